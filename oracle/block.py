@@ -1,0 +1,157 @@
+"""a4-a8: the transformer block, dense and mask-aware (oracle; test infrastructure only).
+
+Block definition (§3.1 "Mask-aware attention", Fig. 5; L134-L138 token-wise
+LayerNorm/GeLU/dropout; Table 1 "(XW1)W2" feed-forward with W1 in R^{H x 4H}):
+
+    h1 = LN(x)(1 + scale1) + shift1                       LN eps 1e-6, no affine   (R3, R2)
+    Q, K, V = h1 Wq^T + bq, h1 Wk^T + bk, h1 Wv^T + bv    split into `heads` heads  (R1)
+    A_j = softmax(Q_j K_j^T / sqrt(d)) V_j                per head j, d = H/heads   (R1)
+    x1 = x + gate1 * (concat_j A_j  Wo^T + bo)
+    h2 = LN(x1)(1 + scale2) + shift2
+    y  = x1 + gate2 * (GELU_tanh(h2 W1^T + b1) W2^T + b2)                          (R3)
+
+Weights use the nn.Linear layout W[out, in]; w_qkv stacks Wq, Wk, Wv as rows [0,H),[H,2H),[2H,3H).
+`mod` is the per-request adaLN vector [6H] = (shift1, scale1, gate1, shift2, scale2, gate2);
+the identity modulation (0, 0, 1, 0, 0, 1) gives plain pre-LN + residual.
+
+Mask-aware block (L157 §3.1, Fig. 5-Bottom; L161 Fig. 7): given the ascending active ids M and
+unmasked ids U of one request (index.build_mask_index),
+  * KV-mode (Fig. 7): compute Q, K, V for rows M only; keys/values of rows U are the
+    cached K[U], V[U] of the template run; attention uses Q_M against the merged key set in
+    original token order (R10); the rest of the block runs on rows M only.
+  * Y-mode (Fig. 5-Bottom): the block input on rows U is the cached previous-block output
+    Y (R4); K, V are projected over all L rows; Q, O-projection and MLP on rows M only.
+Everything is float64.
+"""
+from __future__ import annotations
+
+import math
+
+import numpy as np
+
+LN_EPS = 1e-6
+
+
+def f64(a):
+    return np.asarray(a, dtype=np.float64)
+
+
+def layer_norm(x, eps=LN_EPS):
+    """Row-wise LayerNorm without affine (L134 token-wise; R3)."""
+    x = f64(x)
+    mu = x.mean(axis=-1, keepdims=True)
+    var = ((x - mu) ** 2).mean(axis=-1, keepdims=True)
+    return (x - mu) / np.sqrt(var + eps)
+
+
+def gelu_tanh(x):
+    """GELU, tanh approximation (L134 "GeLU activation"; R3)."""
+    x = f64(x)
+    return 0.5 * x * (1.0 + np.tanh(math.sqrt(2.0 / math.pi) * (x + 0.044715 * x ** 3)))
+
+
+def split_mod(mod, H):
+    mod = f64(mod).reshape(6, H)
+    return mod[0], mod[1], mod[2], mod[3], mod[4], mod[5]
+
+
+def identity_mod(H):
+    m = np.zeros((6, H))
+    m[2] = 1.0
+    m[5] = 1.0
+    return m.reshape(-1)
+
+
+def linear(h, W, b):
+    """h W^T + b (L146 "a linear projection maps X into Q, K, V")."""
+    out = f64(h) @ f64(W).T
+    if b is not None:
+        out = out + f64(b)
+    return out
+
+
+def softmax_rows(s):
+    s = f64(s)
+    s = s - s.max(axis=-1, keepdims=True)
+    e = np.exp(s)
+    return e / e.sum(axis=-1, keepdims=True)
+
+
+def attention(Q, K, V, heads):
+    """Per head j: softmax(Q_j K_j^T / sqrt(d)) V_j  (L146; scale 1/sqrt(d), reading R1).
+
+    Q: [n, H] rows of queries; K, V: [Lk, H]. Returns [n, H] = concat_j A_j.
+    """
+    Q, K, V = f64(Q), f64(K), f64(V)
+    n, H = Q.shape
+    d = H // heads
+    out = np.empty((n, H))
+    for j in range(heads):
+        sl = slice(j * d, (j + 1) * d)
+        S = Q[:, sl] @ K[:, sl].T / math.sqrt(d)
+        out[:, sl] = softmax_rows(S) @ V[:, sl]
+    return out
+
+
+def _qkv_weights(w, H):
+    W, b = f64(w["w_qkv"]), f64(w["b_qkv"])
+    return (W[0:H], b[0:H]), (W[H:2 * H], b[H:2 * H]), (W[2 * H:3 * H], b[2 * H:3 * H])
+
+
+def _attn_out_and_mlp(x_rows, a_rows, w, mod, H):
+    """x1 = x + gate1 (A Wo^T + bo);  y = x1 + gate2 (GELU(h2 W1^T + b1) W2^T + b2)."""
+    _, _, g1, sh2, sc2, g2 = split_mod(mod, H)
+    x1 = f64(x_rows) + g1 * linear(a_rows, w["w_o"], w["b_o"])
+    h2 = layer_norm(x1) * (1.0 + sc2) + sh2
+    y = x1 + g2 * linear(gelu_tanh(linear(h2, w["w_up"], w["b_up"])), w["w_down"], w["b_down"])
+    return y
+
+
+def dense_block(x, w, mod, heads):
+    """Standard block over all L tokens (Fig. 5-Top). Returns (y, K, V)."""
+    x = f64(x)
+    H = x.shape[1]
+    sh1, sc1, _, _, _, _ = split_mod(mod, H)
+    h1 = layer_norm(x) * (1.0 + sc1) + sh1
+    (Wq, bq), (Wk, bk), (Wv, bv) = _qkv_weights(w, H)
+    Q, K, V = linear(h1, Wq, bq), linear(h1, Wk, bk), linear(h1, Wv, bv)
+    a = attention(Q, K, V, heads)
+    return _attn_out_and_mlp(x, a, w, mod, H), K, V
+
+
+def masked_block_kv(x_M, M, U, K_U, V_U, w, mod, heads, L):
+    """KV-cache mode (Fig. 7): fresh Q/K/V on rows M, cached K/V on rows U.
+
+    x_M: [n, H] block input rows M (ascending ids M). K_U, V_U: [u, H] cached keys/values of the
+    template run at rows U. Returns (y_M, K_M, V_M).
+    """
+    x_M = f64(x_M)
+    H = x_M.shape[1]
+    sh1, sc1, _, _, _, _ = split_mod(mod, H)
+    h1_M = layer_norm(x_M) * (1.0 + sc1) + sh1                 # token-wise (L134, L144)
+    (Wq, bq), (Wk, bk), (Wv, bv) = _qkv_weights(w, H)
+    Q_M, K_M, V_M = linear(h1_M, Wq, bq), linear(h1_M, Wk, bk), linear(h1_M, Wv, bv)
+    # merged key set in original token order (R10): fresh rows M, cached rows U
+    K_all = np.empty((L, H))
+    V_all = np.empty((L, H))
+    K_all[M], V_all[M] = K_M, V_M
+    K_all[U], V_all[U] = f64(K_U), f64(V_U)
+    a_M = attention(Q_M, K_all, V_all, heads)                  # queries from masked rows only (L159)
+    return _attn_out_and_mlp(x_M, a_M, w, mod, H), K_M, V_M
+
+
+def masked_block_y(x_M, M, U, x_U, w, mod, heads, L):
+    """Y-cache mode (Fig. 5-Bottom): block input rows U are the cached activations Y of
+    the previous block (R4); K/V over all L rows; Q, O and MLP on rows M. Returns y_M."""
+    x_M = f64(x_M)
+    H = x_M.shape[1]
+    x_full = np.empty((L, H))
+    x_full[M] = x_M
+    x_full[U] = f64(x_U)
+    sh1, sc1, _, _, _, _ = split_mod(mod, H)
+    h1 = layer_norm(x_full) * (1.0 + sc1) + sh1
+    (Wq, bq), (Wk, bk), (Wv, bv) = _qkv_weights(w, H)
+    Q_M = linear(h1[M], Wq, bq)
+    K, V = linear(h1, Wk, bk), linear(h1, Wv, bv)
+    a_M = attention(Q_M, K, V, heads)
+    return _attn_out_and_mlp(x_M, a_M, w, mod, H)

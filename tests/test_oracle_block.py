@@ -1,0 +1,166 @@
+"""Pins for oracle/block.py (a4-a8) against library routines, closed forms and the paper's
+degenerate cases (PAPER.md L134/L144 token-wise ops, L146 all-masked = standard block, L157
+mask-aware block, L161 KV variant)."""
+import math
+
+import numpy as np
+import pytest
+import torch
+import torch.nn.functional as Fn
+
+import synth
+from oracle import block as B
+from oracle.index import build_mask_index
+
+torch.set_default_dtype(torch.float64)
+
+
+def _setup(seed=0, H=48, heads=3, F=80, L=40, dtype="f32", mod=True):
+    g = synth.rng(seed)
+    w = synth.block_weights(g, H, F, dtype)
+    x = synth.latent(g, L, H, dtype)
+    m = synth.mod_table(g, 1, 1, H, dtype, enabled=mod)[0, 0]
+    return g, w, x, m
+
+
+def test_layer_norm_vs_torch_and_moments():
+    g = synth.rng(1)
+    x = g.standard_normal((17, 33)) * 3 + 1
+    ref = Fn.layer_norm(torch.tensor(x), (33,), eps=1e-6).numpy()
+    out = B.layer_norm(x)
+    assert np.allclose(out, ref, rtol=0, atol=1e-12)
+    assert np.allclose(out.mean(-1), 0, atol=1e-12)
+    assert np.allclose(out.var(-1), 1 / (1 + 1e-6 / x.var(-1)), atol=1e-9)
+
+
+def test_gelu_vs_torch():
+    x = np.linspace(-8, 8, 1001)
+    ref = Fn.gelu(torch.tensor(x), approximate="tanh").numpy()
+    assert np.allclose(B.gelu_tanh(x), ref, rtol=0, atol=1e-14)
+
+
+def test_attention_vs_sdpa_and_uniform_case():
+    g = synth.rng(2)
+    n, Lk, heads, d = 7, 19, 3, 16
+    Q, K, V = (g.standard_normal((r, heads * d)) for r in (n, Lk, Lk))
+    out = B.attention(Q, K, V, heads)
+    t = lambda a, r: torch.tensor(a).view(r, heads, d).transpose(0, 1)
+    ref = Fn.scaled_dot_product_attention(t(Q, n), t(K, Lk), t(V, Lk))  # scale 1/sqrt(d)
+    assert np.allclose(out, ref.transpose(0, 1).reshape(n, heads * d).numpy(), atol=1e-12)
+    # Q = 0 -> uniform weights -> every output row is the mean of V (closed form)
+    out0 = B.attention(np.zeros_like(Q), K, V, heads)
+    assert np.allclose(out0, np.broadcast_to(V.mean(0), out0.shape), atol=1e-12)
+
+
+def _torch_block(x, w, mod, heads):
+    """The same block assembled from torch library modules (nn.MultiheadAttention, LayerNorm,
+    Linear, GELU(tanh)) in float64 -- an implementation independent of oracle/block.py."""
+    H = x.shape[1]
+    mha = torch.nn.MultiheadAttention(H, heads, bias=True, batch_first=True)
+    with torch.no_grad():
+        mha.in_proj_weight.copy_(torch.tensor(w["w_qkv"]))
+        mha.in_proj_bias.copy_(torch.tensor(w["b_qkv"]))
+        mha.out_proj.weight.copy_(torch.tensor(w["w_o"]))
+        mha.out_proj.bias.copy_(torch.tensor(w["b_o"]))
+        up = torch.nn.Linear(H, w["w_up"].shape[0])
+        up.weight.copy_(torch.tensor(w["w_up"])); up.bias.copy_(torch.tensor(w["b_up"]))
+        dn = torch.nn.Linear(w["w_up"].shape[0], H)
+        dn.weight.copy_(torch.tensor(w["w_down"])); dn.bias.copy_(torch.tensor(w["b_down"]))
+        sh1, sc1, g1, sh2, sc2, g2 = torch.tensor(np.asarray(mod, np.float64)).view(6, H)
+        xt = torch.tensor(np.asarray(x, np.float64))[None]
+        h1 = Fn.layer_norm(xt, (H,), eps=1e-6) * (1 + sc1) + sh1
+        a, _ = mha(h1, h1, h1, need_weights=False)
+        x1 = xt + g1 * a
+        h2 = Fn.layer_norm(x1, (H,), eps=1e-6) * (1 + sc2) + sh2
+        y = x1 + g2 * dn(Fn.gelu(up(h2), approximate="tanh"))
+    return y[0].numpy()
+
+
+@pytest.mark.parametrize("mod", [True, False])
+def test_dense_block_vs_torch_modules(mod):
+    _, w, x, m = _setup(mod=mod)
+    y, _, _ = B.dense_block(x, w, m, 3)
+    assert np.allclose(y, _torch_block(x, w, m, 3), rtol=0, atol=1e-10)
+
+
+def test_dense_block_zero_weights_closed_form():
+    """W = 0: Q, K const -> uniform attention -> A = bv; o = bo; y = x + g1*bo + g2*b2."""
+    g, w, x, m = _setup(seed=5)
+    for k in ("w_qkv", "w_o", "w_up", "w_down"):
+        w[k] = np.zeros_like(w[k])
+    y, _, _ = B.dense_block(x, w, m, 3)
+    H = x.shape[1]
+    mm = m.astype(np.float64).reshape(6, H)
+    assert np.allclose(y, x + mm[2] * w["b_o"] + mm[5] * w["b_down"], atol=1e-12)
+
+
+def _kv_cache_from_dense(x, w, m, heads, U):
+    _, K, V = B.dense_block(x, w, m, heads)
+    return K[U], V[U]
+
+
+@pytest.mark.parametrize("ratio", [0.0, 0.1, 0.5, 1.0])
+def test_masked_equals_dense_under_identical_input_cache(ratio):
+    """L144/L157: every op but attention is token-wise, so with the cache taken from a dense
+    run on the identical input, masked rows reproduce the dense rows (both modes)."""
+    g, w, x, m = _setup(seed=9, L=64)
+    mask = synth.mask_blobs(g, 8, 8, ratio)
+    M, U = build_mask_index(mask)
+    y_ref, K, V = B.dense_block(x, w, m, 3)
+    y_kv, K_M, V_M = B.masked_block_kv(x[M], M, U, K[U], V[U], w, m, 3, 64)
+    y_y = B.masked_block_y(x[M], M, U, x[U], w, m, 3, 64)
+    assert np.allclose(y_kv, y_ref[M], rtol=0, atol=1e-12)
+    assert np.allclose(y_y, y_ref[M], rtol=0, atol=1e-12)
+    assert np.allclose(K_M, K[M], atol=1e-12) and np.allclose(V_M, V[M], atol=1e-12)
+
+
+def test_all_ones_mask_is_dense():
+    """L146: with every token masked, the mask-aware block is the standard block."""
+    _, w, x, m = _setup(seed=4)
+    L = x.shape[0]
+    M, U = np.arange(L), np.arange(0)
+    y_ref, _, _ = B.dense_block(x, w, m, 3)
+    e = np.zeros((0, x.shape[1]))
+    y_kv, _, _ = B.masked_block_kv(x, M, U, e, e, w, m, 3, L)
+    assert np.allclose(y_kv, y_ref, rtol=0, atol=1e-12)
+    assert np.allclose(B.masked_block_y(x, M, U, e, w, m, 3, L), y_ref, rtol=0, atol=1e-12)
+
+
+def test_cache_is_actually_used():
+    """With a cache from a DIFFERENT template input, masked rows differ from the request's own
+    dense rows, and perturbing one cached key/value row changes the output."""
+    g, w, x, m = _setup(seed=12, L=64)
+    mask = synth.mask_random(g, 64, 0.25)
+    M, U = build_mask_index(mask)
+    x_t = synth.latent(g, 64, x.shape[1], "f32")
+    _, Kt, Vt = B.dense_block(x_t, w, m, 3)
+    y_kv, _, _ = B.masked_block_kv(x[M], M, U, Kt[U], Vt[U], w, m, 3, 64)
+    y_ref, _, _ = B.dense_block(x, w, m, 3)
+    assert not np.allclose(y_kv, y_ref[M], atol=1e-3)
+    Vt2 = Vt.copy(); Vt2[U[0]] += 1.0
+    y2, _, _ = B.masked_block_kv(x[M], M, U, Kt[U], Vt2[U], w, m, 3, 64)
+    assert not np.allclose(y2, y_kv, atol=1e-6)
+    # Y-mode: perturbing an unmasked input row changes masked outputs (through K/V only)
+    xu = x_t[U].copy(); xu[0, 0] += 1.0          # (a whole-row shift would be LN-invariant)
+    assert not np.allclose(B.masked_block_y(x[M], M, U, xu, w, m, 3, 64),
+                           B.masked_block_y(x[M], M, U, x_t[U], w, m, 3, 64), atol=1e-6)
+
+
+def test_key_order_invariance():
+    """Softmax attention does not depend on the key order (R10: order is a layout choice)."""
+    g = synth.rng(21)
+    Q, K, V = g.standard_normal((5, 32)), g.standard_normal((23, 32)), g.standard_normal((23, 32))
+    p = g.permutation(23)
+    assert np.allclose(B.attention(Q, K, V, 2), B.attention(Q, K[p], V[p], 2), atol=1e-12)
+
+
+def test_token_wise_rows_independent():
+    """L134: outside attention each row's result depends only on that row: two different
+    inputs that share rows M and K/V produce identical masked outputs."""
+    g, w, x, m = _setup(seed=13, L=32)
+    mask = synth.mask_random(g, 32, 0.5)
+    M, U = build_mask_index(mask)
+    _, K, V = B.dense_block(x, w, m, 3)
+    y1, _, _ = B.masked_block_kv(x[M], M, U, K[U], V[U], w, m, 3, 32)
+    y2, _, _ = B.masked_block_kv(x[M][::-1].copy(), M[::-1].copy(), U, K[U], V[U], w, m, 3, 32)
+    assert np.allclose(y1, y2[::-1], atol=1e-12)

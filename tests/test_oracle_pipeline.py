@@ -1,0 +1,129 @@
+"""Pins for oracle/pipeline.py (Alg. 1 reading R11) and oracle/counters.py (Table 1)."""
+import json
+import math
+import os
+
+import numpy as np
+import pytest
+
+import synth
+from oracle import counters as C
+from oracle import pipeline as P
+
+
+def _golden():
+    return json.load(open(os.path.join(os.path.dirname(__file__), "golden",
+                                       "pipeline_cases.json")))["cases"]
+
+
+@pytest.mark.parametrize("case", _golden(), ids=lambda c: c["name"])
+def test_hand_timelines(case):
+    v = P.simulate(case["use"], case["Cw"], case["Cwo"], case["Lm"], case["mode"],
+                   case["final"], case.get("slots"))
+    assert v == pytest.approx(case["latency"])
+
+
+def test_limits():
+    """L^m = 0 -> caching every block is optimal; C_w^m >= C_w/o -> caching nothing is."""
+    g = synth.rng(0)
+    for mode in ("kv", "y"):
+        Cw = g.uniform(1, 2, 8); Cwo = Cw + g.uniform(0.5, 2, 8)
+        lat, plan = P.plan_bruteforce(Cw, Cwo, np.zeros(8), mode)
+        assert plan == [1] * 8 and lat == pytest.approx(Cw.sum())
+        lat, plan = P.plan_bruteforce(Cwo + 1, Cwo, g.uniform(0, 1, 8), mode, 0.1)
+        assert plan == [0] * 8 and lat == pytest.approx(Cwo.sum())
+
+
+def test_naive_sequential_is_sum():
+    """Fig. 9-Top: with one staging slot and loads as long as compute, nothing overlaps."""
+    Cw, Lm = [1.0, 2.0, 3.0], [1.5, 0.5, 2.0]
+    v = P.simulate([1, 1, 1], Cw, [9, 9, 9], Lm, "kv", 0.0, slots=1)
+    assert v == pytest.approx(sum(Cw) + sum(Lm))
+
+
+def test_kv_suffix_scan_is_exact():
+    """KV-mode feasible plans are exactly the N+1 suffixes, so the O(N) scan is optimal."""
+    g = synth.rng(1)
+    for _ in range(100):
+        N = int(g.integers(1, 11))
+        Cw, Cwo, Lm = g.uniform(0.5, 2, N), g.uniform(1, 4, N), g.uniform(0, 3, N)
+        fin = float(g.uniform(0, 1))
+        a = P.plan_bruteforce(Cw, Cwo, Lm, "kv", fin)[0]
+        # exhaustive over ALL 2^N plans (infeasible ones score +inf)
+        import itertools
+        b = min(P.simulate(p, Cw, Cwo, Lm, "kv", fin) for p in itertools.product((0, 1), repeat=N))
+        assert a == pytest.approx(b)
+        assert P.plan_suffix_scan(Cw, Cwo, Lm, "kv", fin)[0] == pytest.approx(a)
+
+
+def test_y_bruteforce_beats_or_ties_suffix():
+    g = synth.rng(2)
+    worse = 0
+    for _ in range(60):
+        N = int(g.integers(2, 10))
+        Cw, Cwo, Lm = g.uniform(0.2, 2, N), g.uniform(1, 4, N), g.uniform(0, 4, N)
+        a = P.plan_bruteforce(Cw, Cwo, Lm, "y")[0]
+        b = P.plan_suffix_scan(Cw, Cwo, Lm, "y")[0]
+        assert a <= b + 1e-12
+        worse += b > a + 1e-9
+    assert worse > 0          # heterogeneous Y-mode stacks do need the exhaustive/DP planner
+
+
+def test_more_slots_never_slower():
+    g = synth.rng(3)
+    for _ in range(50):
+        N = 6
+        Cw, Cwo, Lm = g.uniform(0.5, 2, N), g.uniform(1, 4, N), g.uniform(0, 3, N)
+        use = [int(v) for v in g.integers(0, 2, N)]
+        for mode in ("y",):
+            vals = [P.simulate(use, Cw, Cwo, Lm, mode, 0.0, s) for s in (1, 2, 3, None)]
+            assert all(vals[i] >= vals[i + 1] - 1e-12 for i in range(3))
+
+
+def test_table1_scaling():
+    """Table 1 (L165-L173): with image-only tokens, FFN, projection and QK^T FLOPs of the
+    KV-mode block are exactly m times the dense ones; cache shape is ((1-m)L, H)."""
+    L, H, F = 4096, 3072, 12288
+    for m in (0.05, 0.2, 0.5):
+        n = synth.n_masked_for(m, L)
+        ratio = n / L
+        assert C.gemm_flops("kv", n, L, H, F) == pytest.approx(ratio * C.gemm_flops("dense", L, L, H, F))
+        attn_m = C.block_flops("kv", n, L, H, F) - C.gemm_flops("kv", n, L, H, F)
+        attn_d = C.block_flops("dense", L, L, H, F) - C.gemm_flops("dense", L, L, H, F)
+        assert attn_m == pytest.approx(ratio * attn_d)
+        assert C.cache_bytes("y", L - n, H, 2) == (L - n) * H * 2
+        assert C.cache_bytes("kv", L - n, H, 2) == 2 * C.cache_bytes("y", L - n, H, 2)  # L161
+        # Y-mode keeps the K/V projections of the unmasked rows (R5): exactly 4uH^2 more
+        assert C.block_flops("y", n, L, H, F) - C.block_flops("kv", n, L, H, F) == 4 * (L - n) * H * H
+
+
+def test_flops_match_matmul_shapes():
+    """Count 2*m*n*k over the matmuls oracle/block.py performs (instrumented linear/attention)."""
+    from oracle import block as B
+    g = synth.rng(4)
+    H, heads, F, L = 16, 2, 40, 24
+    w = synth.block_weights(g, H, F, "f32")
+    x = synth.latent(g, L, H, "f32")
+    mod = B.identity_mod(H)
+    M = np.arange(0, L, 3); U = np.setdiff1d(np.arange(L), M)
+    count = {"f": 0}
+    orig = B.linear, B.attention
+
+    def lin(h, W, b):
+        count["f"] += 2 * h.shape[0] * W.shape[0] * W.shape[1]
+        return orig[0](h, W, b)
+
+    def att(Q, K, V, heads_):
+        count["f"] += 2 * Q.shape[0] * K.shape[0] * Q.shape[1] * 2
+        return orig[1](Q, K, V, heads_)
+
+    B.linear, B.attention = lin, att
+    try:
+        B.dense_block(x, w, mod, heads)
+        assert count["f"] == C.block_flops("dense", L, L, H, F); count["f"] = 0
+        B.masked_block_kv(x[M], M, U, x[U], x[U], w, mod, heads, L)
+        assert count["f"] == C.block_flops("kv", len(M), L, H, F); count["f"] = 0
+        B.masked_block_y(x[M], M, U, x[U], w, mod, heads, L)
+        assert count["f"] == C.block_flops("y", len(M), L, H, F)
+    finally:
+        B.linear, B.attention = orig
