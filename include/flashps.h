@@ -1,0 +1,267 @@
+/* flashps.h -- C ABI of the B200-native FlashPS hot path (libflashps.so).
+ *
+ * FlashPS (EuroSys '26), /root/reference/PAPER.md: the mask-aware transformer-block forward
+ * (§3.1, Fig. 5/7), its block-granular cache-load pipeline (§4.2,
+ * Alg. 1) and step-level continuous batching (§4.3).  `Lnnn` = PAPER.md line nnn.
+ *
+ * Conventions for every call
+ *  - Pointers prefixed d_ are DEVICE pointers, h_ are HOST pointers. Device buffers are
+ *    caller-owned (allocated with any CUDA allocator, e.g. torch); the library never frees them.
+ *    Library-owned state lives only inside fps_cache_t / fps_engine_t handles.
+ *  - `stream` arguments are cudaStream_t passed as void* (NULL = legacy default stream).
+ *    Every device call is asynchronous on its stream: no allocation and no host
+ *    synchronisation inside hot calls (fps_run_batch documents its one admission sync).
+ *  - Errors: arguments are validated before anything is enqueued, so a failing call has no
+ *    side effect and returns FPS_EINVAL / FPS_EUNSUPPORTED; a failed launch returns FPS_ECUDA.
+ *    Asynchronous device faults surface at the caller's next synchronisation.
+ *    fps_last_error() returns a thread-local message describing the last failure.
+ *  - Rows are contiguous and 16-byte aligned (row_bytes % 16 == 0, pointers 16-B aligned).
+ *  - Determinism: outputs are bit-reproducible run to run (no split-K atomics).
+ *  - There is no CPU fallback: on a machine without a usable sm_100 GPU every device call
+ *    returns FPS_ECUDA.
+ */
+#ifndef FLASHPS_H
+#define FLASHPS_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define FPS_ABI_VERSION 1
+
+typedef enum {
+  FPS_OK = 0,
+  FPS_EINVAL = -1,        /* bad argument (null pointer, size, alignment, layout)        */
+  FPS_ECUDA = -2,         /* CUDA runtime / launch failure, or no usable sm_100 device     */
+  FPS_ENOMEM = -3,        /* host or device allocation failed (handle creation only)       */
+  FPS_EUNSUPPORTED = -4,  /* valid request outside what the kernels implement              */
+  FPS_ESTATE = -5         /* handle in the wrong state (e.g. prefetch of a never-stored entry) */
+} fps_status;
+
+enum { FPS_F32 = 0, FPS_BF16 = 1 };            /* element type of activations and weights */
+enum { FPS_MODE_KV = 0, FPS_MODE_Y = 1 };      /* caching variant: Fig. 7 (K/V) or Fig. 5 (Y) */
+
+const char* fps_last_error(void);
+int32_t fps_abi_version(void);
+/* 1 if a device usable by the kernels (compute capability 10.0) is present, else 0. */
+int32_t fps_device_ok(void);
+/* Test / bench hooks: number of kernels this thread has launched through the library so far;
+ * force the SIMT kernels (bit0: GEMMs, bit1: attention) instead of the tensor-core ones. */
+int64_t fps_launch_count(void);
+void fps_set_disable_tc(int32_t flags);
+
+/* ---------------------------------------------------------------------------------------
+ * a1  Mask -> token index (L130 "categorize the tokens as masked tokens and unmasked tokens").
+ *   d_masks       uint8 [total]: request r's token mask occupies [off[r], off[r+1]);
+ *                 nonzero = active (masked image token, or text token -- set by the caller).
+ *   d_offsets     int32 [n_req+1] on DEVICE, off[0] = 0, non-decreasing.
+ *   d_masked_ids  int32 [total]: request r's ascending LOCAL active ids are written to
+ *                 d_masked_ids[off[r] .. off[r]+n_r).
+ *   d_unmasked_ids int32 [total]: ascending local inactive ids at [off[r] .. off[r]+L_r-n_r).
+ *   d_n_masked    int32 [n_req]: n_r.
+ *   max_len       upper bound on any L_r (launch sizing only).
+ * Bit-exact with the oracle (oracle/index.py). One CTA per request, warp-ballot compaction. */
+fps_status fps_build_mask_index(const uint8_t* d_masks, const int32_t* d_offsets, int32_t n_req,
+                                int32_t max_len, int32_t* d_masked_ids, int32_t* d_unmasked_ids,
+                                int32_t* d_n_masked, void* stream);
+
+/* ---------------------------------------------------------------------------------------
+ * a2 / a9  Row movement (L157 "extract the matrix of masked tokens ... replenishing cached
+ * activations for the unmasked tokens"). 16-B vectorised, bit-exact.
+ *   gather : d_dst[i]          = d_src[d_ids[i]]      i in [0, n)
+ *   scatter: d_dst[d_ids[i]]   = d_src[i]
+ *   copy   : d_dst[d_dst_ids[i]] = d_src[d_src_ids[i]]   (either id array may be NULL = i)
+ * row_bytes % 16 == 0. d_src may be a mapped pinned-host pointer (zero-copy read).          */
+fps_status fps_gather_rows(const void* d_src, const int32_t* d_ids, int32_t n, int32_t row_bytes,
+                           void* d_dst, void* stream);
+fps_status fps_scatter_rows(const void* d_src, const int32_t* d_ids, int32_t n, int32_t row_bytes,
+                            void* d_dst, void* stream);
+fps_status fps_copy_rows(const void* d_src, const int32_t* d_src_ids, const int32_t* d_dst_ids,
+                         int32_t n, int32_t row_bytes, void* d_dst, void* stream);
+
+/* ---------------------------------------------------------------------------------------
+ * a3  Activation cache (L203 host-DRAM store; L207 block granularity; reading R7: key =
+ * (template, step, layer)).  An entry holds L_img rows of width W elements of the template's
+ * full run: KV-mode W = 2H (row = K|V of that token, Fig. 7), Y-mode W = H (block output Y,
+ * Fig. 5).  KV-mode also keeps, per step, the final block's Y rows under layer = n_layers
+ * (width H) for the last replenish (reading R22).                                           */
+typedef struct {
+  int32_t mode;          /* FPS_MODE_KV | FPS_MODE_Y                                        */
+  int32_t dtype;         /* FPS_BF16 | FPS_F32                                              */
+  int32_t H;             /* hidden size                                                     */
+  int32_t L_img;         /* rows per entry (image tokens; text rows are never cached, R9)   */
+  int32_t n_layers;
+  int32_t n_steps;
+  int32_t n_templates;   /* templates addressable: template_id in [0, n_templates)          */
+  int32_t n_entries;     /* physical entries in the pinned arena; 0 = one per key.  When
+                            smaller, key k maps to entry k % n_entries (perf runs only: bytes
+                            moved are identical, contents alias)                            */
+  int32_t copy_method;   /* 0 = SM zero-copy row gather over mapped pinned memory (default);
+                            1 = copy-engine DMA of coalesced row runs                        */
+  int32_t copy_ctas;     /* CTAs used by method 0 (0 = default 32)                          */
+} fps_cache_desc;
+
+typedef struct fps_cache* fps_cache_t;
+
+fps_status fps_cache_create(const fps_cache_desc* desc, fps_cache_t* out);
+fps_status fps_cache_destroy(fps_cache_t c);
+/* Host pointer of an entry (tests / tooling); NULL if out of range. */
+void* fps_cache_entry_host_ptr(fps_cache_t c, uint32_t template_id, int32_t step, int32_t layer);
+size_t fps_cache_entry_bytes(fps_cache_t c, int32_t layer);
+/* D2H: store rows [0, L_img) of d_src (row pitch src_row_bytes >= W*elt) as entry
+ * (template_id, step, layer).  Asynchronous on `stream`. */
+fps_status fps_cache_store(fps_cache_t c, uint32_t template_id, int32_t step, int32_t layer,
+                           const void* d_src, int32_t src_row_bytes, void* stream);
+
+/* H2D layer-ahead prefetch (L207-L209): for each item, rows d_rows[0..n_rows) (LOCAL token
+ * ids < L_img, ascending) of entry (template_id, step, layer) are copied to the SAME row
+ * positions of d_dst (row pitch dst_row_bytes).  All items are issued on `load_stream`; if
+ * `ready_event` (cudaEvent_t) is non-NULL it is recorded after the last copy. */
+typedef struct {
+  uint32_t template_id;
+  int32_t step;
+  int32_t layer;
+  int32_t n_rows;
+  const int32_t* d_rows;   /* device, [n_rows] local row ids (unmasked tokens U)          */
+  const int32_t* h_rows;   /* host mirror of d_rows (used by copy_method 1; may be NULL
+                              for method 0)                                                */
+  void* d_dst;             /* device row 0 of this request's [L, W] region                */
+  int32_t dst_row_bytes;
+} fps_prefetch_item;
+
+fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int32_t n_items,
+                              void* load_stream, void* ready_event);
+
+/* ---------------------------------------------------------------------------------------
+ * a4-a8  Block forward (L146 block definition; L157 mask-aware; L161 KV variant).
+ * Block (oracle/block.py):  h1 = LN(x)(1+sc1)+sh1; Q,K,V = h1 W^T + b; A = softmax(QK^T/sqrt(d))V
+ * per head; x1 = x + g1 (A Wo^T + bo); y = x1 + g2 (GELU_tanh(LN(x1)(1+sc2)+sh2 W1^T + b1) W2^T + b2).
+ * Weights use the nn.Linear layout W[out, in], row-major, dtype = `dtype`; biases may be NULL.
+ */
+typedef struct {
+  int32_t H, heads, head_dim, F;   /* H = heads*head_dim; F = MLP width                    */
+  int32_t dtype;                   /* FPS_BF16 (tcgen05 path) | FPS_F32 (SIMT fp32 path)   */
+  const void *w_qkv, *b_qkv;       /* [3H, H], [3H]  rows: Wq, Wk, Wv                       */
+  const void *w_o, *b_o;           /* [H, H], [H]                                          */
+  const void *w_up, *b_up;         /* [F, H], [F]                                          */
+  const void *w_down, *b_down;     /* [H, F], [H]                                          */
+} fps_block_weights;
+
+/* One varlen launch over a continuous batch (L237): request r owns active rows
+ * [cu_q[r], cu_q[r+1]) of the compact activation arrays and merged key rows
+ * [cu_k[r], cu_k[r+1]) of d_kv. */
+typedef struct {
+  int32_t n_req;
+  int32_t total_q, total_k;        /* sum n_r, sum L_r                                      */
+  int32_t max_q, max_k;            /* max n_r, max L_r                                      */
+  const int32_t* d_cu_q;           /* [n_req+1]                                             */
+  const int32_t* d_cu_k;           /* [n_req+1]                                             */
+  const int32_t* h_cu_q;           /* host mirrors (launch sizing, no device sync)           */
+  const int32_t* h_cu_k;
+  const int32_t* d_q_row;          /* [total_q] merged-buffer row of each active row;
+                                      NULL = identity (dense block: total_q == total_k)      */
+  const void* d_mod;               /* [n_req, 6H] adaLN (shift1,scale1,gate1,shift2,scale2,
+                                      gate2) in dtype, or NULL = identity modulation         */
+  int32_t mode;                    /* FPS_MODE_KV | FPS_MODE_Y                               */
+  /* Y-mode only (Fig. 5-Bottom): cached input rows U feed the K/V projection.             */
+  int32_t total_u;                 /* sum u_r                                               */
+  const int32_t* d_cu_u;           /* [n_req+1]                                             */
+  const int32_t* d_u_src;          /* [total_u] row index into d_xu of each cached row      */
+  const int32_t* d_u_row;          /* [total_u] merged-buffer row of each cached row        */
+} fps_varlen_batch;
+
+/* Workspace bytes fps_masked_block_forward needs for up to max_q active / max_u cached rows. */
+size_t fps_block_workspace_bytes(int32_t H, int32_t F, int32_t dtype, int32_t max_q, int32_t max_u);
+
+/* Mask-aware block over a varlen batch.
+ *   d_x_act [total_q, H]  input rows (active tokens, request-major, ascending ids).
+ *   d_y_act [total_q, H]  output rows. May alias nothing else.
+ *   d_kv    [total_k, 2H] merged key buffer, row = K|V.  KV-mode: rows NOT named by d_q_row
+ *           must already hold (or be in flight to) the cached K|V (fps_cache_prefetch);
+ *           this call writes the fresh rows d_q_row.  Y-mode: fully written by this call.
+ *   d_xu    Y-mode: base of the cached input rows (indexed by b->d_u_src); NULL in KV-mode.
+ *   kv_ready (cudaEvent_t or NULL): waited on `stream` right before the first kernel that
+ *           reads cached rows (attention in KV-mode, the K/V projection in Y-mode), so the
+ *           fresh Q/K/V projection overlaps the in-flight load.
+ *   d_ws / ws_bytes: scratch of at least fps_block_workspace_bytes(...). */
+fps_status fps_masked_block_forward(const fps_block_weights* w, const fps_varlen_batch* b,
+                                    const void* d_x_act, void* d_y_act, void* d_kv,
+                                    const void* d_xu, void* kv_ready, void* d_ws, size_t ws_bytes,
+                                    void* stream);
+
+/* Dense block (Fig. 5-Top; the uncached blocks of Fig. 9-Bottom): all L_r rows of every
+ * request; b->d_q_row must be NULL and total_q == total_k.  d_kv is scratch [total_k, 2H]. */
+fps_status fps_dense_block_forward(const fps_block_weights* w, const fps_varlen_batch* b,
+                                   const void* d_x, void* d_y, void* d_kv, void* d_ws,
+                                   size_t ws_bytes, void* stream);
+
+/* ---------------------------------------------------------------------------------------
+ * a10  Alg. 1 (L211-L219): choose use_cache[l] minimising the step's pipeline latency, under
+ * the pipeline model of reading R11: one load stream (cached blocks' loads in
+ * order, back to back), one compute stream; KV-mode: block l waits for its own load, plans are
+ * monotone, and a final load of `final_load` (the last block's Y rows) ends the step;
+ * Y-mode: block l+1 waits for block l's load.  Unbounded staging slots.  Host only.
+ *   c_cached[N] = C_w^m, c_dense[N] = C_w/o, load[N] = L^m (any time unit).
+ *   use_cache[N] (out), latency (out).  Exact: KV-mode O(N) scan over the N+1 feasible plans;
+ *   Y-mode exact Pareto-front DP over (compute end, load end). */
+fps_status fps_plan_pipeline(const double* c_cached, const double* c_dense, const double* load,
+                             int32_t N, int32_t mode, double final_load, uint8_t* use_cache,
+                             double* latency);
+/* The model itself (for tests and the balancer): latency of a given plan; +inf if infeasible. */
+double fps_pipeline_latency(const uint8_t* use_cache, const double* c_cached,
+                            const double* c_dense, const double* load, int32_t N, int32_t mode,
+                            double final_load);
+
+/* ---------------------------------------------------------------------------------------
+ * Step-level continuous batching over a stack of N blocks (L237, §4.3; Fig. 9 pipeline).
+ */
+typedef struct {
+  int32_t H, heads, F, n_layers, dtype, mode;
+  int32_t L_img, L_txt;            /* per-request tokens (text appended after image, R9)   */
+  int32_t max_batch;               /* max requests per fps_run_batch call (L326: 8)         */
+  int32_t n_steps;                 /* denoising steps of the schedule                       */
+  const fps_block_weights* layers; /* [n_layers], device weight pointers (caller-owned)     */
+  const void* d_mod_table;         /* [n_layers, n_steps, 6H] adaLN vectors, or NULL        */
+  const float* h_deltas;           /* [n_steps] Euler coefficients (copied at create)       */
+  fps_cache_t cache;               /* template activation cache (required)                  */
+  int32_t slots;                   /* staging slots for layer-ahead prefetch (0 = n_layers) */
+  int32_t plan_policy;             /* 0 = Alg. 1 planner; 1 = all cached; 2 = none (dense);
+                                      3 = explicit h_plan                                   */
+  const uint8_t* h_plan;           /* [n_layers] when plan_policy == 3 (copied at create)   */
+  double cost_model[4];            /* planner latency model: comp = a*FLOPs + b,
+                                      load = c*bytes + e  -> {a, b, c, e}  (§4.4)     */
+} fps_engine_desc;
+
+typedef struct fps_engine* fps_engine_t;
+
+typedef struct {
+  uint32_t template_id;
+  int32_t step;            /* in/out: next denoising step of this request                 */
+  int32_t n_steps;         /* request leaves the batch when step == n_steps                */
+  const uint8_t* d_mask;   /* [L_img + L_txt] device token mask (text rows nonzero)         */
+  void* d_x;               /* [L, H] device latent tokens, updated in place                 */
+  int32_t status;          /* out: 0 = running, 1 = finished                                */
+} fps_request;
+
+fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out);
+fps_status fps_engine_destroy(fps_engine_t e);
+/* Run up to n_steps denoising steps over reqs[0..n_req) (n_req <= max_batch).  Each step
+ * every unfinished request advances by one; a request whose step reaches its n_steps leaves
+ * at that step boundary (status = 1) and the batch shrinks.  Admission reads the active-row
+ * counts back to the host once per call (the only host sync).  Each step: mask-aware stack
+ * with the Alg. 1 plan, layer-ahead prefetch on `load_stream`, final replenish + Euler update
+ * x <- x + delta_s * y (reading R21).  The engine's last plan is available below. */
+fps_status fps_run_batch(fps_engine_t e, fps_request* reqs, int32_t n_req, int32_t n_steps,
+                         void* compute_stream, void* load_stream);
+/* Plan and predicted latency (ms) of the last step; use_cache may be NULL. */
+fps_status fps_engine_last_plan(fps_engine_t e, uint8_t* use_cache, double* latency_ms);
+/* Kernels the engine launched in its last fps_run_batch call (own kernels only). */
+int64_t fps_engine_last_launches(fps_engine_t e);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FLASHPS_H */

@@ -1,0 +1,271 @@
+// C ABI entry points of libflashps: validation, dispatch, and the block-forward composition
+// (PAPER.md L146 block; L157 mask-aware Y-mode; L161 KV-mode).  See include/flashps.h.
+#include <cstring>
+#include <mutex>
+
+#include "kernels.h"
+
+namespace fps {
+
+static thread_local std::string g_err;
+thread_local long long g_launches = 0;
+int g_disable_tc = 0;
+
+void set_error(const char* fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+}
+
+fps_status fail(fps_status code, const char* fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return code;
+}
+
+static int elt_size(int dtype) { return dtype == FPS_BF16 ? 2 : 4; }
+
+fps_status launch_gemm(int dtype, const void* A, const void* B, int M, int N, int K,
+                       const Epilogue& ep, cudaStream_t s) {
+  if (M <= 0 || N <= 0) return FPS_OK;
+  if (!(g_disable_tc & 1) && gemm_tc_supported(dtype, M, N, K))
+    return launch_gemm_tc(A, B, M, N, K, ep, s);
+  return launch_gemm_simt(dtype, A, B, M, N, K, ep, s);
+}
+
+fps_status launch_attention(int dtype, const void* q, const void* kv, void* o, int heads,
+                            int head_dim, const int32_t* d_cu_q, const int32_t* d_cu_k,
+                            const int32_t* h_cu_q, const int32_t* h_cu_k, int n_req, int total_q,
+                            int max_q, int max_k, cudaStream_t s) {
+  (void)h_cu_k;
+  (void)max_k;
+  if (total_q <= 0) return FPS_OK;
+  if (!(g_disable_tc & 2) && attention_tc_supported(dtype, head_dim))
+    return launch_attention_tc(q, kv, o, heads, head_dim, d_cu_q, d_cu_k, h_cu_q, n_req, max_q, s);
+  return launch_attention_simt(dtype, q, kv, o, heads, head_dim, d_cu_q, d_cu_k, n_req, total_q, s);
+}
+
+struct BlockWs {
+  char *h, *q, *ao, *x1, *h2, *u, *hu;
+};
+
+static size_t align256(size_t v) { return (v + 255) & ~size_t(255); }
+
+static size_t ws_layout(int H, int F, int dtype, int max_q, int max_u, char* base, BlockWs* ws) {
+  const size_t e = elt_size(dtype);
+  size_t off = 0;
+  auto take = [&](size_t bytes) {
+    char* p = base ? base + off : nullptr;
+    off += align256(bytes);
+    return p;
+  };
+  char* h = take((size_t)max_q * H * e);
+  char* q = take((size_t)max_q * H * e);
+  char* ao = take((size_t)max_q * H * e);
+  char* x1 = take((size_t)max_q * H * e);
+  char* h2 = take((size_t)max_q * H * e);
+  char* u = take((size_t)max_q * F * e);
+  char* hu = take((size_t)max_u * H * e);
+  if (ws) *ws = BlockWs{h, q, ao, x1, h2, u, hu};
+  return off;
+}
+
+static fps_status check_weights(const fps_block_weights* w) {
+  FPS_CHECK_ARG(w, "weights is NULL");
+  FPS_CHECK_ARG(w->dtype == FPS_BF16 || w->dtype == FPS_F32, "dtype %d", w->dtype);
+  FPS_CHECK_ARG(w->H > 0 && w->heads > 0 && w->head_dim > 0 && w->heads * w->head_dim == w->H,
+                "H=%d heads=%d head_dim=%d", w->H, w->heads, w->head_dim);
+  FPS_CHECK_ARG(w->F > 0, "F=%d", w->F);
+  FPS_CHECK_ARG(w->w_qkv && w->w_o && w->w_up && w->w_down, "weight pointer is NULL");
+  const int vec = 16 / elt_size(w->dtype);
+  FPS_CHECK_ARG(w->H % vec == 0 && w->F % vec == 0, "H and F must be multiples of %d", vec);
+  return FPS_OK;
+}
+
+static fps_status check_batch(const fps_varlen_batch* b) {
+  FPS_CHECK_ARG(b, "batch is NULL");
+  FPS_CHECK_ARG(b->n_req >= 0 && b->total_q >= 0 && b->total_k >= 0, "negative sizes");
+  FPS_CHECK_ARG(b->n_req == 0 || (b->d_cu_q && b->d_cu_k), "cu arrays are NULL");
+  FPS_CHECK_ARG(b->mode == FPS_MODE_KV || b->mode == FPS_MODE_Y, "mode %d", b->mode);
+  if (b->mode == FPS_MODE_Y && b->total_u > 0)
+    FPS_CHECK_ARG(b->d_cu_u && b->d_u_src && b->d_u_row, "Y-mode needs cu_u/u_src/u_row");
+  return FPS_OK;
+}
+
+static fps_status block_forward(const fps_block_weights* w, const fps_varlen_batch* b,
+                                const void* x_act, void* y_act, void* kv, const void* xu,
+                                cudaEvent_t kv_ready, void* d_ws, size_t ws_bytes,
+                                cudaStream_t s) {
+  const int H = w->H, F = w->F, dt = w->dtype, tq = b->total_q;
+  const int tu = (b->mode == FPS_MODE_Y) ? b->total_u : 0;
+  const size_t e = elt_size(dt);
+  BlockWs ws;
+  const size_t need = ws_layout(H, F, dt, tq, tu, (char*)d_ws, &ws);
+  FPS_CHECK_ARG(ws_bytes >= need, "workspace %zu < %zu bytes", ws_bytes, need);
+  const char* mod = (const char*)b->d_mod;
+  auto modp = [&](int off) -> const void* { return mod ? mod + (size_t)off * H * e : nullptr; };
+
+  if (tq > 0) {
+    // a4: h1 = LN(x)(1+scale1)+shift1 on active rows
+    FPS_TRY(launch_ln_mod(dt, x_act, nullptr, tq, H, ws.h, b->d_cu_q, b->n_req, b->d_mod, 0, s));
+    // a5: [tq,H] x [3H,H]^T; Q -> compact, K|V -> merged key rows at original positions
+    Epilogue ep{};
+    ep.bias = w->b_qkv;
+    ep.out0 = ws.q; ep.ld0 = H; ep.map0 = nullptr;
+    ep.out1 = kv; ep.ld1 = 2 * H; ep.map1 = b->d_q_row;
+    ep.split = H;
+    FPS_TRY(launch_gemm(dt, ws.h, w->w_qkv, tq, 3 * H, H, ep, s));
+  }
+  if (tu > 0) {
+    // Y-mode: cached block-input rows U -> LN -> K|V projection (Fig. 5-Bottom, reading R5)
+    if (kv_ready) FPS_CUDA_TRY(cudaStreamWaitEvent(s, kv_ready, 0));
+    kv_ready = nullptr;
+    FPS_TRY(launch_ln_mod(dt, xu, b->d_u_src, tu, H, ws.hu, b->d_cu_u, b->n_req, b->d_mod, 0, s));
+    Epilogue ep{};
+    ep.bias = w->b_qkv ? (const char*)w->b_qkv + (size_t)H * e : nullptr;
+    ep.out0 = kv; ep.ld0 = 2 * H; ep.map0 = b->d_u_row;
+    ep.split = 2 * H;
+    FPS_TRY(launch_gemm(dt, ws.hu, (const char*)w->w_qkv + (size_t)H * H * e, tu, 2 * H, H, ep, s));
+  }
+  if (tq == 0) return FPS_OK;
+  // a6: queries from active rows only, keys = merged fresh + cached rows (L159)
+  if (kv_ready) FPS_CUDA_TRY(cudaStreamWaitEvent(s, kv_ready, 0));
+  FPS_TRY(launch_attention(dt, ws.q, kv, ws.ao, w->heads, w->head_dim, b->d_cu_q, b->d_cu_k,
+                           b->h_cu_q, b->h_cu_k, b->n_req, tq, b->max_q, b->max_k, s));
+  {  // a7: x1 = x + gate1 (A Wo^T + bo)
+    Epilogue ep{};
+    ep.bias = w->b_o;
+    ep.resid = x_act; ep.ld_resid = H;
+    ep.gate = modp(2); ep.gate_stride = 6 * H; ep.cu = b->d_cu_q; ep.n_req = b->n_req;
+    ep.out0 = ws.x1; ep.ld0 = H; ep.split = H;
+    FPS_TRY(launch_gemm(dt, ws.ao, w->w_o, tq, H, H, ep, s));
+  }
+  // a8: y = x1 + gate2 (GELU(LN(x1)(1+scale2)+shift2 W1^T + b1) W2^T + b2)
+  FPS_TRY(launch_ln_mod(dt, ws.x1, nullptr, tq, H, ws.h2, b->d_cu_q, b->n_req, b->d_mod, 3 * H, s));
+  {
+    Epilogue ep{};
+    ep.bias = w->b_up; ep.act = 1;
+    ep.out0 = ws.u; ep.ld0 = F; ep.split = F;
+    FPS_TRY(launch_gemm(dt, ws.h2, w->w_up, tq, F, H, ep, s));
+  }
+  {
+    Epilogue ep{};
+    ep.bias = w->b_down;
+    ep.resid = ws.x1; ep.ld_resid = H;
+    ep.gate = modp(5); ep.gate_stride = 6 * H; ep.cu = b->d_cu_q; ep.n_req = b->n_req;
+    ep.out0 = y_act; ep.ld0 = H; ep.split = H;
+    FPS_TRY(launch_gemm(dt, ws.u, w->w_down, tq, H, F, ep, s));
+  }
+  return FPS_OK;
+}
+
+}  // namespace fps
+
+using namespace fps;
+
+extern "C" {
+
+const char* fps_last_error(void) { return fps::g_err.c_str(); }
+int32_t fps_abi_version(void) { return FPS_ABI_VERSION; }
+
+int32_t fps_device_ok(void) {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  cudaDeviceProp p;
+  if (cudaGetDeviceProperties(&p, dev) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  return p.major == 10 && p.minor == 0 ? 1 : 0;
+}
+
+int64_t fps_launch_count(void) { return fps::g_launches; }
+void fps_set_disable_tc(int32_t flags) { fps::g_disable_tc = flags; }
+
+fps_status fps_build_mask_index(const uint8_t* d_masks, const int32_t* d_offsets, int32_t n_req,
+                                int32_t max_len, int32_t* d_masked_ids, int32_t* d_unmasked_ids,
+                                int32_t* d_n_masked, void* stream) {
+  FPS_CHECK_ARG(n_req >= 0, "n_req < 0");
+  if (n_req == 0) return FPS_OK;
+  FPS_CHECK_ARG(d_masks && d_offsets && d_masked_ids && d_unmasked_ids && d_n_masked,
+                "NULL pointer");
+  return launch_mask_index(d_masks, d_offsets, n_req, max_len, d_masked_ids, d_unmasked_ids,
+                           d_n_masked, as_stream(stream));
+}
+
+static fps_status check_rows(const void* src, const void* dst, int32_t n, int32_t row_bytes) {
+  FPS_CHECK_ARG(n >= 0, "n < 0");
+  FPS_CHECK_ARG(row_bytes > 0 && row_bytes % 16 == 0, "row_bytes %d not a positive multiple of 16",
+                row_bytes);
+  if (n == 0) return FPS_OK;
+  FPS_CHECK_ARG(src && dst, "NULL pointer");
+  FPS_CHECK_ARG(aligned16(src) && aligned16(dst), "pointers must be 16-byte aligned");
+  return FPS_OK;
+}
+
+fps_status fps_gather_rows(const void* d_src, const int32_t* d_ids, int32_t n, int32_t row_bytes,
+                           void* d_dst, void* stream) {
+  FPS_TRY(check_rows(d_src, d_dst, n, row_bytes));
+  FPS_CHECK_ARG(n == 0 || d_ids, "ids is NULL");
+  return launch_copy_rows(d_src, d_ids, nullptr, n, row_bytes, d_dst, as_stream(stream));
+}
+
+fps_status fps_scatter_rows(const void* d_src, const int32_t* d_ids, int32_t n, int32_t row_bytes,
+                            void* d_dst, void* stream) {
+  FPS_TRY(check_rows(d_src, d_dst, n, row_bytes));
+  FPS_CHECK_ARG(n == 0 || d_ids, "ids is NULL");
+  return launch_copy_rows(d_src, nullptr, d_ids, n, row_bytes, d_dst, as_stream(stream));
+}
+
+fps_status fps_copy_rows(const void* d_src, const int32_t* d_src_ids, const int32_t* d_dst_ids,
+                         int32_t n, int32_t row_bytes, void* d_dst, void* stream) {
+  FPS_TRY(check_rows(d_src, d_dst, n, row_bytes));
+  return launch_copy_rows(d_src, d_src_ids, d_dst_ids, n, row_bytes, d_dst, as_stream(stream));
+}
+
+size_t fps_block_workspace_bytes(int32_t H, int32_t F, int32_t dtype, int32_t max_q,
+                                 int32_t max_u) {
+  return ws_layout(H, F, dtype, max_q, max_u, nullptr, nullptr);
+}
+
+fps_status fps_masked_block_forward(const fps_block_weights* w, const fps_varlen_batch* b,
+                                    const void* d_x_act, void* d_y_act, void* d_kv,
+                                    const void* d_xu, void* kv_ready, void* d_ws, size_t ws_bytes,
+                                    void* stream) {
+  FPS_TRY(check_weights(w));
+  FPS_TRY(check_batch(b));
+  if (b->total_q > 0) FPS_CHECK_ARG(d_x_act && d_y_act && d_kv && d_ws, "NULL buffer");
+  if (b->mode == FPS_MODE_Y && b->total_u > 0) FPS_CHECK_ARG(d_xu && d_kv, "Y-mode needs d_xu");
+  if (b->total_q > 0 && b->d_q_row == nullptr)
+    FPS_CHECK_ARG(b->total_q == b->total_k, "d_q_row NULL requires total_q == total_k");
+  FPS_CHECK_ARG(w->heads * w->head_dim == w->H, "heads*head_dim != H");
+  return block_forward(w, b, d_x_act, d_y_act, d_kv, d_xu, (cudaEvent_t)kv_ready, d_ws, ws_bytes,
+                       as_stream(stream));
+}
+
+fps_status fps_dense_block_forward(const fps_block_weights* w, const fps_varlen_batch* b,
+                                   const void* d_x, void* d_y, void* d_kv, void* d_ws,
+                                   size_t ws_bytes, void* stream) {
+  FPS_TRY(check_weights(w));
+  FPS_TRY(check_batch(b));
+  FPS_CHECK_ARG(b->d_q_row == nullptr && b->total_q == b->total_k,
+                "dense block: d_q_row must be NULL and total_q == total_k");
+  fps_varlen_batch bb = *b;
+  bb.mode = FPS_MODE_KV;
+  bb.total_u = 0;
+  if (bb.total_q > 0) FPS_CHECK_ARG(d_x && d_y && d_kv && d_ws, "NULL buffer");
+  return block_forward(w, &bb, d_x, d_y, d_kv, nullptr, nullptr, d_ws, ws_bytes,
+                       as_stream(stream));
+}
+
+}  // extern "C"

@@ -1,0 +1,249 @@
+// a3: activation cache in pinned host DRAM + layer-ahead prefetch (PAPER.md L203 host-memory
+// store, L207 block granularity, L209 "while loading the i-th block, the computation stream
+// can concurrently execute the computation of the (i-1)-th block"; reading R7 keys).
+//
+// Two H2D methods (fps_cache_desc.copy_method):
+//  0  SM zero-copy gather: a few CTAs read the unmasked rows straight out of the mapped pinned
+//     arena over PCIe (16-B loads, many in flight) and write them to their token rows in HBM.
+//     One launch per layer for the whole batch, exact bytes, any mask shape.
+//  1  copy-engine DMA: the unmasked rows are coalesced into runs of consecutive tokens and
+//     issued as one cudaMemcpyBatchAsync (no SM time; per-run descriptor overhead).
+#include <algorithm>
+#include <vector>
+
+#include "kernels.h"
+
+struct fps_cache {
+  fps_cache_desc d;
+  int elt = 2;
+  size_t entry_bytes = 0;      // slot size (widest entry)
+  size_t row_bytes_main = 0;   // W * elt
+  size_t row_bytes_final = 0;  // H * elt (KV-mode final Y entry)
+  long long n_keys = 0;
+  long long n_entries = 0;
+  char* host = nullptr;        // pinned, mapped
+  char* dev_alias = nullptr;   // device pointer of `host`
+  std::vector<void*> dsts, srcs;
+  std::vector<size_t> sizes;
+};
+
+namespace fps {
+
+constexpr int kMaxPrefetchItems = 32;
+
+struct PrefetchBatch {
+  const uint4* src[kMaxPrefetchItems];
+  const int32_t* rows[kMaxPrefetchItems];
+  uint4* dst[kMaxPrefetchItems];
+  long long start[kMaxPrefetchItems + 1];   // prefix sums of vectors per item
+  int vpr[kMaxPrefetchItems];
+  int n_items;
+};
+
+__global__ void __launch_bounds__(256) prefetch_kernel(const __grid_constant__ PrefetchBatch b) {
+  const long long total = b.start[b.n_items];
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long i0 = (long long)blockIdx.x * blockDim.x + threadIdx.x; i0 < total;
+       i0 += 4 * stride) {
+    uint4 v[4];
+    uint4* dp[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const long long i = i0 + u * stride;
+      dp[u] = nullptr;
+      if (i < total) {
+        int it = 0;
+        while (i >= b.start[it + 1]) ++it;
+        const long long local = i - b.start[it];
+        const int vpr = b.vpr[it];
+        const int rr = (int)(local / vpr), c = (int)(local - (long long)rr * vpr);
+        const long long row = __ldg(b.rows[it] + rr);
+        v[u] = b.src[it][row * vpr + c];
+        dp[u] = b.dst[it] + row * vpr + c;
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if (dp[u]) *dp[u] = v[u];
+  }
+}
+
+static long long key_of(const fps_cache* c, uint32_t t, int step, int layer) {
+  const int per_step = c->d.n_layers + (c->d.mode == FPS_MODE_KV ? 1 : 0);
+  return ((long long)t * c->d.n_steps + step) * per_step + layer;
+}
+
+static bool key_ok(const fps_cache* c, uint32_t t, int step, int layer) {
+  const int max_layer = c->d.n_layers + (c->d.mode == FPS_MODE_KV ? 1 : 0);
+  return (int)t < c->d.n_templates && step >= 0 && step < c->d.n_steps && layer >= 0 &&
+         layer < max_layer;
+}
+
+static size_t row_bytes_of(const fps_cache* c, int layer) {
+  return (c->d.mode == FPS_MODE_KV && layer == c->d.n_layers) ? c->row_bytes_final
+                                                              : c->row_bytes_main;
+}
+
+static size_t offset_of(const fps_cache* c, uint32_t t, int step, int layer) {
+  return (size_t)(key_of(c, t, step, layer) % c->n_entries) * c->entry_bytes;
+}
+
+}  // namespace fps
+
+using namespace fps;
+
+extern "C" {
+
+fps_status fps_cache_create(const fps_cache_desc* desc, fps_cache_t* out) {
+  FPS_CHECK_ARG(desc && out, "NULL argument");
+  const fps_cache_desc& d = *desc;
+  FPS_CHECK_ARG(d.mode == FPS_MODE_KV || d.mode == FPS_MODE_Y, "mode %d", d.mode);
+  FPS_CHECK_ARG(d.dtype == FPS_BF16 || d.dtype == FPS_F32, "dtype %d", d.dtype);
+  FPS_CHECK_ARG(d.H > 0 && d.L_img > 0 && d.n_layers > 0 && d.n_steps > 0 && d.n_templates > 0,
+                "sizes must be positive");
+  FPS_CHECK_ARG(d.n_entries >= 0 && (d.copy_method == 0 || d.copy_method == 1), "bad desc");
+  auto* c = new (std::nothrow) fps_cache();
+  if (!c) return fail(FPS_ENOMEM, "cache: host allocation");
+  c->d = d;
+  c->elt = d.dtype == FPS_BF16 ? 2 : 4;
+  c->row_bytes_main = (size_t)(d.mode == FPS_MODE_KV ? 2 : 1) * d.H * c->elt;
+  c->row_bytes_final = (size_t)d.H * c->elt;
+  c->entry_bytes = (size_t)d.L_img * c->row_bytes_main;
+  const int per_step = d.n_layers + (d.mode == FPS_MODE_KV ? 1 : 0);
+  c->n_keys = (long long)d.n_templates * d.n_steps * per_step;
+  c->n_entries = d.n_entries > 0 ? std::min<long long>(d.n_entries, c->n_keys) : c->n_keys;
+  const size_t bytes = (size_t)c->n_entries * c->entry_bytes;
+  cudaError_t e = cudaHostAlloc((void**)&c->host, bytes, cudaHostAllocMapped | cudaHostAllocPortable);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    delete c;
+    return fail(e == cudaErrorMemoryAllocation ? FPS_ENOMEM : FPS_ECUDA,
+                "cache: cudaHostAlloc(%zu bytes): %s", bytes, cudaGetErrorString(e));
+  }
+  e = cudaHostGetDevicePointer((void**)&c->dev_alias, c->host, 0);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    cudaFreeHost(c->host);
+    delete c;
+    return fail(FPS_ECUDA, "cache: cudaHostGetDevicePointer: %s", cudaGetErrorString(e));
+  }
+  *out = c;
+  return FPS_OK;
+}
+
+fps_status fps_cache_destroy(fps_cache_t c) {
+  if (!c) return FPS_OK;
+  if (c->host) cudaFreeHost(c->host);
+  delete c;
+  return FPS_OK;
+}
+
+void* fps_cache_entry_host_ptr(fps_cache_t c, uint32_t template_id, int32_t step, int32_t layer) {
+  if (!c || !key_ok(c, template_id, step, layer)) return nullptr;
+  return c->host + offset_of(c, template_id, step, layer);
+}
+
+size_t fps_cache_entry_bytes(fps_cache_t c, int32_t layer) {
+  if (!c) return 0;
+  return (size_t)c->d.L_img * row_bytes_of(c, layer);
+}
+
+fps_status fps_cache_store(fps_cache_t c, uint32_t template_id, int32_t step, int32_t layer,
+                           const void* d_src, int32_t src_row_bytes, void* stream) {
+  FPS_CHECK_ARG(c && d_src, "NULL argument");
+  FPS_CHECK_ARG(key_ok(c, template_id, step, layer), "key (%u,%d,%d) out of range", template_id,
+                step, layer);
+  const size_t rb = row_bytes_of(c, layer);
+  FPS_CHECK_ARG(src_row_bytes >= (int)rb, "src_row_bytes %d < %zu", src_row_bytes, rb);
+  FPS_CUDA_TRY(cudaMemcpy2DAsync(c->host + offset_of(c, template_id, step, layer), rb, d_src,
+                                 src_row_bytes, rb, c->d.L_img, cudaMemcpyDeviceToHost,
+                                 as_stream(stream)));
+  return FPS_OK;
+}
+
+fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int32_t n_items,
+                              void* load_stream, void* ready_event) {
+  FPS_CHECK_ARG(c, "NULL cache");
+  FPS_CHECK_ARG(n_items >= 0 && (n_items == 0 || items), "bad items");
+  cudaStream_t s = as_stream(load_stream);
+  for (int i = 0; i < n_items; ++i) {
+    const fps_prefetch_item& it = items[i];
+    FPS_CHECK_ARG(key_ok(c, it.template_id, it.step, it.layer), "item %d: key out of range", i);
+    FPS_CHECK_ARG(it.n_rows >= 0 && it.n_rows <= c->d.L_img, "item %d: n_rows %d", i, it.n_rows);
+    FPS_CHECK_ARG(it.n_rows == 0 || it.d_dst, "item %d: NULL dst", i);
+    FPS_CHECK_ARG(it.dst_row_bytes == (int)row_bytes_of(c, it.layer),
+                  "item %d: dst_row_bytes %d != entry row bytes %zu", i, it.dst_row_bytes,
+                  row_bytes_of(c, it.layer));
+    if (c->d.copy_method == 0) FPS_CHECK_ARG(it.n_rows == 0 || it.d_rows, "item %d: d_rows", i);
+    else FPS_CHECK_ARG(it.n_rows == 0 || it.h_rows, "item %d: h_rows needed for DMA", i);
+  }
+  if (c->d.copy_method == 0) {
+    for (int base = 0; base < n_items; base += kMaxPrefetchItems) {
+      PrefetchBatch b{};
+      long long acc = 0;
+      int k = 0;
+      for (int i = base; i < n_items && k < kMaxPrefetchItems; ++i) {
+        const fps_prefetch_item& it = items[i];
+        if (it.n_rows == 0) continue;
+        const int vpr = (int)(row_bytes_of(c, it.layer) / 16);
+        b.src[k] = reinterpret_cast<const uint4*>(c->dev_alias +
+                                                  offset_of(c, it.template_id, it.step, it.layer));
+        b.rows[k] = it.d_rows;
+        b.dst[k] = reinterpret_cast<uint4*>(it.d_dst);
+        b.vpr[k] = vpr;
+        b.start[k] = acc;
+        acc += (long long)it.n_rows * vpr;
+        ++k;
+      }
+      b.start[k] = acc;
+      b.n_items = k;
+      if (acc == 0) continue;
+      int ctas = c->d.copy_ctas > 0 ? c->d.copy_ctas : 32;
+      long long want = (acc + 1023) / 1024;
+      if (want < ctas) ctas = (int)want;
+      prefetch_kernel<<<ctas, 256, 0, s>>>(b);
+      count_launch();
+      FPS_LAUNCH_CHECK();
+    }
+  } else {
+    c->dsts.clear();
+    c->srcs.clear();
+    c->sizes.clear();
+    for (int i = 0; i < n_items; ++i) {
+      const fps_prefetch_item& it = items[i];
+      const size_t rb = row_bytes_of(c, it.layer);
+      char* src = c->host + offset_of(c, it.template_id, it.step, it.layer);
+      char* dst = (char*)it.d_dst;
+      int j = 0;
+      while (j < it.n_rows) {
+        int k = j;
+        while (k + 1 < it.n_rows && it.h_rows[k + 1] == it.h_rows[k] + 1) ++k;
+        const size_t r0 = (size_t)it.h_rows[j];
+        c->dsts.push_back(dst + r0 * rb);
+        c->srcs.push_back(src + r0 * rb);
+        c->sizes.push_back((size_t)(k - j + 1) * rb);
+        j = k + 1;
+      }
+    }
+    if (!c->sizes.empty()) {
+      cudaMemcpyAttributes attr{};
+      attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
+      attr.srcLocHint.type = cudaMemLocationTypeHost;
+      attr.dstLocHint.type = cudaMemLocationTypeDevice;
+      attr.flags = cudaMemcpyFlagPreferOverlapWithCompute;
+      size_t attr_idx = 0, fail_idx = 0;
+      cudaError_t e = cudaMemcpyBatchAsync(c->dsts.data(), c->srcs.data(), c->sizes.data(),
+                                           c->sizes.size(), &attr, &attr_idx, 1, &fail_idx, s);
+      if (e != cudaSuccess) {
+        cudaGetLastError();
+        for (size_t q = 0; q < c->sizes.size(); ++q)
+          FPS_CUDA_TRY(cudaMemcpyAsync(c->dsts[q], c->srcs[q], c->sizes[q],
+                                       cudaMemcpyHostToDevice, s));
+      }
+    }
+  }
+  if (ready_event) FPS_CUDA_TRY(cudaEventRecord((cudaEvent_t)ready_event, s));
+  return FPS_OK;
+}
+
+}  // extern "C"

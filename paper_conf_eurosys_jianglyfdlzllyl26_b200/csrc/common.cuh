@@ -1,0 +1,159 @@
+// Shared device/host helpers for libflashps (sm_100a). Internal header.
+#pragma once
+
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <cstdarg>
+#include <cstdio>
+#include <string>
+
+#include "../../include/flashps.h"
+
+namespace fps {
+
+// ---- error reporting (thread-local last error) ----------------------------------------
+void set_error(const char* fmt, ...);
+fps_status fail(fps_status code, const char* fmt, ...);
+
+#define FPS_CHECK_ARG(cond, ...)                              \
+  do {                                                        \
+    if (!(cond)) return ::fps::fail(FPS_EINVAL, __VA_ARGS__); \
+  } while (0)
+
+#define FPS_CUDA_TRY(expr)                                                                  \
+  do {                                                                                      \
+    cudaError_t _e = (expr);                                                                \
+    if (_e != cudaSuccess)                                                                  \
+      return ::fps::fail(FPS_ECUDA, "%s:%d %s: %s", __FILE__, __LINE__, #expr,              \
+                         cudaGetErrorString(_e));                                           \
+  } while (0)
+
+#define FPS_LAUNCH_CHECK()                                                                  \
+  do {                                                                                      \
+    cudaError_t _e = cudaGetLastError();                                                    \
+    if (_e != cudaSuccess)                                                                  \
+      return ::fps::fail(FPS_ECUDA, "%s:%d launch: %s", __FILE__, __LINE__,                 \
+                         cudaGetErrorString(_e));                                           \
+  } while (0)
+
+#define FPS_TRY(expr)                     \
+  do {                                    \
+    fps_status _s = (expr);               \
+    if (_s != FPS_OK) return _s;          \
+  } while (0)
+
+inline cudaStream_t as_stream(void* s) { return reinterpret_cast<cudaStream_t>(s); }
+inline bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+inline int ceil_div(long a, long b) { return (int)((a + b - 1) / b); }
+
+// Counts kernels launched through the library (for the bench's gpu_launches claim).
+extern thread_local long long g_launches;
+inline void count_launch(int n = 1) { g_launches += n; }
+
+constexpr int kNumSMs = 148;
+
+// ---- element access ----------------------------------------------------------------------
+template <typename T> struct Elt;
+template <> struct Elt<float> {
+  __device__ __forceinline__ static float load(const float* p) { return *p; }
+  __device__ __forceinline__ static void store(float* p, float v) { *p = v; }
+  static constexpr int dtype = FPS_F32;
+};
+template <> struct Elt<__nv_bfloat16> {
+  __device__ __forceinline__ static float load(const __nv_bfloat16* p) { return __bfloat162float(*p); }
+  __device__ __forceinline__ static void store(__nv_bfloat16* p, float v) { *p = __float2bfloat16_rn(v); }
+  static constexpr int dtype = FPS_BF16;
+};
+
+__device__ __forceinline__ float to_f(float v) { return v; }
+__device__ __forceinline__ float to_f(__nv_bfloat16 v) { return __bfloat162float(v); }
+template <typename T> __device__ __forceinline__ T from_f(float v);
+template <> __device__ __forceinline__ float from_f<float>(float v) { return v; }
+template <> __device__ __forceinline__ __nv_bfloat16 from_f<__nv_bfloat16>(float v) {
+  return __float2bfloat16_rn(v);
+}
+
+// 16-byte vector <-> floats
+template <typename T> struct Vec16;
+template <> struct Vec16<float> {
+  static constexpr int N = 4;
+  __device__ __forceinline__ static void unpack(const uint4& u, float* f) {
+    f[0] = __uint_as_float(u.x); f[1] = __uint_as_float(u.y);
+    f[2] = __uint_as_float(u.z); f[3] = __uint_as_float(u.w);
+  }
+  __device__ __forceinline__ static uint4 pack(const float* f) {
+    return make_uint4(__float_as_uint(f[0]), __float_as_uint(f[1]), __float_as_uint(f[2]),
+                      __float_as_uint(f[3]));
+  }
+};
+__device__ __forceinline__ uint32_t pack_bf16x2(float lo, float hi) {
+  __nv_bfloat162 v = __floats2bfloat162_rn(lo, hi);
+  return *reinterpret_cast<uint32_t*>(&v);
+}
+__device__ __forceinline__ void unpack_bf16x2(uint32_t u, float& lo, float& hi) {
+  lo = __uint_as_float(u << 16);
+  hi = __uint_as_float(u & 0xffff0000u);
+}
+template <> struct Vec16<__nv_bfloat16> {
+  static constexpr int N = 8;
+  __device__ __forceinline__ static void unpack(const uint4& u, float* f) {
+    unpack_bf16x2(u.x, f[0], f[1]); unpack_bf16x2(u.y, f[2], f[3]);
+    unpack_bf16x2(u.z, f[4], f[5]); unpack_bf16x2(u.w, f[6], f[7]);
+  }
+  __device__ __forceinline__ static uint4 pack(const float* f) {
+    return make_uint4(pack_bf16x2(f[0], f[1]), pack_bf16x2(f[2], f[3]), pack_bf16x2(f[4], f[5]),
+                      pack_bf16x2(f[6], f[7]));
+  }
+};
+
+__device__ __forceinline__ float warp_sum(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+__device__ __forceinline__ float warp_max(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+
+// Request owning row `i` of a prefix-sum array cu[0..n_req] (largest r with cu[r] <= i).
+__device__ __forceinline__ int find_req(const int32_t* __restrict__ cu, int n_req, int i) {
+  int lo = 0, hi = n_req - 1;
+  while (lo < hi) {
+    int mid = (lo + hi + 1) >> 1;
+    if (__ldg(cu + mid) <= i) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+
+__device__ __forceinline__ float gelu_tanh(float x) {
+  const float k0 = 0.7978845608028654f, k1 = 0.044715f;
+  float u = k0 * (x + k1 * x * x * x);
+  return 0.5f * x * (1.0f + tanhf(u));
+}
+
+// ---- GEMM epilogue description (shared by the SIMT and tcgen05 GEMMs) --------------------
+// out[r, c] = epilogue(acc[r, c]) with
+//   v = acc + bias[c]
+//   act == 1: v = GELU_tanh(v)
+//   resid: v = resid[r, c] + gate[req(r), c] * v      (gate NULL -> 1)
+//   routing: columns [0, split) -> out0 (row r, ld0), columns [split, N) -> out1 with row
+//            map1[r] (NULL -> r), column c - split, ld1.  split = N when there is no out1.
+struct Epilogue {
+  const void* bias;          // [N] or null
+  int act;                   // 0 none, 1 gelu_tanh
+  const void* resid;         // [M, ld_resid] or null
+  int ld_resid;
+  const void* gate;          // per-request gate vectors: gate + req * gate_stride, or null
+  int gate_stride;
+  const int32_t* cu;         // request prefix sums over rows (for gate lookup)
+  int n_req;
+  void* out0; int ld0; const int32_t* map0;   // map0: output row for row r (null -> r)
+  void* out1; int ld1; const int32_t* map1;
+  int split;
+};
+
+}  // namespace fps

@@ -1,0 +1,517 @@
+// fps_run_batch: step-level continuous batching over a stack of N mask-aware blocks with the
+// layer-ahead cache pipeline (§4.2 Fig. 9, L237 §4.3).
+//
+// One call = admission (mask index of every request, one host sync to size the varlen batch),
+// then denoising steps.  Per step:
+//   plan     Alg. 1 (planner.cpp) over per-layer costs of this batch (cost model {a,b,c,e});
+//   load     stream: for every cached block, in block order, the unmasked rows of each request's
+//            entry (template, step_r, block) are copied into a ring of `slots` staging buffers;
+//            load j reuses a slot only after the compute stream has consumed load j - slots;
+//   compute  stream: cached blocks run fps_masked_block_forward (waiting for their load only
+//            right before the first kernel that reads cached rows); uncached blocks run the dense
+//            block on all tokens (L211); transitions gather / rebuild rows;
+//   replenish: y[M] from the last block, y[U] from the cache (L157); Euler x += delta_s y (R21).
+#include <algorithm>
+#include <cstring>
+#include <vector>
+
+#include "kernels.h"
+
+struct fps_engine {
+  fps_engine_desc d{};
+  std::vector<fps_block_weights> layers;
+  std::vector<float> deltas;
+  std::vector<uint8_t> fixed_plan;
+  int L = 0, elt = 2, W = 0, D = 0;
+  size_t row_h = 0, row_w = 0;  // bytes of an H row / a W row
+  int maxR = 0;                 // max_batch * L rows
+  // device buffers
+  char *x_full = nullptr, *full[2] = {nullptr, nullptr}, *y_full = nullptr, *act[2] = {nullptr, nullptr};
+  char *kv_scratch = nullptr, *final_slot = nullptr, *ws = nullptr, *mod_batch = nullptr;
+  std::vector<char*> slots;
+  size_t ws_bytes = 0;
+  uint8_t* d_masks = nullptr;
+  int32_t *d_off = nullptr, *d_mids = nullptr, *d_uids = nullptr, *d_nm = nullptr;
+  int32_t *d_meta = nullptr;   // cu_q | cu_k | cu_u | q_row | u_row | mod_ids
+  float* d_delta = nullptr;
+  // pinned host staging
+  int32_t* h_meta = nullptr;
+  int32_t *h_mids = nullptr, *h_uids = nullptr, *h_nm = nullptr, *h_off = nullptr;
+  float* h_delta = nullptr;
+  std::vector<cudaEvent_t> ready, consumed;
+  cudaEvent_t step_start = nullptr, admit_done = nullptr;
+  std::vector<uint8_t> last_plan;
+  double last_latency = 0.0;
+  long long last_launches = 0;
+};
+
+namespace fps {
+
+static void free_engine(fps_engine* e) {
+  if (!e) return;
+  char* bufs[] = {e->x_full, e->full[0], e->full[1], e->y_full, e->act[0], e->act[1],
+                  e->kv_scratch, e->final_slot, e->ws, e->mod_batch};
+  for (char* p : bufs) if (p) cudaFree(p);
+  for (char* p : e->slots) if (p) cudaFree(p);
+  if (e->d_masks) cudaFree(e->d_masks);
+  int32_t* ib[] = {e->d_off, e->d_mids, e->d_uids, e->d_nm, e->d_meta};
+  for (int32_t* p : ib) if (p) cudaFree(p);
+  if (e->d_delta) cudaFree(e->d_delta);
+  void* hb[] = {e->h_meta, e->h_mids, e->h_uids, e->h_nm, e->h_off, e->h_delta};
+  for (void* p : hb) if (p) cudaFreeHost(p);
+  for (auto ev : e->ready) if (ev) cudaEventDestroy(ev);
+  for (auto ev : e->consumed) if (ev) cudaEventDestroy(ev);
+  if (e->step_start) cudaEventDestroy(e->step_start);
+  if (e->admit_done) cudaEventDestroy(e->admit_done);
+  delete e;
+}
+
+// Per-block FLOPs of one request (Table 1, exact per mode; oracle/counters.py restated).
+static double flops_block(int mode, double n, double L, double H, double F) {
+  const double attn = 4.0 * n * L * H;
+  if (mode == FPS_MODE_KV) return 8.0 * n * H * H + 4.0 * n * H * F + attn;
+  return 4.0 * n * H * H + 4.0 * L * H * H + 4.0 * n * H * F + attn;
+}
+
+}  // namespace fps
+
+using namespace fps;
+
+extern "C" {
+
+fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out) {
+  FPS_CHECK_ARG(desc && out, "NULL argument");
+  const fps_engine_desc& d = *desc;
+  FPS_CHECK_ARG(d.H > 0 && d.heads > 0 && d.H % d.heads == 0 && d.F > 0 && d.n_layers > 0,
+                "bad dims");
+  FPS_CHECK_ARG(d.dtype == FPS_BF16 || d.dtype == FPS_F32, "dtype");
+  FPS_CHECK_ARG(d.mode == FPS_MODE_KV || d.mode == FPS_MODE_Y, "mode");
+  FPS_CHECK_ARG(d.L_img > 0 && d.L_txt >= 0 && d.max_batch > 0 && d.n_steps > 0, "bad sizes");
+  FPS_CHECK_ARG(d.layers && d.h_deltas && d.cache, "layers, h_deltas and cache are required");
+  FPS_CHECK_ARG(d.plan_policy >= 0 && d.plan_policy <= 3, "plan_policy");
+  FPS_CHECK_ARG(d.plan_policy != 3 || d.h_plan, "plan_policy 3 needs h_plan");
+  if (d.plan_policy == 3 && d.mode == FPS_MODE_KV) {
+    bool seen = false;
+    for (int l = 0; l < d.n_layers; ++l) {
+      if (d.h_plan[l]) seen = true;
+      else FPS_CHECK_ARG(!seen, "KV-mode plan must be monotone (reading R11)");
+    }
+  }
+  auto* e = new (std::nothrow) fps_engine();
+  if (!e) return fail(FPS_ENOMEM, "engine alloc");
+  e->d = d;
+  e->layers.assign(d.layers, d.layers + d.n_layers);
+  e->deltas.assign(d.h_deltas, d.h_deltas + d.n_steps);
+  if (d.plan_policy == 3) e->fixed_plan.assign(d.h_plan, d.h_plan + d.n_layers);
+  e->d.layers = nullptr;
+  e->d.h_deltas = nullptr;
+  e->d.h_plan = nullptr;
+  e->L = d.L_img + d.L_txt;
+  e->elt = d.dtype == FPS_BF16 ? 2 : 4;
+  e->W = d.mode == FPS_MODE_KV ? 2 * d.H : d.H;
+  e->row_h = (size_t)d.H * e->elt;
+  e->row_w = (size_t)e->W * e->elt;
+  e->maxR = d.max_batch * e->L;
+  const size_t R = e->maxR;
+  size_t slot_bytes = R * e->row_w;
+  int D = d.slots > 0 ? d.slots : d.n_layers;
+  if (d.slots <= 0) {
+    const size_t budget = (size_t)16 << 30;
+    D = (int)std::max<size_t>(2, std::min<size_t>(d.n_layers, budget / std::max<size_t>(slot_bytes, 1)));
+  }
+  e->D = std::min(D, d.n_layers);
+  cudaError_t err = cudaSuccess;
+  auto dmal = [&](char** p, size_t bytes) {
+    if (err == cudaSuccess) err = cudaMalloc((void**)p, std::max<size_t>(bytes, 256));
+  };
+  dmal(&e->x_full, R * e->row_h);
+  dmal(&e->full[0], R * e->row_h);
+  dmal(&e->full[1], R * e->row_h);
+  dmal(&e->y_full, R * e->row_h);
+  dmal(&e->act[0], R * e->row_h);
+  dmal(&e->act[1], R * e->row_h);
+  dmal(&e->kv_scratch, R * 2 * e->row_h);
+  if (d.mode == FPS_MODE_KV) dmal(&e->final_slot, R * e->row_h);
+  e->ws_bytes = fps_block_workspace_bytes(d.H, d.F, d.dtype, (int)R, (int)R);
+  dmal(&e->ws, e->ws_bytes);
+  dmal(&e->mod_batch, (size_t)d.n_layers * d.max_batch * 6 * e->row_h);
+  e->slots.assign(e->D, nullptr);
+  for (int i = 0; i < e->D; ++i) dmal(&e->slots[i], slot_bytes);
+  if (err == cudaSuccess) err = cudaMalloc((void**)&e->d_masks, R);
+  const size_t meta_ints = 3 * (d.max_batch + 1) + 2 * R + (size_t)d.n_layers * d.max_batch;
+  auto imal = [&](int32_t** p, size_t n) {
+    if (err == cudaSuccess) err = cudaMalloc((void**)p, std::max<size_t>(n, 1) * 4);
+  };
+  imal(&e->d_off, d.max_batch + 1);
+  imal(&e->d_mids, R);
+  imal(&e->d_uids, R);
+  imal(&e->d_nm, d.max_batch);
+  imal(&e->d_meta, meta_ints);
+  if (err == cudaSuccess) err = cudaMalloc((void**)&e->d_delta, d.max_batch * 4);
+  auto hmal = [&](void** p, size_t bytes) {
+    if (err == cudaSuccess) err = cudaHostAlloc(p, std::max<size_t>(bytes, 16), cudaHostAllocDefault);
+  };
+  hmal((void**)&e->h_meta, meta_ints * 4);
+  hmal((void**)&e->h_mids, R * 4);
+  hmal((void**)&e->h_uids, R * 4);
+  hmal((void**)&e->h_nm, d.max_batch * 4);
+  hmal((void**)&e->h_off, (d.max_batch + 1) * 4);
+  hmal((void**)&e->h_delta, d.max_batch * 4);
+  e->ready.assign(d.n_layers + 1, nullptr);
+  e->consumed.assign(d.n_layers + 1, nullptr);
+  for (int i = 0; i <= d.n_layers && err == cudaSuccess; ++i) {
+    err = cudaEventCreateWithFlags(&e->ready[i], cudaEventDisableTiming);
+    if (err == cudaSuccess) err = cudaEventCreateWithFlags(&e->consumed[i], cudaEventDisableTiming);
+  }
+  if (err == cudaSuccess) err = cudaEventCreateWithFlags(&e->step_start, cudaEventDisableTiming);
+  if (err == cudaSuccess) err = cudaEventCreateWithFlags(&e->admit_done, cudaEventDisableTiming);
+  if (err != cudaSuccess) {
+    cudaGetLastError();
+    free_engine(e);
+    return fail(err == cudaErrorMemoryAllocation ? FPS_ENOMEM : FPS_ECUDA, "engine create: %s",
+                cudaGetErrorString(err));
+  }
+  *out = e;
+  return FPS_OK;
+}
+
+fps_status fps_engine_destroy(fps_engine_t e) {
+  free_engine(e);
+  return FPS_OK;
+}
+
+fps_status fps_engine_last_plan(fps_engine_t e, uint8_t* use_cache, double* latency_ms) {
+  FPS_CHECK_ARG(e, "NULL engine");
+  if (use_cache)
+    for (size_t i = 0; i < e->last_plan.size(); ++i) use_cache[i] = e->last_plan[i];
+  if (latency_ms) *latency_ms = e->last_latency;
+  return FPS_OK;
+}
+
+int64_t fps_engine_last_launches(fps_engine_t e) { return e ? e->last_launches : -1; }
+
+}  // extern "C"
+
+namespace fps {
+
+struct Batch {
+  int n = 0;                       // requests in the running batch
+  std::vector<int> idx;            // index into the caller's reqs[]
+  std::vector<int> nq, nu;         // active / unmasked rows per request
+  int tq = 0, tu = 0, tk = 0, max_q = 0;
+  int32_t *cu_q, *cu_k, *cu_u, *q_row, *u_row, *mod_ids;      // device (inside d_meta)
+  int32_t *h_cu_q, *h_cu_k, *h_cu_u;                          // host (inside h_meta)
+};
+
+static fps_status admit(fps_engine* e, fps_request* reqs, const std::vector<int>& live, Batch& B,
+                        cudaStream_t cs) {
+  const int L = e->L, n = (int)live.size();
+  B.n = n;
+  B.idx = live;
+  for (int i = 0; i < n; ++i) {
+    FPS_CUDA_TRY(cudaMemcpyAsync(e->d_masks + (size_t)i * L, reqs[live[i]].d_mask, L,
+                                 cudaMemcpyDeviceToDevice, cs));
+    e->h_off[i] = i * L;
+  }
+  e->h_off[n] = n * L;
+  FPS_CUDA_TRY(cudaMemcpyAsync(e->d_off, e->h_off, (n + 1) * 4, cudaMemcpyHostToDevice, cs));
+  FPS_TRY(launch_mask_index(e->d_masks, e->d_off, n, L, e->d_mids, e->d_uids, e->d_nm, cs));
+  FPS_CUDA_TRY(cudaMemcpyAsync(e->h_nm, e->d_nm, n * 4, cudaMemcpyDeviceToHost, cs));
+  FPS_CUDA_TRY(cudaMemcpyAsync(e->h_mids, e->d_mids, (size_t)n * L * 4, cudaMemcpyDeviceToHost, cs));
+  FPS_CUDA_TRY(cudaMemcpyAsync(e->h_uids, e->d_uids, (size_t)n * L * 4, cudaMemcpyDeviceToHost, cs));
+  FPS_CUDA_TRY(cudaEventRecord(e->admit_done, cs));
+  FPS_CUDA_TRY(cudaEventSynchronize(e->admit_done));   // the one admission sync
+  // host metadata, laid out in h_meta exactly like d_meta
+  const int nb = e->d.max_batch;
+  int32_t* m = e->h_meta;
+  int32_t *cu_q = m, *cu_k = m + (nb + 1), *cu_u = m + 2 * (nb + 1);
+  int32_t* q_row = m + 3 * (nb + 1);
+  int32_t* u_row = q_row + e->maxR;
+  int32_t* mod_ids = u_row + e->maxR;
+  B.nq.assign(n, 0);
+  B.nu.assign(n, 0);
+  cu_q[0] = cu_k[0] = cu_u[0] = 0;
+  B.max_q = 0;
+  for (int i = 0; i < n; ++i) {
+    const int nq = e->h_nm[i], nu = L - nq;
+    B.nq[i] = nq;
+    B.nu[i] = nu;
+    for (int j = 0; j < nq; ++j) q_row[cu_q[i] + j] = i * L + e->h_mids[i * L + j];
+    for (int j = 0; j < nu; ++j) u_row[cu_u[i] + j] = i * L + e->h_uids[i * L + j];
+    cu_q[i + 1] = cu_q[i] + nq;
+    cu_k[i + 1] = cu_k[i] + L;
+    cu_u[i + 1] = cu_u[i] + nu;
+    B.max_q = std::max(B.max_q, nq);
+  }
+  B.tq = cu_q[n];
+  B.tk = cu_k[n];
+  B.tu = cu_u[n];
+  (void)mod_ids;
+  FPS_CUDA_TRY(cudaMemcpyAsync(e->d_meta, e->h_meta,
+                               (size_t)(3 * (nb + 1) + 2 * e->maxR) * 4, cudaMemcpyHostToDevice, cs));
+  int32_t* dm = e->d_meta;
+  B.cu_q = dm;
+  B.cu_k = dm + (nb + 1);
+  B.cu_u = dm + 2 * (nb + 1);
+  B.q_row = dm + 3 * (nb + 1);
+  B.u_row = B.q_row + e->maxR;
+  B.mod_ids = B.u_row + e->maxR;
+  B.h_cu_q = cu_q;
+  B.h_cu_k = cu_k;
+  B.h_cu_u = cu_u;
+  return FPS_OK;
+}
+
+static void make_plan(fps_engine* e, const Batch& B) {
+  const int N = e->d.n_layers;
+  e->last_plan.assign(N, 0);
+  const double a = e->d.cost_model[0] > 0 ? e->d.cost_model[0] : 1.0 / 1.0e12;  // ms per FLOP
+  const double b = e->d.cost_model[1] > 0 ? e->d.cost_model[1] : 0.01;
+  const double c = e->d.cost_model[2] > 0 ? e->d.cost_model[2] : 1.0 / 5.0e7;   // ms per byte
+  const double ec = e->d.cost_model[3] > 0 ? e->d.cost_model[3] : 0.01;
+  double fm = 0, fd = 0, by = 0, byf = 0;
+  const double H = e->d.H, F = e->d.F, L = e->L;
+  for (int i = 0; i < B.n; ++i) {
+    fm += flops_block(e->d.mode, B.nq[i], L, H, F);
+    fd += flops_block(FPS_MODE_KV, L, L, H, F);
+    by += (double)B.nu[i] * e->row_w;
+    byf += (double)B.nu[i] * e->row_h;
+  }
+  std::vector<double> Cw(N, a * fm + b), Cwo(N, a * fd + b), Lm(N, by > 0 ? c * by + ec : 0.0);
+  const double fin = byf > 0 ? c * byf + ec : 0.0;
+  if (e->d.plan_policy == 0) {
+    fps_plan_pipeline(Cw.data(), Cwo.data(), Lm.data(), N, e->d.mode, fin, e->last_plan.data(),
+                      &e->last_latency);
+  } else {
+    for (int l = 0; l < N; ++l)
+      e->last_plan[l] = e->d.plan_policy == 1 ? 1 : e->d.plan_policy == 2 ? 0 : e->fixed_plan[l];
+    e->last_latency = fps_pipeline_latency(e->last_plan.data(), Cw.data(), Cwo.data(), Lm.data(),
+                                           N, e->d.mode, fin);
+  }
+}
+
+// One denoising step of the running batch.
+static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStream_t cs,
+                           cudaStream_t ls) {
+  const int N = e->d.n_layers, n = B.n, H = e->d.H;
+  const bool kv = e->d.mode == FPS_MODE_KV;
+  const std::vector<uint8_t>& use = e->last_plan;
+  // adaLN vectors of every block for every request at its own step (rows of the table)
+  if (e->d.d_mod_table) {
+    int32_t* mod_ids = e->h_meta + 3 * (e->d.max_batch + 1) + 2 * e->maxR;
+    for (int l = 0; l < N; ++l)
+      for (int i = 0; i < n; ++i) mod_ids[l * n + i] = l * e->d.n_steps + reqs[B.idx[i]].step;
+    FPS_CUDA_TRY(cudaMemcpyAsync(B.mod_ids, mod_ids, (size_t)N * n * 4, cudaMemcpyHostToDevice, cs));
+    FPS_TRY(launch_copy_rows(e->d.d_mod_table, B.mod_ids, nullptr, N * n, 6 * (int)e->row_h,
+                             e->mod_batch, cs));
+  }
+  for (int i = 0; i < n; ++i) e->h_delta[i] = e->deltas[reqs[B.idx[i]].step];
+  FPS_CUDA_TRY(cudaMemcpyAsync(e->d_delta, e->h_delta, n * 4, cudaMemcpyHostToDevice, cs));
+
+  // ---- load schedule: ring loads (cached blocks in order) + KV-mode final Y load ----------
+  std::vector<int> loads;                  // block of each ring load
+  std::vector<int> pos(N, -1);
+  for (int l = 0; l < N; ++l)
+    if (use[l]) {
+      pos[l] = (int)loads.size();
+      loads.push_back(l);
+    }
+  const int n_ring = (int)loads.size();
+  const bool final_load = kv && n_ring > 0;
+  std::vector<char> consumed_rec(n_ring + 1, 0);
+  int issued = 0;
+  bool final_issued = false;
+  std::vector<fps_prefetch_item> items(n);
+  FPS_CUDA_TRY(cudaEventRecord(e->step_start, cs));
+  FPS_CUDA_TRY(cudaStreamWaitEvent(ls, e->step_start, 0));
+  auto issue = [&](int block, char* dst, size_t row_bytes, cudaEvent_t ev) -> fps_status {
+    for (int i = 0; i < n; ++i) {
+      const fps_request& r = reqs[B.idx[i]];
+      fps_prefetch_item& it = items[i];
+      it.template_id = r.template_id;
+      it.step = r.step;
+      it.layer = block;
+      it.n_rows = B.nu[i];
+      it.d_rows = e->d_uids + (size_t)i * e->L;
+      it.h_rows = e->h_uids + (size_t)i * e->L;
+      it.d_dst = dst + (size_t)B.h_cu_k[i] * row_bytes;
+      it.dst_row_bytes = (int)row_bytes;
+    }
+    return fps_cache_prefetch(e->d.cache, items.data(), n, ls, ev);
+  };
+  auto try_issue = [&]() -> fps_status {
+    while (issued < n_ring && (issued < e->D || consumed_rec[issued - e->D])) {
+      if (issued >= e->D) FPS_CUDA_TRY(cudaStreamWaitEvent(ls, e->consumed[issued - e->D], 0));
+      FPS_TRY(issue(loads[issued], e->slots[issued % e->D], e->row_w, e->ready[issued]));
+      ++issued;
+    }
+    if (final_load && issued == n_ring && !final_issued) {
+      FPS_TRY(issue(N, e->final_slot, e->row_h, e->ready[n_ring]));
+      final_issued = true;
+    }
+    return FPS_OK;
+  };
+  auto consume = [&](int j) -> fps_status {
+    FPS_CUDA_TRY(cudaEventRecord(e->consumed[j], cs));
+    consumed_rec[j] = 1;
+    return FPS_OK;
+  };
+  FPS_TRY(try_issue());
+
+  // ---- compute ------------------------------------------------------------------------
+  fps_varlen_batch vb{};
+  vb.n_req = n;
+  vb.total_q = B.tq;
+  vb.total_k = B.tk;
+  vb.max_q = B.max_q;
+  vb.max_k = e->L;
+  vb.d_cu_q = B.cu_q;
+  vb.d_cu_k = B.cu_k;
+  vb.h_cu_q = B.h_cu_q;
+  vb.h_cu_k = B.h_cu_k;
+  vb.d_q_row = B.q_row;
+  vb.mode = e->d.mode;
+  vb.total_u = B.tu;
+  vb.d_cu_u = B.cu_u;
+  vb.d_u_src = B.u_row;
+  vb.d_u_row = B.u_row;
+  fps_varlen_batch vd = vb;             // dense: every row of every request is active
+  vd.total_q = B.tk;
+  vd.max_q = e->L;
+  vd.d_cu_q = B.cu_k;
+  vd.h_cu_q = B.h_cu_k;
+  vd.d_q_row = nullptr;
+  vd.mode = FPS_MODE_KV;
+  vd.total_u = 0;
+
+  const char* cur_full = e->x_full;     // valid full-row activations when rep == FULL
+  int full_toggle = 0, act_cur = 0;
+  bool rep_full = true;
+  for (int l = 0; l < N; ++l) {
+    const fps_block_weights* w = &e->layers[l];
+    const void* mod = e->d.d_mod_table ? e->mod_batch + (size_t)l * n * 6 * e->row_h : nullptr;
+    vb.d_mod = mod;
+    vd.d_mod = mod;
+    if (!use[l]) {
+      if (!rep_full) {
+        // Y-mode cached -> uncached: rebuild the full input from act rows M and the cached
+        // output rows U of block l-1 (reading R11)
+        char* dst = e->full[full_toggle];
+        FPS_TRY(launch_copy_rows(e->act[act_cur], nullptr, B.q_row, B.tq, (int)e->row_h, dst, cs));
+        FPS_CUDA_TRY(cudaStreamWaitEvent(cs, e->ready[pos[l - 1]], 0));
+        FPS_TRY(launch_copy_rows(e->slots[pos[l - 1] % e->D], B.u_row, B.u_row, B.tu,
+                                 (int)e->row_h, dst, cs));
+        FPS_TRY(consume(pos[l - 1]));
+        cur_full = dst;
+        full_toggle ^= 1;
+      }
+      char* dst = e->full[full_toggle];
+      FPS_TRY(fps_dense_block_forward(w, &vd, cur_full, dst, e->kv_scratch, e->ws, e->ws_bytes, cs));
+      cur_full = dst;
+      full_toggle ^= 1;
+      rep_full = true;
+    } else {
+      const char* x_in;
+      const char* xu = nullptr;
+      cudaEvent_t ev = nullptr;
+      int consumed_after = -1;
+      if (rep_full) {
+        FPS_TRY(launch_copy_rows(cur_full, B.q_row, nullptr, B.tq, (int)e->row_h, e->act[act_cur], cs));
+        xu = cur_full;
+      } else if (!kv) {
+        xu = e->slots[pos[l - 1] % e->D];
+        ev = e->ready[pos[l - 1]];
+        consumed_after = pos[l - 1];
+      }
+      x_in = e->act[act_cur];
+      char* kvbuf;
+      if (kv) {
+        kvbuf = e->slots[pos[l] % e->D];
+        ev = e->ready[pos[l]];
+        consumed_after = pos[l];
+      } else {
+        kvbuf = e->kv_scratch;
+      }
+      FPS_TRY(fps_masked_block_forward(w, &vb, x_in, e->act[act_cur ^ 1], kvbuf, kv ? nullptr : xu,
+                                       ev, e->ws, e->ws_bytes, cs));
+      if (consumed_after >= 0) FPS_TRY(consume(consumed_after));
+      act_cur ^= 1;
+      rep_full = false;
+    }
+    FPS_TRY(try_issue());
+  }
+
+  // ---- replenish (a9) + sampler update ---------------------------------------------------
+  const char* y_src;
+  if (rep_full) {
+    y_src = cur_full;
+  } else {
+    FPS_TRY(launch_copy_rows(e->act[act_cur], nullptr, B.q_row, B.tq, (int)e->row_h, e->y_full, cs));
+    const int j = kv ? n_ring : pos[N - 1];
+    const char* src = kv ? e->final_slot : e->slots[pos[N - 1] % e->D];
+    FPS_CUDA_TRY(cudaStreamWaitEvent(cs, e->ready[j], 0));
+    FPS_TRY(launch_copy_rows(src, B.u_row, B.u_row, B.tu, (int)e->row_h, e->y_full, cs));
+    y_src = e->y_full;
+  }
+  FPS_TRY(launch_euler(e->d.dtype, e->x_full, y_src, B.tk, H, B.cu_k, n, e->d_delta, cs));
+  // the load stream must not run ahead into the next step's slots before this step is done
+  FPS_CUDA_TRY(cudaEventRecord(e->step_start, cs));
+  FPS_CUDA_TRY(cudaStreamWaitEvent(ls, e->step_start, 0));
+  return FPS_OK;
+}
+
+}  // namespace fps
+
+extern "C" fps_status fps_run_batch(fps_engine_t e, fps_request* reqs, int32_t n_req,
+                                    int32_t n_steps, void* compute_stream, void* load_stream) {
+  FPS_CHECK_ARG(e, "NULL engine");
+  FPS_CHECK_ARG(n_req >= 0 && n_req <= e->d.max_batch, "n_req %d > max_batch %d", n_req,
+                e->d.max_batch);
+  FPS_CHECK_ARG(n_req == 0 || reqs, "NULL reqs");
+  FPS_CHECK_ARG(n_steps >= 0, "n_steps < 0");
+  for (int i = 0; i < n_req; ++i) {
+    FPS_CHECK_ARG(reqs[i].d_mask && reqs[i].d_x, "request %d: NULL mask or latent", i);
+    FPS_CHECK_ARG(reqs[i].n_steps <= e->d.n_steps && reqs[i].step >= 0, "request %d: steps", i);
+  }
+  cudaStream_t cs = as_stream(compute_stream);
+  cudaStream_t ls = load_stream ? as_stream(load_stream) : cs;
+  const long long launches0 = g_launches;
+  int done_steps = 0;
+  while (done_steps < n_steps) {
+    std::vector<int> live;
+    for (int i = 0; i < n_req; ++i) {
+      reqs[i].status = reqs[i].step >= reqs[i].n_steps ? 1 : 0;
+      if (!reqs[i].status) live.push_back(i);
+    }
+    if (live.empty()) break;
+    Batch B;
+    FPS_TRY(admit(e, reqs, live, B, cs));
+    // load each request's latent into the contiguous batch buffer
+    for (int i = 0; i < B.n; ++i)
+      FPS_CUDA_TRY(cudaMemcpyAsync(e->x_full + (size_t)i * e->L * e->row_h, reqs[live[i]].d_x,
+                                   (size_t)e->L * e->row_h, cudaMemcpyDeviceToDevice, cs));
+    make_plan(e, B);
+    bool changed = false;
+    while (done_steps < n_steps && !changed) {
+      FPS_TRY(run_step(e, reqs, B, cs, ls));
+      ++done_steps;
+      for (int i = 0; i < B.n; ++i) {
+        fps_request& r = reqs[live[i]];
+        r.step += 1;
+        if (r.step >= r.n_steps) {
+          r.status = 1;
+          changed = true;   // leaves at this step boundary (L237); the batch is rebuilt
+        }
+      }
+    }
+    for (int i = 0; i < B.n; ++i)
+      FPS_CUDA_TRY(cudaMemcpyAsync(reqs[live[i]].d_x, e->x_full + (size_t)i * e->L * e->row_h,
+                                   (size_t)e->L * e->row_h, cudaMemcpyDeviceToDevice, cs));
+  }
+  for (int i = 0; i < n_req; ++i) reqs[i].status = reqs[i].step >= reqs[i].n_steps ? 1 : 0;
+  // make sure the load stream has drained before the caller reuses buffers
+  FPS_CUDA_TRY(cudaEventRecord(e->step_start, ls));
+  FPS_CUDA_TRY(cudaStreamWaitEvent(cs, e->step_start, 0));
+  e->last_launches = g_launches - launches0;
+  return FPS_OK;
+}

@@ -1,0 +1,258 @@
+// a1 mask index, a2/a9/a3 row movement, a4 row-norm + modulation, sampler update.
+// PAPER.md L130 (token categorisation), L157 (extract / replenish rows), L134 (token-wise LN).
+#include "kernels.h"
+
+namespace fps {
+
+// ---------------------------------------------------------------------------------------
+// a1: one CTA (1024 threads) per request; per 1024-token chunk a warp ballot gives each
+// token its rank inside the warp, a warp-0 scan over the 32 warp counts gives the rank
+// inside the chunk, and a running total carries it across chunks. Stable (ascending ids).
+__global__ void __launch_bounds__(1024) mask_index_kernel(const uint8_t* __restrict__ masks,
+                                                          const int32_t* __restrict__ off,
+                                                          int32_t* __restrict__ mids,
+                                                          int32_t* __restrict__ uids,
+                                                          int32_t* __restrict__ nm) {
+  __shared__ int warp_off[32];
+  __shared__ int chunk_total;
+  const int r = blockIdx.x;
+  const int beg = off[r], L = off[r + 1] - beg;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nwarps = blockDim.x >> 5;
+  const unsigned lt_mask = (1u << lane) - 1u;
+  int running = 0;
+  for (int chunk = 0; chunk < L; chunk += blockDim.x) {
+    const int t = chunk + threadIdx.x;
+    const bool valid = t < L;
+    const bool act = valid && masks[beg + t] != 0;
+    const unsigned bal = __ballot_sync(0xffffffffu, act);
+    const int rank_in_warp = __popc(bal & lt_mask);
+    if (lane == 0) warp_off[warp] = __popc(bal);
+    __syncthreads();
+    if (warp == 0) {
+      int v = lane < nwarps ? warp_off[lane] : 0;
+      int incl = v;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        int u = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += u;
+      }
+      if (lane < nwarps) warp_off[lane] = incl - v;
+      if (lane == 31) chunk_total = incl;
+    }
+    __syncthreads();
+    const int before = running + warp_off[warp] + rank_in_warp;   // active tokens with id < t
+    if (valid) {
+      if (act) mids[beg + before] = t;
+      else uids[beg + (t - before)] = t;
+    }
+    running += chunk_total;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) nm[r] = running;
+}
+
+fps_status launch_mask_index(const uint8_t* masks, const int32_t* off, int n_req, int max_len,
+                             int32_t* mids, int32_t* uids, int32_t* nm, cudaStream_t s) {
+  (void)max_len;
+  if (n_req == 0) return FPS_OK;
+  mask_index_kernel<<<n_req, 1024, 0, s>>>(masks, off, mids, uids, nm);
+  count_launch();
+  FPS_LAUNCH_CHECK();
+  return FPS_OK;
+}
+
+// ---------------------------------------------------------------------------------------
+// Row copy by index, 16-B vectors, 4 independent vectors in flight per thread (the source may
+// be mapped pinned host memory read over PCIe, so memory-level parallelism matters).
+__global__ void __launch_bounds__(256) copy_rows_kernel(const uint4* __restrict__ src,
+                                                        const int32_t* __restrict__ src_ids,
+                                                        const int32_t* __restrict__ dst_ids,
+                                                        long long total, int vpr,
+                                                        uint4* __restrict__ dst) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  for (; i < total; i += 4 * stride) {
+    uint4 v[4];
+    long long di[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      long long idx = i + u * stride;
+      di[u] = -1;
+      if (idx < total) {
+        int row = (int)(idx / vpr), c = (int)(idx - (long long)row * vpr);
+        long long sr = src_ids ? __ldg(src_ids + row) : row;
+        long long dr = dst_ids ? __ldg(dst_ids + row) : row;
+        v[u] = src[sr * vpr + c];
+        di[u] = dr * vpr + c;
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if (di[u] >= 0) dst[di[u]] = v[u];
+  }
+}
+
+fps_status launch_copy_rows(const void* src, const int32_t* src_ids, const int32_t* dst_ids,
+                            int n, int row_bytes, void* dst, cudaStream_t s, int max_ctas) {
+  if (n <= 0) return FPS_OK;
+  const int vpr = row_bytes / 16;
+  const long long total = (long long)n * vpr;
+  long long want = (total + 256 * 4 - 1) / (256 * 4);
+  int cap = max_ctas > 0 ? max_ctas : kNumSMs * 8;
+  int grid = (int)(want < cap ? want : cap);
+  if (grid < 1) grid = 1;
+  copy_rows_kernel<<<grid, 256, 0, s>>>(reinterpret_cast<const uint4*>(src), src_ids, dst_ids,
+                                        total, vpr, reinterpret_cast<uint4*>(dst));
+  count_launch();
+  FPS_LAUNCH_CHECK();
+  return FPS_OK;
+}
+
+// ---------------------------------------------------------------------------------------
+// a4: one warp per row; the row stays in registers (VPT 16-B vectors per lane), two-pass
+// mean / variance in fp32, then the per-request adaLN modulation (reading R2/R3).
+template <typename T, int VPT>
+__global__ void __launch_bounds__(128) ln_mod_kernel(const T* __restrict__ x,
+                                                     const int32_t* __restrict__ rows, int n,
+                                                     int H, T* __restrict__ out,
+                                                     const int32_t* __restrict__ cu, int n_req,
+                                                     const T* __restrict__ mod, int shift_off) {
+  constexpr int NV = Vec16<T>::N;
+  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (warp >= n) return;
+  const int src_row = rows ? __ldg(rows + warp) : warp;
+  const int nvec = H / NV;
+  const uint4* xr = reinterpret_cast<const uint4*>(x + (size_t)src_row * H);
+  float v[VPT][NV];
+  float sum = 0.f;
+#pragma unroll
+  for (int k = 0; k < VPT; ++k) {
+    int vi = lane + 32 * k;
+    if (vi < nvec) {
+      Vec16<T>::unpack(xr[vi], v[k]);
+#pragma unroll
+      for (int e = 0; e < NV; ++e) sum += v[k][e];
+    } else {
+#pragma unroll
+      for (int e = 0; e < NV; ++e) v[k][e] = 0.f;
+    }
+  }
+  const float mean = warp_sum(sum) / (float)H;
+  float sq = 0.f;
+#pragma unroll
+  for (int k = 0; k < VPT; ++k) {
+    if (lane + 32 * k < nvec) {
+#pragma unroll
+      for (int e = 0; e < NV; ++e) {
+        float d = v[k][e] - mean;
+        sq += d * d;
+      }
+    }
+  }
+  const float var = warp_sum(sq) / (float)H;
+  const float rstd = 1.0f / sqrtf(var + 1e-6f);
+  const T* shift = nullptr;
+  const T* scale = nullptr;
+  if (mod) {
+    const int r = find_req(cu, n_req, warp);
+    shift = mod + (size_t)r * 6 * H + shift_off;
+    scale = shift + H;
+  }
+  uint4* o = reinterpret_cast<uint4*>(out + (size_t)warp * H);
+#pragma unroll
+  for (int k = 0; k < VPT; ++k) {
+    int vi = lane + 32 * k;
+    if (vi < nvec) {
+      float r[NV];
+      if (mod) {
+        float sh[NV], sc[NV];
+        Vec16<T>::unpack(reinterpret_cast<const uint4*>(shift)[vi], sh);
+        Vec16<T>::unpack(reinterpret_cast<const uint4*>(scale)[vi], sc);
+#pragma unroll
+        for (int e = 0; e < NV; ++e) r[e] = (v[k][e] - mean) * rstd * (1.0f + sc[e]) + sh[e];
+      } else {
+#pragma unroll
+        for (int e = 0; e < NV; ++e) r[e] = (v[k][e] - mean) * rstd;
+      }
+      o[vi] = Vec16<T>::pack(r);
+    }
+  }
+}
+
+template <typename T>
+static fps_status ln_mod_t(const void* x, const int32_t* rows, int n, int H, void* out,
+                           const int32_t* cu, int n_req, const void* mod, int shift_off,
+                           cudaStream_t s) {
+  constexpr int NV = Vec16<T>::N;
+  const int per_lane = ceil_div(H / NV, 32);
+  const int grid = ceil_div(n, 4);
+  auto X = reinterpret_cast<const T*>(x);
+  auto O = reinterpret_cast<T*>(out);
+  auto Md = reinterpret_cast<const T*>(mod);
+#define FPS_LN_CASE(VPT)                                                                  \
+  if (per_lane <= VPT) {                                                                  \
+    ln_mod_kernel<T, VPT><<<grid, 128, 0, s>>>(X, rows, n, H, O, cu, n_req, Md, shift_off); \
+    count_launch();                                                                       \
+    FPS_LAUNCH_CHECK();                                                                   \
+    return FPS_OK;                                                                        \
+  }
+  FPS_LN_CASE(1)
+  FPS_LN_CASE(2)
+  FPS_LN_CASE(4)
+  FPS_LN_CASE(8)
+  FPS_LN_CASE(12)
+  FPS_LN_CASE(16)
+#undef FPS_LN_CASE
+  return fail(FPS_EUNSUPPORTED, "ln_mod: H=%d too large", H);
+}
+
+fps_status launch_ln_mod(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
+                         const int32_t* cu, int n_req, const void* mod, int shift_off,
+                         cudaStream_t s) {
+  if (n <= 0) return FPS_OK;
+  if (dtype == FPS_BF16)
+    return ln_mod_t<__nv_bfloat16>(x, rows, n, H, out, cu, n_req, mod, shift_off, s);
+  return ln_mod_t<float>(x, rows, n, H, out, cu, n_req, mod, shift_off, s);
+}
+
+// ---------------------------------------------------------------------------------------
+// Synthetic sampler update over the full latent (reading R21): x <- x + delta_req * y.
+template <typename T>
+__global__ void __launch_bounds__(256) euler_kernel(T* __restrict__ x, const T* __restrict__ y,
+                                                    long long nvec, int vpr,
+                                                    const int32_t* __restrict__ cu, int n_req,
+                                                    const float* __restrict__ delta) {
+  constexpr int NV = Vec16<T>::N;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nvec;
+       i += (long long)gridDim.x * blockDim.x) {
+    const int row = (int)(i / vpr);
+    const float d = __ldg(delta + find_req(cu, n_req, row));
+    float a[NV], b[NV];
+    Vec16<T>::unpack(reinterpret_cast<const uint4*>(x)[i], a);
+    Vec16<T>::unpack(reinterpret_cast<const uint4*>(y)[i], b);
+#pragma unroll
+    for (int e = 0; e < NV; ++e) a[e] = a[e] + d * b[e];
+    reinterpret_cast<uint4*>(x)[i] = Vec16<T>::pack(a);
+  }
+}
+
+fps_status launch_euler(int dtype, void* x, const void* y, int n, int H, const int32_t* cu,
+                        int n_req, const float* delta, cudaStream_t s) {
+  if (n <= 0) return FPS_OK;
+  const int elt = dtype == FPS_BF16 ? 2 : 4;
+  const int vpr = H * elt / 16;
+  const long long nvec = (long long)n * vpr;
+  int grid = (int)((nvec + 255) / 256);
+  if (grid > kNumSMs * 16) grid = kNumSMs * 16;
+  if (dtype == FPS_BF16)
+    euler_kernel<__nv_bfloat16><<<grid, 256, 0, s>>>((__nv_bfloat16*)x, (const __nv_bfloat16*)y,
+                                                     nvec, vpr, cu, n_req, delta);
+  else
+    euler_kernel<float><<<grid, 256, 0, s>>>((float*)x, (const float*)y, nvec, vpr, cu, n_req,
+                                             delta);
+  count_launch();
+  FPS_LAUNCH_CHECK();
+  return FPS_OK;
+}
+
+}  // namespace fps

@@ -1,0 +1,45 @@
+// Internal launcher declarations (libflashps). Each returns fps_status and never syncs.
+#pragma once
+#include "common.cuh"
+
+namespace fps {
+
+// a1
+fps_status launch_mask_index(const uint8_t* masks, const int32_t* off, int n_req, int max_len,
+                             int32_t* mids, int32_t* uids, int32_t* nm, cudaStream_t s);
+// a2/a9/a3 row movement: dst[dst_ids? dst_ids[i] : i] = src[src_ids ? src_ids[i] : i]
+fps_status launch_copy_rows(const void* src, const int32_t* src_ids, const int32_t* dst_ids,
+                            int n, int row_bytes, void* dst, cudaStream_t s, int max_ctas = 0);
+// a4: out[i] = LN(x[rows ? rows[i] : i]) * (1 + scale[req(i)]) + shift[req(i)]
+fps_status launch_ln_mod(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
+                         const int32_t* cu, int n_req, const void* mod, int shift_off,
+                         cudaStream_t s);
+// x[i] += delta[req(i)] * y[i] over rows of width H (req via cu over rows)
+fps_status launch_euler(int dtype, void* x, const void* y, int n, int H, const int32_t* cu,
+                        int n_req, const float* delta, cudaStream_t s);
+// GEMM C = A[M,K] B[N,K]^T with the fused epilogue
+fps_status launch_gemm(int dtype, const void* A, const void* B, int M, int N, int K,
+                       const Epilogue& ep, cudaStream_t s);
+fps_status launch_gemm_simt(int dtype, const void* A, const void* B, int M, int N, int K,
+                            const Epilogue& ep, cudaStream_t s);
+fps_status launch_gemm_tc(const void* A, const void* B, int M, int N, int K, const Epilogue& ep,
+                          cudaStream_t s);
+bool gemm_tc_supported(int dtype, int M, int N, int K);
+// a6: o[i, head] = softmax(q_i k^T / sqrt(d)) v over the request's merged keys
+fps_status launch_attention(int dtype, const void* q, const void* kv, void* o, int heads,
+                            int head_dim, const int32_t* d_cu_q, const int32_t* d_cu_k,
+                            const int32_t* h_cu_q, const int32_t* h_cu_k, int n_req, int total_q,
+                            int max_q, int max_k, cudaStream_t s);
+fps_status launch_attention_simt(int dtype, const void* q, const void* kv, void* o, int heads,
+                                 int head_dim, const int32_t* cu_q, const int32_t* cu_k,
+                                 int n_req, int total_q, cudaStream_t s);
+fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads, int head_dim,
+                               const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
+                               int n_req, int max_q, cudaStream_t s);
+bool attention_tc_supported(int dtype, int head_dim);
+
+// global switches (tests can force the SIMT kernels): bit0 = no tcgen05 GEMM,
+// bit1 = no tensor-core attention
+extern int g_disable_tc;
+
+}  // namespace fps

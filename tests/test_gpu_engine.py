@@ -1,0 +1,174 @@
+"""GPU parity of fps_run_batch (stack of N blocks, layer-ahead cache pipeline, step-level
+continuous batching) against the oracle's masked_run, plus GPU-internal invariants."""
+import numpy as np
+import pytest
+import torch
+
+import synth
+from oracle import stack as S
+from gpu_util import TOL, check_close, to_dev, to_np
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def F():
+    import paper_conf_eurosys_jianglyfdlzllyl26_b200 as fps
+    fps.require_gpu()
+    return fps
+
+
+def _setup(F, mode, dtype, plan_policy, plan=None, N=3, steps=3, H=256, heads=2, Fd=512,
+           L_img=256, L_txt=16, n_req=3, slots=0, copy_method=0, seed=5000):
+    g = synth.rng(seed)
+    W = synth.stack_weights(g, N, H, Fd, dtype)
+    mods = synth.mod_table(g, N, steps, H, dtype)
+    deltas = synth.delta_table(steps)
+    L = L_img + L_txt
+    n_t = 2
+    # template cache: random activations of the right shapes (both sides consume the same)
+    cache_np = [[[{"K": synth.latent(g, L, H, dtype), "V": synth.latent(g, L, H, dtype),
+                   "Y": synth.latent(g, L, H, dtype)} for _ in range(N)] for _ in range(steps)]
+                for _ in range(n_t)]
+    dt = F.DTYPE_CODE[dtype]
+    m = F.MODE_CODE[mode]
+    cache = F.Cache(m, dt, H, L_img, N, steps, n_templates=n_t, copy_method=copy_method)
+    for t in range(n_t):
+        for s in range(steps):
+            for l in range(N):
+                e = cache_np[t][s][l]
+                if mode == "kv":
+                    cache.store(t, s, l, to_dev(np.concatenate([e["K"], e["V"]], 1), dtype))
+                else:
+                    cache.store(t, s, l, to_dev(e["Y"], dtype))
+            if mode == "kv":
+                cache.store(t, s, N, to_dev(cache_np[t][s][N - 1]["Y"], dtype))
+    torch.cuda.synchronize()
+    layers = [F.BlockWeights(w, heads, dt) for w in W]
+    eng = F.Engine(layers, heads, m, dt, L_img, L_txt, max_batch=4, n_steps=steps, deltas=deltas,
+                   cache=cache, mod_table=to_dev(mods, dtype), slots=slots,
+                   plan_policy=plan_policy, plan=plan)
+    reqs = []
+    ratios = [0.1, 0.45, 0.25, 0.6][:n_req]
+    for i in range(n_req):
+        mask = synth.token_mask(synth.mask_blobs(g, 16, 16, ratios[i]), L_txt)
+        x0 = synth.latent(g, L, H, dtype)
+        reqs.append(dict(template_id=i % n_t, step=i % 2, n_steps=steps, mask_np=mask, x0=x0,
+                         mask=torch.as_tensor(mask).cuda(), x=to_dev(x0, dtype)))
+    return W, mods, deltas, cache_np, eng, reqs
+
+
+def _oracle(W, mods, deltas, cache_np, reqs, plan, mode, heads, steps_run):
+    outs = []
+    for r in reqs:
+        s0 = r["step0"]
+        n = min(steps_run, r["n_steps"] - s0)
+        x = S.masked_run(r["x0"], r["mask_np"], W, mods, deltas, plan, mode,
+                         cache_np[r["template_id"]], heads, n, step0=s0)
+        outs.append(x)
+    return outs
+
+
+@pytest.mark.parametrize("mode,dtype,policy,plan", [
+    ("kv", "bf16", 1, None), ("y", "bf16", 1, None), ("kv", "f32", 1, None),
+    ("y", "f32", 3, [1, 0, 1]), ("kv", "bf16", 3, [0, 1, 1]), ("y", "bf16", 3, [0, 1, 0]),
+    ("kv", "bf16", 2, None)])
+def test_run_batch_matches_oracle(F, mode, dtype, policy, plan):
+    W, mods, deltas, cache_np, eng, reqs = _setup(F, mode, dtype, policy, plan)
+    for r in reqs:
+        r["step0"] = r["step"]
+    eng.run_batch(reqs, 2)
+    torch.cuda.synchronize()
+    used = eng.last_plan()[0]
+    if policy == 1:
+        assert used == [1, 1, 1]
+    if policy == 3:
+        assert used == plan
+    ref = _oracle(W, mods, deltas, cache_np, reqs, used, mode, 2, 2)
+    for r, x in zip(reqs, ref):
+        check_close(to_np(r["x"]), x, TOL[dtype], f"{mode} {dtype} plan={used}")
+        assert r["step"] == min(r["step0"] + 2, r["n_steps"])
+
+
+def test_requests_leave_at_step_boundary(F):
+    """A request reaching its last step leaves; the others keep running (L237)."""
+    W, mods, deltas, cache_np, eng, reqs = _setup(F, "kv", "bf16", 1, steps=3)
+    for r in reqs:
+        r["step0"] = r["step"]
+    eng.run_batch(reqs, 3)
+    torch.cuda.synchronize()
+    assert [r["status"] for r in reqs] == [1, 1, 1]
+    assert [r["step"] for r in reqs] == [3, 3, 3]
+    ref = _oracle(W, mods, deltas, cache_np, reqs, [1, 1, 1], "kv", 2, 3)
+    for r, x in zip(reqs, ref):
+        check_close(to_np(r["x"]), x, TOL["bf16"], "leave")
+
+
+@pytest.mark.parametrize("slots,method", [(1, 0), (2, 1), (0, 0)])
+def test_pipeline_slots_and_copy_methods_bit_identical(F, slots, method):
+    """The staging ring depth and the H2D method change timing only, never the bits."""
+    outs = []
+    for sl, me in ((0, 0), (slots, method)):
+        _, _, _, _, eng, reqs = _setup(F, "kv", "bf16", 1, slots=sl, copy_method=me, seed=5100)
+        eng.run_batch(reqs, 2)
+        torch.cuda.synchronize()
+        outs.append([r["x"].clone() for r in reqs])
+    for a, b in zip(*outs):
+        assert torch.equal(a.view(torch.int16), b.view(torch.int16))
+
+
+def test_delayed_load_stream_bit_identical(F):
+    """Robustness of the event ordering: a busy load stream (a long spin queued before the
+    prefetches) must not change the result."""
+    _, _, _, _, eng, reqs = _setup(F, "y", "bf16", 1, seed=5200)
+    eng.run_batch(reqs, 2)
+    torch.cuda.synchronize()
+    ref = [r["x"].clone() for r in reqs]
+    _, _, _, _, eng, reqs = _setup(F, "y", "bf16", 1, seed=5200)
+    ls = torch.cuda.Stream()
+    with torch.cuda.stream(ls):
+        torch.cuda._sleep(200_000_000)          # ~0.1 s of spinning on the load stream
+    eng.run_batch(reqs, 2, load_stream=ls)
+    torch.cuda.synchronize()
+    for a, r in zip(ref, reqs):
+        assert torch.equal(a.view(torch.int16), r["x"].view(torch.int16))
+
+
+def test_identical_input_cache_gpu_internal_invariant(F):
+    """L144/L157 on the GPU: store the GPU's own dense-run activations as the cache; the masked
+    run on the identical input reproduces the dense run's latents bit-for-bit (token-wise
+    kernels have row-independent arithmetic, attention sees the same keys in the same order)."""
+    g = synth.rng(5300)
+    N, steps, H, heads, Fd, L_img, L_txt = 3, 1, 256, 2, 512, 256, 16
+    L = L_img + L_txt
+    W = synth.stack_weights(g, N, H, Fd, "bf16")
+    mods = synth.mod_table(g, N, steps, H, "bf16")
+    dt = F.FPS_BF16
+    layers = [F.BlockWeights(w, heads, dt) for w in W]
+    x0 = synth.latent(g, L, H, "bf16")
+    mask = synth.token_mask(synth.mask_blobs(g, 16, 16, 0.3), L_txt)
+    for mode in ("kv", "y"):
+        m = F.MODE_CODE[mode]
+        # dense template run on the GPU, one block at a time, capturing K|V and Y
+        b = F.VarlenBatch([L], [L], mod=None)
+        cache = F.Cache(m, dt, H, L_img, N, steps, n_templates=1)
+        cur = to_dev(x0, "bf16")
+        for l in range(N):
+            bl = F.VarlenBatch([L], [L], mod=to_dev(mods[l, 0][None], "bf16"))
+            y, kv = F.dense_block_forward(layers[l], bl, cur)
+            cache.store(0, 0, l, kv if mode == "kv" else y)
+            cur = y
+        if mode == "kv":
+            cache.store(0, 0, N, cur)
+        torch.cuda.synchronize()
+        outs = []
+        for policy in (1, 2):          # all blocks cached vs all blocks dense (no cache)
+            eng = F.Engine(layers, heads, m, dt, L_img, L_txt, 1, steps, synth.delta_table(steps),
+                           cache, mod_table=to_dev(mods, "bf16"), plan_policy=policy)
+            req = dict(template_id=0, step=0, n_steps=steps, mask=torch.as_tensor(mask).cuda(),
+                       x=to_dev(x0, "bf16"))
+            eng.run_batch([req], 1)
+            torch.cuda.synchronize()
+            outs.append(req["x"].clone())
+        diff = (outs[0].float() - outs[1].float()).abs().max().item()
+        assert torch.equal(outs[0].view(torch.int16), outs[1].view(torch.int16)), f"{mode}: {diff}"

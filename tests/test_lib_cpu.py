@@ -1,0 +1,104 @@
+"""CPU-side checks of libflashps: the library loads, exports every symbol include/flashps.h
+declares, its host-only planner (Alg. 1) matches the oracle's exhaustive optimum, and device
+calls fail loudly (no CPU fallback) when no GPU is present."""
+import os
+import re
+
+import numpy as np
+import pytest
+import torch
+
+import synth
+from oracle import pipeline as P
+
+import paper_conf_eurosys_jianglyfdlzllyl26_b200 as fps
+from paper_conf_eurosys_jianglyfdlzllyl26_b200 import _lib
+
+HDR = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "include",
+                   "flashps.h")
+
+
+def _declared():
+    src = open(HDR).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(fps_[a-z0-9_]+)\s*\(", src)))
+
+
+def test_exports_every_declared_symbol():
+    names = _declared()
+    assert len(names) >= 20
+    for n in names:
+        assert hasattr(_lib.lib, n), f"{n} declared in flashps.h but not exported"
+        assert n in _lib.EXPORTED, f"{n} has no Python binding"
+
+
+def test_abi_version():
+    assert fps.fps_abi_version() == 1
+
+
+@pytest.mark.skipif(torch.cuda.is_available(), reason="CPU-only check")
+def test_no_cpu_fallback():
+    assert fps.fps_device_ok() == 0
+    with pytest.raises(fps.FlashPSError) as ei:
+        fps.fps_gather_rows(16, 16, 1, 16, 16, None)      # any device work must fail loudly
+    assert ei.value.code in (_lib.FPS_ECUDA,)
+
+
+def test_argument_validation_before_enqueue():
+    with pytest.raises(fps.FlashPSError) as ei:
+        fps.fps_gather_rows(16, 16, 4, 12, 16, None)      # row_bytes not a multiple of 16
+    assert ei.value.code == _lib.FPS_EINVAL
+    with pytest.raises(fps.FlashPSError):
+        fps.fps_masked_block_forward(None, None, None, None, None, None, None, None, 0, None)
+
+
+def _rand_costs(g, N):
+    return g.uniform(0.2, 2, N), g.uniform(1, 4, N), g.uniform(0, 4, N), float(g.uniform(0, 1))
+
+
+@pytest.mark.parametrize("mode", ["kv", "y"])
+def test_planner_matches_bruteforce(mode):
+    """Alg. 1 in the library (KV: O(N) suffix scan; Y: Pareto DP) vs the oracle's exhaustive
+    optimum over all 2^N plans under the same pipeline model (reading R11)."""
+    g = synth.rng(10 if mode == "kv" else 11)
+    m = fps.MODE_CODE[mode]
+    for _ in range(150):
+        N = int(g.integers(1, 12))
+        Cw, Cwo, Lm, fin = _rand_costs(g, N)
+        if g.uniform() < 0.3:           # uniform layers, like a DiT stack
+            Cw, Cwo, Lm = np.full(N, Cw[0]), np.full(N, Cwo[0]), np.full(N, Lm[0])
+        ref, _ = P.plan_bruteforce(Cw, Cwo, Lm, mode, fin)
+        plan, lat = fps.plan_pipeline(Cw, Cwo, Lm, m, fin)
+        assert lat == pytest.approx(ref, rel=1e-9, abs=1e-12)
+        assert P.simulate(plan, Cw, Cwo, Lm, mode, fin) == pytest.approx(ref, rel=1e-9)
+
+
+@pytest.mark.parametrize("mode", ["kv", "y"])
+def test_latency_model_matches_oracle_simulator(mode):
+    g = synth.rng(12)
+    m = fps.MODE_CODE[mode]
+    for _ in range(200):
+        N = int(g.integers(1, 15))
+        Cw, Cwo, Lm, fin = _rand_costs(g, N)
+        use = [int(v) for v in g.integers(0, 2, N)]
+        ref = P.simulate(use, Cw, Cwo, Lm, mode, fin)
+        got = fps.pipeline_latency(use, Cw, Cwo, Lm, m, fin)
+        if np.isinf(ref):
+            assert np.isinf(got)
+        else:
+            assert got == pytest.approx(ref, rel=1e-12)
+
+
+def test_planner_large_stack_properties():
+    """N = 57 / 70 (Flux-, SDXL-scale): no plan the oracle can evaluate beats the library's."""
+    g = synth.rng(13)
+    for N in (57, 70):
+        for mode in ("kv", "y"):
+            m = fps.MODE_CODE[mode]
+            Cw, Cwo, Lm, fin = _rand_costs(g, N)
+            plan, lat = fps.plan_pipeline(Cw, Cwo, Lm, m, fin)
+            assert P.simulate(plan, Cw, Cwo, Lm, mode, fin) == pytest.approx(lat, rel=1e-9)
+            assert lat <= P.plan_suffix_scan(Cw, Cwo, Lm, mode, fin)[0] + 1e-9
+            for _ in range(200):
+                use = [int(v) for v in g.integers(0, 2, N)]
+                assert lat <= P.simulate(use, Cw, Cwo, Lm, mode, fin) + 1e-9
