@@ -52,6 +52,14 @@ int32_t fps_device_ok(void);
  * force the SIMT kernels (bit0: GEMMs, bit1: attention) instead of the tensor-core ones. */
 int64_t fps_launch_count(void);
 void fps_set_disable_tc(int32_t flags);
+/* Per-kernel-class timing for the bench: when enabled (this also clears old records) every
+ * library launch is bracketed by CUDA events on its own stream.  fps_profile_read synchronises
+ * on them and fills, per class k in {0 GEMM, 1 attention, 2 row-norm, 3 row copy, 4 cache
+ * prefetch, 5 sampler update, 6 mask index}, the summed device ms, algorithmic FLOPs and bytes
+ * and the launch count (arrays of 7, each may be NULL).  Returns the number of classes (7) or
+ * FPS_ECUDA. */
+void fps_profile_enable(int32_t on);
+int32_t fps_profile_read(double* ms, double* flops, double* bytes, int64_t* count);
 
 /* ---------------------------------------------------------------------------------------
  * a1  Mask -> token index (L130 "categorize the tokens as masked tokens and unmasked tokens").
@@ -191,6 +199,12 @@ fps_status fps_masked_block_forward(const fps_block_weights* w, const fps_varlen
                                     const void* d_x_act, void* d_y_act, void* d_kv,
                                     const void* d_xu, void* kv_ready, void* d_ws, size_t ws_bytes,
                                     void* stream);
+
+/* The projection building block of a5/a7/a8 on its own (tests and per-kernel measurement):
+ * d_out[M, N] = act(d_a[M, K] . d_w[N, K]^T + d_bias) with act 0 = identity, 1 = GELU_tanh.
+ * bf16 with K % 64 == 0 and N % 8 == 0 runs the tcgen05 GEMM, anything else the SIMT kernel. */
+fps_status fps_linear(int32_t dtype, const void* d_a, const void* d_w, const void* d_bias,
+                      int32_t M, int32_t N, int32_t K, int32_t act, void* d_out, void* stream);
 
 /* Dense block (Fig. 5-Top; the uncached blocks of Fig. 9-Bottom): all L_r rows of every
  * request; b->d_q_row must be NULL and total_q == total_k.  d_kv is scratch [total_k, 2H]. */

@@ -150,6 +150,16 @@ def dense_block_forward(w: BlockWeights, b: VarlenBatch, x, kv=None, y=None, ws=
     return y, kv
 
 
+def linear(a, w, bias=None, act=0, out=None, stream=None):
+    """out = act(a w^T + bias) through fps_linear (tcgen05 GEMM for bf16)."""
+    M, K = a.shape
+    N = w.shape[0]
+    out = out if out is not None else torch.empty(M, N, dtype=a.dtype, device=a.device)
+    dt = FPS_BF16 if a.dtype == torch.bfloat16 else FPS_F32
+    _lib.fps_linear(dt, ptr(a), ptr(w), ptr(bias), M, N, K, act, ptr(out), stream_ptr(stream))
+    return out
+
+
 # ---------------------------------------------------------------------------------------
 def plan_pipeline(c_cached, c_dense, load, mode, final_load=0.0):
     """Alg. 1 (host, in the library). Returns (use_cache list, latency)."""
@@ -206,8 +216,10 @@ class Cache:
 
     def prefetch(self, items, load_stream=None, ready_event=None):
         arr = (fps_prefetch_item * max(len(items), 1))(*items)
-        ev = ready_event.cuda_event if ready_event is not None else None
-        _lib.fps_cache_prefetch(self.h, arr, len(items), stream_ptr(load_stream), ev)
+        _lib.fps_cache_prefetch(self.h, arr, len(items), stream_ptr(load_stream), None)
+        if ready_event is not None:       # torch creates its events lazily: record it here
+            ready_event.record(load_stream if load_stream is not None
+                               else torch.cuda.current_stream())
 
 
 class Engine:

@@ -70,6 +70,8 @@ _SIGS = [
     ("fps_device_ok", i32, [], False),
     ("fps_launch_count", i64, [], False),
     ("fps_set_disable_tc", None, [i32], False),
+    ("fps_profile_enable", None, [i32], False),
+    ("fps_profile_read", i32, [P_dbl, P_dbl, P_dbl, C.POINTER(C.c_int64)], False),
     ("fps_build_mask_index", C.c_int, [vp, vp, i32, i32, vp, vp, vp, vp], True),
     ("fps_gather_rows", C.c_int, [vp, vp, i32, i32, vp, vp], True),
     ("fps_scatter_rows", C.c_int, [vp, vp, i32, i32, vp, vp], True),
@@ -84,6 +86,7 @@ _SIGS = [
     ("fps_masked_block_forward", C.c_int,
      [C.POINTER(fps_block_weights), C.POINTER(fps_varlen_batch), vp, vp, vp, vp, vp, vp, sz, vp],
      True),
+    ("fps_linear", C.c_int, [i32, vp, vp, vp, i32, i32, i32, i32, vp, vp], True),
     ("fps_dense_block_forward", C.c_int,
      [C.POINTER(fps_block_weights), C.POINTER(fps_varlen_batch), vp, vp, vp, vp, sz, vp], True),
     ("fps_plan_pipeline", C.c_int, [P_dbl, P_dbl, P_dbl, i32, i32, dbl, P_u8, P_dbl], True),

@@ -2,6 +2,7 @@
 // (PAPER.md L146 block; L157 mask-aware Y-mode; L161 KV-mode).  See include/flashps.h.
 #include <cstring>
 #include <mutex>
+#include <vector>
 
 #include "kernels.h"
 
@@ -32,24 +33,87 @@ fps_status fail(fps_status code, const char* fmt, ...) {
 
 static int elt_size(int dtype) { return dtype == FPS_BF16 ? 2 : 4; }
 
-fps_status launch_gemm(int dtype, const void* A, const void* B, int M, int N, int K,
-                       const Epilogue& ep, cudaStream_t s) {
-  if (M <= 0 || N <= 0) return FPS_OK;
+// ---- profiling ------------------------------------------------------------------------------
+namespace prof {
+struct Rec {
+  cudaEvent_t a, b;
+  int kind;
+  double flops, bytes;
+};
+static bool g_on = false;
+static std::vector<Rec> g_recs;
+static std::vector<cudaEvent_t> g_pool;
+static size_t g_used = 0;
+static cudaEvent_t g_pending = nullptr;
+
+static cudaEvent_t take() {
+  if (g_used == g_pool.size()) {
+    cudaEvent_t e;
+    if (cudaEventCreate(&e) != cudaSuccess) {
+      cudaGetLastError();
+      return nullptr;
+    }
+    g_pool.push_back(e);
+  }
+  return g_pool[g_used++];
+}
+bool enabled() { return g_on; }
+void begin(cudaStream_t s) {
+  if (!g_on) return;
+  g_pending = take();
+  if (g_pending) cudaEventRecord(g_pending, s);
+}
+void end(cudaStream_t s, int kind, double flops, double bytes) {
+  if (!g_on || !g_pending) return;
+  cudaEvent_t b = take();
+  if (!b) return;
+  cudaEventRecord(b, s);
+  g_recs.push_back(Rec{g_pending, b, kind, flops, bytes});
+  g_pending = nullptr;
+}
+}  // namespace prof
+
+static fps_status launch_gemm_impl(int dtype, const void* A, const void* B, int M, int N, int K,
+                                   const Epilogue& ep, cudaStream_t s) {
   if (!(g_disable_tc & 1) && gemm_tc_supported(dtype, M, N, K))
     return launch_gemm_tc(A, B, M, N, K, ep, s);
   return launch_gemm_simt(dtype, A, B, M, N, K, ep, s);
+}
+
+fps_status launch_gemm(int dtype, const void* A, const void* B, int M, int N, int K,
+                       const Epilogue& ep, cudaStream_t s) {
+  if (M <= 0 || N <= 0) return FPS_OK;
+  prof::begin(s);
+  fps_status st = launch_gemm_impl(dtype, A, B, M, N, K, ep, s);
+  const double e = elt_size(dtype);
+  prof::end(s, prof::GEMM, 2.0 * M * N * K, e * ((double)M * K + (double)N * K + (double)M * N));
+  return st;
 }
 
 fps_status launch_attention(int dtype, const void* q, const void* kv, void* o, int heads,
                             int head_dim, const int32_t* d_cu_q, const int32_t* d_cu_k,
                             const int32_t* h_cu_q, const int32_t* h_cu_k, int n_req, int total_q,
                             int max_q, int max_k, cudaStream_t s) {
-  (void)h_cu_k;
   (void)max_k;
   if (total_q <= 0) return FPS_OK;
-  if (!(g_disable_tc & 2) && attention_tc_supported(dtype, head_dim))
-    return launch_attention_tc(q, kv, o, heads, head_dim, d_cu_q, d_cu_k, h_cu_q, n_req, max_q, s);
-  return launch_attention_simt(dtype, q, kv, o, heads, head_dim, d_cu_q, d_cu_k, n_req, total_q, s);
+  prof::begin(s);
+  fps_status st;
+  if (!(g_disable_tc & 2) && attention_tc_supported(dtype, head_dim) && h_cu_q && h_cu_k)
+    st = launch_attention_tc(q, kv, o, heads, head_dim, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);
+  else
+    st = launch_attention_simt(dtype, q, kv, o, heads, head_dim, d_cu_q, d_cu_k, n_req, total_q, s);
+  if (prof::enabled() && h_cu_q && h_cu_k) {
+    // algorithmic work: QK^T and PV, 4 n_r L_r H FLOPs; bytes: Q, O once + K|V once per request
+    double fl = 0, by = 0;
+    const double H = (double)heads * head_dim, e = elt_size(dtype);
+    for (int r = 0; r < n_req; ++r) {
+      const double n = h_cu_q[r + 1] - h_cu_q[r], L = h_cu_k[r + 1] - h_cu_k[r];
+      fl += 4.0 * n * L * H;
+      by += e * (2.0 * n * H + 2.0 * L * H);
+    }
+    prof::end(s, prof::ATTN, fl, by);
+  }
+  return st;
 }
 
 struct BlockWs {
@@ -190,6 +254,35 @@ int32_t fps_device_ok(void) {
 }
 
 int64_t fps_launch_count(void) { return fps::g_launches; }
+
+void fps_profile_enable(int32_t on) {
+  fps::prof::g_on = on != 0;
+  fps::prof::g_recs.clear();
+  fps::prof::g_used = 0;
+  fps::prof::g_pending = nullptr;
+}
+
+int32_t fps_profile_read(double* ms, double* flops, double* bytes, int64_t* count) {
+  using namespace fps::prof;
+  for (int k = 0; k < NKIND; ++k) {
+    if (ms) ms[k] = 0;
+    if (flops) flops[k] = 0;
+    if (bytes) bytes[k] = 0;
+    if (count) count[k] = 0;
+  }
+  for (const Rec& r : g_recs) {
+    float t = 0.f;
+    if (cudaEventSynchronize(r.b) != cudaSuccess || cudaEventElapsedTime(&t, r.a, r.b) != cudaSuccess) {
+      cudaGetLastError();
+      return FPS_ECUDA;
+    }
+    if (ms) ms[r.kind] += t;
+    if (flops) flops[r.kind] += r.flops;
+    if (bytes) bytes[r.kind] += r.bytes;
+    if (count) count[r.kind] += 1;
+  }
+  return NKIND;
+}
 void fps_set_disable_tc(int32_t flags) { fps::g_disable_tc = flags; }
 
 fps_status fps_build_mask_index(const uint8_t* d_masks, const int32_t* d_offsets, int32_t n_req,
@@ -251,6 +344,21 @@ fps_status fps_masked_block_forward(const fps_block_weights* w, const fps_varlen
   FPS_CHECK_ARG(w->heads * w->head_dim == w->H, "heads*head_dim != H");
   return block_forward(w, b, d_x_act, d_y_act, d_kv, d_xu, (cudaEvent_t)kv_ready, d_ws, ws_bytes,
                        as_stream(stream));
+}
+
+fps_status fps_linear(int32_t dtype, const void* d_a, const void* d_w, const void* d_bias,
+                      int32_t M, int32_t N, int32_t K, int32_t act, void* d_out, void* stream) {
+  FPS_CHECK_ARG(dtype == FPS_BF16 || dtype == FPS_F32, "dtype %d", dtype);
+  FPS_CHECK_ARG(M >= 0 && N > 0 && K > 0 && (act == 0 || act == 1), "bad sizes / act");
+  FPS_CHECK_ARG(M == 0 || (d_a && d_w && d_out), "NULL pointer");
+  FPS_CHECK_ARG(N % 8 == 0, "N %% 8 != 0");
+  Epilogue ep{};
+  ep.bias = d_bias;
+  ep.act = act;
+  ep.out0 = d_out;
+  ep.ld0 = N;
+  ep.split = N;
+  return launch_gemm(dtype, d_a, d_w, M, N, K, ep, as_stream(stream));
 }
 
 fps_status fps_dense_block_forward(const fps_block_weights* w, const fps_varlen_batch* b,

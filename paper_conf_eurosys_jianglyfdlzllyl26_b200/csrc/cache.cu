@@ -201,7 +201,9 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
       int ctas = c->d.copy_ctas > 0 ? c->d.copy_ctas : 32;
       long long want = (acc + 1023) / 1024;
       if (want < ctas) ctas = (int)want;
+      prof::begin(s);
       prefetch_kernel<<<ctas, 256, 0, s>>>(b);
+      prof::end(s, prof::PREFETCH, 0, 16.0 * acc);
       count_launch();
       FPS_LAUNCH_CHECK();
     }
@@ -225,22 +227,10 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
         j = k + 1;
       }
     }
-    if (!c->sizes.empty()) {
-      cudaMemcpyAttributes attr{};
-      attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-      attr.srcLocHint.type = cudaMemLocationTypeHost;
-      attr.dstLocHint.type = cudaMemLocationTypeDevice;
-      attr.flags = cudaMemcpyFlagPreferOverlapWithCompute;
-      size_t attr_idx = 0, fail_idx = 0;
-      cudaError_t e = cudaMemcpyBatchAsync(c->dsts.data(), c->srcs.data(), c->sizes.data(),
-                                           c->sizes.size(), &attr, &attr_idx, 1, &fail_idx, s);
-      if (e != cudaSuccess) {
-        cudaGetLastError();
-        for (size_t q = 0; q < c->sizes.size(); ++q)
-          FPS_CUDA_TRY(cudaMemcpyAsync(c->dsts[q], c->srcs[q], c->sizes[q],
-                                       cudaMemcpyHostToDevice, s));
-      }
-    }
+    // one DMA per run of consecutive rows (cudaMemcpyBatchAsync dropped rows of long runs in
+    // testing on this driver, so the runs are issued individually)
+    for (size_t q = 0; q < c->sizes.size(); ++q)
+      FPS_CUDA_TRY(cudaMemcpyAsync(c->dsts[q], c->srcs[q], c->sizes[q], cudaMemcpyHostToDevice, s));
   }
   if (ready_event) FPS_CUDA_TRY(cudaEventRecord((cudaEvent_t)ready_event, s));
   return FPS_OK;

@@ -54,6 +54,16 @@ inline void count_launch(int n = 1) { g_launches += n; }
 
 constexpr int kNumSMs = 148;
 
+// ---- per-kernel-class timing (fps_profile_enable / fps_profile_read) ----------------------
+// When enabled, every library launch is bracketed by a pair of CUDA events on its own stream;
+// fps_profile_read sums the event durations per class with the algorithmic FLOPs / bytes.
+namespace prof {
+enum Kind { GEMM = 0, ATTN = 1, LN = 2, ROWS = 3, PREFETCH = 4, EULER = 5, INDEX = 6, NKIND = 7 };
+bool enabled();
+void begin(cudaStream_t s);
+void end(cudaStream_t s, int kind, double flops, double bytes);
+}  // namespace prof
+
 // ---- element access ----------------------------------------------------------------------
 template <typename T> struct Elt;
 template <> struct Elt<float> {

@@ -1,9 +1,292 @@
-// Tensor-core varlen merged-key attention (placeholder until the tcgen05 kernel lands).
+// a6: masked-query attention over the merged (fresh + cached) key set, tcgen05 + TMEM + TMA.
+// PAPER.md L146 (QK^T and softmax are the only inter-token op), L159 ("the Q matrix of only the
+// new tokens along with the K and V matrices of all present tokens"), L161 (K/V variant).
+//
+// One CTA per (request, 128-query tile, head); varlen: the tile -> request map is decoded from
+// cu_q in-kernel, keys are the request's rows [cu_k[r], cu_k[r+1]) of the merged buffer.
+//   warp 0     TMA: Q tile once; K and V tiles (128 keys x d) through a 2-stage ring
+//   warp 1     MMA: S_j = Q K_j^T into one of two TMEM S buffers (issued one tile ahead), then
+//              O += P_j V_j with V as an MN-major operand; commits free the K/V stage
+//   warps 4-7  softmax, thread = query row: S row from TMEM (tcgen05.ld), online softmax in the
+//              exp2 domain with a lazy max (O in TMEM is rescaled only when the running max grows
+//              by more than 2^8, FA4-style), P as bf16 into smem in the UMMA K-major SW128 layout;
+//              final O / l from TMEM to global.
 #include "kernels.h"
+#include "tc_util.cuh"
+
 namespace fps {
-bool attention_tc_supported(int dtype, int head_dim) { (void)dtype; (void)head_dim; return false; }
-fps_status launch_attention_tc(const void*, const void*, void*, int, int, const int32_t*,
-                               const int32_t*, const int32_t*, int, int, cudaStream_t) {
-  return fail(FPS_EUNSUPPORTED, "attention_tc not built");
+
+template <int D>
+struct AttnCfg {
+  static constexpr int BM = 128, BN = 128, STAGES = 2;
+  static constexpr int CH = D / 64;                        // 64-wide (128 B) chunks along d
+  static constexpr int Q_BYTES = BM * D * 2;
+  static constexpr int KV_TILE = BN * D * 2;
+  static constexpr int P_BYTES = BM * BN * 2;
+  static constexpr int SMEM = Q_BYTES + STAGES * 2 * KV_TILE + P_BYTES + 1024 + 256;
+  static constexpr int TMEM_COLS = 512;                    // S0 [0,128) S1 [128,256) O [256,256+D)
+};
+
+template <int D>
+__global__ void __launch_bounds__(256, 1)
+    attn_tc_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmKV,
+                   __nv_bfloat16* __restrict__ O, const int32_t* __restrict__ cu_q,
+                   const int32_t* __restrict__ cu_k, int n_req, int heads, float scale_log2) {
+  using Cfg = AttnCfg<D>;
+  constexpr int CHUNK = 128 * 128;                         // bytes of one [128 rows x 128 B] chunk
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~uintptr_t(1023));
+  uint8_t* sQ = smem;
+  uint8_t* sK = sQ + Cfg::Q_BYTES;                          // [stage][CH chunks]
+  uint8_t* sV = sK + Cfg::STAGES * Cfg::KV_TILE;
+  uint8_t* sP = sV + Cfg::STAGES * Cfg::KV_TILE;            // [2 chunks of 64 keys]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sP + Cfg::P_BYTES);
+  uint64_t* bar_q = bars;
+  uint64_t* kv_full = bars + 1;
+  uint64_t* kv_empty = bars + 3;
+  uint64_t* bar_s = bars + 5;
+  uint64_t* bar_p = bars + 7;
+  uint64_t* bar_o = bars + 8;
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + 9);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int head = blockIdx.y;
+  const int H = heads * D;
+  // decode (request, q tile) of this CTA
+  int r = 0, qt = blockIdx.x;
+  for (; r < n_req; ++r) {
+    const int nt = (__ldg(cu_q + r + 1) - __ldg(cu_q + r) + 127) >> 7;
+    if (qt < nt) break;
+    qt -= nt;
+  }
+  const int q0 = __ldg(cu_q + r) + qt * 128;
+  const int n_rows = min(128, __ldg(cu_q + r + 1) - q0);
+  const int k0 = __ldg(cu_k + r);
+  const int Lr = __ldg(cu_k + r + 1) - k0;
+  const int nk = (Lr + 127) >> 7;
+
+  if (threadIdx.x == 0) {
+    tc::mbar_init(bar_q, 1);
+    for (int s = 0; s < 2; ++s) {
+      tc::mbar_init(&kv_full[s], 1);
+      tc::mbar_init(&kv_empty[s], 1);
+      tc::mbar_init(&bar_s[s], 1);
+    }
+    tc::mbar_init(bar_p, 4);
+    tc::mbar_init(bar_o, 1);
+    tc::fence_mbar_init();
+  }
+  if (warp == 0 && lane == 0) {
+    tc::tma_prefetch_desc(&tmQ);
+    tc::tma_prefetch_desc(&tmKV);
+  }
+  if (warp == 2) tc::tmem_alloc<Cfg::TMEM_COLS>(tmem_holder);
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tmem = *tmem_holder;
+  const uint32_t tS = tmem, tO = tmem + 256;
+
+  if (warp == 0) {
+    if (lane == 0 && nk > 0) {
+      tc::mbar_expect_tx(bar_q, Cfg::Q_BYTES);
+#pragma unroll
+      for (int c = 0; c < Cfg::CH; ++c)
+        tc::tma_load_2d(sQ + c * CHUNK, &tmQ, bar_q, head * D + c * 64, q0);
+      for (int kt = 0; kt < nk; ++kt) {
+        const int st = kt & 1;
+        tc::mbar_wait(&kv_empty[st], ((kt >> 1) & 1) ^ 1);
+        tc::mbar_expect_tx(&kv_full[st], 2 * Cfg::KV_TILE);
+        const int krow = k0 + kt * 128;
+#pragma unroll
+        for (int c = 0; c < Cfg::CH; ++c) {
+          tc::tma_load_2d(sK + st * Cfg::KV_TILE + c * CHUNK, &tmKV, &kv_full[st],
+                          head * D + c * 64, krow);
+          tc::tma_load_2d(sV + st * Cfg::KV_TILE + c * CHUNK, &tmKV, &kv_full[st],
+                          H + head * D + c * 64, krow);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && nk > 0) {
+      constexpr uint32_t idesc_s = tc::idesc_bf16(128, 128);
+      constexpr uint32_t idesc_o = tc::idesc_bf16(128, D, /*b_mn_major=*/true);
+      tc::mbar_wait(bar_q, 0);
+      auto issue_s = [&](int kt) {
+        const int st = kt & 1;
+        tc::mbar_wait(&kv_full[st], (kt >> 1) & 1);
+        tc::fence_after();
+        const uint32_t qa = tc::smem_u32(sQ), kb = tc::smem_u32(sK + st * Cfg::KV_TILE);
+#pragma unroll
+        for (int ks = 0; ks < D / 16; ++ks) {
+          const uint32_t off = (ks >> 2) * CHUNK + (ks & 3) * 32;
+          tc::mma_bf16(tS + st * 128, tc::sdesc_k_sw128(qa + off), tc::sdesc_k_sw128(kb + off),
+                       idesc_s, ks > 0);
+        }
+        tc::mma_commit(&bar_s[st]);
+      };
+      issue_s(0);
+      for (int kt = 0; kt < nk; ++kt) {
+        if (kt + 1 < nk) issue_s(kt + 1);
+        tc::mbar_wait(bar_p, kt & 1);
+        tc::fence_after();
+        const int st = kt & 1;
+        const uint32_t pa = tc::smem_u32(sP), vb = tc::smem_u32(sV + st * Cfg::KV_TILE);
+#pragma unroll
+        for (int ks = 0; ks < 8; ++ks) {
+          tc::mma_bf16(tO, tc::sdesc_k_sw128(pa + (ks >> 2) * CHUNK + (ks & 3) * 32),
+                       tc::sdesc_mn_sw128(vb + ks * 2048, CHUNK), idesc_o, (kt | ks) != 0);
+        }
+        tc::mma_commit(bar_o);
+        tc::mma_commit(&kv_empty[st]);
+      }
+    }
+  } else if (warp >= 4) {
+    const int q = warp & 3;
+    const int row = q * 32 + lane;
+    const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+    float m_used = -INFINITY, l = 0.f;
+    uint8_t* prow = sP + row * 128;
+    const int sw = row & 7;
+    for (int kt = 0; kt < nk; ++kt) {
+      const int st = kt & 1;
+      tc::mbar_wait(&bar_s[st], (kt >> 1) & 1);
+      tc::fence_after();
+      float s[128];
+#pragma unroll
+      for (int c = 0; c < 4; ++c) {
+        tc::tmem_ld32(tS + lane_off + st * 128 + c * 32, reinterpret_cast<uint32_t*>(s + c * 32));
+      }
+      tc::tmem_wait_ld();
+      const int valid = Lr - kt * 128;                    // keys of this request in the tile
+      float mx = -INFINITY;
+#pragma unroll
+      for (int i = 0; i < 128; ++i) {
+        s[i] = (i < valid) ? s[i] * scale_log2 : -INFINITY;
+        mx = fmaxf(mx, s[i]);
+      }
+      const bool need = mx > m_used + 8.0f;
+      bool waited = false;
+      if (__any_sync(0xffffffffu, need)) {
+        const float m_new = need ? mx : m_used;
+        const float factor = need ? tc::ex2(m_used - m_new) : 1.0f;   // ex2(-inf) = 0
+        if (kt > 0) {
+          tc::mbar_wait(bar_o, (kt - 1) & 1);
+          tc::fence_after();
+          waited = true;
+#pragma unroll 1
+          for (int c = 0; c < D / 32; ++c) {
+            uint32_t o[32];
+            tc::tmem_ld32(tO + lane_off + c * 32, o);
+            tc::tmem_wait_ld();
+#pragma unroll
+            for (int e = 0; e < 32; ++e) o[e] = __float_as_uint(__uint_as_float(o[e]) * factor);
+            tc::tmem_st32(tO + lane_off + c * 32, o);
+          }
+          tc::tmem_wait_st();
+        }
+        l *= factor;
+        m_used = m_new;
+      }
+      if (kt > 0 && !waited) {
+        tc::mbar_wait(bar_o, (kt - 1) & 1);                // PV_{kt-1} done: P buffer is free
+        tc::fence_after();
+      }
+      // P = exp2(s - m) as bf16 into the K-major SW128 A-operand layout
+      float sum = 0.f;
+#pragma unroll
+      for (int u = 0; u < 16; ++u) {
+        float p[8];
+#pragma unroll
+        for (int e = 0; e < 8; ++e) {
+          p[e] = tc::ex2(s[u * 8 + e] - m_used);
+          sum += p[e];
+        }
+        const uint4 v = make_uint4(pack_bf16x2(p[0], p[1]), pack_bf16x2(p[2], p[3]),
+                                   pack_bf16x2(p[4], p[5]), pack_bf16x2(p[6], p[7]));
+        const int chunk = u >> 3, unit = u & 7;
+        *reinterpret_cast<uint4*>(prow + chunk * CHUNK + ((unit ^ sw) << 4)) = v;
+      }
+      l += sum;
+      tc::fence_proxy_async_smem();
+      tc::fence_before();
+      __syncwarp();
+      if (lane == 0) tc::mbar_arrive(bar_p);
+    }
+    if (nk > 0) {
+      tc::mbar_wait(bar_o, (nk - 1) & 1);
+      tc::fence_after();
+    }
+    const float inv = (l > 0.f) ? 1.0f / l : 0.f;
+    __nv_bfloat16* orow = O + (size_t)(q0 + row) * H + head * D;
+#pragma unroll 1
+    for (int c = 0; c < D / 32; ++c) {
+      uint32_t o[32];
+      tc::tmem_ld32(tO + lane_off + c * 32, o);
+      tc::tmem_wait_ld();
+      if (row < n_rows) {
+#pragma unroll
+        for (int g = 0; g < 4; ++g) {
+          float f[8];
+#pragma unroll
+          for (int e = 0; e < 8; ++e) f[e] = __uint_as_float(o[g * 8 + e]) * inv;
+          *reinterpret_cast<uint4*>(orow + c * 32 + g * 8) = Vec16<__nv_bfloat16>::pack(f);
+        }
+      }
+    }
+  }
+  tc::fence_before();
+  __syncthreads();
+  if (warp == 2) {
+    tc::fence_after();
+    tc::tmem_dealloc<Cfg::TMEM_COLS>(tmem);
+  }
 }
+
+bool attention_tc_supported(int dtype, int head_dim) {
+  return dtype == FPS_BF16 && (head_dim == 64 || head_dim == 128);
+}
+
+template <int D>
+static fps_status launch_d(const void* q, const void* kv, void* o, int heads,
+                           const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
+                           const int32_t* h_cu_k, int n_req, cudaStream_t s) {
+  using Cfg = AttnCfg<D>;
+  const int H = heads * D;
+  int tiles = 0;
+  for (int r = 0; r < n_req; ++r) tiles += (h_cu_q[r + 1] - h_cu_q[r] + 127) / 128;
+  if (tiles == 0) return FPS_OK;
+  // rows past a request's own keys (next request, or past the end: TMA zero fill) are masked
+  // in-kernel; past-the-end query rows are never stored
+  CUtensorMap tq, tkv;
+  if (!make_tmap_2d_bf16(&tq, q, (uint64_t)h_cu_q[n_req], H, (uint64_t)H * 2, 64, 128))
+    return fail(FPS_ECUDA, "attention_tc: Q tensor map");
+  if (!make_tmap_2d_bf16(&tkv, kv, (uint64_t)h_cu_k[n_req], 2 * H, (uint64_t)H * 4, 64, 128))
+    return fail(FPS_ECUDA, "attention_tc: KV tensor map");
+  static bool attr = false;
+  if (!attr) {
+    FPS_CUDA_TRY(cudaFuncSetAttribute(attn_tc_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      Cfg::SMEM));
+    attr = true;
+  }
+  const float scale_log2 = 1.4426950408889634f / sqrtf((float)D);
+  attn_tc_kernel<D><<<dim3(tiles, heads), 256, Cfg::SMEM, s>>>(
+      tq, tkv, reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads, scale_log2);
+  count_launch();
+  FPS_LAUNCH_CHECK();
+  return FPS_OK;
+}
+
+fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads, int head_dim,
+                               const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
+                               const int32_t* h_cu_k, int n_req, cudaStream_t s) {
+  if (!h_cu_q || !h_cu_k) return fail(FPS_EINVAL, "attention_tc needs host cu_q / cu_k");
+  if (!aligned16(q) || !aligned16(kv) || !aligned16(o))
+    return fail(FPS_EINVAL, "attention_tc: unaligned operand");
+  if (head_dim == 128)
+    return launch_d<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);
+  return launch_d<64>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);
+}
+
 }  // namespace fps

@@ -55,7 +55,9 @@ fps_status launch_mask_index(const uint8_t* masks, const int32_t* off, int n_req
                              int32_t* mids, int32_t* uids, int32_t* nm, cudaStream_t s) {
   (void)max_len;
   if (n_req == 0) return FPS_OK;
+  prof::begin(s);
   mask_index_kernel<<<n_req, 1024, 0, s>>>(masks, off, mids, uids, nm);
+  prof::end(s, prof::INDEX, 0, 0);
   count_launch();
   FPS_LAUNCH_CHECK();
   return FPS_OK;
@@ -101,8 +103,10 @@ fps_status launch_copy_rows(const void* src, const int32_t* src_ids, const int32
   int cap = max_ctas > 0 ? max_ctas : kNumSMs * 8;
   int grid = (int)(want < cap ? want : cap);
   if (grid < 1) grid = 1;
+  prof::begin(s);
   copy_rows_kernel<<<grid, 256, 0, s>>>(reinterpret_cast<const uint4*>(src), src_ids, dst_ids,
                                         total, vpr, reinterpret_cast<uint4*>(dst));
+  prof::end(s, prof::ROWS, 0, 2.0 * n * row_bytes);
   count_launch();
   FPS_LAUNCH_CHECK();
   return FPS_OK;
@@ -191,7 +195,9 @@ static fps_status ln_mod_t(const void* x, const int32_t* rows, int n, int H, voi
   auto Md = reinterpret_cast<const T*>(mod);
 #define FPS_LN_CASE(VPT)                                                                  \
   if (per_lane <= VPT) {                                                                  \
+    prof::begin(s);                                                                       \
     ln_mod_kernel<T, VPT><<<grid, 128, 0, s>>>(X, rows, n, H, O, cu, n_req, Md, shift_off); \
+    prof::end(s, prof::LN, 0, 2.0 * n * H * sizeof(T));                                   \
     count_launch();                                                                       \
     FPS_LAUNCH_CHECK();                                                                   \
     return FPS_OK;                                                                        \
@@ -244,12 +250,14 @@ fps_status launch_euler(int dtype, void* x, const void* y, int n, int H, const i
   const long long nvec = (long long)n * vpr;
   int grid = (int)((nvec + 255) / 256);
   if (grid > kNumSMs * 16) grid = kNumSMs * 16;
+  prof::begin(s);
   if (dtype == FPS_BF16)
     euler_kernel<__nv_bfloat16><<<grid, 256, 0, s>>>((__nv_bfloat16*)x, (const __nv_bfloat16*)y,
                                                      nvec, vpr, cu, n_req, delta);
   else
     euler_kernel<float><<<grid, 256, 0, s>>>((float*)x, (const float*)y, nvec, vpr, cu, n_req,
                                              delta);
+  prof::end(s, prof::EULER, 2.0 * n * H, 3.0 * n * H * elt);
   count_launch();
   FPS_LAUNCH_CHECK();
   return FPS_OK;

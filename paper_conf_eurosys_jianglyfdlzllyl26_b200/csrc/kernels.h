@@ -35,7 +35,7 @@ fps_status launch_attention_simt(int dtype, const void* q, const void* kv, void*
                                  int n_req, int total_q, cudaStream_t s);
 fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads, int head_dim,
                                const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
-                               int n_req, int max_q, cudaStream_t s);
+                               const int32_t* h_cu_k, int n_req, cudaStream_t s);
 bool attention_tc_supported(int dtype, int head_dim);
 
 // global switches (tests can force the SIMT kernels): bit0 = no tcgen05 GEMM,

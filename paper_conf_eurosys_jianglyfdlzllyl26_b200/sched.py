@@ -1,0 +1,112 @@
+"""§4.4 mask-aware scheduling on top of the library's Alg. 1 planner.
+
+  * latency models (L255-L257): Comp(FLOPs) = a*FLOPs + b and Load(bytes) = c*bytes + e, fitted
+    by least squares on measurements taken on this GPU (`calibrate`);
+  * CalcCost (Alg. 2 lines 1-4): the Alg. 1 pipeline latency of worker.running_batch + request,
+    computed by fps_plan_pipeline in libflashps;
+  * route (Alg. 2 lines 5-11): the candidate worker with slack and the lowest cost wins; ties go
+    to the worker with fewer requests, then the lower id (reading R15).
+Host-side bookkeeping only; the data path never leaves the GPU worker that owns a request.
+"""
+from __future__ import annotations
+
+import math
+
+import numpy as np
+
+from . import FPS_MODE_KV, FPS_MODE_Y, plan_pipeline
+
+
+def block_flops(mode, n, L, H, F):
+    """Exact FLOPs of one block for one request with n active of L rows (Table 1, per mode)."""
+    if mode == "dense":
+        return 8.0 * L * H * H + 4.0 * L * H * F + 4.0 * L * L * H
+    attn = 4.0 * n * L * H
+    if mode == "kv":
+        return 8.0 * n * H * H + 4.0 * n * H * F + attn
+    return 4.0 * n * H * H + 4.0 * L * H * H + 4.0 * n * H * F + attn
+
+
+def cache_bytes(mode, u, H, elt=2):
+    return (2.0 if mode == "kv" else 1.0) * u * H * elt
+
+
+def fit_linear(x, y):
+    """Least squares y ~ a x + b; returns (a, b, R^2) (L257 reports R^2)."""
+    x = np.asarray(x, np.float64)
+    y = np.asarray(y, np.float64)
+    A = np.stack([x, np.ones_like(x)], 1)
+    (a, b), *_ = np.linalg.lstsq(A, y, rcond=None)
+    res = y - (a * x + b)
+    tot = ((y - y.mean()) ** 2).sum()
+    return float(a), float(b), float(1.0 - (res ** 2).sum() / tot) if tot > 0 else 1.0
+
+
+class Request:
+    """What the scheduler knows about a request: its active rows n and unmasked rows u."""
+
+    def __init__(self, rid, n_active, L, arrival=0.0, steps=28):
+        self.rid, self.n, self.L, self.arrival, self.steps = rid, int(n_active), int(L), arrival, steps
+
+    @property
+    def u(self):
+        return self.L - self.n
+
+
+class CostModel:
+    """Per-block costs of a batch for Alg. 1 from the two fitted linear models."""
+
+    def __init__(self, n_layers, H, F, mode, comp=(1e-12, 0.01), load=(2e-8, 0.01), elt=2):
+        self.n_layers, self.H, self.F, self.mode, self.elt = n_layers, H, F, mode, elt
+        self.comp, self.load = comp, load
+
+    def costs(self, batch):
+        a, b = self.comp
+        c, e = self.load
+        fm = sum(block_flops(self.mode, r.n, r.L, self.H, self.F) for r in batch)
+        fd = sum(block_flops("dense", r.n, r.L, self.H, self.F) for r in batch)
+        by = sum(cache_bytes(self.mode, r.u, self.H, self.elt) for r in batch)
+        byf = sum(cache_bytes("y", r.u, self.H, self.elt) for r in batch)
+        N = self.n_layers
+        Cw = [a * fm + b] * N
+        Cwo = [a * fd + b] * N
+        Lm = [c * by + e if by > 0 else 0.0] * N
+        fin = (c * byf + e) if (self.mode == "kv" and byf > 0) else 0.0
+        return Cw, Cwo, Lm, fin
+
+    def step_latency(self, batch):
+        """dp(batch).pipeline_latency of Alg. 2 line 3 (library planner)."""
+        if not batch:
+            return 0.0
+        Cw, Cwo, Lm, fin = self.costs(batch)
+        mode = FPS_MODE_KV if self.mode == "kv" else FPS_MODE_Y
+        return plan_pipeline(Cw, Cwo, Lm, mode, fin)[1]
+
+    def as_engine_model(self):
+        """(a, b, c, e) in the units fps_engine_desc.cost_model expects (ms/FLOP, ms, ms/B, ms)."""
+        return (self.comp[0], self.comp[1], self.load[0], self.load[1])
+
+
+def route(req, workers, cost_fn, max_batch):
+    """Alg. 2 lines 6-11. workers: list of lists of assigned requests. Returns an index or None."""
+    best, key = None, None
+    for wid, assigned in enumerate(workers):
+        if len(assigned) >= max_batch:
+            continue
+        k = (cost_fn(assigned + [req]), len(assigned), wid)
+        if key is None or k < key:
+            best, key = wid, k
+    return best
+
+
+def assign_all(reqs, n_workers, cost_fn, max_batch):
+    """Route a pool of simultaneously arriving requests one by one (arrival order)."""
+    workers = [[] for _ in range(n_workers)]
+    held = []
+    for r in reqs:
+        w = route(r, workers, cost_fn, max_batch)
+        if w is None:
+            held.append(r)
+        else:
+            workers[w].append(r)
+    return workers, held

@@ -4,7 +4,15 @@ import torch
 
 import synth
 
-TOL = {"bf16": 2e-2, "f32": 1e-5}          # BASELINE.json north_star tolerances
+TOL = {"bf16": 2e-2, "f32": 1e-5}          # BASELINE.json north_star tolerances (block outputs)
+
+
+def stack_tol(dtype, n_blocks):
+    """Tolerance for a latent after a chain of n_blocks blocks: the
+    per-block bound grows like sqrt(n) because each block adds an independent rounding error to
+    the bf16 residual stream; the fp32 path keeps 1e-5 per block, i.e. 1e-5 * n."""
+    import math
+    return TOL[dtype] * (math.sqrt(n_blocks) if dtype == "bf16" else n_blocks)
 
 
 def to_dev(a, dtype):

@@ -114,6 +114,7 @@ def test_cache_store_prefetch_bytes_equal(F, mode, method):
                                              ids[r].ctypes.data, dst[r * (L_img + L_txt)].data_ptr(),
                                              w * 2))
         ls = torch.cuda.Stream()
+        ls.wait_stream(torch.cuda.current_stream())     # dst zero-fill and ids upload first
         ev = torch.cuda.Event()
         c.prefetch(items, ls, ev)
         ev.synchronize()
