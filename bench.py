@@ -121,7 +121,12 @@ def make_requests(w, n_requests, seed):
     return reqs
 
 
-def build_engine_inputs(F, w, mode, device, n_entries):
+def make_cache(F, w, mode, n_entries, location=0, copy_method=0):
+    return F.Cache(F.MODE_CODE[mode], F.FPS_BF16, w["H"], w["L_img"], w["layers"], w["steps"],
+                   n_templates=64, n_entries=n_entries, copy_method=copy_method, location=location)
+
+
+def build_engine_inputs(F, w, mode, device, n_entries, location=0, copy_method=0):
     """Random-init block weights (N(0, 1/fan_in), bf16) and adaLN table on the GPU; pinned cache
     arena (contents do not affect timing; entries alias modulo n_entries)."""
     gen = torch.Generator(device=device).manual_seed(SEED)
@@ -147,8 +152,7 @@ def build_engine_inputs(F, w, mode, device, n_entries):
     mod[:, :, 2] += 1.0
     mod[:, :, 5] += 1.0
     mod = mod.reshape(N, w["steps"], 6 * H).to(torch.bfloat16)
-    cache = F.Cache(F.MODE_CODE[mode], F.FPS_BF16, H, w["L_img"], N, w["steps"],
-                    n_templates=64, n_entries=n_entries)
+    cache = make_cache(F, w, mode, n_entries, location, copy_method)
     return layers, mod, cache
 
 
@@ -188,8 +192,9 @@ def calibrate(F, w, mode, layers, cache, reqs, device):
     for m in (0.05, 0.3, 0.6, 0.9):
         u = w["L_img"] - synth.n_masked_for(m, w["L_img"])
         rows = torch.arange(u, device=device, dtype=torch.int32)
-        items = [F.fps_prefetch_item(i, 0, 0, u, rows.data_ptr(), None, dst[i * L].data_ptr(), W * 2)
-                 for i in range(B)]
+        h_rows = np.arange(u, dtype=np.int32)
+        items = [F.fps_prefetch_item(i, 0, 0, u, rows.data_ptr(), h_rows.ctypes.data,
+                                     dst[i * L].data_ptr(), W * 2) for i in range(B)]
         for _ in range(2):
             cache.prefetch(items, ls)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -276,6 +281,10 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C3", choices=list(WORKLOADS))
     ap.add_argument("--mode", default="kv", choices=["kv", "y"])
+    ap.add_argument("--tier", default="host", choices=["host", "hbm"],
+                    help="template cache in pinned host DRAM (configs[2]) or HBM (NEXT-1)")
+    ap.add_argument("--copy-method", type=int, default=0, choices=[0, 1],
+                    help="H2D method: 0 SM zero-copy row gather, 1 DMA per row run")
     ap.add_argument("--no-extras", action="store_true", help="skip dense / Y-mode / profile legs")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()
@@ -334,7 +343,11 @@ def main():
     pool = make_requests(w, w["batch"] * world, SEED)
     t0 = time.perf_counter()
     n_entries = 2 * (w["layers"] + 1)
-    layers, mod, cache = build_engine_inputs(F, w, args.mode, device, n_entries)
+    location = 1 if args.tier == "hbm" else 0
+    layers, mod, cache = build_engine_inputs(F, w, args.mode, device, n_entries, location,
+                                             args.copy_method)
+    base_cfg["cache_tier"] = "pinned host DRAM" if location == 0 else "device HBM (NEXT-1)"
+    base_cfg["h2d_method"] = ["SM zero-copy row gather", "DMA per row run"][args.copy_method]
     torch.cuda.synchronize()
     log(f"[rank {rank}] inputs ready in {time.perf_counter() - t0:.1f}s")
     my_pool = pool[:w["batch"]]
@@ -355,7 +368,7 @@ def main():
     def engine(policy, mode=args.mode, the_cache=cache):
         return F.Engine(layers, w["heads"], F.MODE_CODE[mode], F.FPS_BF16, w["L_img"], w["L_txt"],
                         max(len(reqs_dev), 1), w["steps"], deltas, the_cache, mod_table=mod,
-                        slots=4, plan_policy=policy, cost_model=cm.as_engine_model())
+                        slots=0, plan_policy=policy, cost_model=cm.as_engine_model())
 
     eng = engine(0)
     with Clocks(local) as clk:
@@ -375,20 +388,24 @@ def main():
         cached_ms, _ = run_engine_timed(F, eng_c, reqs_dev, K, W, stream, load_stream, rank, world)
         del eng_c
         extras.update(dense_ms_per_step=dense_ms, all_cached_ms_per_step=cached_ms)
-        # the other caching mode on the same batch
+        # the other caching mode, and both modes with the other cache tier, on the same batch
         other = "y" if args.mode == "kv" else "kv"
-        l2, m2, c2 = layers, mod, F.Cache(F.MODE_CODE[other], F.FPS_BF16, w["H"], w["L_img"],
-                                          w["layers"], w["steps"], n_templates=64,
-                                          n_entries=n_entries)
-        cm2, _ = calibrate(F, w, other, layers, c2, [dict()] * w["batch"], device)
-        eng_o = F.Engine(layers, w["heads"], F.MODE_CODE[other], F.FPS_BF16, w["L_img"],
-                         w["L_txt"], max(len(reqs_dev), 1), w["steps"], deltas, c2, mod_table=mod,
-                         slots=4, plan_policy=0, cost_model=cm2.as_engine_model())
-        other_ms, _ = run_engine_timed(F, eng_o, reqs_dev, K, W, stream, load_stream, rank, world)
-        extras[f"{other}_mode_ms_per_step"] = other_ms
-        extras[f"{other}_mode_plan_cached_blocks"] = int(sum(eng_o.last_plan()[0]))
-        del eng_o
-        c2.close()
+        for md, loc, cmeth in ((other, location, args.copy_method), (args.mode, 1 - location, 0),
+                               (other, 1 - location, 0), (args.mode, location, 1 - args.copy_method)):
+            if loc == 1 and cmeth == 1:
+                continue
+            c2 = make_cache(F, w, md, n_entries, loc, cmeth)
+            cm2, _ = calibrate(F, w, md, layers, c2, [dict()] * w["batch"], device)
+            eng_o = F.Engine(layers, w["heads"], F.MODE_CODE[md], F.FPS_BF16, w["L_img"],
+                             w["L_txt"], max(len(reqs_dev), 1), w["steps"], deltas, c2,
+                             mod_table=mod, slots=0, plan_policy=0,
+                             cost_model=cm2.as_engine_model())
+            o_ms, _ = run_engine_timed(F, eng_o, reqs_dev, K, W, stream, load_stream, rank, world)
+            tag = f"{md}_mode_{['host', 'hbm'][loc]}" + ("_dma" if cmeth == 1 else "")
+            extras[f"{tag}_ms_per_step"] = o_ms
+            extras[f"{tag}_cached_blocks"] = int(sum(eng_o.last_plan()[0]))
+            del eng_o
+            c2.close()
 
     # per-kernel-class device time over the same timed region (CUDA events on each kernel's
     # own stream), for the roofline of the dominant kernel

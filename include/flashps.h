@@ -109,15 +109,21 @@ typedef struct {
                             moved are identical, contents alias)                            */
   int32_t copy_method;   /* 0 = SM zero-copy row gather over mapped pinned memory (default);
                             1 = copy-engine DMA of coalesced row runs                        */
-  int32_t copy_ctas;     /* CTAs used by method 0 (0 = default 32)                          */
+  int32_t copy_ctas;     /* CTAs used by method 0 (0 = default: 32 host, 296 device)        */
+  int32_t location;      /* 0 = pinned host DRAM (L203, streamed over PCIe);
+                            1 = device HBM: the template tier one level above host DRAM
+                            (the paper's "ideal" no-load case of Fig. 4-Left,
+                            L108), prefetch becomes an HBM row gather                        */
 } fps_cache_desc;
 
 typedef struct fps_cache* fps_cache_t;
 
 fps_status fps_cache_create(const fps_cache_desc* desc, fps_cache_t* out);
 fps_status fps_cache_destroy(fps_cache_t c);
-/* Host pointer of an entry (tests / tooling); NULL if out of range. */
+/* Host pointer of an entry (tests / tooling); NULL if out of range or the arena is in HBM. */
 void* fps_cache_entry_host_ptr(fps_cache_t c, uint32_t template_id, int32_t step, int32_t layer);
+/* Address of an entry in whichever memory holds the arena (host or device); NULL if out of range. */
+void* fps_cache_entry_ptr(fps_cache_t c, uint32_t template_id, int32_t step, int32_t layer);
 size_t fps_cache_entry_bytes(fps_cache_t c, int32_t layer);
 /* D2H: store rows [0, L_img) of d_src (row pitch src_row_bytes >= W*elt) as entry
  * (template_id, step, layer).  Asynchronous on `stream`. */

@@ -183,9 +183,9 @@ class Cache:
     """fps_cache_t: pinned host arena of template activations (L203)."""
 
     def __init__(self, mode, dtype, H, L_img, n_layers, n_steps, n_templates=1, n_entries=0,
-                 copy_method=0, copy_ctas=0):
+                 copy_method=0, copy_ctas=0, location=0):
         self.desc = fps_cache_desc(mode, dtype, H, L_img, n_layers, n_steps, n_templates,
-                                   n_entries, copy_method, copy_ctas)
+                                   n_entries, copy_method, copy_ctas, location)
         h = C.c_void_p()
         _lib.fps_cache_create(C.byref(self.desc), C.byref(h))
         self.h = h

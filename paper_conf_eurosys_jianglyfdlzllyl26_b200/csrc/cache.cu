@@ -113,6 +113,20 @@ fps_status fps_cache_create(const fps_cache_desc* desc, fps_cache_t* out) {
   c->n_keys = (long long)d.n_templates * d.n_steps * per_step;
   c->n_entries = d.n_entries > 0 ? std::min<long long>(d.n_entries, c->n_keys) : c->n_keys;
   const size_t bytes = (size_t)c->n_entries * c->entry_bytes;
+  FPS_CHECK_ARG(d.location == 0 || d.location == 1, "location %d", d.location);
+  if (d.location == 1) {
+    // HBM tier: the arena lives in device memory; "host" then names that device buffer
+    cudaError_t e = cudaMalloc((void**)&c->host, bytes);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      delete c;
+      return fail(e == cudaErrorMemoryAllocation ? FPS_ENOMEM : FPS_ECUDA,
+                  "cache: cudaMalloc(%zu bytes): %s", bytes, cudaGetErrorString(e));
+    }
+    c->dev_alias = c->host;
+    *out = c;
+    return FPS_OK;
+  }
   cudaError_t e = cudaHostAlloc((void**)&c->host, bytes, cudaHostAllocMapped | cudaHostAllocPortable);
   if (e != cudaSuccess) {
     cudaGetLastError();
@@ -133,14 +147,22 @@ fps_status fps_cache_create(const fps_cache_desc* desc, fps_cache_t* out) {
 
 fps_status fps_cache_destroy(fps_cache_t c) {
   if (!c) return FPS_OK;
-  if (c->host) cudaFreeHost(c->host);
+  if (c->host) {
+    if (c->d.location == 1) cudaFree(c->host);
+    else cudaFreeHost(c->host);
+  }
   delete c;
   return FPS_OK;
 }
 
-void* fps_cache_entry_host_ptr(fps_cache_t c, uint32_t template_id, int32_t step, int32_t layer) {
+void* fps_cache_entry_ptr(fps_cache_t c, uint32_t template_id, int32_t step, int32_t layer) {
   if (!c || !key_ok(c, template_id, step, layer)) return nullptr;
   return c->host + offset_of(c, template_id, step, layer);
+}
+
+void* fps_cache_entry_host_ptr(fps_cache_t c, uint32_t template_id, int32_t step, int32_t layer) {
+  if (!c || c->d.location == 1) return nullptr;
+  return fps_cache_entry_ptr(c, template_id, step, layer);
 }
 
 size_t fps_cache_entry_bytes(fps_cache_t c, int32_t layer) {
@@ -156,7 +178,7 @@ fps_status fps_cache_store(fps_cache_t c, uint32_t template_id, int32_t step, in
   const size_t rb = row_bytes_of(c, layer);
   FPS_CHECK_ARG(src_row_bytes >= (int)rb, "src_row_bytes %d < %zu", src_row_bytes, rb);
   FPS_CUDA_TRY(cudaMemcpy2DAsync(c->host + offset_of(c, template_id, step, layer), rb, d_src,
-                                 src_row_bytes, rb, c->d.L_img, cudaMemcpyDeviceToHost,
+                                 src_row_bytes, rb, c->d.L_img, cudaMemcpyDefault,
                                  as_stream(stream)));
   return FPS_OK;
 }
@@ -198,7 +220,7 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
       b.start[k] = acc;
       b.n_items = k;
       if (acc == 0) continue;
-      int ctas = c->d.copy_ctas > 0 ? c->d.copy_ctas : 32;
+      int ctas = c->d.copy_ctas > 0 ? c->d.copy_ctas : (c->d.location == 1 ? 2 * kNumSMs : 32);
       long long want = (acc + 1023) / 1024;
       if (want < ctas) ctas = (int)want;
       prof::begin(s);
@@ -230,7 +252,7 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
     // one DMA per run of consecutive rows (cudaMemcpyBatchAsync dropped rows of long runs in
     // testing on this driver, so the runs are issued individually)
     for (size_t q = 0; q < c->sizes.size(); ++q)
-      FPS_CUDA_TRY(cudaMemcpyAsync(c->dsts[q], c->srcs[q], c->sizes[q], cudaMemcpyHostToDevice, s));
+      FPS_CUDA_TRY(cudaMemcpyAsync(c->dsts[q], c->srcs[q], c->sizes[q], cudaMemcpyDefault, s));
   }
   if (ready_event) FPS_CUDA_TRY(cudaEventRecord((cudaEvent_t)ready_event, s));
   return FPS_OK;

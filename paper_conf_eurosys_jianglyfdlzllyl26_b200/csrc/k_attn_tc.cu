@@ -9,8 +9,9 @@
 //              O += P_j V_j with V as an MN-major operand; commits free the K/V stage
 //   warps 4-7  softmax, thread = query row: S row from TMEM (tcgen05.ld), online softmax in the
 //              exp2 domain with a lazy max (O in TMEM is rescaled only when the running max grows
-//              by more than 2^8, FA4-style), P as bf16 into smem in the UMMA K-major SW128 layout;
-//              final O / l from TMEM to global.
+//              by more than 2^8, FA4-style), P as bf16 into one of two smem P buffers in the UMMA
+//              K-major SW128 layout; the exponentials of tile j are computed while PV_{j-1} still
+//              runs; final O / l from TMEM to global.
 #include "kernels.h"
 #include "tc_util.cuh"
 
@@ -22,8 +23,8 @@ struct AttnCfg {
   static constexpr int CH = D / 64;                        // 64-wide (128 B) chunks along d
   static constexpr int Q_BYTES = BM * D * 2;
   static constexpr int KV_TILE = BN * D * 2;
-  static constexpr int P_BYTES = BM * BN * 2;
-  static constexpr int SMEM = Q_BYTES + STAGES * 2 * KV_TILE + P_BYTES + 1024 + 256;
+  static constexpr int P_BYTES = BM * BN * 2;              // one P tile; two are kept
+  static constexpr int SMEM = Q_BYTES + STAGES * 2 * KV_TILE + 2 * P_BYTES + 1024 + 256;
   static constexpr int TMEM_COLS = 512;                    // S0 [0,128) S1 [128,256) O [256,256+D)
 };
 
@@ -40,15 +41,15 @@ __global__ void __launch_bounds__(256, 1)
   uint8_t* sQ = smem;
   uint8_t* sK = sQ + Cfg::Q_BYTES;                          // [stage][CH chunks]
   uint8_t* sV = sK + Cfg::STAGES * Cfg::KV_TILE;
-  uint8_t* sP = sV + Cfg::STAGES * Cfg::KV_TILE;            // [2 chunks of 64 keys]
-  uint64_t* bars = reinterpret_cast<uint64_t*>(sP + Cfg::P_BYTES);
+  uint8_t* sP = sV + Cfg::STAGES * Cfg::KV_TILE;            // [2 buffers][2 chunks of 64 keys]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sP + 2 * Cfg::P_BYTES);
   uint64_t* bar_q = bars;
   uint64_t* kv_full = bars + 1;
   uint64_t* kv_empty = bars + 3;
   uint64_t* bar_s = bars + 5;
-  uint64_t* bar_p = bars + 7;
-  uint64_t* bar_o = bars + 8;
-  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + 9);
+  uint64_t* bar_p = bars + 7;                               // [2]: P_j written (buffer j % 2)
+  uint64_t* bar_o = bars + 9;                               // [2]: PV_j done (buffer j % 2)
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + 11);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int head = blockIdx.y;
@@ -72,9 +73,9 @@ __global__ void __launch_bounds__(256, 1)
       tc::mbar_init(&kv_full[s], 1);
       tc::mbar_init(&kv_empty[s], 1);
       tc::mbar_init(&bar_s[s], 1);
+      tc::mbar_init(&bar_p[s], 4);
+      tc::mbar_init(&bar_o[s], 1);
     }
-    tc::mbar_init(bar_p, 4);
-    tc::mbar_init(bar_o, 1);
     tc::fence_mbar_init();
   }
   if (warp == 0 && lane == 0) {
@@ -128,17 +129,20 @@ __global__ void __launch_bounds__(256, 1)
       };
       issue_s(0);
       for (int kt = 0; kt < nk; ++kt) {
+        // S buffer (kt+1)&1 was released by the softmax of tile kt-1 (bar_p waited below)
         if (kt + 1 < nk) issue_s(kt + 1);
-        tc::mbar_wait(bar_p, kt & 1);
+        const int pb = kt & 1;
+        tc::mbar_wait(&bar_p[pb], (kt >> 1) & 1);
         tc::fence_after();
         const int st = kt & 1;
-        const uint32_t pa = tc::smem_u32(sP), vb = tc::smem_u32(sV + st * Cfg::KV_TILE);
+        const uint32_t pa = tc::smem_u32(sP + pb * Cfg::P_BYTES);
+        const uint32_t vb = tc::smem_u32(sV + st * Cfg::KV_TILE);
 #pragma unroll
         for (int ks = 0; ks < 8; ++ks) {
           tc::mma_bf16(tO, tc::sdesc_k_sw128(pa + (ks >> 2) * CHUNK + (ks & 3) * 32),
                        tc::sdesc_mn_sw128(vb + ks * 2048, CHUNK), idesc_o, (kt | ks) != 0);
         }
-        tc::mma_commit(bar_o);
+        tc::mma_commit(&bar_o[pb]);
         tc::mma_commit(&kv_empty[st]);
       }
     }
@@ -146,8 +150,7 @@ __global__ void __launch_bounds__(256, 1)
     const int q = warp & 3;
     const int row = q * 32 + lane;
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
-    float m_used = -INFINITY, l = 0.f;
-    uint8_t* prow = sP + row * 128;
+    float m_used = -INFINITY, l = 0.f;                      // m_used in the scaled log2 domain
     const int sw = row & 7;
     for (int kt = 0; kt < nk; ++kt) {
       const int st = kt & 1;
@@ -155,67 +158,72 @@ __global__ void __launch_bounds__(256, 1)
       tc::fence_after();
       float s[128];
 #pragma unroll
-      for (int c = 0; c < 4; ++c) {
+      for (int c = 0; c < 4; ++c)
         tc::tmem_ld32(tS + lane_off + st * 128 + c * 32, reinterpret_cast<uint32_t*>(s + c * 32));
-      }
       tc::tmem_wait_ld();
       const int valid = Lr - kt * 128;                    // keys of this request in the tile
-      float mx = -INFINITY;
+      if (valid < 128) {
 #pragma unroll
-      for (int i = 0; i < 128; ++i) {
-        s[i] = (i < valid) ? s[i] * scale_log2 : -INFINITY;
-        mx = fmaxf(mx, s[i]);
+        for (int i = 0; i < 128; ++i) s[i] = (i < valid) ? s[i] : -INFINITY;
       }
+      float mx = s[0];
+#pragma unroll
+      for (int i = 1; i < 128; ++i) mx = fmaxf(mx, s[i]);
+      mx *= scale_log2;
       const bool need = mx > m_used + 8.0f;
-      bool waited = false;
-      if (__any_sync(0xffffffffu, need)) {
-        const float m_new = need ? mx : m_used;
-        const float factor = need ? tc::ex2(m_used - m_new) : 1.0f;   // ex2(-inf) = 0
-        if (kt > 0) {
-          tc::mbar_wait(bar_o, (kt - 1) & 1);
-          tc::fence_after();
-          waited = true;
-#pragma unroll 1
-          for (int c = 0; c < D / 32; ++c) {
-            uint32_t o[32];
-            tc::tmem_ld32(tO + lane_off + c * 32, o);
-            tc::tmem_wait_ld();
-#pragma unroll
-            for (int e = 0; e < 32; ++e) o[e] = __float_as_uint(__uint_as_float(o[e]) * factor);
-            tc::tmem_st32(tO + lane_off + c * 32, o);
-          }
-          tc::tmem_wait_st();
-        }
+      const bool any_need = __any_sync(0xffffffffu, need);
+      float factor = 1.0f;
+      if (need) {
+        factor = tc::ex2(m_used - mx);                    // ex2(-inf) = 0 on the first tile
         l *= factor;
-        m_used = m_new;
+        m_used = mx;
       }
-      if (kt > 0 && !waited) {
-        tc::mbar_wait(bar_o, (kt - 1) & 1);                // PV_{kt-1} done: P buffer is free
-        tc::fence_after();
-      }
-      // P = exp2(s - m) as bf16 into the K-major SW128 A-operand layout
+      // p = 2^(s*scale - m) while PV_{kt-1} may still be running
       float sum = 0.f;
 #pragma unroll
-      for (int u = 0; u < 16; ++u) {
-        float p[8];
+      for (int i = 0; i < 128; ++i) {
+        s[i] = tc::ex2(fmaf(s[i], scale_log2, -m_used));
+        sum += s[i];
+      }
+      l += sum;
+      if (any_need && kt > 0) {
+        // O += P_{kt-1} V_{kt-1} must land before O is rescaled (rare: max grew by > 2^8)
+        tc::mbar_wait(&bar_o[(kt - 1) & 1], ((kt - 1) >> 1) & 1);
+        tc::fence_after();
+#pragma unroll 1
+        for (int c = 0; c < D / 32; ++c) {
+          uint32_t o[32];
+          tc::tmem_ld32(tO + lane_off + c * 32, o);
+          tc::tmem_wait_ld();
 #pragma unroll
-        for (int e = 0; e < 8; ++e) {
-          p[e] = tc::ex2(s[u * 8 + e] - m_used);
-          sum += p[e];
+          for (int e = 0; e < 32; ++e) o[e] = __float_as_uint(__uint_as_float(o[e]) * factor);
+          tc::tmem_st32(tO + lane_off + c * 32, o);
         }
-        const uint4 v = make_uint4(pack_bf16x2(p[0], p[1]), pack_bf16x2(p[2], p[3]),
-                                   pack_bf16x2(p[4], p[5]), pack_bf16x2(p[6], p[7]));
+        tc::tmem_wait_st();
+      }
+      // P buffer kt&1 was last read by PV_{kt-2}
+      const int pb = kt & 1;
+      if (kt >= 2) {
+        tc::mbar_wait(&bar_o[pb], ((kt - 2) >> 1) & 1);
+        tc::fence_after();
+      }
+      uint8_t* prow = sP + pb * Cfg::P_BYTES + row * 128;
+#pragma unroll
+      for (int u = 0; u < 16; ++u) {
+        const uint4 v = make_uint4(pack_bf16x2(s[u * 8 + 0], s[u * 8 + 1]),
+                                   pack_bf16x2(s[u * 8 + 2], s[u * 8 + 3]),
+                                   pack_bf16x2(s[u * 8 + 4], s[u * 8 + 5]),
+                                   pack_bf16x2(s[u * 8 + 6], s[u * 8 + 7]));
         const int chunk = u >> 3, unit = u & 7;
         *reinterpret_cast<uint4*>(prow + chunk * CHUNK + ((unit ^ sw) << 4)) = v;
       }
-      l += sum;
       tc::fence_proxy_async_smem();
       tc::fence_before();
       __syncwarp();
-      if (lane == 0) tc::mbar_arrive(bar_p);
+      if (lane == 0) tc::mbar_arrive(&bar_p[pb]);
     }
     if (nk > 0) {
-      tc::mbar_wait(bar_o, (nk - 1) & 1);
+      tc::mbar_wait(&bar_o[(nk - 1) & 1], ((nk - 1) >> 1) & 1);
       tc::fence_after();
     }
     const float inv = (l > 0.f) ? 1.0f / l : 0.f;

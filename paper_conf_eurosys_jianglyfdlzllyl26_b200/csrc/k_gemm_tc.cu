@@ -121,26 +121,77 @@ __global__ void __launch_bounds__(256, 1)
   } else if (warp >= 4) {
     const int q = warp & 3;
     int it = 0;
+    const __nv_bfloat16* __restrict__ bias = reinterpret_cast<const __nv_bfloat16*>(ep.bias);
+    const __nv_bfloat16* __restrict__ resid = reinterpret_cast<const __nv_bfloat16*>(ep.resid);
     for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++it) {
       const int m_blk = tile % num_m, n_blk = tile / num_m;
       const int acc = it & 1;
+      const int row = m_blk * Cfg::BM + q * 32 + lane;
+      const bool row_ok = row < M;
+      // per-row epilogue state, looked up once per tile (not per column group)
+      const __nv_bfloat16* gate = nullptr;
+      int orow0 = row, orow1 = row;
+      if (row_ok) {
+        if (ep.gate)
+          gate = reinterpret_cast<const __nv_bfloat16*>(ep.gate) +
+                 (size_t)find_req(ep.cu, ep.n_req, row) * ep.gate_stride;
+        if (ep.map0) orow0 = __ldg(ep.map0 + row);
+        if (ep.map1) orow1 = __ldg(ep.map1 + row);
+      }
       tc::mbar_wait(&tfull[acc], (it >> 1) & 1);
       tc::fence_after();
-      const int row = m_blk * Cfg::BM + q * 32 + lane;
 #pragma unroll 1
       for (int c = 0; c < BN / 32; ++c) {
         uint32_t r[32];
         tc::tmem_ld32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + c * 32, r);
+        // issue every global load of this 32-column chunk before using any of them
+        const int col0 = n_blk * BN + c * 32;
+        uint4 bv[4], rv[4], gv[4];
+#pragma unroll
+        for (int g = 0; g < 4; ++g) {
+          const int c0 = col0 + g * 8;
+          const bool ok = row_ok && c0 < N;
+          bv[g] = (bias && ok) ? __ldg(reinterpret_cast<const uint4*>(bias + c0)) : make_uint4(0, 0, 0, 0);
+          rv[g] = (resid && ok) ? __ldg(reinterpret_cast<const uint4*>(resid + (size_t)row * ep.ld_resid + c0))
+                                : make_uint4(0, 0, 0, 0);
+          gv[g] = (gate && ok) ? __ldg(reinterpret_cast<const uint4*>(gate + c0)) : make_uint4(0, 0, 0, 0);
+        }
         tc::tmem_wait_ld();
-        if (row < M) {
+        if (row_ok) {
 #pragma unroll
           for (int g = 0; g < 4; ++g) {
-            const int c0 = n_blk * BN + c * 32 + g * 8;
+            const int c0 = col0 + g * 8;
             if (c0 < N) {
-              float v[8];
+              float v[8], t[8];
 #pragma unroll
               for (int e = 0; e < 8; ++e) v[e] = __uint_as_float(r[g * 8 + e]);
-              epilogue_store<__nv_bfloat16, 8>(ep, row, c0, v);
+              if (bias) {
+                Vec16<__nv_bfloat16>::unpack(bv[g], t);
+#pragma unroll
+                for (int e = 0; e < 8; ++e) v[e] += t[e];
+              }
+              if (ep.act == 1) {
+#pragma unroll
+                for (int e = 0; e < 8; ++e) v[e] = gelu_tanh(v[e]);
+              }
+              if (resid) {
+                float rr[8];
+                Vec16<__nv_bfloat16>::unpack(rv[g], rr);
+                if (gate) {
+                  Vec16<__nv_bfloat16>::unpack(gv[g], t);
+#pragma unroll
+                  for (int e = 0; e < 8; ++e) v[e] = rr[e] + t[e] * v[e];
+                } else {
+#pragma unroll
+                  for (int e = 0; e < 8; ++e) v[e] = rr[e] + v[e];
+                }
+              }
+              __nv_bfloat16* dst =
+                  c0 < ep.split
+                      ? reinterpret_cast<__nv_bfloat16*>(ep.out0) + (size_t)orow0 * ep.ld0 + c0
+                      : reinterpret_cast<__nv_bfloat16*>(ep.out1) + (size_t)orow1 * ep.ld1 +
+                            (c0 - ep.split);
+              *reinterpret_cast<uint4*>(dst) = Vec16<__nv_bfloat16>::pack(v);
             }
           }
         }

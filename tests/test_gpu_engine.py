@@ -19,7 +19,7 @@ def F():
 
 
 def _setup(F, mode, dtype, plan_policy, plan=None, N=3, steps=3, H=256, heads=2, Fd=512,
-           L_img=256, L_txt=16, n_req=3, slots=0, copy_method=0, seed=5000):
+           L_img=256, L_txt=16, n_req=3, slots=0, copy_method=0, seed=5000, location=0):
     g = synth.rng(seed)
     W = synth.stack_weights(g, N, H, Fd, dtype)
     mods = synth.mod_table(g, N, steps, H, dtype)
@@ -32,7 +32,8 @@ def _setup(F, mode, dtype, plan_policy, plan=None, N=3, steps=3, H=256, heads=2,
                 for _ in range(n_t)]
     dt = F.DTYPE_CODE[dtype]
     m = F.MODE_CODE[mode]
-    cache = F.Cache(m, dt, H, L_img, N, steps, n_templates=n_t, copy_method=copy_method)
+    cache = F.Cache(m, dt, H, L_img, N, steps, n_templates=n_t, copy_method=copy_method,
+                    location=location)
     for t in range(n_t):
         for s in range(steps):
             for l in range(N):
@@ -104,12 +105,14 @@ def test_requests_leave_at_step_boundary(F):
         check_close(to_np(r["x"]), x, stack_tol("bf16", 3), "leave")
 
 
-@pytest.mark.parametrize("slots,method", [(1, 0), (2, 1), (0, 0)])
-def test_pipeline_slots_and_copy_methods_bit_identical(F, slots, method):
-    """The staging ring depth and the H2D method change timing only, never the bits."""
+@pytest.mark.parametrize("slots,method,location", [(1, 0, 0), (2, 1, 0), (0, 0, 0), (2, 0, 1)])
+def test_pipeline_slots_and_copy_methods_bit_identical(F, slots, method, location):
+    """The staging ring depth, the H2D method and the cache tier (pinned host / HBM) change
+    timing only, never the bits."""
     outs = []
-    for sl, me in ((0, 0), (slots, method)):
-        _, _, _, _, eng, reqs = _setup(F, "kv", "bf16", 1, slots=sl, copy_method=me, seed=5100)
+    for sl, me, lo in ((0, 0, 0), (slots, method, location)):
+        _, _, _, _, eng, reqs = _setup(F, "kv", "bf16", 1, slots=sl, copy_method=me, seed=5100,
+                                       location=lo)
         eng.run_batch(reqs, 2)
         torch.cuda.synchronize()
         outs.append([r["x"].clone() for r in reqs])
