@@ -220,7 +220,8 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
       b.start[k] = acc;
       b.n_items = k;
       if (acc == 0) continue;
-      int ctas = c->d.copy_ctas > 0 ? c->d.copy_ctas : (c->d.location == 1 ? 2 * kNumSMs : 32);
+      // few CTAs: the copy overlaps the compute stream and should not crowd it out
+      int ctas = c->d.copy_ctas > 0 ? c->d.copy_ctas : (c->d.location == 1 ? 64 : 32);
       long long want = (acc + 1023) / 1024;
       if (want < ctas) ctas = (int)want;
       prof::begin(s);

@@ -44,12 +44,14 @@ __global__ void __launch_bounds__(256, 1)
   uint8_t* sP = sV + Cfg::STAGES * Cfg::KV_TILE;            // [2 buffers][2 chunks of 64 keys]
   uint64_t* bars = reinterpret_cast<uint64_t*>(sP + 2 * Cfg::P_BYTES);
   uint64_t* bar_q = bars;
-  uint64_t* kv_full = bars + 1;
-  uint64_t* kv_empty = bars + 3;
-  uint64_t* bar_s = bars + 5;
+  uint64_t* k_full = bars + 1;                              // K and V rings are separate so
+  uint64_t* k_empty = bars + 3;                             // K_j+2 loads as soon as S_j is
+  uint64_t* bar_s = bars + 5;                               // done, long before PV_j frees V
   uint64_t* bar_p = bars + 7;                               // [2]: P_j written (buffer j % 2)
   uint64_t* bar_o = bars + 9;                               // [2]: PV_j done (buffer j % 2)
-  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + 11);
+  uint64_t* v_full = bars + 11;
+  uint64_t* v_empty = bars + 13;
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + 15);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int head = blockIdx.y;
@@ -70,8 +72,10 @@ __global__ void __launch_bounds__(256, 1)
   if (threadIdx.x == 0) {
     tc::mbar_init(bar_q, 1);
     for (int s = 0; s < 2; ++s) {
-      tc::mbar_init(&kv_full[s], 1);
-      tc::mbar_init(&kv_empty[s], 1);
+      tc::mbar_init(&k_full[s], 1);
+      tc::mbar_init(&k_empty[s], 1);
+      tc::mbar_init(&v_full[s], 1);
+      tc::mbar_init(&v_empty[s], 1);
       tc::mbar_init(&bar_s[s], 1);
       tc::mbar_init(&bar_p[s], 4);
       tc::mbar_init(&bar_o[s], 1);
@@ -97,16 +101,24 @@ __global__ void __launch_bounds__(256, 1)
         tc::tma_load_2d(sQ + c * CHUNK, &tmQ, bar_q, head * D + c * 64, q0);
       for (int kt = 0; kt < nk; ++kt) {
         const int st = kt & 1;
-        tc::mbar_wait(&kv_empty[st], ((kt >> 1) & 1) ^ 1);
-        tc::mbar_expect_tx(&kv_full[st], 2 * Cfg::KV_TILE);
-        const int krow = k0 + kt * 128;
+        tc::mbar_wait(&k_empty[st], ((kt >> 1) & 1) ^ 1);
+        tc::mbar_expect_tx(&k_full[st], Cfg::KV_TILE);
 #pragma unroll
-        for (int c = 0; c < Cfg::CH; ++c) {
-          tc::tma_load_2d(sK + st * Cfg::KV_TILE + c * CHUNK, &tmKV, &kv_full[st],
-                          head * D + c * 64, krow);
-          tc::tma_load_2d(sV + st * Cfg::KV_TILE + c * CHUNK, &tmKV, &kv_full[st],
-                          H + head * D + c * 64, krow);
-        }
+        for (int c = 0; c < Cfg::CH; ++c)
+          tc::tma_load_2d(sK + st * Cfg::KV_TILE + c * CHUNK, &tmKV, &k_full[st],
+                          head * D + c * 64, k0 + kt * 128);
+      }
+    }
+  } else if (warp == 3) {
+    if (lane == 0) {
+      for (int kt = 0; kt < nk; ++kt) {
+        const int st = kt & 1;
+        tc::mbar_wait(&v_empty[st], ((kt >> 1) & 1) ^ 1);
+        tc::mbar_expect_tx(&v_full[st], Cfg::KV_TILE);
+#pragma unroll
+        for (int c = 0; c < Cfg::CH; ++c)
+          tc::tma_load_2d(sV + st * Cfg::KV_TILE + c * CHUNK, &tmKV, &v_full[st],
+                          H + head * D + c * 64, k0 + kt * 128);
       }
     }
   } else if (warp == 1) {
@@ -116,7 +128,7 @@ __global__ void __launch_bounds__(256, 1)
       tc::mbar_wait(bar_q, 0);
       auto issue_s = [&](int kt) {
         const int st = kt & 1;
-        tc::mbar_wait(&kv_full[st], (kt >> 1) & 1);
+        tc::mbar_wait(&k_full[st], (kt >> 1) & 1);
         tc::fence_after();
         const uint32_t qa = tc::smem_u32(sQ), kb = tc::smem_u32(sK + st * Cfg::KV_TILE);
 #pragma unroll
@@ -126,6 +138,7 @@ __global__ void __launch_bounds__(256, 1)
                        idesc_s, ks > 0);
         }
         tc::mma_commit(&bar_s[st]);
+        tc::mma_commit(&k_empty[st]);
       };
       issue_s(0);
       for (int kt = 0; kt < nk; ++kt) {
@@ -135,6 +148,8 @@ __global__ void __launch_bounds__(256, 1)
         tc::mbar_wait(&bar_p[pb], (kt >> 1) & 1);
         tc::fence_after();
         const int st = kt & 1;
+        tc::mbar_wait(&v_full[st], (kt >> 1) & 1);
+        tc::fence_after();
         const uint32_t pa = tc::smem_u32(sP + pb * Cfg::P_BYTES);
         const uint32_t vb = tc::smem_u32(sV + st * Cfg::KV_TILE);
 #pragma unroll
@@ -143,7 +158,7 @@ __global__ void __launch_bounds__(256, 1)
                        tc::sdesc_mn_sw128(vb + ks * 2048, CHUNK), idesc_o, (kt | ks) != 0);
         }
         tc::mma_commit(&bar_o[pb]);
-        tc::mma_commit(&kv_empty[st]);
+        tc::mma_commit(&v_empty[st]);
       }
     }
   } else if (warp >= 4) {

@@ -183,6 +183,80 @@ __global__ void __launch_bounds__(128) ln_mod_kernel(const T* __restrict__ x,
   }
 }
 
+// Wide rows (H >= 1024 bf16): one 128-thread CTA per row, VPT 16-B vectors per thread.  Every
+// global load of the row -- x and the request's shift / scale vectors -- is issued up front, so a
+// row costs one memory round trip plus two block reductions (mean, then centred variance).
+template <typename T, int VPT>
+__global__ void __launch_bounds__(128) ln_mod_row_kernel(const T* __restrict__ x,
+                                                         const int32_t* __restrict__ rows, int H,
+                                                         T* __restrict__ out,
+                                                         const int32_t* __restrict__ cu, int n_req,
+                                                         const T* __restrict__ mod, int shift_off) {
+  constexpr int NV = Vec16<T>::N;
+  __shared__ float red[4];
+  const int row = blockIdx.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int nvec = H / NV;
+  const int src_row = rows ? __ldg(rows + row) : row;
+  const uint4* xr = reinterpret_cast<const uint4*>(x + (size_t)src_row * H);
+  const uint4* sh = nullptr;
+  const uint4* sc = nullptr;
+  if (mod) {
+    const T* base = mod + (size_t)find_req(cu, n_req, row) * 6 * H + shift_off;
+    sh = reinterpret_cast<const uint4*>(base);
+    sc = reinterpret_cast<const uint4*>(base + H);
+  }
+  uint4 xv[VPT], shv[VPT], scv[VPT];
+#pragma unroll
+  for (int k = 0; k < VPT; ++k) {
+    const int vi = tid + 128 * k;
+    const bool ok = vi < nvec;
+    xv[k] = ok ? __ldg(xr + vi) : make_uint4(0, 0, 0, 0);
+    shv[k] = (ok && mod) ? __ldg(sh + vi) : make_uint4(0, 0, 0, 0);
+    scv[k] = (ok && mod) ? __ldg(sc + vi) : make_uint4(0, 0, 0, 0);
+  }
+  float v[VPT][NV];
+  float sum = 0.f;
+#pragma unroll
+  for (int k = 0; k < VPT; ++k) {
+    Vec16<T>::unpack(xv[k], v[k]);
+#pragma unroll
+    for (int e = 0; e < NV; ++e) sum += v[k][e];
+  }
+  sum = warp_sum(sum);
+  if (lane == 0) red[warp] = sum;
+  __syncthreads();
+  const float mean = (red[0] + red[1] + red[2] + red[3]) / (float)H;
+  __syncthreads();
+  float sq = 0.f;
+#pragma unroll
+  for (int k = 0; k < VPT; ++k) {
+    if (tid + 128 * k < nvec) {
+#pragma unroll
+      for (int e = 0; e < NV; ++e) {
+        const float d = v[k][e] - mean;
+        sq += d * d;
+      }
+    }
+  }
+  sq = warp_sum(sq);
+  if (lane == 0) red[warp] = sq;
+  __syncthreads();
+  const float rstd = 1.0f / sqrtf((red[0] + red[1] + red[2] + red[3]) / (float)H + 1e-6f);
+  uint4* o = reinterpret_cast<uint4*>(out + (size_t)row * H);
+#pragma unroll
+  for (int k = 0; k < VPT; ++k) {
+    const int vi = tid + 128 * k;
+    if (vi < nvec) {
+      float r[NV], a[NV], b[NV];
+      Vec16<T>::unpack(shv[k], a);
+      Vec16<T>::unpack(scv[k], b);
+#pragma unroll
+      for (int e = 0; e < NV; ++e) r[e] = (v[k][e] - mean) * rstd * (1.0f + b[e]) + a[e];
+      o[vi] = Vec16<T>::pack(r);
+    }
+  }
+}
+
 template <typename T>
 static fps_status ln_mod_t(const void* x, const int32_t* rows, int n, int H, void* out,
                            const int32_t* cu, int n_req, const void* mod, int shift_off,
@@ -193,6 +267,21 @@ static fps_status ln_mod_t(const void* x, const int32_t* rows, int n, int H, voi
   auto X = reinterpret_cast<const T*>(x);
   auto O = reinterpret_cast<T*>(out);
   auto Md = reinterpret_cast<const T*>(mod);
+  const int per_thread = ceil_div(H / NV, 128);
+  if (H / NV >= 128 && per_thread <= 8) {
+    prof::begin(s);
+#define FPS_LNR_CASE(VPT)                                                                  \
+    if (per_thread <= VPT)                                                                 \
+      ln_mod_row_kernel<T, VPT><<<n, 128, 0, s>>>(X, rows, H, O, cu, n_req, Md, shift_off); \
+    else
+    FPS_LNR_CASE(1) FPS_LNR_CASE(2) FPS_LNR_CASE(3) FPS_LNR_CASE(4) FPS_LNR_CASE(6)
+    ln_mod_row_kernel<T, 8><<<n, 128, 0, s>>>(X, rows, H, O, cu, n_req, Md, shift_off);
+#undef FPS_LNR_CASE
+    prof::end(s, prof::LN, 0, 2.0 * n * H * sizeof(T));
+    count_launch();
+    FPS_LAUNCH_CHECK();
+    return FPS_OK;
+  }
 #define FPS_LN_CASE(VPT)                                                                  \
   if (per_lane <= VPT) {                                                                  \
     prof::begin(s);                                                                       \
