@@ -53,6 +53,16 @@ def log(*a):
     print(*a, file=sys.stderr, flush=True)
 
 
+def ncu_traffic(kernel):
+    """DRAM bytes per launch of `kernel` from the newest committed ncu capture (profiles/)."""
+    import glob
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_traffic.json")))
+    if not files:
+        return None
+    d = json.load(open(files[-1]))
+    return d.get(kernel, {}).get("dram_bytes_per_launch")
+
+
 def peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -74,7 +84,7 @@ class Clocks:
              "clocks_event_reasons.sw_power_cap")
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}",
-                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                          "--format=csv,noheader,nounits", "-lms", "50"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
@@ -431,7 +441,11 @@ def main():
     roofline = {"bound": "tensor", "kernel": "gemm_tcgen05 (a5/a7/a8 projections + MLP)",
                 "achieved": gemm_achieved, "peak": bf16_sust, "unit": "TFLOP/s",
                 "frac": gemm_achieved / bf16_sust, "peak_source": f"{src} bf16_tflops_sustained",
-                "traffic": None, "avg_launch_ms": gemm_avg_ms,
+                "traffic": ncu_traffic("gemm_tcgen05"),
+                "traffic_source": "dram__bytes_read.sum + dram__bytes_write.sum per launch, "
+                                  "ncu --set full capture in profiles/ (one masked block's GEMMs)",
+                "algorithmic_bytes_per_launch": by[0] / max(cnt[0], 1),
+                "avg_launch_ms": gemm_avg_ms,
                 "flops_per_launch": fl[0] / max(cnt[0], 1)}
 
     # e2e through the public call with HOST buffers: per step H2D latents, one step, D2H latents
