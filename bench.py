@@ -316,6 +316,12 @@ def main():
     if w["L_txt"] == 0:
         base_cfg["l2"] = "inputs > L2 (weights + activations streamed per step)"
 
+    metric_name = ("masked-block stack images/s (Flux-scale, 20% mask) [ms/step alongside]"
+                   if args.config == "C3" else f"masked-block stack images/s ({args.config})")
+    base_cfg["cache_tier"] = "pinned host DRAM" if args.tier == "host" else "device HBM (NEXT-1)"
+    base_cfg["h2d_method"] = ["SM zero-copy row gather", "DMA per row run"][args.copy_method]
+    base_cfg["parallelism"] = f"request-parallel x{world} (Alg. 2 routing)"
+
     if args.impl == "reference":
         if rank != 0:
             return
@@ -331,7 +337,7 @@ def main():
         cpu = {"value": ips, "unit": metric_unit, "cores": cpu_threads(), "kind": "oracle",
                "sample": f"1 mask-aware block x 1 request per step (fp64 numpy), extrapolated x"
                          f"{w['layers']} blocks x{w['batch']} requests x{w['steps']} steps"}
-        print(json.dumps({"impl": "reference", "metric": "images/s (masked-block stack)",
+        print(json.dumps({"impl": "reference", "metric": metric_name,
                           "value": ips, "unit": metric_unit, "n_gpus": world, "steps": K,
                           "warmup": W, "ms_per_step": step_ms, "higher_is_better": True,
                           "scaling": "weak", "vs_baseline": None, "dtype": "f64",
@@ -362,9 +368,9 @@ def main():
     log(f"[rank {rank}] inputs ready in {time.perf_counter() - t0:.1f}s")
     my_pool = pool[:w["batch"]]
     cm, fit = calibrate(F, w, args.mode, layers, cache, [dict()] * w["batch"], device)
-    sreqs = [sched.Request(i, p["n_active"], L) for i, p in enumerate(pool)]
-    assign, held = sched.assign_all(sreqs, world, cm.step_latency, w["batch"])
-    mine = [pool[r.rid] for r in assign[rank]]
+    my_ids, assign, held = sched.shard_requests([p["n_active"] for p in pool], L, world, rank, cm,
+                                                w["batch"])
+    mine = [pool[i] for i in my_ids]
     g = torch.Generator(device=device).manual_seed(SEED + rank)
     reqs_dev = []
     for i, p in enumerate(mine):
@@ -490,8 +496,7 @@ def main():
                    "block_s": blk}
         mean_n = statistics.mean(p["n_active"] for p in mine) if mine else 0
         out = {
-            "metric": "masked-block stack images/s (Flux-scale, 20% mask) [ms/step alongside]"
-            if args.config == "C3" else f"masked-block stack images/s ({args.config})",
+            "metric": metric_name,
             "value": value, "unit": metric_unit, "n_gpus": world, "steps": K, "warmup": W,
             "ms_per_step": step_ms, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "bf16", "data": "synthetic (random-init weights, blob masks)",

@@ -99,6 +99,15 @@ def route(req, workers, cost_fn, max_batch):
     return best
 
 
+def shard_requests(n_active, L, world, rank, cost_model, max_batch):
+    """Request-parallel sharding for `world` GPU workers (§8(e)): every rank routes the same
+    pool with Alg. 2 (deterministic, so no communication is needed) and keeps its share.
+    Returns (indices of this rank's requests, the full assignment, held requests)."""
+    reqs = [Request(i, n, L) for i, n in enumerate(n_active)]
+    workers, held = assign_all(reqs, world, cost_model.step_latency, max_batch)
+    return [r.rid for r in workers[rank]], [[r.rid for r in w] for w in workers], [r.rid for r in held]
+
+
 def assign_all(reqs, n_workers, cost_fn, max_batch):
     """Route a pool of simultaneously arriving requests one by one (arrival order)."""
     workers = [[] for _ in range(n_workers)]
