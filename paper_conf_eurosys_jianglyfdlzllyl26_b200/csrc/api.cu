@@ -283,7 +283,10 @@ int32_t fps_profile_read(double* ms, double* flops, double* bytes, int64_t* coun
   }
   return NKIND;
 }
-void fps_set_disable_tc(int32_t flags) { fps::g_disable_tc = flags; }
+void fps_set_disable_tc(int32_t flags) {
+  fps::g_disable_tc = flags & 3;
+  fps::g_gemm_force = (flags >> 2) & 3;
+}
 
 fps_status fps_build_mask_index(const uint8_t* d_masks, const int32_t* d_offsets, int32_t n_req,
                                 int32_t max_len, int32_t* d_masked_ids, int32_t* d_unmasked_ids,

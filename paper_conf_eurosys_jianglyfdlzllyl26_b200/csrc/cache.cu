@@ -30,6 +30,7 @@ struct fps_cache {
 namespace fps {
 
 constexpr int kMaxPrefetchItems = 32;
+constexpr int kPrefetchUnroll = 8;     // 16-B loads in flight per thread (PCIe latency hiding)
 
 struct PrefetchBatch {
   const uint4* src[kMaxPrefetchItems];
@@ -44,11 +45,11 @@ __global__ void __launch_bounds__(256) prefetch_kernel(const __grid_constant__ P
   const long long total = b.start[b.n_items];
   const long long stride = (long long)gridDim.x * blockDim.x;
   for (long long i0 = (long long)blockIdx.x * blockDim.x + threadIdx.x; i0 < total;
-       i0 += 4 * stride) {
-    uint4 v[4];
-    uint4* dp[4];
+       i0 += kPrefetchUnroll * stride) {
+    uint4 v[kPrefetchUnroll];
+    uint4* dp[kPrefetchUnroll];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
+    for (int u = 0; u < kPrefetchUnroll; ++u) {
       const long long i = i0 + u * stride;
       dp[u] = nullptr;
       if (i < total) {
@@ -63,7 +64,7 @@ __global__ void __launch_bounds__(256) prefetch_kernel(const __grid_constant__ P
       }
     }
 #pragma unroll
-    for (int u = 0; u < 4; ++u)
+    for (int u = 0; u < kPrefetchUnroll; ++u)
       if (dp[u]) *dp[u] = v[u];
   }
 }
@@ -221,8 +222,10 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
       b.n_items = k;
       if (acc == 0) continue;
       // few CTAs: the copy overlaps the compute stream and should not crowd it out
-      int ctas = c->d.copy_ctas > 0 ? c->d.copy_ctas : (c->d.location == 1 ? 64 : 32);
-      long long want = (acc + 1023) / 1024;
+      // measured on B200 (bench --copy-ctas sweep): 16 CTAs x 8 loads in flight sustain the
+      // PCIe link while stealing the least issue bandwidth from the compute stream
+      int ctas = c->d.copy_ctas > 0 ? c->d.copy_ctas : (c->d.location == 1 ? 64 : 16);
+      long long want = (acc + 2047) / 2048;
       if (want < ctas) ctas = (int)want;
       prof::begin(s);
       prefetch_kernel<<<ctas, 256, 0, s>>>(b);

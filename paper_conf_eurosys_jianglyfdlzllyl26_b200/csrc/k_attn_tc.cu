@@ -181,10 +181,15 @@ __global__ void __launch_bounds__(256, 1)
 #pragma unroll
         for (int i = 0; i < 128; ++i) s[i] = (i < valid) ? s[i] : -INFINITY;
       }
-      float mx = s[0];
+      // row max as 8 independent chains (latency 16 + 3 steps instead of 127)
+      float m8[8];
 #pragma unroll
-      for (int i = 1; i < 128; ++i) mx = fmaxf(mx, s[i]);
-      mx *= scale_log2;
+      for (int j = 0; j < 8; ++j) m8[j] = s[j];
+#pragma unroll
+      for (int i = 8; i < 128; ++i) m8[i & 7] = fmaxf(m8[i & 7], s[i]);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) m8[j] = fmaxf(m8[j], m8[j + 4]);
+      float mx = fmaxf(fmaxf(m8[0], m8[1]), fmaxf(m8[2], m8[3])) * scale_log2;
       const bool need = mx > m_used + 8.0f;
       const bool any_need = __any_sync(0xffffffffu, need);
       float factor = 1.0f;
@@ -193,14 +198,19 @@ __global__ void __launch_bounds__(256, 1)
         l *= factor;
         m_used = mx;
       }
-      // p = 2^(s*scale - m) while PV_{kt-1} may still be running
-      float sum = 0.f;
+      // p = 2^(s*scale - m) while PV_{kt-1} may still be running; packed FFMA2 for the
+      // scale-and-shift, packed FADD2 into 8 independent partial sums
+      const float nm = -m_used;
+      float a8[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
 #pragma unroll
-      for (int i = 0; i < 128; ++i) {
-        s[i] = tc::ex2(fmaf(s[i], scale_log2, -m_used));
-        sum += s[i];
+      for (int i = 0; i < 128; i += 2) {
+        tc::ffma2(s[i], s[i + 1], s[i], s[i + 1], scale_log2, scale_log2, nm, nm);
+        s[i] = tc::ex2(s[i]);
+        s[i + 1] = tc::ex2(s[i + 1]);
+        const int j = (i >> 1) & 3;
+        tc::fadd2(a8[2 * j], a8[2 * j + 1], a8[2 * j], a8[2 * j + 1], s[i], s[i + 1]);
       }
-      l += sum;
+      l += ((a8[0] + a8[1]) + (a8[2] + a8[3])) + ((a8[4] + a8[5]) + (a8[6] + a8[7]));
       if (any_need && kt > 0) {
         // O += P_{kt-1} V_{kt-1} must land before O is rescaled (rare: max grew by > 2^8)
         tc::mbar_wait(&bar_o[(kt - 1) & 1], ((kt - 1) >> 1) & 1);

@@ -2,20 +2,115 @@
 // C[M, N] = A[M, K] . B[N, K]^T, bf16 in, fp32 accumulate in TMEM, fused epilogue (bias, GELU,
 // gated residual, K/V row scatter into the merged key buffer -- PAPER.md L157/L161).
 //
-//   warp 0      TMA producer: A tile 128 x 64 and B tile BN x 64 per k-block, 128-B swizzle,
-//               STAGES-deep smem ring (full/empty mbarriers)
-//   warp 1      MMA issuer: one thread issues 4 x tcgen05.mma (M=128, N=BN, K=16) per k-block
-//               into one of two TMEM accumulators; tcgen05.commit frees the smem stage
-//   warp 2      TMEM allocator (2 x BN columns)
+// Two kernels share the epilogue:
+//  * gemm_tc_kernel (1 SM per tile, M=128 x BN): for small M.
+//  * gemm_tc2_kernel (CTA pair, tcgen05 cta_group::2, 256 x 256 tile): each CTA of the pair loads
+//    its 128 rows of A and its 128 rows of B; the leader's single thread issues M=256 MMAs that read
+//    both CTAs' shared memory and accumulate rows 0-127 in CTA 0's TMEM, 128-255 in CTA 1's.
+//    Per SM this halves the operand bytes per FLOP (L2 -> SM traffic) and the 6-stage ring gives
+//    a deeper prefetch than the 4-stage 1-SM ring; 256-row tiles also cut wave quantisation for
+//    the M of masked blocks (e.g. M = 1331: 72 or 216 pair tiles on 74 SM pairs).
+//
+//   warp 0      TMA producer (both CTAs), STAGES-deep 128B-swizzled smem ring
+//   warp 1      MMA issuer (one thread; leader CTA only in the pair kernel)
+//   warp 2      TMEM allocator (two accumulators: tile i's epilogue overlaps tile i+1's MMAs)
 //   warps 4-7   epilogue: tcgen05.ld 32 columns at a time (thread = output row), fused ops,
-//               16-B stores; the second accumulator lets tile i's epilogue overlap tile i+1's MMAs
+//               all global loads of a chunk issued before use, 16-B stores
 // Tiles are visited n-major so the CTAs working at the same time share one weight tile (L2).
+#include <algorithm>
+
 #include "epilogue.cuh"
 #include "kernels.h"
 #include "tc_util.cuh"
 
 namespace fps {
 
+// Grouped raster: tiles walk groups of GM m-blocks, n-major inside a group, so the CTAs running
+// at the same time touch GM row panels of A and a few column panels of B -- both stay in L2 even
+// when A is large (continuous batches: M ~ 30k rows).  For num_m <= GM this is plain n-major.
+template <int GM>
+__device__ __forceinline__ void tile_coords(int tile, int num_m, int num_n, int& m_blk, int& n_blk) {
+  const int group = tile / (GM * num_n);
+  const int first_m = group * GM;
+  const int gm = min(num_m - first_m, GM);
+  const int local = tile - group * GM * num_n;
+  m_blk = first_m + local % gm;
+  n_blk = local / gm;
+}
+
+// Epilogue of one accumulator tile for the calling thread's output row (thread = TMEM lane).
+template <int BN>
+__device__ __forceinline__ void epilogue_tile(const Epilogue& ep, int M, int N, int row,
+                                              int col_base, uint32_t taddr) {
+  const __nv_bfloat16* __restrict__ bias = reinterpret_cast<const __nv_bfloat16*>(ep.bias);
+  const __nv_bfloat16* __restrict__ resid = reinterpret_cast<const __nv_bfloat16*>(ep.resid);
+  const bool row_ok = row < M;
+  const __nv_bfloat16* gate = nullptr;
+  int orow0 = row, orow1 = row;
+  if (row_ok) {
+    if (ep.gate)
+      gate = reinterpret_cast<const __nv_bfloat16*>(ep.gate) +
+             (size_t)find_req(ep.cu, ep.n_req, row) * ep.gate_stride;
+    if (ep.map0) orow0 = __ldg(ep.map0 + row);
+    if (ep.map1) orow1 = __ldg(ep.map1 + row);
+  }
+#pragma unroll 1
+  for (int c = 0; c < BN / 32; ++c) {
+    uint32_t r[32];
+    tc::tmem_ld32(taddr + c * 32, r);
+    const int col0 = col_base + c * 32;
+    uint4 bv[4], rv[4], gv[4];
+#pragma unroll
+    for (int g = 0; g < 4; ++g) {
+      const int c0 = col0 + g * 8;
+      const bool ok = row_ok && c0 < N;
+      bv[g] = (bias && ok) ? __ldg(reinterpret_cast<const uint4*>(bias + c0)) : make_uint4(0, 0, 0, 0);
+      rv[g] = (resid && ok)
+                  ? __ldg(reinterpret_cast<const uint4*>(resid + (size_t)row * ep.ld_resid + c0))
+                  : make_uint4(0, 0, 0, 0);
+      gv[g] = (gate && ok) ? __ldg(reinterpret_cast<const uint4*>(gate + c0)) : make_uint4(0, 0, 0, 0);
+    }
+    tc::tmem_wait_ld();
+    if (!row_ok) continue;
+#pragma unroll
+    for (int g = 0; g < 4; ++g) {
+      const int c0 = col0 + g * 8;
+      if (c0 >= N) continue;
+      float v[8], t[8];
+#pragma unroll
+      for (int e = 0; e < 8; ++e) v[e] = __uint_as_float(r[g * 8 + e]);
+      if (bias) {
+        Vec16<__nv_bfloat16>::unpack(bv[g], t);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) v[e] += t[e];
+      }
+      if (ep.act == 1) {
+#pragma unroll
+        for (int e = 0; e < 8; ++e) v[e] = gelu_tanh(v[e]);
+      }
+      if (resid) {
+        float rr[8];
+        Vec16<__nv_bfloat16>::unpack(rv[g], rr);
+        if (gate) {
+          Vec16<__nv_bfloat16>::unpack(gv[g], t);
+#pragma unroll
+          for (int e = 0; e < 8; ++e) v[e] = rr[e] + t[e] * v[e];
+        } else {
+#pragma unroll
+          for (int e = 0; e < 8; ++e) v[e] = rr[e] + v[e];
+        }
+      }
+      __nv_bfloat16* dst =
+          c0 < ep.split ? reinterpret_cast<__nv_bfloat16*>(ep.out0) + (size_t)orow0 * ep.ld0 + c0
+                        : reinterpret_cast<__nv_bfloat16*>(ep.out1) + (size_t)orow1 * ep.ld1 +
+                              (c0 - ep.split);
+      *reinterpret_cast<uint4*>(dst) = Vec16<__nv_bfloat16>::pack(v);
+    }
+  }
+}
+
+// ============================================================================================
+// 1-SM kernel
 template <int BN, int STAGES>
 struct GemmCfg {
   static constexpr int BM = 128, BK = 64;
@@ -31,6 +126,7 @@ __global__ void __launch_bounds__(256, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    int M, int N, int K, Epilogue ep) {
   using Cfg = GemmCfg<BN, STAGES>;
+  constexpr int kGroupM = 16;                              // 2048 rows of A per group
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~uintptr_t(1023));
@@ -74,7 +170,8 @@ __global__ void __launch_bounds__(256, 1)
       int stage = 0;
       uint32_t phase = 0;
       for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
-        const int m_blk = tile % num_m, n_blk = tile / num_m;
+        int m_blk, n_blk;
+        tile_coords<kGroupM>(tile, num_m, num_n, m_blk, n_blk);
         for (int kb = 0; kb < num_k; ++kb) {
           tc::mbar_wait(&empty[stage], phase ^ 1);
           tc::mbar_expect_tx(&full[stage], Cfg::STAGE_BYTES);
@@ -96,8 +193,7 @@ __global__ void __launch_bounds__(256, 1)
       int it = 0;
       for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++it) {
         const int acc = it & 1;
-        const uint32_t aphase = (it >> 1) & 1;
-        tc::mbar_wait(&tempty[acc], aphase ^ 1);
+        tc::mbar_wait(&tempty[acc], ((it >> 1) & 1) ^ 1);
         tc::fence_after();
         const uint32_t d = tmem_base + acc * BN;
         for (int kb = 0; kb < num_k; ++kb) {
@@ -121,81 +217,14 @@ __global__ void __launch_bounds__(256, 1)
   } else if (warp >= 4) {
     const int q = warp & 3;
     int it = 0;
-    const __nv_bfloat16* __restrict__ bias = reinterpret_cast<const __nv_bfloat16*>(ep.bias);
-    const __nv_bfloat16* __restrict__ resid = reinterpret_cast<const __nv_bfloat16*>(ep.resid);
     for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++it) {
-      const int m_blk = tile % num_m, n_blk = tile / num_m;
+      int m_blk, n_blk;
+      tile_coords<kGroupM>(tile, num_m, num_n, m_blk, n_blk);
       const int acc = it & 1;
-      const int row = m_blk * Cfg::BM + q * 32 + lane;
-      const bool row_ok = row < M;
-      // per-row epilogue state, looked up once per tile (not per column group)
-      const __nv_bfloat16* gate = nullptr;
-      int orow0 = row, orow1 = row;
-      if (row_ok) {
-        if (ep.gate)
-          gate = reinterpret_cast<const __nv_bfloat16*>(ep.gate) +
-                 (size_t)find_req(ep.cu, ep.n_req, row) * ep.gate_stride;
-        if (ep.map0) orow0 = __ldg(ep.map0 + row);
-        if (ep.map1) orow1 = __ldg(ep.map1 + row);
-      }
       tc::mbar_wait(&tfull[acc], (it >> 1) & 1);
       tc::fence_after();
-#pragma unroll 1
-      for (int c = 0; c < BN / 32; ++c) {
-        uint32_t r[32];
-        tc::tmem_ld32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + c * 32, r);
-        // issue every global load of this 32-column chunk before using any of them
-        const int col0 = n_blk * BN + c * 32;
-        uint4 bv[4], rv[4], gv[4];
-#pragma unroll
-        for (int g = 0; g < 4; ++g) {
-          const int c0 = col0 + g * 8;
-          const bool ok = row_ok && c0 < N;
-          bv[g] = (bias && ok) ? __ldg(reinterpret_cast<const uint4*>(bias + c0)) : make_uint4(0, 0, 0, 0);
-          rv[g] = (resid && ok) ? __ldg(reinterpret_cast<const uint4*>(resid + (size_t)row * ep.ld_resid + c0))
-                                : make_uint4(0, 0, 0, 0);
-          gv[g] = (gate && ok) ? __ldg(reinterpret_cast<const uint4*>(gate + c0)) : make_uint4(0, 0, 0, 0);
-        }
-        tc::tmem_wait_ld();
-        if (row_ok) {
-#pragma unroll
-          for (int g = 0; g < 4; ++g) {
-            const int c0 = col0 + g * 8;
-            if (c0 < N) {
-              float v[8], t[8];
-#pragma unroll
-              for (int e = 0; e < 8; ++e) v[e] = __uint_as_float(r[g * 8 + e]);
-              if (bias) {
-                Vec16<__nv_bfloat16>::unpack(bv[g], t);
-#pragma unroll
-                for (int e = 0; e < 8; ++e) v[e] += t[e];
-              }
-              if (ep.act == 1) {
-#pragma unroll
-                for (int e = 0; e < 8; ++e) v[e] = gelu_tanh(v[e]);
-              }
-              if (resid) {
-                float rr[8];
-                Vec16<__nv_bfloat16>::unpack(rv[g], rr);
-                if (gate) {
-                  Vec16<__nv_bfloat16>::unpack(gv[g], t);
-#pragma unroll
-                  for (int e = 0; e < 8; ++e) v[e] = rr[e] + t[e] * v[e];
-                } else {
-#pragma unroll
-                  for (int e = 0; e < 8; ++e) v[e] = rr[e] + v[e];
-                }
-              }
-              __nv_bfloat16* dst =
-                  c0 < ep.split
-                      ? reinterpret_cast<__nv_bfloat16*>(ep.out0) + (size_t)orow0 * ep.ld0 + c0
-                      : reinterpret_cast<__nv_bfloat16*>(ep.out1) + (size_t)orow1 * ep.ld1 +
-                            (c0 - ep.split);
-              *reinterpret_cast<uint4*>(dst) = Vec16<__nv_bfloat16>::pack(v);
-            }
-          }
-        }
-      }
+      epilogue_tile<BN>(ep, M, N, m_blk * Cfg::BM + q * 32 + lane, n_blk * BN,
+                        tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN);
       tc::fence_before();
       __syncwarp();
       if (lane == 0) tc::mbar_arrive(&tempty[acc]);
@@ -208,9 +237,145 @@ __global__ void __launch_bounds__(256, 1)
   }
 }
 
+// ============================================================================================
+// CTA-pair kernel (cta_group::2): 256 x 256 tile per pair
+template <int STAGES>
+struct Gemm2Cfg {
+  static constexpr int BM = 256, BN = 256, BK = 64;        // per pair
+  static constexpr int A_BYTES = 128 * BK * 2;             // per CTA: its 128 rows of A
+  static constexpr int B_BYTES = 128 * BK * 2;             // per CTA: its 128 rows of B
+  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr int TMEM_COLS = 512;                    // 2 accumulators x 256 columns
+  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 + 256;
+};
+
+template <int STAGES>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
+    gemm_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                    int M, int N, int K, Epilogue ep) {
+  using Cfg = Gemm2Cfg<STAGES>;
+  constexpr int kGroupM = 8;                               // 2048 rows of A per group
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~uintptr_t(1023));
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + STAGES * Cfg::A_BYTES;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + STAGES * Cfg::STAGE_BYTES);
+  uint64_t* empty = full + STAGES;
+  uint64_t* tfull = empty + STAGES;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(tempty + 2);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = tc::cluster_ctarank();
+  const int pair = blockIdx.x >> 1, num_pairs = gridDim.x >> 1;
+  const int num_m = (M + Cfg::BM - 1) / Cfg::BM;
+  const int num_n = (N + Cfg::BN - 1) / Cfg::BN;
+  const int num_tiles = num_m * num_n;
+  const int num_k = K / Cfg::BK;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < STAGES; ++s) {
+      tc::mbar_init(&full[s], 1);                          // used in the leader only
+      tc::mbar_init(&empty[s], 1);                         // both: leader's MMA commit multicasts
+    }
+    for (int a = 0; a < 2; ++a) {
+      tc::mbar_init(&tfull[a], 1);                         // both: multicast commit
+      tc::mbar_init(&tempty[a], 8);                        // leader: 4 epilogue warps x 2 CTAs
+    }
+    tc::fence_mbar_init();
+  }
+  if (warp == 0 && lane == 0) {
+    tc::tma_prefetch_desc(&tmA);
+    tc::tma_prefetch_desc(&tmB);
+  }
+  if (warp == 2) tc::tmem_alloc_2sm<Cfg::TMEM_COLS>(tmem_holder);
+  tc::fence_before();
+  __syncthreads();
+  tc::cluster_sync();                                      // peer barriers initialised
+  tc::fence_after();
+  const uint32_t tmem_base = *tmem_holder;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int tile = pair; tile < num_tiles; tile += num_pairs) {
+        int m_blk, n_blk;
+        tile_coords<kGroupM>(tile, num_m, num_n, m_blk, n_blk);
+        const int arow = m_blk * Cfg::BM + rank * 128, brow = n_blk * Cfg::BN + rank * 128;
+        for (int kb = 0; kb < num_k; ++kb) {
+          tc::mbar_wait(&empty[stage], phase ^ 1);
+          if (rank == 0) tc::mbar_expect_tx(&full[stage], 2 * Cfg::STAGE_BYTES);
+          tc::tma_load_2d_2sm(sA + stage * Cfg::A_BYTES, &tmA, &full[stage], kb * Cfg::BK, arow);
+          tc::tma_load_2d_2sm(sB + stage * Cfg::B_BYTES, &tmB, &full[stage], kb * Cfg::BK, brow);
+          if (++stage == STAGES) {
+            stage = 0;
+            phase ^= 1;
+          }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && rank == 0) {
+      constexpr uint32_t idesc = tc::idesc_bf16(256, 256);
+      int stage = 0;
+      uint32_t phase = 0;
+      int it = 0;
+      for (int tile = pair; tile < num_tiles; tile += num_pairs, ++it) {
+        const int acc = it & 1;
+        tc::mbar_wait(&tempty[acc], ((it >> 1) & 1) ^ 1);
+        tc::fence_after();
+        const uint32_t d = tmem_base + acc * 256;
+        for (int kb = 0; kb < num_k; ++kb) {
+          tc::mbar_wait(&full[stage], phase);
+          tc::fence_after();
+          const uint32_t a0 = tc::smem_u32(sA + stage * Cfg::A_BYTES);
+          const uint32_t b0 = tc::smem_u32(sB + stage * Cfg::B_BYTES);
+#pragma unroll
+          for (int k = 0; k < Cfg::BK / 16; ++k)
+            tc::mma_bf16_2sm(d, tc::sdesc_k_sw128(a0 + k * 32), tc::sdesc_k_sw128(b0 + k * 32),
+                             idesc, (kb | k) != 0);
+          tc::mma_commit_2sm(&empty[stage]);
+          if (++stage == STAGES) {
+            stage = 0;
+            phase ^= 1;
+          }
+        }
+        tc::mma_commit_2sm(&tfull[acc]);
+      }
+    }
+  } else if (warp >= 4) {
+    const int q = warp & 3;
+    const uint32_t tempty_leader = tc::mapa(tc::smem_u32(tempty), 0);
+    int it = 0;
+    for (int tile = pair; tile < num_tiles; tile += num_pairs, ++it) {
+      int m_blk, n_blk;
+      tile_coords<kGroupM>(tile, num_m, num_n, m_blk, n_blk);
+      const int acc = it & 1;
+      tc::mbar_wait(&tfull[acc], (it >> 1) & 1);
+      tc::fence_after();
+      epilogue_tile<256>(ep, M, N, m_blk * Cfg::BM + rank * 128 + q * 32 + lane, n_blk * Cfg::BN,
+                         tmem_base + ((uint32_t)(q * 32) << 16) + acc * 256);
+      tc::fence_before();
+      __syncwarp();
+      if (lane == 0) tc::mbar_arrive_cluster(tempty_leader + acc * 8);
+    }
+  }
+  __syncthreads();
+  tc::cluster_sync();                                      // both CTAs done with TMEM / barriers
+  if (warp == 2) {
+    tc::fence_after();
+    tc::tmem_dealloc_2sm<Cfg::TMEM_COLS>(tmem_base);
+  }
+}
+
+// ============================================================================================
 bool gemm_tc_supported(int dtype, int M, int N, int K) {
   return dtype == FPS_BF16 && M > 0 && K >= 64 && K % 64 == 0 && N % 8 == 0;
 }
+
+int g_gemm_force = 0;   // tests: 1 = force the 1-SM kernel, 2 = force the CTA-pair kernel
 
 template <int BN, int STAGES>
 static fps_status launch_cfg(const void* A, const void* B, int M, int N, int K,
@@ -234,14 +399,47 @@ static fps_status launch_cfg(const void* A, const void* B, int M, int N, int K,
   return FPS_OK;
 }
 
+template <int STAGES>
+static fps_status launch_pair(const void* A, const void* B, int M, int N, int K,
+                              const Epilogue& ep, cudaStream_t s) {
+  using Cfg = Gemm2Cfg<STAGES>;
+  CUtensorMap ta, tb;
+  if (!make_tmap_2d_bf16(&ta, A, M, K, (uint64_t)K * 2, Cfg::BK, 128) ||
+      !make_tmap_2d_bf16(&tb, B, N, K, (uint64_t)K * 2, Cfg::BK, 128))
+    return fail(FPS_ECUDA, "gemm_tc2: cuTensorMapEncodeTiled failed (M=%d N=%d K=%d)", M, N, K);
+  static bool attr_set = false;
+  if (!attr_set) {
+    FPS_CUDA_TRY(cudaFuncSetAttribute(gemm_tc2_kernel<STAGES>,
+                                      cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
+    attr_set = true;
+  }
+  const int tiles = ceil_div(M, Cfg::BM) * ceil_div(N, Cfg::BN);
+  const int pairs = tiles < kNumSMs / 2 ? tiles : kNumSMs / 2;
+  gemm_tc2_kernel<STAGES><<<2 * pairs, 256, Cfg::SMEM, s>>>(ta, tb, M, N, K, ep);
+  count_launch();
+  FPS_LAUNCH_CHECK();
+  return FPS_OK;
+}
+
 fps_status launch_gemm_tc(const void* A, const void* B, int M, int N, int K, const Epilogue& ep,
                           cudaStream_t s) {
   if (!aligned16(A) || !aligned16(B)) return fail(FPS_EINVAL, "gemm_tc: unaligned operand");
-  // pick the N tile that minimises (waves x tile width); ties -> the wider tile (less L2 traffic)
-  const int m_blocks = ceil_div(M, 128);
-  const long t256 = (long)m_blocks * ceil_div(N, 256), t128 = (long)m_blocks * ceil_div(N, 128);
+  // Cost model: time ~ waves x tile work; the pair kernel's 256x256 tile does 2x the work of a
+  // 128x256 tile on two SMs, i.e. the same per-SM time per wave, but at half the operand traffic
+  // per FLOP.  Prefer it unless it needs more waves.
+  const int m1 = ceil_div(M, 128), m2 = ceil_div(M, 256);
+  const long t256 = (long)m1 * ceil_div(N, 256), t128 = (long)m1 * ceil_div(N, 128);
+  const long tp = (long)m2 * ceil_div(N, 256);
   const long c256 = ((t256 + kNumSMs - 1) / kNumSMs) * 256;
   const long c128 = ((t128 + kNumSMs - 1) / kNumSMs) * 128;
+  const long cp = ((tp + kNumSMs / 2 - 1) / (kNumSMs / 2)) * 256;
+  // Measured (tools/gemm_probe.py, B200): the pair kernel reaches 95% tensor-pipe activity at
+  // large M where the 1-SM kernel is L2-bound (1480 vs 1070 TFLOP/s at M = 29491); at one wave
+  // the extra M padding of 256-row tiles can make it lose, so then padding decides.
+  const long cmin = std::min(c256, c128);
+  const bool pair_wins = cp < cmin || (cp == cmin && (tp > kNumSMs / 2 || m2 * 256 - M < 128));
+  if (g_gemm_force == 2 || (g_gemm_force == 0 && pair_wins))
+    return launch_pair<6>(A, B, M, N, K, ep, s);
   if (c256 <= c128) return launch_cfg<256, 4>(A, B, M, N, K, ep, s);
   return launch_cfg<128, 6>(A, B, M, N, K, ep, s);
 }

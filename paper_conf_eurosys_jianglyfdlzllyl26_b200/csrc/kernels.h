@@ -41,5 +41,7 @@ bool attention_tc_supported(int dtype, int head_dim);
 // global switches (tests can force the SIMT kernels): bit0 = no tcgen05 GEMM,
 // bit1 = no tensor-core attention
 extern int g_disable_tc;
+// tests: 0 = choose, 1 = force the 1-SM tcgen05 GEMM, 2 = force the CTA-pair GEMM
+extern int g_gemm_force;
 
 }  // namespace fps

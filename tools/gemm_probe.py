@@ -1,0 +1,26 @@
+"""Time one fps_linear shape: python tools/gemm_probe.py M N K [force: 0 auto, 4 1-SM, 8 pair]."""
+import os
+import sys
+
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_eurosys_jianglyfdlzllyl26_b200 as F
+
+M, N, K = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3])
+force = int(sys.argv[4]) if len(sys.argv) > 4 else 0
+a = torch.randn(M, K, device="cuda").to(torch.bfloat16)
+w = (torch.randn(N, K, device="cuda") / K ** 0.5).to(torch.bfloat16)
+out = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
+F.fps_set_disable_tc(force)
+for _ in range(3):
+    F.linear(a, w, out=out)
+e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+torch.cuda.synchronize()
+e0.record()
+for _ in range(10):
+    F.linear(a, w, out=out)
+e1.record()
+torch.cuda.synchronize()
+ms = e0.elapsed_time(e1) / 10
+print(f"{M}x{N}x{K} force={force}: {ms:.4f} ms {2 * M * N * K / ms / 1e9:.0f} TF/s")
