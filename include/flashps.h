@@ -213,6 +213,16 @@ fps_status fps_masked_block_forward(const fps_block_weights* w, const fps_varlen
 fps_status fps_linear(int32_t dtype, const void* d_a, const void* d_w, const void* d_bias,
                       int32_t M, int32_t N, int32_t K, int32_t act, void* d_out, void* stream);
 
+/* a6 on its own (tests and per-kernel measurement): for request r and head j,
+ * d_o[i, j] = softmax(q_i K_j^T / sqrt(head_dim)) V_j over the request's merged key rows
+ * [cu_k[r], cu_k[r+1]) of d_kv ([total_k, 2H], row = K|V), for its active rows
+ * [cu_q[r], cu_q[r+1]) of d_q / d_o ([total_q, H]).  Device and host copies of both prefix-sum
+ * arrays are required (launch sizing without a device sync). */
+fps_status fps_masked_attention(int32_t dtype, const void* d_q, const void* d_kv, void* d_o,
+                                int32_t heads, int32_t head_dim, const int32_t* d_cu_q,
+                                const int32_t* d_cu_k, const int32_t* h_cu_q,
+                                const int32_t* h_cu_k, int32_t n_req, void* stream);
+
 /* Dense block (Fig. 5-Top; the uncached blocks of Fig. 9-Bottom): all L_r rows of every
  * request; b->d_q_row must be NULL and total_q == total_k.  d_kv is scratch [total_k, 2H]. */
 fps_status fps_dense_block_forward(const fps_block_weights* w, const fps_varlen_batch* b,

@@ -150,6 +150,22 @@ def dense_block_forward(w: BlockWeights, b: VarlenBatch, x, kv=None, y=None, ws=
     return y, kv
 
 
+def masked_attention(q, kv, n_active, L, heads, out=None, stream=None):
+    """a6 through fps_masked_attention: q [sum n, H], kv [sum L, 2H] (K|V rows)."""
+    H = q.shape[1]
+    cu_q = np.concatenate([[0], np.cumsum(n_active)]).astype(np.int32)
+    cu_k = np.concatenate([[0], np.cumsum(L)]).astype(np.int32)
+    d_cu_q = torch.tensor(cu_q, device=q.device)
+    d_cu_k = torch.tensor(cu_k, device=q.device)
+    out = out if out is not None else torch.empty_like(q)
+    dt = FPS_BF16 if q.dtype == torch.bfloat16 else FPS_F32
+    _lib.fps_masked_attention(dt, ptr(q), ptr(kv), ptr(out), heads, H // heads, ptr(d_cu_q),
+                              ptr(d_cu_k), cu_q.ctypes.data, cu_k.ctypes.data, len(n_active),
+                              stream_ptr(stream))
+    out._fps_keep = (d_cu_q, d_cu_k, cu_q, cu_k)          # keep the index arrays alive
+    return out
+
+
 def linear(a, w, bias=None, act=0, out=None, stream=None):
     """out = act(a w^T + bias) through fps_linear (tcgen05 GEMM for bf16)."""
     M, K = a.shape

@@ -88,6 +88,7 @@ _SIGS = [
      [C.POINTER(fps_block_weights), C.POINTER(fps_varlen_batch), vp, vp, vp, vp, vp, vp, sz, vp],
      True),
     ("fps_linear", C.c_int, [i32, vp, vp, vp, i32, i32, i32, i32, vp, vp], True),
+    ("fps_masked_attention", C.c_int, [i32, vp, vp, vp, i32, i32, vp, vp, vp, vp, i32, vp], True),
     ("fps_dense_block_forward", C.c_int,
      [C.POINTER(fps_block_weights), C.POINTER(fps_varlen_batch), vp, vp, vp, vp, sz, vp], True),
     ("fps_plan_pipeline", C.c_int, [P_dbl, P_dbl, P_dbl, i32, i32, dbl, P_u8, P_dbl], True),

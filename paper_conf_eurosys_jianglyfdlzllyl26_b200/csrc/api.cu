@@ -364,6 +364,24 @@ fps_status fps_linear(int32_t dtype, const void* d_a, const void* d_w, const voi
   return launch_gemm(dtype, d_a, d_w, M, N, K, ep, as_stream(stream));
 }
 
+fps_status fps_masked_attention(int32_t dtype, const void* d_q, const void* d_kv, void* d_o,
+                                int32_t heads, int32_t head_dim, const int32_t* d_cu_q,
+                                const int32_t* d_cu_k, const int32_t* h_cu_q,
+                                const int32_t* h_cu_k, int32_t n_req, void* stream) {
+  FPS_CHECK_ARG(dtype == FPS_BF16 || dtype == FPS_F32, "dtype %d", dtype);
+  FPS_CHECK_ARG(heads > 0 && head_dim > 0 && n_req >= 0, "bad sizes");
+  if (n_req == 0) return FPS_OK;
+  FPS_CHECK_ARG(d_q && d_kv && d_o && d_cu_q && d_cu_k && h_cu_q && h_cu_k, "NULL pointer");
+  const int total_q = h_cu_q[n_req];
+  int max_q = 0, max_k = 0;
+  for (int r = 0; r < n_req; ++r) {
+    max_q = std::max(max_q, h_cu_q[r + 1] - h_cu_q[r]);
+    max_k = std::max(max_k, h_cu_k[r + 1] - h_cu_k[r]);
+  }
+  return launch_attention(dtype, d_q, d_kv, d_o, heads, head_dim, d_cu_q, d_cu_k, h_cu_q, h_cu_k,
+                          n_req, total_q, max_q, max_k, as_stream(stream));
+}
+
 fps_status fps_dense_block_forward(const fps_block_weights* w, const fps_varlen_batch* b,
                                    const void* d_x, void* d_y, void* d_kv, void* d_ws,
                                    size_t ws_bytes, void* stream) {

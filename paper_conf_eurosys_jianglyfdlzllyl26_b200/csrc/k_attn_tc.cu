@@ -205,8 +205,12 @@ __global__ void __launch_bounds__(256, 1)
 #pragma unroll
       for (int i = 0; i < 128; i += 2) {
         tc::ffma2(s[i], s[i + 1], s[i], s[i + 1], scale_log2, scale_log2, nm, nm);
-        s[i] = tc::ex2(s[i]);
-        s[i + 1] = tc::ex2(s[i + 1]);
+        if (((i >> 3) & 3) == 3) {                         // 1/4 of the exponentials on the FMA pipe
+          tc::ex2_poly2(s[i], s[i + 1]);
+        } else {                                           // 3/4 on the MUFU unit
+          s[i] = tc::ex2(s[i]);
+          s[i + 1] = tc::ex2(s[i + 1]);
+        }
         const int j = (i >> 1) & 3;
         tc::fadd2(a8[2 * j], a8[2 * j + 1], a8[2 * j], a8[2 * j + 1], s[i], s[i + 1]);
       }

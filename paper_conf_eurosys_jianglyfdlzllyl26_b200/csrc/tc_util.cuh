@@ -246,6 +246,27 @@ __device__ __forceinline__ void fadd2(float& d0, float& d1, float a0, float a1, 
       : "=f"(d0), "=f"(d1)
       : "f"(a0), "f"(a1), "f"(b0), "f"(b1));
 }
+// 2^x for a pair on the FMA pipe (offloads the MUFU unit, FA4-style): x = n + f, n = round(x),
+// f in [-0.5, 0.5], 2^f by a degree-5 polynomial (Taylor in ln 2, rel. error < 3e-6), then n is
+// added to the exponent field.  x is clamped to >= -126 (results below 2^-126 flush towards 0;
+// they are far below bf16 P resolution relative to the row max, which is >= 1).
+__device__ __forceinline__ void ex2_poly2(float& x0, float& x1) {
+  const float magic = 12582912.0f;                          // 1.5 * 2^23: round-to-nearest trick
+  x0 = fmaxf(x0, -126.0f);
+  x1 = fmaxf(x1, -126.0f);
+  float r0, r1, n0, n1, f0, f1;
+  fadd2(r0, r1, x0, x1, magic, magic);
+  fadd2(n0, n1, r0, r1, -magic, -magic);
+  fadd2(f0, f1, x0, x1, -n0, -n1);
+  float p0 = 1.3333558e-3f, p1 = 1.3333558e-3f;
+  ffma2(p0, p1, p0, p1, f0, f1, 9.6181291e-3f, 9.6181291e-3f);
+  ffma2(p0, p1, p0, p1, f0, f1, 5.5504109e-2f, 5.5504109e-2f);
+  ffma2(p0, p1, p0, p1, f0, f1, 2.4022651e-1f, 2.4022651e-1f);
+  ffma2(p0, p1, p0, p1, f0, f1, 6.9314718e-1f, 6.9314718e-1f);
+  ffma2(p0, p1, p0, p1, f0, f1, 1.0f, 1.0f);
+  x0 = __int_as_float(__float_as_int(p0) + (__float_as_int(r0) << 23));
+  x1 = __int_as_float(__float_as_int(p1) + (__float_as_int(r1) << 23));
+}
 __device__ __forceinline__ float ex2(float x) {
   float y;
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
