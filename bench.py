@@ -373,6 +373,8 @@ def main():
     torch.cuda.set_device(local)
     device = torch.device("cuda", local)
     F.require_gpu()
+    if os.environ.get("FPS_KERNEL_FLAGS"):            # experiments: force kernel variants
+        F.fps_set_disable_tc(int(os.environ["FPS_KERNEL_FLAGS"]))
     if world > 1:
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=device)

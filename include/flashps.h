@@ -50,7 +50,8 @@ int32_t fps_abi_version(void);
 int32_t fps_device_ok(void);
 /* Test / bench hooks: number of kernels this thread has launched through the library so far;
  * force the SIMT kernels (bit0: GEMMs, bit1: attention) instead of the tensor-core ones;
- * bits 2-3 = 1 force the 1-SM tcgen05 GEMM, = 2 force the CTA-pair (cta_group::2) GEMM. */
+ * bits 2-3 = 1 force the 1-SM tcgen05 GEMM, = 2 force the CTA-pair (cta_group::2) GEMM;
+ * bits 4-5 = 1 force the one-query-tile attention kernel, = 2 the two-tile (ping-pong) one. */
 int64_t fps_launch_count(void);
 void fps_set_disable_tc(int32_t flags);
 /* Per-kernel-class timing for the bench: when enabled (this also clears old records) every
@@ -110,7 +111,9 @@ typedef struct {
                             moved are identical, contents alias)                            */
   int32_t copy_method;   /* 0 = SM zero-copy row gather over mapped pinned memory (default);
                             1 = copy-engine DMA of coalesced row runs                        */
-  int32_t copy_ctas;     /* CTAs used by method 0 (0 = default: 16 host, 64 device)         */
+  int32_t copy_ctas;     /* CTAs used by method 0 (0 = default: 16 for the host link -- enough
+                            for PCIe, few enough not to crowd out the compute stream -- and 64
+                            for the HBM tier)                                               */
   int32_t location;      /* 0 = pinned host DRAM (L203, streamed over PCIe);
                             1 = device HBM: the template tier one level above host DRAM
                             (the paper's "ideal" no-load case of Fig. 4-Left,

@@ -286,6 +286,7 @@ int32_t fps_profile_read(double* ms, double* flops, double* bytes, int64_t* coun
 void fps_set_disable_tc(int32_t flags) {
   fps::g_disable_tc = flags & 3;
   fps::g_gemm_force = (flags >> 2) & 3;
+  fps::g_attn_force = (flags >> 4) & 3;
 }
 
 fps_status fps_build_mask_index(const uint8_t* d_masks, const int32_t* d_offsets, int32_t n_req,

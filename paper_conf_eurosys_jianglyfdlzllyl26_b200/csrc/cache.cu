@@ -224,6 +224,8 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
       // few CTAs: the copy overlaps the compute stream and should not crowd it out
       // measured on B200 (bench --copy-ctas sweep): 16 CTAs x 8 loads in flight sustain the
       // PCIe link while stealing the least issue bandwidth from the compute stream
+      // HBM tier: 64 CTAs keep the HBM row gather (~0.1 ms per Flux block) well under the
+      // compute of a block; 16 were measured too slow (0.35 ms, on the critical path)
       int ctas = c->d.copy_ctas > 0 ? c->d.copy_ctas : (c->d.location == 1 ? 64 : 16);
       long long want = (acc + 2047) / 2048;
       if (want < ctas) ctas = (int)want;

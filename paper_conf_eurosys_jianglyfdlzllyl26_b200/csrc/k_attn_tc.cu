@@ -281,6 +281,322 @@ __global__ void __launch_bounds__(256, 1)
   }
 }
 
+// ============================================================================================
+// Two query tiles per CTA (A = rows q0..q0+127, B = the next 128), FA4-style ping-pong: the
+// tensor core alternates between the tiles (S_A, S_B, PV_A, S_A', PV_B, S_B', ...) while two
+// softmax warpgroups (warps 4-7 for A, 8-11 for B) work on the other tile, so MUFU/issue time of
+// one warpgroup hides behind MMAs of the other.  Every K/V tile feeds four MMAs (half the smem
+// traffic per FLOP), and a CTA covers 256 query rows (e.g. 6 x 24 = 144 CTAs for n = 1331: one
+// wave).  TMEM: S_A [0,128) S_B [128,256) O_A [256,256+D) O_B [384,384+D); one shared smem P tile
+// is written alternately by the two warpgroups.  S rows are read from TMEM in two 64-column
+// halves (max pass, then exp pass) to stay within 168 registers at 384 threads.
+template <int D>
+struct Attn2Cfg {
+  static constexpr int CH = D / 64;
+  static constexpr int Q_BYTES = 128 * D * 2;              // one query tile
+  static constexpr int KV_TILE = 128 * D * 2;
+  static constexpr int P_BYTES = 128 * 128 * 2;
+  static constexpr int SMEM = 2 * Q_BYTES + 4 * KV_TILE + P_BYTES + 1024 + 256;
+  static constexpr int TMEM_COLS = 512;
+};
+
+template <int D>
+__global__ void __launch_bounds__(384, 1)
+    attn_tc2_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmKV,
+                    __nv_bfloat16* __restrict__ O, const int32_t* __restrict__ cu_q,
+                    const int32_t* __restrict__ cu_k, int n_req, int heads, float scale_log2) {
+  using Cfg = Attn2Cfg<D>;
+  constexpr int CHUNK = 128 * 128;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~uintptr_t(1023));
+  uint8_t* sQ = smem;                                       // [2 tiles][CH chunks]
+  uint8_t* sK = sQ + 2 * Cfg::Q_BYTES;                      // [2 stages][CH chunks]
+  uint8_t* sV = sK + 2 * Cfg::KV_TILE;
+  uint8_t* sP = sV + 2 * Cfg::KV_TILE;                      // [2 chunks of 64 keys]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sP + Cfg::P_BYTES);
+  uint64_t* bar_q = bars;
+  uint64_t* k_full = bars + 1;
+  uint64_t* k_empty = bars + 3;
+  uint64_t* v_full = bars + 5;
+  uint64_t* v_empty = bars + 7;
+  uint64_t* bar_s = bars + 9;                               // [tile]
+  uint64_t* bar_p = bars + 11;                              // [tile]
+  uint64_t* bar_o = bars + 13;                              // [tile]
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + 15);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int head = blockIdx.y;
+  const int H = heads * D;
+  int r = 0, qp = blockIdx.x, ntile = 0;
+  for (; r < n_req; ++r) {
+    ntile = (__ldg(cu_q + r + 1) - __ldg(cu_q + r) + 127) >> 7;
+    const int np = (ntile + 1) >> 1;
+    if (qp < np) break;
+    qp -= np;
+  }
+  const bool hasB = 2 * qp + 1 < ntile;
+  const int q_end = __ldg(cu_q + r + 1);
+  const int q0 = __ldg(cu_q + r) + qp * 256;
+  const int k0 = __ldg(cu_k + r);
+  const int Lr = __ldg(cu_k + r + 1) - k0;
+  const int nk = (Lr + 127) >> 7;
+
+  if (threadIdx.x == 0) {
+    tc::mbar_init(bar_q, 1);
+    for (int s = 0; s < 2; ++s) {
+      tc::mbar_init(&k_full[s], 1);
+      tc::mbar_init(&k_empty[s], 1);
+      tc::mbar_init(&v_full[s], 1);
+      tc::mbar_init(&v_empty[s], 1);
+      tc::mbar_init(&bar_s[s], 1);
+      tc::mbar_init(&bar_p[s], 4);
+      tc::mbar_init(&bar_o[s], 1);
+    }
+    tc::fence_mbar_init();
+  }
+  if (warp == 0 && lane == 0) {
+    tc::tma_prefetch_desc(&tmQ);
+    tc::tma_prefetch_desc(&tmKV);
+  }
+  if (warp == 2) tc::tmem_alloc<Cfg::TMEM_COLS>(tmem_holder);
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tmem = *tmem_holder;
+
+  if (warp == 0) {
+    if (lane == 0 && nk > 0) {
+      tc::mbar_expect_tx(bar_q, (hasB ? 2 : 1) * Cfg::Q_BYTES);
+      for (int t = 0; t < (hasB ? 2 : 1); ++t)
+#pragma unroll
+        for (int c = 0; c < Cfg::CH; ++c)
+          tc::tma_load_2d(sQ + t * Cfg::Q_BYTES + c * CHUNK, &tmQ, bar_q, head * D + c * 64,
+                          q0 + t * 128);
+      for (int kt = 0; kt < nk; ++kt) {
+        const int st = kt & 1;
+        tc::mbar_wait(&k_empty[st], ((kt >> 1) & 1) ^ 1);
+        tc::mbar_expect_tx(&k_full[st], Cfg::KV_TILE);
+#pragma unroll
+        for (int c = 0; c < Cfg::CH; ++c)
+          tc::tma_load_2d(sK + st * Cfg::KV_TILE + c * CHUNK, &tmKV, &k_full[st],
+                          head * D + c * 64, k0 + kt * 128);
+      }
+    }
+  } else if (warp == 3) {
+    if (lane == 0) {
+      for (int kt = 0; kt < nk; ++kt) {
+        const int st = kt & 1;
+        tc::mbar_wait(&v_empty[st], ((kt >> 1) & 1) ^ 1);
+        tc::mbar_expect_tx(&v_full[st], Cfg::KV_TILE);
+#pragma unroll
+        for (int c = 0; c < Cfg::CH; ++c)
+          tc::tma_load_2d(sV + st * Cfg::KV_TILE + c * CHUNK, &tmKV, &v_full[st],
+                          H + head * D + c * 64, k0 + kt * 128);
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && nk > 0) {
+      constexpr uint32_t idesc_s = tc::idesc_bf16(128, 128);
+      constexpr uint32_t idesc_o = tc::idesc_bf16(128, D, /*b_mn_major=*/true);
+      tc::mbar_wait(bar_q, 0);
+      auto issue_s = [&](int t, int kt) {           // S_t = Q_t K_kt^T  (K stage must be full)
+        const uint32_t qa = tc::smem_u32(sQ + t * Cfg::Q_BYTES);
+        const uint32_t kb = tc::smem_u32(sK + (kt & 1) * Cfg::KV_TILE);
+#pragma unroll
+        for (int ks = 0; ks < D / 16; ++ks) {
+          const uint32_t off = (ks >> 2) * CHUNK + (ks & 3) * 32;
+          tc::mma_bf16(tmem + t * 128, tc::sdesc_k_sw128(qa + off), tc::sdesc_k_sw128(kb + off),
+                       idesc_s, ks > 0);
+        }
+        tc::mma_commit(&bar_s[t]);
+      };
+      auto issue_pv = [&](int t, int kt) {          // O_t += P V_kt  (P and V stage ready)
+        const uint32_t pa = tc::smem_u32(sP), vb = tc::smem_u32(sV + (kt & 1) * Cfg::KV_TILE);
+#pragma unroll
+        for (int ks = 0; ks < 8; ++ks)
+          tc::mma_bf16(tmem + 256 + t * 128,
+                       tc::sdesc_k_sw128(pa + (ks >> 2) * CHUNK + (ks & 3) * 32),
+                       tc::sdesc_mn_sw128(vb + ks * 2048, CHUNK), idesc_o, (kt | ks) != 0);
+        tc::mma_commit(&bar_o[t]);
+      };
+      tc::mbar_wait(&k_full[0], 0);
+      tc::fence_after();
+      issue_s(0, 0);
+      if (hasB) issue_s(1, 0);
+      tc::mma_commit(&k_empty[0]);
+      for (int kt = 0; kt < nk; ++kt) {
+        const bool more = kt + 1 < nk;
+        tc::mbar_wait(&v_full[kt & 1], (kt >> 1) & 1);
+        tc::mbar_wait(&bar_p[0], kt & 1);
+        tc::fence_after();
+        issue_pv(0, kt);
+        if (!hasB) tc::mma_commit(&v_empty[kt & 1]);
+        if (more) {
+          tc::mbar_wait(&k_full[(kt + 1) & 1], ((kt + 1) >> 1) & 1);
+          tc::fence_after();
+          issue_s(0, kt + 1);
+          if (!hasB) tc::mma_commit(&k_empty[(kt + 1) & 1]);
+        }
+        if (hasB) {
+          tc::mbar_wait(&bar_p[1], kt & 1);
+          tc::fence_after();
+          issue_pv(1, kt);
+          tc::mma_commit(&v_empty[kt & 1]);
+          if (more) {
+            issue_s(1, kt + 1);
+            tc::mma_commit(&k_empty[(kt + 1) & 1]);
+          }
+        }
+      }
+    }
+  } else if (warp >= 4) {
+    const int t = (warp >= 8) ? 1 : 0;                     // query tile of this warpgroup
+    if (t == 1 && !hasB) goto done;
+    {
+      const int q = warp & 3;
+      const int row = q * 32 + lane;
+      const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+      const uint32_t tS = tmem + t * 128, tO = tmem + 256 + t * 128;
+      float m_used = -INFINITY, l = 0.f;
+      const int sw = row & 7;
+      uint8_t* prow = sP + row * 128;
+      for (int kt = 0; kt < nk; ++kt) {
+        tc::mbar_wait(&bar_s[t], kt & 1);
+        tc::fence_after();
+        const int valid = Lr - kt * 128;
+        // pass 1: row max over the two 64-column halves
+        float mx = -INFINITY;
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          float s[64];
+          tc::tmem_ld32(tS + lane_off + h * 64, reinterpret_cast<uint32_t*>(s));
+          tc::tmem_ld32(tS + lane_off + h * 64 + 32, reinterpret_cast<uint32_t*>(s + 32));
+          tc::tmem_wait_ld();
+          if (valid < (h + 1) * 64) {                     // only the request's last key tile
+#pragma unroll
+            for (int i = 0; i < 64; ++i) s[i] = (h * 64 + i < valid) ? s[i] : -INFINITY;
+          }
+          float m8[8];
+#pragma unroll
+          for (int j = 0; j < 8; ++j) m8[j] = s[j];
+#pragma unroll
+          for (int i = 8; i < 64; ++i) m8[i & 7] = fmaxf(m8[i & 7], s[i]);
+#pragma unroll
+          for (int j = 0; j < 4; ++j) m8[j] = fmaxf(m8[j], m8[j + 4]);
+          mx = fmaxf(mx, fmaxf(fmaxf(m8[0], m8[1]), fmaxf(m8[2], m8[3])));
+        }
+        mx *= scale_log2;
+        const bool need = mx > m_used + 8.0f;
+        const bool any_need = __any_sync(0xffffffffu, need);
+        float factor = 1.0f;
+        if (need) {
+          factor = tc::ex2(m_used - mx);
+          l *= factor;
+          m_used = mx;
+        }
+        if (any_need && kt > 0) {                           // rescale O_t after PV_t(kt-1)
+          tc::mbar_wait(&bar_o[t], (kt - 1) & 1);
+          tc::fence_after();
+#pragma unroll 1
+          for (int c = 0; c < D / 32; ++c) {
+            uint32_t o[32];
+            tc::tmem_ld32(tO + lane_off + c * 32, o);
+            tc::tmem_wait_ld();
+#pragma unroll
+            for (int e = 0; e < 32; ++e) o[e] = __float_as_uint(__uint_as_float(o[e]) * factor);
+            tc::tmem_st32(tO + lane_off + c * 32, o);
+          }
+          tc::tmem_wait_st();
+        }
+        // pass 2: exponentials per half, then P into the shared P tile once it is free
+        const float nm = -m_used;
+        float a8[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          float s[64];
+          tc::tmem_ld32(tS + lane_off + h * 64, reinterpret_cast<uint32_t*>(s));
+          tc::tmem_ld32(tS + lane_off + h * 64 + 32, reinterpret_cast<uint32_t*>(s + 32));
+          tc::tmem_wait_ld();
+          if (valid < (h + 1) * 64) {
+#pragma unroll
+            for (int i = 0; i < 64; ++i) s[i] = (h * 64 + i < valid) ? s[i] : -INFINITY;
+          }
+#pragma unroll
+          for (int i = 0; i < 64; i += 2) {
+            tc::ffma2(s[i], s[i + 1], s[i], s[i + 1], scale_log2, scale_log2, nm, nm);
+            if (((i >> 3) & 3) == 3) {
+              tc::ex2_poly2(s[i], s[i + 1]);
+            } else {
+              s[i] = tc::ex2(s[i]);
+              s[i + 1] = tc::ex2(s[i + 1]);
+            }
+            const int j = (i >> 1) & 3;
+            tc::fadd2(a8[2 * j], a8[2 * j + 1], a8[2 * j], a8[2 * j + 1], s[i], s[i + 1]);
+          }
+          if (h == 0) {
+            // the P tile is free once the other tile's previous PV (or, for tile B, this
+            // tile-pair's PV_A) has completed; S_t is fully read after the second half's load
+            if (t == 0) {
+              if (kt > 0) {
+                if (hasB) tc::mbar_wait(&bar_o[1], (kt - 1) & 1);
+                else tc::mbar_wait(&bar_o[0], (kt - 1) & 1);
+              }
+            } else {
+              tc::mbar_wait(&bar_o[0], kt & 1);
+            }
+            tc::fence_after();
+          }
+#pragma unroll
+          for (int u = 0; u < 8; ++u) {
+            const uint4 v = make_uint4(pack_bf16x2(s[u * 8 + 0], s[u * 8 + 1]),
+                                       pack_bf16x2(s[u * 8 + 2], s[u * 8 + 3]),
+                                       pack_bf16x2(s[u * 8 + 4], s[u * 8 + 5]),
+                                       pack_bf16x2(s[u * 8 + 6], s[u * 8 + 7]));
+            *reinterpret_cast<uint4*>(prow + h * CHUNK + ((u ^ sw) << 4)) = v;
+          }
+        }
+        l += ((a8[0] + a8[1]) + (a8[2] + a8[3])) + ((a8[4] + a8[5]) + (a8[6] + a8[7]));
+        tc::fence_proxy_async_smem();
+        tc::fence_before();
+        __syncwarp();
+        if (lane == 0) tc::mbar_arrive(&bar_p[t]);
+      }
+      if (nk > 0) {
+        tc::mbar_wait(&bar_o[t], (nk - 1) & 1);
+        tc::fence_after();
+      }
+      const float inv = (l > 0.f) ? 1.0f / l : 0.f;
+      const int grow = q0 + t * 128 + row;
+      __nv_bfloat16* orow = O + (size_t)grow * H + head * D;
+#pragma unroll 1
+      for (int c = 0; c < D / 32; ++c) {
+        uint32_t o[32];
+        tc::tmem_ld32(tO + lane_off + c * 32, o);
+        tc::tmem_wait_ld();
+        if (grow < q_end) {
+#pragma unroll
+          for (int g = 0; g < 4; ++g) {
+            float f[8];
+#pragma unroll
+            for (int e = 0; e < 8; ++e) f[e] = __uint_as_float(o[g * 8 + e]) * inv;
+            *reinterpret_cast<uint4*>(orow + c * 32 + g * 8) = Vec16<__nv_bfloat16>::pack(f);
+          }
+        }
+      }
+    }
+  done:;
+  }
+  tc::fence_before();
+  __syncthreads();
+  if (warp == 2) {
+    tc::fence_after();
+    tc::tmem_dealloc<Cfg::TMEM_COLS>(tmem);
+  }
+}
+
+int g_attn_force = 0;   // tests: 1 = force the one-tile kernel
+
 bool attention_tc_supported(int dtype, int head_dim) {
   return dtype == FPS_BF16 && (head_dim == 64 || head_dim == 128);
 }
@@ -315,12 +631,50 @@ static fps_status launch_d(const void* q, const void* kv, void* o, int heads,
   return FPS_OK;
 }
 
+template <int D>
+static fps_status launch_d2(const void* q, const void* kv, void* o, int heads,
+                            const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
+                            const int32_t* h_cu_k, int n_req, cudaStream_t s) {
+  using Cfg = Attn2Cfg<D>;
+  const int H = heads * D;
+  int pairs = 0;
+  for (int r = 0; r < n_req; ++r) pairs += ((h_cu_q[r + 1] - h_cu_q[r] + 127) / 128 + 1) / 2;
+  if (pairs == 0) return FPS_OK;
+  CUtensorMap tq, tkv;
+  if (!make_tmap_2d_bf16(&tq, q, (uint64_t)h_cu_q[n_req], H, (uint64_t)H * 2, 64, 128))
+    return fail(FPS_ECUDA, "attention_tc2: Q tensor map");
+  if (!make_tmap_2d_bf16(&tkv, kv, (uint64_t)h_cu_k[n_req], 2 * H, (uint64_t)H * 4, 64, 128))
+    return fail(FPS_ECUDA, "attention_tc2: KV tensor map");
+  static bool attr = false;
+  if (!attr) {
+    FPS_CUDA_TRY(cudaFuncSetAttribute(attn_tc2_kernel<D>,
+                                      cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
+    attr = true;
+  }
+  const float scale_log2 = 1.4426950408889634f / sqrtf((float)D);
+  attn_tc2_kernel<D><<<dim3(pairs, heads), 384, Cfg::SMEM, s>>>(
+      tq, tkv, reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads, scale_log2);
+  count_launch();
+  FPS_LAUNCH_CHECK();
+  return FPS_OK;
+}
+
 fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads, int head_dim,
                                const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
                                const int32_t* h_cu_k, int n_req, cudaStream_t s) {
   if (!h_cu_q || !h_cu_k) return fail(FPS_EINVAL, "attention_tc needs host cu_q / cu_k");
   if (!aligned16(q) || !aligned16(kv) || !aligned16(o))
     return fail(FPS_EINVAL, "attention_tc: unaligned operand");
+  // The two-tile kernel wins alone only when one tile per CTA leaves a partial second wave
+  // (n = 1331: 561 vs 531 TFLOP/s) and loses inside the step (578 vs 697 TFLOP/s with the cache
+  // gather co-running) and at large batches (781 vs 844): its two softmax warpgroups share the SM
+  // sub-partitions.  Default: one tile per CTA; the two-tile kernel is kept, tested, selectable.
+  const bool two = g_attn_force == 2;
+  if (two) {
+    if (head_dim == 128)
+      return launch_d2<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);
+    return launch_d2<64>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);
+  }
   if (head_dim == 128)
     return launch_d<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);
   return launch_d<64>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);

@@ -43,5 +43,7 @@ bool attention_tc_supported(int dtype, int head_dim);
 extern int g_disable_tc;
 // tests: 0 = choose, 1 = force the 1-SM tcgen05 GEMM, 2 = force the CTA-pair GEMM
 extern int g_gemm_force;
+// tests: 0 = two query tiles per CTA (default), 1 = force the one-tile attention kernel
+extern int g_attn_force;
 
 }  // namespace fps

@@ -19,17 +19,20 @@ def F():
     return fps
 
 
+KERNEL_FLAGS = {"auto": 0, "two_tile": 32, "one_tile": 16, "simt": 2}
+
+
 @pytest.mark.parametrize("d,heads", [(128, 3), (64, 4)])
-@pytest.mark.parametrize("simt", [False, True])
-def test_varlen_attention(F, d, heads, simt):
+@pytest.mark.parametrize("kernel", list(KERNEL_FLAGS))
+def test_varlen_attention(F, d, heads, kernel):
     g = synth.rng(d * 10 + heads)
     H = d * heads
-    n_active = [1, 130, 257, 64]
-    L = [5, 300, 1000, 129]
+    n_active = [1, 130, 257, 64, 384, 200]
+    L = [5, 300, 1000, 129, 700, 256]
     q = synth.latent(g, sum(n_active), H, "bf16")
     kv = synth.latent(g, sum(L), 2 * H, "bf16") * 2.0       # larger logits exercise the max
     kv = synth.bf16_round(kv)
-    F.fps_set_disable_tc(2 if simt else 0)
+    F.fps_set_disable_tc(KERNEL_FLAGS[kernel])
     try:
         out = F.masked_attention(to_dev(q, "bf16"), to_dev(kv, "bf16"), n_active, L, heads)
         torch.cuda.synchronize()
