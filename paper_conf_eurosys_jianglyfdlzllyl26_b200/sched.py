@@ -119,3 +119,75 @@ def assign_all(reqs, n_workers, cost_fn, max_batch):
         else:
             workers[w].append(r)
     return workers, held
+
+
+def simulate_serving(reqs, n_workers, max_batch, step_latency, policy="mask_aware"):
+    """Cluster of `n_workers` step-level continuous-batching workers (Fig. 8 workflow, L191-L199;
+    L237: join / leave at step boundaries) fed by a router (Alg. 2, or a baseline policy:
+    "round_robin" = request-level, "least_requests" = fewest assigned requests).
+
+    reqs: Request objects with .arrival (ms) and .steps, sorted by arrival.
+    step_latency(batch) -> ms of one denoising step of that batch (e.g. CostModel.step_latency,
+    the Alg. 1 pipeline latency from latency models fitted on this GPU).
+    Returns {rid: (arrival, finish)}; requests no worker can take are held FIFO (reading R15)."""
+    import heapq
+    workers = [[] for _ in range(n_workers)]
+    running = [[] for _ in range(n_workers)]
+    remaining, busy, held, out, ev = {}, [False] * n_workers, [], {}, []
+    seq = 0
+    for r in reqs:
+        heapq.heappush(ev, (r.arrival, 1, seq, "arr", r))
+        seq += 1
+    rr = [0]
+
+    def start_step(wid, now):
+        nonlocal seq
+        running[wid] = list(workers[wid])
+        busy[wid] = bool(running[wid])
+        if busy[wid]:
+            heapq.heappush(ev, (now + step_latency(running[wid]), 0, seq, "step", wid))
+            seq += 1
+
+    def assign(r, now):
+        free = [w for w in range(n_workers) if len(workers[w]) < max_batch]
+        if policy == "mask_aware":
+            wid = route(r, workers, step_latency, max_batch)
+        elif not free:
+            wid = None
+        elif policy == "round_robin":
+            wid = min(free, key=lambda w: (w - rr[0]) % n_workers)
+            rr[0] = (wid + 1) % n_workers
+        else:
+            wid = min(free, key=lambda w: (len(workers[w]), w))
+        if wid is None:
+            held.append(r)
+            return
+        workers[wid].append(r)
+        remaining[r.rid] = r.steps
+        if not busy[wid]:
+            start_step(wid, now)
+
+    while ev:
+        now, _, _, kind, obj = heapq.heappop(ev)
+        if kind == "arr":
+            assign(obj, now)
+            continue
+        wid = obj
+        for r in running[wid]:
+            remaining[r.rid] -= 1
+            if remaining[r.rid] == 0:
+                workers[wid].remove(r)
+                out[r.rid] = (r.arrival, now)
+        while held and len(workers[wid]) < max_batch:
+            assign(held.pop(0), now)
+        start_step(wid, now)
+    return out
+
+
+def latency_stats(out):
+    lat = sorted(f - a for a, f in out.values())
+    if not lat:
+        return {}
+    pick = lambda q: lat[min(len(lat) - 1, int(math.ceil(q * len(lat))) - 1)]
+    return {"mean_ms": sum(lat) / len(lat), "p50_ms": pick(0.5), "p95_ms": pick(0.95),
+            "makespan_ms": max(f for _, f in out.values()) - min(a for a, _ in out.values())}

@@ -91,6 +91,49 @@ def test_run_batch_matches_oracle(F, mode, dtype, policy, plan):
         assert r["step"] == min(r["step0"] + 2, r["n_steps"])
 
 
+@pytest.mark.parametrize("mode", ["kv", "y"])
+def test_degenerate_masks_in_one_batch(F, mode):
+    """Continuous batch mixing an empty mask (no masked image token: only text rows active), a
+    full mask (every row active: no cache rows), tiny and large masks, and requests at different
+    steps -- one varlen launch per kernel."""
+    g = synth.rng(5400)
+    N, steps, H, heads, Fd, L_img, L_txt = 2, 3, 256, 2, 512, 256, 16
+    L = L_img + L_txt
+    W = synth.stack_weights(g, N, H, Fd, "bf16")
+    mods = synth.mod_table(g, N, steps, H, "bf16")
+    deltas = synth.delta_table(steps)
+    cache_np = [[{"K": synth.latent(g, L, H, "bf16"), "V": synth.latent(g, L, H, "bf16"),
+                  "Y": synth.latent(g, L, H, "bf16")} for _ in range(N)] for _ in range(steps)]
+    m = F.MODE_CODE[mode]
+    cache = F.Cache(m, F.FPS_BF16, H, L_img, N, steps, n_templates=1)
+    for s in range(steps):
+        for l in range(N):
+            e = cache_np[s][l]
+            cache.store(0, s, l, to_dev(np.concatenate([e["K"], e["V"]], 1) if mode == "kv"
+                                        else e["Y"], "bf16"))
+        if mode == "kv":
+            cache.store(0, s, N, to_dev(cache_np[s][N - 1]["Y"], "bf16"))
+    torch.cuda.synchronize()
+    layers = [F.BlockWeights(w, heads, F.FPS_BF16) for w in W]
+    eng = F.Engine(layers, heads, m, F.FPS_BF16, L_img, L_txt, 6, steps, deltas, cache,
+                   mod_table=to_dev(mods, "bf16"), plan_policy=1)
+    reqs = []
+    for i, ratio in enumerate([0.0, 1.0, 1 / 256, 0.6, 0.3, 0.05]):
+        mask = synth.token_mask(synth.mask_random(g, L_img, ratio), L_txt)
+        x0 = synth.latent(g, L, H, "bf16")
+        reqs.append(dict(template_id=0, step=i % 3 if i % 3 < 2 else 0, n_steps=steps,
+                         mask_np=mask, x0=x0, mask=torch.as_tensor(mask).cuda(),
+                         x=to_dev(x0, "bf16")))
+    for r in reqs:
+        r["step0"] = r["step"]
+    eng.run_batch(reqs, 1)
+    torch.cuda.synchronize()
+    for r in reqs:
+        ref = S.masked_run(r["x0"], r["mask_np"], W, mods, deltas, [1] * N, mode, cache_np, heads,
+                           1, step0=r["step0"])
+        check_close(to_np(r["x"]), ref, stack_tol("bf16", N), f"{mode} n={r['mask_np'].sum()}")
+
+
 def test_requests_leave_at_step_boundary(F):
     """A request reaching its last step leaves; the others keep running (L237)."""
     W, mods, deltas, cache_np, eng, reqs = _setup(F, "kv", "bf16", 1, steps=3)

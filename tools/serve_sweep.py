@@ -1,0 +1,55 @@
+"""configs[4]-style serving sweep, simulated: Poisson arrivals of Flux-scale editing requests
+(mask ratios ~ Beta(2, 8.5)) routed to 1/2/4/8 GPU workers by Alg. 2 (mask-aware)
+or by request-count baselines, each worker running step-level continuous batching (max batch 8,
+L326).  Step latencies come from the Alg. 1 planner over the linear latency models the bench
+fitted on a B200 (`plan.fit` of a bench JSON line): a prediction from measured models, not a
+multi-GPU measurement (gpurun exposes one GPU).
+
+  python tools/serve_sweep.py profiles/r01_bench_c3_kv_host_tier.json > profiles/r01_serving_sim.json
+"""
+import json
+import os
+import sys
+
+import numpy as np
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import synth
+from paper_conf_eurosys_jianglyfdlzllyl26_b200 import sched
+
+
+def main():
+    b = json.load(open(sys.argv[1]))
+    fit = b["plan"]["fit"]
+    mode = b["config"]["cache_mode"]
+    comp = (fit["comp_ms_per_tflop"] / 1e12, max(fit["comp_b_ms"], 1e-3))
+    load = (1.0 / (fit["load_gbs"] * 1e6), max(fit["load_e_ms"], 1e-3))
+    cm = sched.CostModel(57, 3072, 12288, mode, comp=comp, load=load)
+    L_img, L_txt, steps = 4096, 512, 28
+    g = synth.rng(2024)
+    n_req = 400
+    ratios = synth.sample_mask_ratios(g, n_req)
+    n_active = [synth.n_masked_for(float(m), L_img) + L_txt for m in ratios]
+    # capacity of one worker: closed-loop step time of a full batch of 8 typical requests
+    typical = [sched.Request(i, int(np.median(n_active)), L_img + L_txt) for i in range(8)]
+    cap_img_s = 8 / (cm.step_latency(typical) * steps / 1e3)
+    out = {"source_bench": sys.argv[1], "mode": mode, "fit": fit,
+           "one_gpu_capacity_images_per_s": cap_img_s, "runs": []}
+    for n_gpu in (1, 2, 4, 8):
+        for load_frac in (0.5, 0.8, 0.95):
+            rate = load_frac * cap_img_s * n_gpu                     # requests per second
+            gaps = g.exponential(1e3 / rate, n_req)
+            t = np.cumsum(gaps)
+            reqs = [sched.Request(i, n_active[i], L_img + L_txt, arrival=float(t[i]), steps=steps)
+                    for i in range(n_req)]
+            for pol in ("mask_aware", "least_requests", "round_robin"):
+                res = sched.simulate_serving(reqs, n_gpu, 8, cm.step_latency, pol)
+                st = sched.latency_stats(res)
+                st.update(n_gpus=n_gpu, load=load_frac, policy=pol,
+                          images_per_s=n_req / (st["makespan_ms"] / 1e3))
+                out["runs"].append(st)
+    print(json.dumps(out, indent=1))
+
+
+if __name__ == "__main__":
+    main()
