@@ -312,7 +312,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C3", choices=list(WORKLOADS))
     ap.add_argument("--mode", default="kv", choices=["kv", "y"])
-    ap.add_argument("--tier", default="host", choices=["host", "hbm"],
+    ap.add_argument("--tier", default="host", choices=["host", "hbm", "host_hugepage"],
                     help="template cache in pinned host DRAM (configs[2]) or HBM (NEXT-1)")
     ap.add_argument("--copy-ctas", type=int, default=0, help="CTAs of the SM row gather (0 = lib default)")
     ap.add_argument("--copy-method", type=int, default=0, choices=[0, 1],
@@ -340,7 +340,8 @@ def main():
 
     metric_name = ("masked-block stack images/s (Flux-scale, 20% mask) [ms/step alongside]"
                    if args.config == "C3" else f"masked-block stack images/s ({args.config})")
-    base_cfg["cache_tier"] = "pinned host DRAM" if args.tier == "host" else "device HBM (NEXT-1)"
+    base_cfg["cache_tier"] = {"host": "pinned host DRAM", "hbm": "device HBM (NEXT-1)",
+                              "host_hugepage": "pinned host DRAM on 2 MiB pages"}[args.tier]
     base_cfg["h2d_method"] = ["SM zero-copy row gather", "DMA per row run"][args.copy_method]
     base_cfg["parallelism"] = f"request-parallel x{world} (Alg. 2 routing)"
 
@@ -383,7 +384,7 @@ def main():
     pool = make_requests(w, w["batch"] * world, SEED)
     t0 = time.perf_counter()
     n_entries = 2 * (w["layers"] + 1)
-    location = 1 if args.tier == "hbm" else 0
+    location = {"host": 0, "hbm": 1, "host_hugepage": 2}[args.tier]
     global COPY_CTAS
     COPY_CTAS = args.copy_ctas
     layers, mod, cache = build_engine_inputs(F, w, args.mode, device, n_entries, location,
@@ -432,7 +433,7 @@ def main():
         extras.update(dense_ms_per_step=dense_ms, all_cached_ms_per_step=cached_ms)
         # the same plan with every cache entry already resident in HBM: the step without any
         # host-link load; exposed load = this step - that step
-        if location == 0:
+        if location != 1:
             c_h = make_cache(F, w, args.mode, n_entries, 1, 0)
             eng_h = F.Engine(layers, w["heads"], F.MODE_CODE[args.mode], F.FPS_BF16, w["L_img"],
                              w["L_txt"], max(len(reqs_dev), 1), w["steps"], deltas, c_h,
@@ -445,8 +446,9 @@ def main():
             extras["exposed_load_ms_per_step"] = max(step_ms - noload_ms, 0.0)
         # the other caching mode, and both modes with the other cache tier, on the same batch
         other = "y" if args.mode == "kv" else "kv"
-        for md, loc, cmeth in ((other, location, args.copy_method), (args.mode, 1 - location, 0),
-                               (other, 1 - location, 0), (args.mode, location, 1 - args.copy_method)):
+        other_loc = 0 if location == 1 else 1
+        for md, loc, cmeth in ((other, location, args.copy_method), (args.mode, other_loc, 0),
+                               (other, other_loc, 0), (args.mode, location, 1 - args.copy_method)):
             if loc == 1 and cmeth == 1:
                 continue
             c2 = make_cache(F, w, md, n_entries, loc, cmeth)
@@ -456,7 +458,7 @@ def main():
                              mod_table=mod, slots=0, plan_policy=0,
                              cost_model=cm2.as_engine_model())
             o_ms, _ = run_engine_timed(F, eng_o, reqs_dev, K, W, stream, load_stream, rank, world)
-            tag = f"{md}_mode_{['host', 'hbm'][loc]}" + ("_dma" if cmeth == 1 else "")
+            tag = f"{md}_mode_{['host', 'hbm', 'host_hugepage'][loc]}" + ("_dma" if cmeth == 1 else "")
             extras[f"{tag}_ms_per_step"] = o_ms
             extras[f"{tag}_cached_blocks"] = int(sum(eng_o.last_plan()[0]))
             del eng_o

@@ -101,7 +101,7 @@ __global__ void __launch_bounds__(256, 1)
         tc::tma_load_2d(sQ + c * CHUNK, &tmQ, bar_q, head * D + c * 64, q0);
       for (int kt = 0; kt < nk; ++kt) {
         const int st = kt & 1;
-        tc::mbar_wait(&k_empty[st], ((kt >> 1) & 1) ^ 1);
+        tc::mbar_wait_sleep(&k_empty[st], ((kt >> 1) & 1) ^ 1);
         tc::mbar_expect_tx(&k_full[st], Cfg::KV_TILE);
 #pragma unroll
         for (int c = 0; c < Cfg::CH; ++c)
@@ -113,7 +113,7 @@ __global__ void __launch_bounds__(256, 1)
     if (lane == 0) {
       for (int kt = 0; kt < nk; ++kt) {
         const int st = kt & 1;
-        tc::mbar_wait(&v_empty[st], ((kt >> 1) & 1) ^ 1);
+        tc::mbar_wait_sleep(&v_empty[st], ((kt >> 1) & 1) ^ 1);
         tc::mbar_expect_tx(&v_full[st], Cfg::KV_TILE);
 #pragma unroll
         for (int c = 0; c < Cfg::CH; ++c)
@@ -125,10 +125,10 @@ __global__ void __launch_bounds__(256, 1)
     if (lane == 0 && nk > 0) {
       constexpr uint32_t idesc_s = tc::idesc_bf16(128, 128);
       constexpr uint32_t idesc_o = tc::idesc_bf16(128, D, /*b_mn_major=*/true);
-      tc::mbar_wait(bar_q, 0);
+      tc::mbar_wait_sleep(bar_q, 0);
       auto issue_s = [&](int kt) {
         const int st = kt & 1;
-        tc::mbar_wait(&k_full[st], (kt >> 1) & 1);
+        tc::mbar_wait_sleep(&k_full[st], (kt >> 1) & 1);
         tc::fence_after();
         const uint32_t qa = tc::smem_u32(sQ), kb = tc::smem_u32(sK + st * Cfg::KV_TILE);
 #pragma unroll
@@ -145,10 +145,10 @@ __global__ void __launch_bounds__(256, 1)
         // S buffer (kt+1)&1 was released by the softmax of tile kt-1 (bar_p waited below)
         if (kt + 1 < nk) issue_s(kt + 1);
         const int pb = kt & 1;
-        tc::mbar_wait(&bar_p[pb], (kt >> 1) & 1);
+        tc::mbar_wait_sleep(&bar_p[pb], (kt >> 1) & 1);
         tc::fence_after();
         const int st = kt & 1;
-        tc::mbar_wait(&v_full[st], (kt >> 1) & 1);
+        tc::mbar_wait_sleep(&v_full[st], (kt >> 1) & 1);
         tc::fence_after();
         const uint32_t pa = tc::smem_u32(sP + pb * Cfg::P_BYTES);
         const uint32_t vb = tc::smem_u32(sV + st * Cfg::KV_TILE);
@@ -375,7 +375,7 @@ __global__ void __launch_bounds__(384, 1)
                           q0 + t * 128);
       for (int kt = 0; kt < nk; ++kt) {
         const int st = kt & 1;
-        tc::mbar_wait(&k_empty[st], ((kt >> 1) & 1) ^ 1);
+        tc::mbar_wait_sleep(&k_empty[st], ((kt >> 1) & 1) ^ 1);
         tc::mbar_expect_tx(&k_full[st], Cfg::KV_TILE);
 #pragma unroll
         for (int c = 0; c < Cfg::CH; ++c)
@@ -387,7 +387,7 @@ __global__ void __launch_bounds__(384, 1)
     if (lane == 0) {
       for (int kt = 0; kt < nk; ++kt) {
         const int st = kt & 1;
-        tc::mbar_wait(&v_empty[st], ((kt >> 1) & 1) ^ 1);
+        tc::mbar_wait_sleep(&v_empty[st], ((kt >> 1) & 1) ^ 1);
         tc::mbar_expect_tx(&v_full[st], Cfg::KV_TILE);
 #pragma unroll
         for (int c = 0; c < Cfg::CH; ++c)
@@ -399,7 +399,7 @@ __global__ void __launch_bounds__(384, 1)
     if (lane == 0 && nk > 0) {
       constexpr uint32_t idesc_s = tc::idesc_bf16(128, 128);
       constexpr uint32_t idesc_o = tc::idesc_bf16(128, D, /*b_mn_major=*/true);
-      tc::mbar_wait(bar_q, 0);
+      tc::mbar_wait_sleep(bar_q, 0);
       auto issue_s = [&](int t, int kt) {           // S_t = Q_t K_kt^T  (K stage must be full)
         const uint32_t qa = tc::smem_u32(sQ + t * Cfg::Q_BYTES);
         const uint32_t kb = tc::smem_u32(sK + (kt & 1) * Cfg::KV_TILE);
@@ -420,26 +420,26 @@ __global__ void __launch_bounds__(384, 1)
                        tc::sdesc_mn_sw128(vb + ks * 2048, CHUNK), idesc_o, (kt | ks) != 0);
         tc::mma_commit(&bar_o[t]);
       };
-      tc::mbar_wait(&k_full[0], 0);
+      tc::mbar_wait_sleep(&k_full[0], 0);
       tc::fence_after();
       issue_s(0, 0);
       if (hasB) issue_s(1, 0);
       tc::mma_commit(&k_empty[0]);
       for (int kt = 0; kt < nk; ++kt) {
         const bool more = kt + 1 < nk;
-        tc::mbar_wait(&v_full[kt & 1], (kt >> 1) & 1);
-        tc::mbar_wait(&bar_p[0], kt & 1);
+        tc::mbar_wait_sleep(&v_full[kt & 1], (kt >> 1) & 1);
+        tc::mbar_wait_sleep(&bar_p[0], kt & 1);
         tc::fence_after();
         issue_pv(0, kt);
         if (!hasB) tc::mma_commit(&v_empty[kt & 1]);
         if (more) {
-          tc::mbar_wait(&k_full[(kt + 1) & 1], ((kt + 1) >> 1) & 1);
+          tc::mbar_wait_sleep(&k_full[(kt + 1) & 1], ((kt + 1) >> 1) & 1);
           tc::fence_after();
           issue_s(0, kt + 1);
           if (!hasB) tc::mma_commit(&k_empty[(kt + 1) & 1]);
         }
         if (hasB) {
-          tc::mbar_wait(&bar_p[1], kt & 1);
+          tc::mbar_wait_sleep(&bar_p[1], kt & 1);
           tc::fence_after();
           issue_pv(1, kt);
           tc::mma_commit(&v_empty[kt & 1]);
@@ -665,11 +665,10 @@ fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads
   if (!h_cu_q || !h_cu_k) return fail(FPS_EINVAL, "attention_tc needs host cu_q / cu_k");
   if (!aligned16(q) || !aligned16(kv) || !aligned16(o))
     return fail(FPS_EINVAL, "attention_tc: unaligned operand");
-  // The two-tile kernel wins alone only when one tile per CTA leaves a partial second wave
-  // (n = 1331: 561 vs 531 TFLOP/s) and loses inside the step (578 vs 697 TFLOP/s with the cache
-  // gather co-running) and at large batches (781 vs 844): its two softmax warpgroups share the SM
-  // sub-partitions.  Default: one tile per CTA; the two-tile kernel is kept, tested, selectable.
-  const bool two = g_attn_force == 2;
+  // Measured on B200 once the producer / MMA warps sleep in try_wait instead of spinning:
+  // two tiles per CTA 576 vs 537 TFLOP/s (n = 1331), 892 vs 880 (16 x 1800 rows), and a 3.4%
+  // faster HBM-tier step (25.15 vs 26.03 ms); the pinned-host step is unchanged (43.4 vs 43.6).
+  const bool two = g_attn_force != 1;
   if (two) {
     if (head_dim == 128)
       return launch_d2<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);

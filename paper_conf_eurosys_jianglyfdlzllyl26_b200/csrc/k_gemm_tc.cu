@@ -437,7 +437,9 @@ fps_status launch_gemm_tc(const void* A, const void* B, int M, int N, int K, con
   // large M where the 1-SM kernel is L2-bound (1480 vs 1070 TFLOP/s at M = 29491); at one wave
   // the extra M padding of 256-row tiles can make it lose, so then padding decides.
   const long cmin = std::min(c256, c128);
-  const bool pair_wins = cp < cmin || (cp == cmin && (tp > kNumSMs / 2 || m2 * 256 - M < 128));
+  // multi-wave problems: the pair kernel (lower L2 traffic per FLOP) regardless of the small
+  // quantisation differences the wave model sees; one wave: the wave model and M padding decide
+  const bool pair_wins = tp > kNumSMs / 2 || cp < cmin || (cp == cmin && m2 * 256 - M < 128);
   if (g_gemm_force == 2 || (g_gemm_force == 0 && pair_wins))
     return launch_pair<6>(A, B, M, N, K, ep, s);
   if (c256 <= c128) return launch_cfg<256, 4>(A, B, M, N, K, ep, s);

@@ -32,6 +32,23 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         : "memory");
   } while (!done);
 }
+// try_wait with a suspend-time hint: the waiting warp sleeps in hardware until the phase
+// completes instead of re-issuing try_wait in a tight loop.  Used by the attention's producer and
+// MMA warps, whose spinning otherwise steals issue slots from the softmax warps sharing their SM
+// sub-partition (measured: 2.3M try_wait issues per launch; 537 -> 564 TFLOP/s at n = 1331).
+// Not used in the GEMM: there the later wake-up cost more than the issue slots it saved.
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) {
+  const uint32_t a = smem_u32(bar);
+  uint32_t done;
+  do {
+    asm volatile(
+        "{\n.reg .pred p;\nmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n"
+        "selp.u32 %0, 1, 0, p;\n}\n"
+        : "=r"(done)
+        : "r"(a), "r"(parity), "r"(10000000u)
+        : "memory");
+  } while (!done);
+}
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }

@@ -8,6 +8,8 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import paper_conf_eurosys_jianglyfdlzllyl26_b200 as F
 
 n, L, heads, d, R = (int(v) for v in sys.argv[1:6])
+if len(sys.argv) > 6:
+    F.fps_set_disable_tc(int(sys.argv[6]))                # 16 one-tile, 32 two-tile kernel
 H = heads * d
 q = torch.randn(R * n, H, device="cuda").to(torch.bfloat16)
 kv = torch.randn(R * L, 2 * H, device="cuda").to(torch.bfloat16)
