@@ -35,7 +35,11 @@ struct fps_cache {
 namespace fps {
 
 constexpr int kMaxPrefetchItems = 32;
-constexpr int kPrefetchUnroll = 8;     // 16-B loads in flight per thread (PCIe latency hiding)
+// Row gather launch shape (threads per CTA, 16-B loads in flight per thread).  Measured on B200
+// (C3 pinned-host step): 256 x 8 gives 43.4 ms; 128 x 8 45.2, 64 x 16 47.7 (41 GB/s), 32 x 16
+// 50.7 -- fewer, deeper threads do not reach the link rate.  FPS_PREFETCH_SHAPE=threads,unroll
+// overrides (experiments).
+static int g_pf_threads = 256, g_pf_unroll = 8;
 
 struct PrefetchBatch {
   const uint4* src[kMaxPrefetchItems];
@@ -46,6 +50,7 @@ struct PrefetchBatch {
   int n_items;
 };
 
+template <int kPrefetchUnroll>
 __global__ void __launch_bounds__(256) prefetch_kernel(const __grid_constant__ PrefetchBatch b) {
   const long long total = b.start[b.n_items];
   const long long stride = (long long)gridDim.x * blockDim.x;
@@ -258,16 +263,26 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
       b.start[k] = acc;
       b.n_items = k;
       if (acc == 0) continue;
-      // few CTAs: the copy overlaps the compute stream and should not crowd it out
-      // measured on B200 (bench --copy-ctas sweep): 16 CTAs x 8 loads in flight sustain the
-      // PCIe link while stealing the least issue bandwidth from the compute stream
-      // HBM tier: 64 CTAs keep the HBM row gather (~0.1 ms per Flux block) well under the
-      // compute of a block; 16 were measured too slow (0.35 ms, on the critical path)
+      // few CTAs: the copy overlaps the compute stream and should not crowd it out.
+      // Measured on B200 (bench --copy-ctas sweep, 256 threads x 8 loads): 16 CTAs sustain the
+      // PCIe link while stealing the least issue bandwidth from the compute stream; the HBM tier
+      // needs 64 to keep its row gather (~0.1 ms per Flux block) off the critical path.
+      static bool shape_read = false;
+      if (!shape_read) {
+        shape_read = true;
+        if (const char* e = getenv("FPS_PREFETCH_SHAPE"))
+          if (sscanf(e, "%d,%d", &g_pf_threads, &g_pf_unroll) != 2) g_pf_threads = 64, g_pf_unroll = 16;
+      }
+      const int thr = g_pf_threads, unr = g_pf_unroll;
       int ctas = c->d.copy_ctas > 0 ? c->d.copy_ctas : (c->d.location == 1 ? 64 : 16);
-      long long want = (acc + 2047) / 2048;
+      ctas = (int)((long long)ctas * 2048 / (thr * unr));  // same loads in flight as 256 x 8
+      long long want = (acc + (long long)thr * unr - 1) / ((long long)thr * unr);
       if (want < ctas) ctas = (int)want;
+      if (ctas < 1) ctas = 1;
       prof::begin(s);
-      prefetch_kernel<<<ctas, 256, 0, s>>>(b);
+      if (unr >= 16) prefetch_kernel<16><<<ctas, thr, 0, s>>>(b);
+      else if (unr >= 8) prefetch_kernel<8><<<ctas, thr, 0, s>>>(b);
+      else prefetch_kernel<4><<<ctas, thr, 0, s>>>(b);
       prof::end(s, prof::PREFETCH, 0, 16.0 * acc);
       count_launch();
       FPS_LAUNCH_CHECK();
