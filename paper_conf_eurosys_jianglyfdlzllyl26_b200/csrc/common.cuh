@@ -144,6 +144,16 @@ __device__ __forceinline__ float gelu_tanh(float x) {
   float u = k0 * (x + k1 * x * x * x);
   return 0.5f * x * (1.0f + tanhf(u));
 }
+// bf16-output epilogues: tanh.approx.f32 (MUFU, ~2^-11 relative error, far below the bf16 output
+// rounding of 2^-9) instead of the ~20-instruction accurate tanhf, which made the MLP-up GEMM's
+// epilogue the slowest part of its last tile.  The fp32 path keeps gelu_tanh (1e-5 parity).
+__device__ __forceinline__ float gelu_tanh_fast(float x) {
+  const float k0 = 0.7978845608028654f, k1 = 0.044715f;
+  const float u = k0 * fmaf(k1 * x, x * x, x);
+  float t;
+  asm("tanh.approx.f32 %0, %1;" : "=f"(t) : "f"(u));
+  return 0.5f * x * (1.0f + t);
+}
 
 // ---- GEMM epilogue description (shared by the SIMT and tcgen05 GEMMs) --------------------
 // out[r, c] = epilogue(acc[r, c]) with

@@ -86,7 +86,7 @@ __device__ __forceinline__ void epilogue_tile(const Epilogue& ep, int M, int N, 
       }
       if (ep.act == 1) {
 #pragma unroll
-        for (int e = 0; e < 8; ++e) v[e] = gelu_tanh(v[e]);
+        for (int e = 0; e < 8; ++e) v[e] = gelu_tanh_fast(v[e]);
       }
       if (resid) {
         float rr[8];
@@ -439,7 +439,10 @@ fps_status launch_gemm_tc(const void* A, const void* B, int M, int N, int K, con
   const long cmin = std::min(c256, c128);
   // multi-wave problems: the pair kernel (lower L2 traffic per FLOP) regardless of the small
   // quantisation differences the wave model sees; one wave: the wave model and M padding decide
-  const bool pair_wins = tp > kNumSMs / 2 || cp < cmin || (cp == cmin && m2 * 256 - M < 128);
+  // (one wave, long K: the pair's deeper ring wins -- 80.5 vs 83.3 us at 1331x3072x12288;
+  //  short K: its longer prologue / epilogue lose -- 27.3 vs 23.2 us at 1331x3072x3072)
+  const bool pair_wins = tp > kNumSMs / 2 || cp < cmin ||
+                         (cp == cmin && (m2 * 256 - M < 128 || K >= 8192));
   if (g_gemm_force == 2 || (g_gemm_force == 0 && pair_wins))
     return launch_pair<6>(A, B, M, N, K, ep, s);
   if (c256 <= c128) return launch_cfg<256, 4>(A, B, M, N, K, ep, s);

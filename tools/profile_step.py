@@ -10,10 +10,11 @@ import paper_conf_eurosys_jianglyfdlzllyl26_b200 as F
 ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C3"); ap.add_argument("--mode", default="kv")
 ap.add_argument("--policy", type=int, default=1); ap.add_argument("--steps", type=int, default=2)
+ap.add_argument("--location", type=int, default=0)
 a = ap.parse_args()
 w = bench.WORKLOADS[a.config]
 dev = torch.device("cuda", 0)
-layers, mod, cache = bench.build_engine_inputs(F, w, a.mode, dev, 2 * (w["layers"] + 1))
+layers, mod, cache = bench.build_engine_inputs(F, w, a.mode, dev, 2 * (w["layers"] + 1), a.location)
 pool = bench.make_requests(w, w["batch"], bench.SEED)
 L = w["L_img"] + w["L_txt"]
 reqs = [dict(template_id=i, step=0, n_steps=w["steps"], mask=torch.as_tensor(p["mask_np"]).to(dev),
