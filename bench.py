@@ -237,7 +237,10 @@ def calibrate(F, w, mode, layers, cache, reqs, device):
         bx.append(B * u * W * 2)
         by.append(e0.elapsed_time(e1) / 4)
     c, e, r2l = sched.fit_linear(bx, by)
-    cm = sched.CostModel(w["layers"], H, Fd, mode, comp=(a, max(bb, 1e-4)), load=(c, max(e, 1e-4)))
+    # a whole-entry DMA (copy_method 2) moves the same bytes whatever the mask: its load time is
+    # flat in the row count, the fitted slope ~0 (or slightly negative by noise) -> clamp at 0
+    cm = sched.CostModel(w["layers"], H, Fd, mode, comp=(max(a, 1e-16), max(bb, 1e-4)),
+                         load=(max(c, 0.0), max(e, 1e-4)))
     info = {"comp_ms_per_tflop": a * 1e12, "comp_b_ms": bb, "comp_r2": r2c,
             "load_gbs": 1.0 / (c * 1e6) if c > 0 else None, "load_e_ms": e, "load_r2": r2l}
     return cm, info
@@ -315,11 +318,13 @@ def main():
     ap.add_argument("--tier", default="host", choices=["host", "hbm", "host_hugepage"],
                     help="template cache in pinned host DRAM (configs[2]) or HBM (NEXT-1)")
     ap.add_argument("--copy-ctas", type=int, default=0, help="CTAs of the SM row gather (0 = lib default)")
-    ap.add_argument("--copy-method", type=int, default=0, choices=[0, 1],
+    ap.add_argument("--copy-method", type=int, default=None, choices=[0, 1, 2],
                     help="H2D method: 0 SM zero-copy row gather, 1 DMA per row run")
     ap.add_argument("--no-extras", action="store_true", help="skip dense / Y-mode / profile legs")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()
+    if args.copy_method is None:          # HBM tier: whole-entry DMA (no SM time); host: gather
+        args.copy_method = 2 if args.tier == "hbm" else 0
 
     rank = int(os.environ.get("RANK", 0))
     world = int(os.environ.get("WORLD_SIZE", 1))
@@ -342,7 +347,7 @@ def main():
                    if args.config == "C3" else f"masked-block stack images/s ({args.config})")
     base_cfg["cache_tier"] = {"host": "pinned host DRAM", "hbm": "device HBM (NEXT-1)",
                               "host_hugepage": "pinned host DRAM on 2 MiB pages"}[args.tier]
-    base_cfg["h2d_method"] = ["SM zero-copy row gather", "DMA per row run"][args.copy_method]
+    base_cfg["h2d_method"] = ["SM row gather", "DMA per row run", "DMA of whole entries"][args.copy_method]
     base_cfg["parallelism"] = f"request-parallel x{world} (Alg. 2 routing)"
 
     if args.impl == "reference":
@@ -390,7 +395,7 @@ def main():
     layers, mod, cache = build_engine_inputs(F, w, args.mode, device, n_entries, location,
                                              args.copy_method)
     base_cfg["cache_tier"] = "pinned host DRAM" if location == 0 else "device HBM (NEXT-1)"
-    base_cfg["h2d_method"] = ["SM zero-copy row gather", "DMA per row run"][args.copy_method]
+    base_cfg["h2d_method"] = ["SM row gather", "DMA per row run", "DMA of whole entries"][args.copy_method]
     torch.cuda.synchronize()
     log(f"[rank {rank}] inputs ready in {time.perf_counter() - t0:.1f}s")
     my_pool = pool[:w["batch"]]
@@ -434,7 +439,7 @@ def main():
         # the same plan with every cache entry already resident in HBM: the step without any
         # host-link load; exposed load = this step - that step
         if location != 1:
-            c_h = make_cache(F, w, args.mode, n_entries, 1, 0)
+            c_h = make_cache(F, w, args.mode, n_entries, 1, 2)
             eng_h = F.Engine(layers, w["heads"], F.MODE_CODE[args.mode], F.FPS_BF16, w["L_img"],
                              w["L_txt"], max(len(reqs_dev), 1), w["steps"], deltas, c_h,
                              mod_table=mod, slots=0, plan_policy=3, plan=list(plan))
@@ -447,8 +452,10 @@ def main():
         # the other caching mode, and both modes with the other cache tier, on the same batch
         other = "y" if args.mode == "kv" else "kv"
         other_loc = 0 if location == 1 else 1
-        for md, loc, cmeth in ((other, location, args.copy_method), (args.mode, other_loc, 0),
-                               (other, other_loc, 0), (args.mode, location, 1 - args.copy_method)):
+        other_cm = 2 if other_loc == 1 else 0
+        for md, loc, cmeth in ((other, location, args.copy_method),
+                               (args.mode, other_loc, other_cm), (other, other_loc, other_cm),
+                               (args.mode, location, 1 if args.copy_method != 1 else 0)):
             if loc == 1 and cmeth == 1:
                 continue
             c2 = make_cache(F, w, md, n_entries, loc, cmeth)

@@ -109,8 +109,14 @@ typedef struct {
   int32_t n_entries;     /* physical entries in the pinned arena; 0 = one per key.  When
                             smaller, key k maps to entry k % n_entries (perf runs only: bytes
                             moved are identical, contents alias)                            */
-  int32_t copy_method;   /* 0 = SM zero-copy row gather over mapped pinned memory (default);
-                            1 = copy-engine DMA of coalesced row runs                        */
+  int32_t copy_method;   /* 0 = SM row gather (zero-copy over mapped pinned memory, or from
+                                the HBM arena) -- exactly the rows U (default);
+                            1 = copy-engine DMA of coalesced row runs of U;
+                            2 = copy-engine DMA of the WHOLE entry (all L_img rows, one copy
+                                per request): no SM time, but rows outside U are overwritten
+                                too, so fresh K/V must be written only after `ready_event`
+                                (fps_run_batch orders this itself).  Meant for the HBM tier,
+                                where the extra bytes are cheap and SM time is not.            */
   int32_t copy_ctas;     /* CTAs used by method 0 (0 = default: 16 for the host link -- enough
                             for PCIe, few enough not to crowd out the compute stream -- and 64
                             for the HBM tier)                                               */

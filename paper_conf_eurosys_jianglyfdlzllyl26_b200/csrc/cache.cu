@@ -99,6 +99,8 @@ static size_t offset_of(const fps_cache* c, uint32_t t, int step, int layer) {
   return (size_t)(key_of(c, t, step, layer) % c->n_entries) * c->entry_bytes;
 }
 
+bool cache_writes_all_rows(const fps_cache* c) { return c && c->d.copy_method == 2; }
+
 }  // namespace fps
 
 using namespace fps;
@@ -112,7 +114,7 @@ fps_status fps_cache_create(const fps_cache_desc* desc, fps_cache_t* out) {
   FPS_CHECK_ARG(d.dtype == FPS_BF16 || d.dtype == FPS_F32, "dtype %d", d.dtype);
   FPS_CHECK_ARG(d.H > 0 && d.L_img > 0 && d.n_layers > 0 && d.n_steps > 0 && d.n_templates > 0,
                 "sizes must be positive");
-  FPS_CHECK_ARG(d.n_entries >= 0 && (d.copy_method == 0 || d.copy_method == 1), "bad desc");
+  FPS_CHECK_ARG(d.n_entries >= 0 && d.copy_method >= 0 && d.copy_method <= 2, "bad desc");
   auto* c = new (std::nothrow) fps_cache();
   if (!c) return fail(FPS_ENOMEM, "cache: host allocation");
   c->d = d;
@@ -240,9 +242,19 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
                   "item %d: dst_row_bytes %d != entry row bytes %zu", i, it.dst_row_bytes,
                   row_bytes_of(c, it.layer));
     if (c->d.copy_method == 0) FPS_CHECK_ARG(it.n_rows == 0 || it.d_rows, "item %d: d_rows", i);
-    else FPS_CHECK_ARG(it.n_rows == 0 || it.h_rows, "item %d: h_rows needed for DMA", i);
+    else if (c->d.copy_method == 1)
+      FPS_CHECK_ARG(it.n_rows == 0 || it.h_rows, "item %d: h_rows needed for DMA", i);
   }
-  if (c->d.copy_method == 0) {
+  if (c->d.copy_method == 2) {
+    // whole entries: one contiguous DMA per request (rows [0, L_img) land at their token rows)
+    for (int i = 0; i < n_items; ++i) {
+      const fps_prefetch_item& it = items[i];
+      if (it.n_rows == 0) continue;
+      FPS_CUDA_TRY(cudaMemcpyAsync(it.d_dst, c->host + offset_of(c, it.template_id, it.step, it.layer),
+                                   (size_t)c->d.L_img * row_bytes_of(c, it.layer),
+                                   cudaMemcpyDefault, s));
+    }
+  } else if (c->d.copy_method == 0) {
     for (int base = 0; base < n_items; base += kMaxPrefetchItems) {
       PrefetchBatch b{};
       long long acc = 0;

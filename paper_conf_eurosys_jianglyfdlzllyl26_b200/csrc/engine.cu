@@ -429,6 +429,12 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
         kvbuf = e->slots[pos[l] % e->D];
         ev = e->ready[pos[l]];
         consumed_after = pos[l];
+        if (cache_writes_all_rows(e->d.cache)) {
+          // whole-entry DMA also lands on the masked rows: the QKV epilogue's fresh K/V must
+          // come after it (the load was issued layers ahead, so this rarely waits)
+          FPS_CUDA_TRY(cudaStreamWaitEvent(cs, ev, 0));
+          ev = nullptr;
+        }
       } else {
         kvbuf = e->kv_scratch;
       }

@@ -38,6 +38,10 @@ fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads
                                const int32_t* h_cu_k, int n_req, cudaStream_t s);
 bool attention_tc_supported(int dtype, int head_dim);
 
+// true if fps_cache_prefetch also overwrites rows outside U (copy_method 2): fresh rows written
+// into the same buffer must then be ordered after the load's ready event
+bool cache_writes_all_rows(const fps_cache* c);
+
 // global switches (tests can force the SIMT kernels): bit0 = no tcgen05 GEMM,
 // bit1 = no tensor-core attention
 extern int g_disable_tc;

@@ -148,7 +148,8 @@ def test_requests_leave_at_step_boundary(F):
         check_close(to_np(r["x"]), x, stack_tol("bf16", 3), "leave")
 
 
-@pytest.mark.parametrize("slots,method,location", [(1, 0, 0), (2, 1, 0), (0, 0, 0), (2, 0, 1)])
+@pytest.mark.parametrize("slots,method,location", [(1, 0, 0), (2, 1, 0), (0, 0, 0), (2, 0, 1),
+                                                  (0, 2, 1), (1, 2, 1), (2, 2, 0)])
 def test_pipeline_slots_and_copy_methods_bit_identical(F, slots, method, location):
     """The staging ring depth, the H2D method and the cache tier (pinned host / HBM) change
     timing only, never the bits."""
@@ -163,14 +164,19 @@ def test_pipeline_slots_and_copy_methods_bit_identical(F, slots, method, locatio
         assert torch.equal(a.view(torch.int16), b.view(torch.int16))
 
 
-def test_delayed_load_stream_bit_identical(F):
+@pytest.mark.parametrize("mode,method,location", [("y", 0, 0), ("kv", 0, 0), ("kv", 2, 1),
+                                                  ("y", 2, 1)])
+def test_delayed_load_stream_bit_identical(F, mode, method, location):
     """Robustness of the event ordering: a busy load stream (a long spin queued before the
-    prefetches) must not change the result."""
-    _, _, _, _, eng, reqs = _setup(F, "y", "bf16", 1, seed=5200)
+    prefetches) must not change the result -- in particular a late whole-entry DMA (method 2)
+    must not land on fresh K/V rows."""
+    _, _, _, _, eng, reqs = _setup(F, mode, "bf16", 1, seed=5200, copy_method=method,
+                                   location=location)
     eng.run_batch(reqs, 2)
     torch.cuda.synchronize()
     ref = [r["x"].clone() for r in reqs]
-    _, _, _, _, eng, reqs = _setup(F, "y", "bf16", 1, seed=5200)
+    _, _, _, _, eng, reqs = _setup(F, mode, "bf16", 1, seed=5200, copy_method=method,
+                                   location=location)
     ls = torch.cuda.Stream()
     with torch.cuda.stream(ls):
         torch.cuda._sleep(200_000_000)          # ~0.1 s of spinning on the load stream
