@@ -220,12 +220,16 @@ def calibrate(F, w, mode, layers, cache, reqs, device):
     W = (2 if mode == "kv" else 1) * H
     dst = torch.empty(B * L, W, dtype=torch.bfloat16, device=device)
     ls = torch.cuda.Stream(device=device)
-    for m in (0.05, 0.3, 0.6, 0.9):
+    whole = cache.desc.copy_method == 2
+    for k, m in enumerate((0.05, 0.3, 0.6, 0.9)):
         u = w["L_img"] - synth.n_masked_for(m, w["L_img"])
         rows = torch.arange(u, device=device, dtype=torch.int32)
         h_rows = np.arange(u, dtype=np.int32)
         items = [F.fps_prefetch_item(i, 0, 0, u, rows.data_ptr(), h_rows.ctypes.data,
                                      dst[i * L].data_ptr(), W * 2) for i in range(B)]
+        if whole:                 # whole-entry DMA: bytes do not depend on u; vary the count
+            items = items * (k + 1)
+            u = w["L_img"] * (k + 1)
         for _ in range(2):
             cache.prefetch(items, ls)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -240,7 +244,8 @@ def calibrate(F, w, mode, layers, cache, reqs, device):
     # a whole-entry DMA (copy_method 2) moves the same bytes whatever the mask: its load time is
     # flat in the row count, the fitted slope ~0 (or slightly negative by noise) -> clamp at 0
     cm = sched.CostModel(w["layers"], H, Fd, mode, comp=(max(a, 1e-16), max(bb, 1e-4)),
-                         load=(max(c, 0.0), max(e, 1e-4)))
+                         load=(max(c, 0.0), max(e, 1e-4)),
+                         full_entry_rows=w["L_img"] if whole else None)
     info = {"comp_ms_per_tflop": a * 1e12, "comp_b_ms": bb, "comp_r2": r2c,
             "load_gbs": 1.0 / (c * 1e6) if c > 0 else None, "load_e_ms": e, "load_r2": r2l}
     return cm, info
@@ -323,8 +328,13 @@ def main():
     ap.add_argument("--no-extras", action="store_true", help="skip dense / Y-mode / profile legs")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()
+    import faulthandler                   # a stuck run dumps every thread's stack and exits
+    faulthandler.dump_traceback_later(900, exit=True)
     if args.copy_method is None:          # HBM tier: whole-entry DMA (no SM time); host: gather
-        args.copy_method = 2 if args.tier == "hbm" else 0
+        # measured on B200 (C3) with the planner's load model counting whole entries: KV-mode
+        # host 38.1 ms with whole-entry DMA vs 43.3 with the SM row gather (no SM interference
+        # outweighs +25% bytes), Y-mode host 30.8 vs 36.4, HBM tier 23.0 vs 24.4
+        args.copy_method = 2
 
     rank = int(os.environ.get("RANK", 0))
     world = int(os.environ.get("WORLD_SIZE", 1))
@@ -399,7 +409,9 @@ def main():
     torch.cuda.synchronize()
     log(f"[rank {rank}] inputs ready in {time.perf_counter() - t0:.1f}s")
     my_pool = pool[:w["batch"]]
+    log(f"[rank {rank}] calibrating")
     cm, fit = calibrate(F, w, args.mode, layers, cache, [dict()] * w["batch"], device)
+    log(f"[rank {rank}] fit {fit}")
     my_ids, assign, held = sched.shard_requests([p["n_active"] for p in pool], L, world, rank, cm,
                                                 w["batch"])
     mine = [pool[i] for i in my_ids]
@@ -419,6 +431,7 @@ def main():
                         slots=0, plan_policy=policy, cost_model=cm.as_engine_model())
 
     eng = engine(0)
+    log(f"[rank {rank}] timed run")
     with Clocks(local) as clk:
         step_ms, launches = run_engine_timed(F, eng, reqs_dev, K, W, stream, load_stream, rank, world)
     plan, pred_ms = eng.last_plan()
@@ -427,6 +440,7 @@ def main():
 
     extras = {}
     if not args.no_extras:
+        log(f"[rank {rank}] extras")
         # same batch, every block dense (all tokens, no cache): the compute-saving reference
         eng_d = engine(2)
         dense_ms, _ = run_engine_timed(F, eng_d, reqs_dev, K, W, stream, load_stream, rank, world)
@@ -473,6 +487,7 @@ def main():
 
     # per-kernel-class device time over the same timed region (CUDA events on each kernel's
     # own stream), for the roofline of the dominant kernel
+    log(f"[rank {rank}] profile pass")
     F.fps_profile_enable(1)
     run_engine_timed(F, eng, reqs_dev, K, W, stream, load_stream, rank, world)
     ms = (torch.zeros(7, dtype=torch.float64)).numpy()
@@ -502,6 +517,7 @@ def main():
                 "avg_launch_ms": gemm_avg_ms,
                 "flops_per_launch": fl[0] / max(cnt[0], 1)}
 
+    log(f"[rank {rank}] e2e")
     # e2e through the public call with HOST buffers: per step H2D latents, one step, D2H latents
     host_x = [torch.empty(L, w["H"], dtype=torch.bfloat16).pin_memory() for _ in reqs_dev]
     for h, r in zip(host_x, reqs_dev):

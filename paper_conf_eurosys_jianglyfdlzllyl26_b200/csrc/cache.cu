@@ -2,12 +2,16 @@
 // store, L207 block granularity, L209 "while loading the i-th block, the computation stream
 // can concurrently execute the computation of the (i-1)-th block"; reading R7 keys).
 //
-// Two H2D methods (fps_cache_desc.copy_method):
+// Three load methods (fps_cache_desc.copy_method):
 //  0  SM zero-copy gather: a few CTAs read the unmasked rows straight out of the mapped pinned
 //     arena over PCIe (16-B loads, many in flight) and write them to their token rows in HBM.
-//     One launch per layer for the whole batch, exact bytes, any mask shape.
-//  1  copy-engine DMA: the unmasked rows are coalesced into runs of consecutive tokens and
-//     issued as one cudaMemcpyBatchAsync (no SM time; per-run descriptor overhead).
+//     One launch per layer for the whole batch, exact bytes, any mask shape -- but the gather
+//     warps share the SMs with the compute stream (~10% slower GEMMs in the step).
+//  1  copy-engine DMA: the unmasked rows coalesced into runs of consecutive tokens, one
+//     cudaMemcpyAsync per run (no SM time; per-run overhead).
+//  2  copy-engine DMA of whole entries (all L_img rows, one copy per request and block): +25%
+//     bytes at m = 0.2 but no SM time and no per-run overhead; the caller orders fresh-row writes
+//     after the ready event.  Fastest measured step on B200 for both tiers.
 #include <sys/mman.h>
 
 #include <algorithm>
@@ -247,13 +251,17 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
   }
   if (c->d.copy_method == 2) {
     // whole entries: one contiguous DMA per request (rows [0, L_img) land at their token rows)
+    double bytes = 0;
+    prof::begin(s);
     for (int i = 0; i < n_items; ++i) {
       const fps_prefetch_item& it = items[i];
       if (it.n_rows == 0) continue;
+      const size_t nb = (size_t)c->d.L_img * row_bytes_of(c, it.layer);
       FPS_CUDA_TRY(cudaMemcpyAsync(it.d_dst, c->host + offset_of(c, it.template_id, it.step, it.layer),
-                                   (size_t)c->d.L_img * row_bytes_of(c, it.layer),
-                                   cudaMemcpyDefault, s));
+                                   nb, cudaMemcpyDefault, s));
+      bytes += nb;
     }
+    prof::end(s, prof::PREFETCH, 0, bytes);
   } else if (c->d.copy_method == 0) {
     for (int base = 0; base < n_items; base += kMaxPrefetchItems) {
       PrefetchBatch b{};
@@ -321,8 +329,13 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
     }
     // one DMA per run of consecutive rows (cudaMemcpyBatchAsync dropped rows of long runs in
     // testing on this driver, so the runs are issued individually)
-    for (size_t q = 0; q < c->sizes.size(); ++q)
+    double bytes = 0;
+    prof::begin(s);
+    for (size_t q = 0; q < c->sizes.size(); ++q) {
       FPS_CUDA_TRY(cudaMemcpyAsync(c->dsts[q], c->srcs[q], c->sizes[q], cudaMemcpyDefault, s));
+      bytes += c->sizes[q];
+    }
+    prof::end(s, prof::PREFETCH, 0, bytes);
   }
   if (ready_event) FPS_CUDA_TRY(cudaEventRecord((cudaEvent_t)ready_event, s));
   return FPS_OK;

@@ -274,8 +274,10 @@ static void make_plan(fps_engine* e, const Batch& B) {
   for (int i = 0; i < B.n; ++i) {
     fm += flops_block(e->d.mode, B.nq[i], L, H, F);
     fd += flops_block(FPS_MODE_KV, L, L, H, F);
-    by += (double)B.nu[i] * e->row_w;
-    byf += (double)B.nu[i] * e->row_h;
+    // rows the load moves: U, or the whole entry for the whole-entry DMA method
+    const double rows = (B.nu[i] > 0 && cache_writes_all_rows(e->d.cache)) ? e->d.L_img : B.nu[i];
+    by += rows * e->row_w;
+    byf += rows * e->row_h;
   }
   std::vector<double> Cw(N, a * fm + b), Cwo(N, a * fd + b), Lm(N, by > 0 ? c * by + ec : 0.0);
   const double fin = byf > 0 ? c * byf + ec : 0.0;

@@ -56,17 +56,23 @@ class Request:
 class CostModel:
     """Per-block costs of a batch for Alg. 1 from the two fitted linear models."""
 
-    def __init__(self, n_layers, H, F, mode, comp=(1e-12, 0.01), load=(2e-8, 0.01), elt=2):
+    def __init__(self, n_layers, H, F, mode, comp=(1e-12, 0.01), load=(2e-8, 0.01), elt=2,
+                 full_entry_rows=None):
         self.n_layers, self.H, self.F, self.mode, self.elt = n_layers, H, F, mode, elt
         self.comp, self.load = comp, load
+        # whole-entry DMA loads (copy_method 2) move L_img rows whatever the mask
+        self.full_entry_rows = full_entry_rows
+
+    def _rows(self, r):
+        return self.full_entry_rows if (self.full_entry_rows and r.u > 0) else r.u
 
     def costs(self, batch):
         a, b = self.comp
         c, e = self.load
         fm = sum(block_flops(self.mode, r.n, r.L, self.H, self.F) for r in batch)
         fd = sum(block_flops("dense", r.n, r.L, self.H, self.F) for r in batch)
-        by = sum(cache_bytes(self.mode, r.u, self.H, self.elt) for r in batch)
-        byf = sum(cache_bytes("y", r.u, self.H, self.elt) for r in batch)
+        by = sum(cache_bytes(self.mode, self._rows(r), self.H, self.elt) for r in batch)
+        byf = sum(cache_bytes("y", self._rows(r), self.H, self.elt) for r in batch)
         N = self.n_layers
         Cw = [a * fm + b] * N
         Cwo = [a * fd + b] * N
