@@ -5,7 +5,7 @@ L326).  Step latencies come from the Alg. 1 planner over the linear latency mode
 fitted on a B200 (`plan.fit` of a bench JSON line): a prediction from measured models, not a
 multi-GPU measurement (gpurun exposes one GPU).
 
-  python tools/serve_sweep.py profiles/r01_bench_c3_kv_host_tier.json > profiles/r01_serving_sim.json
+  python tools/serve_sweep.py profiles/r01_bench_c3_default.json > profiles/r01_serving_sim.json
 """
 import json
 import os
@@ -24,8 +24,10 @@ def main():
     mode = b["config"]["cache_mode"]
     comp = (fit["comp_ms_per_tflop"] / 1e12, max(fit["comp_b_ms"], 1e-3))
     load = (1.0 / (fit["load_gbs"] * 1e6), max(fit["load_e_ms"], 1e-3))
-    cm = sched.CostModel(57, 3072, 12288, mode, comp=comp, load=load)
     L_img, L_txt, steps = 4096, 512, 28
+    whole = "whole" in b["config"].get("h2d_method", "")
+    cm = sched.CostModel(57, 3072, 12288, mode, comp=comp, load=load,
+                         full_entry_rows=L_img if whole else None)
     g = synth.rng(2024)
     n_req = 400
     ratios = synth.sample_mask_ratios(g, n_req)
