@@ -11,6 +11,7 @@ namespace fps {
 static thread_local std::string g_err;
 thread_local long long g_launches = 0;
 int g_disable_tc = 0;
+int g_pdl = 1;
 
 void set_error(const char* fmt, ...) {
   char buf[1024];
@@ -287,6 +288,7 @@ void fps_set_disable_tc(int32_t flags) {
   fps::g_disable_tc = flags & 3;
   fps::g_gemm_force = (flags >> 2) & 3;
   fps::g_attn_force = (flags >> 4) & 3;
+  fps::g_pdl = (flags & 64) ? 0 : 1;
 }
 
 fps_status fps_build_mask_index(const uint8_t* d_masks, const int32_t* d_offsets, int32_t n_req,

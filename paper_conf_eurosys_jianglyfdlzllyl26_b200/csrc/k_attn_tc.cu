@@ -91,6 +91,8 @@ __global__ void __launch_bounds__(256, 1)
   __syncthreads();
   tc::fence_after();
   const uint32_t tmem = *tmem_holder;
+  pdl_trigger();
+  pdl_wait();
   const uint32_t tS = tmem, tO = tmem + 256;
 
   if (warp == 0) {
@@ -364,6 +366,8 @@ __global__ void __launch_bounds__(384, 1)
   __syncthreads();
   tc::fence_after();
   const uint32_t tmem = *tmem_holder;
+  pdl_trigger();
+  pdl_wait();
 
   if (warp == 0) {
     if (lane == 0 && nk > 0) {
@@ -624,8 +628,9 @@ static fps_status launch_d(const void* q, const void* kv, void* o, int heads,
     attr = true;
   }
   const float scale_log2 = 1.4426950408889634f / sqrtf((float)D);
-  attn_tc_kernel<D><<<dim3(tiles, heads), 256, Cfg::SMEM, s>>>(
-      tq, tkv, reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads, scale_log2);
+  FPS_CUDA_TRY(launch_k(attn_tc_kernel<D>, dim3(tiles, heads), dim3(256), Cfg::SMEM, s, tq, tkv,
+                        reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads,
+                        scale_log2));
   count_launch();
   FPS_LAUNCH_CHECK();
   return FPS_OK;
@@ -652,8 +657,9 @@ static fps_status launch_d2(const void* q, const void* kv, void* o, int heads,
     attr = true;
   }
   const float scale_log2 = 1.4426950408889634f / sqrtf((float)D);
-  attn_tc2_kernel<D><<<dim3(pairs, heads), 384, Cfg::SMEM, s>>>(
-      tq, tkv, reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads, scale_log2);
+  FPS_CUDA_TRY(launch_k(attn_tc2_kernel<D>, dim3(pairs, heads), dim3(384), Cfg::SMEM, s, tq, tkv,
+                        reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads,
+                        scale_log2));
   count_launch();
   FPS_LAUNCH_CHECK();
   return FPS_OK;

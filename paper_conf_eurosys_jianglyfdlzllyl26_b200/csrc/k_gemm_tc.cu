@@ -164,6 +164,8 @@ __global__ void __launch_bounds__(256, 1)
   __syncthreads();
   tc::fence_after();
   const uint32_t tmem_base = *tmem_holder;
+  pdl_trigger();   // setup done: let the next kernel's CTAs start as ours retire
+  pdl_wait();      // inputs of this GEMM come from the previous kernel
 
   if (warp == 0) {
     if (lane == 0) {
@@ -295,6 +297,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
   tc::cluster_sync();                                      // peer barriers initialised
   tc::fence_after();
   const uint32_t tmem_base = *tmem_holder;
+  pdl_trigger();   // setup done: let the next kernel's CTAs start as ours retire
+  pdl_wait();      // inputs of this GEMM come from the previous kernel
 
   if (warp == 0) {
     if (lane == 0) {
@@ -393,7 +397,8 @@ static fps_status launch_cfg(const void* A, const void* B, int M, int N, int K,
   }
   const int tiles = ceil_div(M, Cfg::BM) * ceil_div(N, BN);
   const int grid = tiles < kNumSMs ? tiles : kNumSMs;
-  gemm_tc_kernel<BN, STAGES><<<grid, 256, Cfg::SMEM, s>>>(ta, tb, M, N, K, ep);
+  FPS_CUDA_TRY(launch_k(gemm_tc_kernel<BN, STAGES>, dim3(grid), dim3(256), Cfg::SMEM, s, ta, tb,
+                        M, N, K, ep));
   count_launch();
   FPS_LAUNCH_CHECK();
   return FPS_OK;
@@ -415,7 +420,8 @@ static fps_status launch_pair(const void* A, const void* B, int M, int N, int K,
   }
   const int tiles = ceil_div(M, Cfg::BM) * ceil_div(N, Cfg::BN);
   const int pairs = tiles < kNumSMs / 2 ? tiles : kNumSMs / 2;
-  gemm_tc2_kernel<STAGES><<<2 * pairs, 256, Cfg::SMEM, s>>>(ta, tb, M, N, K, ep);
+  FPS_CUDA_TRY(launch_k(gemm_tc2_kernel<STAGES>, dim3(2 * pairs), dim3(256), Cfg::SMEM, s, ta, tb,
+                        M, N, K, ep));
   count_launch();
   FPS_LAUNCH_CHECK();
   return FPS_OK;

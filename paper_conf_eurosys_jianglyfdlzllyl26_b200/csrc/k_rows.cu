@@ -71,6 +71,8 @@ __global__ void __launch_bounds__(256) copy_rows_kernel(const uint4* __restrict_
                                                         const int32_t* __restrict__ dst_ids,
                                                         long long total, int vpr,
                                                         uint4* __restrict__ dst) {
+  pdl_trigger();
+  pdl_wait();
   const long long stride = (long long)gridDim.x * blockDim.x;
   long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   for (; i < total; i += 4 * stride) {
@@ -104,8 +106,9 @@ fps_status launch_copy_rows(const void* src, const int32_t* src_ids, const int32
   int grid = (int)(want < cap ? want : cap);
   if (grid < 1) grid = 1;
   prof::begin(s);
-  copy_rows_kernel<<<grid, 256, 0, s>>>(reinterpret_cast<const uint4*>(src), src_ids, dst_ids,
-                                        total, vpr, reinterpret_cast<uint4*>(dst));
+  FPS_CUDA_TRY(launch_k(copy_rows_kernel, dim3(grid), dim3(256), 0, s,
+                        reinterpret_cast<const uint4*>(src), src_ids, dst_ids, total, vpr,
+                        reinterpret_cast<uint4*>(dst)));
   prof::end(s, prof::ROWS, 0, 2.0 * n * row_bytes);
   count_launch();
   FPS_LAUNCH_CHECK();
@@ -194,6 +197,8 @@ __global__ void __launch_bounds__(128) ln_mod_row_kernel(const T* __restrict__ x
                                                          const T* __restrict__ mod, int shift_off) {
   constexpr int NV = Vec16<T>::N;
   __shared__ float red[4];
+  pdl_trigger();
+  pdl_wait();
   const int row = blockIdx.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int nvec = H / NV;
   const int src_row = rows ? __ldg(rows + row) : row;
@@ -270,13 +275,17 @@ static fps_status ln_mod_t(const void* x, const int32_t* rows, int n, int H, voi
   const int per_thread = ceil_div(H / NV, 128);
   if (H / NV >= 128 && per_thread <= 8) {
     prof::begin(s);
+    cudaError_t le;
 #define FPS_LNR_CASE(VPT)                                                                  \
     if (per_thread <= VPT)                                                                 \
-      ln_mod_row_kernel<T, VPT><<<n, 128, 0, s>>>(X, rows, H, O, cu, n_req, Md, shift_off); \
+      le = launch_k(ln_mod_row_kernel<T, VPT>, dim3(n), dim3(128), 0, s, X, rows, H, O, cu, \
+                    n_req, Md, shift_off);                                                 \
     else
     FPS_LNR_CASE(1) FPS_LNR_CASE(2) FPS_LNR_CASE(3) FPS_LNR_CASE(4) FPS_LNR_CASE(6)
-    ln_mod_row_kernel<T, 8><<<n, 128, 0, s>>>(X, rows, H, O, cu, n_req, Md, shift_off);
+    le = launch_k(ln_mod_row_kernel<T, 8>, dim3(n), dim3(128), 0, s, X, rows, H, O, cu, n_req,
+                  Md, shift_off);
 #undef FPS_LNR_CASE
+    FPS_CUDA_TRY(le);
     prof::end(s, prof::LN, 0, 2.0 * n * H * sizeof(T));
     count_launch();
     FPS_LAUNCH_CHECK();
