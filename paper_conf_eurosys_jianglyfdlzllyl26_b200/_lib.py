@@ -10,7 +10,8 @@ import ctypes as C
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libflashps.so")
+# FPS_LIB selects another in-tree build of the same library (used by tools/ for A/B timing)
+LIB_PATH = os.environ.get("FPS_LIB") or os.path.join(_HERE, "libflashps.so")
 
 FPS_OK, FPS_EINVAL, FPS_ECUDA, FPS_ENOMEM, FPS_EUNSUPPORTED, FPS_ESTATE = 0, -1, -2, -3, -4, -5
 FPS_F32, FPS_BF16 = 0, 1
