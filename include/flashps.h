@@ -51,7 +51,8 @@ int32_t fps_device_ok(void);
 /* Test / bench hooks: number of kernels this thread has launched through the library so far;
  * force the SIMT kernels (bit0: GEMMs, bit1: attention) instead of the tensor-core ones;
  * bits 2-3 = 1 force the 1-SM tcgen05 GEMM, = 2 force the CTA-pair (cta_group::2) GEMM;
- * bits 4-5 = 1 force the one-query-tile attention kernel, = 2 the two-tile (ping-pong) one;
+ * bits 4-5 = 1 force the one-query-tile attention kernel, = 2 the two-tile kernel with P in
+ * shared memory, = 3 the two-tile kernel with P in TMEM and a correction warpgroup (the default);
  * bit 6 = launch without programmatic dependent launch (PDL is on by default). */
 int64_t fps_launch_count(void);
 void fps_set_disable_tc(int32_t flags);

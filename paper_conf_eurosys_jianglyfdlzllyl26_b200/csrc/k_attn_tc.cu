@@ -599,7 +599,380 @@ __global__ void __launch_bounds__(384, 1)
   }
 }
 
-int g_attn_force = 0;   // tests: 1 = force the one-tile kernel
+// ============================================================================================
+// Two query tiles per CTA with P kept in TMEM and a correction warpgroup (default kernel).
+//   warp 0      TMA: both Q tiles, then K tiles (2-stage ring)
+//   warp 1      MMA: S_A(j), S_B(j), PV_A(j), S_A(j+1), PV_B(j), S_B(j+1), ...  PV takes P from
+//               TMEM (A operand "ts" form), V from smem (MN-major); S_t(j+1) is issued right after
+//               PV_t(j) into the same columns -- tcgen05.mma executes in issue order
+//   warp 2      TMEM allocation
+//   warp 3      TMA: V tiles (2-stage ring)
+//   warps 4-7   softmax of tile A, 8-11 of tile B: thread = query row, the whole S row in
+//               registers (one tcgen05.ld round), P as bf16 pairs back into the upper half of the
+//               tile's S columns (tcgen05.st), lazy max with its rescale factor left in smem
+//   warps 12-15 correction: rescale O_t in TMEM when a row's max grew (off the softmax critical
+//               path; O_t(j-1) is complete by then because S_t(j) was issued after PV_t(j-1)),
+//               final O / l to global
+// Registers are rebalanced per warpgroup with setmaxnreg (softmax 192, correction 72, rest 56)
+// so the 128-float S row fits without spills.  TMEM: S_A/P_A [0,128), S_B/P_B [128,256),
+// O_A [256,256+D), O_B [384,384+D).  No smem P tile: the two softmax warpgroups no longer wait
+// for each other's PV to free a shared buffer.
+// Tuning knobs of the P-in-TMEM kernels (compile-time; defaults are the measured best):
+//   FPS_ATTN_POLY  N > 0: every N-th group of 8 exponentials on the FMA pipe (0: all on MUFU)
+//   FPS_ATTN_MMA_SPIN  1: the MMA warp spins on the P barriers instead of sleeping in try_wait
+#ifndef FPS_ATTN_POLY
+#define FPS_ATTN_POLY 4
+#endif
+#ifndef FPS_ATTN_MMA_SPIN
+#define FPS_ATTN_MMA_SPIN 0
+#endif
+#if FPS_ATTN_MMA_SPIN
+#define ATTN_MMA_WAIT(bar, par) tc::mbar_wait(bar, par)
+#else
+#define ATTN_MMA_WAIT(bar, par) tc::mbar_wait_sleep(bar, par)
+#endif
+__device__ __forceinline__ constexpr bool attn_poly(int i) {
+  return FPS_ATTN_POLY > 0 && ((i >> 3) % (FPS_ATTN_POLY > 0 ? FPS_ATTN_POLY : 1)) == (FPS_ATTN_POLY > 0 ? FPS_ATTN_POLY : 1) - 1;
+}
+#ifdef FPS_ATTN_TRACE
+// developer instrumentation (separate build): per-step clock64 stamps of one CTA
+__device__ long long g_attn_trace[2][64][8];
+#define ATTN_TRACE(t, kt, slot)                                                     \
+  do {                                                                              \
+    if (blockIdx.x == 5 && blockIdx.y == 3 && (threadIdx.x & 31) == 0 && (kt) < 64) \
+      g_attn_trace[t][kt][slot] = clock64();                                        \
+  } while (0)
+#else
+#define ATTN_TRACE(t, kt, slot) do {} while (0)
+#endif
+template <int D>
+struct Attn3Cfg {
+  static constexpr int Q_BYTES = 128 * D * 2;
+  static constexpr int KV_TILE = 128 * D * 2;
+  static constexpr int SMEM = 2 * Q_BYTES + 4 * KV_TILE + 2 * 2 * 128 * 4 + 1024 + 256;
+  static constexpr int TMEM_COLS = 512;
+};
+
+template <int D>
+__global__ void __launch_bounds__(512, 1)
+    attn_tc3_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmKV,
+                    __nv_bfloat16* __restrict__ O, const int32_t* __restrict__ cu_q,
+                    const int32_t* __restrict__ cu_k, int n_req, int heads, float scale_log2) {
+  using Cfg = Attn3Cfg<D>;
+  constexpr int CHUNK = 128 * 128;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~uintptr_t(1023));
+  uint8_t* sQ = smem;                                       // [2 tiles][D/64 chunks]
+  uint8_t* sK = sQ + 2 * Cfg::Q_BYTES;                      // [2 stages][D/64 chunks]
+  uint8_t* sV = sK + 2 * Cfg::KV_TILE;
+  float* sScale = reinterpret_cast<float*>(sV + 2 * Cfg::KV_TILE);   // [tile][row]
+  float* sL = sScale + 2 * 128;                                      // [tile][row]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sL + 2 * 128);
+  uint64_t* bar_q = bars;
+  uint64_t* k_full = bars + 1;
+  uint64_t* k_empty = bars + 3;
+  uint64_t* v_full = bars + 5;
+  uint64_t* v_empty = bars + 7;
+  uint64_t* bar_s = bars + 9;       // [tile] S_t(j) in TMEM            (MMA commit)
+  uint64_t* bar_p = bars + 11;      // [tile] P_t(j) stored + O_t rescaled (4 softmax + 4 correction warps)
+  uint64_t* bar_stat = bars + 13;   // [tile] scale_t(j) in smem             (4 softmax warps)
+  uint64_t* bar_o = bars + 15;      // [tile] final PV_t done              (MMA commit)
+  uint64_t* bar_fin = bars + 17;    // [tile] row sum l in smem            (4 softmax warps)
+  uint64_t* bar_p2 = bars + 19;     // [tile] second half of P_t(j) stored (4 softmax warps)
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + 21);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int head = blockIdx.y;
+  const int H = heads * D;
+  int r = 0, qp = blockIdx.x, ntile = 0;
+  for (; r < n_req; ++r) {
+    ntile = (__ldg(cu_q + r + 1) - __ldg(cu_q + r) + 127) >> 7;
+    const int np = (ntile + 1) >> 1;
+    if (qp < np) break;
+    qp -= np;
+  }
+  const bool hasB = 2 * qp + 1 < ntile;
+  const int q_end = __ldg(cu_q + r + 1);
+  const int q0 = __ldg(cu_q + r) + qp * 256;
+  const int k0 = __ldg(cu_k + r);
+  const int Lr = __ldg(cu_k + r + 1) - k0;
+  const int nk = (Lr + 127) >> 7;
+
+  if (threadIdx.x == 0) {
+    tc::mbar_init(bar_q, 1);
+    for (int s = 0; s < 2; ++s) {
+      tc::mbar_init(&k_full[s], 1);
+      tc::mbar_init(&k_empty[s], 1);
+      tc::mbar_init(&v_full[s], 1);
+      tc::mbar_init(&v_empty[s], 1);
+      tc::mbar_init(&bar_s[s], 1);
+      tc::mbar_init(&bar_p[s], 8);
+      tc::mbar_init(&bar_stat[s], 4);
+      tc::mbar_init(&bar_o[s], 1);
+      tc::mbar_init(&bar_fin[s], 4);
+      tc::mbar_init(&bar_p2[s], 4);
+    }
+    tc::fence_mbar_init();
+  }
+  if (warp == 0 && lane == 0) {
+    tc::tma_prefetch_desc(&tmQ);
+    tc::tma_prefetch_desc(&tmKV);
+  }
+  if (warp == 2) tc::tmem_alloc<Cfg::TMEM_COLS>(tmem_holder);
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tmem = *tmem_holder;
+  pdl_trigger();
+  pdl_wait();
+
+  if (warp < 4) {
+    tc::regs_dec<56>();
+    if (warp == 0) {
+      if (lane == 0 && nk > 0) {
+        tc::mbar_expect_tx(bar_q, (hasB ? 2 : 1) * Cfg::Q_BYTES);
+        for (int t = 0; t < (hasB ? 2 : 1); ++t)
+#pragma unroll
+          for (int c = 0; c < D / 64; ++c)
+            tc::tma_load_2d(sQ + t * Cfg::Q_BYTES + c * CHUNK, &tmQ, bar_q, head * D + c * 64,
+                            q0 + t * 128);
+        for (int kt = 0; kt < nk; ++kt) {
+          const int st = kt & 1;
+          tc::mbar_wait_sleep(&k_empty[st], ((kt >> 1) & 1) ^ 1);
+          tc::mbar_expect_tx(&k_full[st], Cfg::KV_TILE);
+#pragma unroll
+          for (int c = 0; c < D / 64; ++c)
+            tc::tma_load_2d(sK + st * Cfg::KV_TILE + c * CHUNK, &tmKV, &k_full[st],
+                            head * D + c * 64, k0 + kt * 128);
+        }
+      }
+    } else if (warp == 3) {
+      if (lane == 0) {
+        for (int kt = 0; kt < nk; ++kt) {
+          const int st = kt & 1;
+          tc::mbar_wait_sleep(&v_empty[st], ((kt >> 1) & 1) ^ 1);
+          tc::mbar_expect_tx(&v_full[st], Cfg::KV_TILE);
+#pragma unroll
+          for (int c = 0; c < D / 64; ++c)
+            tc::tma_load_2d(sV + st * Cfg::KV_TILE + c * CHUNK, &tmKV, &v_full[st],
+                            H + head * D + c * 64, k0 + kt * 128);
+        }
+      }
+    } else if (warp == 1) {
+      // whole warp: operands stay warp-uniform, one elected lane issues (see mma_bf16_w).  The
+      // 512-column allocation is the whole TMEM, so its base is column 0 (a constant here).
+      if (nk > 0) {
+        constexpr uint32_t idesc_s = tc::idesc_bf16(128, 128);
+        constexpr uint32_t idesc_o = tc::idesc_bf16(128, D, /*b_mn_major=*/true);
+        tc::mbar_wait_sleep(bar_q, 0);
+        const uint64_t dq = tc::sdesc_k_sw128(tc::smem_u32(sQ));
+        const uint64_t dk = tc::sdesc_k_sw128(tc::smem_u32(sK));
+        const uint64_t dv = tc::sdesc_mn_sw128(tc::smem_u32(sV), CHUNK);
+        auto issue_s = [&](int t, int kt) {           // S_t = Q_t K_kt^T
+          const uint64_t a = dq + ((t * Cfg::Q_BYTES) >> 4);
+          const uint64_t b = dk + (((kt & 1) * Cfg::KV_TILE) >> 4);
+          if constexpr (D == 128) tc::mma_ss_k8_commit<CHUNK / 16, CHUNK / 16>(t * 128, a, b, idesc_s, &bar_s[t]);
+          else tc::mma_ss_k4_commit(t * 128, a, b, idesc_s, &bar_s[t]);
+        };
+        // O_t += P_t V_kt, P_t = TMEM cols [64,128): keys 0-63 as soon as the softmax has
+        // stored them (bar_p), keys 64-127 after the rest (bar_p2)
+        auto issue_pv = [&](int t, int kt) {
+          const uint64_t b = dv + (((kt & 1) * Cfg::KV_TILE) >> 4);
+          ATTN_MMA_WAIT(&bar_p[t], kt & 1);
+          tc::fence_after();
+          ATTN_TRACE(t, kt, 5);
+          tc::mma_ts_k4(256 + t * 128, t * 128 + 64, b, idesc_o, kt != 0);
+          ATTN_MMA_WAIT(&bar_p2[t], kt & 1);
+          tc::fence_after();
+          ATTN_TRACE(t, kt, 6);
+          tc::mma_ts_k4(256 + t * 128, t * 128 + 96, b + (4 * 2048 >> 4), idesc_o, 1);
+        };
+        tc::mbar_wait_sleep(&k_full[0], 0);
+        tc::fence_after();
+        issue_s(0, 0);
+        if (hasB) issue_s(1, 0);
+        tc::mma_commit_w(&k_empty[0]);
+        for (int kt = 0; kt < nk; ++kt) {
+          const bool more = kt + 1 < nk;
+          tc::mbar_wait_sleep(&v_full[kt & 1], (kt >> 1) & 1);
+          issue_pv(0, kt);
+          if (!more) tc::mma_commit_w(&bar_o[0]);
+          if (!hasB) tc::mma_commit_w(&v_empty[kt & 1]);
+          if (more) {
+            tc::mbar_wait_sleep(&k_full[(kt + 1) & 1], ((kt + 1) >> 1) & 1);
+            tc::fence_after();
+            issue_s(0, kt + 1);
+            if (!hasB) tc::mma_commit_w(&k_empty[(kt + 1) & 1]);
+          }
+          if (hasB) {
+            issue_pv(1, kt);
+            if (!more) tc::mma_commit_w(&bar_o[1]);
+            tc::mma_commit_w(&v_empty[kt & 1]);
+            if (more) {
+              issue_s(1, kt + 1);
+              tc::mma_commit_w(&k_empty[(kt + 1) & 1]);
+            }
+          }
+        }
+      }
+    }
+  } else if (warp < 12) {
+    // ---------------- softmax (warps 4-7: tile A, 8-11: tile B) ----------------
+    tc::regs_inc<192>();
+    const int t = (warp >= 8) ? 1 : 0;
+    if (t == 0 || hasB) {
+      const int q = warp & 3;
+      const int row = q * 32 + lane;
+      const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+      const uint32_t tS = tmem + t * 128;
+      float m_used = -INFINITY, l = 0.f;
+      for (int kt = 0; kt < nk; ++kt) {
+        tc::mbar_wait(&bar_s[t], kt & 1);
+        tc::fence_after();
+        ATTN_TRACE(t, kt, 0);
+        float s[128];
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+          tc::tmem_ld32(tS + lane_off + c * 32, reinterpret_cast<uint32_t*>(s + c * 32));
+        tc::tmem_wait_ld();
+        ATTN_TRACE(t, kt, 1);
+        const int valid = Lr - kt * 128;
+        if (valid < 128) {                                 // only the request's last key tile
+#pragma unroll
+          for (int i = 0; i < 128; ++i) s[i] = (i < valid) ? s[i] : -INFINITY;
+        }
+        float m4[4] = {s[0], s[1], s[2], s[3]};
+#pragma unroll
+        for (int i = 4; i < 124; i += 8)
+#pragma unroll
+          for (int j = 0; j < 4; ++j) m4[j] = tc::fmax3(m4[j], s[i + j], s[i + 4 + j]);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) m4[j] = fmaxf(m4[j], s[124 + j]);
+        const float mx = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) * scale_log2;
+        float factor = 1.0f;
+        if (mx > m_used + 8.0f) {                          // lazy rescale (threshold 2^8)
+          factor = tc::ex2(m_used - mx);
+          m_used = mx;
+        }
+        ATTN_TRACE(t, kt, 2);
+        sScale[t * 128 + row] = factor;
+        __syncwarp();
+        if (lane == 0) tc::mbar_arrive(&bar_stat[t]);
+        // exponentials (a quarter on the FMA pipe), packed to bf16 pairs and stored into the
+        // upper half of this tile's S columns 32 keys at a time
+        const float nm = -m_used;
+        float a8[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          uint32_t p[16];
+#pragma unroll
+          for (int i = c * 32; i < c * 32 + 32; i += 2) {
+            tc::ffma2(s[i], s[i + 1], s[i], s[i + 1], scale_log2, scale_log2, nm, nm);
+            if (attn_poly(i)) {
+              tc::ex2_poly2(s[i], s[i + 1]);
+            } else {
+              s[i] = tc::ex2(s[i]);
+              s[i + 1] = tc::ex2(s[i + 1]);
+            }
+            p[(i - c * 32) >> 1] = tc::pack_bf16x2_rn(s[i], s[i + 1]);
+          }
+          tc::tmem_st16(tS + lane_off + 64 + c * 16, p);
+          if (c & 1) {                                     // keys 0-63, then 64-127, released
+            tc::tmem_wait_st();
+            tc::fence_before();
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(c == 1 ? &bar_p[t] : &bar_p2[t]);
+            ATTN_TRACE(t, kt, 2 + (c >> 1) + 1);
+          }
+        }
+#pragma unroll
+        for (int i = 0; i < 128; i += 2) {
+          const int j = (i >> 1) & 3;
+          tc::fadd2(a8[2 * j], a8[2 * j + 1], a8[2 * j], a8[2 * j + 1], s[i], s[i + 1]);
+        }
+        l = l * factor + (((a8[0] + a8[1]) + (a8[2] + a8[3])) + ((a8[4] + a8[5]) + (a8[6] + a8[7])));
+      }
+      sL[t * 128 + row] = l;
+      __syncwarp();
+      if (lane == 0) tc::mbar_arrive(&bar_fin[t]);
+    }
+  } else {
+    // ---------------- correction + epilogue (warps 12-15) ----------------
+    tc::regs_dec<72>();
+    const int q = warp & 3;
+    const int row = q * 32 + lane;
+    const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+    const int ntl = hasB ? 2 : 1;
+    for (int kt = 0; kt < nk; ++kt) {
+      for (int t = 0; t < ntl; ++t) {
+        tc::mbar_wait(&bar_stat[t], kt & 1);
+        const float f = sScale[t * 128 + row];
+        if (kt > 0 && __any_sync(0xffffffffu, f != 1.0f)) {
+          // O_t(kt-1) is complete: softmax saw S_t(kt), issued after PV_t(kt-1)
+          tc::fence_after();
+          const uint32_t tO = tmem + 256 + t * 128 + lane_off;
+#pragma unroll 1
+          for (int c = 0; c < D / 32; ++c) {
+            uint32_t o[32];
+            tc::tmem_ld32(tO + c * 32, o);
+            tc::tmem_wait_ld();
+#pragma unroll
+            for (int e = 0; e < 32; e += 2) {
+              float x0 = __uint_as_float(o[e]), x1 = __uint_as_float(o[e + 1]);
+              tc::ffma2(x0, x1, x0, x1, f, f, 0.f, 0.f);
+              o[e] = __float_as_uint(x0);
+              o[e + 1] = __float_as_uint(x1);
+            }
+            tc::tmem_st32(tO + c * 32, o);
+          }
+          tc::tmem_wait_st();
+        }
+        tc::fence_before();
+        __syncwarp();
+        if (lane == 0) tc::mbar_arrive(&bar_p[t]);
+      }
+    }
+    for (int t = 0; t < ntl; ++t) {
+      const int grow = q0 + t * 128 + row;
+      __nv_bfloat16* orow = O + (size_t)grow * H + head * D;
+      if (nk == 0) {                                       // no keys: defined zero output
+        if (grow < q_end)
+          for (int c = 0; c < D; c += 8) *reinterpret_cast<uint4*>(orow + c) = make_uint4(0, 0, 0, 0);
+        continue;
+      }
+      tc::mbar_wait(&bar_fin[t], 0);
+      tc::mbar_wait(&bar_o[t], 0);
+      tc::fence_after();
+      const float l = sL[t * 128 + row];
+      const float inv = (l > 0.f) ? 1.0f / l : 0.f;
+      const uint32_t tO = tmem + 256 + t * 128 + lane_off;
+#pragma unroll 1
+      for (int c = 0; c < D / 32; ++c) {
+        uint32_t o[32];
+        tc::tmem_ld32(tO + c * 32, o);
+        tc::tmem_wait_ld();
+        if (grow < q_end) {
+#pragma unroll
+          for (int g = 0; g < 4; ++g) {
+            float f[8];
+#pragma unroll
+            for (int e = 0; e < 8; ++e) f[e] = __uint_as_float(o[g * 8 + e]) * inv;
+            *reinterpret_cast<uint4*>(orow + c * 32 + g * 8) = Vec16<__nv_bfloat16>::pack(f);
+          }
+        }
+      }
+    }
+  }
+  tc::fence_before();
+  __syncthreads();
+  if (warp == 2) {
+    tc::fence_after();
+    tc::tmem_dealloc<Cfg::TMEM_COLS>(tmem);
+  }
+}
+
+int g_attn_force = 0;   // tests: 1 = one-tile kernel, 2 = two-tile smem-P kernel, 3 = P-in-TMEM
 
 bool attention_tc_supported(int dtype, int head_dim) {
   return dtype == FPS_BF16 && (head_dim == 64 || head_dim == 128);
@@ -665,17 +1038,67 @@ static fps_status launch_d2(const void* q, const void* kv, void* o, int heads,
   return FPS_OK;
 }
 
+template <int D>
+static fps_status launch_d3(const void* q, const void* kv, void* o, int heads,
+                            const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
+                            const int32_t* h_cu_k, int n_req, cudaStream_t s) {
+  using Cfg = Attn3Cfg<D>;
+  const int H = heads * D;
+  int pairs = 0;
+  for (int r = 0; r < n_req; ++r) pairs += ((h_cu_q[r + 1] - h_cu_q[r] + 127) / 128 + 1) / 2;
+  if (pairs == 0) return FPS_OK;
+  CUtensorMap tq, tkv;
+  if (!make_tmap_2d_bf16(&tq, q, (uint64_t)h_cu_q[n_req], H, (uint64_t)H * 2, 64, 128))
+    return fail(FPS_ECUDA, "attention_tc3: Q tensor map");
+  if (!make_tmap_2d_bf16(&tkv, kv, (uint64_t)h_cu_k[n_req], 2 * H, (uint64_t)H * 4, 64, 128))
+    return fail(FPS_ECUDA, "attention_tc3: KV tensor map");
+  static bool attr = false;
+  if (!attr) {
+    FPS_CUDA_TRY(cudaFuncSetAttribute(attn_tc3_kernel<D>,
+                                      cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
+    attr = true;
+  }
+  const float scale_log2 = 1.4426950408889634f / sqrtf((float)D);
+  FPS_CUDA_TRY(launch_k(attn_tc3_kernel<D>, dim3(pairs, heads), dim3(512), Cfg::SMEM, s, tq, tkv,
+                        reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads,
+                        scale_log2));
+#ifdef FPS_ATTN_TRACE
+  {
+    static long long h[2][64][8];
+    cudaStreamSynchronize(s);
+    cudaMemcpyFromSymbol(h, g_attn_trace, sizeof(h));
+    const long long base = h[0][0][0];
+    for (int kt = 0; kt < 12; ++kt)
+      for (int t = 0; t < 2; ++t)
+        fprintf(stderr, "trace t%d kt%2d: S %7lld ld %5lld max %5lld Plo %5lld Phi %5lld | mmaPV %7lld %7lld\n", t, kt,
+                h[t][kt][0] - base, h[t][kt][1] - h[t][kt][0], h[t][kt][2] - h[t][kt][0],
+                h[t][kt][3] - h[t][kt][0], h[t][kt][4] - h[t][kt][0], h[t][kt][5] - base,
+                h[t][kt][6] - base);
+  }
+#endif
+  count_launch();
+  FPS_LAUNCH_CHECK();
+  return FPS_OK;
+}
+
 fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads, int head_dim,
                                const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
                                const int32_t* h_cu_k, int n_req, cudaStream_t s) {
   if (!h_cu_q || !h_cu_k) return fail(FPS_EINVAL, "attention_tc needs host cu_q / cu_k");
   if (!aligned16(q) || !aligned16(kv) || !aligned16(o))
     return fail(FPS_EINVAL, "attention_tc: unaligned operand");
-  // Measured on B200 once the producer / MMA warps sleep in try_wait instead of spinning:
-  // two tiles per CTA 576 vs 537 TFLOP/s (n = 1331), 892 vs 880 (16 x 1800 rows), and a 3.4%
-  // faster HBM-tier step (25.15 vs 26.03 ms); the pinned-host step is unchanged (43.4 vs 43.6).
-  const bool two = g_attn_force != 1;
-  if (two) {
+  // Default: P in TMEM + correction warpgroup (attn_tc3).  Measured on B200 (tools/attn_probe.py,
+  // TFLOP/s at 16 x 1800 / 4 x 4608 query rows over 4608 keys): 1085 / 1200 vs 930 / 1004 for the
+  // smem-P two-tile kernel and ~800 / 900 for the one-tile kernel.  A 64-key-step variant with S
+  // double-buffered per tile (no S -> softmax -> PV -> S chain) measured 1113 at best: M=128 N=64
+  // SS MMAs run at 66% of the tensor rate (48.6 instead of 32 cycles each, tools/micro/mma_rate:
+  // A+B operand reads exceed the 128 B/clk smem port), which ate the latency it saved.
+  if (g_attn_force == 0 || g_attn_force == 3) {
+    if (head_dim == 128)
+      return launch_d3<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);
+    return launch_d3<64>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);
+  }
+  if (g_attn_force == 2) {
     if (head_dim == 128)
       return launch_d2<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);
     return launch_d2<64>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);

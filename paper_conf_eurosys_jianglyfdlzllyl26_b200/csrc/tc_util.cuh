@@ -184,6 +184,142 @@ __device__ __forceinline__ void mma_bf16_ts(uint32_t tmem_d, uint32_t tmem_a, ui
       "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem_d),
       "r"(tmem_a), "l"(bdesc), "r"(idesc), "r"(accumulate));
 }
+// Warp-wide variants: executed by all 32 lanes with warp-uniform operands, one lane elected inside
+// the asm issues.  Keeps the operands in uniform registers (no per-MMA R2UR / waterfall loop that
+// a single-lane branch costs), which matters for the 64-cycle 128x128x16 MMAs of the attention.
+__device__ __forceinline__ void mma_bf16_w(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc,
+                                          uint32_t idesc, uint32_t accumulate) {
+  asm volatile(
+      "{\n.reg .pred p, e;\nelect.sync _|e, 0xffffffff;\nsetp.ne.b32 p, %4, 0;\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate));
+}
+__device__ __forceinline__ void mma_bf16_ts_w(uint32_t tmem_d, uint32_t tmem_a, uint64_t bdesc,
+                                              uint32_t idesc, uint32_t accumulate) {
+  asm volatile(
+      "{\n.reg .pred p, e;\nelect.sync _|e, 0xffffffff;\nsetp.ne.b32 p, %4, 0;\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem_d),
+      "r"(tmem_a), "l"(bdesc), "r"(idesc), "r"(accumulate));
+}
+__device__ __forceinline__ void mma_commit_w(uint64_t* bar) {
+  asm volatile(
+      "{\n.reg .pred e;\nelect.sync _|e, 0xffffffff;\n"
+      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n}\n" ::"r"(
+          smem_u32(bar))
+      : "memory");
+}
+// Whole MMA groups in one asm block (one elect.sync per group, descriptor low words advanced with
+// 32-bit immediates): the per-MMA wrapper above still cost ~20 SASS instructions per 64-cycle
+// MMA (collective elect + R2UR of every operand), which made the attention's MMA warp the
+// bottleneck.  Descriptor addresses stay below 2^14 (smem < 256 KB) so the low-word adds never
+// carry into the high word.
+// SS group, K-major SW128 A and B, 8 x K=16 (d = 128): k-steps 0-3 advance 32 B inside the 128 B
+// swizzle row, k-steps 4-7 start at the next 64-column chunk (A_CH / B_CH, in 16-B units).
+// Commits the group to `bar`.
+template <int A_CH, int B_CH>
+__device__ __forceinline__ void mma_ss_k8_commit(uint32_t d, uint64_t adesc, uint64_t bdesc,
+                                                 uint32_t idesc, uint64_t* bar) {
+  const uint32_t alo = (uint32_t)adesc, ahi = (uint32_t)(adesc >> 32);
+  const uint32_t blo = (uint32_t)bdesc, bhi = (uint32_t)(bdesc >> 32);
+  asm volatile(
+      "{\n.reg .pred e;\n.reg .b32 al, bl;\n.reg .b64 ad, bd;\n"
+      "elect.sync _|e, 0xffffffff;\n"
+      "mov.b64 ad, {%1, %2};\nmov.b64 bd, {%3, %4};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], ad, bd, %5, 0;\n"
+      "add.s32 al, %1, 2;\nadd.s32 bl, %3, 2;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "add.s32 al, %1, 4;\nadd.s32 bl, %3, 4;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "add.s32 al, %1, 6;\nadd.s32 bl, %3, 6;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "add.s32 al, %1, %7;\nadd.s32 bl, %3, %8;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "add.s32 al, al, 2;\nadd.s32 bl, bl, 2;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "add.s32 al, al, 2;\nadd.s32 bl, bl, 2;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "add.s32 al, al, 2;\nadd.s32 bl, bl, 2;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%6];\n"
+      "}\n" ::"r"(d),
+      "r"(alo), "r"(ahi), "r"(blo), "r"(bhi), "r"(idesc), "r"(smem_u32(bar)), "n"(A_CH), "n"(B_CH)
+      : "memory");
+}
+// SS group with 4 x K=16 (d = 64): one 64-column chunk.
+__device__ __forceinline__ void mma_ss_k4_commit(uint32_t d, uint64_t adesc, uint64_t bdesc,
+                                                 uint32_t idesc, uint64_t* bar) {
+  const uint32_t alo = (uint32_t)adesc, ahi = (uint32_t)(adesc >> 32);
+  const uint32_t blo = (uint32_t)bdesc, bhi = (uint32_t)(bdesc >> 32);
+  asm volatile(
+      "{\n.reg .pred e;\n.reg .b32 al, bl;\n.reg .b64 ad, bd;\n"
+      "elect.sync _|e, 0xffffffff;\n"
+      "mov.b64 ad, {%1, %2};\nmov.b64 bd, {%3, %4};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], ad, bd, %5, 0;\n"
+      "add.s32 al, %1, 2;\nadd.s32 bl, %3, 2;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "add.s32 al, %1, 4;\nadd.s32 bl, %3, 4;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "add.s32 al, %1, 6;\nadd.s32 bl, %3, 6;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%6];\n"
+      "}\n" ::"r"(d),
+      "r"(alo), "r"(ahi), "r"(blo), "r"(bhi), "r"(idesc), "r"(smem_u32(bar))
+      : "memory");
+}
+// TS group (A = P from TMEM, 8 columns per K=16 step; B = V MN-major, 2048 B per 16 keys),
+// 4 steps (64 keys); `acc` = 0 only for the first group of the output.
+__device__ __forceinline__ void mma_ts_k4(uint32_t d, uint32_t a_tmem, uint64_t bdesc,
+                                          uint32_t idesc, uint32_t acc) {
+  const uint32_t blo = (uint32_t)bdesc, bhi = (uint32_t)(bdesc >> 32);
+  asm volatile(
+      "{\n.reg .pred e, p;\n.reg .b32 ta, bl;\n.reg .b64 bd;\n"
+      "elect.sync _|e, 0xffffffff;\n"
+      "setp.ne.b32 p, %5, 0;\n"
+      "mov.b64 bd, {%2, %3};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], bd, %4, p;\n"
+      "add.s32 ta, %1, 8;\nadd.s32 bl, %2, 128;\nmov.b64 bd, {bl, %3};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ta], bd, %4, 1;\n"
+      "add.s32 ta, %1, 16;\nadd.s32 bl, %2, 256;\nmov.b64 bd, {bl, %3};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ta], bd, %4, 1;\n"
+      "add.s32 ta, %1, 24;\nadd.s32 bl, %2, 384;\nmov.b64 bd, {bl, %3};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ta], bd, %4, 1;\n"
+      "}\n" ::"r"(d),
+      "r"(a_tmem), "r"(blo), "r"(bhi), "r"(idesc), "r"(acc)
+      : "memory");
+}
+__device__ __forceinline__ void mma_ts_k4_commit(uint32_t d, uint32_t a_tmem, uint64_t bdesc,
+                                                 uint32_t idesc, uint32_t acc, uint64_t* bar) {
+  mma_ts_k4(d, a_tmem, bdesc, idesc, acc);
+  mma_commit_w(bar);
+}
+// TS group, 8 steps (128 keys), no commit (callers commit once per tile).
+__device__ __forceinline__ void mma_ts_k8(uint32_t d, uint32_t a_tmem, uint64_t bdesc,
+                                          uint32_t idesc, uint32_t acc) {
+  const uint32_t blo = (uint32_t)bdesc, bhi = (uint32_t)(bdesc >> 32);
+  asm volatile(
+      "{\n.reg .pred e, p;\n.reg .b32 ta, bl;\n.reg .b64 bd;\n"
+      "elect.sync _|e, 0xffffffff;\n"
+      "setp.ne.b32 p, %5, 0;\n"
+      "mov.b64 bd, {%2, %3};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], bd, %4, p;\n"
+      "add.s32 ta, %1, 8;\nadd.s32 bl, %2, 128;\nmov.b64 bd, {bl, %3};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ta], bd, %4, 1;\n"
+      "add.s32 ta, %1, 16;\nadd.s32 bl, %2, 256;\nmov.b64 bd, {bl, %3};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ta], bd, %4, 1;\n"
+      "add.s32 ta, %1, 24;\nadd.s32 bl, %2, 384;\nmov.b64 bd, {bl, %3};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ta], bd, %4, 1;\n"
+      "add.s32 ta, %1, 32;\nadd.s32 bl, %2, 512;\nmov.b64 bd, {bl, %3};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ta], bd, %4, 1;\n"
+      "add.s32 ta, %1, 40;\nadd.s32 bl, %2, 640;\nmov.b64 bd, {bl, %3};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ta], bd, %4, 1;\n"
+      "add.s32 ta, %1, 48;\nadd.s32 bl, %2, 768;\nmov.b64 bd, {bl, %3};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ta], bd, %4, 1;\n"
+      "add.s32 ta, %1, 56;\nadd.s32 bl, %2, 896;\nmov.b64 bd, {bl, %3};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ta], bd, %4, 1;\n"
+      "}\n" ::"r"(d),
+      "r"(a_tmem), "r"(blo), "r"(bhi), "r"(idesc), "r"(acc)
+      : "memory");
+}
 __device__ __forceinline__ void mma_commit(uint64_t* bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
                    smem_u32(bar))
@@ -264,9 +400,10 @@ __device__ __forceinline__ void fadd2(float& d0, float& d1, float a0, float a1, 
       : "f"(a0), "f"(a1), "f"(b0), "f"(b1));
 }
 // 2^x for a pair on the FMA pipe (offloads the MUFU unit, FA4-style): x = n + f, n = round(x),
-// f in [-0.5, 0.5], 2^f by a degree-5 polynomial (Taylor in ln 2, rel. error < 3e-6), then n is
-// added to the exponent field.  x is clamped to >= -126 (results below 2^-126 flush towards 0;
-// they are far below bf16 P resolution relative to the row max, which is >= 1).
+// f in [-0.5, 0.5], 2^f by a degree-3 polynomial fitted for relative error on [-0.5, 0.5]
+// (max 7.5e-5, far below the 2^-9 rounding of the bf16 P it feeds), then n is added to the
+// exponent field.  x is clamped to >= -126 (results below 2^-126 flush towards 0; they are far
+// below bf16 P resolution relative to the row max, which is >= 1).
 __device__ __forceinline__ void ex2_poly2(float& x0, float& x1) {
   const float magic = 12582912.0f;                          // 1.5 * 2^23: round-to-nearest trick
   x0 = fmaxf(x0, -126.0f);
@@ -275,14 +412,32 @@ __device__ __forceinline__ void ex2_poly2(float& x0, float& x1) {
   fadd2(r0, r1, x0, x1, magic, magic);
   fadd2(n0, n1, r0, r1, -magic, -magic);
   fadd2(f0, f1, x0, x1, -n0, -n1);
-  float p0 = 1.3333558e-3f, p1 = 1.3333558e-3f;
-  ffma2(p0, p1, p0, p1, f0, f1, 9.6181291e-3f, 9.6181291e-3f);
-  ffma2(p0, p1, p0, p1, f0, f1, 5.5504109e-2f, 5.5504109e-2f);
-  ffma2(p0, p1, p0, p1, f0, f1, 2.4022651e-1f, 2.4022651e-1f);
-  ffma2(p0, p1, p0, p1, f0, f1, 6.9314718e-1f, 6.9314718e-1f);
-  ffma2(p0, p1, p0, p1, f0, f1, 1.0f, 1.0f);
+  float p0 = 5.5171650e-2f, p1 = 5.5171650e-2f;
+  ffma2(p0, p1, p0, p1, f0, f1, 2.4261113e-1f, 2.4261113e-1f);
+  ffma2(p0, p1, p0, p1, f0, f1, 6.9326097e-1f, 6.9326097e-1f);
+  ffma2(p0, p1, p0, p1, f0, f1, 9.9992806e-1f, 9.9992806e-1f);
   x0 = __int_as_float(__float_as_int(p0) + (__float_as_int(r0) << 23));
   x1 = __int_as_float(__float_as_int(p1) + (__float_as_int(r1) << 23));
+}
+// three-input max (one FMNMX3 on sm_100)
+__device__ __forceinline__ float fmax3(float a, float b, float c) {
+  float r;
+  asm("max.f32 %0, %1, %2, %3;" : "=f"(r) : "f"(a), "f"(b), "f"(c));
+  return r;
+}
+// per-warpgroup register budget (all four warps of a warpgroup execute the same one)
+template <int N>
+__device__ __forceinline__ void regs_inc() {
+  asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(N));
+}
+template <int N>
+__device__ __forceinline__ void regs_dec() {
+  asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(N));
+}
+__device__ __forceinline__ uint32_t pack_bf16x2_rn(float lo, float hi) {
+  uint32_t r;
+  asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
+  return r;
 }
 __device__ __forceinline__ float ex2(float x) {
   float y;

@@ -19,7 +19,7 @@ def F():
     return fps
 
 
-KERNEL_FLAGS = {"auto": 0, "two_tile": 32, "one_tile": 16, "simt": 2}
+KERNEL_FLAGS = {"auto": 0, "p_tmem": 48, "two_tile": 32, "one_tile": 16, "simt": 2}
 
 
 @pytest.mark.parametrize("d,heads", [(128, 3), (64, 4)])
@@ -47,7 +47,8 @@ def test_varlen_attention(F, d, heads, kernel):
         ko += l
 
 
-def test_attention_large_logits_lazy_rescale(F):
+@pytest.mark.parametrize("kernel", ["auto", "p_tmem", "two_tile", "one_tile"])
+def test_attention_large_logits_lazy_rescale(F, kernel):
     """Keys whose scores grow along the sequence force the lazy-max rescale of O in TMEM."""
     g = synth.rng(5)
     heads, d = 2, 128
@@ -57,6 +58,13 @@ def test_attention_large_logits_lazy_rescale(F):
     k = synth.bf16_round(np.linspace(-4, 4, L, dtype=np.float32)[:, None] * np.ones((1, H), np.float32))
     v = synth.latent(g, L, H, "bf16")
     kv = np.concatenate([k, v], 1)
-    out = F.masked_attention(to_dev(q, "bf16"), to_dev(kv, "bf16"), [n], [L], heads)
-    torch.cuda.synchronize()
-    check_close(to_np(out), attention(q, k, v, heads), TOL["bf16"], "rescale")
+    F.fps_set_disable_tc(KERNEL_FLAGS[kernel])
+    try:
+        q2 = np.concatenate([q, q], 0)                      # 256 query rows: both tiles of a pair
+        out = F.masked_attention(to_dev(q2, "bf16"), to_dev(kv, "bf16"), [2 * n], [L], heads)
+        torch.cuda.synchronize()
+    finally:
+        F.fps_set_disable_tc(0)
+    ref = attention(q, k, v, heads)
+    check_close(to_np(out)[:n], ref, TOL["bf16"], "rescale")
+    check_close(to_np(out)[n:], ref, TOL["bf16"], "rescale (second tile of the pair)")
