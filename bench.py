@@ -223,8 +223,19 @@ def calibrate(F, w, mode, layers, cache, reqs, device):
     whole = cache.desc.copy_method == 2
     for k, m in enumerate((0.05, 0.3, 0.6, 0.9)):
         u = w["L_img"] - synth.n_masked_for(m, w["L_img"])
-        rows = torch.arange(u, device=device, dtype=torch.int32)
-        h_rows = np.arange(u, dtype=np.int32)
+        # unmasked rows with the run structure of a blob mask: the masked rows form chunks of
+        # ~28 consecutive tokens spread over the grid (one per image row the blob crosses)
+        nm = w["L_img"] - u
+        keep = np.ones(w["L_img"], bool)
+        n_chunks = max(1, nm // 28)
+        starts = np.linspace(0, w["L_img"] - 28, n_chunks).astype(int)
+        for c0 in starts:
+            keep[c0:c0 + 28] = False
+        drop = np.flatnonzero(keep)[:max(0, keep.sum() - u)]   # exact count u
+        keep[drop] = False
+        h_rows = np.flatnonzero(keep).astype(np.int32)
+        u = len(h_rows)
+        rows = torch.as_tensor(h_rows, device=device)
         items = [F.fps_prefetch_item(i, 0, 0, u, rows.data_ptr(), h_rows.ctypes.data,
                                      dst[i * L].data_ptr(), W * 2) for i in range(B)]
         if whole:                 # whole-entry DMA: bytes do not depend on u; vary the count
@@ -324,17 +335,19 @@ def main():
                     help="template cache in pinned host DRAM (configs[2]) or HBM (NEXT-1)")
     ap.add_argument("--copy-ctas", type=int, default=0, help="CTAs of the SM row gather (0 = lib default)")
     ap.add_argument("--copy-method", type=int, default=None, choices=[0, 1, 2],
-                    help="H2D method: 0 SM zero-copy row gather, 1 DMA per row run")
+                    help="H2D method: 0 SM zero-copy row gather, 1 batched DMA of the unmasked row "
+                         "runs (host default), 2 whole-entry DMA (HBM default)")
     ap.add_argument("--no-extras", action="store_true", help="skip dense / Y-mode / profile legs")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()
     import faulthandler                   # a stuck run dumps every thread's stack and exits
     faulthandler.dump_traceback_later(900, exit=True)
-    if args.copy_method is None:          # HBM tier: whole-entry DMA (no SM time); host: gather
-        # measured on B200 (C3) with the planner's load model counting whole entries: KV-mode
-        # host 38.1 ms with whole-entry DMA vs 43.3 with the SM row gather (no SM interference
-        # outweighs +25% bytes), Y-mode host 30.8 vs 36.4, HBM tier 23.0 vs 24.4
-        args.copy_method = 2
+    if args.copy_method is None:
+        # measured on B200 (C3): pinned host tier -- batched DMA of the unmasked row runs 32.8
+        # ms/step vs 36.7 with whole-entry DMA (-20% bytes at the same 55 GB/s) and 43.3 with the
+        # SM row gather (SM interference); HBM tier -- whole-entry DMA 21.6 vs 44.4 for the run
+        # batch (device-to-device run copies reach only ~145 GB/s on the copy engine)
+        args.copy_method = 2 if args.tier == "hbm" else 1
 
     rank = int(os.environ.get("RANK", 0))
     world = int(os.environ.get("WORLD_SIZE", 1))
@@ -357,7 +370,7 @@ def main():
                    if args.config == "C3" else f"masked-block stack images/s ({args.config})")
     base_cfg["cache_tier"] = {"host": "pinned host DRAM", "hbm": "device HBM (NEXT-1)",
                               "host_hugepage": "pinned host DRAM on 2 MiB pages"}[args.tier]
-    base_cfg["h2d_method"] = ["SM row gather", "DMA per row run", "DMA of whole entries"][args.copy_method]
+    base_cfg["h2d_method"] = ["SM row gather", "batched DMA of the unmasked row runs", "DMA of whole entries"][args.copy_method]
     base_cfg["parallelism"] = f"request-parallel x{world} (Alg. 2 routing)"
 
     if args.impl == "reference":
@@ -405,7 +418,7 @@ def main():
     layers, mod, cache = build_engine_inputs(F, w, args.mode, device, n_entries, location,
                                              args.copy_method)
     base_cfg["cache_tier"] = "pinned host DRAM" if location == 0 else "device HBM (NEXT-1)"
-    base_cfg["h2d_method"] = ["SM row gather", "DMA per row run", "DMA of whole entries"][args.copy_method]
+    base_cfg["h2d_method"] = ["SM row gather", "batched DMA of the unmasked row runs", "DMA of whole entries"][args.copy_method]
     torch.cuda.synchronize()
     log(f"[rank {rank}] inputs ready in {time.perf_counter() - t0:.1f}s")
     my_pool = pool[:w["batch"]]
@@ -466,10 +479,11 @@ def main():
         # the other caching mode, and both modes with the other cache tier, on the same batch
         other = "y" if args.mode == "kv" else "kv"
         other_loc = 0 if location == 1 else 1
-        other_cm = 2 if other_loc == 1 else 0
+        default_cm = lambda loc: 2 if loc == 1 else 1
+        other_cm = default_cm(other_loc)
         for md, loc, cmeth in ((other, location, args.copy_method),
                                (args.mode, other_loc, other_cm), (other, other_loc, other_cm),
-                               (args.mode, location, 1 if args.copy_method != 1 else 0)):
+                               (args.mode, location, 2 if args.copy_method != 2 else 1)):
             if loc == 1 and cmeth == 1:
                 continue
             c2 = make_cache(F, w, md, n_entries, loc, cmeth)
@@ -479,7 +493,9 @@ def main():
                              mod_table=mod, slots=0, plan_policy=0,
                              cost_model=cm2.as_engine_model())
             o_ms, _ = run_engine_timed(F, eng_o, reqs_dev, K, W, stream, load_stream, rank, world)
-            tag = f"{md}_mode_{['host', 'hbm', 'host_hugepage'][loc]}" + ("_dma" if cmeth == 1 else "")
+            tag = f"{md}_mode_{['host', 'hbm', 'host_hugepage'][loc]}"
+            if cmeth != default_cm(loc):
+                tag += "_" + ["row_gather", "run_dma", "whole_entry_dma"][cmeth]
             extras[f"{tag}_ms_per_step"] = o_ms
             extras[f"{tag}_cached_blocks"] = int(sum(eng_o.last_plan()[0]))
             del eng_o

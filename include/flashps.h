@@ -113,7 +113,11 @@ typedef struct {
                             moved are identical, contents alias)                            */
   int32_t copy_method;   /* 0 = SM row gather (zero-copy over mapped pinned memory, or from
                                 the HBM arena) -- exactly the rows U (default);
-                            1 = copy-engine DMA of coalesced row runs of U;
+                            1 = copy-engine DMA of exactly the rows U: their runs of
+                                consecutive tokens go out as one cudaMemcpyBatchAsync per call
+                                (one cudaMemcpyAsync per run on the legacy default stream).
+                                Full link rate on only the unmasked bytes: the pinned-host
+                                default of the bench;
                             2 = copy-engine DMA of the WHOLE entry (all L_img rows, one copy
                                 per request): no SM time, but rows outside U are overwritten
                                 too, so fresh K/V must be written only after `ready_event`

@@ -164,8 +164,24 @@ def test_pipeline_slots_and_copy_methods_bit_identical(F, slots, method, locatio
         assert torch.equal(a.view(torch.int16), b.view(torch.int16))
 
 
+@pytest.mark.parametrize("mode,slots", [("kv", 2), ("y", 2), ("kv", 1)])
+def test_batched_run_dma_bit_identical(F, mode, slots):
+    """copy_method 1 on a real load stream goes through one cudaMemcpyBatchAsync per prefetch
+    (exact unmasked rows); with a shallow staging ring the slot reuse must still be ordered."""
+    outs = []
+    for me, use_ls in ((0, False), (1, True)):
+        _, _, _, _, eng, reqs = _setup(F, mode, "bf16", 1, slots=slots if me else 0,
+                                       copy_method=me, seed=5150)
+        ls = torch.cuda.Stream() if use_ls else None
+        eng.run_batch(reqs, 2, load_stream=ls)
+        torch.cuda.synchronize()
+        outs.append([r["x"].clone() for r in reqs])
+    for a, b in zip(*outs):
+        assert torch.equal(a.view(torch.int16), b.view(torch.int16))
+
+
 @pytest.mark.parametrize("mode,method,location", [("y", 0, 0), ("kv", 0, 0), ("kv", 2, 1),
-                                                  ("y", 2, 1)])
+                                                  ("y", 2, 1), ("kv", 1, 0), ("y", 1, 0)])
 def test_delayed_load_stream_bit_identical(F, mode, method, location):
     """Robustness of the event ordering: a busy load stream (a long spin queued before the
     prefetches) must not change the result -- in particular a late whole-entry DMA (method 2)
