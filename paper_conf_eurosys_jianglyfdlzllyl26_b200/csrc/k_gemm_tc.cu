@@ -38,74 +38,100 @@ __device__ __forceinline__ void tile_coords(int tile, int num_m, int num_n, int&
   n_blk = local / gm;
 }
 
+// Per-row epilogue context: gate vector of the row's request and the output rows of both
+// column ranges (K/V scatter into the merged key buffer).
+struct RowCtx {
+  const __nv_bfloat16* gate;
+  int orow0, orow1;
+  bool ok;
+};
+__device__ __forceinline__ RowCtx row_ctx(const Epilogue& ep, int M, int row) {
+  RowCtx c{nullptr, row, row, row < M};
+  if (c.ok) {
+    if (ep.gate)
+      c.gate = reinterpret_cast<const __nv_bfloat16*>(ep.gate) +
+               (size_t)find_req(ep.cu, ep.n_req, row) * ep.gate_stride;
+    if (ep.map0) c.orow0 = __ldg(ep.map0 + row);
+    if (ep.map1) c.orow1 = __ldg(ep.map1 + row);
+  }
+  return c;
+}
+
+// Global loads of the fused operands of 32 columns col0.. of one row (issued before use).
+struct ChunkIn {
+  uint4 bv[4], rv[4], gv[4];
+};
+__device__ __forceinline__ void chunk_load(const Epilogue& ep, const RowCtx& rc, int N, int row,
+                                           int col0, ChunkIn& in) {
+  const __nv_bfloat16* __restrict__ bias = reinterpret_cast<const __nv_bfloat16*>(ep.bias);
+  const __nv_bfloat16* __restrict__ resid = reinterpret_cast<const __nv_bfloat16*>(ep.resid);
+#pragma unroll
+  for (int g = 0; g < 4; ++g) {
+    const int c0 = col0 + g * 8;
+    const bool ok = rc.ok && c0 < N;
+    in.bv[g] = (bias && ok) ? __ldg(reinterpret_cast<const uint4*>(bias + c0)) : make_uint4(0, 0, 0, 0);
+    in.rv[g] = (resid && ok)
+                   ? __ldg(reinterpret_cast<const uint4*>(resid + (size_t)row * ep.ld_resid + c0))
+                   : make_uint4(0, 0, 0, 0);
+    in.gv[g] = (rc.gate && ok) ? __ldg(reinterpret_cast<const uint4*>(rc.gate + c0))
+                               : make_uint4(0, 0, 0, 0);
+  }
+}
+
+// Fused ops + 16-B stores of 32 accumulator values (fp32 bits) of one row, columns col0..
+__device__ __forceinline__ void chunk_store(const Epilogue& ep, const RowCtx& rc, int N, int col0,
+                                            const uint32_t* r, const ChunkIn& in) {
+  if (!rc.ok) return;
+#pragma unroll
+  for (int g = 0; g < 4; ++g) {
+    const int c0 = col0 + g * 8;
+    if (c0 >= N) continue;
+    float v[8], t[8];
+#pragma unroll
+    for (int e = 0; e < 8; ++e) v[e] = __uint_as_float(r[g * 8 + e]);
+    if (ep.bias) {
+      Vec16<__nv_bfloat16>::unpack(in.bv[g], t);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) v[e] += t[e];
+    }
+    if (ep.act == 1) {
+#pragma unroll
+      for (int e = 0; e < 8; ++e) v[e] = gelu_tanh_fast(v[e]);
+    }
+    if (ep.resid) {
+      float rr[8];
+      Vec16<__nv_bfloat16>::unpack(in.rv[g], rr);
+      if (rc.gate) {
+        Vec16<__nv_bfloat16>::unpack(in.gv[g], t);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) v[e] = rr[e] + t[e] * v[e];
+      } else {
+#pragma unroll
+        for (int e = 0; e < 8; ++e) v[e] = rr[e] + v[e];
+      }
+    }
+    __nv_bfloat16* dst =
+        c0 < ep.split ? reinterpret_cast<__nv_bfloat16*>(ep.out0) + (size_t)rc.orow0 * ep.ld0 + c0
+                      : reinterpret_cast<__nv_bfloat16*>(ep.out1) + (size_t)rc.orow1 * ep.ld1 +
+                            (c0 - ep.split);
+    *reinterpret_cast<uint4*>(dst) = Vec16<__nv_bfloat16>::pack(v);
+  }
+}
+
 // Epilogue of one accumulator tile for the calling thread's output row (thread = TMEM lane).
 template <int BN>
 __device__ __forceinline__ void epilogue_tile(const Epilogue& ep, int M, int N, int row,
                                               int col_base, uint32_t taddr) {
-  const __nv_bfloat16* __restrict__ bias = reinterpret_cast<const __nv_bfloat16*>(ep.bias);
-  const __nv_bfloat16* __restrict__ resid = reinterpret_cast<const __nv_bfloat16*>(ep.resid);
-  const bool row_ok = row < M;
-  const __nv_bfloat16* gate = nullptr;
-  int orow0 = row, orow1 = row;
-  if (row_ok) {
-    if (ep.gate)
-      gate = reinterpret_cast<const __nv_bfloat16*>(ep.gate) +
-             (size_t)find_req(ep.cu, ep.n_req, row) * ep.gate_stride;
-    if (ep.map0) orow0 = __ldg(ep.map0 + row);
-    if (ep.map1) orow1 = __ldg(ep.map1 + row);
-  }
+  const RowCtx rc = row_ctx(ep, M, row);
 #pragma unroll 1
   for (int c = 0; c < BN / 32; ++c) {
     uint32_t r[32];
     tc::tmem_ld32(taddr + c * 32, r);
     const int col0 = col_base + c * 32;
-    uint4 bv[4], rv[4], gv[4];
-#pragma unroll
-    for (int g = 0; g < 4; ++g) {
-      const int c0 = col0 + g * 8;
-      const bool ok = row_ok && c0 < N;
-      bv[g] = (bias && ok) ? __ldg(reinterpret_cast<const uint4*>(bias + c0)) : make_uint4(0, 0, 0, 0);
-      rv[g] = (resid && ok)
-                  ? __ldg(reinterpret_cast<const uint4*>(resid + (size_t)row * ep.ld_resid + c0))
-                  : make_uint4(0, 0, 0, 0);
-      gv[g] = (gate && ok) ? __ldg(reinterpret_cast<const uint4*>(gate + c0)) : make_uint4(0, 0, 0, 0);
-    }
+    ChunkIn in;
+    chunk_load(ep, rc, N, row, col0, in);
     tc::tmem_wait_ld();
-    if (!row_ok) continue;
-#pragma unroll
-    for (int g = 0; g < 4; ++g) {
-      const int c0 = col0 + g * 8;
-      if (c0 >= N) continue;
-      float v[8], t[8];
-#pragma unroll
-      for (int e = 0; e < 8; ++e) v[e] = __uint_as_float(r[g * 8 + e]);
-      if (bias) {
-        Vec16<__nv_bfloat16>::unpack(bv[g], t);
-#pragma unroll
-        for (int e = 0; e < 8; ++e) v[e] += t[e];
-      }
-      if (ep.act == 1) {
-#pragma unroll
-        for (int e = 0; e < 8; ++e) v[e] = gelu_tanh_fast(v[e]);
-      }
-      if (resid) {
-        float rr[8];
-        Vec16<__nv_bfloat16>::unpack(rv[g], rr);
-        if (gate) {
-          Vec16<__nv_bfloat16>::unpack(gv[g], t);
-#pragma unroll
-          for (int e = 0; e < 8; ++e) v[e] = rr[e] + t[e] * v[e];
-        } else {
-#pragma unroll
-          for (int e = 0; e < 8; ++e) v[e] = rr[e] + v[e];
-        }
-      }
-      __nv_bfloat16* dst =
-          c0 < ep.split ? reinterpret_cast<__nv_bfloat16*>(ep.out0) + (size_t)orow0 * ep.ld0 + c0
-                        : reinterpret_cast<__nv_bfloat16*>(ep.out1) + (size_t)orow1 * ep.ld1 +
-                              (c0 - ep.split);
-      *reinterpret_cast<uint4*>(dst) = Vec16<__nv_bfloat16>::pack(v);
-    }
+    chunk_store(ep, rc, N, col0, r, in);
   }
 }
 
@@ -375,6 +401,178 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
 }
 
 // ============================================================================================
+// CTA-pair kernel, operands swapped (C^T = B . A^T): the MMA's M=256 side walks the weight rows
+// (N of the GEMM, a multiple of 256 at every block shape) and its N side walks the activation
+// rows in blocks of NA (runtime, multiple of 16, <= 256).  For the active-row counts of masked
+// blocks this removes the M padding of 256-row tiles (M = 1331: 6 x 224 = 1344 rows instead of
+// 6 x 256 = 1536, -12.5% tensor work at the same number of waves).  Each CTA loads its 128
+// weight rows and NA/2 activation rows per k-step; the accumulator holds D[n][m] (TMEM lane =
+// output column), so the epilogue warps transpose 32 x 32 chunks through shared memory and then
+// run the same per-row fused epilogue (thread = output row, 16-B stores) as the other kernels.
+template <int STAGES>
+struct Gemm2sCfg {
+  static constexpr int BK = 64;
+  static constexpr int A_BYTES = 128 * BK * 2;             // per CTA: 128 weight rows
+  static constexpr int B_BYTES = 128 * BK * 2;             // per CTA: up to 128 activation rows
+  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr int TMEM_COLS = 512;                    // 2 accumulators x up to 256 columns
+  static constexpr int XPOSE_BYTES = 4 * 32 * 33 * 4;      // per epilogue warp: 32 x 33 floats
+  static constexpr int SMEM = STAGES * STAGE_BYTES + XPOSE_BYTES + 1024 + 256;
+};
+
+template <int STAGES>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
+    gemm_tc2s_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                     int M, int N, int K, int NA, Epilogue ep) {
+  using Cfg = Gemm2sCfg<STAGES>;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~uintptr_t(1023));
+  uint8_t* sW = smem;                                      // weight rows (MMA operand A)
+  uint8_t* sX = smem + STAGES * Cfg::A_BYTES;              // activation rows (MMA operand B)
+  float* sT = reinterpret_cast<float*>(smem + STAGES * Cfg::STAGE_BYTES);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + STAGES * Cfg::STAGE_BYTES + Cfg::XPOSE_BYTES);
+  uint64_t* empty = full + STAGES;
+  uint64_t* tfull = empty + STAGES;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(tempty + 2);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = tc::cluster_ctarank();
+  const int pair = blockIdx.x >> 1, num_pairs = gridDim.x >> 1;
+  const int num_m = (M + NA - 1) / NA;                     // activation blocks
+  const int num_n = (N + 255) / 256;                       // weight blocks
+  const int num_tiles = num_m * num_n;
+  const int num_k = K / Cfg::BK;
+  const int half = NA >> 1;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < STAGES; ++s) {
+      tc::mbar_init(&full[s], 1);
+      tc::mbar_init(&empty[s], 1);
+    }
+    for (int a = 0; a < 2; ++a) {
+      tc::mbar_init(&tfull[a], 1);
+      tc::mbar_init(&tempty[a], 8);
+    }
+    tc::fence_mbar_init();
+  }
+  if (warp == 0 && lane == 0) {
+    tc::tma_prefetch_desc(&tmA);
+    tc::tma_prefetch_desc(&tmB);
+  }
+  if (warp == 2) tc::tmem_alloc_2sm<Cfg::TMEM_COLS>(tmem_holder);
+  tc::fence_before();
+  __syncthreads();
+  tc::cluster_sync();
+  tc::fence_after();
+  const uint32_t tmem_base = *tmem_holder;
+  pdl_trigger();
+  pdl_wait();
+
+  // tile t: weight block t / num_m, activation block t % num_m -- the pairs running at the same
+  // time share a few weight panels (read from HBM once) and all of A (L2-resident)
+  if (warp == 0) {
+    if (lane == 0) {
+      const uint32_t bytes = 2 * (Cfg::A_BYTES + half * Cfg::BK * 2);
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int tile = pair; tile < num_tiles; tile += num_pairs) {
+        const int n_blk = tile / num_m, m_blk = tile - n_blk * num_m;
+        const int wrow = n_blk * 256 + rank * 128, xrow = m_blk * NA + rank * half;
+        for (int kb = 0; kb < num_k; ++kb) {
+          tc::mbar_wait(&empty[stage], phase ^ 1);
+          if (rank == 0) tc::mbar_expect_tx(&full[stage], bytes);
+          tc::tma_load_2d_2sm(sW + stage * Cfg::A_BYTES, &tmB, &full[stage], kb * Cfg::BK, wrow);
+          tc::tma_load_2d_2sm(sX + stage * Cfg::B_BYTES, &tmA, &full[stage], kb * Cfg::BK, xrow);
+          if (++stage == STAGES) {
+            stage = 0;
+            phase ^= 1;
+          }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && rank == 0) {
+      const uint32_t idesc = tc::idesc_bf16(256, NA);
+      int stage = 0;
+      uint32_t phase = 0;
+      int it = 0;
+      for (int tile = pair; tile < num_tiles; tile += num_pairs, ++it) {
+        const int acc = it & 1;
+        tc::mbar_wait(&tempty[acc], ((it >> 1) & 1) ^ 1);
+        tc::fence_after();
+        const uint32_t d = tmem_base + acc * 256;
+        for (int kb = 0; kb < num_k; ++kb) {
+          tc::mbar_wait(&full[stage], phase);
+          tc::fence_after();
+          const uint32_t a0 = tc::smem_u32(sW + stage * Cfg::A_BYTES);
+          const uint32_t b0 = tc::smem_u32(sX + stage * Cfg::B_BYTES);
+#pragma unroll
+          for (int k = 0; k < Cfg::BK / 16; ++k)
+            tc::mma_bf16_2sm(d, tc::sdesc_k_sw128(a0 + k * 32), tc::sdesc_k_sw128(b0 + k * 32),
+                             idesc, (kb | k) != 0);
+          tc::mma_commit_2sm(&empty[stage]);
+          if (++stage == STAGES) {
+            stage = 0;
+            phase ^= 1;
+          }
+        }
+        tc::mma_commit_2sm(&tfull[acc]);
+      }
+    }
+  } else if (warp >= 4) {
+    const int q = warp & 3;
+    float* xt = sT + q * 32 * 33;
+    const uint32_t tempty_leader = tc::mapa(tc::smem_u32(tempty), 0);
+    int it = 0;
+    for (int tile = pair; tile < num_tiles; tile += num_pairs, ++it) {
+      const int n_blk = tile / num_m, m_blk = tile - n_blk * num_m;
+      const int acc = it & 1;
+      tc::mbar_wait(&tfull[acc], (it >> 1) & 1);
+      tc::fence_after();
+      // this warp's 32 output columns; TMEM column j of the tile = activation row m_blk*NA + j
+      const int col0 = n_blk * 256 + rank * 128 + q * 32;
+      const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16) + acc * 256;
+      const int nchunk = NA >> 5, rem = NA & 31;
+#pragma unroll 1
+      for (int c = 0; c < nchunk + (rem ? 1 : 0); ++c) {
+        uint32_t r[32];
+        if (c < nchunk) {
+          tc::tmem_ld32(taddr + c * 32, r);
+        } else {                                           // NA % 32 == 16: last 16 columns
+          tc::tmem_ld16(taddr + c * 32, r);
+#pragma unroll
+          for (int j = 16; j < 32; ++j) r[j] = 0u;
+        }
+        tc::tmem_wait_ld();
+        // transpose: lane = column (col0 + lane), r[j] = row j  ->  lane = row, 32 columns
+#pragma unroll
+        for (int j = 0; j < 32; ++j) xt[j * 33 + lane] = __uint_as_float(r[j]);
+        __syncwarp();
+#pragma unroll
+        for (int j = 0; j < 32; ++j) r[j] = __float_as_uint(xt[lane * 33 + j]);
+        __syncwarp();
+        const int row = m_blk * NA + c * 32 + lane;
+        const RowCtx rc = row_ctx(ep, (c * 32 + lane < NA) ? M : 0, row);
+        ChunkIn in;
+        chunk_load(ep, rc, N, row, col0, in);
+        chunk_store(ep, rc, N, col0, r, in);
+      }
+      tc::fence_before();
+      __syncwarp();
+      if (lane == 0) tc::mbar_arrive_cluster(tempty_leader + acc * 8);
+    }
+  }
+  __syncthreads();
+  tc::cluster_sync();
+  if (warp == 2) {
+    tc::fence_after();
+    tc::tmem_dealloc_2sm<Cfg::TMEM_COLS>(tmem_base);
+  }
+}
+
+// ============================================================================================
 bool gemm_tc_supported(int dtype, int M, int N, int K) {
   return dtype == FPS_BF16 && M > 0 && K >= 64 && K % 64 == 0 && N % 8 == 0;
 }
@@ -427,6 +625,46 @@ static fps_status launch_pair(const void* A, const void* B, int M, int N, int K,
   return FPS_OK;
 }
 
+template <int STAGES>
+static fps_status launch_pair_swap(const void* A, const void* B, int M, int N, int K, int NA,
+                                   const Epilogue& ep, cudaStream_t s) {
+  using Cfg = Gemm2sCfg<STAGES>;
+  CUtensorMap ta, tb;
+  if (!make_tmap_2d_bf16(&ta, A, M, K, (uint64_t)K * 2, Cfg::BK, NA / 2) ||
+      !make_tmap_2d_bf16(&tb, B, N, K, (uint64_t)K * 2, Cfg::BK, 128))
+    return fail(FPS_ECUDA, "gemm_tc2s: cuTensorMapEncodeTiled failed (M=%d N=%d K=%d)", M, N, K);
+  static bool attr_set = false;
+  if (!attr_set) {
+    FPS_CUDA_TRY(cudaFuncSetAttribute(gemm_tc2s_kernel<STAGES>,
+                                      cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
+    attr_set = true;
+  }
+  const int tiles = ceil_div(M, NA) * ceil_div(N, 256);
+  const int pairs = tiles < kNumSMs / 2 ? tiles : kNumSMs / 2;
+  FPS_CUDA_TRY(launch_k(gemm_tc2s_kernel<STAGES>, dim3(2 * pairs), dim3(256), Cfg::SMEM, s, ta,
+                        tb, M, N, K, NA, ep));
+  count_launch();
+  FPS_LAUNCH_CHECK();
+  return FPS_OK;
+}
+
+// Activation-block height for the swapped pair kernel: minimise waves x NA (per-SM tensor work
+// of the critical path), ties to the larger NA (fewer tiles, fewer epilogue passes).
+static int swap_block(int M, int N, long* cost) {
+  int best = 256;
+  long bc = -1;
+  for (int na = 256; na >= 64; na -= 16) {
+    const long tiles = (long)ceil_div(M, na) * ceil_div(N, 256);
+    const long c = ((tiles + kNumSMs / 2 - 1) / (kNumSMs / 2)) * na;
+    if (bc < 0 || c < bc) {
+      bc = c;
+      best = na;
+    }
+  }
+  *cost = bc;
+  return best;
+}
+
 fps_status launch_gemm_tc(const void* A, const void* B, int M, int N, int K, const Epilogue& ep,
                           cudaStream_t s) {
   if (!aligned16(A) || !aligned16(B)) return fail(FPS_EINVAL, "gemm_tc: unaligned operand");
@@ -449,6 +687,14 @@ fps_status launch_gemm_tc(const void* A, const void* B, int M, int N, int K, con
   //  short K: its longer prologue / epilogue lose -- 27.3 vs 23.2 us at 1331x3072x3072)
   const bool pair_wins = tp > kNumSMs / 2 || cp < cmin ||
                          (cp == cmin && (m2 * 256 - M < 128 || K >= 8192));
+  // swapped operands (activation rows on the MMA's N side, no 256-row M padding): correct and
+  // tested, but measured no faster at the masked-block shapes (1331x9216x3072: 59.8 vs 59.2 us
+  // for the pair kernel -- under the power cap the MMAs on TMA zero-fill rows cost little) and
+  // slow for small activation blocks (NA = 144: 3.6x), so it is only selectable by force
+  if (g_gemm_force == 3) {
+    long cs = 0;
+    return launch_pair_swap<6>(A, B, M, N, K, swap_block(M, N, &cs), ep, s);
+  }
   if (g_gemm_force == 2 || (g_gemm_force == 0 && pair_wins))
     return launch_pair<6>(A, B, M, N, K, ep, s);
   if (c256 <= c128) return launch_cfg<256, 4>(A, B, M, N, K, ep, s);
