@@ -154,17 +154,24 @@ def build_engine_inputs(F, w, mode, device, n_entries, location=0, copy_method=0
         return (torch.randn(*shape, generator=gen, device=device) * scale).to(torch.bfloat16)
 
     layers = []
+    par = w.get("block") == "par"
     for _ in range(N):
-        t = {"w_qkv": rnd(3 * H, H, scale=H ** -0.5), "b_qkv": rnd(3 * H, scale=0.02),
-             "w_o": rnd(H, H, scale=H ** -0.5), "b_o": rnd(H, scale=0.02),
-             "w_up": rnd(Fd, H, scale=H ** -0.5), "b_up": rnd(Fd, scale=0.02),
-             "w_down": rnd(H, Fd, scale=Fd ** -0.5), "b_down": rnd(H, scale=0.02)}
+        if par:      # parallel (Flux single-stream) block: W1 [3H+F, H], W2 [H, H+F] (R23)
+            t = {"w_qkv": rnd(3 * H + Fd, H, scale=H ** -0.5), "b_qkv": rnd(3 * H + Fd, scale=0.02),
+                 "w_down": rnd(H, H + Fd, scale=(H + Fd) ** -0.5), "b_down": rnd(H, scale=0.02)}
+        else:
+            t = {"w_qkv": rnd(3 * H, H, scale=H ** -0.5), "b_qkv": rnd(3 * H, scale=0.02),
+                 "w_o": rnd(H, H, scale=H ** -0.5), "b_o": rnd(H, scale=0.02),
+                 "w_up": rnd(Fd, H, scale=H ** -0.5), "b_up": rnd(Fd, scale=0.02),
+                 "w_down": rnd(H, Fd, scale=Fd ** -0.5), "b_down": rnd(H, scale=0.02)}
         layers.append(F.BlockWeights.__new__(F.BlockWeights))
         bw = layers[-1]
         bw.t, bw.H, bw.F, bw.heads, bw.dtype = t, H, Fd, w["heads"], F.FPS_BF16
+        bw.kind = F.FPS_BLOCK_PAR if par else F.FPS_BLOCK_SEQ
         bw.c = F.fps_block_weights(H, w["heads"], H // w["heads"], Fd, F.FPS_BF16,
-                                   *[t[k].data_ptr() for k in ("w_qkv", "b_qkv", "w_o", "b_o", "w_up",
-                                                               "b_up", "w_down", "b_down")])
+                                   *[t[k].data_ptr() if k in t else None
+                                     for k in ("w_qkv", "b_qkv", "w_o", "b_o", "w_up", "b_up",
+                                               "w_down", "b_down")], bw.kind)
     mod = torch.zeros(N, w["steps"], 6, H, device=device)
     mod += 0.02 * torch.randn(N, w["steps"], 6, H, generator=gen, device=device)
     mod[:, :, 2] += 1.0
@@ -305,7 +312,7 @@ def oracle_block_sample(w, mode, ratio, seed=7):
     g = synth.rng(seed)
     H, Fd, L_img, L_txt = w["H"], w["F"], w["L_img"], w["L_txt"]
     L = L_img + L_txt
-    wt = synth.block_weights(g, H, Fd, "bf16")
+    wt = synth.block_weights(g, H, Fd, "bf16", w.get("block", "seq"))
     mask = synth.token_mask(synth.mask_blobs(g, *w["grid"], ratio), L_txt)
     M, U = build_mask_index(mask)
     x = synth.latent(g, L, H, "bf16")
@@ -339,6 +346,9 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C3", choices=list(WORKLOADS))
     ap.add_argument("--mode", default="kv", choices=["kv", "y"])
+    ap.add_argument("--block", default="seq", choices=["seq", "par"],
+                    help="block kind: sequential attention -> MLP, or the parallel (Flux "
+                         "single-stream) block with fused input / output projections (NEXT-2)")
     ap.add_argument("--tier", default="host", choices=["host", "hbm", "host_hugepage"],
                     help="template cache in pinned host DRAM (configs[2]) or HBM (NEXT-1)")
     ap.add_argument("--copy-ctas", type=int, default=0, help="CTAs of the SM row gather (0 = lib default)")
@@ -360,7 +370,7 @@ def main():
     rank = int(os.environ.get("RANK", 0))
     world = int(os.environ.get("WORLD_SIZE", 1))
     local = int(os.environ.get("LOCAL_RANK", 0))
-    w = WORKLOADS[args.config]
+    w = dict(WORKLOADS[args.config], block=args.block)
     K, W = args.steps, max(args.warmup, 0)
     if W + K > w["steps"]:
         raise SystemExit(f"--warmup + --steps must be <= {w['steps']} denoising steps")
@@ -370,7 +380,7 @@ def main():
                 "head_dim": w["H"] // w["heads"], "mlp": w["F"], "tokens": L,
                 "image_tokens": w["L_img"], "text_tokens": w["L_txt"], "blocks": w["layers"],
                 "denoise_steps": w["steps"], "cache_mode": args.mode,
-                "batch_per_gpu": w["batch"], "l2": "inputs > L2 (12.9 GB of weights streamed per step)"}
+                "batch_per_gpu": w["batch"], "block": args.block, "l2": "inputs > L2 (12.9 GB of weights streamed per step)"}
     if w["L_txt"] == 0:
         base_cfg["l2"] = "inputs > L2 (weights + activations streamed per step)"
 
@@ -433,6 +443,13 @@ def main():
     log(f"[rank {rank}] calibrating")
     cm, fit = calibrate(F, w, args.mode, layers, cache, [dict()] * w["batch"], device)
     log(f"[rank {rank}] fit {fit}")
+    if world > 1:
+        # every rank routes the same pool with Alg. 2; the cost models must be identical for the
+        # assignments to agree, so all ranks use rank 0's fit (setup only, not on the data path)
+        import torch.distributed as dist
+        obj = [(cm.comp, cm.load, fit)]
+        dist.broadcast_object_list(obj, src=0)
+        cm.comp, cm.load, fit = obj[0]
     my_ids, assign, held = sched.shard_requests([p["n_active"] for p in pool], L, world, rank, cm,
                                                 w["batch"])
     mine = [pool[i] for i in my_ids]

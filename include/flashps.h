@@ -66,6 +66,18 @@ void fps_profile_enable(int32_t on);
 int32_t fps_profile_read(double* ms, double* flops, double* bytes, int64_t* count);
 
 /* ---------------------------------------------------------------------------------------
+ * a1 input (NEXT-4)  Pixel mask -> token mask.  L79 (§2.1): the latent (B, C, H, W) is reshaped
+ * to (B, H x W, C), one token per latent position; a token covers an f x f block of editing-mask
+ * pixels (VAE down-sampling x patchify).  Reading R8: a token is active iff ANY of
+ * its pixels is nonzero; reading R9: L_txt text tokens are appended, always active.
+ *   d_pix   uint8 [n_req][Hp * Wp] row-major pixel masks (nonzero = edit this pixel).
+ *   f       block edge; must divide Hp and Wp (else FPS_EINVAL).
+ *   d_tok   uint8 [n_req][(Hp/f) * (Wp/f) + L_txt] written with 0/1 (caller-owned).
+ * Bit-exact with oracle/index.py pixel_to_token_mask.  Output feeds fps_build_mask_index. */
+fps_status fps_mask_to_tokens(const uint8_t* d_pix, int32_t n_req, int32_t Hp, int32_t Wp,
+                              int32_t f, int32_t L_txt, uint8_t* d_tok, void* stream);
+
+/* ---------------------------------------------------------------------------------------
  * a1  Mask -> token index (L130 "categorize the tokens as masked tokens and unmasked tokens").
  *   d_masks       uint8 [total]: request r's token mask occupies [off[r], off[r+1]);
  *                 nonzero = active (masked image token, or text token -- set by the caller).
@@ -170,14 +182,22 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
  * Block (oracle/block.py):  h1 = LN(x)(1+sc1)+sh1; Q,K,V = h1 W^T + b; A = softmax(QK^T/sqrt(d))V
  * per head; x1 = x + g1 (A Wo^T + bo); y = x1 + g2 (GELU_tanh(LN(x1)(1+sc2)+sh2 W1^T + b1) W2^T + b2).
  * Weights use the nn.Linear layout W[out, in], row-major, dtype = `dtype`; biases may be NULL.
+ *
+ * kind = FPS_BLOCK_PAR (NEXT-2, reading R23): the parallel (Flux single-stream) block
+ *   h = LN(x)(1+sc1)+sh1; [Q|K|V|Z] = h W1^T + b1; y = x + g1 ([A | GELU_tanh(Z)] W2^T + b2)
+ * with W1 = w_qkv [3H+F, H] (rows Wq, Wk, Wv, then the F MLP-input rows), b1 = b_qkv [3H+F],
+ * W2 = w_down [H, H+F], b2 = b_down [H]; w_o, b_o, w_up, b_up must be NULL; only
+ * (shift1, scale1, gate1) of the modulation vector are read.  Same masked modes and cache.
  */
+enum { FPS_BLOCK_SEQ = 0, FPS_BLOCK_PAR = 1 };
 typedef struct {
   int32_t H, heads, head_dim, F;   /* H = heads*head_dim; F = MLP width                    */
   int32_t dtype;                   /* FPS_BF16 (tcgen05 path) | FPS_F32 (SIMT fp32 path)   */
-  const void *w_qkv, *b_qkv;       /* [3H, H], [3H]  rows: Wq, Wk, Wv                       */
-  const void *w_o, *b_o;           /* [H, H], [H]                                          */
-  const void *w_up, *b_up;         /* [F, H], [F]                                          */
-  const void *w_down, *b_down;     /* [H, F], [H]                                          */
+  const void *w_qkv, *b_qkv;       /* [3H, H], [3H]  rows: Wq, Wk, Wv  (PAR: W1, b1)        */
+  const void *w_o, *b_o;           /* [H, H], [H]                      (PAR: NULL)          */
+  const void *w_up, *b_up;         /* [F, H], [F]                      (PAR: NULL)          */
+  const void *w_down, *b_down;     /* [H, F], [H]                      (PAR: W2 [H, H+F], b2) */
+  int32_t kind;                    /* FPS_BLOCK_SEQ | FPS_BLOCK_PAR                         */
 } fps_block_weights;
 
 /* One varlen launch over a continuous batch (L237): request r owns active rows

@@ -22,6 +22,18 @@ unmasked ids U of one request (index.build_mask_index),
   * Y-mode (Fig. 5-Bottom): the block input on rows U is the cached previous-block output
     Y (R4); K, V are projected over all L rows; Q, O-projection and MLP on rows M only.
 Everything is float64.
+
+Parallel block variant (NEXT-2, weights["kind"] == "par"; reading R23): the Flux single-stream
+block, where attention and MLP read the same normalised input and share one input and one
+output projection (Flux is a stack of such transformer blocks, L79 / L92 footnote):
+
+    h  = LN(x)(1 + scale1) + shift1
+    [Q | K | V | Z] = h W1^T + b1                         W1 in R^{(3H+F) x H}
+    y  = x + gate1 * ([A | GELU_tanh(Z)] W2^T + b2)       A = concat_j A_j, W2 in R^{H x (H+F)}
+
+Only (shift1, scale1, gate1) of `mod` are used.  Its FLOPs per row equal the sequential block's
+(12 H^2 multiply-adds with F = 4H), and the same masked modes apply: Z is token-wise (rows M
+only), K/V follow KV- or Y-mode exactly as above.
 """
 from __future__ import annotations
 
@@ -93,9 +105,28 @@ def attention(Q, K, V, heads):
     return out
 
 
+def is_parallel(w):
+    return w.get("kind", "seq") == "par"
+
+
 def _qkv_weights(w, H):
-    W, b = f64(w["w_qkv"]), f64(w["b_qkv"])
+    if is_parallel(w):
+        W, b = f64(w["w_1"]), f64(w["b_1"])
+    else:
+        W, b = f64(w["w_qkv"]), f64(w["b_qkv"])
     return (W[0:H], b[0:H]), (W[H:2 * H], b[H:2 * H]), (W[2 * H:3 * H], b[2 * H:3 * H])
+
+
+def _block_out(x_rows, h_rows, a_rows, w, mod, H):
+    """The block output on the given rows from their input x, normalised input h and attention
+    output A: the sequential block's O projection + MLP, or the parallel block's fused output."""
+    if not is_parallel(w):
+        return _attn_out_and_mlp(x_rows, a_rows, w, mod, H)
+    _, _, g1, _, _, _ = split_mod(mod, H)
+    W1, b1 = f64(w["w_1"]), f64(w["b_1"])
+    z = gelu_tanh(linear(h_rows, W1[3 * H:], b1[3 * H:]))          # MLP branch, token-wise
+    cat = np.concatenate([f64(a_rows), z], axis=1)                  # [A | GELU(Z)]
+    return f64(x_rows) + g1 * linear(cat, w["w_2"], w["b_2"])
 
 
 def _attn_out_and_mlp(x_rows, a_rows, w, mod, H):
@@ -116,7 +147,7 @@ def dense_block(x, w, mod, heads):
     (Wq, bq), (Wk, bk), (Wv, bv) = _qkv_weights(w, H)
     Q, K, V = linear(h1, Wq, bq), linear(h1, Wk, bk), linear(h1, Wv, bv)
     a = attention(Q, K, V, heads)
-    return _attn_out_and_mlp(x, a, w, mod, H), K, V
+    return _block_out(x, h1, a, w, mod, H), K, V
 
 
 def masked_block_kv(x_M, M, U, K_U, V_U, w, mod, heads, L):
@@ -137,7 +168,7 @@ def masked_block_kv(x_M, M, U, K_U, V_U, w, mod, heads, L):
     K_all[M], V_all[M] = K_M, V_M
     K_all[U], V_all[U] = f64(K_U), f64(V_U)
     a_M = attention(Q_M, K_all, V_all, heads)                  # queries from masked rows only (L159)
-    return _attn_out_and_mlp(x_M, a_M, w, mod, H), K_M, V_M
+    return _block_out(x_M, h1_M, a_M, w, mod, H), K_M, V_M
 
 
 def masked_block_y(x_M, M, U, x_U, w, mod, heads, L):
@@ -154,4 +185,4 @@ def masked_block_y(x_M, M, U, x_U, w, mod, heads, L):
     Q_M = linear(h1[M], Wq, bq)
     K, V = linear(h1, Wk, bk), linear(h1, Wv, bv)
     a_M = attention(Q_M, K, V, heads)
-    return _attn_out_and_mlp(x_M, a_M, w, mod, H)
+    return _block_out(x_M, h1[M], a_M, w, mod, H)

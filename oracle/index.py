@@ -37,3 +37,31 @@ def scatter_rows(rows, ids, out):
     for i, t in enumerate(ids):
         out[t] = rows[i]
     return out
+
+
+def pixel_to_token_mask(pix, f, L_txt=0):
+    """Pixel-level editing mask -> token mask (NEXT-4; reading R8 of DESIGN.md).
+
+    PAPER.md L79 (§2.1): "a latent of shape (B, C, H, W) is reshaped to (B, H x W, C)", i.e. one
+    token per latent position; a token covers an f x f block of mask pixels (VAE down-sampling
+    x patchify; f = 16 for Flux-scale 1024^2 -> 64 x 64 tokens, 16 / 32 for the SDXL-scale 64^2 /
+    32^2 levels).  Reading R8: the token is masked iff ANY covered pixel is masked (so every
+    edited pixel is regenerated).  Text tokens (reading R9) are appended, always active.
+    pix: 2-D array [Hp, Wp], nonzero = masked; Hp, Wp multiples of f.  Returns uint8 [T + L_txt].
+    """
+    Hp, Wp = pix.shape
+    Ht, Wt = Hp // f, Wp // f
+    out = np.zeros(Ht * Wt + L_txt, dtype=np.uint8)
+    for i in range(Ht):
+        for j in range(Wt):
+            hit = 0
+            for y in range(i * f, (i + 1) * f):
+                for x in range(j * f, (j + 1) * f):
+                    if pix[y, x]:
+                        hit = 1
+                        break
+                if hit:
+                    break
+            out[i * Wt + j] = hit
+    out[Ht * Wt:] = 1
+    return out

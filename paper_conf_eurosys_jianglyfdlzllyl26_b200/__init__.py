@@ -40,6 +40,16 @@ def require_gpu():
 
 
 # ---------------------------------------------------------------------------------------
+def mask_to_tokens(pix, f, L_txt=0, stream=None):
+    """NEXT-4 on the GPU: pixel masks (uint8 cuda tensor [n_req, Hp, Wp] or [Hp, Wp]) -> token
+    masks [n_req, (Hp/f)*(Wp/f) + L_txt] (uint8, text tokens active)."""
+    p = pix.reshape((-1,) + tuple(pix.shape[-2:])).contiguous().to(torch.uint8)
+    n, Hp, Wp = p.shape
+    tok = torch.empty(n, (Hp // f) * (Wp // f) + L_txt, dtype=torch.uint8, device=pix.device)
+    _lib.fps_mask_to_tokens(ptr(p), n, Hp, Wp, f, L_txt, ptr(tok), stream_ptr(stream))
+    return tok
+
+
 def build_mask_index(masks, stream=None):
     """a1 on the GPU. masks: list of uint8 cuda tensors (one per request, text rows set).
     Returns (masked_ids, unmasked_ids, n_masked, offsets) as cuda int32 tensors; request r's
@@ -76,16 +86,20 @@ class BlockWeights:
     """Holds one block's device weights (nn.Linear layout) and its C descriptor."""
 
     def __init__(self, w: dict, heads: int, dtype: int, device="cuda"):
+        """w: the sequential block's w_qkv, b_qkv, w_o, b_o, w_up, b_up, w_down, b_down, or with
+        w["kind"] == "par" the parallel block's w_1 [3H+F, H], b_1, w_2 [H, H+F], b_2."""
         td = TORCH_DTYPE[dtype]
-        self.t = {k: torch.as_tensor(np.ascontiguousarray(v)).to(device=device, dtype=td)
-                  for k, v in w.items()}
-        H = self.t["w_o"].shape[0]
-        F = self.t["w_up"].shape[0]
+        self.kind = _lib.FPS_BLOCK_PAR if w.get("kind", "seq") == "par" else _lib.FPS_BLOCK_SEQ
+        alias = {"w_1": "w_qkv", "b_1": "b_qkv", "w_2": "w_down", "b_2": "b_down"}
+        self.t = {alias.get(k, k): torch.as_tensor(np.ascontiguousarray(v)).to(device=device, dtype=td)
+                  for k, v in w.items() if k != "kind"}
+        H = self.t["w_down"].shape[0]
+        F = (self.t["w_qkv"].shape[0] - 3 * H) if self.kind else self.t["w_up"].shape[0]
         self.H, self.F, self.heads, self.dtype = H, F, heads, dtype
         self.c = fps_block_weights(H, heads, H // heads, F, dtype,
                                    *[ptr(self.t.get(k)) for k in
                                      ("w_qkv", "b_qkv", "w_o", "b_o", "w_up", "b_up", "w_down",
-                                      "b_down")])
+                                      "b_down")], self.kind)
 
 
 class VarlenBatch:

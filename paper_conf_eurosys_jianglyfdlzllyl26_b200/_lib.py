@@ -16,6 +16,7 @@ LIB_PATH = os.environ.get("FPS_LIB") or os.path.join(_HERE, "libflashps.so")
 FPS_OK, FPS_EINVAL, FPS_ECUDA, FPS_ENOMEM, FPS_EUNSUPPORTED, FPS_ESTATE = 0, -1, -2, -3, -4, -5
 FPS_F32, FPS_BF16 = 0, 1
 FPS_MODE_KV, FPS_MODE_Y = 0, 1
+FPS_BLOCK_SEQ, FPS_BLOCK_PAR = 0, 1
 
 vp, i32, u32, i64, sz, dbl = C.c_void_p, C.c_int32, C.c_uint32, C.c_int64, C.c_size_t, C.c_double
 P_i32, P_u8, P_dbl, P_f32 = C.POINTER(C.c_int32), C.POINTER(C.c_uint8), C.POINTER(C.c_double), C.POINTER(C.c_float)
@@ -41,7 +42,7 @@ class fps_prefetch_item(C.Structure):
 class fps_block_weights(C.Structure):
     _fields_ = [("H", i32), ("heads", i32), ("head_dim", i32), ("F", i32), ("dtype", i32),
                 ("w_qkv", vp), ("b_qkv", vp), ("w_o", vp), ("b_o", vp), ("w_up", vp),
-                ("b_up", vp), ("w_down", vp), ("b_down", vp)]
+                ("b_up", vp), ("w_down", vp), ("b_down", vp), ("kind", i32)]
 
 
 class fps_varlen_batch(C.Structure):
@@ -73,6 +74,7 @@ _SIGS = [
     ("fps_set_disable_tc", None, [i32], False),
     ("fps_profile_enable", None, [i32], False),
     ("fps_profile_read", i32, [P_dbl, P_dbl, P_dbl, C.POINTER(C.c_int64)], False),
+    ("fps_mask_to_tokens", C.c_int, [vp, i32, i32, i32, i32, i32, vp, vp], True),
     ("fps_build_mask_index", C.c_int, [vp, vp, i32, i32, vp, vp, vp, vp], True),
     ("fps_gather_rows", C.c_int, [vp, vp, i32, i32, vp, vp], True),
     ("fps_scatter_rows", C.c_int, [vp, vp, i32, i32, vp, vp], True),

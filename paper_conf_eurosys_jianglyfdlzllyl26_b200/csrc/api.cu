@@ -94,15 +94,17 @@ fps_status launch_gemm(int dtype, const void* A, const void* B, int M, int N, in
 fps_status launch_attention(int dtype, const void* q, const void* kv, void* o, int heads,
                             int head_dim, const int32_t* d_cu_q, const int32_t* d_cu_k,
                             const int32_t* h_cu_q, const int32_t* h_cu_k, int n_req, int total_q,
-                            int max_q, int max_k, cudaStream_t s) {
+                            int max_q, int max_k, cudaStream_t s, int ldo) {
   (void)max_k;
   if (total_q <= 0) return FPS_OK;
   prof::begin(s);
   fps_status st;
   if (!(g_disable_tc & 2) && attention_tc_supported(dtype, head_dim) && h_cu_q && h_cu_k)
-    st = launch_attention_tc(q, kv, o, heads, head_dim, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);
+    st = launch_attention_tc(q, kv, o, heads, head_dim, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s,
+                             ldo);
   else
-    st = launch_attention_simt(dtype, q, kv, o, heads, head_dim, d_cu_q, d_cu_k, n_req, total_q, s);
+    st = launch_attention_simt(dtype, q, kv, o, heads, head_dim, d_cu_q, d_cu_k, n_req, total_q, s,
+                               ldo);
   if (prof::enabled() && h_cu_q && h_cu_k) {
     // algorithmic work: QK^T and PV, 4 n_r L_r H FLOPs; bytes: Q, O once + K|V once per request
     double fl = 0, by = 0;
@@ -148,7 +150,12 @@ static fps_status check_weights(const fps_block_weights* w) {
   FPS_CHECK_ARG(w->H > 0 && w->heads > 0 && w->head_dim > 0 && w->heads * w->head_dim == w->H,
                 "H=%d heads=%d head_dim=%d", w->H, w->heads, w->head_dim);
   FPS_CHECK_ARG(w->F > 0, "F=%d", w->F);
-  FPS_CHECK_ARG(w->w_qkv && w->w_o && w->w_up && w->w_down, "weight pointer is NULL");
+  FPS_CHECK_ARG(w->kind == FPS_BLOCK_SEQ || w->kind == FPS_BLOCK_PAR, "kind %d", w->kind);
+  if (w->kind == FPS_BLOCK_PAR)
+    FPS_CHECK_ARG(w->w_qkv && w->w_down && !w->w_o && !w->b_o && !w->w_up && !w->b_up,
+                  "parallel block: w_qkv (W1) and w_down (W2) set, w_o/b_o/w_up/b_up NULL");
+  else
+    FPS_CHECK_ARG(w->w_qkv && w->w_o && w->w_up && w->w_down, "weight pointer is NULL");
   const int vec = 16 / elt_size(w->dtype);
   FPS_CHECK_ARG(w->H % vec == 0 && w->F % vec == 0, "H and F must be multiples of %d", vec);
   return FPS_OK;
@@ -186,7 +193,13 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
     ep.out0 = ws.q; ep.ld0 = H; ep.map0 = nullptr;
     ep.out1 = kv; ep.ld1 = 2 * H; ep.map1 = b->d_q_row;
     ep.split = H;
-    FPS_TRY(launch_gemm(dt, ws.h, w->w_qkv, tq, 3 * H, H, ep, s));
+    int n_out = 3 * H;
+    if (w->kind == FPS_BLOCK_PAR) {     // + MLP input rows: GELU(Z) -> cat[:, H:H+F]
+      ep.out2 = (char*)ws.ao + (size_t)H * e; ep.ld2 = H + F; ep.split2 = 3 * H;
+      ep.act = 1; ep.act_from = 3 * H;
+      n_out += F;
+    }
+    FPS_TRY(launch_gemm(dt, ws.h, w->w_qkv, tq, n_out, H, ep, s));
   }
   if (tu > 0) {
     // Y-mode: cached block-input rows U -> LN -> K|V projection (Fig. 5-Bottom, reading R5)
@@ -200,6 +213,19 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
     FPS_TRY(launch_gemm(dt, ws.hu, (const char*)w->w_qkv + (size_t)H * H * e, tu, 2 * H, H, ep, s));
   }
   if (tq == 0) return FPS_OK;
+  if (w->kind == FPS_BLOCK_PAR) {
+    // parallel block (reading R23): ws.ao..ws.u hold cat = [A | GELU(Z)], [tq, H+F]
+    char* cat = ws.ao;
+    if (kv_ready) FPS_CUDA_TRY(cudaStreamWaitEvent(s, kv_ready, 0));
+    FPS_TRY(launch_attention(dt, ws.q, kv, cat, w->heads, w->head_dim, b->d_cu_q, b->d_cu_k,
+                             b->h_cu_q, b->h_cu_k, b->n_req, tq, b->max_q, b->max_k, s, H + F));
+    Epilogue ep{};
+    ep.bias = w->b_down;
+    ep.resid = x_act; ep.ld_resid = H;
+    ep.gate = modp(2); ep.gate_stride = 6 * H; ep.cu = b->d_cu_q; ep.n_req = b->n_req;
+    ep.out0 = y_act; ep.ld0 = H; ep.split = H;
+    return launch_gemm(dt, cat, w->w_down, tq, H, H + F, ep, s);
+  }
   // a6: queries from active rows only, keys = merged fresh + cached rows (L159)
   if (kv_ready) FPS_CUDA_TRY(cudaStreamWaitEvent(s, kv_ready, 0));
   FPS_TRY(launch_attention(dt, ws.q, kv, ws.ao, w->heads, w->head_dim, b->d_cu_q, b->d_cu_k,
@@ -300,6 +326,15 @@ fps_status fps_build_mask_index(const uint8_t* d_masks, const int32_t* d_offsets
                 "NULL pointer");
   return launch_mask_index(d_masks, d_offsets, n_req, max_len, d_masked_ids, d_unmasked_ids,
                            d_n_masked, as_stream(stream));
+}
+
+fps_status fps_mask_to_tokens(const uint8_t* d_pix, int32_t n_req, int32_t Hp, int32_t Wp,
+                              int32_t f, int32_t L_txt, uint8_t* d_tok, void* stream) {
+  FPS_CHECK_ARG(n_req >= 0 && Hp >= 0 && Wp >= 0 && L_txt >= 0, "negative size");
+  FPS_CHECK_ARG(f > 0 && Hp % f == 0 && Wp % f == 0, "f=%d must divide Hp=%d and Wp=%d", f, Hp, Wp);
+  if (n_req == 0 || (Hp * Wp == 0 && L_txt == 0)) return FPS_OK;
+  FPS_CHECK_ARG(d_tok && (d_pix || Hp * Wp == 0), "NULL pointer");
+  return launch_mask_pool(d_pix, n_req, Hp, Wp, f, L_txt, d_tok, as_stream(stream));
 }
 
 static fps_status check_rows(const void* src, const void* dst, int32_t n, int32_t row_bytes) {

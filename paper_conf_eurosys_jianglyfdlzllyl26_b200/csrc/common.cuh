@@ -202,6 +202,10 @@ struct Epilogue {
   void* out0; int ld0; const int32_t* map0;   // map0: output row for row r (null -> r)
   void* out1; int ld1; const int32_t* map1;
   int split;
+  // optional third column range [split2, N) -> out2 (row r, no remap), and the activation
+  // applied only to columns >= act_from (the parallel block's fused QKV|MLP projection)
+  void* out2; int ld2; int split2;
+  int act_from;
 };
 
 }  // namespace fps

@@ -7,7 +7,7 @@
 namespace fps {
 
 // Apply the epilogue to NC consecutive columns c0..c0+NC-1 of row r (NC | 8, c0 % NC == 0,
-// and all NC columns on the same side of `split`).  Vectorised 16-B stores when possible.
+// and all NC columns on the same side of `split`, `split2` and `act_from`).  Vectorised 16-B stores when possible.
 template <typename T, int NC>
 __device__ __forceinline__ void epilogue_store(const Epilogue& ep, int r, int c0, float* v) {
   if (ep.bias) {
@@ -15,7 +15,7 @@ __device__ __forceinline__ void epilogue_store(const Epilogue& ep, int r, int c0
 #pragma unroll
     for (int e = 0; e < NC; ++e) v[e] += to_f(b[e]);
   }
-  if (ep.act == 1) {
+  if (ep.act == 1 && c0 >= ep.act_from) {
 #pragma unroll
     for (int e = 0; e < NC; ++e) v[e] = gelu_tanh(v[e]);
   }
@@ -35,6 +35,8 @@ __device__ __forceinline__ void epilogue_store(const Epilogue& ep, int r, int c0
   if (c0 < ep.split) {
     const int orow = ep.map0 ? __ldg(ep.map0 + r) : r;
     dst = reinterpret_cast<T*>(ep.out0) + (size_t)orow * ep.ld0 + c0;
+  } else if (ep.out2 && c0 >= ep.split2) {
+    dst = reinterpret_cast<T*>(ep.out2) + (size_t)r * ep.ld2 + (c0 - ep.split2);
   } else {
     const int orow = ep.map1 ? __ldg(ep.map1 + r) : r;
     dst = reinterpret_cast<T*>(ep.out1) + (size_t)orow * ep.ld1 + (c0 - ep.split);

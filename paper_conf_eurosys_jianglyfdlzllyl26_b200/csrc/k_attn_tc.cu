@@ -32,7 +32,7 @@ template <int D>
 __global__ void __launch_bounds__(256, 1)
     attn_tc_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmKV,
                    __nv_bfloat16* __restrict__ O, const int32_t* __restrict__ cu_q,
-                   const int32_t* __restrict__ cu_k, int n_req, int heads, float scale_log2) {
+                   const int32_t* __restrict__ cu_k, int n_req, int heads, float scale_log2, int ldo) {
   using Cfg = AttnCfg<D>;
   constexpr int CHUNK = 128 * 128;                         // bytes of one [128 rows x 128 B] chunk
   extern __shared__ uint8_t smem_raw[];
@@ -258,7 +258,7 @@ __global__ void __launch_bounds__(256, 1)
       tc::fence_after();
     }
     const float inv = (l > 0.f) ? 1.0f / l : 0.f;
-    __nv_bfloat16* orow = O + (size_t)(q0 + row) * H + head * D;
+    __nv_bfloat16* orow = O + (size_t)(q0 + row) * ldo + head * D;
 #pragma unroll 1
     for (int c = 0; c < D / 32; ++c) {
       uint32_t o[32];
@@ -306,7 +306,7 @@ template <int D>
 __global__ void __launch_bounds__(384, 1)
     attn_tc2_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmKV,
                     __nv_bfloat16* __restrict__ O, const int32_t* __restrict__ cu_q,
-                    const int32_t* __restrict__ cu_k, int n_req, int heads, float scale_log2) {
+                    const int32_t* __restrict__ cu_k, int n_req, int heads, float scale_log2, int ldo) {
   using Cfg = Attn2Cfg<D>;
   constexpr int CHUNK = 128 * 128;
   extern __shared__ uint8_t smem_raw[];
@@ -572,7 +572,7 @@ __global__ void __launch_bounds__(384, 1)
       }
       const float inv = (l > 0.f) ? 1.0f / l : 0.f;
       const int grow = q0 + t * 128 + row;
-      __nv_bfloat16* orow = O + (size_t)grow * H + head * D;
+      __nv_bfloat16* orow = O + (size_t)grow * ldo + head * D;
 #pragma unroll 1
       for (int c = 0; c < D / 32; ++c) {
         uint32_t o[32];
@@ -657,7 +657,7 @@ template <int D>
 __global__ void __launch_bounds__(512, 1)
     attn_tc3_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmKV,
                     __nv_bfloat16* __restrict__ O, const int32_t* __restrict__ cu_q,
-                    const int32_t* __restrict__ cu_k, int n_req, int heads, float scale_log2) {
+                    const int32_t* __restrict__ cu_k, int n_req, int heads, float scale_log2, int ldo) {
   using Cfg = Attn3Cfg<D>;
   constexpr int CHUNK = 128 * 128;
   extern __shared__ uint8_t smem_raw[];
@@ -935,7 +935,7 @@ __global__ void __launch_bounds__(512, 1)
     }
     for (int t = 0; t < ntl; ++t) {
       const int grow = q0 + t * 128 + row;
-      __nv_bfloat16* orow = O + (size_t)grow * H + head * D;
+      __nv_bfloat16* orow = O + (size_t)grow * ldo + head * D;
       if (nk == 0) {                                       // no keys: defined zero output
         if (grow < q_end)
           for (int c = 0; c < D; c += 8) *reinterpret_cast<uint4*>(orow + c) = make_uint4(0, 0, 0, 0);
@@ -981,7 +981,7 @@ bool attention_tc_supported(int dtype, int head_dim) {
 template <int D>
 static fps_status launch_d(const void* q, const void* kv, void* o, int heads,
                            const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
-                           const int32_t* h_cu_k, int n_req, cudaStream_t s) {
+                           const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo) {
   using Cfg = AttnCfg<D>;
   const int H = heads * D;
   int tiles = 0;
@@ -1003,7 +1003,7 @@ static fps_status launch_d(const void* q, const void* kv, void* o, int heads,
   const float scale_log2 = 1.4426950408889634f / sqrtf((float)D);
   FPS_CUDA_TRY(launch_k(attn_tc_kernel<D>, dim3(tiles, heads), dim3(256), Cfg::SMEM, s, tq, tkv,
                         reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads,
-                        scale_log2));
+                        scale_log2, ldo));
   count_launch();
   FPS_LAUNCH_CHECK();
   return FPS_OK;
@@ -1012,7 +1012,7 @@ static fps_status launch_d(const void* q, const void* kv, void* o, int heads,
 template <int D>
 static fps_status launch_d2(const void* q, const void* kv, void* o, int heads,
                             const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
-                            const int32_t* h_cu_k, int n_req, cudaStream_t s) {
+                            const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo) {
   using Cfg = Attn2Cfg<D>;
   const int H = heads * D;
   int pairs = 0;
@@ -1032,7 +1032,7 @@ static fps_status launch_d2(const void* q, const void* kv, void* o, int heads,
   const float scale_log2 = 1.4426950408889634f / sqrtf((float)D);
   FPS_CUDA_TRY(launch_k(attn_tc2_kernel<D>, dim3(pairs, heads), dim3(384), Cfg::SMEM, s, tq, tkv,
                         reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads,
-                        scale_log2));
+                        scale_log2, ldo));
   count_launch();
   FPS_LAUNCH_CHECK();
   return FPS_OK;
@@ -1041,7 +1041,7 @@ static fps_status launch_d2(const void* q, const void* kv, void* o, int heads,
 template <int D>
 static fps_status launch_d3(const void* q, const void* kv, void* o, int heads,
                             const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
-                            const int32_t* h_cu_k, int n_req, cudaStream_t s) {
+                            const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo) {
   using Cfg = Attn3Cfg<D>;
   const int H = heads * D;
   int pairs = 0;
@@ -1061,7 +1061,7 @@ static fps_status launch_d3(const void* q, const void* kv, void* o, int heads,
   const float scale_log2 = 1.4426950408889634f / sqrtf((float)D);
   FPS_CUDA_TRY(launch_k(attn_tc3_kernel<D>, dim3(pairs, heads), dim3(512), Cfg::SMEM, s, tq, tkv,
                         reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads,
-                        scale_log2));
+                        scale_log2, ldo));
 #ifdef FPS_ATTN_TRACE
   {
     static long long h[2][64][8];
@@ -1083,7 +1083,10 @@ static fps_status launch_d3(const void* q, const void* kv, void* o, int heads,
 
 fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads, int head_dim,
                                const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
-                               const int32_t* h_cu_k, int n_req, cudaStream_t s) {
+                               const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo) {
+  if (ldo == 0) ldo = heads * head_dim;
+  if (ldo < heads * head_dim || ldo % 8 != 0)
+    return fail(FPS_EINVAL, "attention_tc: output row stride %d", ldo);
   if (!h_cu_q || !h_cu_k) return fail(FPS_EINVAL, "attention_tc needs host cu_q / cu_k");
   if (!aligned16(q) || !aligned16(kv) || !aligned16(o))
     return fail(FPS_EINVAL, "attention_tc: unaligned operand");
@@ -1095,17 +1098,17 @@ fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads
   // A+B operand reads exceed the 128 B/clk smem port), which ate the latency it saved.
   if (g_attn_force == 0 || g_attn_force == 3) {
     if (head_dim == 128)
-      return launch_d3<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);
-    return launch_d3<64>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);
+      return launch_d3<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo);
+    return launch_d3<64>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo);
   }
   if (g_attn_force == 2) {
     if (head_dim == 128)
-      return launch_d2<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);
-    return launch_d2<64>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);
+      return launch_d2<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo);
+    return launch_d2<64>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo);
   }
   if (head_dim == 128)
-    return launch_d<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);
-  return launch_d<64>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s);
+    return launch_d<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo);
+  return launch_d<64>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo);
 }
 
 }  // namespace fps

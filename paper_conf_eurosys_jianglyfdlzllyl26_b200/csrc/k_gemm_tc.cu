@@ -42,11 +42,11 @@ __device__ __forceinline__ void tile_coords(int tile, int num_m, int num_n, int&
 // column ranges (K/V scatter into the merged key buffer).
 struct RowCtx {
   const __nv_bfloat16* gate;
-  int orow0, orow1;
+  int row, orow0, orow1;
   bool ok;
 };
 __device__ __forceinline__ RowCtx row_ctx(const Epilogue& ep, int M, int row) {
-  RowCtx c{nullptr, row, row, row < M};
+  RowCtx c{nullptr, row, row, row, row < M};
   if (c.ok) {
     if (ep.gate)
       c.gate = reinterpret_cast<const __nv_bfloat16*>(ep.gate) +
@@ -94,7 +94,7 @@ __device__ __forceinline__ void chunk_store(const Epilogue& ep, const RowCtx& rc
 #pragma unroll
       for (int e = 0; e < 8; ++e) v[e] += t[e];
     }
-    if (ep.act == 1) {
+    if (ep.act == 1 && c0 >= ep.act_from) {
 #pragma unroll
       for (int e = 0; e < 8; ++e) v[e] = gelu_tanh_fast(v[e]);
     }
@@ -112,8 +112,10 @@ __device__ __forceinline__ void chunk_store(const Epilogue& ep, const RowCtx& rc
     }
     __nv_bfloat16* dst =
         c0 < ep.split ? reinterpret_cast<__nv_bfloat16*>(ep.out0) + (size_t)rc.orow0 * ep.ld0 + c0
-                      : reinterpret_cast<__nv_bfloat16*>(ep.out1) + (size_t)rc.orow1 * ep.ld1 +
-                            (c0 - ep.split);
+        : (ep.out2 && c0 >= ep.split2)
+            ? reinterpret_cast<__nv_bfloat16*>(ep.out2) + (size_t)rc.row * ep.ld2 + (c0 - ep.split2)
+            : reinterpret_cast<__nv_bfloat16*>(ep.out1) + (size_t)rc.orow1 * ep.ld1 +
+                  (c0 - ep.split);
     *reinterpret_cast<uint4*>(dst) = Vec16<__nv_bfloat16>::pack(v);
   }
 }

@@ -64,6 +64,49 @@ fps_status launch_mask_index(const uint8_t* masks, const int32_t* off, int n_req
 }
 
 // ---------------------------------------------------------------------------------------
+// NEXT-4 (reading R8): pixel mask [Hp, Wp] -> token mask; token (i, j) is active iff any pixel
+// of its f x f block is nonzero; L_txt text tokens appended active.  Thread per token; rows of
+// the block read as 16-B vectors when the geometry allows (f % 16 == 0, Wp % 16 == 0).
+__global__ void __launch_bounds__(256) mask_pool_kernel(const uint8_t* __restrict__ pix, int Hp,
+                                                        int Wp, int f, int L_txt,
+                                                        uint8_t* __restrict__ tok) {
+  const int Wt = Wp / f, T = (Hp / f) * Wt;
+  const int r = blockIdx.y;
+  const int t = blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= T + L_txt) return;
+  uint8_t* out = tok + (size_t)r * (T + L_txt);
+  if (t >= T) {
+    out[t] = 1;
+    return;
+  }
+  const uint8_t* p = pix + (size_t)r * Hp * Wp + (size_t)(t / Wt) * f * Wp + (t % Wt) * f;
+  bool hit = false;
+  if ((f & 15) == 0 && (Wp & 15) == 0 && (reinterpret_cast<uintptr_t>(pix) & 15) == 0) {
+    for (int y = 0; y < f && !hit; ++y)
+      for (int x = 0; x < f; x += 16) {
+        const uint4 v = __ldg(reinterpret_cast<const uint4*>(p + (size_t)y * Wp + x));
+        hit |= (v.x | v.y | v.z | v.w) != 0u;
+      }
+  } else {
+    for (int y = 0; y < f && !hit; ++y)
+      for (int x = 0; x < f; ++x) hit |= __ldg(p + (size_t)y * Wp + x) != 0;
+  }
+  out[t] = hit ? 1 : 0;
+}
+
+fps_status launch_mask_pool(const uint8_t* pix, int n_req, int Hp, int Wp, int f, int L_txt,
+                            uint8_t* tok, cudaStream_t s) {
+  const int T = (Hp / f) * (Wp / f) + L_txt;
+  if (n_req == 0 || T == 0) return FPS_OK;
+  prof::begin(s);
+  mask_pool_kernel<<<dim3(ceil_div(T, 256), n_req), 256, 0, s>>>(pix, Hp, Wp, f, L_txt, tok);
+  prof::end(s, prof::INDEX, 0, (double)n_req * ((double)Hp * Wp + T));
+  count_launch();
+  FPS_LAUNCH_CHECK();
+  return FPS_OK;
+}
+
+// ---------------------------------------------------------------------------------------
 // Row copy by index, 16-B vectors, 4 independent vectors in flight per thread (the source may
 // be mapped pinned host memory read over PCIe, so memory-level parallelism matters).
 __global__ void __launch_bounds__(256) copy_rows_kernel(const uint4* __restrict__ src,

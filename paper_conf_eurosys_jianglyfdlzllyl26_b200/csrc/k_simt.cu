@@ -53,8 +53,8 @@ __global__ void __launch_bounds__(256) gemm_simt_kernel(const T* __restrict__ A,
 fps_status launch_gemm_simt(int dtype, const void* A, const void* B, int M, int N, int K,
                             const Epilogue& ep, cudaStream_t s) {
   if (M <= 0) return FPS_OK;
-  if (N % 4 != 0 || ep.split % 4 != 0)
-    return fail(FPS_EUNSUPPORTED, "gemm_simt: N=%d split=%d must be multiples of 4", N, ep.split);
+  if (N % 4 != 0 || ep.split % 4 != 0 || ep.split2 % 4 != 0 || ep.act_from % 4 != 0)
+    return fail(FPS_EUNSUPPORTED, "gemm_simt: N=%d and the epilogue splits must be multiples of 4", N);
   dim3 grid(ceil_div(N, SBN), ceil_div(M, SBM));
   if (dtype == FPS_BF16)
     gemm_simt_kernel<__nv_bfloat16><<<grid, 256, 0, s>>>(
@@ -74,7 +74,7 @@ __global__ void __launch_bounds__(128) attn_simt_kernel(const T* __restrict__ q,
                                                         T* __restrict__ o, int heads, int total_q,
                                                         const int32_t* __restrict__ cu_q,
                                                         const int32_t* __restrict__ cu_k,
-                                                        int n_req) {
+                                                        int n_req, int ldo) {
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   const int i = gw / heads, j = gw - (gw / heads) * heads;
   if (i >= total_q) return;
@@ -104,7 +104,7 @@ __global__ void __launch_bounds__(128) attn_simt_kernel(const T* __restrict__ q,
     for (int e = 0; e < DPL; ++e) acc[e] = acc[e] * c + p * to_f(vr[e]);
     m = mn;
   }
-  T* op = o + (size_t)i * H + j * d + lane * DPL;
+  T* op = o + (size_t)i * ldo + j * d + lane * DPL;
   const float inv = 1.0f / l;
 #pragma unroll
   for (int e = 0; e < DPL; ++e) op[e] = from_f<T>(acc[e] * inv);
@@ -112,8 +112,9 @@ __global__ void __launch_bounds__(128) attn_simt_kernel(const T* __restrict__ q,
 
 fps_status launch_attention_simt(int dtype, const void* q, const void* kv, void* o, int heads,
                                  int head_dim, const int32_t* cu_q, const int32_t* cu_k,
-                                 int n_req, int total_q, cudaStream_t s) {
+                                 int n_req, int total_q, cudaStream_t s, int ldo) {
   if (total_q <= 0) return FPS_OK;
+  if (ldo == 0) ldo = heads * head_dim;
   const long long warps = (long long)total_q * heads;
   const int grid = (int)((warps * 32 + 127) / 128);
 #define FPS_ATT_CASE(D)                                                                      \
@@ -121,10 +122,10 @@ fps_status launch_attention_simt(int dtype, const void* q, const void* kv, void*
     if (dtype == FPS_BF16)                                                                   \
       attn_simt_kernel<__nv_bfloat16, D / 32><<<grid, 128, 0, s>>>(                          \
           (const __nv_bfloat16*)q, (const __nv_bfloat16*)kv, (__nv_bfloat16*)o, heads,       \
-          total_q, cu_q, cu_k, n_req);                                                       \
+          total_q, cu_q, cu_k, n_req, ldo);                                                       \
     else                                                                                     \
       attn_simt_kernel<float, D / 32><<<grid, 128, 0, s>>>(                                  \
-          (const float*)q, (const float*)kv, (float*)o, heads, total_q, cu_q, cu_k, n_req);  \
+          (const float*)q, (const float*)kv, (float*)o, heads, total_q, cu_q, cu_k, n_req, ldo);  \
     count_launch();                                                                          \
     FPS_LAUNCH_CHECK();                                                                      \
     return FPS_OK;                                                                           \

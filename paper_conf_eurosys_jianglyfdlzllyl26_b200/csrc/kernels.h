@@ -7,6 +7,9 @@ namespace fps {
 // a1
 fps_status launch_mask_index(const uint8_t* masks, const int32_t* off, int n_req, int max_len,
                              int32_t* mids, int32_t* uids, int32_t* nm, cudaStream_t s);
+// NEXT-4: pixel mask -> token mask (max-pool over f x f blocks, text tokens appended active)
+fps_status launch_mask_pool(const uint8_t* pix, int n_req, int Hp, int Wp, int f, int L_txt,
+                            uint8_t* tok, cudaStream_t s);
 // a2/a9/a3 row movement: dst[dst_ids? dst_ids[i] : i] = src[src_ids ? src_ids[i] : i]
 fps_status launch_copy_rows(const void* src, const int32_t* src_ids, const int32_t* dst_ids,
                             int n, int row_bytes, void* dst, cudaStream_t s, int max_ctas = 0);
@@ -25,17 +28,18 @@ fps_status launch_gemm_simt(int dtype, const void* A, const void* B, int M, int 
 fps_status launch_gemm_tc(const void* A, const void* B, int M, int N, int K, const Epilogue& ep,
                           cudaStream_t s);
 bool gemm_tc_supported(int dtype, int M, int N, int K);
-// a6: o[i, head] = softmax(q_i k^T / sqrt(d)) v over the request's merged keys
+// a6: o[i, head] = softmax(q_i k^T / sqrt(d)) v over the request's merged keys; o rows are
+// ldo elements apart (0 = heads * head_dim)
 fps_status launch_attention(int dtype, const void* q, const void* kv, void* o, int heads,
                             int head_dim, const int32_t* d_cu_q, const int32_t* d_cu_k,
                             const int32_t* h_cu_q, const int32_t* h_cu_k, int n_req, int total_q,
-                            int max_q, int max_k, cudaStream_t s);
+                            int max_q, int max_k, cudaStream_t s, int ldo = 0);
 fps_status launch_attention_simt(int dtype, const void* q, const void* kv, void* o, int heads,
                                  int head_dim, const int32_t* cu_q, const int32_t* cu_k,
-                                 int n_req, int total_q, cudaStream_t s);
+                                 int n_req, int total_q, cudaStream_t s, int ldo = 0);
 fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads, int head_dim,
                                const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
-                               const int32_t* h_cu_k, int n_req, cudaStream_t s);
+                               const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo = 0);
 bool attention_tc_supported(int dtype, int head_dim);
 
 // true if fps_cache_prefetch also overwrites rows outside U (copy_method 2): fresh rows written

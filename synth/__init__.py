@@ -89,8 +89,22 @@ CONFIGS = {
 }
 
 
-def block_weights(g: np.random.Generator, H: int, F: int, dtype: str = "bf16") -> dict:
-    """nn.Linear layout: W[out, in]. Q/K/V stacked as rows [0,H), [H,2H), [2H,3H) of w_qkv."""
+def block_weights(g: np.random.Generator, H: int, F: int, dtype: str = "bf16",
+                  kind: str = "seq") -> dict:
+    """nn.Linear layout: W[out, in]. Q/K/V stacked as rows [0,H), [H,2H), [2H,3H) of w_qkv.
+
+    kind="par" (parallel block, NEXT-2): w_1 [3H+F, H] stacks Q, K, V and the MLP input rows;
+    w_2 [H, H+F] maps the concatenation [attention | GELU(MLP)] back to H."""
+    if kind == "par":
+        w = {
+            "w_1": g.standard_normal((3 * H + F, H), dtype=np.float32) / math.sqrt(H),
+            "b_1": 0.02 * g.standard_normal(3 * H + F, dtype=np.float32),
+            "w_2": g.standard_normal((H, H + F), dtype=np.float32) / math.sqrt(H + F),
+            "b_2": 0.02 * g.standard_normal(H, dtype=np.float32),
+        }
+        out = {k: _store(v, dtype) for k, v in w.items()}
+        out["kind"] = "par"
+        return out
     w = {
         "w_qkv": g.standard_normal((3 * H, H), dtype=np.float32) / math.sqrt(H),
         "b_qkv": 0.02 * g.standard_normal(3 * H, dtype=np.float32),
@@ -104,8 +118,9 @@ def block_weights(g: np.random.Generator, H: int, F: int, dtype: str = "bf16") -
     return {k: _store(v, dtype) for k, v in w.items()}
 
 
-def stack_weights(g: np.random.Generator, layers: int, H: int, F: int, dtype: str = "bf16"):
-    return [block_weights(g, H, F, dtype) for _ in range(layers)]
+def stack_weights(g: np.random.Generator, layers: int, H: int, F: int, dtype: str = "bf16",
+                  kind: str = "seq"):
+    return [block_weights(g, H, F, dtype, kind) for _ in range(layers)]
 
 
 def mod_table(g: np.random.Generator, layers: int, steps: int, H: int, dtype: str = "bf16",

@@ -21,9 +21,9 @@ def F():
     return fps
 
 
-def _problem(seed, dtype, H, heads, Fd, L_img, L_txt, ratios, mod=True, blobs=False):
+def _problem(seed, dtype, H, heads, Fd, L_img, L_txt, ratios, mod=True, blobs=False, kind="seq"):
     g = synth.rng(seed)
-    w = synth.block_weights(g, H, Fd, dtype)
+    w = synth.block_weights(g, H, Fd, dtype, kind)
     reqs = []
     for m in ratios:
         L = L_img + L_txt
@@ -45,7 +45,7 @@ def _problem(seed, dtype, H, heads, Fd, L_img, L_txt, ratios, mod=True, blobs=Fa
 
 def _run_masked(F, w, reqs, heads, dtype, mode):
     dt = F.DTYPE_CODE[dtype]
-    H = w["w_o"].shape[0]
+    H = (w["w_2"] if w.get("kind") == "par" else w["w_o"]).shape[0]
     bw = F.BlockWeights(w, heads, dt)
     Ls = [r["L"] for r in reqs]
     cu_k = np.concatenate([[0], np.cumsum(Ls)])
@@ -175,3 +175,44 @@ def test_flux_scale_sampled_rows(F):
     a = B.attention(Q, Kall, Vall, heads)
     ref = B._attn_out_and_mlp(x[M][sample], a, w, mod, H)
     check_close(y[sample], ref, TOL["bf16"], "flux sampled")
+
+
+# ---- NEXT-2: parallel (Flux single-stream) block, reading R23 ------------------------------
+@pytest.mark.parametrize("mode", ["kv", "y"])
+def test_parallel_fp32_masked(F, mode):
+    w, reqs = _problem(4001, "f32", 64, 2, 256, 256, 8, [0.25, 0.6], kind="par")
+    y, _ = _run_masked(F, w, reqs, 2, "f32", mode)
+    check_close(y, _ref_masked(w, reqs, 2, mode), TOL["f32"], f"parallel fp32 {mode}")
+
+
+@pytest.mark.parametrize("mode", ["kv", "y"])
+@pytest.mark.parametrize("simt", [False, True])
+def test_parallel_bf16_varlen_batch(F, mode, simt):
+    w, reqs = _problem(4002, "bf16", 256, 2, 1024, 576, 40, [0.05, 0.6, 0.3], blobs=True,
+                       kind="par")
+    F.fps_set_disable_tc(3 if simt else 0)
+    try:
+        y, _ = _run_masked(F, w, reqs, 2, "bf16", mode)
+    finally:
+        F.fps_set_disable_tc(0)
+    check_close(y, _ref_masked(w, reqs, 2, mode), TOL["bf16"], f"parallel bf16 {mode} simt={simt}")
+
+
+def test_parallel_dense_and_head64(F):
+    w, reqs = _problem(4003, "bf16", 640, 10, 2560, 300, 20, [1.0], kind="par")
+    r = reqs[0]
+    bw = F.BlockWeights(w, 10, F.FPS_BF16)
+    b = F.VarlenBatch([r["L"]], [r["L"]], mod=to_dev(r["mod"][None], "bf16"))
+    y, _ = F.dense_block_forward(bw, b, to_dev(r["x"], "bf16"))
+    torch.cuda.synchronize()
+    ref, _, _ = B.dense_block(r["x"], w, r["mod"], 10)
+    check_close(to_np(y), ref, TOL["bf16"], "parallel dense H=640")
+
+
+def test_parallel_weights_validated(F):
+    w, _ = _problem(4004, "bf16", 128, 2, 512, 64, 0, [0.5], kind="par")
+    bw = F.BlockWeights(w, 2, F.FPS_BF16)
+    bw.c.w_o = bw.c.w_qkv                         # a sequential-only pointer set -> EINVAL
+    b = F.VarlenBatch([64], [64])
+    with pytest.raises(F.FlashPSError):
+        F.dense_block_forward(bw, b, torch.zeros(64, 128, dtype=torch.bfloat16, device="cuda"))

@@ -19,9 +19,10 @@ def F():
 
 
 def _setup(F, mode, dtype, plan_policy, plan=None, N=3, steps=3, H=256, heads=2, Fd=512,
-           L_img=256, L_txt=16, n_req=3, slots=0, copy_method=0, seed=5000, location=0):
+           L_img=256, L_txt=16, n_req=3, slots=0, copy_method=0, seed=5000, location=0,
+           kind="seq"):
     g = synth.rng(seed)
-    W = synth.stack_weights(g, N, H, Fd, dtype)
+    W = synth.stack_weights(g, N, H, Fd, dtype, kind)
     mods = synth.mod_table(g, N, steps, H, dtype)
     deltas = synth.delta_table(steps)
     L = L_img + L_txt
@@ -89,6 +90,21 @@ def test_run_batch_matches_oracle(F, mode, dtype, policy, plan):
     for r, x in zip(reqs, ref):
         check_close(to_np(r["x"]), x, stack_tol(dtype, 3), f"{mode} {dtype} plan={used}")
         assert r["step"] == min(r["step0"] + 2, r["n_steps"])
+
+
+@pytest.mark.parametrize("mode,dtype,policy,plan", [
+    ("kv", "bf16", 1, None), ("y", "bf16", 3, [1, 0, 1]), ("kv", "f32", 3, [0, 1, 1])])
+def test_run_batch_parallel_blocks(F, mode, dtype, policy, plan):
+    """A stack of parallel (Flux single-stream) blocks through fps_run_batch (NEXT-2, R23)."""
+    W, mods, deltas, cache_np, eng, reqs = _setup(F, mode, dtype, policy, plan, kind="par")
+    for r in reqs:
+        r["step0"] = r["step"]
+    eng.run_batch(reqs, 2)
+    torch.cuda.synchronize()
+    used = eng.last_plan()[0]
+    ref = _oracle(W, mods, deltas, cache_np, reqs, used, mode, 2, 2)
+    for r, x in zip(reqs, ref):
+        check_close(to_np(r["x"]), x, stack_tol(dtype, 3), f"parallel {mode} {dtype} plan={used}")
 
 
 @pytest.mark.parametrize("mode", ["kv", "y"])

@@ -128,3 +128,28 @@ def test_cache_store_prefetch_bytes_equal(F, mode, method, location):
             exp[ids[r]] = ents[(t, s, layer)][ids[r]]
             assert np.array_equal(got[base:base + L_img + L_txt], exp)
     c.close()
+
+
+@pytest.mark.parametrize("Hp,Wp,f,L_txt,n_req,p", [(1024, 1024, 16, 512, 2, 0.0005),
+                                                  (1024, 1024, 32, 0, 3, 0.0002),
+                                                  (30, 45, 3, 5, 2, 0.02), (64, 48, 16, 0, 1, 0.0),
+                                                  (64, 64, 16, 3, 1, 1.0), (8, 8, 1, 0, 1, 0.3),
+                                                  (96, 80, 8, 1, 4, 0.01)])
+def test_mask_to_tokens_bit_exact(F, Hp, Wp, f, L_txt, n_req, p):
+    from oracle.index import pixel_to_token_mask
+    g = synth.rng(Hp + Wp + f)
+    pix = (g.random((n_req, Hp, Wp)) < p).astype(np.uint8)
+    if Hp >= 64:                                    # plus an irregular blob region
+        yy, xx = np.mgrid[:Hp, :Wp]
+        pix[0] |= (((yy - Hp / 3) / (Hp / 6)) ** 2 + ((xx - Wp / 2) / (Wp / 5)) ** 2 < 1).astype(np.uint8)
+    tok = F.mask_to_tokens(torch.as_tensor(pix).cuda(), f, L_txt)
+    torch.cuda.synchronize()
+    got = tok.cpu().numpy()
+    for r in range(n_req):
+        assert got[r].tolist() == pixel_to_token_mask(pix[r], f, L_txt).tolist()
+
+
+def test_mask_to_tokens_rejects_bad_geometry(F):
+    pix = torch.zeros(1, 30, 40, dtype=torch.uint8, device="cuda")
+    with pytest.raises(F.FlashPSError):
+        F.mask_to_tokens(pix, 16)

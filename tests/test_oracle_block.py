@@ -164,3 +164,79 @@ def test_token_wise_rows_independent():
     y1, _, _ = B.masked_block_kv(x[M], M, U, K[U], V[U], w, m, 3, 32)
     y2, _, _ = B.masked_block_kv(x[M][::-1].copy(), M[::-1].copy(), U, K[U], V[U], w, m, 3, 32)
     assert np.allclose(y1, y2[::-1], atol=1e-12)
+
+
+# ---- NEXT-2: parallel (Flux single-stream) block, reading R23 ------------------------------
+def _setup_par(seed=0, H=48, heads=3, F=80, L=40, dtype="f32"):
+    g = synth.rng(seed)
+    w = synth.block_weights(g, H, F, dtype, kind="par")
+    x = synth.latent(g, L, H, dtype)
+    m = synth.mod_table(g, 1, 1, H, dtype)[0, 0]
+    return g, w, x, m
+
+
+def _torch_parallel_block(x, w, mod, heads):
+    """The parallel block from torch library modules in float64: nn.MultiheadAttention takes
+    W1's Q/K/V rows and W2's first H columns as its output projection; the MLP branch is two
+    nn.Linear layers over W1's last F rows and W2's last F columns."""
+    H = x.shape[1]
+    F = w["w_1"].shape[0] - 3 * H
+    W1, b1 = np.asarray(w["w_1"], np.float64), np.asarray(w["b_1"], np.float64)
+    W2 = np.asarray(w["w_2"], np.float64)
+    mha = torch.nn.MultiheadAttention(H, heads, bias=True, batch_first=True)
+    up, dn = torch.nn.Linear(H, F), torch.nn.Linear(F, H)
+    with torch.no_grad():
+        mha.in_proj_weight.copy_(torch.tensor(W1[:3 * H])); mha.in_proj_bias.copy_(torch.tensor(b1[:3 * H]))
+        mha.out_proj.weight.copy_(torch.tensor(W2[:, :H])); mha.out_proj.bias.zero_()
+        up.weight.copy_(torch.tensor(W1[3 * H:])); up.bias.copy_(torch.tensor(b1[3 * H:]))
+        dn.weight.copy_(torch.tensor(W2[:, H:])); dn.bias.copy_(torch.tensor(np.asarray(w["b_2"], np.float64)))
+        sh1, sc1, g1 = torch.tensor(np.asarray(mod, np.float64)).view(6, H)[:3]
+        xt = torch.tensor(np.asarray(x, np.float64))[None]
+        h = Fn.layer_norm(xt, (H,), eps=1e-6) * (1 + sc1) + sh1
+        a, _ = mha(h, h, h, need_weights=False)
+        y = xt + g1 * (a + dn(Fn.gelu(up(h), approximate="tanh")))
+    return y[0].numpy()
+
+
+def test_parallel_block_vs_torch_modules():
+    _, w, x, m = _setup_par()
+    y, K, V = B.dense_block(x, w, m, 3)
+    assert np.allclose(y, _torch_parallel_block(x, w, m, 3), rtol=0, atol=1e-10)
+    # K, V are W1's rows [H, 3H) applied to the normalised input
+    H = x.shape[1]
+    mm = np.asarray(m, np.float64).reshape(6, H)
+    h = B.layer_norm(x) * (1 + mm[1]) + mm[0]
+    assert np.allclose(K, h @ np.asarray(w["w_1"], np.float64)[H:2 * H].T + w["b_1"][H:2 * H], atol=1e-12)
+
+
+def test_parallel_block_zero_weights_closed_form():
+    """W1 = W2 = 0: y = x + gate1 * b2 (the MLP branch GELU(b1) meets a zero W2)."""
+    _, w, x, m = _setup_par(seed=3)
+    w["w_1"], w["w_2"] = np.zeros_like(w["w_1"]), np.zeros_like(w["w_2"])
+    y, _, _ = B.dense_block(x, w, m, 3)
+    H = x.shape[1]
+    assert np.allclose(y, x + m.reshape(6, H)[2] * w["b_2"], atol=1e-12)
+
+
+@pytest.mark.parametrize("ratio", [0.0, 0.3, 1.0])
+def test_parallel_masked_equals_dense_under_identical_input_cache(ratio):
+    g, w, x, m = _setup_par(seed=19, L=64)
+    mask = synth.mask_blobs(g, 8, 8, ratio)
+    M, U = build_mask_index(mask)
+    y_ref, K, V = B.dense_block(x, w, m, 3)
+    y_kv, K_M, V_M = B.masked_block_kv(x[M], M, U, K[U], V[U], w, m, 3, 64)
+    y_y = B.masked_block_y(x[M], M, U, x[U], w, m, 3, 64)
+    assert np.allclose(y_kv, y_ref[M], rtol=0, atol=1e-12)
+    assert np.allclose(y_y, y_ref[M], rtol=0, atol=1e-12)
+    assert np.allclose(K_M, K[M], atol=1e-12) and np.allclose(V_M, V[M], atol=1e-12)
+
+
+def test_parallel_cache_is_actually_used():
+    g, w, x, m = _setup_par(seed=23, L=64)
+    mask = synth.mask_random(g, 64, 0.25)
+    M, U = build_mask_index(mask)
+    x_t = synth.latent(g, 64, x.shape[1], "f32")
+    _, Kt, Vt = B.dense_block(x_t, w, m, 3)
+    y_kv, _, _ = B.masked_block_kv(x[M], M, U, Kt[U], Vt[U], w, m, 3, 64)
+    y_ref, _, _ = B.dense_block(x, w, m, 3)
+    assert not np.allclose(y_kv, y_ref[M], atol=1e-3)

@@ -52,3 +52,37 @@ def test_gather_scatter_roundtrip_bit_exact():
     scatter_rows(xm, M, out)
     scatter_rows(xu, U, out)
     assert np.array_equal(out.view(np.uint32), x.view(np.uint32))    # identity, bit-exact
+
+
+# ---- NEXT-4: pixel mask -> token mask (reading R8) -------------------------------------------
+from oracle.index import pixel_to_token_mask
+
+
+def test_pixel_to_token_golden():
+    # hand-derived: 4 x 6 pixels, f = 2 -> 2 x 3 tokens; pixels set at (0,0), (3,5), (2,2)
+    pix = np.zeros((4, 6), np.uint8)
+    pix[0, 0] = pix[3, 5] = pix[2, 2] = 1
+    # token (0,0) covers rows 0-1 cols 0-1 -> 1; (1,2) covers rows 2-3 cols 4-5 -> 1;
+    # (1,1) covers rows 2-3 cols 2-3 -> 1; all others 0; then 2 text tokens
+    assert pixel_to_token_mask(pix, 2, 2).tolist() == [1, 0, 0, 0, 1, 1, 1, 1]
+
+
+def test_pixel_to_token_vs_reshape_max_and_identities():
+    g = synth.rng(21)
+    for (Hp, Wp, f) in ((32, 48, 4), (30, 45, 3), (64, 64, 16), (16, 16, 1), (40, 8, 8)):
+        pix = (g.random((Hp, Wp)) < 0.02).astype(np.uint8)
+        tok = pixel_to_token_mask(pix, f, 3)
+        ref = pix.reshape(Hp // f, f, Wp // f, f).max(axis=(1, 3)).reshape(-1)  # library max-pool
+        assert tok[:-3].tolist() == (ref != 0).astype(np.uint8).tolist()
+        assert tok[-3:].tolist() == [1, 1, 1]
+        if f == 1:
+            assert tok[:-3].tolist() == (pix.reshape(-1) != 0).tolist()       # identity
+    # monotone: adding masked pixels never clears a token; empty / full masks
+    pix = np.zeros((64, 64), np.uint8)
+    assert pixel_to_token_mask(pix, 16).sum() == 0
+    assert pixel_to_token_mask(pix + 1, 16).sum() == 16
+    pix[5, 7] = 1
+    a = pixel_to_token_mask(pix, 16)
+    pix[40, 60] = 1
+    b = pixel_to_token_mask(pix, 16)
+    assert np.all(b >= a) and a.sum() == 1 and b.sum() == 2

@@ -6,9 +6,9 @@ import synth
 from oracle import stack as S
 
 
-def _setup(N=3, steps=2, H=32, heads=2, F=64, L_img=36, L_txt=4, seed=0):
+def _setup(N=3, steps=2, H=32, heads=2, F=64, L_img=36, L_txt=4, seed=0, kind="seq"):
     g = synth.rng(seed)
-    W = synth.stack_weights(g, N, H, F, "f32")
+    W = synth.stack_weights(g, N, H, F, "f32", kind)
     mods = synth.mod_table(g, N, steps, H, "f32")
     x0 = synth.latent(g, L_img + L_txt, H, "f32")
     return g, W, mods, x0, synth.delta_table(steps)
@@ -19,10 +19,12 @@ PLANS_Y = PLANS_KV + [[1, 0, 1], [1, 1, 0], [0, 1, 0], [1, 0, 0]]
 
 
 @pytest.mark.parametrize("mode,plan", [("kv", p) for p in PLANS_KV] + [("y", p) for p in PLANS_Y])
-def test_identical_input_cache_reproduces_template(mode, plan):
+@pytest.mark.parametrize("kind", ["seq", "par"])
+def test_identical_input_cache_reproduces_template(mode, plan, kind):
     """L144/L157 + L211: with the cache from the template run on the identical input, every
-    feasible plan reproduces the dense trajectory over a whole stack and several steps."""
-    g, W, mods, x0, deltas = _setup()
+    feasible plan reproduces the dense trajectory over a whole stack and several steps (both
+    block kinds)."""
+    g, W, mods, x0, deltas = _setup(kind=kind)
     cache, xs = S.template_run(x0, W, mods, deltas, 2, 2)
     mask = synth.token_mask(synth.mask_blobs(g, 6, 6, 0.3), 4)
     x = S.masked_run(x0, mask, W, mods, deltas, plan, mode, cache, 2, 2)
