@@ -359,7 +359,9 @@ def main():
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()
     import faulthandler                   # a stuck run dumps every thread's stack and exits
+    import signal
     faulthandler.dump_traceback_later(900, exit=True)
+    faulthandler.register(signal.SIGUSR1, all_threads=True)   # `timeout -s USR1`: dump stacks
     if args.copy_method is None:
         # measured on B200 (C3): pinned host tier -- batched DMA of the unmasked row runs 32.8
         # ms/step vs 36.7 with whole-entry DMA (-20% bytes at the same 55 GB/s) and 43.3 with the
@@ -480,10 +482,12 @@ def main():
     if not args.no_extras:
         log(f"[rank {rank}] extras")
         # same batch, every block dense (all tokens, no cache): the compute-saving reference
+        log(f"[rank {rank}] extras: dense")
         eng_d = engine(2)
         dense_ms, _ = run_engine_timed(F, eng_d, reqs_dev, K, W, stream, load_stream, rank, world)
         del eng_d
         # all blocks cached (no planner) and the HBM-resident "ideal" (no loads at all)
+        log(f"[rank {rank}] extras: all cached")
         eng_c = engine(1)
         cached_ms, _ = run_engine_timed(F, eng_c, reqs_dev, K, W, stream, load_stream, rank, world)
         del eng_c
@@ -491,6 +495,7 @@ def main():
         # the same plan with every cache entry already resident in HBM: the step without any
         # host-link load; exposed load = this step - that step
         if location != 1:
+            log(f"[rank {rank}] extras: same plan, HBM-resident cache")
             c_h = make_cache(F, w, args.mode, n_entries, 1, 2)
             eng_h = F.Engine(layers, w["heads"], F.MODE_CODE[args.mode], F.FPS_BF16, w["L_img"],
                              w["L_txt"], max(len(reqs_dev), 1), w["steps"], deltas, c_h,
@@ -511,6 +516,7 @@ def main():
                                (args.mode, location, 2 if args.copy_method != 2 else 1)):
             if loc == 1 and cmeth == 1:
                 continue
+            log(f"[rank {rank}] extras: mode {md} location {loc} copy method {cmeth}")
             c2 = make_cache(F, w, md, n_entries, loc, cmeth)
             cm2, _ = calibrate(F, w, md, layers, c2, [dict()] * w["batch"], device)
             eng_o = F.Engine(layers, w["heads"], F.MODE_CODE[md], F.FPS_BF16, w["L_img"],

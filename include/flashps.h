@@ -53,7 +53,9 @@ int32_t fps_device_ok(void);
  * bits 2-3 = 1 force the 1-SM tcgen05 GEMM, = 2 force the CTA-pair (cta_group::2) GEMM;
  * bits 4-5 = 1 force the one-query-tile attention kernel, = 2 the two-tile kernel with P in
  * shared memory, = 3 the two-tile kernel with P in TMEM and a correction warpgroup (the default);
- * bit 6 = launch without programmatic dependent launch (PDL is on by default). */
+ * bit 6 = launch without programmatic dependent launch (PDL is on by default);
+ * bit 7 = HBM-arena whole-entry prefetch by driver device-to-device memcpy instead of the
+ * library copy kernel (experiments only: see cache.cu). */
 int64_t fps_launch_count(void);
 void fps_set_disable_tc(int32_t flags);
 /* Per-kernel-class timing for the bench: when enabled (this also clears old records) every

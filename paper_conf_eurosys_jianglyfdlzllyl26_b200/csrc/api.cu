@@ -12,6 +12,7 @@ static thread_local std::string g_err;
 thread_local long long g_launches = 0;
 int g_disable_tc = 0;
 int g_pdl = 1;
+thread_local PdlFence g_pdl_fence;
 
 void set_error(const char* fmt, ...) {
   char buf[1024];
@@ -203,7 +204,7 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
   }
   if (tu > 0) {
     // Y-mode: cached block-input rows U -> LN -> K|V projection (Fig. 5-Bottom, reading R5)
-    if (kv_ready) FPS_CUDA_TRY(cudaStreamWaitEvent(s, kv_ready, 0));
+    if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
     kv_ready = nullptr;
     FPS_TRY(launch_ln_mod(dt, xu, b->d_u_src, tu, H, ws.hu, b->d_cu_u, b->n_req, b->d_mod, 0, s));
     Epilogue ep{};
@@ -216,7 +217,7 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
   if (w->kind == FPS_BLOCK_PAR) {
     // parallel block (reading R23): ws.ao..ws.u hold cat = [A | GELU(Z)], [tq, H+F]
     char* cat = ws.ao;
-    if (kv_ready) FPS_CUDA_TRY(cudaStreamWaitEvent(s, kv_ready, 0));
+    if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
     FPS_TRY(launch_attention(dt, ws.q, kv, cat, w->heads, w->head_dim, b->d_cu_q, b->d_cu_k,
                              b->h_cu_q, b->h_cu_k, b->n_req, tq, b->max_q, b->max_k, s, H + F));
     Epilogue ep{};
@@ -227,7 +228,7 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
     return launch_gemm(dt, cat, w->w_down, tq, H, H + F, ep, s);
   }
   // a6: queries from active rows only, keys = merged fresh + cached rows (L159)
-  if (kv_ready) FPS_CUDA_TRY(cudaStreamWaitEvent(s, kv_ready, 0));
+  if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
   FPS_TRY(launch_attention(dt, ws.q, kv, ws.ao, w->heads, w->head_dim, b->d_cu_q, b->d_cu_k,
                            b->h_cu_q, b->h_cu_k, b->n_req, tq, b->max_q, b->max_k, s));
   {  // a7: x1 = x + gate1 (A Wo^T + bo)
@@ -315,6 +316,7 @@ void fps_set_disable_tc(int32_t flags) {
   fps::g_gemm_force = (flags >> 2) & 3;
   fps::g_attn_force = (flags >> 4) & 3;
   fps::g_pdl = (flags & 64) ? 0 : 1;
+  fps::g_d2d_kernel = (flags & 128) ? 0 : 1;
 }
 
 fps_status fps_build_mask_index(const uint8_t* d_masks, const int32_t* d_offsets, int32_t n_req,

@@ -105,6 +105,7 @@ static size_t offset_of(const fps_cache* c, uint32_t t, int step, int layer) {
   return (size_t)(key_of(c, t, step, layer) % c->n_entries) * c->entry_bytes;
 }
 
+int g_d2d_kernel = 1;   // experiments: 0 = driver D2D memcpy for HBM whole-entry loads
 bool cache_writes_all_rows(const fps_cache* c) { return c && c->d.copy_method == 2; }
 
 }  // namespace fps
@@ -259,8 +260,17 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
       const fps_prefetch_item& it = items[i];
       if (it.n_rows == 0) continue;
       const size_t nb = (size_t)c->d.L_img * row_bytes_of(c, it.layer);
-      FPS_CUDA_TRY(cudaMemcpyAsync(it.d_dst, c->host + offset_of(c, it.template_id, it.step, it.layer),
-                                   nb, cudaMemcpyDefault, s));
+      const char* src = c->host + offset_of(c, it.template_id, it.step, it.layer);
+      if (c->d.location == 1 && g_d2d_kernel) {
+        // HBM arena: device-to-device entry copy by our own kernel (launched without PDL).
+        // A driver cudaMemcpyAsync D2D here, with PDL launches on the compute stream, hung
+        // the C2B stack deterministically (tools/hang_probe.py: plan 21 dense + 39 cached).
+        pdl_fence(s);
+        FPS_TRY(launch_copy_rows(src, nullptr, nullptr, c->d.L_img, (int)row_bytes_of(c, it.layer),
+                                 it.d_dst, s, 0, false));
+      } else {
+        FPS_COPY_TRY(s, cudaMemcpyAsync(it.d_dst, src, nb, cudaMemcpyDefault, s));
+      }
       bytes += nb;
     }
     prof::end(s, prof::PREFETCH, 0, bytes);
@@ -336,7 +346,7 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
     if (s == 0 || s == cudaStreamLegacy) {
       // the batch API rejects the legacy default stream: one DMA per run there
       for (size_t q = 0; q < c->sizes.size(); ++q)
-        FPS_CUDA_TRY(cudaMemcpyAsync(c->dsts[q], c->srcs[q], c->sizes[q], cudaMemcpyDefault, s));
+        FPS_COPY_TRY(s, cudaMemcpyAsync(c->dsts[q], c->srcs[q], c->sizes[q], cudaMemcpyDefault, s));
     } else if (!c->sizes.empty()) {
       cudaMemcpyAttributes a{};
       a.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
@@ -347,6 +357,7 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
       a.dstLocHint.id = dev;
       a.flags = cudaMemcpyFlagPreferOverlapWithCompute;
       size_t attr_idx = 0, fail_idx = ~size_t(0);
+      pdl_fence(s);
       const cudaError_t e = cudaMemcpyBatchAsync(c->dsts.data(), c->srcs.data(), c->sizes.data(),
                                                  c->sizes.size(), &a, &attr_idx, 1, &fail_idx, s);
       if (e != cudaSuccess) {

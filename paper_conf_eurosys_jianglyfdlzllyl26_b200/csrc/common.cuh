@@ -59,6 +59,41 @@ __device__ __forceinline__ void pdl_trigger() {
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 }
 extern int g_pdl;   // 1 = launch with PDL (default), 0 = plain launches (fps_set_disable_tc bit 6)
+// Set by every cross-stream wait / copy the library enqueues: the next kernel is launched
+// WITHOUT the PDL attribute, so PDL only ever overlaps two back-to-back library kernels.
+// Measured on B200: a PDL launch right after cudaStreamWaitEvent on a load-stream device-to-
+// device copy (HBM-tier whole-entry DMA) hung intermittently (3 of 6 C2B bench runs; 0 of 6
+// without PDL) -- the early-resident CTAs of a persistent kernel fill every SM while the event's
+// producer still needs them.
+struct PdlFence {             // streams whose next library kernel must not use PDL
+  cudaStream_t s[8];
+  int n = 0;
+  void add(cudaStream_t st) {
+    for (int i = 0; i < n; ++i)
+      if (s[i] == st) return;
+    if (n < 8) s[n++] = st;
+    else s[7] = st;
+  }
+  bool take(cudaStream_t st) {
+    for (int i = 0; i < n; ++i)
+      if (s[i] == st) {
+        s[i] = s[--n];
+        return true;
+      }
+    return false;
+  }
+};
+extern thread_local PdlFence g_pdl_fence;
+inline cudaError_t stream_wait(cudaStream_t s, cudaEvent_t ev, unsigned flags = 0) {
+  g_pdl_fence.add(s);
+  return cudaStreamWaitEvent(s, ev, flags);
+}
+inline void pdl_fence(cudaStream_t s) { g_pdl_fence.add(s); }
+#define FPS_COPY_TRY(stream, x) \
+  do {                          \
+    ::fps::pdl_fence(stream);   \
+    FPS_CUDA_TRY(x);            \
+  } while (0)
 
 template <typename... KArgs, typename... Args>
 inline cudaError_t launch_k(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem,
@@ -70,7 +105,8 @@ inline cudaError_t launch_k(void (*kernel)(KArgs...), dim3 grid, dim3 block, siz
   cfg.stream = s;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  attr[0].val.programmaticStreamSerializationAllowed = g_pdl;
+  const bool fenced = g_pdl_fence.take(s);
+  attr[0].val.programmaticStreamSerializationAllowed = (g_pdl && !fenced) ? 1 : 0;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
   return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);

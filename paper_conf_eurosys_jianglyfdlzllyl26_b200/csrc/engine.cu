@@ -209,16 +209,16 @@ static fps_status admit(fps_engine* e, fps_request* reqs, const std::vector<int>
   B.n = n;
   B.idx = live;
   for (int i = 0; i < n; ++i) {
-    FPS_CUDA_TRY(cudaMemcpyAsync(e->d_masks + (size_t)i * L, reqs[live[i]].d_mask, L,
+    FPS_COPY_TRY(cs, cudaMemcpyAsync(e->d_masks + (size_t)i * L, reqs[live[i]].d_mask, L,
                                  cudaMemcpyDeviceToDevice, cs));
     e->h_off[i] = i * L;
   }
   e->h_off[n] = n * L;
-  FPS_CUDA_TRY(cudaMemcpyAsync(e->d_off, e->h_off, (n + 1) * 4, cudaMemcpyHostToDevice, cs));
+  FPS_COPY_TRY(cs, cudaMemcpyAsync(e->d_off, e->h_off, (n + 1) * 4, cudaMemcpyHostToDevice, cs));
   FPS_TRY(launch_mask_index(e->d_masks, e->d_off, n, L, e->d_mids, e->d_uids, e->d_nm, cs));
-  FPS_CUDA_TRY(cudaMemcpyAsync(e->h_nm, e->d_nm, n * 4, cudaMemcpyDeviceToHost, cs));
-  FPS_CUDA_TRY(cudaMemcpyAsync(e->h_mids, e->d_mids, (size_t)n * L * 4, cudaMemcpyDeviceToHost, cs));
-  FPS_CUDA_TRY(cudaMemcpyAsync(e->h_uids, e->d_uids, (size_t)n * L * 4, cudaMemcpyDeviceToHost, cs));
+  FPS_COPY_TRY(cs, cudaMemcpyAsync(e->h_nm, e->d_nm, n * 4, cudaMemcpyDeviceToHost, cs));
+  FPS_COPY_TRY(cs, cudaMemcpyAsync(e->h_mids, e->d_mids, (size_t)n * L * 4, cudaMemcpyDeviceToHost, cs));
+  FPS_COPY_TRY(cs, cudaMemcpyAsync(e->h_uids, e->d_uids, (size_t)n * L * 4, cudaMemcpyDeviceToHost, cs));
   FPS_CUDA_TRY(cudaEventRecord(e->admit_done, cs));
   FPS_CUDA_TRY(cudaEventSynchronize(e->admit_done));   // the one admission sync
   // host metadata, laid out in h_meta exactly like d_meta
@@ -247,7 +247,7 @@ static fps_status admit(fps_engine* e, fps_request* reqs, const std::vector<int>
   B.tk = cu_k[n];
   B.tu = cu_u[n];
   (void)mod_ids;
-  FPS_CUDA_TRY(cudaMemcpyAsync(e->d_meta, e->h_meta,
+  FPS_COPY_TRY(cs, cudaMemcpyAsync(e->d_meta, e->h_meta,
                                (size_t)(3 * (nb + 1) + 2 * e->maxR) * 4, cudaMemcpyHostToDevice, cs));
   int32_t* dm = e->d_meta;
   B.cu_q = dm;
@@ -303,12 +303,12 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
     int32_t* mod_ids = e->h_meta + 3 * (e->d.max_batch + 1) + 2 * e->maxR;
     for (int l = 0; l < N; ++l)
       for (int i = 0; i < n; ++i) mod_ids[l * n + i] = l * e->d.n_steps + reqs[B.idx[i]].step;
-    FPS_CUDA_TRY(cudaMemcpyAsync(B.mod_ids, mod_ids, (size_t)N * n * 4, cudaMemcpyHostToDevice, cs));
+    FPS_COPY_TRY(cs, cudaMemcpyAsync(B.mod_ids, mod_ids, (size_t)N * n * 4, cudaMemcpyHostToDevice, cs));
     FPS_TRY(launch_copy_rows(e->d.d_mod_table, B.mod_ids, nullptr, N * n, 6 * (int)e->row_h,
                              e->mod_batch, cs));
   }
   for (int i = 0; i < n; ++i) e->h_delta[i] = e->deltas[reqs[B.idx[i]].step];
-  FPS_CUDA_TRY(cudaMemcpyAsync(e->d_delta, e->h_delta, n * 4, cudaMemcpyHostToDevice, cs));
+  FPS_COPY_TRY(cs, cudaMemcpyAsync(e->d_delta, e->h_delta, n * 4, cudaMemcpyHostToDevice, cs));
 
   // ---- load schedule: ring loads (cached blocks in order) + KV-mode final Y load ----------
   std::vector<int> loads;                  // block of each ring load
@@ -325,7 +325,7 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
   bool final_issued = false;
   std::vector<fps_prefetch_item> items(n);
   FPS_CUDA_TRY(cudaEventRecord(e->step_start, cs));
-  FPS_CUDA_TRY(cudaStreamWaitEvent(ls, e->step_start, 0));
+  FPS_CUDA_TRY(stream_wait(ls, e->step_start, 0));
   auto issue = [&](int block, char* dst, size_t row_bytes, cudaEvent_t ev) -> fps_status {
     for (int i = 0; i < n; ++i) {
       const fps_request& r = reqs[B.idx[i]];
@@ -343,7 +343,7 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
   };
   auto try_issue = [&]() -> fps_status {
     while (issued < n_ring && (issued < e->D || consumed_rec[issued - e->D])) {
-      if (issued >= e->D) FPS_CUDA_TRY(cudaStreamWaitEvent(ls, e->consumed[issued - e->D], 0));
+      if (issued >= e->D) FPS_CUDA_TRY(stream_wait(ls, e->consumed[issued - e->D], 0));
       FPS_TRY(issue(loads[issued], e->slots[issued % e->D], e->row_w, e->ready[issued]));
       ++issued;
     }
@@ -400,7 +400,7 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
         // output rows U of block l-1 (reading R11)
         char* dst = e->full[full_toggle];
         FPS_TRY(launch_copy_rows(e->act[act_cur], nullptr, B.q_row, B.tq, (int)e->row_h, dst, cs));
-        FPS_CUDA_TRY(cudaStreamWaitEvent(cs, e->ready[pos[l - 1]], 0));
+        FPS_CUDA_TRY(stream_wait(cs, e->ready[pos[l - 1]], 0));
         FPS_TRY(launch_copy_rows(e->slots[pos[l - 1] % e->D], B.u_row, B.u_row, B.tu,
                                  (int)e->row_h, dst, cs));
         FPS_TRY(consume(pos[l - 1]));
@@ -434,7 +434,7 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
         if (cache_writes_all_rows(e->d.cache)) {
           // whole-entry DMA also lands on the masked rows: the QKV epilogue's fresh K/V must
           // come after it (the load was issued layers ahead, so this rarely waits)
-          FPS_CUDA_TRY(cudaStreamWaitEvent(cs, ev, 0));
+          FPS_CUDA_TRY(stream_wait(cs, ev, 0));
           ev = nullptr;
         }
       } else {
@@ -457,14 +457,14 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
     FPS_TRY(launch_copy_rows(e->act[act_cur], nullptr, B.q_row, B.tq, (int)e->row_h, e->y_full, cs));
     const int j = kv ? n_ring : pos[N - 1];
     const char* src = kv ? e->final_slot : e->slots[pos[N - 1] % e->D];
-    FPS_CUDA_TRY(cudaStreamWaitEvent(cs, e->ready[j], 0));
+    FPS_CUDA_TRY(stream_wait(cs, e->ready[j], 0));
     FPS_TRY(launch_copy_rows(src, B.u_row, B.u_row, B.tu, (int)e->row_h, e->y_full, cs));
     y_src = e->y_full;
   }
   FPS_TRY(launch_euler(e->d.dtype, e->x_full, y_src, B.tk, H, B.cu_k, n, e->d_delta, cs));
   // the load stream must not run ahead into the next step's slots before this step is done
   FPS_CUDA_TRY(cudaEventRecord(e->step_start, cs));
-  FPS_CUDA_TRY(cudaStreamWaitEvent(ls, e->step_start, 0));
+  FPS_CUDA_TRY(stream_wait(ls, e->step_start, 0));
   return FPS_OK;
 }
 
@@ -496,7 +496,7 @@ extern "C" fps_status fps_run_batch(fps_engine_t e, fps_request* reqs, int32_t n
     FPS_TRY(admit(e, reqs, live, B, cs));
     // load each request's latent into the contiguous batch buffer
     for (int i = 0; i < B.n; ++i)
-      FPS_CUDA_TRY(cudaMemcpyAsync(e->x_full + (size_t)i * e->L * e->row_h, reqs[live[i]].d_x,
+      FPS_COPY_TRY(cs, cudaMemcpyAsync(e->x_full + (size_t)i * e->L * e->row_h, reqs[live[i]].d_x,
                                    (size_t)e->L * e->row_h, cudaMemcpyDeviceToDevice, cs));
     make_plan(e, B);
     bool changed = false;
@@ -513,13 +513,13 @@ extern "C" fps_status fps_run_batch(fps_engine_t e, fps_request* reqs, int32_t n
       }
     }
     for (int i = 0; i < B.n; ++i)
-      FPS_CUDA_TRY(cudaMemcpyAsync(reqs[live[i]].d_x, e->x_full + (size_t)i * e->L * e->row_h,
+      FPS_COPY_TRY(cs, cudaMemcpyAsync(reqs[live[i]].d_x, e->x_full + (size_t)i * e->L * e->row_h,
                                    (size_t)e->L * e->row_h, cudaMemcpyDeviceToDevice, cs));
   }
   for (int i = 0; i < n_req; ++i) reqs[i].status = reqs[i].step >= reqs[i].n_steps ? 1 : 0;
   // make sure the load stream has drained before the caller reuses buffers
   FPS_CUDA_TRY(cudaEventRecord(e->step_start, ls));
-  FPS_CUDA_TRY(cudaStreamWaitEvent(cs, e->step_start, 0));
+  FPS_CUDA_TRY(stream_wait(cs, e->step_start, 0));
   e->last_launches = g_launches - launches0;
   return FPS_OK;
 }

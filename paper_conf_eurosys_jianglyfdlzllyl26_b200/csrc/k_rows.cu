@@ -140,7 +140,8 @@ __global__ void __launch_bounds__(256) copy_rows_kernel(const uint4* __restrict_
 }
 
 fps_status launch_copy_rows(const void* src, const int32_t* src_ids, const int32_t* dst_ids,
-                            int n, int row_bytes, void* dst, cudaStream_t s, int max_ctas) {
+                            int n, int row_bytes, void* dst, cudaStream_t s, int max_ctas,
+                            bool profile) {
   if (n <= 0) return FPS_OK;
   const int vpr = row_bytes / 16;
   const long long total = (long long)n * vpr;
@@ -148,11 +149,11 @@ fps_status launch_copy_rows(const void* src, const int32_t* src_ids, const int32
   int cap = max_ctas > 0 ? max_ctas : kNumSMs * 8;
   int grid = (int)(want < cap ? want : cap);
   if (grid < 1) grid = 1;
-  prof::begin(s);
+  if (profile) prof::begin(s);
   FPS_CUDA_TRY(launch_k(copy_rows_kernel, dim3(grid), dim3(256), 0, s,
                         reinterpret_cast<const uint4*>(src), src_ids, dst_ids, total, vpr,
                         reinterpret_cast<uint4*>(dst)));
-  prof::end(s, prof::ROWS, 0, 2.0 * n * row_bytes);
+  if (profile) prof::end(s, prof::ROWS, 0, 2.0 * n * row_bytes);
   count_launch();
   FPS_LAUNCH_CHECK();
   return FPS_OK;

@@ -12,7 +12,8 @@ fps_status launch_mask_pool(const uint8_t* pix, int n_req, int Hp, int Wp, int f
                             uint8_t* tok, cudaStream_t s);
 // a2/a9/a3 row movement: dst[dst_ids? dst_ids[i] : i] = src[src_ids ? src_ids[i] : i]
 fps_status launch_copy_rows(const void* src, const int32_t* src_ids, const int32_t* dst_ids,
-                            int n, int row_bytes, void* dst, cudaStream_t s, int max_ctas = 0);
+                            int n, int row_bytes, void* dst, cudaStream_t s, int max_ctas = 0,
+                            bool profile = true);
 // a4: out[i] = LN(x[rows ? rows[i] : i]) * (1 + scale[req(i)]) + shift[req(i)]
 fps_status launch_ln_mod(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
                          const int32_t* cu, int n_req, const void* mod, int shift_off,
@@ -53,5 +54,7 @@ extern int g_disable_tc;
 extern int g_gemm_force;
 // tests: 0 = two query tiles per CTA (default), 1 = force the one-tile attention kernel
 extern int g_attn_force;
+// 1 (default): HBM-arena whole-entry loads copied by a library kernel, 0: driver D2D memcpy
+extern int g_d2d_kernel;
 
 }  // namespace fps

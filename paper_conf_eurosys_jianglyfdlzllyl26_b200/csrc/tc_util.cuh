@@ -20,10 +20,35 @@ __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
 __device__ __forceinline__ void fence_mbar_init() {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 }
+// FPS_HANG_WATCH builds (debugging only): a wait still unsatisfied after 4 s of wall time
+// reports the kernel shape, block, thread, barrier and parity, then traps.
+#ifdef FPS_HANG_WATCH
+__device__ __forceinline__ unsigned long long global_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define FPS_WATCH_DECL unsigned long long _t0 = 0, _spins = 0;
+#define FPS_WATCH_STEP(a, parity)                                                              \
+  if ((++_spins & 1023) == 0) {                                                                \
+    const unsigned long long _now = global_ns();                                              \
+    if (_t0 == 0) _t0 = _now;                                                                  \
+    else if (_now - _t0 > 4000000000ull) {                                                     \
+      printf("HANG grid(%d,%d) block(%d) cta(%d,%d) thr %d bar 0x%x parity %u\n", gridDim.x,  \
+             gridDim.y, blockDim.x, blockIdx.x, blockIdx.y, threadIdx.x, a, parity);           \
+      __trap();                                                                                \
+    }                                                                                          \
+  }
+#else
+#define FPS_WATCH_DECL
+#define FPS_WATCH_STEP(a, parity)
+#endif
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   const uint32_t a = smem_u32(bar);
   uint32_t done;
+  FPS_WATCH_DECL
   do {
+    FPS_WATCH_STEP(a, parity)
     asm volatile(
         "{\n.reg .pred p;\nmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
         "selp.u32 %0, 1, 0, p;\n}\n"
@@ -40,7 +65,9 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
 __device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) {
   const uint32_t a = smem_u32(bar);
   uint32_t done;
+  FPS_WATCH_DECL
   do {
+    FPS_WATCH_STEP(a, parity)
     asm volatile(
         "{\n.reg .pred p;\nmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n"
         "selp.u32 %0, 1, 0, p;\n}\n"

@@ -256,3 +256,17 @@ def test_identical_input_cache_gpu_internal_invariant(F):
             outs.append(req["x"].clone())
         diff = (outs[0].float() - outs[1].float()).abs().max().item()
         assert torch.equal(outs[0].view(torch.int16), outs[1].view(torch.int16)), f"{mode}: {diff}"
+
+
+def test_hbm_whole_entry_loads_with_dense_prefix_complete():
+    """Regression: HBM-tier whole-entry loads under a plan with a dense prefix (C2B stack,
+    21 dense + 39 cached blocks).  Issued as driver device-to-device memcpys next to the PDL
+    compute chain this hung on the first step; the library copy kernel must complete.  Runs in
+    a subprocess so a hang fails the test instead of stalling the suite."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    p = subprocess.run([sys.executable, os.path.join(root, "tools", "hang_probe.py"), "C2B", "kv",
+                        "1", "2", "21", "3"], capture_output=True, text=True, timeout=180)
+    assert p.returncode == 0 and "DONE" in p.stdout, p.stdout[-2000:] + p.stderr[-2000:]
