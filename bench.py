@@ -297,11 +297,20 @@ def run_engine_timed(F, eng, reqs_dev, K, W, stream, load_stream, rank, world):
     launches = F.fps_launch_count() - l0
     ms = e0.elapsed_time(e1)
     if world > 1:
-        t = torch.tensor([ms], device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+        ms = dist_max(ms)
         dist.barrier()
     return ms / K, launches
+
+
+DIST_DEVICE = None   # device of the all-reduce tensors: the GPU (NCCL) or the CPU (gloo)
+
+
+def dist_max(v):
+    """Max over ranks of a host float (device-timed values are reduced, never wall clock)."""
+    import torch.distributed as dist
+    t = torch.tensor([float(v)], dtype=torch.float64, device=DIST_DEVICE)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
 
 
 def oracle_block_sample(w, mode, ratio, seed=7):
@@ -419,14 +428,24 @@ def main():
 
     import paper_conf_eurosys_jianglyfdlzllyl26_b200 as F
     from paper_conf_eurosys_jianglyfdlzllyl26_b200 import sched
-    torch.cuda.set_device(local)
-    device = torch.device("cuda", local)
     F.require_gpu()
+    # one process per GPU; only on a box with fewer GPUs than ranks (a functional check of the
+    # multi-rank path on one GPU) do ranks share devices, with gloo for the two host reductions
+    n_dev = torch.cuda.device_count()
+    torch.cuda.set_device(local % n_dev)
+    device = torch.device("cuda", local % n_dev)
     if os.environ.get("FPS_KERNEL_FLAGS"):            # experiments: force kernel variants
         F.fps_set_disable_tc(int(os.environ["FPS_KERNEL_FLAGS"]))
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=device)
+        global DIST_DEVICE
+        if n_dev >= world:
+            dist.init_process_group("nccl", device_id=device)
+            DIST_DEVICE = device
+        else:
+            dist.init_process_group("gloo")
+            DIST_DEVICE = torch.device("cpu")
+            log(f"[rank {rank}] {world} ranks on {n_dev} GPU(s): shared devices, gloo reductions")
 
     # requests of the whole job, routed to GPUs by Alg. 2 (identical on every rank: no comms)
     pool = make_requests(w, w["batch"] * world, SEED)
@@ -472,7 +491,7 @@ def main():
 
     eng = engine(0)
     log(f"[rank {rank}] timed run")
-    with Clocks(local) as clk:
+    with Clocks(local % n_dev) as clk:
         step_ms, launches = run_engine_timed(F, eng, reqs_dev, K, W, stream, load_stream, rank, world)
     plan, pred_ms = eng.last_plan()
     imgs = sum(len(a) for a in assign)
@@ -585,10 +604,7 @@ def main():
     torch.cuda.synchronize()
     e2e_ms = e0.elapsed_time(e1) / K
     if world > 1:
-        import torch.distributed as dist
-        t = torch.tensor([e2e_ms], device=device)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        e2e_ms = float(t.item())
+        e2e_ms = dist_max(e2e_ms)
     bytes_io = len(reqs_dev) * L * w["H"] * 2
     e2e = {"value": imgs / (e2e_ms * 1e-3 * w["steps"]), "unit": metric_unit,
            "ms_per_step": e2e_ms, "h2d_bytes_per_step": bytes_io, "d2h_bytes_per_step": bytes_io}

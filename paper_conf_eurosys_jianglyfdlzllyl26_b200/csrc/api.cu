@@ -140,7 +140,7 @@ static size_t ws_layout(int H, int F, int dtype, int max_q, int max_u, char* bas
   char* x1 = take((size_t)max_q * H * e);
   char* h2 = take((size_t)max_q * H * e);
   char* u = take((size_t)max_q * F * e);
-  char* hu = take((size_t)max_u * H * e);
+  char* hu = take((size_t)(max_q + max_u) * H * e);   // Y-mode: LN of all rows, token order
   if (ws) *ws = BlockWs{h, q, ao, x1, h2, u, hu};
   return off;
 }
@@ -167,8 +167,12 @@ static fps_status check_batch(const fps_varlen_batch* b) {
   FPS_CHECK_ARG(b->n_req >= 0 && b->total_q >= 0 && b->total_k >= 0, "negative sizes");
   FPS_CHECK_ARG(b->n_req == 0 || (b->d_cu_q && b->d_cu_k), "cu arrays are NULL");
   FPS_CHECK_ARG(b->mode == FPS_MODE_KV || b->mode == FPS_MODE_Y, "mode %d", b->mode);
-  if (b->mode == FPS_MODE_Y && b->total_u > 0)
+  if (b->mode == FPS_MODE_Y && b->total_u > 0) {
     FPS_CHECK_ARG(b->d_cu_u && b->d_u_src && b->d_u_row, "Y-mode needs cu_u/u_src/u_row");
+    FPS_CHECK_ARG(b->total_q + b->total_u == b->total_k,
+                  "Y-mode: every merged row must be active or cached (%d + %d != %d)", b->total_q,
+                  b->total_u, b->total_k);
+  }
   return FPS_OK;
 }
 
@@ -185,7 +189,30 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
   const char* mod = (const char*)b->d_mod;
   auto modp = [&](int off) -> const void* { return mod ? mod + (size_t)off * H * e : nullptr; };
 
-  if (tq > 0) {
+  // Y-mode, sequential block: Q over the active rows, K|V in ONE GEMM over all rows of the
+  // merged buffer (fresh rows M and cached input rows U, normalised into token order) -- the same
+  // FLOPs as the QKV GEMM on M plus a K|V GEMM on U, in fewer waves with no 256-row padding at
+  // the M/U split (C3: 6 + 1 waves instead of 3 + 5)
+  const bool y_split = tu > 0 && tq > 0 && w->kind == FPS_BLOCK_SEQ;
+  if (y_split) {
+    FPS_TRY(launch_ln_mod(dt, x_act, nullptr, tq, H, ws.h, b->d_cu_q, b->n_req, b->d_mod, 0, s));
+    Epilogue eq{};
+    eq.bias = w->b_qkv;
+    eq.out0 = ws.q; eq.ld0 = H; eq.split = H;
+    FPS_TRY(launch_gemm(dt, ws.h, w->w_qkv, tq, H, H, eq, s));
+    FPS_TRY(launch_ln_mod(dt, x_act, nullptr, tq, H, ws.hu, b->d_cu_q, b->n_req, b->d_mod, 0, s,
+                          b->d_q_row));
+    if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
+    kv_ready = nullptr;
+    FPS_TRY(launch_ln_mod(dt, xu, b->d_u_src, tu, H, ws.hu, b->d_cu_u, b->n_req, b->d_mod, 0, s,
+                          b->d_u_row));
+    Epilogue ek{};
+    ek.bias = w->b_qkv ? (const char*)w->b_qkv + (size_t)H * e : nullptr;
+    ek.out0 = kv; ek.ld0 = 2 * H; ek.split = 2 * H;
+    FPS_TRY(launch_gemm(dt, ws.hu, (const char*)w->w_qkv + (size_t)H * H * e, b->total_k, 2 * H, H,
+                        ek, s));
+  }
+  if (tq > 0 && !y_split) {
     // a4: h1 = LN(x)(1+scale1)+shift1 on active rows
     FPS_TRY(launch_ln_mod(dt, x_act, nullptr, tq, H, ws.h, b->d_cu_q, b->n_req, b->d_mod, 0, s));
     // a5: [tq,H] x [3H,H]^T; Q -> compact, K|V -> merged key rows at original positions
@@ -202,7 +229,7 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
     }
     FPS_TRY(launch_gemm(dt, ws.h, w->w_qkv, tq, n_out, H, ep, s));
   }
-  if (tu > 0) {
+  if (tu > 0 && !y_split) {
     // Y-mode: cached block-input rows U -> LN -> K|V projection (Fig. 5-Bottom, reading R5)
     if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
     kv_ready = nullptr;

@@ -167,7 +167,8 @@ __global__ void __launch_bounds__(128) ln_mod_kernel(const T* __restrict__ x,
                                                      const int32_t* __restrict__ rows, int n,
                                                      int H, T* __restrict__ out,
                                                      const int32_t* __restrict__ cu, int n_req,
-                                                     const T* __restrict__ mod, int shift_off) {
+                                                     const T* __restrict__ mod, int shift_off,
+                                                     const int32_t* __restrict__ out_rows) {
   constexpr int NV = Vec16<T>::N;
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (warp >= n) return;
@@ -209,7 +210,7 @@ __global__ void __launch_bounds__(128) ln_mod_kernel(const T* __restrict__ x,
     shift = mod + (size_t)r * 6 * H + shift_off;
     scale = shift + H;
   }
-  uint4* o = reinterpret_cast<uint4*>(out + (size_t)warp * H);
+  uint4* o = reinterpret_cast<uint4*>(out + (size_t)(out_rows ? __ldg(out_rows + warp) : warp) * H);
 #pragma unroll
   for (int k = 0; k < VPT; ++k) {
     int vi = lane + 32 * k;
@@ -238,7 +239,8 @@ __global__ void __launch_bounds__(128) ln_mod_row_kernel(const T* __restrict__ x
                                                          const int32_t* __restrict__ rows, int H,
                                                          T* __restrict__ out,
                                                          const int32_t* __restrict__ cu, int n_req,
-                                                         const T* __restrict__ mod, int shift_off) {
+                                                         const T* __restrict__ mod, int shift_off,
+                                                         const int32_t* __restrict__ out_rows) {
   constexpr int NV = Vec16<T>::N;
   __shared__ float red[4];
   pdl_trigger();
@@ -291,7 +293,7 @@ __global__ void __launch_bounds__(128) ln_mod_row_kernel(const T* __restrict__ x
   if (lane == 0) red[warp] = sq;
   __syncthreads();
   const float rstd = 1.0f / sqrtf((red[0] + red[1] + red[2] + red[3]) / (float)H + 1e-6f);
-  uint4* o = reinterpret_cast<uint4*>(out + (size_t)row * H);
+  uint4* o = reinterpret_cast<uint4*>(out + (size_t)(out_rows ? __ldg(out_rows + row) : row) * H);
 #pragma unroll
   for (int k = 0; k < VPT; ++k) {
     const int vi = tid + 128 * k;
@@ -309,7 +311,7 @@ __global__ void __launch_bounds__(128) ln_mod_row_kernel(const T* __restrict__ x
 template <typename T>
 static fps_status ln_mod_t(const void* x, const int32_t* rows, int n, int H, void* out,
                            const int32_t* cu, int n_req, const void* mod, int shift_off,
-                           cudaStream_t s) {
+                           cudaStream_t s, const int32_t* out_rows) {
   constexpr int NV = Vec16<T>::N;
   const int per_lane = ceil_div(H / NV, 32);
   const int grid = ceil_div(n, 4);
@@ -323,11 +325,11 @@ static fps_status ln_mod_t(const void* x, const int32_t* rows, int n, int H, voi
 #define FPS_LNR_CASE(VPT)                                                                  \
     if (per_thread <= VPT)                                                                 \
       le = launch_k(ln_mod_row_kernel<T, VPT>, dim3(n), dim3(128), 0, s, X, rows, H, O, cu, \
-                    n_req, Md, shift_off);                                                 \
+                    n_req, Md, shift_off, out_rows);                                       \
     else
     FPS_LNR_CASE(1) FPS_LNR_CASE(2) FPS_LNR_CASE(3) FPS_LNR_CASE(4) FPS_LNR_CASE(6)
     le = launch_k(ln_mod_row_kernel<T, 8>, dim3(n), dim3(128), 0, s, X, rows, H, O, cu, n_req,
-                  Md, shift_off);
+                  Md, shift_off, out_rows);
 #undef FPS_LNR_CASE
     FPS_CUDA_TRY(le);
     prof::end(s, prof::LN, 0, 2.0 * n * H * sizeof(T));
@@ -338,7 +340,7 @@ static fps_status ln_mod_t(const void* x, const int32_t* rows, int n, int H, voi
 #define FPS_LN_CASE(VPT)                                                                  \
   if (per_lane <= VPT) {                                                                  \
     prof::begin(s);                                                                       \
-    ln_mod_kernel<T, VPT><<<grid, 128, 0, s>>>(X, rows, n, H, O, cu, n_req, Md, shift_off); \
+    ln_mod_kernel<T, VPT><<<grid, 128, 0, s>>>(X, rows, n, H, O, cu, n_req, Md, shift_off, out_rows); \
     prof::end(s, prof::LN, 0, 2.0 * n * H * sizeof(T));                                   \
     count_launch();                                                                       \
     FPS_LAUNCH_CHECK();                                                                   \
@@ -356,11 +358,11 @@ static fps_status ln_mod_t(const void* x, const int32_t* rows, int n, int H, voi
 
 fps_status launch_ln_mod(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
                          const int32_t* cu, int n_req, const void* mod, int shift_off,
-                         cudaStream_t s) {
+                         cudaStream_t s, const int32_t* out_rows) {
   if (n <= 0) return FPS_OK;
   if (dtype == FPS_BF16)
-    return ln_mod_t<__nv_bfloat16>(x, rows, n, H, out, cu, n_req, mod, shift_off, s);
-  return ln_mod_t<float>(x, rows, n, H, out, cu, n_req, mod, shift_off, s);
+    return ln_mod_t<__nv_bfloat16>(x, rows, n, H, out, cu, n_req, mod, shift_off, s, out_rows);
+  return ln_mod_t<float>(x, rows, n, H, out, cu, n_req, mod, shift_off, s, out_rows);
 }
 
 // ---------------------------------------------------------------------------------------

@@ -14,10 +14,11 @@ fps_status launch_mask_pool(const uint8_t* pix, int n_req, int Hp, int Wp, int f
 fps_status launch_copy_rows(const void* src, const int32_t* src_ids, const int32_t* dst_ids,
                             int n, int row_bytes, void* dst, cudaStream_t s, int max_ctas = 0,
                             bool profile = true);
-// a4: out[i] = LN(x[rows ? rows[i] : i]) * (1 + scale[req(i)]) + shift[req(i)]
+// a4: out[out_rows ? out_rows[i] : i] = LN(x[rows ? rows[i] : i]) * (1 + scale[req(i)])
+//                                        + shift[req(i)]
 fps_status launch_ln_mod(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
                          const int32_t* cu, int n_req, const void* mod, int shift_off,
-                         cudaStream_t s);
+                         cudaStream_t s, const int32_t* out_rows = nullptr);
 // x[i] += delta[req(i)] * y[i] over rows of width H (req via cu over rows)
 fps_status launch_euler(int dtype, void* x, const void* y, int n, int H, const int32_t* cu,
                         int n_req, const float* delta, cudaStream_t s);
