@@ -216,3 +216,45 @@ def test_parallel_weights_validated(F):
     b = F.VarlenBatch([64], [64])
     with pytest.raises(F.FlashPSError):
         F.dense_block_forward(bw, b, torch.zeros(64, 128, dtype=torch.bfloat16, device="cuda"))
+
+
+@pytest.mark.parametrize("mode", ["kv", "y"])
+def test_c4_continuous_batch_sampled_rows(F, mode):
+    """configs[3] in the bench's launch configuration: 16 Flux-scale requests with masks from 5 %
+    to 60 % in ONE varlen launch per GEMM / attention; the oracle checks sampled rows of four
+    requests (first, last and two inner ones, incl. the smallest and largest masks)."""
+    g = synth.rng(3004 + (mode == "y"))
+    H, heads, Fd, L_img, L_txt = 3072, 24, 12288, 4096, 512
+    L = L_img + L_txt
+    w = synth.block_weights(g, H, Fd, "bf16")
+    reqs = []
+    for m in np.linspace(0.05, 0.60, 16):
+        mask = synth.token_mask(synth.mask_blobs(g, 64, 64, float(m)), L_txt)
+        M, U = build_mask_index(mask)
+        reqs.append(dict(mask=mask, M=M, U=U, L=L, x=synth.latent(g, L, H, "bf16"),
+                         K=synth.latent(g, L, H, "bf16"), V=synth.latent(g, L, H, "bf16"),
+                         xu=synth.latent(g, L, H, "bf16"),
+                         mod=synth.mod_table(g, 1, 1, H, "bf16")[0, 0]))
+    y, _ = _run_masked(F, w, reqs, heads, "bf16", mode)
+    cu = np.concatenate([[0], np.cumsum([len(r["M"]) for r in reqs])])
+    Wq, bq = w["w_qkv"][:H], w["b_qkv"][:H]
+    Wk, bk = w["w_qkv"][H:2 * H], w["b_qkv"][H:2 * H]
+    Wv, bv = w["w_qkv"][2 * H:], w["b_qkv"][2 * H:]
+    for i in (0, 5, 10, 15):
+        r = reqs[i]
+        M, U = r["M"], r["U"]
+        sh1, sc1 = r["mod"][:H], r["mod"][H:2 * H]
+        x_in = np.array(r["x"], np.float64)
+        if mode == "y":
+            x_in[U] = r["xu"][U]
+        h1 = B.layer_norm(x_in) * (1 + sc1) + sh1
+        if mode == "kv":
+            Kall, Vall = np.array(r["K"], np.float64), np.array(r["V"], np.float64)
+            Kall[M] = B.linear(h1[M], Wk, bk)
+            Vall[M] = B.linear(h1[M], Wv, bv)
+        else:
+            Kall, Vall = B.linear(h1, Wk, bk), B.linear(h1, Wv, bv)
+        sample = np.unique(np.concatenate([g.choice(len(M), 12, replace=False), [0, len(M) - 1]]))
+        a = B.attention(B.linear(h1[M][sample], Wq, bq), Kall, Vall, heads)
+        ref = B._attn_out_and_mlp(r["x"][M][sample], a, w, r["mod"], H)
+        check_close(y[cu[i] + sample], ref, TOL["bf16"], f"C4 {mode} request {i}")

@@ -270,3 +270,60 @@ def test_hbm_whole_entry_loads_with_dense_prefix_complete():
     p = subprocess.run([sys.executable, os.path.join(root, "tools", "hang_probe.py"), "C2B", "kv",
                         "1", "2", "21", "3"], capture_output=True, text=True, timeout=180)
     assert p.returncode == 0 and "DONE" in p.stdout, p.stdout[-2000:] + p.stderr[-2000:]
+
+
+@pytest.mark.parametrize("mode", ["kv", "y"])
+def test_full_scale_stack_identical_input_invariant(F, mode):
+    """configs[2] at its full size (57 Flux-scale blocks, 4096 + 512 tokens, m = 0.2): with the
+    cache taken from the GPU's own dense template run on the identical input, the mask-aware
+    step (every block cached) reproduces the dense step bit-for-bit -- a property that holds at
+    any size (L144/L157), checked where the fp64 oracle cannot run the whole stack."""
+    H, heads, Fd, L_img, L_txt, N, steps = 3072, 24, 12288, 4096, 512, 57, 1
+    L = L_img + L_txt
+    dev = torch.device("cuda")
+    gen = torch.Generator(device=dev).manual_seed(57)
+    rnd = lambda *s, sc=1.0: (torch.randn(*s, generator=gen, device=dev) * sc).to(torch.bfloat16)
+    dt = F.FPS_BF16
+    layers = []
+    for _ in range(N):
+        t = {"w_qkv": rnd(3 * H, H, sc=H ** -0.5), "b_qkv": rnd(3 * H, sc=0.02),
+             "w_o": rnd(H, H, sc=H ** -0.5), "b_o": rnd(H, sc=0.02),
+             "w_up": rnd(Fd, H, sc=H ** -0.5), "b_up": rnd(Fd, sc=0.02),
+             "w_down": rnd(H, Fd, sc=Fd ** -0.5), "b_down": rnd(H, sc=0.02)}
+        bw = F.BlockWeights.__new__(F.BlockWeights)
+        bw.t, bw.H, bw.F, bw.heads, bw.dtype, bw.kind = t, H, Fd, heads, dt, 0
+        bw.c = F.fps_block_weights(H, heads, H // heads, Fd, dt,
+                                   *[t[k].data_ptr() for k in ("w_qkv", "b_qkv", "w_o", "b_o",
+                                                               "w_up", "b_up", "w_down", "b_down")], 0)
+        layers.append(bw)
+    mods = (0.02 * torch.randn(N, steps, 6, H, generator=gen, device=dev))
+    mods[:, :, 2] += 1.0
+    mods[:, :, 5] += 1.0
+    mods = mods.reshape(N, steps, 6 * H).to(torch.bfloat16)
+    x0 = torch.randn(L, H, generator=gen, device=dev).to(torch.bfloat16)
+    mask = synth.token_mask(synth.mask_blobs(synth.rng(57), 64, 64, 0.2), L_txt)
+    m = F.MODE_CODE[mode]
+    cache = F.Cache(m, dt, H, L_img, N, steps, n_templates=1)
+    cur = x0.clone()
+    for l in range(N):
+        bl = F.VarlenBatch([L], [L], mod=mods[l, 0][None].contiguous())
+        y, kv = F.dense_block_forward(layers[l], bl, cur)
+        cache.store(0, 0, l, kv if mode == "kv" else y)
+        cur = y
+    if mode == "kv":
+        cache.store(0, 0, N, cur)
+    torch.cuda.synchronize()
+    outs = []
+    for policy in (1, 2):                 # every block cached vs every block dense
+        eng = F.Engine(layers, heads, m, dt, L_img, L_txt, 1, steps, synth.delta_table(steps),
+                       cache, mod_table=mods, plan_policy=policy)
+        req = dict(template_id=0, step=0, n_steps=steps, mask=torch.as_tensor(mask).cuda(),
+                   x=x0.clone())
+        eng.run_batch([req], 1)
+        torch.cuda.synchronize()
+        outs.append(req["x"].clone())
+        eng.close()
+    cache.close()
+    assert torch.isfinite(outs[0].float()).all()
+    assert torch.equal(outs[0].view(torch.int16), outs[1].view(torch.int16)), \
+        f"{mode}: max diff {(outs[0].float() - outs[1].float()).abs().max().item()}"
