@@ -47,6 +47,7 @@ WORKLOADS = {
                 desc="SDXL-scale 64x64 level (640 ch), masks 10/30/50%, batch 4"),
 }
 SEED = 1003
+SDXL_CTX = (77, 2048)          # SDXL prompt encoding: 77 tokens x 2048 channels (R24)
 
 
 def log(*a):
@@ -155,8 +156,24 @@ def build_engine_inputs(F, w, mode, device, n_entries, location=0, copy_method=0
 
     layers = []
     par = w.get("block") == "par"
+    sdxl = w.get("block") == "sdxl"
+    D = SDXL_CTX[1]
     for _ in range(N):
-        if par:      # parallel (Flux single-stream) block: W1 [3H+F, H], W2 [H, H+F] (R23)
+        if sdxl:     # SDXL UNet transformer block (R24): self-attn, cross-attn, GEGLU
+            t = {"w_qkv": rnd(3 * H, H, scale=H ** -0.5),
+                 "w_o": rnd(H, H, scale=H ** -0.5), "b_o": rnd(H, scale=0.02),
+                 "w_up": rnd(2 * Fd, H, scale=H ** -0.5), "b_up": rnd(2 * Fd, scale=0.02),
+                 "w_down": rnd(H, Fd, scale=Fd ** -0.5), "b_down": rnd(H, scale=0.02),
+                 "w_q2": rnd(H, H, scale=H ** -0.5), "w_kv2": rnd(2 * H, D, scale=D ** -0.5),
+                 "w_o2": rnd(H, H, scale=H ** -0.5), "b_o2": rnd(H, scale=0.02)}
+            for i in (1, 2, 3):
+                t[f"ln{i}_w"] = (1.0 + rnd(H, scale=0.02).float()).to(torch.bfloat16)
+                t[f"ln{i}_b"] = rnd(H, scale=0.02)
+            wp, bp = torch.empty_like(t["w_up"]), torch.empty_like(t["b_up"])
+            F.fps_geglu_pack(F.FPS_BF16, t["w_up"].data_ptr(), t["b_up"].data_ptr(), Fd, H,
+                             wp.data_ptr(), bp.data_ptr(), F.stream_ptr())
+            t["w_up"], t["b_up"] = wp, bp
+        elif par:    # parallel (Flux single-stream) block: W1 [3H+F, H], W2 [H, H+F] (R23)
             t = {"w_qkv": rnd(3 * H + Fd, H, scale=H ** -0.5), "b_qkv": rnd(3 * H + Fd, scale=0.02),
                  "w_down": rnd(H, H + Fd, scale=(H + Fd) ** -0.5), "b_down": rnd(H, scale=0.02)}
         else:
@@ -167,16 +184,20 @@ def build_engine_inputs(F, w, mode, device, n_entries, location=0, copy_method=0
         layers.append(F.BlockWeights.__new__(F.BlockWeights))
         bw = layers[-1]
         bw.t, bw.H, bw.F, bw.heads, bw.dtype = t, H, Fd, w["heads"], F.FPS_BF16
-        bw.kind = F.FPS_BLOCK_PAR if par else F.FPS_BLOCK_SEQ
+        bw.kind = F.FPS_BLOCK_SDXL if sdxl else F.FPS_BLOCK_PAR if par else F.FPS_BLOCK_SEQ
+        bw.D_ctx = D if sdxl else 0
+        ptrs = lambda keys: [t[k].data_ptr() if k in t else None for k in keys]
         bw.c = F.fps_block_weights(H, w["heads"], H // w["heads"], Fd, F.FPS_BF16,
-                                   *[t[k].data_ptr() if k in t else None
-                                     for k in ("w_qkv", "b_qkv", "w_o", "b_o", "w_up", "b_up",
-                                               "w_down", "b_down")], bw.kind)
+                                   *ptrs(("w_qkv", "b_qkv", "w_o", "b_o", "w_up", "b_up",
+                                          "w_down", "b_down")), bw.kind, bw.D_ctx,
+                                   *ptrs(F._SDXL_KEYS))
     mod = torch.zeros(N, w["steps"], 6, H, device=device)
     mod += 0.02 * torch.randn(N, w["steps"], 6, H, generator=gen, device=device)
     mod[:, :, 2] += 1.0
     mod[:, :, 5] += 1.0
     mod = mod.reshape(N, w["steps"], 6 * H).to(torch.bfloat16)
+    if sdxl:
+        mod = None                    # SDXL blocks are not adaLN-modulated (R24)
     cache = make_cache(F, w, mode, n_entries, location, copy_method)
     return layers, mod, cache
 
@@ -199,11 +220,15 @@ def calibrate(F, w, mode, layers, cache, reqs, device):
     ld_items = [F.fps_prefetch_item(i, 0, 0, w["L_img"], ld_rows.data_ptr(), h_ld_rows.ctypes.data,
                                     ld_dst[i * L].data_ptr(), Wl * 2) for i in range(B)]
     ld_stream = torch.cuda.Stream(device=device)
+    kind = w.get("block", "seq")
+    Lc = SDXL_CTX[0] if kind == "sdxl" else 0
+    ctx_kv = (torch.randn(B * Lc, 2 * H, device=device).to(torch.bfloat16) if Lc else None)
     for m in (0.05, 0.2, 0.4, 0.7, 1.0):
         n_img = synth.n_masked_for(m, w["L_img"])
         n = n_img + w["L_txt"]
         q_row = torch.cat([torch.arange(n, device=device, dtype=torch.int32) + i * L for i in range(B)])
-        b = F.VarlenBatch([n] * B, [L] * B, q_row=q_row, mode=F.FPS_MODE_KV)
+        b = F.VarlenBatch([n] * B, [L] * B, q_row=q_row, mode=F.FPS_MODE_KV,
+                          ctx_kv=ctx_kv, n_ctx=[Lc] * B)
         x = torch.randn(B * n, H, device=device).to(torch.bfloat16)
         ws = F.workspace(H, Fd, F.FPS_BF16, B * n, 0, device)
         y = torch.empty_like(x)
@@ -228,7 +253,7 @@ def calibrate(F, w, mode, layers, cache, reqs, device):
             fn()
         e1.record(s)
         torch.cuda.synchronize()
-        xs.append(B * sched.block_flops("kv", n, L, H, Fd))
+        xs.append(B * sched.block_flops("kv", n, L, H, Fd, kind, Lc))
         ys.append(e0.elapsed_time(e1) / (3 * nl))
     a, bb, r2c = sched.fit_linear(xs, ys)
     # loads: rows of one layer for the batch at several unmasked counts
@@ -271,7 +296,7 @@ def calibrate(F, w, mode, layers, cache, reqs, device):
     # flat in the row count, the fitted slope ~0 (or slightly negative by noise) -> clamp at 0
     cm = sched.CostModel(w["layers"], H, Fd, mode, comp=(max(a, 1e-16), max(bb, 1e-4)),
                          load=(max(c, 0.0), max(e, 1e-4)),
-                         full_entry_rows=w["L_img"] if whole else None)
+                         full_entry_rows=w["L_img"] if whole else None, kind=kind, Lc=Lc)
     info = {"comp_ms_per_tflop": a * 1e12, "comp_b_ms": bb, "comp_r2": r2c,
             "load_gbs": 1.0 / (c * 1e6) if c > 0 else None, "load_e_ms": e, "load_r2": r2l}
     return cm, info
@@ -321,7 +346,9 @@ def oracle_block_sample(w, mode, ratio, seed=7):
     g = synth.rng(seed)
     H, Fd, L_img, L_txt = w["H"], w["F"], w["L_img"], w["L_txt"]
     L = L_img + L_txt
-    wt = synth.block_weights(g, H, Fd, "bf16", w.get("block", "seq"))
+    kind = w.get("block", "seq")
+    wt = synth.block_weights(g, H, Fd, "bf16", kind, D_ctx=SDXL_CTX[1])
+    ctx = synth.context(g, *SDXL_CTX, "bf16") if kind == "sdxl" else None
     mask = synth.token_mask(synth.mask_blobs(g, *w["grid"], ratio), L_txt)
     M, U = build_mask_index(mask)
     x = synth.latent(g, L, H, "bf16")
@@ -329,9 +356,9 @@ def oracle_block_sample(w, mode, ratio, seed=7):
     mod = synth.mod_table(g, 1, 1, H, "bf16")[0, 0]
     t0 = time.perf_counter()
     if mode == "kv":
-        OB.masked_block_kv(x[M], M, U, K[U], V[U], wt, mod, w["heads"], L)
+        OB.masked_block_kv(x[M], M, U, K[U], V[U], wt, mod, w["heads"], L, ctx)
     else:
-        OB.masked_block_y(x[M], M, U, x[U], wt, mod, w["heads"], L)
+        OB.masked_block_y(x[M], M, U, x[U], wt, mod, w["heads"], L, ctx)
     return time.perf_counter() - t0
 
 
@@ -355,9 +382,11 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C3", choices=list(WORKLOADS))
     ap.add_argument("--mode", default="kv", choices=["kv", "y"])
-    ap.add_argument("--block", default="seq", choices=["seq", "par"],
-                    help="block kind: sequential attention -> MLP, or the parallel (Flux "
-                         "single-stream) block with fused input / output projections (NEXT-2)")
+    ap.add_argument("--block", default=None, choices=["seq", "par", "sdxl"],
+                    help="block kind: sequential attention -> MLP, the parallel (Flux "
+                         "single-stream) block with fused input / output projections, or the SDXL "
+                         "block with cross-attention and GEGLU (NEXT-2); default: sdxl for the "
+                         "SDXL-scale configs (C2A/C2B), seq otherwise")
     ap.add_argument("--tier", default="host", choices=["host", "hbm", "host_hugepage"],
                     help="template cache in pinned host DRAM (configs[2]) or HBM (NEXT-1)")
     ap.add_argument("--copy-ctas", type=int, default=0, help="CTAs of the SM row gather (0 = lib default)")
@@ -381,6 +410,8 @@ def main():
     rank = int(os.environ.get("RANK", 0))
     world = int(os.environ.get("WORLD_SIZE", 1))
     local = int(os.environ.get("LOCAL_RANK", 0))
+    if args.block is None:
+        args.block = "sdxl" if args.config.startswith("C2") else "seq"
     w = dict(WORKLOADS[args.config], block=args.block)
     K, W = args.steps, max(args.warmup, 0)
     if W + K > w["steps"]:
@@ -476,10 +507,13 @@ def main():
     mine = [pool[i] for i in my_ids]
     g = torch.Generator(device=device).manual_seed(SEED + rank)
     reqs_dev = []
+    L_ctx = SDXL_CTX[0] if args.block == "sdxl" else 0
     for i, p in enumerate(mine):
         reqs_dev.append(dict(template_id=i, step=0, n_steps=w["steps"],
                              mask=torch.as_tensor(p["mask_np"]).to(device),
                              x=torch.randn(L, w["H"], generator=g, device=device).to(torch.bfloat16)))
+        if L_ctx:
+            reqs_dev[-1]["ctx"] = torch.randn(*SDXL_CTX, generator=g, device=device).to(torch.bfloat16)
     stream = torch.cuda.current_stream()
     load_stream = torch.cuda.Stream(device=device)
     deltas = synth.delta_table(w["steps"])
@@ -487,7 +521,7 @@ def main():
     def engine(policy, mode=args.mode, the_cache=cache):
         return F.Engine(layers, w["heads"], F.MODE_CODE[mode], F.FPS_BF16, w["L_img"], w["L_txt"],
                         max(len(reqs_dev), 1), w["steps"], deltas, the_cache, mod_table=mod,
-                        slots=0, plan_policy=policy, cost_model=cm.as_engine_model())
+                        slots=0, plan_policy=policy, cost_model=cm.as_engine_model(), L_ctx=L_ctx)
 
     eng = engine(0)
     log(f"[rank {rank}] timed run")
@@ -518,7 +552,7 @@ def main():
             c_h = make_cache(F, w, args.mode, n_entries, 1, 2)
             eng_h = F.Engine(layers, w["heads"], F.MODE_CODE[args.mode], F.FPS_BF16, w["L_img"],
                              w["L_txt"], max(len(reqs_dev), 1), w["steps"], deltas, c_h,
-                             mod_table=mod, slots=0, plan_policy=3, plan=list(plan))
+                             mod_table=mod, slots=0, plan_policy=3, plan=list(plan), L_ctx=L_ctx)
             noload_ms, _ = run_engine_timed(F, eng_h, reqs_dev, K, W, stream, load_stream, rank,
                                             world)
             del eng_h
@@ -541,7 +575,7 @@ def main():
             eng_o = F.Engine(layers, w["heads"], F.MODE_CODE[md], F.FPS_BF16, w["L_img"],
                              w["L_txt"], max(len(reqs_dev), 1), w["steps"], deltas, c2,
                              mod_table=mod, slots=0, plan_policy=0,
-                             cost_model=cm2.as_engine_model())
+                             cost_model=cm2.as_engine_model(), L_ctx=L_ctx)
             o_ms, _ = run_engine_timed(F, eng_o, reqs_dev, K, W, stream, load_stream, rank, world)
             tag = f"{md}_mode_{['host', 'hbm', 'host_hugepage'][loc]}"
             if cmeth != default_cm(loc):

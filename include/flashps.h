@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define FPS_ABI_VERSION 1
+#define FPS_ABI_VERSION 2
 
 typedef enum {
   FPS_OK = 0,
@@ -190,16 +190,32 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
  * with W1 = w_qkv [3H+F, H] (rows Wq, Wk, Wv, then the F MLP-input rows), b1 = b_qkv [3H+F],
  * W2 = w_down [H, H+F], b2 = b_down [H]; w_o, b_o, w_up, b_up must be NULL; only
  * (shift1, scale1, gate1) of the modulation vector are read.  Same masked modes and cache.
+ *
+ * kind = FPS_BLOCK_SDXL (NEXT-2, reading R24): the SDXL UNet transformer block (the paper
+ *   evaluates SDXL, L65 / L305) -- self-attention, cross-attention to the request's prompt
+ *   encoding, GEGLU feed-forward, each behind an affine LayerNorm, ungated residuals:
+ *   h1 = LN(x) g1 + b1;  x1 = x + (A(h1 Wq^T, h1 Wk^T, h1 Wv^T) Wo^T + bo)
+ *   h2 = LN(x1) g2 + b2; x2 = x1 + (A(h2 Wq2^T, Kc, Vc) Wo2^T + bo2),  [Kc | Vc] = ctx Wkv2^T
+ *   h3 = LN(x2) g3 + b3; [P | G] = h3 Wup^T + bup;  y = x2 + ((P * GELU_tanh(G)) Wdown^T + bdown)
+ *   w_up / b_up must be in the PACKED layout fps_geglu_pack writes ([2F, H], F % 32 == 0);
+ *   the per-request context keys / values Kc | Vc come precomputed in the batch (d_ctx_kv,
+ *   written by fps_context_kv); d_mod is ignored.  bf16 only (tcgen05 path; H, F % 64 == 0).
  */
-enum { FPS_BLOCK_SEQ = 0, FPS_BLOCK_PAR = 1 };
+enum { FPS_BLOCK_SEQ = 0, FPS_BLOCK_PAR = 1, FPS_BLOCK_SDXL = 2 };
 typedef struct {
   int32_t H, heads, head_dim, F;   /* H = heads*head_dim; F = MLP width                    */
   int32_t dtype;                   /* FPS_BF16 (tcgen05 path) | FPS_F32 (SIMT fp32 path)   */
   const void *w_qkv, *b_qkv;       /* [3H, H], [3H]  rows: Wq, Wk, Wv  (PAR: W1, b1)        */
   const void *w_o, *b_o;           /* [H, H], [H]                      (PAR: NULL)          */
-  const void *w_up, *b_up;         /* [F, H], [F]                      (PAR: NULL)          */
+  const void *w_up, *b_up;         /* [F, H], [F]  (PAR: NULL; SDXL: packed GEGLU [2F, H])  */
   const void *w_down, *b_down;     /* [H, F], [H]                      (PAR: W2 [H, H+F], b2) */
-  int32_t kind;                    /* FPS_BLOCK_SEQ | FPS_BLOCK_PAR                         */
+  int32_t kind;                    /* FPS_BLOCK_SEQ | FPS_BLOCK_PAR | FPS_BLOCK_SDXL        */
+  /* SDXL block only (NULL / 0 otherwise); biases may be NULL, LN vectors may not.          */
+  int32_t D_ctx;                   /* prompt-encoding width (2048 in SDXL)                  */
+  const void *ln1_w, *ln1_b, *ln2_w, *ln2_b, *ln3_w, *ln3_b;   /* [H] gamma, beta          */
+  const void *w_q2, *b_q2;         /* [H, H], [H]   cross-attention query projection       */
+  const void *w_kv2, *b_kv2;       /* [2H, D_ctx], [2H]  rows Wk2 then Wv2 (fps_context_kv) */
+  const void *w_o2, *b_o2;         /* [H, H], [H]   cross-attention output projection      */
 } fps_block_weights;
 
 /* One varlen launch over a continuous batch (L237): request r owns active rows
@@ -223,7 +239,24 @@ typedef struct {
   const int32_t* d_cu_u;           /* [n_req+1]                                             */
   const int32_t* d_u_src;          /* [total_u] row index into d_xu of each cached row      */
   const int32_t* d_u_row;          /* [total_u] merged-buffer row of each cached row        */
+  /* SDXL blocks only: request r's cross-attention keys / values are rows
+   * [cu_ctx[r], cu_ctx[r+1]) of d_ctx_kv ([total_ctx, 2H], row = Kc|Vc, fps_context_kv).    */
+  const void* d_ctx_kv;
+  const int32_t* d_cu_ctx;         /* [n_req+1] device                                      */
+  const int32_t* h_cu_ctx;         /* [n_req+1] host mirror                                  */
 } fps_varlen_batch;
+
+/* SDXL block helpers (R24), run once per weight load / per request prompt, not per step.
+ * fps_geglu_pack: d_w [2F, K] (rows: GEGLU value half, then gate half -- diffusers' GEGLU
+ *   proj layout) and optional d_b [2F] -> d_w_out / d_b_out in the packed layout the block's
+ *   fused GEGLU epilogue reads (32-row groups: value rows 32j..32j+31, then gate rows
+ *   F+32j..F+32j+31).  F % 32 == 0, K*elt % 16 == 0; outputs must not alias inputs.
+ * fps_context_kv: d_ctx_kv[n_rows, 2H] = d_ctx[n_rows, D_ctx] Wkv2^T (+ b_kv2) with the
+ *   block's cross-attention weights -- the K|V rows fps_varlen_batch.d_ctx_kv expects. */
+fps_status fps_geglu_pack(int32_t dtype, const void* d_w, const void* d_b, int32_t F, int32_t K,
+                          void* d_w_out, void* d_b_out, void* stream);
+fps_status fps_context_kv(const fps_block_weights* w, const void* d_ctx, int32_t n_rows,
+                          void* d_ctx_kv, void* stream);
 
 /* Workspace bytes fps_masked_block_forward needs for up to max_q active / max_u cached rows. */
 size_t fps_block_workspace_bytes(int32_t H, int32_t F, int32_t dtype, int32_t max_q, int32_t max_u);
@@ -301,6 +334,8 @@ typedef struct {
   const uint8_t* h_plan;           /* [n_layers] when plan_policy == 3 (copied at create)   */
   double cost_model[4];            /* planner latency model: comp = a*FLOPs + b,
                                       load = c*bytes + e  -> {a, b, c, e}  (§4.4)     */
+  int32_t L_ctx, D_ctx;            /* SDXL blocks: prompt tokens / width of each request's
+                                      fps_request.d_ctx (0 if no layer is FPS_BLOCK_SDXL)   */
 } fps_engine_desc;
 
 typedef struct fps_engine* fps_engine_t;
@@ -312,6 +347,7 @@ typedef struct {
   const uint8_t* d_mask;   /* [L_img + L_txt] device token mask (text rows nonzero)         */
   void* d_x;               /* [L, H] device latent tokens, updated in place                 */
   int32_t status;          /* out: 0 = running, 1 = finished                                */
+  const void* d_ctx;       /* [L_ctx, D_ctx] device prompt encoding (SDXL blocks), or NULL  */
 } fps_request;
 
 fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out);
@@ -321,7 +357,9 @@ fps_status fps_engine_destroy(fps_engine_t e);
  * at that step boundary (status = 1) and the batch shrinks.  Admission reads the active-row
  * counts back to the host once per call (the only host sync).  Each step: mask-aware stack
  * with the Alg. 1 plan, layer-ahead prefetch on `load_stream`, final replenish + Euler update
- * x <- x + delta_s * y (reading R21).  The engine's last plan is available below. */
+ * x <- x + delta_s * y (reading R21).  The engine's last plan is available below.
+ * SDXL blocks: at admission the engine projects every request's d_ctx to the cross-attention
+ * K|V of each SDXL block once (fps_context_kv); the prompt is fixed over the steps. */
 fps_status fps_run_batch(fps_engine_t e, fps_request* reqs, int32_t n_req, int32_t n_steps,
                          void* compute_stream, void* load_stream);
 /* Plan and predicted latency (ms) of the last step; use_cache may be NULL. */

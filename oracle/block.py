@@ -34,6 +34,21 @@ output projection (Flux is a stack of such transformer blocks, L79 / L92 footnot
 Only (shift1, scale1, gate1) of `mod` are used.  Its FLOPs per row equal the sequential block's
 (12 H^2 multiply-adds with F = 4H), and the same masked modes apply: Z is token-wise (rows M
 only), K/V follow KV- or Y-mode exactly as above.
+
+SDXL block variant (NEXT-2, weights["kind"] == "sdxl"; reading R24): the UNet transformer
+block of the SDXL model the paper evaluates (L65, L305), i.e. self-attention, cross-attention
+to the request's prompt encoding ctx [L_ctx, D_ctx], and a GEGLU feed-forward, each pre-norm
+with an affine LayerNorm (gamma, beta) and an ungated residual; `mod` is not used:
+
+    h1 = LN(x) g1 + b1 ;  Q, K, V = h1 Wqkv^T (+ b) ;  x1 = x + (A(Q, K, V) Wo^T + bo)
+    h2 = LN(x1) g2 + b2 ; Q2 = h2 Wq2^T (+ bq2) ; [Kc | Vc] = ctx Wkv2^T (+ bkv2)
+                          x2 = x1 + (A(Q2, Kc, Vc) Wo2^T + bo2)
+    h3 = LN(x2) g3 + b3 ; [P | G] = h3 Wup^T + bup      Wup in R^{2F x H}: rows [0,F) -> P,
+                          y  = x2 + ((P * GELU_tanh(G)) Wdown^T + bdown)    rows [F,2F) -> G
+
+Cross-attention and GEGLU are token-wise in the latent (each row's output depends only on that
+row and ctx), so on a masked block they run on rows M only; the self-attention's K/V follow
+KV- or Y-mode exactly as for the sequential block.
 """
 from __future__ import annotations
 
@@ -54,6 +69,11 @@ def layer_norm(x, eps=LN_EPS):
     mu = x.mean(axis=-1, keepdims=True)
     var = ((x - mu) ** 2).mean(axis=-1, keepdims=True)
     return (x - mu) / np.sqrt(var + eps)
+
+
+def layer_norm_affine(x, gamma, beta):
+    """LayerNorm with per-channel affine (the SDXL block's norms, R24): LN(x) * gamma + beta."""
+    return layer_norm(x) * f64(gamma) + f64(beta)
 
 
 def gelu_tanh(x):
@@ -109,17 +129,59 @@ def is_parallel(w):
     return w.get("kind", "seq") == "par"
 
 
+def is_sdxl(w):
+    return w.get("kind", "seq") == "sdxl"
+
+
+def geglu(h, W, b):
+    """GEGLU feed-forward input (R24): [P | G] = h W^T + b with P the first F output rows of W,
+    G the last F; returns P * GELU_tanh(G)."""
+    pg = linear(h, W, b)
+    F = pg.shape[1] // 2
+    return pg[:, :F] * gelu_tanh(pg[:, F:])
+
+
+def context_kv(ctx, w):
+    """Cross-attention keys / values of the prompt encoding: ctx Wkv2^T + bkv2 -> (Kc, Vc)."""
+    kv = linear(ctx, w["w_kv2"], w.get("b_kv2"))
+    H = kv.shape[1] // 2
+    return kv[:, :H], kv[:, H:]
+
+
+def _norm1(x, w, mod, H):
+    """The block's first normalised input: affine LN (SDXL) or adaLN-modulated LN."""
+    if is_sdxl(w):
+        return layer_norm_affine(x, w["ln1_w"], w["ln1_b"])
+    sh1, sc1, _, _, _, _ = split_mod(mod, H)
+    return layer_norm(x) * (1.0 + sc1) + sh1
+
+
+def _sdxl_out(x_rows, a_rows, w, ctx, heads):
+    """SDXL block after the self-attention, on the given rows (all token-wise in the latent)."""
+    x1 = f64(x_rows) + linear(a_rows, w["w_o"], w.get("b_o"))
+    h2 = layer_norm_affine(x1, w["ln2_w"], w["ln2_b"])
+    Kc, Vc = context_kv(ctx, w)
+    a2 = attention(linear(h2, w["w_q2"], w.get("b_q2")), Kc, Vc, heads)
+    x2 = x1 + linear(a2, w["w_o2"], w.get("b_o2"))
+    h3 = layer_norm_affine(x2, w["ln3_w"], w["ln3_b"])
+    return x2 + linear(geglu(h3, w["w_up"], w.get("b_up")), w["w_down"], w.get("b_down"))
+
+
 def _qkv_weights(w, H):
     if is_parallel(w):
         W, b = f64(w["w_1"]), f64(w["b_1"])
     else:
-        W, b = f64(w["w_qkv"]), f64(w["b_qkv"])
+        W = f64(w["w_qkv"])
+        b = f64(w["b_qkv"]) if w.get("b_qkv") is not None else np.zeros(3 * H)
     return (W[0:H], b[0:H]), (W[H:2 * H], b[H:2 * H]), (W[2 * H:3 * H], b[2 * H:3 * H])
 
 
-def _block_out(x_rows, h_rows, a_rows, w, mod, H):
+def _block_out(x_rows, h_rows, a_rows, w, mod, H, ctx=None, heads=None):
     """The block output on the given rows from their input x, normalised input h and attention
-    output A: the sequential block's O projection + MLP, or the parallel block's fused output."""
+    output A: the sequential block's O projection + MLP, the parallel block's fused output, or
+    the SDXL block's O projection + cross-attention + GEGLU."""
+    if is_sdxl(w):
+        return _sdxl_out(x_rows, a_rows, w, ctx, heads)
     if not is_parallel(w):
         return _attn_out_and_mlp(x_rows, a_rows, w, mod, H)
     _, _, g1, _, _, _ = split_mod(mod, H)
@@ -138,19 +200,19 @@ def _attn_out_and_mlp(x_rows, a_rows, w, mod, H):
     return y
 
 
-def dense_block(x, w, mod, heads):
-    """Standard block over all L tokens (Fig. 5-Top). Returns (y, K, V)."""
+def dense_block(x, w, mod, heads, ctx=None):
+    """Standard block over all L tokens (Fig. 5-Top). Returns (y, K, V).
+    ctx: the request's prompt encoding [L_ctx, D_ctx] (SDXL block only)."""
     x = f64(x)
     H = x.shape[1]
-    sh1, sc1, _, _, _, _ = split_mod(mod, H)
-    h1 = layer_norm(x) * (1.0 + sc1) + sh1
+    h1 = _norm1(x, w, mod, H)
     (Wq, bq), (Wk, bk), (Wv, bv) = _qkv_weights(w, H)
     Q, K, V = linear(h1, Wq, bq), linear(h1, Wk, bk), linear(h1, Wv, bv)
     a = attention(Q, K, V, heads)
-    return _block_out(x, h1, a, w, mod, H), K, V
+    return _block_out(x, h1, a, w, mod, H, ctx, heads), K, V
 
 
-def masked_block_kv(x_M, M, U, K_U, V_U, w, mod, heads, L):
+def masked_block_kv(x_M, M, U, K_U, V_U, w, mod, heads, L, ctx=None):
     """KV-cache mode (Fig. 7): fresh Q/K/V on rows M, cached K/V on rows U.
 
     x_M: [n, H] block input rows M (ascending ids M). K_U, V_U: [u, H] cached keys/values of the
@@ -158,8 +220,7 @@ def masked_block_kv(x_M, M, U, K_U, V_U, w, mod, heads, L):
     """
     x_M = f64(x_M)
     H = x_M.shape[1]
-    sh1, sc1, _, _, _, _ = split_mod(mod, H)
-    h1_M = layer_norm(x_M) * (1.0 + sc1) + sh1                 # token-wise (L134, L144)
+    h1_M = _norm1(x_M, w, mod, H)                              # token-wise (L134, L144)
     (Wq, bq), (Wk, bk), (Wv, bv) = _qkv_weights(w, H)
     Q_M, K_M, V_M = linear(h1_M, Wq, bq), linear(h1_M, Wk, bk), linear(h1_M, Wv, bv)
     # merged key set in original token order (R10): fresh rows M, cached rows U
@@ -168,10 +229,10 @@ def masked_block_kv(x_M, M, U, K_U, V_U, w, mod, heads, L):
     K_all[M], V_all[M] = K_M, V_M
     K_all[U], V_all[U] = f64(K_U), f64(V_U)
     a_M = attention(Q_M, K_all, V_all, heads)                  # queries from masked rows only (L159)
-    return _block_out(x_M, h1_M, a_M, w, mod, H), K_M, V_M
+    return _block_out(x_M, h1_M, a_M, w, mod, H, ctx, heads), K_M, V_M
 
 
-def masked_block_y(x_M, M, U, x_U, w, mod, heads, L):
+def masked_block_y(x_M, M, U, x_U, w, mod, heads, L, ctx=None):
     """Y-cache mode (Fig. 5-Bottom): block input rows U are the cached activations Y of
     the previous block (R4); K/V over all L rows; Q, O and MLP on rows M. Returns y_M."""
     x_M = f64(x_M)
@@ -179,10 +240,9 @@ def masked_block_y(x_M, M, U, x_U, w, mod, heads, L):
     x_full = np.empty((L, H))
     x_full[M] = x_M
     x_full[U] = f64(x_U)
-    sh1, sc1, _, _, _, _ = split_mod(mod, H)
-    h1 = layer_norm(x_full) * (1.0 + sc1) + sh1
+    h1 = _norm1(x_full, w, mod, H)
     (Wq, bq), (Wk, bk), (Wv, bv) = _qkv_weights(w, H)
     Q_M = linear(h1[M], Wq, bq)
     K, V = linear(h1, Wk, bk), linear(h1, Wv, bv)
     a_M = attention(Q_M, K, V, heads)
-    return _block_out(x_M, h1[M], a_M, w, mod, H)
+    return _block_out(x_M, h1[M], a_M, w, mod, H, ctx, heads)

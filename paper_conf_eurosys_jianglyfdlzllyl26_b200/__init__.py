@@ -82,24 +82,51 @@ def scatter_rows(src, ids, out, stream=None):
     return out
 
 
+_KIND = {"seq": _lib.FPS_BLOCK_SEQ, "par": _lib.FPS_BLOCK_PAR, "sdxl": _lib.FPS_BLOCK_SDXL}
+_SDXL_KEYS = ("ln1_w", "ln1_b", "ln2_w", "ln2_b", "ln3_w", "ln3_b", "w_q2", "b_q2", "w_kv2",
+              "b_kv2", "w_o2", "b_o2")
+
+
 class BlockWeights:
     """Holds one block's device weights (nn.Linear layout) and its C descriptor."""
 
-    def __init__(self, w: dict, heads: int, dtype: int, device="cuda"):
+    def __init__(self, w: dict, heads: int, dtype: int, device="cuda", stream=None):
         """w: the sequential block's w_qkv, b_qkv, w_o, b_o, w_up, b_up, w_down, b_down, or with
-        w["kind"] == "par" the parallel block's w_1 [3H+F, H], b_1, w_2 [H, H+F], b_2."""
+        w["kind"] == "par" the parallel block's w_1 [3H+F, H], b_1, w_2 [H, H+F], b_2, or with
+        w["kind"] == "sdxl" the SDXL block's weights (synth.block_weights names); its GEGLU input
+        projection w_up [2F, H] is repacked on the device by fps_geglu_pack."""
         td = TORCH_DTYPE[dtype]
-        self.kind = _lib.FPS_BLOCK_PAR if w.get("kind", "seq") == "par" else _lib.FPS_BLOCK_SEQ
+        self.kind = _KIND[w.get("kind", "seq")]
         alias = {"w_1": "w_qkv", "b_1": "b_qkv", "w_2": "w_down", "b_2": "b_down"}
         self.t = {alias.get(k, k): torch.as_tensor(np.ascontiguousarray(v)).to(device=device, dtype=td)
-                  for k, v in w.items() if k != "kind"}
+                  for k, v in w.items() if k != "kind" and v is not None}
         H = self.t["w_down"].shape[0]
-        F = (self.t["w_qkv"].shape[0] - 3 * H) if self.kind else self.t["w_up"].shape[0]
+        if self.kind == _lib.FPS_BLOCK_PAR:
+            F = self.t["w_qkv"].shape[0] - 3 * H
+        elif self.kind == _lib.FPS_BLOCK_SDXL:
+            F = self.t["w_up"].shape[0] // 2
+            K = self.t["w_up"].shape[1]
+            wp = torch.empty_like(self.t["w_up"])
+            bp = torch.empty_like(self.t["b_up"]) if "b_up" in self.t else None
+            _lib.fps_geglu_pack(dtype, ptr(self.t["w_up"]), ptr(self.t.get("b_up")), F, K,
+                                ptr(wp), ptr(bp), stream_ptr(stream))
+            self.t["w_up"], self.t["b_up"] = wp, bp
+        else:
+            F = self.t["w_up"].shape[0]
         self.H, self.F, self.heads, self.dtype = H, F, heads, dtype
+        self.D_ctx = self.t["w_kv2"].shape[1] if "w_kv2" in self.t else 0
         self.c = fps_block_weights(H, heads, H // heads, F, dtype,
                                    *[ptr(self.t.get(k)) for k in
                                      ("w_qkv", "b_qkv", "w_o", "b_o", "w_up", "b_up", "w_down",
-                                      "b_down")], self.kind)
+                                      "b_down")], self.kind, self.D_ctx,
+                                   *[ptr(self.t.get(k)) for k in _SDXL_KEYS])
+
+    def context_kv(self, ctx, out=None, stream=None):
+        """SDXL block: the cross-attention K|V rows [n, 2H] of prompt encodings ctx [n, D_ctx]."""
+        out = out if out is not None else torch.empty(ctx.shape[0], 2 * self.H, dtype=ctx.dtype,
+                                                      device=ctx.device)
+        _lib.fps_context_kv(C.byref(self.c), ptr(ctx), ctx.shape[0], ptr(out), stream_ptr(stream))
+        return out
 
 
 class VarlenBatch:
@@ -109,7 +136,7 @@ class VarlenBatch:
     u_row / u_src: Y-mode cached rows. mod: [n_req, 6H] device tensor or None."""
 
     def __init__(self, n_active, L, q_row=None, mod=None, mode=FPS_MODE_KV, u_row=None,
-                 u_src=None, n_unmasked=None, device="cuda"):
+                 u_src=None, n_unmasked=None, device="cuda", ctx_kv=None, n_ctx=None):
         self.n_active = list(map(int, n_active))
         self.L = list(map(int, L))
         cu_q = np.concatenate([[0], np.cumsum(self.n_active)]).astype(np.int32)
@@ -128,6 +155,12 @@ class VarlenBatch:
             max(self.L, default=0), ptr(self.cu_q), ptr(self.cu_k),
             self.h_cu_q.ctypes.data_as(C.c_void_p), self.h_cu_k.ctypes.data_as(C.c_void_p),
             ptr(q_row), ptr(mod), mode, int(cu_u[-1]), ptr(self.cu_u), ptr(u_src), ptr(u_row))
+        if ctx_kv is not None:       # SDXL blocks: request r's prompt K|V rows (n_ctx[r] each)
+            cu_c = np.concatenate([[0], np.cumsum(n_ctx)]).astype(np.int32)
+            self.h_cu_ctx, self.cu_ctx, self.ctx_kv = cu_c, torch.tensor(cu_c, device=device), ctx_kv
+            self.c.d_ctx_kv = ptr(ctx_kv)
+            self.c.d_cu_ctx = ptr(self.cu_ctx)
+            self.c.h_cu_ctx = self.h_cu_ctx.ctypes.data_as(C.c_void_p)
 
     @property
     def total_q(self):
@@ -257,7 +290,7 @@ class Engine:
 
     def __init__(self, layers, heads, mode, dtype, L_img, L_txt, max_batch, n_steps, deltas,
                  cache: Cache, mod_table=None, slots=0, plan_policy=0, plan=None,
-                 cost_model=(0.0, 0.0, 0.0, 0.0)):
+                 cost_model=(0.0, 0.0, 0.0, 0.0), L_ctx=0):
         self.layers = layers                      # list[BlockWeights] (keeps tensors alive)
         self._w = (fps_block_weights * len(layers))(*[l.c for l in layers])
         self._deltas = (C.c_float * n_steps)(*map(float, deltas))
@@ -268,7 +301,8 @@ class Engine:
         d = fps_engine_desc(H, heads, F, len(layers), dtype, mode, L_img, L_txt, max_batch,
                             n_steps, C.cast(self._w, C.c_void_p), ptr(mod_table),
                             C.cast(self._deltas, C.c_void_p), cache.h, slots, plan_policy,
-                            C.cast(self._plan, C.c_void_p), (C.c_double * 4)(*cost_model))
+                            C.cast(self._plan, C.c_void_p), (C.c_double * 4)(*cost_model),
+                            L_ctx, max((getattr(l, "D_ctx", 0) for l in layers), default=0))
         self.desc = d
         h = C.c_void_p()
         _lib.fps_engine_create(C.byref(d), C.byref(h))
@@ -287,12 +321,12 @@ class Engine:
             pass
 
     def run_batch(self, reqs, n_steps, stream=None, load_stream=None):
-        """reqs: list of dicts with template_id, step, n_steps, mask (cuda uint8), x (cuda).
-        Updates each dict's step/status in place."""
+        """reqs: list of dicts with template_id, step, n_steps, mask (cuda uint8), x (cuda),
+        and ctx (cuda [L_ctx, D_ctx]) for SDXL blocks. Updates each dict's step/status in place."""
         arr = (fps_request * max(len(reqs), 1))()
         for i, r in enumerate(reqs):
             arr[i] = fps_request(r["template_id"], r["step"], r["n_steps"], ptr(r["mask"]),
-                                 ptr(r["x"]), 0)
+                                 ptr(r["x"]), 0, ptr(r.get("ctx")))
         ls = stream_ptr(load_stream) if load_stream is not None else None
         _lib.fps_run_batch(self.h, arr, len(reqs), n_steps, stream_ptr(stream), ls)
         for i, r in enumerate(reqs):

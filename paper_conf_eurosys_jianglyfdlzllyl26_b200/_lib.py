@@ -16,7 +16,7 @@ LIB_PATH = os.environ.get("FPS_LIB") or os.path.join(_HERE, "libflashps.so")
 FPS_OK, FPS_EINVAL, FPS_ECUDA, FPS_ENOMEM, FPS_EUNSUPPORTED, FPS_ESTATE = 0, -1, -2, -3, -4, -5
 FPS_F32, FPS_BF16 = 0, 1
 FPS_MODE_KV, FPS_MODE_Y = 0, 1
-FPS_BLOCK_SEQ, FPS_BLOCK_PAR = 0, 1
+FPS_BLOCK_SEQ, FPS_BLOCK_PAR, FPS_BLOCK_SDXL = 0, 1, 2
 
 vp, i32, u32, i64, sz, dbl = C.c_void_p, C.c_int32, C.c_uint32, C.c_int64, C.c_size_t, C.c_double
 P_i32, P_u8, P_dbl, P_f32 = C.POINTER(C.c_int32), C.POINTER(C.c_uint8), C.POINTER(C.c_double), C.POINTER(C.c_float)
@@ -42,14 +42,18 @@ class fps_prefetch_item(C.Structure):
 class fps_block_weights(C.Structure):
     _fields_ = [("H", i32), ("heads", i32), ("head_dim", i32), ("F", i32), ("dtype", i32),
                 ("w_qkv", vp), ("b_qkv", vp), ("w_o", vp), ("b_o", vp), ("w_up", vp),
-                ("b_up", vp), ("w_down", vp), ("b_down", vp), ("kind", i32)]
+                ("b_up", vp), ("w_down", vp), ("b_down", vp), ("kind", i32), ("D_ctx", i32),
+                ("ln1_w", vp), ("ln1_b", vp), ("ln2_w", vp), ("ln2_b", vp), ("ln3_w", vp),
+                ("ln3_b", vp), ("w_q2", vp), ("b_q2", vp), ("w_kv2", vp), ("b_kv2", vp),
+                ("w_o2", vp), ("b_o2", vp)]
 
 
 class fps_varlen_batch(C.Structure):
     _fields_ = [("n_req", i32), ("total_q", i32), ("total_k", i32), ("max_q", i32),
                 ("max_k", i32), ("d_cu_q", vp), ("d_cu_k", vp), ("h_cu_q", vp), ("h_cu_k", vp),
                 ("d_q_row", vp), ("d_mod", vp), ("mode", i32), ("total_u", i32),
-                ("d_cu_u", vp), ("d_u_src", vp), ("d_u_row", vp)]
+                ("d_cu_u", vp), ("d_u_src", vp), ("d_u_row", vp), ("d_ctx_kv", vp),
+                ("d_cu_ctx", vp), ("h_cu_ctx", vp)]
 
 
 class fps_engine_desc(C.Structure):
@@ -57,12 +61,12 @@ class fps_engine_desc(C.Structure):
                 ("mode", i32), ("L_img", i32), ("L_txt", i32), ("max_batch", i32),
                 ("n_steps", i32), ("layers", vp), ("d_mod_table", vp), ("h_deltas", vp),
                 ("cache", vp), ("slots", i32), ("plan_policy", i32), ("h_plan", vp),
-                ("cost_model", dbl * 4)]
+                ("cost_model", dbl * 4), ("L_ctx", i32), ("D_ctx", i32)]
 
 
 class fps_request(C.Structure):
     _fields_ = [("template_id", u32), ("step", i32), ("n_steps", i32), ("d_mask", vp),
-                ("d_x", vp), ("status", i32)]
+                ("d_x", vp), ("status", i32), ("d_ctx", vp)]
 
 
 # (name, restype, argtypes, checked)
@@ -86,6 +90,8 @@ _SIGS = [
     ("fps_cache_entry_bytes", sz, [vp, i32], False),
     ("fps_cache_store", C.c_int, [vp, u32, i32, i32, vp, i32, vp], True),
     ("fps_cache_prefetch", C.c_int, [vp, C.POINTER(fps_prefetch_item), i32, vp, vp], True),
+    ("fps_geglu_pack", C.c_int, [i32, vp, vp, i32, i32, vp, vp, vp], True),
+    ("fps_context_kv", C.c_int, [C.POINTER(fps_block_weights), vp, i32, vp, vp], True),
     ("fps_block_workspace_bytes", sz, [i32, i32, i32, i32, i32], False),
     ("fps_masked_block_forward", C.c_int,
      [C.POINTER(fps_block_weights), C.POINTER(fps_varlen_batch), vp, vp, vp, vp, vp, vp, sz, vp],

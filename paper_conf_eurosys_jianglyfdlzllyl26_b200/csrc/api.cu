@@ -121,7 +121,7 @@ fps_status launch_attention(int dtype, const void* q, const void* kv, void* o, i
 }
 
 struct BlockWs {
-  char *h, *q, *ao, *x1, *h2, *u, *hu;
+  char *h, *q, *ao, *x1, *h2, *u, *hu, *x2;
 };
 
 static size_t align256(size_t v) { return (v + 255) & ~size_t(255); }
@@ -137,11 +137,12 @@ static size_t ws_layout(int H, int F, int dtype, int max_q, int max_u, char* bas
   char* h = take((size_t)max_q * H * e);
   char* q = take((size_t)max_q * H * e);
   char* ao = take((size_t)max_q * H * e);
-  char* x1 = take((size_t)max_q * H * e);
+  char* x1 = take((size_t)max_q * H * 4);              // fp32 for the SDXL block's residual stream
   char* h2 = take((size_t)max_q * H * e);
   char* u = take((size_t)max_q * F * e);
   char* hu = take((size_t)(max_q + max_u) * H * e);   // Y-mode: LN of all rows, token order
-  if (ws) *ws = BlockWs{h, q, ao, x1, h2, u, hu};
+  char* x2 = take((size_t)max_q * H * 4);              // SDXL block: after cross-attention (fp32)
+  if (ws) *ws = BlockWs{h, q, ao, x1, h2, u, hu, x2};
   return off;
 }
 
@@ -151,8 +152,19 @@ static fps_status check_weights(const fps_block_weights* w) {
   FPS_CHECK_ARG(w->H > 0 && w->heads > 0 && w->head_dim > 0 && w->heads * w->head_dim == w->H,
                 "H=%d heads=%d head_dim=%d", w->H, w->heads, w->head_dim);
   FPS_CHECK_ARG(w->F > 0, "F=%d", w->F);
-  FPS_CHECK_ARG(w->kind == FPS_BLOCK_SEQ || w->kind == FPS_BLOCK_PAR, "kind %d", w->kind);
-  if (w->kind == FPS_BLOCK_PAR)
+  FPS_CHECK_ARG(w->kind == FPS_BLOCK_SEQ || w->kind == FPS_BLOCK_PAR || w->kind == FPS_BLOCK_SDXL,
+                "kind %d", w->kind);
+  if (w->kind == FPS_BLOCK_SDXL) {
+    FPS_CHECK_ARG(w->w_qkv && w->w_o && w->w_up && w->w_down && w->w_q2 && w->w_kv2 && w->w_o2,
+                  "SDXL block: weight pointer is NULL");
+    FPS_CHECK_ARG(w->ln1_w && w->ln1_b && w->ln2_w && w->ln2_b && w->ln3_w && w->ln3_b,
+                  "SDXL block: LayerNorm gamma / beta is NULL");
+    FPS_CHECK_ARG(w->D_ctx > 0, "SDXL block: D_ctx=%d", w->D_ctx);
+    if (w->dtype != FPS_BF16 || (g_disable_tc & 1) || w->H % 64 || w->F % 64 || w->D_ctx % 64)
+      return fail(FPS_EUNSUPPORTED,
+                  "SDXL block: bf16 tcgen05 path only (H=%d, F=%d, D_ctx=%d multiples of 64)",
+                  w->H, w->F, w->D_ctx);
+  } else if (w->kind == FPS_BLOCK_PAR)
     FPS_CHECK_ARG(w->w_qkv && w->w_down && !w->w_o && !w->b_o && !w->w_up && !w->b_up,
                   "parallel block: w_qkv (W1) and w_down (W2) set, w_o/b_o/w_up/b_up NULL");
   else
@@ -176,6 +188,16 @@ static fps_status check_batch(const fps_varlen_batch* b) {
   return FPS_OK;
 }
 
+static fps_status check_ctx(const fps_block_weights* w, const fps_varlen_batch* b) {
+  if (w->kind != FPS_BLOCK_SDXL || b->n_req == 0 || b->total_q == 0) return FPS_OK;
+  FPS_CHECK_ARG(b->d_ctx_kv && b->d_cu_ctx && b->h_cu_ctx && b->h_cu_q,
+                "SDXL block: d_ctx_kv / cu_ctx (device and host) / h_cu_q required");
+  for (int r = 0; r < b->n_req; ++r)
+    FPS_CHECK_ARG(b->h_cu_ctx[r + 1] > b->h_cu_ctx[r],
+                  "SDXL block: request %d has an empty prompt context", r);
+  return FPS_OK;
+}
+
 static fps_status block_forward(const fps_block_weights* w, const fps_varlen_batch* b,
                                 const void* x_act, void* y_act, void* kv, const void* xu,
                                 cudaEvent_t kv_ready, void* d_ws, size_t ws_bytes,
@@ -186,26 +208,31 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
   BlockWs ws;
   const size_t need = ws_layout(H, F, dt, tq, tu, (char*)d_ws, &ws);
   FPS_CHECK_ARG(ws_bytes >= need, "workspace %zu < %zu bytes", ws_bytes, need);
-  const char* mod = (const char*)b->d_mod;
+  const bool sdxl = w->kind == FPS_BLOCK_SDXL;
+  const char* mod = sdxl ? nullptr : (const char*)b->d_mod;
   auto modp = [&](int off) -> const void* { return mod ? mod + (size_t)off * H * e : nullptr; };
+  // a4, the first norm: adaLN-modulated LN, or the SDXL block's affine LN (reading R24)
+  auto ln1 = [&](const void* x, const int32_t* rows, int n, void* out, const int32_t* cu,
+                 const int32_t* out_rows) -> fps_status {
+    if (sdxl) return launch_ln_affine(dt, x, rows, n, H, out, w->ln1_w, w->ln1_b, s, out_rows);
+    return launch_ln_mod(dt, x, rows, n, H, out, cu, b->n_req, mod, 0, s, out_rows);
+  };
 
   // Y-mode, sequential block: Q over the active rows, K|V in ONE GEMM over all rows of the
   // merged buffer (fresh rows M and cached input rows U, normalised into token order) -- the same
   // FLOPs as the QKV GEMM on M plus a K|V GEMM on U, in fewer waves with no 256-row padding at
   // the M/U split (C3: 6 + 1 waves instead of 3 + 5)
-  const bool y_split = tu > 0 && tq > 0 && w->kind == FPS_BLOCK_SEQ;
+  const bool y_split = tu > 0 && tq > 0 && w->kind != FPS_BLOCK_PAR;
   if (y_split) {
-    FPS_TRY(launch_ln_mod(dt, x_act, nullptr, tq, H, ws.h, b->d_cu_q, b->n_req, b->d_mod, 0, s));
+    FPS_TRY(ln1(x_act, nullptr, tq, ws.h, b->d_cu_q, nullptr));
     Epilogue eq{};
     eq.bias = w->b_qkv;
     eq.out0 = ws.q; eq.ld0 = H; eq.split = H;
     FPS_TRY(launch_gemm(dt, ws.h, w->w_qkv, tq, H, H, eq, s));
-    FPS_TRY(launch_ln_mod(dt, x_act, nullptr, tq, H, ws.hu, b->d_cu_q, b->n_req, b->d_mod, 0, s,
-                          b->d_q_row));
+    FPS_TRY(ln1(x_act, nullptr, tq, ws.hu, b->d_cu_q, b->d_q_row));
     if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
     kv_ready = nullptr;
-    FPS_TRY(launch_ln_mod(dt, xu, b->d_u_src, tu, H, ws.hu, b->d_cu_u, b->n_req, b->d_mod, 0, s,
-                          b->d_u_row));
+    FPS_TRY(ln1(xu, b->d_u_src, tu, ws.hu, b->d_cu_u, b->d_u_row));
     Epilogue ek{};
     ek.bias = w->b_qkv ? (const char*)w->b_qkv + (size_t)H * e : nullptr;
     ek.out0 = kv; ek.ld0 = 2 * H; ek.split = 2 * H;
@@ -214,7 +241,7 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
   }
   if (tq > 0 && !y_split) {
     // a4: h1 = LN(x)(1+scale1)+shift1 on active rows
-    FPS_TRY(launch_ln_mod(dt, x_act, nullptr, tq, H, ws.h, b->d_cu_q, b->n_req, b->d_mod, 0, s));
+    FPS_TRY(ln1(x_act, nullptr, tq, ws.h, b->d_cu_q, nullptr));
     // a5: [tq,H] x [3H,H]^T; Q -> compact, K|V -> merged key rows at original positions
     Epilogue ep{};
     ep.bias = w->b_qkv;
@@ -233,7 +260,7 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
     // Y-mode: cached block-input rows U -> LN -> K|V projection (Fig. 5-Bottom, reading R5)
     if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
     kv_ready = nullptr;
-    FPS_TRY(launch_ln_mod(dt, xu, b->d_u_src, tu, H, ws.hu, b->d_cu_u, b->n_req, b->d_mod, 0, s));
+    FPS_TRY(ln1(xu, b->d_u_src, tu, ws.hu, b->d_cu_u, nullptr));
     Epilogue ep{};
     ep.bias = w->b_qkv ? (const char*)w->b_qkv + (size_t)H * e : nullptr;
     ep.out0 = kv; ep.ld0 = 2 * H; ep.map0 = b->d_u_row;
@@ -264,7 +291,42 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
     ep.resid = x_act; ep.ld_resid = H;
     ep.gate = modp(2); ep.gate_stride = 6 * H; ep.cu = b->d_cu_q; ep.n_req = b->n_req;
     ep.out0 = ws.x1; ep.ld0 = H; ep.split = H;
+    ep.out0_f32 = sdxl;          // SDXL: keep the residual stream x1, x2 in fp32 (R24)
     FPS_TRY(launch_gemm(dt, ws.ao, w->w_o, tq, H, H, ep, s));
+  }
+  if (sdxl) {
+    // SDXL block (reading R24): cross-attention of the active rows to the request's prompt
+    // K|V (token-wise in the latent, so rows M only), then the GEGLU feed-forward
+    FPS_TRY(launch_ln_affine_f32in((const float*)ws.x1, tq, H, ws.h2, w->ln2_w, w->ln2_b, s));
+    {
+      Epilogue ep{};
+      ep.bias = w->b_q2;
+      ep.out0 = ws.q; ep.ld0 = H; ep.split = H;
+      FPS_TRY(launch_gemm(dt, ws.h2, w->w_q2, tq, H, H, ep, s));
+    }
+    int max_c = 0;
+    for (int r = 0; r < b->n_req; ++r) max_c = std::max(max_c, b->h_cu_ctx[r + 1] - b->h_cu_ctx[r]);
+    FPS_TRY(launch_attention(dt, ws.q, b->d_ctx_kv, ws.ao, w->heads, w->head_dim, b->d_cu_q,
+                             b->d_cu_ctx, b->h_cu_q, b->h_cu_ctx, b->n_req, tq, b->max_q, max_c, s));
+    {
+      Epilogue ep{};
+      ep.bias = w->b_o2;
+      ep.resid = ws.x1; ep.ld_resid = H; ep.resid_f32 = 1;
+      ep.out0 = ws.x2; ep.ld0 = H; ep.split = H; ep.out0_f32 = 1;
+      FPS_TRY(launch_gemm(dt, ws.ao, w->w_o2, tq, H, H, ep, s));
+    }
+    FPS_TRY(launch_ln_affine_f32in((const float*)ws.x2, tq, H, ws.h2, w->ln3_w, w->ln3_b, s));
+    {
+      Epilogue ep{};
+      ep.bias = w->b_up; ep.act = 2;
+      ep.out0 = ws.u; ep.ld0 = F; ep.split = 2 * F;
+      FPS_TRY(launch_gemm(dt, ws.h2, w->w_up, tq, 2 * F, H, ep, s));
+    }
+    Epilogue ep{};
+    ep.bias = w->b_down;
+    ep.resid = ws.x2; ep.ld_resid = H; ep.resid_f32 = 1;
+    ep.out0 = y_act; ep.ld0 = H; ep.split = H;
+    return launch_gemm(dt, ws.u, w->w_down, tq, H, F, ep, s);
   }
   // a8: y = x1 + gate2 (GELU(LN(x1)(1+scale2)+shift2 W1^T + b1) W2^T + b2)
   FPS_TRY(launch_ln_mod(dt, ws.x1, nullptr, tq, H, ws.h2, b->d_cu_q, b->n_req, b->d_mod, 3 * H, s));
@@ -412,8 +474,34 @@ fps_status fps_masked_block_forward(const fps_block_weights* w, const fps_varlen
   if (b->total_q > 0 && b->d_q_row == nullptr)
     FPS_CHECK_ARG(b->total_q == b->total_k, "d_q_row NULL requires total_q == total_k");
   FPS_CHECK_ARG(w->heads * w->head_dim == w->H, "heads*head_dim != H");
+  FPS_TRY(check_ctx(w, b));
   return block_forward(w, b, d_x_act, d_y_act, d_kv, d_xu, (cudaEvent_t)kv_ready, d_ws, ws_bytes,
                        as_stream(stream));
+}
+
+fps_status fps_geglu_pack(int32_t dtype, const void* d_w, const void* d_b, int32_t F, int32_t K,
+                          void* d_w_out, void* d_b_out, void* stream) {
+  FPS_CHECK_ARG(dtype == FPS_BF16 || dtype == FPS_F32, "dtype %d", dtype);
+  FPS_CHECK_ARG(F > 0 && F % 32 == 0 && K > 0 && (K * elt_size(dtype)) % 16 == 0,
+                "F=%d must be a positive multiple of 32, K*elt a multiple of 16 (K=%d)", F, K);
+  FPS_CHECK_ARG(d_w && d_w_out && (!d_b || d_b_out), "NULL pointer");
+  FPS_CHECK_ARG(d_w != d_w_out && (!d_b || d_b != d_b_out), "outputs must not alias inputs");
+  FPS_CHECK_ARG(aligned16(d_w) && aligned16(d_w_out), "weights must be 16-byte aligned");
+  return launch_geglu_pack(dtype, d_w, d_b, F, K, d_w_out, d_b ? d_b_out : nullptr,
+                           as_stream(stream));
+}
+
+fps_status fps_context_kv(const fps_block_weights* w, const void* d_ctx, int32_t n_rows,
+                          void* d_ctx_kv, void* stream) {
+  FPS_TRY(check_weights(w));
+  FPS_CHECK_ARG(w->kind == FPS_BLOCK_SDXL, "fps_context_kv: SDXL block weights required");
+  FPS_CHECK_ARG(n_rows >= 0, "n_rows < 0");
+  if (n_rows == 0) return FPS_OK;
+  FPS_CHECK_ARG(d_ctx && d_ctx_kv, "NULL pointer");
+  Epilogue ep{};
+  ep.bias = w->b_kv2;
+  ep.out0 = d_ctx_kv; ep.ld0 = 2 * w->H; ep.split = 2 * w->H;
+  return launch_gemm(w->dtype, d_ctx, w->w_kv2, n_rows, 2 * w->H, w->D_ctx, ep, as_stream(stream));
 }
 
 fps_status fps_linear(int32_t dtype, const void* d_a, const void* d_w, const void* d_bias,
@@ -456,6 +544,7 @@ fps_status fps_dense_block_forward(const fps_block_weights* w, const fps_varlen_
   FPS_TRY(check_batch(b));
   FPS_CHECK_ARG(b->d_q_row == nullptr && b->total_q == b->total_k,
                 "dense block: d_q_row must be NULL and total_q == total_k");
+  FPS_TRY(check_ctx(w, b));
   fps_varlen_batch bb = *b;
   bb.mode = FPS_MODE_KV;
   bb.total_u = 0;

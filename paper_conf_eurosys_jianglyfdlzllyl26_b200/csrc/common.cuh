@@ -226,9 +226,24 @@ __device__ __forceinline__ float gelu_tanh_fast(float x) {
 //   resid: v = resid[r, c] + gate[req(r), c] * v      (gate NULL -> 1)
 //   routing: columns [0, split) -> out0 (row r, ld0), columns [split, N) -> out1 with row
 //            map1[r] (NULL -> r), column c - split, ld1.  split = N when there is no out1.
+// Row-norm output transform: out = LN(x) * (one + scale[req]) + shift[req], the request's vectors
+// `stride` elements apart (req from cu over rows); stride 0 = one shared vector (affine LN with
+// scale = gamma, shift = beta, one = 0); shift == nullptr = plain LN.
+template <typename T>
+struct LnMod {
+  const T* shift;
+  const T* scale;
+  int stride;
+  float one;
+  const int32_t* cu;
+  int n_req;
+};
+
 struct Epilogue {
   const void* bias;          // [N] or null
-  int act;                   // 0 none, 1 gelu_tanh
+  int act;                   // 0 none, 1 gelu_tanh, 2 GEGLU over 32-column (value, gate) pairs:
+                             //   columns [64j, 64j+32) x GELU_tanh([64j+32, 64j+64)) -> output
+                             //   columns [32j, 32j+32) of out0 (tcgen05 path; no resid/gate)
   const void* resid;         // [M, ld_resid] or null
   int ld_resid;
   const void* gate;          // per-request gate vectors: gate + req * gate_stride, or null
@@ -242,6 +257,8 @@ struct Epilogue {
   // applied only to columns >= act_from (the parallel block's fused QKV|MLP projection)
   void* out2; int ld2; int split2;
   int act_from;
+  // fp32 residual stream (SDXL block, tcgen05 path only): out0 and/or resid hold fp32 rows
+  int out0_f32, resid_f32;
 };
 
 }  // namespace fps

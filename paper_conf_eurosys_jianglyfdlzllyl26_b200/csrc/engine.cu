@@ -33,6 +33,11 @@ struct fps_engine {
   uint8_t* d_masks = nullptr;
   int32_t *d_off = nullptr, *d_mids = nullptr, *d_uids = nullptr, *d_nm = nullptr;
   int32_t *d_meta = nullptr;   // cu_q | cu_k | cu_u | q_row | u_row | mod_ids
+  // SDXL blocks: batch prompt encodings and their per-block cross-attention K|V
+  int n_sdxl = 0;
+  std::vector<int> sdxl_slot;  // per layer: index into ctx_kv, or -1
+  char *ctx_in = nullptr, *ctx_kv = nullptr;
+  int32_t *d_cu_ctx = nullptr, *h_cu_ctx = nullptr;
   float* d_delta = nullptr;
   // pinned host staging
   int32_t* h_meta = nullptr;
@@ -53,6 +58,10 @@ static void free_engine(fps_engine* e) {
                   e->kv_scratch, e->final_slot, e->ws, e->mod_batch};
   for (char* p : bufs) if (p) cudaFree(p);
   for (char* p : e->slots) if (p) cudaFree(p);
+  if (e->ctx_in) cudaFree(e->ctx_in);
+  if (e->ctx_kv) cudaFree(e->ctx_kv);
+  if (e->d_cu_ctx) cudaFree(e->d_cu_ctx);
+  if (e->h_cu_ctx) cudaFreeHost(e->h_cu_ctx);
   if (e->d_masks) cudaFree(e->d_masks);
   int32_t* ib[] = {e->d_off, e->d_mids, e->d_uids, e->d_nm, e->d_meta};
   for (int32_t* p : ib) if (p) cudaFree(p);
@@ -67,10 +76,14 @@ static void free_engine(fps_engine* e) {
 }
 
 // Per-block FLOPs of one request (Table 1, exact per mode; oracle/counters.py restated).
-static double flops_block(int mode, double n, double L, double H, double F) {
+// SDXL blocks (R24) add, per active row, the cross-attention Q / O projections (4 H^2), its
+// attention over Lc prompt tokens (4 Lc H) and the GEGLU's doubled up-projection (2 H F).
+static double flops_block(int mode, double n, double L, double H, double F, int kind = 0,
+                          double Lc = 0) {
   const double attn = 4.0 * n * L * H;
-  if (mode == FPS_MODE_KV) return 8.0 * n * H * H + 4.0 * n * H * F + attn;
-  return 4.0 * n * H * H + 4.0 * L * H * H + 4.0 * n * H * F + attn;
+  const double extra = kind == FPS_BLOCK_SDXL ? n * (4.0 * H * H + 4.0 * Lc * H + 2.0 * H * F) : 0.0;
+  if (mode == FPS_MODE_KV) return 8.0 * n * H * H + 4.0 * n * H * F + attn + extra;
+  return 4.0 * n * H * H + 4.0 * L * H * H + 4.0 * n * H * F + attn + extra;
 }
 
 }  // namespace fps
@@ -97,6 +110,13 @@ fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out) {
       else FPS_CHECK_ARG(!seen, "KV-mode plan must be monotone (reading R11)");
     }
   }
+  for (int l = 0; l < d.n_layers; ++l) {
+    FPS_CHECK_ARG(d.layers[l].H == d.H && d.layers[l].F == d.F && d.layers[l].dtype == d.dtype,
+                  "layer %d: H / F / dtype differ from the engine's", l);
+    if (d.layers[l].kind == FPS_BLOCK_SDXL)
+      FPS_CHECK_ARG(d.L_ctx > 0 && d.layers[l].D_ctx == d.D_ctx,
+                    "layer %d: SDXL block needs L_ctx > 0 and D_ctx == the engine's", l);
+  }
   auto* e = new (std::nothrow) fps_engine();
   if (!e) return fail(FPS_ENOMEM, "engine alloc");
   e->d = d;
@@ -106,6 +126,9 @@ fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out) {
   e->d.layers = nullptr;
   e->d.h_deltas = nullptr;
   e->d.h_plan = nullptr;
+  e->sdxl_slot.assign(d.n_layers, -1);
+  for (int l = 0; l < d.n_layers; ++l)
+    if (d.layers[l].kind == FPS_BLOCK_SDXL) e->sdxl_slot[l] = e->n_sdxl++;
   e->L = d.L_img + d.L_txt;
   e->elt = d.dtype == FPS_BF16 ? 2 : 4;
   e->W = d.mode == FPS_MODE_KV ? 2 * d.H : d.H;
@@ -137,6 +160,13 @@ fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out) {
   dmal(&e->mod_batch, (size_t)d.n_layers * d.max_batch * 6 * e->row_h);
   e->slots.assign(e->D, nullptr);
   for (int i = 0; i < e->D; ++i) dmal(&e->slots[i], slot_bytes);
+  if (e->n_sdxl) {
+    dmal(&e->ctx_in, (size_t)d.max_batch * d.L_ctx * d.D_ctx * e->elt);
+    dmal(&e->ctx_kv, (size_t)e->n_sdxl * d.max_batch * d.L_ctx * 2 * e->row_h);
+    if (err == cudaSuccess) err = cudaMalloc((void**)&e->d_cu_ctx, (d.max_batch + 1) * 4);
+    if (err == cudaSuccess)
+      err = cudaHostAlloc((void**)&e->h_cu_ctx, (d.max_batch + 1) * 4, cudaHostAllocDefault);
+  }
   if (err == cudaSuccess) err = cudaMalloc((void**)&e->d_masks, R);
   const size_t meta_ints = 3 * (d.max_batch + 1) + 2 * R + (size_t)d.n_layers * d.max_batch;
   auto imal = [&](int32_t** p, size_t n) {
@@ -259,6 +289,24 @@ static fps_status admit(fps_engine* e, fps_request* reqs, const std::vector<int>
   B.h_cu_q = cu_q;
   B.h_cu_k = cu_k;
   B.h_cu_u = cu_u;
+  if (e->n_sdxl) {
+    // SDXL blocks: the prompt is fixed over the steps, so each block's cross-attention K|V
+    // is projected once per admission (one GEMM per SDXL block over the batch's prompts)
+    const int Lc = e->d.L_ctx;
+    const size_t ctx_row = (size_t)e->d.D_ctx * e->elt;
+    for (int i = 0; i < n; ++i) {
+      FPS_CHECK_ARG(reqs[live[i]].d_ctx, "request %d: SDXL blocks need d_ctx", live[i]);
+      FPS_COPY_TRY(cs, cudaMemcpyAsync(e->ctx_in + (size_t)i * Lc * ctx_row, reqs[live[i]].d_ctx,
+                                       Lc * ctx_row, cudaMemcpyDeviceToDevice, cs));
+    }
+    for (int i = 0; i <= n; ++i) e->h_cu_ctx[i] = i * Lc;
+    FPS_COPY_TRY(cs, cudaMemcpyAsync(e->d_cu_ctx, e->h_cu_ctx, (n + 1) * 4, cudaMemcpyHostToDevice, cs));
+    for (int l = 0; l < e->d.n_layers; ++l)
+      if (e->sdxl_slot[l] >= 0)
+        FPS_TRY(fps_context_kv(&e->layers[l], e->ctx_in, n * Lc,
+                               e->ctx_kv + (size_t)e->sdxl_slot[l] * e->d.max_batch * Lc * 2 * e->row_h,
+                               cs));
+  }
   return FPS_OK;
 }
 
@@ -269,17 +317,26 @@ static void make_plan(fps_engine* e, const Batch& B) {
   const double b = e->d.cost_model[1] > 0 ? e->d.cost_model[1] : 0.01;
   const double c = e->d.cost_model[2] > 0 ? e->d.cost_model[2] : 1.0 / 5.0e7;   // ms per byte
   const double ec = e->d.cost_model[3] > 0 ? e->d.cost_model[3] : 0.01;
-  double fm = 0, fd = 0, by = 0, byf = 0;
-  const double H = e->d.H, F = e->d.F, L = e->L;
+  double by = 0, byf = 0;
+  const double H = e->d.H, F = e->d.F, L = e->L, Lc = e->d.L_ctx;
+  std::vector<double> Cw(N), Cwo(N), Lm(N);
+  for (int l = 0; l < N; ++l) {
+    const int kind = e->layers[l].kind;
+    double fm = 0, fd = 0;
+    for (int i = 0; i < B.n; ++i) {
+      fm += flops_block(e->d.mode, B.nq[i], L, H, F, kind, Lc);
+      fd += flops_block(FPS_MODE_KV, L, L, H, F, kind, Lc);
+    }
+    Cw[l] = a * fm + b;
+    Cwo[l] = a * fd + b;
+  }
   for (int i = 0; i < B.n; ++i) {
-    fm += flops_block(e->d.mode, B.nq[i], L, H, F);
-    fd += flops_block(FPS_MODE_KV, L, L, H, F);
     // rows the load moves: U, or the whole entry for the whole-entry DMA method
     const double rows = (B.nu[i] > 0 && cache_writes_all_rows(e->d.cache)) ? e->d.L_img : B.nu[i];
     by += rows * e->row_w;
     byf += rows * e->row_h;
   }
-  std::vector<double> Cw(N, a * fm + b), Cwo(N, a * fd + b), Lm(N, by > 0 ? c * by + ec : 0.0);
+  for (int l = 0; l < N; ++l) Lm[l] = by > 0 ? c * by + ec : 0.0;
   const double fin = byf > 0 ? c * byf + ec : 0.0;
   if (e->d.plan_policy == 0) {
     fps_plan_pipeline(Cw.data(), Cwo.data(), Lm.data(), N, e->d.mode, fin, e->last_plan.data(),
@@ -394,6 +451,18 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
     const void* mod = e->d.d_mod_table ? e->mod_batch + (size_t)l * n * 6 * e->row_h : nullptr;
     vb.d_mod = mod;
     vd.d_mod = mod;
+    if (e->sdxl_slot[l] >= 0) {
+      vb.d_ctx_kv = e->ctx_kv +
+                    (size_t)e->sdxl_slot[l] * e->d.max_batch * e->d.L_ctx * 2 * e->row_h;
+      vb.d_cu_ctx = e->d_cu_ctx;
+      vb.h_cu_ctx = e->h_cu_ctx;
+    } else {
+      vb.d_ctx_kv = nullptr;
+      vb.d_cu_ctx = vb.h_cu_ctx = nullptr;
+    }
+    vd.d_ctx_kv = vb.d_ctx_kv;
+    vd.d_cu_ctx = vb.d_cu_ctx;
+    vd.h_cu_ctx = vb.h_cu_ctx;
     if (!use[l]) {
       if (!rep_full) {
         // Y-mode cached -> uncached: rebuild the full input from act rows M and the cached

@@ -59,7 +59,7 @@ __device__ __forceinline__ RowCtx row_ctx(const Epilogue& ep, int M, int row) {
 
 // Global loads of the fused operands of 32 columns col0.. of one row (issued before use).
 struct ChunkIn {
-  uint4 bv[4], rv[4], gv[4];
+  uint4 bv[4], rv[8], gv[4];   // rv[4..7]: second halves of an fp32 residual
 };
 __device__ __forceinline__ void chunk_load(const Epilogue& ep, const RowCtx& rc, int N, int row,
                                            int col0, ChunkIn& in) {
@@ -70,9 +70,15 @@ __device__ __forceinline__ void chunk_load(const Epilogue& ep, const RowCtx& rc,
     const int c0 = col0 + g * 8;
     const bool ok = rc.ok && c0 < N;
     in.bv[g] = (bias && ok) ? __ldg(reinterpret_cast<const uint4*>(bias + c0)) : make_uint4(0, 0, 0, 0);
-    in.rv[g] = (resid && ok)
-                   ? __ldg(reinterpret_cast<const uint4*>(resid + (size_t)row * ep.ld_resid + c0))
-                   : make_uint4(0, 0, 0, 0);
+    if (ep.resid_f32) {
+      const float* rf = reinterpret_cast<const float*>(ep.resid) + (size_t)row * ep.ld_resid + c0;
+      in.rv[g] = (resid && ok) ? __ldg(reinterpret_cast<const uint4*>(rf)) : make_uint4(0, 0, 0, 0);
+      in.rv[g + 4] = (resid && ok) ? __ldg(reinterpret_cast<const uint4*>(rf + 4)) : make_uint4(0, 0, 0, 0);
+    } else {
+      in.rv[g] = (resid && ok)
+                     ? __ldg(reinterpret_cast<const uint4*>(resid + (size_t)row * ep.ld_resid + c0))
+                     : make_uint4(0, 0, 0, 0);
+    }
     in.gv[g] = (rc.gate && ok) ? __ldg(reinterpret_cast<const uint4*>(rc.gate + c0))
                                : make_uint4(0, 0, 0, 0);
   }
@@ -100,7 +106,12 @@ __device__ __forceinline__ void chunk_store(const Epilogue& ep, const RowCtx& rc
     }
     if (ep.resid) {
       float rr[8];
-      Vec16<__nv_bfloat16>::unpack(in.rv[g], rr);
+      if (ep.resid_f32) {
+        Vec16<float>::unpack(in.rv[g], rr);
+        Vec16<float>::unpack(in.rv[g + 4], rr + 4);
+      } else {
+        Vec16<__nv_bfloat16>::unpack(in.rv[g], rr);
+      }
       if (rc.gate) {
         Vec16<__nv_bfloat16>::unpack(in.gv[g], t);
 #pragma unroll
@@ -109,6 +120,12 @@ __device__ __forceinline__ void chunk_store(const Epilogue& ep, const RowCtx& rc
 #pragma unroll
         for (int e = 0; e < 8; ++e) v[e] = rr[e] + v[e];
       }
+    }
+    if (ep.out0_f32 && c0 < ep.split) {
+      float* df = reinterpret_cast<float*>(ep.out0) + (size_t)rc.orow0 * ep.ld0 + c0;
+      reinterpret_cast<uint4*>(df)[0] = Vec16<float>::pack(v);
+      reinterpret_cast<uint4*>(df)[1] = Vec16<float>::pack(v + 4);
+      continue;
     }
     __nv_bfloat16* dst =
         c0 < ep.split ? reinterpret_cast<__nv_bfloat16*>(ep.out0) + (size_t)rc.orow0 * ep.ld0 + c0
@@ -120,11 +137,57 @@ __device__ __forceinline__ void chunk_store(const Epilogue& ep, const RowCtx& rc
   }
 }
 
+// GEGLU (act 2, SDXL block R24): accumulator columns col0..+31 are the value half and
+// col0+32..+63 the gate half of output columns col0/2..+31 (weights packed by
+// launch_geglu_pack); out = (value + b) * GELU_tanh(gate + b').
+__device__ __forceinline__ void geglu_store(const Epilogue& ep, const RowCtx& rc, int N, int col0,
+                                            const uint32_t* ra, const uint32_t* rg,
+                                            const ChunkIn& ia, const ChunkIn& ig) {
+  if (!rc.ok || col0 >= N) return;
+  __nv_bfloat16* out =
+      reinterpret_cast<__nv_bfloat16*>(ep.out0) + (size_t)rc.orow0 * ep.ld0 + (col0 >> 1);
+#pragma unroll
+  for (int g = 0; g < 4; ++g) {
+    float v[8], t[8], b[8];
+#pragma unroll
+    for (int e = 0; e < 8; ++e) {
+      v[e] = __uint_as_float(ra[g * 8 + e]);
+      t[e] = __uint_as_float(rg[g * 8 + e]);
+    }
+    if (ep.bias) {
+      Vec16<__nv_bfloat16>::unpack(ia.bv[g], b);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) v[e] += b[e];
+      Vec16<__nv_bfloat16>::unpack(ig.bv[g], b);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) t[e] += b[e];
+    }
+#pragma unroll
+    for (int e = 0; e < 8; ++e) v[e] *= gelu_tanh_fast(t[e]);
+    *reinterpret_cast<uint4*>(out + g * 8) = Vec16<__nv_bfloat16>::pack(v);
+  }
+}
+
 // Epilogue of one accumulator tile for the calling thread's output row (thread = TMEM lane).
 template <int BN>
 __device__ __forceinline__ void epilogue_tile(const Epilogue& ep, int M, int N, int row,
                                               int col_base, uint32_t taddr) {
   const RowCtx rc = row_ctx(ep, M, row);
+  if (ep.act == 2) {
+#pragma unroll 1
+    for (int c = 0; c < BN / 64; ++c) {
+      uint32_t ra[32], rg[32];
+      tc::tmem_ld32(taddr + c * 64, ra);
+      tc::tmem_ld32(taddr + c * 64 + 32, rg);
+      const int col0 = col_base + c * 64;
+      ChunkIn ia, ig;
+      chunk_load(ep, rc, N, row, col0, ia);
+      chunk_load(ep, rc, N, row, col0 + 32, ig);
+      tc::tmem_wait_ld();
+      geglu_store(ep, rc, N, col0, ra, rg, ia, ig);
+    }
+    return;
+  }
 #pragma unroll 1
   for (int c = 0; c < BN / 32; ++c) {
     uint32_t r[32];
@@ -693,7 +756,7 @@ fps_status launch_gemm_tc(const void* A, const void* B, int M, int N, int K, con
   // tested, but measured no faster at the masked-block shapes (1331x9216x3072: 59.8 vs 59.2 us
   // for the pair kernel -- under the power cap the MMAs on TMA zero-fill rows cost little) and
   // slow for small activation blocks (NA = 144: 3.6x), so it is only selectable by force
-  if (g_gemm_force == 3) {
+  if (g_gemm_force == 3 && ep.act != 2) {
     long cs = 0;
     return launch_pair_swap<6>(A, B, M, N, K, swap_block(M, N, &cs), ep, s);
   }

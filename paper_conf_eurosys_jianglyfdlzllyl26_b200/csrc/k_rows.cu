@@ -1,5 +1,7 @@
 // a1 mask index, a2/a9/a3 row movement, a4 row-norm + modulation, sampler update.
 // PAPER.md L130 (token categorisation), L157 (extract / replenish rows), L134 (token-wise LN).
+#include <algorithm>
+
 #include "kernels.h"
 
 namespace fps {
@@ -160,14 +162,51 @@ fps_status launch_copy_rows(const void* src, const int32_t* src_ids, const int32
 }
 
 // ---------------------------------------------------------------------------------------
+// GEGLU weight packing (SDXL block, R24): output row j of group k = j / 64 takes value row
+// 32k + (j % 64) for j % 64 < 32, else gate row F + 32k + (j % 64 - 32).  Not on the hot path
+// (run once when weights are loaded).
+__device__ __forceinline__ int geglu_src_row(int j, int F) {
+  const int k = j >> 6, w = j & 63;
+  return w < 32 ? 32 * k + w : F + 32 * k + (w - 32);
+}
+
+__global__ void __launch_bounds__(256) geglu_pack_kernel(const uint4* __restrict__ w,
+                                                         uint4* __restrict__ w_out, int F, int vpr,
+                                                         const char* __restrict__ b,
+                                                         char* __restrict__ b_out, int elt) {
+  const long long total = 2LL * F * vpr;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < total;
+       i += (long long)gridDim.x * blockDim.x) {
+    const int row = (int)(i / vpr), c = (int)(i - (long long)row * vpr);
+    w_out[i] = w[(long long)geglu_src_row(row, F) * vpr + c];
+  }
+  if (b && blockIdx.x == 0)
+    for (int j = threadIdx.x; j < 2 * F; j += blockDim.x)
+      for (int e = 0; e < elt; ++e) b_out[(size_t)j * elt + e] = b[(size_t)geglu_src_row(j, F) * elt + e];
+}
+
+fps_status launch_geglu_pack(int dtype, const void* w, const void* b, int F, int K, void* w_out,
+                             void* b_out, cudaStream_t s) {
+  const int elt = dtype == FPS_BF16 ? 2 : 4;
+  const int vpr = K * elt / 16;
+  const long long total = 2LL * F * vpr;
+  const int grid = (int)std::min<long long>((total + 255) / 256, kNumSMs * 8LL);
+  geglu_pack_kernel<<<grid, 256, 0, s>>>(reinterpret_cast<const uint4*>(w),
+                                         reinterpret_cast<uint4*>(w_out), F, vpr,
+                                         reinterpret_cast<const char*>(b),
+                                         reinterpret_cast<char*>(b_out), elt);
+  count_launch();
+  FPS_LAUNCH_CHECK();
+  return FPS_OK;
+}
+
+// ---------------------------------------------------------------------------------------
 // a4: one warp per row; the row stays in registers (VPT 16-B vectors per lane), two-pass
 // mean / variance in fp32, then the per-request adaLN modulation (reading R2/R3).
 template <typename T, int VPT>
 __global__ void __launch_bounds__(128) ln_mod_kernel(const T* __restrict__ x,
                                                      const int32_t* __restrict__ rows, int n,
-                                                     int H, T* __restrict__ out,
-                                                     const int32_t* __restrict__ cu, int n_req,
-                                                     const T* __restrict__ mod, int shift_off,
+                                                     int H, T* __restrict__ out, LnMod<T> md,
                                                      const int32_t* __restrict__ out_rows) {
   constexpr int NV = Vec16<T>::N;
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
@@ -203,12 +242,13 @@ __global__ void __launch_bounds__(128) ln_mod_kernel(const T* __restrict__ x,
   }
   const float var = warp_sum(sq) / (float)H;
   const float rstd = 1.0f / sqrtf(var + 1e-6f);
+  const bool mod = md.shift != nullptr;
   const T* shift = nullptr;
   const T* scale = nullptr;
   if (mod) {
-    const int r = find_req(cu, n_req, warp);
-    shift = mod + (size_t)r * 6 * H + shift_off;
-    scale = shift + H;
+    const size_t off = md.stride ? (size_t)find_req(md.cu, md.n_req, warp) * md.stride : 0;
+    shift = md.shift + off;
+    scale = md.scale + off;
   }
   uint4* o = reinterpret_cast<uint4*>(out + (size_t)(out_rows ? __ldg(out_rows + warp) : warp) * H);
 #pragma unroll
@@ -221,7 +261,7 @@ __global__ void __launch_bounds__(128) ln_mod_kernel(const T* __restrict__ x,
         Vec16<T>::unpack(reinterpret_cast<const uint4*>(shift)[vi], sh);
         Vec16<T>::unpack(reinterpret_cast<const uint4*>(scale)[vi], sc);
 #pragma unroll
-        for (int e = 0; e < NV; ++e) r[e] = (v[k][e] - mean) * rstd * (1.0f + sc[e]) + sh[e];
+        for (int e = 0; e < NV; ++e) r[e] = (v[k][e] - mean) * rstd * (md.one + sc[e]) + sh[e];
       } else {
 #pragma unroll
         for (int e = 0; e < NV; ++e) r[e] = (v[k][e] - mean) * rstd;
@@ -237,9 +277,7 @@ __global__ void __launch_bounds__(128) ln_mod_kernel(const T* __restrict__ x,
 template <typename T, int VPT>
 __global__ void __launch_bounds__(128) ln_mod_row_kernel(const T* __restrict__ x,
                                                          const int32_t* __restrict__ rows, int H,
-                                                         T* __restrict__ out,
-                                                         const int32_t* __restrict__ cu, int n_req,
-                                                         const T* __restrict__ mod, int shift_off,
+                                                         T* __restrict__ out, LnMod<T> md,
                                                          const int32_t* __restrict__ out_rows) {
   constexpr int NV = Vec16<T>::N;
   __shared__ float red[4];
@@ -249,12 +287,13 @@ __global__ void __launch_bounds__(128) ln_mod_row_kernel(const T* __restrict__ x
   const int nvec = H / NV;
   const int src_row = rows ? __ldg(rows + row) : row;
   const uint4* xr = reinterpret_cast<const uint4*>(x + (size_t)src_row * H);
+  const bool mod = md.shift != nullptr;
   const uint4* sh = nullptr;
   const uint4* sc = nullptr;
   if (mod) {
-    const T* base = mod + (size_t)find_req(cu, n_req, row) * 6 * H + shift_off;
-    sh = reinterpret_cast<const uint4*>(base);
-    sc = reinterpret_cast<const uint4*>(base + H);
+    const size_t off = md.stride ? (size_t)find_req(md.cu, md.n_req, row) * md.stride : 0;
+    sh = reinterpret_cast<const uint4*>(md.shift + off);
+    sc = reinterpret_cast<const uint4*>(md.scale + off);
   }
   uint4 xv[VPT], shv[VPT], scv[VPT];
 #pragma unroll
@@ -302,7 +341,7 @@ __global__ void __launch_bounds__(128) ln_mod_row_kernel(const T* __restrict__ x
       Vec16<T>::unpack(shv[k], a);
       Vec16<T>::unpack(scv[k], b);
 #pragma unroll
-      for (int e = 0; e < NV; ++e) r[e] = (v[k][e] - mean) * rstd * (1.0f + b[e]) + a[e];
+      for (int e = 0; e < NV; ++e) r[e] = (v[k][e] - mean) * rstd * (md.one + b[e]) + a[e];
       o[vi] = Vec16<T>::pack(r);
     }
   }
@@ -310,26 +349,24 @@ __global__ void __launch_bounds__(128) ln_mod_row_kernel(const T* __restrict__ x
 
 template <typename T>
 static fps_status ln_mod_t(const void* x, const int32_t* rows, int n, int H, void* out,
-                           const int32_t* cu, int n_req, const void* mod, int shift_off,
-                           cudaStream_t s, const int32_t* out_rows) {
+                           LnMod<T> Md, cudaStream_t s, const int32_t* out_rows) {
   constexpr int NV = Vec16<T>::N;
   const int per_lane = ceil_div(H / NV, 32);
   const int grid = ceil_div(n, 4);
   auto X = reinterpret_cast<const T*>(x);
   auto O = reinterpret_cast<T*>(out);
-  auto Md = reinterpret_cast<const T*>(mod);
+  if (!Md.shift) Md.one = 1.0f;
   const int per_thread = ceil_div(H / NV, 128);
   if (H / NV >= 128 && per_thread <= 8) {
     prof::begin(s);
     cudaError_t le;
 #define FPS_LNR_CASE(VPT)                                                                  \
     if (per_thread <= VPT)                                                                 \
-      le = launch_k(ln_mod_row_kernel<T, VPT>, dim3(n), dim3(128), 0, s, X, rows, H, O, cu, \
-                    n_req, Md, shift_off, out_rows);                                       \
+      le = launch_k(ln_mod_row_kernel<T, VPT>, dim3(n), dim3(128), 0, s, X, rows, H, O, Md, \
+                    out_rows);                                                             \
     else
     FPS_LNR_CASE(1) FPS_LNR_CASE(2) FPS_LNR_CASE(3) FPS_LNR_CASE(4) FPS_LNR_CASE(6)
-    le = launch_k(ln_mod_row_kernel<T, 8>, dim3(n), dim3(128), 0, s, X, rows, H, O, cu, n_req,
-                  Md, shift_off, out_rows);
+    le = launch_k(ln_mod_row_kernel<T, 8>, dim3(n), dim3(128), 0, s, X, rows, H, O, Md, out_rows);
 #undef FPS_LNR_CASE
     FPS_CUDA_TRY(le);
     prof::end(s, prof::LN, 0, 2.0 * n * H * sizeof(T));
@@ -340,7 +377,7 @@ static fps_status ln_mod_t(const void* x, const int32_t* rows, int n, int H, voi
 #define FPS_LN_CASE(VPT)                                                                  \
   if (per_lane <= VPT) {                                                                  \
     prof::begin(s);                                                                       \
-    ln_mod_kernel<T, VPT><<<grid, 128, 0, s>>>(X, rows, n, H, O, cu, n_req, Md, shift_off, out_rows); \
+    ln_mod_kernel<T, VPT><<<grid, 128, 0, s>>>(X, rows, n, H, O, Md, out_rows);           \
     prof::end(s, prof::LN, 0, 2.0 * n * H * sizeof(T));                                   \
     count_launch();                                                                       \
     FPS_LAUNCH_CHECK();                                                                   \
@@ -356,13 +393,114 @@ static fps_status ln_mod_t(const void* x, const int32_t* rows, int n, int H, voi
   return fail(FPS_EUNSUPPORTED, "ln_mod: H=%d too large", H);
 }
 
+// SDXL block norms over the fp32 residual stream (R24): one 128-thread CTA per row, fp32 input
+// (VPT float4 per thread), bf16 output LN(x) * gamma + beta.
+template <int VPT>
+__global__ void __launch_bounds__(128) ln_affine_f32_kernel(const float* __restrict__ x, int H,
+                                                            __nv_bfloat16* __restrict__ out,
+                                                            const __nv_bfloat16* __restrict__ gamma,
+                                                            const __nv_bfloat16* __restrict__ beta) {
+  __shared__ float red[4];
+  pdl_trigger();
+  pdl_wait();
+  const int row = blockIdx.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int nvec = H / 4;
+  const float4* xr = reinterpret_cast<const float4*>(x + (size_t)row * H);
+  float4 v[VPT];
+  float sum = 0.f;
+#pragma unroll
+  for (int k = 0; k < VPT; ++k) {
+    const int vi = tid + 128 * k;
+    v[k] = vi < nvec ? __ldg(xr + vi) : make_float4(0.f, 0.f, 0.f, 0.f);
+    sum += (v[k].x + v[k].y) + (v[k].z + v[k].w);
+  }
+  sum = warp_sum(sum);
+  if (lane == 0) red[warp] = sum;
+  __syncthreads();
+  const float mean = (red[0] + red[1] + red[2] + red[3]) / (float)H;
+  __syncthreads();
+  float sq = 0.f;
+#pragma unroll
+  for (int k = 0; k < VPT; ++k)
+    if (tid + 128 * k < nvec) {
+      const float a = v[k].x - mean, b = v[k].y - mean, c = v[k].z - mean, d = v[k].w - mean;
+      sq += (a * a + b * b) + (c * c + d * d);
+    }
+  sq = warp_sum(sq);
+  if (lane == 0) red[warp] = sq;
+  __syncthreads();
+  const float rstd = 1.0f / sqrtf((red[0] + red[1] + red[2] + red[3]) / (float)H + 1e-6f);
+  uint2* o = reinterpret_cast<uint2*>(out + (size_t)row * H);
+  const uint2* gp = reinterpret_cast<const uint2*>(gamma);
+  const uint2* bp = reinterpret_cast<const uint2*>(beta);
+#pragma unroll
+  for (int k = 0; k < VPT; ++k) {
+    const int vi = tid + 128 * k;
+    if (vi < nvec) {
+      const uint2 gv = __ldg(gp + vi), bv = __ldg(bp + vi);
+      float g0, g1, g2, g3, b0, b1, b2, b3;
+      unpack_bf16x2(gv.x, g0, g1); unpack_bf16x2(gv.y, g2, g3);
+      unpack_bf16x2(bv.x, b0, b1); unpack_bf16x2(bv.y, b2, b3);
+      o[vi] = make_uint2(pack_bf16x2((v[k].x - mean) * rstd * g0 + b0, (v[k].y - mean) * rstd * g1 + b1),
+                         pack_bf16x2((v[k].z - mean) * rstd * g2 + b2, (v[k].w - mean) * rstd * g3 + b3));
+    }
+  }
+}
+
+fps_status launch_ln_affine_f32in(const float* x, int n, int H, void* out, const void* gamma,
+                                  const void* beta, cudaStream_t s) {
+  if (n <= 0) return FPS_OK;
+  if (H % 4) return fail(FPS_EUNSUPPORTED, "ln_affine_f32: H=%d not a multiple of 4", H);
+  const int per = ceil_div(H / 4, 128);
+  auto G = reinterpret_cast<const __nv_bfloat16*>(gamma);
+  auto Bt = reinterpret_cast<const __nv_bfloat16*>(beta);
+  auto O = reinterpret_cast<__nv_bfloat16*>(out);
+  prof::begin(s);
+  cudaError_t le;
+  if (per <= 2) le = launch_k(ln_affine_f32_kernel<2>, dim3(n), dim3(128), 0, s, x, H, O, G, Bt);
+  else if (per <= 4) le = launch_k(ln_affine_f32_kernel<4>, dim3(n), dim3(128), 0, s, x, H, O, G, Bt);
+  else if (per <= 8) le = launch_k(ln_affine_f32_kernel<8>, dim3(n), dim3(128), 0, s, x, H, O, G, Bt);
+  else if (per <= 16) le = launch_k(ln_affine_f32_kernel<16>, dim3(n), dim3(128), 0, s, x, H, O, G, Bt);
+  else return fail(FPS_EUNSUPPORTED, "ln_affine_f32: H=%d too large", H);
+  FPS_CUDA_TRY(le);
+  prof::end(s, prof::LN, 0, 6.0 * n * H);
+  count_launch();
+  FPS_LAUNCH_CHECK();
+  return FPS_OK;
+}
+
+template <typename T>
+static LnMod<T> ln_params(const void* shift, const void* scale, int stride, float one,
+                          const int32_t* cu, int n_req) {
+  return LnMod<T>{reinterpret_cast<const T*>(shift), reinterpret_cast<const T*>(scale), stride, one,
+                  cu, n_req};
+}
+
 fps_status launch_ln_mod(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
                          const int32_t* cu, int n_req, const void* mod, int shift_off,
                          cudaStream_t s, const int32_t* out_rows) {
   if (n <= 0) return FPS_OK;
+  const size_t e = dtype == FPS_BF16 ? 2 : 4;
+  const char* sh = mod ? (const char*)mod + (size_t)shift_off * e : nullptr;
+  const char* sc = mod ? sh + (size_t)H * e : nullptr;
   if (dtype == FPS_BF16)
-    return ln_mod_t<__nv_bfloat16>(x, rows, n, H, out, cu, n_req, mod, shift_off, s, out_rows);
-  return ln_mod_t<float>(x, rows, n, H, out, cu, n_req, mod, shift_off, s, out_rows);
+    return ln_mod_t<__nv_bfloat16>(x, rows, n, H, out,
+                                   ln_params<__nv_bfloat16>(sh, sc, 6 * H, 1.0f, cu, n_req), s,
+                                   out_rows);
+  return ln_mod_t<float>(x, rows, n, H, out, ln_params<float>(sh, sc, 6 * H, 1.0f, cu, n_req), s,
+                         out_rows);
+}
+
+fps_status launch_ln_affine(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
+                            const void* gamma, const void* beta, cudaStream_t s,
+                            const int32_t* out_rows) {
+  if (n <= 0) return FPS_OK;
+  if (dtype == FPS_BF16)
+    return ln_mod_t<__nv_bfloat16>(x, rows, n, H, out,
+                                   ln_params<__nv_bfloat16>(beta, gamma, 0, 0.0f, nullptr, 0), s,
+                                   out_rows);
+  return ln_mod_t<float>(x, rows, n, H, out, ln_params<float>(beta, gamma, 0, 0.0f, nullptr, 0), s,
+                         out_rows);
 }
 
 // ---------------------------------------------------------------------------------------

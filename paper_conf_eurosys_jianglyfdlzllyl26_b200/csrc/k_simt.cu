@@ -53,6 +53,8 @@ __global__ void __launch_bounds__(256) gemm_simt_kernel(const T* __restrict__ A,
 fps_status launch_gemm_simt(int dtype, const void* A, const void* B, int M, int N, int K,
                             const Epilogue& ep, cudaStream_t s) {
   if (M <= 0) return FPS_OK;
+  if (ep.act == 2 || ep.out0_f32 || ep.resid_f32)
+    return fail(FPS_EUNSUPPORTED, "gemm_simt: GEGLU / fp32-residual epilogues are tcgen05-only");
   if (N % 4 != 0 || ep.split % 4 != 0 || ep.split2 % 4 != 0 || ep.act_from % 4 != 0)
     return fail(FPS_EUNSUPPORTED, "gemm_simt: N=%d and the epilogue splits must be multiples of 4", N);
   dim3 grid(ceil_div(N, SBN), ceil_div(M, SBM));

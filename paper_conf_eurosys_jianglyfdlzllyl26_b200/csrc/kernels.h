@@ -19,6 +19,17 @@ fps_status launch_copy_rows(const void* src, const int32_t* src_ids, const int32
 fps_status launch_ln_mod(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
                          const int32_t* cu, int n_req, const void* mod, int shift_off,
                          cudaStream_t s, const int32_t* out_rows = nullptr);
+// a4 (SDXL block, R24): out[out_rows ? out_rows[i] : i] = LN(x[rows ? rows[i] : i]) * gamma + beta
+fps_status launch_ln_affine(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
+                            const void* gamma, const void* beta, cudaStream_t s,
+                            const int32_t* out_rows = nullptr);
+// same over an fp32 residual stream: x [n, H] fp32 -> out [n, H] bf16
+fps_status launch_ln_affine_f32in(const float* x, int n, int H, void* out, const void* gamma,
+                                  const void* beta, cudaStream_t s);
+// GEGLU weight packing: rows of w [2F, K] (value half, then gate half) -> 32-row interleave
+// (value rows 32j.., gate rows 32j..) so one 64-column GEMM chunk holds a (value, gate) pair
+fps_status launch_geglu_pack(int dtype, const void* w, const void* b, int F, int K, void* w_out,
+                             void* b_out, cudaStream_t s);
 // x[i] += delta[req(i)] * y[i] over rows of width H (req via cu over rows)
 fps_status launch_euler(int dtype, void* x, const void* y, int n, int H, const int32_t* cu,
                         int n_req, const float* delta, cudaStream_t s);

@@ -17,14 +17,17 @@ import numpy as np
 from . import FPS_MODE_KV, FPS_MODE_Y, plan_pipeline
 
 
-def block_flops(mode, n, L, H, F):
-    """Exact FLOPs of one block for one request with n active of L rows (Table 1, per mode)."""
+def block_flops(mode, n, L, H, F, kind="seq", Lc=0):
+    """Exact FLOPs of one block for one request with n active of L rows (Table 1, per mode);
+    the SDXL block (R24) adds cross-attention (4H^2 + 4 Lc H) and the GEGLU's 2HF per row."""
+    rows = L if mode == "dense" else n
+    extra = rows * (4.0 * H * H + 4.0 * Lc * H + 2.0 * H * F) if kind == "sdxl" else 0.0
     if mode == "dense":
-        return 8.0 * L * H * H + 4.0 * L * H * F + 4.0 * L * L * H
+        return 8.0 * L * H * H + 4.0 * L * H * F + 4.0 * L * L * H + extra
     attn = 4.0 * n * L * H
     if mode == "kv":
-        return 8.0 * n * H * H + 4.0 * n * H * F + attn
-    return 4.0 * n * H * H + 4.0 * L * H * H + 4.0 * n * H * F + attn
+        return 8.0 * n * H * H + 4.0 * n * H * F + attn + extra
+    return 4.0 * n * H * H + 4.0 * L * H * H + 4.0 * n * H * F + attn + extra
 
 
 def cache_bytes(mode, u, H, elt=2):
@@ -57,8 +60,9 @@ class CostModel:
     """Per-block costs of a batch for Alg. 1 from the two fitted linear models."""
 
     def __init__(self, n_layers, H, F, mode, comp=(1e-12, 0.01), load=(2e-8, 0.01), elt=2,
-                 full_entry_rows=None):
+                 full_entry_rows=None, kind="seq", Lc=0):
         self.n_layers, self.H, self.F, self.mode, self.elt = n_layers, H, F, mode, elt
+        self.kind, self.Lc = kind, Lc
         self.comp, self.load = comp, load
         # whole-entry DMA loads (copy_method 2) move L_img rows whatever the mask
         self.full_entry_rows = full_entry_rows
@@ -69,8 +73,8 @@ class CostModel:
     def costs(self, batch):
         a, b = self.comp
         c, e = self.load
-        fm = sum(block_flops(self.mode, r.n, r.L, self.H, self.F) for r in batch)
-        fd = sum(block_flops("dense", r.n, r.L, self.H, self.F) for r in batch)
+        fm = sum(block_flops(self.mode, r.n, r.L, self.H, self.F, self.kind, self.Lc) for r in batch)
+        fd = sum(block_flops("dense", r.n, r.L, self.H, self.F, self.kind, self.Lc) for r in batch)
         by = sum(cache_bytes(self.mode, self._rows(r), self.H, self.elt) for r in batch)
         byf = sum(cache_bytes("y", self._rows(r), self.H, self.elt) for r in batch)
         N = self.n_layers

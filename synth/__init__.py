@@ -25,7 +25,7 @@ import numpy as np
 
 __all__ = [
     "rng", "bf16_round", "BlockDims", "CONFIGS", "block_weights", "stack_weights", "mod_table",
-    "delta_table", "latent", "mask_random", "mask_blobs", "token_mask", "n_masked_for",
+    "delta_table", "latent", "context", "mask_random", "mask_blobs", "token_mask", "n_masked_for",
     "sample_mask_ratios",
 ]
 
@@ -90,11 +90,34 @@ CONFIGS = {
 
 
 def block_weights(g: np.random.Generator, H: int, F: int, dtype: str = "bf16",
-                  kind: str = "seq") -> dict:
+                  kind: str = "seq", D_ctx: int = 2048) -> dict:
     """nn.Linear layout: W[out, in]. Q/K/V stacked as rows [0,H), [H,2H), [2H,3H) of w_qkv.
 
     kind="par" (parallel block, NEXT-2): w_1 [3H+F, H] stacks Q, K, V and the MLP input rows;
-    w_2 [H, H+F] maps the concatenation [attention | GELU(MLP)] back to H."""
+    w_2 [H, H+F] maps the concatenation [attention | GELU(MLP)] back to H.
+
+    kind="sdxl" (SDXL UNet transformer block, NEXT-2): bias-free Q/K/V projections (w_qkv, and
+    w_q2 / w_kv2 [2H, D_ctx] for the cross-attention, K rows then V rows), biased output
+    projections w_o / w_o2, GEGLU input w_up [2F, H] (first F rows the value half, last F the
+    gate half), w_down [H, F], and three affine LayerNorms ln{1,2,3}_w ~ 1 + N(0, 0.02^2),
+    ln{1,2,3}_b ~ N(0, 0.02^2)."""
+    if kind == "sdxl":
+        n = lambda *shape: g.standard_normal(shape, dtype=np.float32)
+        w = {
+            "w_qkv": n(3 * H, H) / math.sqrt(H),
+            "w_o": n(H, H) / math.sqrt(H), "b_o": 0.02 * n(H),
+            "w_q2": n(H, H) / math.sqrt(H),
+            "w_kv2": n(2 * H, D_ctx) / math.sqrt(D_ctx),
+            "w_o2": n(H, H) / math.sqrt(H), "b_o2": 0.02 * n(H),
+            "w_up": n(2 * F, H) / math.sqrt(H), "b_up": 0.02 * n(2 * F),
+            "w_down": n(H, F) / math.sqrt(F), "b_down": 0.02 * n(H),
+        }
+        for i in (1, 2, 3):
+            w[f"ln{i}_w"] = 1.0 + 0.02 * n(H)
+            w[f"ln{i}_b"] = 0.02 * n(H)
+        out = {k: _store(v, dtype) for k, v in w.items()}
+        out["kind"] = "sdxl"
+        return out
     if kind == "par":
         w = {
             "w_1": g.standard_normal((3 * H + F, H), dtype=np.float32) / math.sqrt(H),
@@ -119,8 +142,15 @@ def block_weights(g: np.random.Generator, H: int, F: int, dtype: str = "bf16",
 
 
 def stack_weights(g: np.random.Generator, layers: int, H: int, F: int, dtype: str = "bf16",
-                  kind: str = "seq"):
-    return [block_weights(g, H, F, dtype, kind) for _ in range(layers)]
+                  kind: str = "seq", D_ctx: int = 2048):
+    return [block_weights(g, H, F, dtype, kind, D_ctx) for _ in range(layers)]
+
+
+def context(g: np.random.Generator, L_ctx: int = 77, D_ctx: int = 2048,
+            dtype: str = "bf16") -> np.ndarray:
+    """A request's prompt encoding for the SDXL cross-attention (77 tokens x 2048 channels in
+    SDXL), ~ N(0, 1)."""
+    return _store(g.standard_normal((L_ctx, D_ctx), dtype=np.float32), dtype)
 
 
 def mod_table(g: np.random.Generator, layers: int, steps: int, H: int, dtype: str = "bf16",

@@ -240,3 +240,110 @@ def test_parallel_cache_is_actually_used():
     y_kv, _, _ = B.masked_block_kv(x[M], M, U, Kt[U], Vt[U], w, m, 3, 64)
     y_ref, _, _ = B.dense_block(x, w, m, 3)
     assert not np.allclose(y_kv, y_ref[M], atol=1e-3)
+
+
+# ---- NEXT-2: SDXL UNet transformer block (self-attn + cross-attn + GEGLU), reading R24 -----
+def _setup_sdxl(seed=0, H=48, heads=3, F=80, L=40, L_ctx=7, D_ctx=24, dtype="f32"):
+    g = synth.rng(seed)
+    w = synth.block_weights(g, H, F, dtype, kind="sdxl", D_ctx=D_ctx)
+    x = synth.latent(g, L, H, dtype)
+    ctx = synth.context(g, L_ctx, D_ctx, dtype)
+    return g, w, x, ctx
+
+
+def _torch_sdxl_block(x, w, ctx, heads):
+    """The SDXL block assembled from torch library modules in float64, as diffusers'
+    BasicTransformerBlock is: nn.LayerNorm (affine), nn.MultiheadAttention for self-attention
+    (bias-free in-projection, biased out-projection) and for cross-attention (kdim = vdim =
+    D_ctx, separate q/k/v projection weights), and GEGLU as Linear -> chunk(2) -> value *
+    gelu(gate) -> Linear."""
+    t = lambda a: torch.tensor(np.asarray(a, np.float64))
+    H, D = x.shape[1], ctx.shape[1]
+    F = w["w_up"].shape[0] // 2
+    lns = [torch.nn.LayerNorm(H, eps=1e-6) for _ in range(3)]
+    sa = torch.nn.MultiheadAttention(H, heads, bias=True, batch_first=True)
+    ca = torch.nn.MultiheadAttention(H, heads, bias=True, batch_first=True, kdim=D, vdim=D)
+    up, dn = torch.nn.Linear(H, 2 * F), torch.nn.Linear(F, H)
+    with torch.no_grad():
+        for i, ln in enumerate(lns, 1):
+            ln.weight.copy_(t(w[f"ln{i}_w"])); ln.bias.copy_(t(w[f"ln{i}_b"]))
+        sa.in_proj_weight.copy_(t(w["w_qkv"])); sa.in_proj_bias.zero_()
+        sa.out_proj.weight.copy_(t(w["w_o"])); sa.out_proj.bias.copy_(t(w["b_o"]))
+        ca.q_proj_weight.copy_(t(w["w_q2"]))
+        ca.k_proj_weight.copy_(t(w["w_kv2"][:H])); ca.v_proj_weight.copy_(t(w["w_kv2"][H:]))
+        ca.in_proj_bias.zero_()
+        ca.out_proj.weight.copy_(t(w["w_o2"])); ca.out_proj.bias.copy_(t(w["b_o2"]))
+        up.weight.copy_(t(w["w_up"])); up.bias.copy_(t(w["b_up"]))
+        dn.weight.copy_(t(w["w_down"])); dn.bias.copy_(t(w["b_down"]))
+        xt, ct = t(x)[None], t(ctx)[None]
+        h = lns[0](xt)
+        x1 = xt + sa(h, h, h, need_weights=False)[0]
+        h = lns[1](x1)
+        x2 = x1 + ca(h, ct, ct, need_weights=False)[0]
+        v, gate = up(lns[2](x2)).chunk(2, dim=-1)
+        y = x2 + dn(v * Fn.gelu(gate, approximate="tanh"))
+    return y[0].numpy()
+
+
+def test_sdxl_block_vs_torch_modules():
+    _, w, x, ctx = _setup_sdxl()
+    y, K, V = B.dense_block(x, w, None, 3, ctx)
+    assert np.allclose(y, _torch_sdxl_block(x, w, ctx, 3), rtol=0, atol=1e-10)
+    H = x.shape[1]
+    h = Fn.layer_norm(torch.tensor(np.asarray(x, np.float64)), (H,),
+                      weight=torch.tensor(np.asarray(w["ln1_w"], np.float64)),
+                      bias=torch.tensor(np.asarray(w["ln1_b"], np.float64)), eps=1e-6).numpy()
+    assert np.allclose(K, h @ np.asarray(w["w_qkv"], np.float64)[H:2 * H].T, atol=1e-12)
+
+
+def test_sdxl_single_context_token_closed_form():
+    """L_ctx = 1: the cross-attention softmax is 1 for every query, so its output is the one
+    context value row ctx Wv2^T for every latent row; with W_o2 = I the block's x2 - x1 equals
+    that row (checked through y with a zero feed-forward)."""
+    _, w, x, ctx = _setup_sdxl(seed=31, L_ctx=1)
+    H = x.shape[1]
+    w["w_o2"], w["b_o2"] = np.eye(H, dtype=np.float32), np.zeros(H, np.float32)
+    w["w_down"], w["b_down"] = np.zeros_like(w["w_down"]), np.zeros_like(w["b_down"])
+    y, _, _ = B.dense_block(x, w, None, 3, ctx)
+    w0 = dict(w); w0["w_kv2"] = np.zeros_like(w["w_kv2"])   # same block, zero context values
+    y0, _, _ = B.dense_block(x, w0, None, 3, ctx)
+    v_row = np.asarray(ctx, np.float64) @ np.asarray(w["w_kv2"], np.float64)[H:].T
+    assert np.allclose(y - y0, np.broadcast_to(v_row, y.shape), atol=1e-12)
+
+
+def test_sdxl_geglu_halves_closed_form():
+    """GEGLU chunk order: gate weights 0 and gate bias c give P * GELU(c) with P the FIRST F
+    output rows; swapping the halves would give GELU(P) * ... instead."""
+    g = synth.rng(33)
+    h = g.standard_normal((5, 8))
+    W = g.standard_normal((12, 8)); W[6:] = 0.0
+    b = np.zeros(12); b[6:] = 3.0
+    gelu3 = 0.5 * 3.0 * (1 + math.tanh(math.sqrt(2 / math.pi) * (3.0 + 0.044715 * 27.0)))
+    assert np.allclose(B.geglu(h, W, b), (h @ W[:6].T) * gelu3, atol=1e-12)
+
+
+@pytest.mark.parametrize("ratio", [0.0, 0.3, 1.0])
+def test_sdxl_masked_equals_dense_under_identical_input_cache(ratio):
+    g, w, x, ctx = _setup_sdxl(seed=35, L=64)
+    mask = synth.mask_blobs(g, 8, 8, ratio)
+    M, U = build_mask_index(mask)
+    y_ref, K, V = B.dense_block(x, w, None, 3, ctx)
+    y_kv, K_M, V_M = B.masked_block_kv(x[M], M, U, K[U], V[U], w, None, 3, 64, ctx)
+    y_y = B.masked_block_y(x[M], M, U, x[U], w, None, 3, 64, ctx)
+    assert np.allclose(y_kv, y_ref[M], rtol=0, atol=1e-12)
+    assert np.allclose(y_y, y_ref[M], rtol=0, atol=1e-12)
+    assert np.allclose(K_M, K[M], atol=1e-12) and np.allclose(V_M, V[M], atol=1e-12)
+
+
+def test_sdxl_context_and_cache_are_used():
+    g, w, x, ctx = _setup_sdxl(seed=37, L=64)
+    mask = synth.mask_random(g, 64, 0.25)
+    M, U = build_mask_index(mask)
+    x_t = synth.latent(g, 64, x.shape[1], "f32")
+    _, Kt, Vt = B.dense_block(x_t, w, None, 3, ctx)
+    y_kv, _, _ = B.masked_block_kv(x[M], M, U, Kt[U], Vt[U], w, None, 3, 64, ctx)
+    y_ref, _, _ = B.dense_block(x, w, None, 3, ctx)
+    assert not np.allclose(y_kv, y_ref[M], atol=1e-3)
+    ctx2 = ctx.copy(); ctx2[0, 0] += 1.0
+    y2, _, _ = B.masked_block_kv(x[M], M, U, Kt[U], Vt[U], w, None, 3, 64, ctx2)
+    assert not np.allclose(y2, y_kv, atol=1e-6)

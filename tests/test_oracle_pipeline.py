@@ -127,3 +127,36 @@ def test_flops_match_matmul_shapes():
         assert count["f"] == C.block_flops("y", len(M), L, H, F)
     finally:
         B.linear, B.attention = orig
+
+
+def test_sdxl_flops_match_matmul_shapes():
+    """The SDXL block's counts (R24) against the matmuls oracle/block.py performs."""
+    from oracle import block as B
+    g = synth.rng(5)
+    H, heads, F, L, Lc, D = 16, 2, 32, 24, 5, 12
+    w = synth.block_weights(g, H, F, "f32", "sdxl", D_ctx=D)
+    x = synth.latent(g, L, H, "f32")
+    ctx = synth.context(g, Lc, D, "f32")
+    M = np.arange(0, L, 3); U = np.setdiff1d(np.arange(L), M)
+    count = {"f": 0}
+    orig = B.linear, B.attention
+
+    def lin(h, W, b):
+        count["f"] += 2 * h.shape[0] * W.shape[0] * W.shape[1]
+        return orig[0](h, W, b)
+
+    def att(Q, K, V, heads_):
+        count["f"] += 2 * Q.shape[0] * K.shape[0] * Q.shape[1] * 2
+        return orig[1](Q, K, V, heads_)
+
+    B.linear, B.attention = lin, att
+    cf = C.context_flops(Lc, D, H)
+    try:
+        B.dense_block(x, w, None, heads, ctx)
+        assert count["f"] == C.block_flops("dense", L, L, H, F, "sdxl", Lc) + cf; count["f"] = 0
+        B.masked_block_kv(x[M], M, U, x[U], x[U], w, None, heads, L, ctx)
+        assert count["f"] == C.block_flops("kv", len(M), L, H, F, "sdxl", Lc) + cf; count["f"] = 0
+        B.masked_block_y(x[M], M, U, x[U], w, None, heads, L, ctx)
+        assert count["f"] == C.block_flops("y", len(M), L, H, F, "sdxl", Lc) + cf
+    finally:
+        B.linear, B.attention = orig
