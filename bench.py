@@ -48,6 +48,7 @@ WORKLOADS = {
 }
 SEED = 1003
 SDXL_CTX = (77, 2048)          # SDXL prompt encoding: 77 tokens x 2048 channels (R24)
+FLUX_DOUBLE = 19               # Flux: 19 double-stream blocks, then 38 single-stream (R19, R25)
 
 
 def log(*a):
@@ -155,11 +156,19 @@ def build_engine_inputs(F, w, mode, device, n_entries, location=0, copy_method=0
         return (torch.randn(*shape, generator=gen, device=device) * scale).to(torch.bfloat16)
 
     layers = []
-    par = w.get("block") == "par"
-    sdxl = w.get("block") == "sdxl"
     D = SDXL_CTX[1]
-    for _ in range(N):
-        if sdxl:     # SDXL UNet transformer block (R24): self-attn, cross-attn, GEGLU
+    flux = w.get("block") == "flux"
+    for li in range(N):
+        kind = (("double" if li < FLUX_DOUBLE else "par") if flux else w.get("block", "seq"))
+        par, sdxl = kind == "par", kind == "sdxl"
+        if kind == "double":  # Flux double-stream block: a sequential set per stream (R25)
+            t = {}
+            for pre, bpre in (("w_", "b_"), ("t_", "tb_")):
+                t.update({pre + "qkv": rnd(3 * H, H, scale=H ** -0.5), bpre + "qkv": rnd(3 * H, scale=0.02),
+                          pre + "o": rnd(H, H, scale=H ** -0.5), bpre + "o": rnd(H, scale=0.02),
+                          pre + "up": rnd(Fd, H, scale=H ** -0.5), bpre + "up": rnd(Fd, scale=0.02),
+                          pre + "down": rnd(H, Fd, scale=Fd ** -0.5), bpre + "down": rnd(H, scale=0.02)})
+        elif sdxl:     # SDXL UNet transformer block (R24): self-attn, cross-attn, GEGLU
             t = {"w_qkv": rnd(3 * H, H, scale=H ** -0.5),
                  "w_o": rnd(H, H, scale=H ** -0.5), "b_o": rnd(H, scale=0.02),
                  "w_up": rnd(2 * Fd, H, scale=H ** -0.5), "b_up": rnd(2 * Fd, scale=0.02),
@@ -184,19 +193,20 @@ def build_engine_inputs(F, w, mode, device, n_entries, location=0, copy_method=0
         layers.append(F.BlockWeights.__new__(F.BlockWeights))
         bw = layers[-1]
         bw.t, bw.H, bw.F, bw.heads, bw.dtype = t, H, Fd, w["heads"], F.FPS_BF16
-        bw.kind = F.FPS_BLOCK_SDXL if sdxl else F.FPS_BLOCK_PAR if par else F.FPS_BLOCK_SEQ
+        bw.kind = F._KIND[kind]
         bw.D_ctx = D if sdxl else 0
         ptrs = lambda keys: [t[k].data_ptr() if k in t else None for k in keys]
         bw.c = F.fps_block_weights(H, w["heads"], H // w["heads"], Fd, F.FPS_BF16,
-                                   *ptrs(("w_qkv", "b_qkv", "w_o", "b_o", "w_up", "b_up",
-                                          "w_down", "b_down")), bw.kind, bw.D_ctx,
-                                   *ptrs(F._SDXL_KEYS))
-    mod = torch.zeros(N, w["steps"], 6, H, device=device)
-    mod += 0.02 * torch.randn(N, w["steps"], 6, H, generator=gen, device=device)
-    mod[:, :, 2] += 1.0
-    mod[:, :, 5] += 1.0
-    mod = mod.reshape(N, w["steps"], 6 * H).to(torch.bfloat16)
-    if sdxl:
+                                   *ptrs(F._SEQ_KEYS), bw.kind, bw.D_ctx, *ptrs(F._SDXL_KEYS),
+                                   *ptrs(("t_qkv", "tb_qkv", "t_o", "tb_o", "t_up", "tb_up",
+                                          "t_down", "tb_down")))
+    ns = 2 if flux else 1              # double-stream blocks: image 6H then text 6H per row
+    mod = torch.zeros(N, w["steps"], ns, 6, H, device=device)
+    mod += 0.02 * torch.randn(N, w["steps"], ns, 6, H, generator=gen, device=device)
+    mod[:, :, :, 2] += 1.0
+    mod[:, :, :, 5] += 1.0
+    mod = mod.reshape(N, w["steps"], ns * 6 * H).to(torch.bfloat16)
+    if w.get("block") == "sdxl":
         mod = None                    # SDXL blocks are not adaLN-modulated (R24)
     cache = make_cache(F, w, mode, n_entries, location, copy_method)
     return layers, mod, cache
@@ -221,14 +231,16 @@ def calibrate(F, w, mode, layers, cache, reqs, device):
                                     ld_dst[i * L].data_ptr(), Wl * 2) for i in range(B)]
     ld_stream = torch.cuda.Stream(device=device)
     kind = w.get("block", "seq")
+    kind = "double" if kind == "flux" else kind         # FLOPs per row: double == seq
     Lc = SDXL_CTX[0] if kind == "sdxl" else 0
     ctx_kv = (torch.randn(B * Lc, 2 * H, device=device).to(torch.bfloat16) if Lc else None)
     for m in (0.05, 0.2, 0.4, 0.7, 1.0):
         n_img = synth.n_masked_for(m, w["L_img"])
         n = n_img + w["L_txt"]
         q_row = torch.cat([torch.arange(n, device=device, dtype=torch.int32) + i * L for i in range(B)])
+        ids = np.concatenate([np.arange(n_img), np.arange(w["L_img"], L)])
         b = F.VarlenBatch([n] * B, [L] * B, q_row=q_row, mode=F.FPS_MODE_KV,
-                          ctx_kv=ctx_kv, n_ctx=[Lc] * B)
+                          ctx_kv=ctx_kv, n_ctx=[Lc] * B, act_ids=[ids] * B, L_img=w["L_img"])
         x = torch.randn(B * n, H, device=device).to(torch.bfloat16)
         ws = F.workspace(H, Fd, F.FPS_BF16, B * n, 0, device)
         y = torch.empty_like(x)
@@ -347,18 +359,19 @@ def oracle_block_sample(w, mode, ratio, seed=7):
     H, Fd, L_img, L_txt = w["H"], w["F"], w["L_img"], w["L_txt"]
     L = L_img + L_txt
     kind = w.get("block", "seq")
+    kind = "double" if kind == "flux" else kind
     wt = synth.block_weights(g, H, Fd, "bf16", kind, D_ctx=SDXL_CTX[1])
     ctx = synth.context(g, *SDXL_CTX, "bf16") if kind == "sdxl" else None
     mask = synth.token_mask(synth.mask_blobs(g, *w["grid"], ratio), L_txt)
     M, U = build_mask_index(mask)
     x = synth.latent(g, L, H, "bf16")
     K, V = synth.latent(g, L, H, "bf16"), synth.latent(g, L, H, "bf16")
-    mod = synth.mod_table(g, 1, 1, H, "bf16")[0, 0]
+    mod = synth.mod_table(g, 1, 1, H, "bf16", streams=2 if kind == "double" else 1)[0, 0]
     t0 = time.perf_counter()
     if mode == "kv":
-        OB.masked_block_kv(x[M], M, U, K[U], V[U], wt, mod, w["heads"], L, ctx)
+        OB.masked_block_kv(x[M], M, U, K[U], V[U], wt, mod, w["heads"], L, ctx, L_txt)
     else:
-        OB.masked_block_y(x[M], M, U, x[U], wt, mod, w["heads"], L, ctx)
+        OB.masked_block_y(x[M], M, U, x[U], wt, mod, w["heads"], L, ctx, L_txt)
     return time.perf_counter() - t0
 
 
@@ -382,10 +395,11 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C3", choices=list(WORKLOADS))
     ap.add_argument("--mode", default="kv", choices=["kv", "y"])
-    ap.add_argument("--block", default=None, choices=["seq", "par", "sdxl"],
+    ap.add_argument("--block", default=None, choices=["seq", "par", "sdxl", "flux"],
                     help="block kind: sequential attention -> MLP, the parallel (Flux "
                          "single-stream) block with fused input / output projections, or the SDXL "
-                         "block with cross-attention and GEGLU (NEXT-2); default: sdxl for the "
+                         "block with cross-attention and GEGLU, or Flux's stack of 19 double-stream "
+                         "then 38 single-stream blocks (NEXT-2); default: sdxl for the "
                          "SDXL-scale configs (C2A/C2B), seq otherwise")
     ap.add_argument("--tier", default="host", choices=["host", "hbm", "host_hugepage"],
                     help="template cache in pinned host DRAM (configs[2]) or HBM (NEXT-1)")
@@ -508,6 +522,7 @@ def main():
     g = torch.Generator(device=device).manual_seed(SEED + rank)
     reqs_dev = []
     L_ctx = SDXL_CTX[0] if args.block == "sdxl" else 0
+    MODW = 12 * w["H"] if args.block == "flux" else 0
     for i, p in enumerate(mine):
         reqs_dev.append(dict(template_id=i, step=0, n_steps=w["steps"],
                              mask=torch.as_tensor(p["mask_np"]).to(device),
@@ -521,7 +536,8 @@ def main():
     def engine(policy, mode=args.mode, the_cache=cache):
         return F.Engine(layers, w["heads"], F.MODE_CODE[mode], F.FPS_BF16, w["L_img"], w["L_txt"],
                         max(len(reqs_dev), 1), w["steps"], deltas, the_cache, mod_table=mod,
-                        slots=0, plan_policy=policy, cost_model=cm.as_engine_model(), L_ctx=L_ctx)
+                        slots=0, plan_policy=policy, cost_model=cm.as_engine_model(), L_ctx=L_ctx,
+                        mod_width=MODW)
 
     eng = engine(0)
     log(f"[rank {rank}] timed run")
@@ -552,7 +568,8 @@ def main():
             c_h = make_cache(F, w, args.mode, n_entries, 1, 2)
             eng_h = F.Engine(layers, w["heads"], F.MODE_CODE[args.mode], F.FPS_BF16, w["L_img"],
                              w["L_txt"], max(len(reqs_dev), 1), w["steps"], deltas, c_h,
-                             mod_table=mod, slots=0, plan_policy=3, plan=list(plan), L_ctx=L_ctx)
+                             mod_table=mod, slots=0, plan_policy=3, plan=list(plan), L_ctx=L_ctx,
+                             mod_width=MODW)
             noload_ms, _ = run_engine_timed(F, eng_h, reqs_dev, K, W, stream, load_stream, rank,
                                             world)
             del eng_h
@@ -575,7 +592,7 @@ def main():
             eng_o = F.Engine(layers, w["heads"], F.MODE_CODE[md], F.FPS_BF16, w["L_img"],
                              w["L_txt"], max(len(reqs_dev), 1), w["steps"], deltas, c2,
                              mod_table=mod, slots=0, plan_policy=0,
-                             cost_model=cm2.as_engine_model(), L_ctx=L_ctx)
+                             cost_model=cm2.as_engine_model(), L_ctx=L_ctx, mod_width=MODW)
             o_ms, _ = run_engine_timed(F, eng_o, reqs_dev, K, W, stream, load_stream, rank, world)
             tag = f"{md}_mode_{['host', 'hbm', 'host_hugepage'][loc]}"
             if cmeth != default_cm(loc):

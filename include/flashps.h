@@ -200,8 +200,15 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
  *   w_up / b_up must be in the PACKED layout fps_geglu_pack writes ([2F, H], F % 32 == 0);
  *   the per-request context keys / values Kc | Vc come precomputed in the batch (d_ctx_kv,
  *   written by fps_context_kv); d_mod is ignored.  bf16 only (tcgen05 path; H, F % 64 == 0).
+ *
+ * kind = FPS_BLOCK_DOUBLE (NEXT-2, reading R25): Flux's double-stream (MM-DiT) block.  Image
+ *   rows and text rows keep their own sequential-block weights (image: the fields above; text:
+ *   the t_* fields) and adaLN vectors (the request's modulation vector is [12H]: image 6H, then
+ *   text 6H) and meet in ONE joint attention over all rows.  The batch must describe the
+ *   stream-major order of its active rows (fps_varlen_batch.d_sm_perm etc.); text rows are
+ *   always active (R9), so cached rows U are image rows.
  */
-enum { FPS_BLOCK_SEQ = 0, FPS_BLOCK_PAR = 1, FPS_BLOCK_SDXL = 2 };
+enum { FPS_BLOCK_SEQ = 0, FPS_BLOCK_PAR = 1, FPS_BLOCK_SDXL = 2, FPS_BLOCK_DOUBLE = 3 };
 typedef struct {
   int32_t H, heads, head_dim, F;   /* H = heads*head_dim; F = MLP width                    */
   int32_t dtype;                   /* FPS_BF16 (tcgen05 path) | FPS_F32 (SIMT fp32 path)   */
@@ -216,6 +223,8 @@ typedef struct {
   const void *w_q2, *b_q2;         /* [H, H], [H]   cross-attention query projection       */
   const void *w_kv2, *b_kv2;       /* [2H, D_ctx], [2H]  rows Wk2 then Wv2 (fps_context_kv) */
   const void *w_o2, *b_o2;         /* [H, H], [H]   cross-attention output projection      */
+  /* DOUBLE block only: the text stream's weights, same shapes as w_qkv .. b_down.           */
+  const void *t_qkv, *tb_qkv, *t_o, *tb_o, *t_up, *tb_up, *t_down, *tb_down;
 } fps_block_weights;
 
 /* One varlen launch over a continuous batch (L237): request r owns active rows
@@ -244,6 +253,16 @@ typedef struct {
   const void* d_ctx_kv;
   const int32_t* d_cu_ctx;         /* [n_req+1] device                                      */
   const int32_t* h_cu_ctx;         /* [n_req+1] host mirror                                  */
+  /* Elements between consecutive requests' modulation vectors in d_mod (0 = 6H, or 12H for
+   * a DOUBLE block).                                                                       */
+  int32_t mod_stride;
+  /* DOUBLE blocks only: the stream-major order of the active rows -- every request's image
+   * rows (request-major, ascending), then every request's text rows.                        */
+  int32_t total_q_img;             /* active image rows of the batch                        */
+  const int32_t* d_sm_perm;        /* [total_q] compact (request-major) row of stream row i  */
+  const int32_t* d_sm_kvrow;       /* [total_q] merged-buffer row of stream row i            */
+  const int32_t* d_cu_img;         /* [n_req+1] prefix sums of active image rows            */
+  const int32_t* d_cu_txt;         /* [n_req+1] prefix sums of text rows                    */
 } fps_varlen_batch;
 
 /* SDXL block helpers (R24), run once per weight load / per request prompt, not per step.
@@ -336,6 +355,9 @@ typedef struct {
                                       load = c*bytes + e  -> {a, b, c, e}  (§4.4)     */
   int32_t L_ctx, D_ctx;            /* SDXL blocks: prompt tokens / width of each request's
                                       fps_request.d_ctx (0 if no layer is FPS_BLOCK_SDXL)   */
+  int32_t mod_width;               /* elements per d_mod_table row: 0 = 6H; 12H when any
+                                      layer is FPS_BLOCK_DOUBLE (image 6H, text 6H; other
+                                      blocks read the first 6H)                              */
 } fps_engine_desc;
 
 typedef struct fps_engine* fps_engine_t;

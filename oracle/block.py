@@ -49,6 +49,17 @@ with an affine LayerNorm (gamma, beta) and an ungated residual; `mod` is not use
 Cross-attention and GEGLU are token-wise in the latent (each row's output depends only on that
 row and ctx), so on a masked block they run on rows M only; the self-attention's K/V follow
 KV- or Y-mode exactly as for the sequential block.
+
+Double-stream block variant (NEXT-2, weights["kind"] == "double"; reading R25): Flux's
+MM-DiT block, where image rows [0, L_img) and text rows [L_img, L) keep their own weights
+(w["img"], w["txt"], each a sequential block's set) and adaLN vectors (mod [12H] = image 6H,
+then text 6H) and meet only in one joint attention over all L rows:
+
+    per stream s of the row:  h1 = LN(x)(1 + scale1_s) + shift1_s ;  Q, K, V = h1 W_s^T + b_s
+    A = softmax(Q K^T / sqrt(d)) V over all rows (joint)
+    per stream:  x1 = x + gate1_s (A Wo_s^T + bo_s) ;  y = x1 + gate2_s MLP_s(LN(x1)(1+scale2_s)+shift2_s)
+
+Text rows are always active (R9), so a masked block has fresh text rows and cached image rows U.
 """
 from __future__ import annotations
 
@@ -133,6 +144,46 @@ def is_sdxl(w):
     return w.get("kind", "seq") == "sdxl"
 
 
+def is_double(w):
+    return w.get("kind", "seq") == "double"
+
+
+def _per_stream(f, ids, L_img, mod, H):
+    """Row-wise op of the double-stream block (R25): f(stream weights key, stream mod [6H])
+    evaluated for both streams, each row taking its own stream's result (ids >= L_img: text)."""
+    mod = f64(mod).reshape(-1)
+    img, txt = f("img", mod[:6 * H]), f("txt", mod[6 * H:])
+    return np.where((np.asarray(ids) >= L_img)[:, None], txt, img)
+
+
+def _double_block(x_rows, ids, w, mod, heads, L_img, K_U=None, V_U=None, U=None, x_U=None,
+                  L=None):
+    """Double-stream block on rows `ids` (ascending) of one request.  Dense: ids = all rows.
+    KV-mode: K_U / V_U cached at rows U.  Y-mode: x_U = cached input rows U.  Returns (y, K, V)
+    over the rows `ids`."""
+    x_rows = f64(x_rows)
+    H = x_rows.shape[1]
+    ln1 = lambda xr: (lambda s, m: layer_norm(xr) * (1.0 + split_mod(m, H)[1]) + split_mod(m, H)[0])
+    proj = lambda hr, j: (lambda s, m: linear(hr, *_qkv_weights(w[s], H)[j]))
+    h1 = _per_stream(ln1(x_rows), ids, L_img, mod, H)
+    Q, K, V = (_per_stream(proj(h1, j), ids, L_img, mod, H) for j in range(3))
+    if U is None or len(U) == 0:
+        Kall, Vall = K, V
+    else:
+        L = L if L is not None else len(ids) + len(U)
+        Kall, Vall = np.empty((L, H)), np.empty((L, H))
+        Kall[ids], Vall[ids] = K, V
+        if x_U is None:                                            # KV-mode: cached K/V rows U
+            Kall[U], Vall[U] = f64(K_U), f64(V_U)
+        else:                                                      # Y-mode: project x[U]
+            hU = _per_stream(ln1(f64(x_U)), U, L_img, mod, H)
+            Kall[U] = _per_stream(proj(hU, 1), U, L_img, mod, H)
+            Vall[U] = _per_stream(proj(hU, 2), U, L_img, mod, H)
+    a = attention(Q, Kall, Vall, heads)
+    y = _per_stream(lambda s, m: _attn_out_and_mlp(x_rows, a, w[s], m, H), ids, L_img, mod, H)
+    return y, K, V
+
+
 def geglu(h, W, b):
     """GEGLU feed-forward input (R24): [P | G] = h W^T + b with P the first F output rows of W,
     G the last F; returns P * GELU_tanh(G)."""
@@ -200,11 +251,15 @@ def _attn_out_and_mlp(x_rows, a_rows, w, mod, H):
     return y
 
 
-def dense_block(x, w, mod, heads, ctx=None):
+def dense_block(x, w, mod, heads, ctx=None, L_txt=0):
     """Standard block over all L tokens (Fig. 5-Top). Returns (y, K, V).
-    ctx: the request's prompt encoding [L_ctx, D_ctx] (SDXL block only)."""
+    ctx: the request's prompt encoding [L_ctx, D_ctx] (SDXL block only); L_txt: text rows at
+    the end of x (double-stream block only)."""
     x = f64(x)
     H = x.shape[1]
+    if is_double(w):
+        L = x.shape[0]
+        return _double_block(x, np.arange(L), w, mod, heads, L - L_txt)
     h1 = _norm1(x, w, mod, H)
     (Wq, bq), (Wk, bk), (Wv, bv) = _qkv_weights(w, H)
     Q, K, V = linear(h1, Wq, bq), linear(h1, Wk, bk), linear(h1, Wv, bv)
@@ -212,12 +267,14 @@ def dense_block(x, w, mod, heads, ctx=None):
     return _block_out(x, h1, a, w, mod, H, ctx, heads), K, V
 
 
-def masked_block_kv(x_M, M, U, K_U, V_U, w, mod, heads, L, ctx=None):
+def masked_block_kv(x_M, M, U, K_U, V_U, w, mod, heads, L, ctx=None, L_txt=0):
     """KV-cache mode (Fig. 7): fresh Q/K/V on rows M, cached K/V on rows U.
 
     x_M: [n, H] block input rows M (ascending ids M). K_U, V_U: [u, H] cached keys/values of the
     template run at rows U. Returns (y_M, K_M, V_M).
     """
+    if is_double(w):
+        return _double_block(x_M, M, w, mod, heads, L - L_txt, K_U, V_U, U, L=L)
     x_M = f64(x_M)
     H = x_M.shape[1]
     h1_M = _norm1(x_M, w, mod, H)                              # token-wise (L134, L144)
@@ -232,9 +289,11 @@ def masked_block_kv(x_M, M, U, K_U, V_U, w, mod, heads, L, ctx=None):
     return _block_out(x_M, h1_M, a_M, w, mod, H, ctx, heads), K_M, V_M
 
 
-def masked_block_y(x_M, M, U, x_U, w, mod, heads, L, ctx=None):
+def masked_block_y(x_M, M, U, x_U, w, mod, heads, L, ctx=None, L_txt=0):
     """Y-cache mode (Fig. 5-Bottom): block input rows U are the cached activations Y of
     the previous block (R4); K/V over all L rows; Q, O and MLP on rows M. Returns y_M."""
+    if is_double(w):
+        return _double_block(x_M, M, w, mod, heads, L - L_txt, U=U, x_U=x_U, L=L)[0]
     x_M = f64(x_M)
     H = x_M.shape[1]
     x_full = np.empty((L, H))

@@ -18,11 +18,11 @@ from .block import dense_block, f64, masked_block_kv, masked_block_y
 from .index import build_mask_index, gather_rows, scatter_rows
 
 
-def template_run(x0, weights, mods, deltas, heads, steps, ctx=None):
+def template_run(x0, weights, mods, deltas, heads, steps, ctx=None, L_txt=0):
     """Full (dense) inference of the template: the producer of the activation cache (L130,
     L203). mods[l][s] is block l's adaLN vector at step s.
 
-    ctx: the request's prompt encoding (SDXL blocks only).
+    ctx: the request's prompt encoding (SDXL blocks only); L_txt: text rows (double-stream).
     Returns (cache, xs): cache[s][l] = {"K", "V", "Y"} full-L arrays; xs[s] = latent entering
     step s (xs[steps] = final latent)."""
     x = f64(x0)
@@ -32,7 +32,7 @@ def template_run(x0, weights, mods, deltas, heads, steps, ctx=None):
         cur = x
         entries = []
         for l, w in enumerate(weights):
-            y, K, V = dense_block(cur, w, mods[l][s], heads, ctx)
+            y, K, V = dense_block(cur, w, mods[l][s], heads, ctx, L_txt)
             entries.append({"K": K, "V": V, "Y": y})
             cur = y
         cache.append(entries)
@@ -53,7 +53,7 @@ def check_plan(use_cache, mode):
                 raise ValueError("KV-mode plan must be monotone (0..0 1..1)")
 
 
-def masked_stack(x, mask, weights, mods_s, use_cache, mode, cache_s, heads, ctx=None):
+def masked_stack(x, mask, weights, mods_s, use_cache, mode, cache_s, heads, ctx=None, L_txt=0):
     """One denoising step's block stack for one request (a2-a9).
 
     x: full latent [L, H] entering the step; mask: [L] (text rows set); mods_s[l]: block l's
@@ -71,7 +71,7 @@ def masked_stack(x, mask, weights, mods_s, use_cache, mode, cache_s, heads, ctx=
                 scatter_rows(act, M, full)
                 scatter_rows(gather_rows(cache_s[l - 1]["Y"], U), U, full)
                 cur = full
-            cur, _, _ = dense_block(cur, weights[l], mods_s[l], heads, ctx)   # L211: all tokens
+            cur, _, _ = dense_block(cur, weights[l], mods_s[l], heads, ctx, L_txt)   # L211: all tokens
             rep = "full"
             continue
         if rep == "full":
@@ -82,9 +82,9 @@ def masked_stack(x, mask, weights, mods_s, use_cache, mode, cache_s, heads, ctx=
         if mode == "kv":
             act, _, _ = masked_block_kv(act, M, U, gather_rows(cache_s[l]["K"], U),
                                         gather_rows(cache_s[l]["V"], U), weights[l],
-                                        mods_s[l], heads, L, ctx)
+                                        mods_s[l], heads, L, ctx, L_txt)
         else:
-            act = masked_block_y(act, M, U, x_U, weights[l], mods_s[l], heads, L, ctx)
+            act = masked_block_y(act, M, U, x_U, weights[l], mods_s[l], heads, L, ctx, L_txt)
         rep = "act"
     if rep == "full":
         return cur
@@ -100,11 +100,11 @@ def euler_update(x, y, delta):
 
 
 def masked_run(x0, mask, weights, mods, deltas, use_cache, mode, cache, heads, steps,
-               step0=0, ctx=None):
+               step0=0, ctx=None, L_txt=0):
     """Steps step0..step0+steps-1 of one request against the template cache."""
     x = f64(x0)
     for s in range(step0, step0 + steps):
         mods_s = [mods[l][s] for l in range(len(weights))]
-        y = masked_stack(x, mask, weights, mods_s, use_cache, mode, cache[s], heads, ctx)
+        y = masked_stack(x, mask, weights, mods_s, use_cache, mode, cache[s], heads, ctx, L_txt)
         x = euler_update(x, y, deltas[s])
     return x

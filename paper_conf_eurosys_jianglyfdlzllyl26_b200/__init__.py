@@ -82,7 +82,9 @@ def scatter_rows(src, ids, out, stream=None):
     return out
 
 
-_KIND = {"seq": _lib.FPS_BLOCK_SEQ, "par": _lib.FPS_BLOCK_PAR, "sdxl": _lib.FPS_BLOCK_SDXL}
+_KIND = {"seq": _lib.FPS_BLOCK_SEQ, "par": _lib.FPS_BLOCK_PAR, "sdxl": _lib.FPS_BLOCK_SDXL,
+         "double": _lib.FPS_BLOCK_DOUBLE}
+_SEQ_KEYS = ("w_qkv", "b_qkv", "w_o", "b_o", "w_up", "b_up", "w_down", "b_down")
 _SDXL_KEYS = ("ln1_w", "ln1_b", "ln2_w", "ln2_b", "ln3_w", "ln3_b", "w_q2", "b_q2", "w_kv2",
               "b_kv2", "w_o2", "b_o2")
 
@@ -98,6 +100,9 @@ class BlockWeights:
         td = TORCH_DTYPE[dtype]
         self.kind = _KIND[w.get("kind", "seq")]
         alias = {"w_1": "w_qkv", "b_1": "b_qkv", "w_2": "w_down", "b_2": "b_down"}
+        if self.kind == _lib.FPS_BLOCK_DOUBLE:     # image stream = the primary fields
+            w = dict(w["img"], **{"t" + k[1:] if k.startswith("w_") else "tb" + k[1:]: v
+                                  for k, v in w["txt"].items()})
         self.t = {alias.get(k, k): torch.as_tensor(np.ascontiguousarray(v)).to(device=device, dtype=td)
                   for k, v in w.items() if k != "kind" and v is not None}
         H = self.t["w_down"].shape[0]
@@ -119,7 +124,9 @@ class BlockWeights:
                                    *[ptr(self.t.get(k)) for k in
                                      ("w_qkv", "b_qkv", "w_o", "b_o", "w_up", "b_up", "w_down",
                                       "b_down")], self.kind, self.D_ctx,
-                                   *[ptr(self.t.get(k)) for k in _SDXL_KEYS])
+                                   *[ptr(self.t.get(k)) for k in _SDXL_KEYS],
+                                   *[ptr(self.t.get("t" + k[1:] if k.startswith("w_") else
+                                                    "tb" + k[1:])) for k in _SEQ_KEYS])
 
     def context_kv(self, ctx, out=None, stream=None):
         """SDXL block: the cross-attention K|V rows [n, 2H] of prompt encodings ctx [n, D_ctx]."""
@@ -136,7 +143,8 @@ class VarlenBatch:
     u_row / u_src: Y-mode cached rows. mod: [n_req, 6H] device tensor or None."""
 
     def __init__(self, n_active, L, q_row=None, mod=None, mode=FPS_MODE_KV, u_row=None,
-                 u_src=None, n_unmasked=None, device="cuda", ctx_kv=None, n_ctx=None):
+                 u_src=None, n_unmasked=None, device="cuda", ctx_kv=None, n_ctx=None,
+                 act_ids=None, L_img=None, mod_stride=0):
         self.n_active = list(map(int, n_active))
         self.L = list(map(int, L))
         cu_q = np.concatenate([[0], np.cumsum(self.n_active)]).astype(np.int32)
@@ -155,6 +163,23 @@ class VarlenBatch:
             max(self.L, default=0), ptr(self.cu_q), ptr(self.cu_k),
             self.h_cu_q.ctypes.data_as(C.c_void_p), self.h_cu_k.ctypes.data_as(C.c_void_p),
             ptr(q_row), ptr(mod), mode, int(cu_u[-1]), ptr(self.cu_u), ptr(u_src), ptr(u_row))
+        self.c.mod_stride = mod_stride
+        if act_ids is not None:      # double-stream blocks: stream-major order of the rows
+            # act_ids[r]: ascending token ids of request r's active rows (all rows if dense)
+            perm, kvr, ni, nt = [], [], [], []
+            for st in (0, 1):
+                for r, ids in enumerate(act_ids):
+                    ids = np.asarray(ids)
+                    sel = np.flatnonzero((ids >= L_img) if st else (ids < L_img))
+                    perm.append(cu_q[r] + sel)
+                    kvr.append(cu_k[r] + ids[sel])
+                    (nt if st else ni).append(len(sel))
+            arrs = (np.concatenate(perm), np.concatenate(kvr),
+                    np.concatenate([[0], np.cumsum(ni)]), np.concatenate([[0], np.cumsum(nt)]))
+            self.sm = [torch.as_tensor(a.astype(np.int32), device=device) for a in arrs]
+            self.c.total_q_img = int(sum(ni))
+            self.c.d_sm_perm, self.c.d_sm_kvrow, self.c.d_cu_img, self.c.d_cu_txt = \
+                (ptr(t) for t in self.sm)
         if ctx_kv is not None:       # SDXL blocks: request r's prompt K|V rows (n_ctx[r] each)
             cu_c = np.concatenate([[0], np.cumsum(n_ctx)]).astype(np.int32)
             self.h_cu_ctx, self.cu_ctx, self.ctx_kv = cu_c, torch.tensor(cu_c, device=device), ctx_kv
@@ -290,7 +315,7 @@ class Engine:
 
     def __init__(self, layers, heads, mode, dtype, L_img, L_txt, max_batch, n_steps, deltas,
                  cache: Cache, mod_table=None, slots=0, plan_policy=0, plan=None,
-                 cost_model=(0.0, 0.0, 0.0, 0.0), L_ctx=0):
+                 cost_model=(0.0, 0.0, 0.0, 0.0), L_ctx=0, mod_width=0):
         self.layers = layers                      # list[BlockWeights] (keeps tensors alive)
         self._w = (fps_block_weights * len(layers))(*[l.c for l in layers])
         self._deltas = (C.c_float * n_steps)(*map(float, deltas))
@@ -302,7 +327,8 @@ class Engine:
                             n_steps, C.cast(self._w, C.c_void_p), ptr(mod_table),
                             C.cast(self._deltas, C.c_void_p), cache.h, slots, plan_policy,
                             C.cast(self._plan, C.c_void_p), (C.c_double * 4)(*cost_model),
-                            L_ctx, max((getattr(l, "D_ctx", 0) for l in layers), default=0))
+                            L_ctx, max((getattr(l, "D_ctx", 0) for l in layers), default=0),
+                            mod_width)
         self.desc = d
         h = C.c_void_p()
         _lib.fps_engine_create(C.byref(d), C.byref(h))

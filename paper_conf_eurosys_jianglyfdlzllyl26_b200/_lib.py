@@ -16,7 +16,7 @@ LIB_PATH = os.environ.get("FPS_LIB") or os.path.join(_HERE, "libflashps.so")
 FPS_OK, FPS_EINVAL, FPS_ECUDA, FPS_ENOMEM, FPS_EUNSUPPORTED, FPS_ESTATE = 0, -1, -2, -3, -4, -5
 FPS_F32, FPS_BF16 = 0, 1
 FPS_MODE_KV, FPS_MODE_Y = 0, 1
-FPS_BLOCK_SEQ, FPS_BLOCK_PAR, FPS_BLOCK_SDXL = 0, 1, 2
+FPS_BLOCK_SEQ, FPS_BLOCK_PAR, FPS_BLOCK_SDXL, FPS_BLOCK_DOUBLE = 0, 1, 2, 3
 
 vp, i32, u32, i64, sz, dbl = C.c_void_p, C.c_int32, C.c_uint32, C.c_int64, C.c_size_t, C.c_double
 P_i32, P_u8, P_dbl, P_f32 = C.POINTER(C.c_int32), C.POINTER(C.c_uint8), C.POINTER(C.c_double), C.POINTER(C.c_float)
@@ -45,7 +45,8 @@ class fps_block_weights(C.Structure):
                 ("b_up", vp), ("w_down", vp), ("b_down", vp), ("kind", i32), ("D_ctx", i32),
                 ("ln1_w", vp), ("ln1_b", vp), ("ln2_w", vp), ("ln2_b", vp), ("ln3_w", vp),
                 ("ln3_b", vp), ("w_q2", vp), ("b_q2", vp), ("w_kv2", vp), ("b_kv2", vp),
-                ("w_o2", vp), ("b_o2", vp)]
+                ("w_o2", vp), ("b_o2", vp), ("t_qkv", vp), ("tb_qkv", vp), ("t_o", vp),
+                ("tb_o", vp), ("t_up", vp), ("tb_up", vp), ("t_down", vp), ("tb_down", vp)]
 
 
 class fps_varlen_batch(C.Structure):
@@ -53,7 +54,8 @@ class fps_varlen_batch(C.Structure):
                 ("max_k", i32), ("d_cu_q", vp), ("d_cu_k", vp), ("h_cu_q", vp), ("h_cu_k", vp),
                 ("d_q_row", vp), ("d_mod", vp), ("mode", i32), ("total_u", i32),
                 ("d_cu_u", vp), ("d_u_src", vp), ("d_u_row", vp), ("d_ctx_kv", vp),
-                ("d_cu_ctx", vp), ("h_cu_ctx", vp)]
+                ("d_cu_ctx", vp), ("h_cu_ctx", vp), ("mod_stride", i32), ("total_q_img", i32),
+                ("d_sm_perm", vp), ("d_sm_kvrow", vp), ("d_cu_img", vp), ("d_cu_txt", vp)]
 
 
 class fps_engine_desc(C.Structure):
@@ -61,7 +63,7 @@ class fps_engine_desc(C.Structure):
                 ("mode", i32), ("L_img", i32), ("L_txt", i32), ("max_batch", i32),
                 ("n_steps", i32), ("layers", vp), ("d_mod_table", vp), ("h_deltas", vp),
                 ("cache", vp), ("slots", i32), ("plan_policy", i32), ("h_plan", vp),
-                ("cost_model", dbl * 4), ("L_ctx", i32), ("D_ctx", i32)]
+                ("cost_model", dbl * 4), ("L_ctx", i32), ("D_ctx", i32), ("mod_width", i32)]
 
 
 class fps_request(C.Structure):

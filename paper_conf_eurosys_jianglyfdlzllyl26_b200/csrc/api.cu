@@ -152,8 +152,10 @@ static fps_status check_weights(const fps_block_weights* w) {
   FPS_CHECK_ARG(w->H > 0 && w->heads > 0 && w->head_dim > 0 && w->heads * w->head_dim == w->H,
                 "H=%d heads=%d head_dim=%d", w->H, w->heads, w->head_dim);
   FPS_CHECK_ARG(w->F > 0, "F=%d", w->F);
-  FPS_CHECK_ARG(w->kind == FPS_BLOCK_SEQ || w->kind == FPS_BLOCK_PAR || w->kind == FPS_BLOCK_SDXL,
-                "kind %d", w->kind);
+  FPS_CHECK_ARG(w->kind >= FPS_BLOCK_SEQ && w->kind <= FPS_BLOCK_DOUBLE, "kind %d", w->kind);
+  if (w->kind == FPS_BLOCK_DOUBLE)
+    FPS_CHECK_ARG(w->w_qkv && w->w_o && w->w_up && w->w_down && w->t_qkv && w->t_o && w->t_up &&
+                  w->t_down, "double-stream block: image or text weight pointer is NULL");
   if (w->kind == FPS_BLOCK_SDXL) {
     FPS_CHECK_ARG(w->w_qkv && w->w_o && w->w_up && w->w_down && w->w_q2 && w->w_kv2 && w->w_o2,
                   "SDXL block: weight pointer is NULL");
@@ -164,6 +166,7 @@ static fps_status check_weights(const fps_block_weights* w) {
       return fail(FPS_EUNSUPPORTED,
                   "SDXL block: bf16 tcgen05 path only (H=%d, F=%d, D_ctx=%d multiples of 64)",
                   w->H, w->F, w->D_ctx);
+  } else if (w->kind == FPS_BLOCK_DOUBLE) {
   } else if (w->kind == FPS_BLOCK_PAR)
     FPS_CHECK_ARG(w->w_qkv && w->w_down && !w->w_o && !w->b_o && !w->w_up && !w->b_up,
                   "parallel block: w_qkv (W1) and w_down (W2) set, w_o/b_o/w_up/b_up NULL");
@@ -188,6 +191,16 @@ static fps_status check_batch(const fps_varlen_batch* b) {
   return FPS_OK;
 }
 
+static fps_status check_streams(const fps_block_weights* w, const fps_varlen_batch* b) {
+  if (w->kind != FPS_BLOCK_DOUBLE || b->n_req == 0 || b->total_q == 0) return FPS_OK;
+  FPS_CHECK_ARG(b->d_sm_perm && b->d_sm_kvrow && b->d_cu_img && b->d_cu_txt,
+                "double-stream block: stream-major order (d_sm_perm, d_sm_kvrow, d_cu_img, "
+                "d_cu_txt) required");
+  FPS_CHECK_ARG(b->total_q_img >= 0 && b->total_q_img <= b->total_q, "total_q_img %d",
+                b->total_q_img);
+  return FPS_OK;
+}
+
 static fps_status check_ctx(const fps_block_weights* w, const fps_varlen_batch* b) {
   if (w->kind != FPS_BLOCK_SDXL || b->n_req == 0 || b->total_q == 0) return FPS_OK;
   FPS_CHECK_ARG(b->d_ctx_kv && b->d_cu_ctx && b->h_cu_ctx && b->h_cu_q,
@@ -195,6 +208,101 @@ static fps_status check_ctx(const fps_block_weights* w, const fps_varlen_batch* 
   for (int r = 0; r < b->n_req; ++r)
     FPS_CHECK_ARG(b->h_cu_ctx[r + 1] > b->h_cu_ctx[r],
                   "SDXL block: request %d has an empty prompt context", r);
+  return FPS_OK;
+}
+
+// Double-stream (Flux MM-DiT) block, reading R25.  The active rows are processed in
+// stream-major order (all image rows, then all text rows) so each stream's projections are
+// one GEMM over contiguous rows with that stream's weights; Q is scattered back to the
+// request-major order the varlen attention reads, its output gathered to stream-major again,
+// and the final epilogue writes y in request-major order.
+static fps_status double_block_forward(const fps_block_weights* w, const fps_varlen_batch* b,
+                                       const void* x_act, void* y_act, void* kv, const void* xu,
+                                       cudaEvent_t kv_ready, void* d_ws, size_t ws_bytes,
+                                       cudaStream_t s) {
+  const int H = w->H, F = w->F, dt = w->dtype, tq = b->total_q;
+  const int tu = (b->mode == FPS_MODE_Y) ? b->total_u : 0;
+  const int ti = b->total_q_img, tt = tq - ti;
+  const size_t e = elt_size(dt), rowb = (size_t)H * e;
+  BlockWs ws;
+  const size_t need = ws_layout(H, F, dt, tq, tu, (char*)d_ws, &ws);
+  FPS_CHECK_ARG(ws_bytes >= need, "workspace %zu < %zu bytes", ws_bytes, need);
+  const int MS = b->mod_stride > 0 ? b->mod_stride : 12 * H;
+  const char* mod = (const char*)b->d_mod;
+  auto modp = [&](int stream, int off) -> const void* {
+    return mod ? mod + ((size_t)stream * 6 * H + (size_t)off * H) * e : nullptr;
+  };
+  const int32_t* perm = b->d_sm_perm;
+  const int32_t* kvrow = b->d_sm_kvrow;
+  const int32_t* cu[2] = {b->d_cu_img, b->d_cu_txt};
+  const int rows0[2] = {0, ti}, nrows[2] = {ti, tt};
+  const void* Wqkv[2] = {w->w_qkv, w->t_qkv};
+  const void* Bqkv[2] = {w->b_qkv, w->tb_qkv};
+  const void* Wo[2] = {w->w_o, w->t_o};
+  const void* Bo[2] = {w->b_o, w->tb_o};
+  const void* Wup[2] = {w->w_up, w->t_up};
+  const void* Bup[2] = {w->b_up, w->tb_up};
+  const void* Wdn[2] = {w->w_down, w->t_down};
+  const void* Bdn[2] = {w->b_down, w->tb_down};
+  char* x_sm = ws.x2;      // x in stream-major order (the fp32-sized buffer is free here)
+  char* ao_sm = ws.h2;     // attention output, stream-major (h2 is written only after its use)
+  auto at = [&](char* base, int st, size_t width = 0) {
+    return base + (size_t)rows0[st] * (width ? width : rowb);
+  };
+  if (tq > 0) {
+    FPS_TRY(launch_copy_rows(x_act, perm, nullptr, tq, (int)rowb, x_sm, s));
+    for (int st = 0; st < 2; ++st) {
+      // a4 per stream, a5 per stream: Q -> request-major rows, K|V -> merged key rows
+      FPS_TRY(launch_ln_mod(dt, at(x_sm, st), nullptr, nrows[st], H, at(ws.h, st), cu[st],
+                            b->n_req, mod, 6 * H * st, s, nullptr, MS));
+      Epilogue ep{};
+      ep.bias = Bqkv[st];
+      ep.out0 = ws.q; ep.ld0 = H; ep.map0 = perm + rows0[st];
+      ep.out1 = kv; ep.ld1 = 2 * H; ep.map1 = kvrow + rows0[st];
+      ep.split = H;
+      FPS_TRY(launch_gemm(dt, at(ws.h, st), Wqkv[st], nrows[st], 3 * H, H, ep, s));
+    }
+  }
+  if (tu > 0) {
+    // Y-mode: cached input rows U (image rows, R9) -> image-stream LN -> K|V projection
+    if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
+    kv_ready = nullptr;
+    FPS_TRY(launch_ln_mod(dt, xu, b->d_u_src, tu, H, ws.hu, b->d_cu_u, b->n_req, mod, 0, s,
+                          nullptr, MS));
+    Epilogue ep{};
+    ep.bias = w->b_qkv ? (const char*)w->b_qkv + (size_t)H * e : nullptr;
+    ep.out0 = kv; ep.ld0 = 2 * H; ep.map0 = b->d_u_row;
+    ep.split = 2 * H;
+    FPS_TRY(launch_gemm(dt, ws.hu, (const char*)w->w_qkv + (size_t)H * H * e, tu, 2 * H, H, ep, s));
+  }
+  if (tq == 0) return FPS_OK;
+  // a6: joint attention of both streams' queries over the merged keys
+  if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
+  FPS_TRY(launch_attention(dt, ws.q, kv, ws.ao, w->heads, w->head_dim, b->d_cu_q, b->d_cu_k,
+                           b->h_cu_q, b->h_cu_k, b->n_req, tq, b->max_q, b->max_k, s));
+  FPS_TRY(launch_copy_rows(ws.ao, perm, nullptr, tq, (int)rowb, ao_sm, s));
+  for (int st = 0; st < 2; ++st) {   // a7 per stream: x1 = x + gate1 (A Wo^T + bo)
+    Epilogue ep{};
+    ep.bias = Bo[st];
+    ep.resid = at(x_sm, st); ep.ld_resid = H;
+    ep.gate = modp(st, 2); ep.gate_stride = MS; ep.cu = cu[st]; ep.n_req = b->n_req;
+    ep.out0 = at(ws.x1, st); ep.ld0 = H; ep.split = H;
+    FPS_TRY(launch_gemm(dt, at(ao_sm, st), Wo[st], nrows[st], H, H, ep, s));
+  }
+  for (int st = 0; st < 2; ++st) {   // a8 per stream; y written back in request-major order
+    FPS_TRY(launch_ln_mod(dt, at(ws.x1, st), nullptr, nrows[st], H, at(ws.h2, st), cu[st],
+                          b->n_req, mod, 6 * H * st + 3 * H, s, nullptr, MS));
+    Epilogue eu{};
+    eu.bias = Bup[st]; eu.act = 1;
+    eu.out0 = at(ws.u, st, (size_t)F * e); eu.ld0 = F; eu.split = F;
+    FPS_TRY(launch_gemm(dt, at(ws.h2, st), Wup[st], nrows[st], F, H, eu, s));
+    Epilogue ed{};
+    ed.bias = Bdn[st];
+    ed.resid = at(ws.x1, st); ed.ld_resid = H;
+    ed.gate = modp(st, 5); ed.gate_stride = MS; ed.cu = cu[st]; ed.n_req = b->n_req;
+    ed.out0 = y_act; ed.ld0 = H; ed.map0 = perm + rows0[st]; ed.split = H;
+    FPS_TRY(launch_gemm(dt, at(ws.u, st, (size_t)F * e), Wdn[st], nrows[st], H, F, ed, s));
+  }
   return FPS_OK;
 }
 
@@ -208,14 +316,17 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
   BlockWs ws;
   const size_t need = ws_layout(H, F, dt, tq, tu, (char*)d_ws, &ws);
   FPS_CHECK_ARG(ws_bytes >= need, "workspace %zu < %zu bytes", ws_bytes, need);
+  if (w->kind == FPS_BLOCK_DOUBLE)
+    return double_block_forward(w, b, x_act, y_act, kv, xu, kv_ready, d_ws, ws_bytes, s);
   const bool sdxl = w->kind == FPS_BLOCK_SDXL;
+  const int MS = b->mod_stride > 0 ? b->mod_stride : 6 * H;
   const char* mod = sdxl ? nullptr : (const char*)b->d_mod;
   auto modp = [&](int off) -> const void* { return mod ? mod + (size_t)off * H * e : nullptr; };
   // a4, the first norm: adaLN-modulated LN, or the SDXL block's affine LN (reading R24)
   auto ln1 = [&](const void* x, const int32_t* rows, int n, void* out, const int32_t* cu,
                  const int32_t* out_rows) -> fps_status {
     if (sdxl) return launch_ln_affine(dt, x, rows, n, H, out, w->ln1_w, w->ln1_b, s, out_rows);
-    return launch_ln_mod(dt, x, rows, n, H, out, cu, b->n_req, mod, 0, s, out_rows);
+    return launch_ln_mod(dt, x, rows, n, H, out, cu, b->n_req, mod, 0, s, out_rows, MS);
   };
 
   // Y-mode, sequential block: Q over the active rows, K|V in ONE GEMM over all rows of the
@@ -277,7 +388,7 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
     Epilogue ep{};
     ep.bias = w->b_down;
     ep.resid = x_act; ep.ld_resid = H;
-    ep.gate = modp(2); ep.gate_stride = 6 * H; ep.cu = b->d_cu_q; ep.n_req = b->n_req;
+    ep.gate = modp(2); ep.gate_stride = MS; ep.cu = b->d_cu_q; ep.n_req = b->n_req;
     ep.out0 = y_act; ep.ld0 = H; ep.split = H;
     return launch_gemm(dt, cat, w->w_down, tq, H, H + F, ep, s);
   }
@@ -289,7 +400,7 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
     Epilogue ep{};
     ep.bias = w->b_o;
     ep.resid = x_act; ep.ld_resid = H;
-    ep.gate = modp(2); ep.gate_stride = 6 * H; ep.cu = b->d_cu_q; ep.n_req = b->n_req;
+    ep.gate = modp(2); ep.gate_stride = MS; ep.cu = b->d_cu_q; ep.n_req = b->n_req;
     ep.out0 = ws.x1; ep.ld0 = H; ep.split = H;
     ep.out0_f32 = sdxl;          // SDXL: keep the residual stream x1, x2 in fp32 (R24)
     FPS_TRY(launch_gemm(dt, ws.ao, w->w_o, tq, H, H, ep, s));
@@ -329,7 +440,8 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
     return launch_gemm(dt, ws.u, w->w_down, tq, H, F, ep, s);
   }
   // a8: y = x1 + gate2 (GELU(LN(x1)(1+scale2)+shift2 W1^T + b1) W2^T + b2)
-  FPS_TRY(launch_ln_mod(dt, ws.x1, nullptr, tq, H, ws.h2, b->d_cu_q, b->n_req, b->d_mod, 3 * H, s));
+  FPS_TRY(launch_ln_mod(dt, ws.x1, nullptr, tq, H, ws.h2, b->d_cu_q, b->n_req, b->d_mod, 3 * H, s,
+                        nullptr, MS));
   {
     Epilogue ep{};
     ep.bias = w->b_up; ep.act = 1;
@@ -340,7 +452,7 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
     Epilogue ep{};
     ep.bias = w->b_down;
     ep.resid = ws.x1; ep.ld_resid = H;
-    ep.gate = modp(5); ep.gate_stride = 6 * H; ep.cu = b->d_cu_q; ep.n_req = b->n_req;
+    ep.gate = modp(5); ep.gate_stride = MS; ep.cu = b->d_cu_q; ep.n_req = b->n_req;
     ep.out0 = y_act; ep.ld0 = H; ep.split = H;
     FPS_TRY(launch_gemm(dt, ws.u, w->w_down, tq, H, F, ep, s));
   }
@@ -475,6 +587,7 @@ fps_status fps_masked_block_forward(const fps_block_weights* w, const fps_varlen
     FPS_CHECK_ARG(b->total_q == b->total_k, "d_q_row NULL requires total_q == total_k");
   FPS_CHECK_ARG(w->heads * w->head_dim == w->H, "heads*head_dim != H");
   FPS_TRY(check_ctx(w, b));
+  FPS_TRY(check_streams(w, b));
   return block_forward(w, b, d_x_act, d_y_act, d_kv, d_xu, (cudaEvent_t)kv_ready, d_ws, ws_bytes,
                        as_stream(stream));
 }
@@ -545,6 +658,7 @@ fps_status fps_dense_block_forward(const fps_block_weights* w, const fps_varlen_
   FPS_CHECK_ARG(b->d_q_row == nullptr && b->total_q == b->total_k,
                 "dense block: d_q_row must be NULL and total_q == total_k");
   FPS_TRY(check_ctx(w, b));
+  FPS_TRY(check_streams(w, b));
   fps_varlen_batch bb = *b;
   bb.mode = FPS_MODE_KV;
   bb.total_u = 0;

@@ -38,6 +38,11 @@ struct fps_engine {
   std::vector<int> sdxl_slot;  // per layer: index into ctx_kv, or -1
   char *ctx_in = nullptr, *ctx_kv = nullptr;
   int32_t *d_cu_ctx = nullptr, *h_cu_ctx = nullptr;
+  // double-stream blocks: stream-major order of the masked and the dense batch
+  // (perm | kvrow | cu_img | cu_txt, masked then dense)
+  bool has_double = false;
+  int MW = 0;                   // modulation elements per request and block
+  int32_t *d_sm = nullptr, *h_sm = nullptr;
   float* d_delta = nullptr;
   // pinned host staging
   int32_t* h_meta = nullptr;
@@ -58,6 +63,8 @@ static void free_engine(fps_engine* e) {
                   e->kv_scratch, e->final_slot, e->ws, e->mod_batch};
   for (char* p : bufs) if (p) cudaFree(p);
   for (char* p : e->slots) if (p) cudaFree(p);
+  if (e->d_sm) cudaFree(e->d_sm);
+  if (e->h_sm) cudaFreeHost(e->h_sm);
   if (e->ctx_in) cudaFree(e->ctx_in);
   if (e->ctx_kv) cudaFree(e->ctx_kv);
   if (e->d_cu_ctx) cudaFree(e->d_cu_ctx);
@@ -117,6 +124,12 @@ fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out) {
       FPS_CHECK_ARG(d.L_ctx > 0 && d.layers[l].D_ctx == d.D_ctx,
                     "layer %d: SDXL block needs L_ctx > 0 and D_ctx == the engine's", l);
   }
+  bool any_double = false;
+  for (int l = 0; l < d.n_layers; ++l) any_double |= d.layers[l].kind == FPS_BLOCK_DOUBLE;
+  FPS_CHECK_ARG(!any_double || !d.d_mod_table || d.mod_width == 12 * d.H,
+                "double-stream blocks need mod_width = 12H (got %d)", d.mod_width);
+  FPS_CHECK_ARG(d.mod_width == 0 || d.mod_width == 6 * d.H || d.mod_width == 12 * d.H,
+                "mod_width %d", d.mod_width);
   auto* e = new (std::nothrow) fps_engine();
   if (!e) return fail(FPS_ENOMEM, "engine alloc");
   e->d = d;
@@ -127,8 +140,11 @@ fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out) {
   e->d.h_deltas = nullptr;
   e->d.h_plan = nullptr;
   e->sdxl_slot.assign(d.n_layers, -1);
-  for (int l = 0; l < d.n_layers; ++l)
+  for (int l = 0; l < d.n_layers; ++l) {
     if (d.layers[l].kind == FPS_BLOCK_SDXL) e->sdxl_slot[l] = e->n_sdxl++;
+    if (d.layers[l].kind == FPS_BLOCK_DOUBLE) e->has_double = true;
+  }
+  e->MW = d.mod_width > 0 ? d.mod_width : 6 * d.H;
   e->L = d.L_img + d.L_txt;
   e->elt = d.dtype == FPS_BF16 ? 2 : 4;
   e->W = d.mode == FPS_MODE_KV ? 2 * d.H : d.H;
@@ -157,7 +173,12 @@ fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out) {
   if (d.mode == FPS_MODE_KV) dmal(&e->final_slot, R * e->row_h);
   e->ws_bytes = fps_block_workspace_bytes(d.H, d.F, d.dtype, (int)R, (int)R);
   dmal(&e->ws, e->ws_bytes);
-  dmal(&e->mod_batch, (size_t)d.n_layers * d.max_batch * 6 * e->row_h);
+  dmal(&e->mod_batch, (size_t)d.n_layers * d.max_batch * e->MW * e->elt);
+  const size_t sm_ints = 2 * (2 * R + 2 * (d.max_batch + 1));
+  if (e->has_double) {
+    if (err == cudaSuccess) err = cudaMalloc((void**)&e->d_sm, sm_ints * 4);
+    if (err == cudaSuccess) err = cudaHostAlloc((void**)&e->h_sm, sm_ints * 4, cudaHostAllocDefault);
+  }
   e->slots.assign(e->D, nullptr);
   for (int i = 0; i < e->D; ++i) dmal(&e->slots[i], slot_bytes);
   if (e->n_sdxl) {
@@ -231,6 +252,10 @@ struct Batch {
   int tq = 0, tu = 0, tk = 0, max_q = 0;
   int32_t *cu_q, *cu_k, *cu_u, *q_row, *u_row, *mod_ids;      // device (inside d_meta)
   int32_t *h_cu_q, *h_cu_k, *h_cu_u;                          // host (inside h_meta)
+  // double-stream blocks: [0] masked batch, [1] dense batch (device, inside e->d_sm)
+  int ti[2] = {0, 0};
+  int32_t *sm_perm[2] = {nullptr, nullptr}, *sm_kvrow[2] = {nullptr, nullptr};
+  int32_t *cu_img[2] = {nullptr, nullptr}, *cu_txt[2] = {nullptr, nullptr};
 };
 
 static fps_status admit(fps_engine* e, fps_request* reqs, const std::vector<int>& live, Batch& B,
@@ -289,6 +314,46 @@ static fps_status admit(fps_engine* e, fps_request* reqs, const std::vector<int>
   B.h_cu_q = cu_q;
   B.h_cu_k = cu_k;
   B.h_cu_u = cu_u;
+  if (e->has_double) {
+    // stream-major order (all image rows, then all text rows) of the masked and dense batches
+    const int R = e->maxR, nb1 = e->d.max_batch + 1, Li = e->d.L_img;
+    for (int v = 0; v < 2; ++v) {
+      int32_t* base = e->h_sm + (size_t)v * (2 * R + 2 * nb1);
+      int32_t *perm = base, *kvr = base + R, *ci = base + 2 * R, *ct = ci + nb1;
+      int k = 0;
+      ci[0] = ct[0] = 0;
+      for (int i = 0; i < n; ++i) {          // image rows
+        const int cnt = v == 0 ? B.nq[i] : L;
+        int ni = 0;
+        for (int j = 0; j < cnt; ++j) {
+          const int tok = v == 0 ? e->h_mids[i * L + j] : j;
+          if (tok >= Li) break;                // ascending ids: text rows come last
+          perm[k] = v == 0 ? cu_q[i] + j : i * L + j;
+          kvr[k] = v == 0 ? q_row[cu_q[i] + j] : i * L + j;
+          ++k, ++ni;
+        }
+        ci[i + 1] = ci[i] + ni;
+      }
+      B.ti[v] = k;
+      for (int i = 0; i < n; ++i) {          // text rows
+        const int cnt = v == 0 ? B.nq[i] : L;
+        const int first = ci[i + 1] - ci[i];
+        for (int j = first; j < cnt; ++j) {
+          perm[k] = v == 0 ? cu_q[i] + j : i * L + j;
+          kvr[k] = v == 0 ? q_row[cu_q[i] + j] : i * L + j;
+          ++k;
+        }
+        ct[i + 1] = ct[i] + (cnt - first);
+      }
+      int32_t* dbase = e->d_sm + (size_t)v * (2 * R + 2 * nb1);
+      B.sm_perm[v] = dbase;
+      B.sm_kvrow[v] = dbase + R;
+      B.cu_img[v] = dbase + 2 * R;
+      B.cu_txt[v] = dbase + 2 * R + nb1;
+    }
+    FPS_COPY_TRY(cs, cudaMemcpyAsync(e->d_sm, e->h_sm, (size_t)2 * (2 * R + 2 * nb1) * 4,
+                                     cudaMemcpyHostToDevice, cs));
+  }
   if (e->n_sdxl) {
     // SDXL blocks: the prompt is fixed over the steps, so each block's cross-attention K|V
     // is projected once per admission (one GEMM per SDXL block over the batch's prompts)
@@ -361,7 +426,7 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
     for (int l = 0; l < N; ++l)
       for (int i = 0; i < n; ++i) mod_ids[l * n + i] = l * e->d.n_steps + reqs[B.idx[i]].step;
     FPS_COPY_TRY(cs, cudaMemcpyAsync(B.mod_ids, mod_ids, (size_t)N * n * 4, cudaMemcpyHostToDevice, cs));
-    FPS_TRY(launch_copy_rows(e->d.d_mod_table, B.mod_ids, nullptr, N * n, 6 * (int)e->row_h,
+    FPS_TRY(launch_copy_rows(e->d.d_mod_table, B.mod_ids, nullptr, N * n, e->MW * e->elt,
                              e->mod_batch, cs));
   }
   for (int i = 0; i < n; ++i) e->h_delta[i] = e->deltas[reqs[B.idx[i]].step];
@@ -434,7 +499,18 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
   vb.d_cu_u = B.cu_u;
   vb.d_u_src = B.u_row;
   vb.d_u_row = B.u_row;
+  vb.mod_stride = e->MW;
+  vb.total_q_img = B.ti[0];
+  vb.d_sm_perm = B.sm_perm[0];
+  vb.d_sm_kvrow = B.sm_kvrow[0];
+  vb.d_cu_img = B.cu_img[0];
+  vb.d_cu_txt = B.cu_txt[0];
   fps_varlen_batch vd = vb;             // dense: every row of every request is active
+  vd.total_q_img = B.ti[1];
+  vd.d_sm_perm = B.sm_perm[1];
+  vd.d_sm_kvrow = B.sm_kvrow[1];
+  vd.d_cu_img = B.cu_img[1];
+  vd.d_cu_txt = B.cu_txt[1];
   vd.total_q = B.tk;
   vd.max_q = e->L;
   vd.d_cu_q = B.cu_k;
@@ -448,7 +524,7 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
   bool rep_full = true;
   for (int l = 0; l < N; ++l) {
     const fps_block_weights* w = &e->layers[l];
-    const void* mod = e->d.d_mod_table ? e->mod_batch + (size_t)l * n * 6 * e->row_h : nullptr;
+    const void* mod = e->d.d_mod_table ? e->mod_batch + (size_t)l * n * e->MW * e->elt : nullptr;
     vb.d_mod = mod;
     vd.d_mod = mod;
     if (e->sdxl_slot[l] >= 0) {

@@ -623,6 +623,9 @@ __global__ void __launch_bounds__(384, 1)
 #ifndef FPS_ATTN_POLY
 #define FPS_ATTN_POLY 4
 #endif
+#ifndef FPS_ATTN_POLY64          // the same for head_dim 64 (twice the exponentials per MMA FLOP)
+#define FPS_ATTN_POLY64 4
+#endif
 #ifndef FPS_ATTN_MMA_SPIN
 #define FPS_ATTN_MMA_SPIN 0
 #endif
@@ -631,8 +634,10 @@ __global__ void __launch_bounds__(384, 1)
 #else
 #define ATTN_MMA_WAIT(bar, par) tc::mbar_wait_sleep(bar, par)
 #endif
+template <int D>
 __device__ __forceinline__ constexpr bool attn_poly(int i) {
-  return FPS_ATTN_POLY > 0 && ((i >> 3) % (FPS_ATTN_POLY > 0 ? FPS_ATTN_POLY : 1)) == (FPS_ATTN_POLY > 0 ? FPS_ATTN_POLY : 1) - 1;
+  constexpr int N = D == 64 ? FPS_ATTN_POLY64 : FPS_ATTN_POLY;
+  return N > 0 && ((i >> 3) % (N > 0 ? N : 1)) == (N > 0 ? N : 1) - 1;
 }
 #ifdef FPS_ATTN_TRACE
 // developer instrumentation (separate build): per-step clock64 stamps of one CTA
@@ -869,7 +874,7 @@ __global__ void __launch_bounds__(512, 1)
 #pragma unroll
           for (int i = c * 32; i < c * 32 + 32; i += 2) {
             tc::ffma2(s[i], s[i + 1], s[i], s[i + 1], scale_log2, scale_log2, nm, nm);
-            if (attn_poly(i)) {
+            if (attn_poly<D>(i)) {
               tc::ex2_poly2(s[i], s[i + 1]);
             } else {
               s[i] = tc::ex2(s[i]);

@@ -478,17 +478,18 @@ static LnMod<T> ln_params(const void* shift, const void* scale, int stride, floa
 
 fps_status launch_ln_mod(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
                          const int32_t* cu, int n_req, const void* mod, int shift_off,
-                         cudaStream_t s, const int32_t* out_rows) {
+                         cudaStream_t s, const int32_t* out_rows, int mod_stride) {
   if (n <= 0) return FPS_OK;
+  if (mod_stride <= 0) mod_stride = 6 * H;
   const size_t e = dtype == FPS_BF16 ? 2 : 4;
   const char* sh = mod ? (const char*)mod + (size_t)shift_off * e : nullptr;
   const char* sc = mod ? sh + (size_t)H * e : nullptr;
   if (dtype == FPS_BF16)
     return ln_mod_t<__nv_bfloat16>(x, rows, n, H, out,
-                                   ln_params<__nv_bfloat16>(sh, sc, 6 * H, 1.0f, cu, n_req), s,
-                                   out_rows);
-  return ln_mod_t<float>(x, rows, n, H, out, ln_params<float>(sh, sc, 6 * H, 1.0f, cu, n_req), s,
-                         out_rows);
+                                   ln_params<__nv_bfloat16>(sh, sc, mod_stride, 1.0f, cu, n_req),
+                                   s, out_rows);
+  return ln_mod_t<float>(x, rows, n, H, out, ln_params<float>(sh, sc, mod_stride, 1.0f, cu, n_req),
+                         s, out_rows);
 }
 
 fps_status launch_ln_affine(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,

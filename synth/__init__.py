@@ -101,6 +101,9 @@ def block_weights(g: np.random.Generator, H: int, F: int, dtype: str = "bf16",
     projections w_o / w_o2, GEGLU input w_up [2F, H] (first F rows the value half, last F the
     gate half), w_down [H, F], and three affine LayerNorms ln{1,2,3}_w ~ 1 + N(0, 0.02^2),
     ln{1,2,3}_b ~ N(0, 0.02^2)."""
+    if kind == "double":     # Flux double-stream block: one sequential set per stream (R25)
+        return {"kind": "double", "img": block_weights(g, H, F, dtype),
+                "txt": block_weights(g, H, F, dtype)}
     if kind == "sdxl":
         n = lambda *shape: g.standard_normal(shape, dtype=np.float32)
         w = {
@@ -154,17 +157,19 @@ def context(g: np.random.Generator, L_ctx: int = 77, D_ctx: int = 2048,
 
 
 def mod_table(g: np.random.Generator, layers: int, steps: int, H: int, dtype: str = "bf16",
-              enabled: bool = True) -> np.ndarray:
-    """adaLN vectors [layers, steps, 6H] = (shift1, scale1, gate1, shift2, scale2, gate2).
+              enabled: bool = True, streams: int = 1) -> np.ndarray:
+    """adaLN vectors [layers, steps, 6H] = (shift1, scale1, gate1, shift2, scale2, gate2);
+    streams=2 (double-stream blocks): [layers, steps, 12H], the image stream's 6H then the text
+    stream's.
 
     enabled=False gives the identity modulation (shift 0, scale 0, gate 1): plain LN + residual.
     """
-    t = np.zeros((layers, steps, 6, H), dtype=np.float32)
+    t = np.zeros((layers, steps, streams, 6, H), dtype=np.float32)
     if enabled:
         t[:] = 0.02 * g.standard_normal(t.shape, dtype=np.float32)
-    t[:, :, 2] += 1.0
-    t[:, :, 5] += 1.0
-    return _store(t.reshape(layers, steps, 6 * H), dtype)
+    t[:, :, :, 2] += 1.0
+    t[:, :, :, 5] += 1.0
+    return _store(t.reshape(layers, steps, streams * 6 * H), dtype)
 
 
 def delta_table(steps: int) -> np.ndarray:

@@ -347,3 +347,90 @@ def test_sdxl_context_and_cache_are_used():
     ctx2 = ctx.copy(); ctx2[0, 0] += 1.0
     y2, _, _ = B.masked_block_kv(x[M], M, U, Kt[U], Vt[U], w, None, 3, 64, ctx2)
     assert not np.allclose(y2, y_kv, atol=1e-6)
+
+
+# ---- NEXT-2: Flux double-stream (MM-DiT) block, reading R25 --------------------------------
+def _setup_double(seed=0, H=48, heads=3, F=80, L_img=32, L_txt=8, dtype="f32"):
+    g = synth.rng(seed)
+    w = synth.block_weights(g, H, F, dtype, kind="double")
+    x = synth.latent(g, L_img + L_txt, H, dtype)
+    m = synth.mod_table(g, 1, 1, H, dtype, streams=2)[0, 0]
+    return g, w, x, m
+
+
+def _torch_double_block(x, w, mod, heads, L_img):
+    """The double-stream block from torch library routines in float64: per-stream Linear /
+    LayerNorm, and ONE scaled_dot_product_attention over the concatenated streams."""
+    t = lambda a: torch.tensor(np.asarray(a, np.float64))
+    H = x.shape[1]
+    d = H // heads
+    m = t(mod).view(2, 6, H)
+    xs = [t(x[:L_img]), t(x[L_img:])]
+    ws = [w["img"], w["txt"]]
+    lin = lambda h, W, b: Fn.linear(h, t(W), t(b))
+    hs = [Fn.layer_norm(xs[i], (H,), eps=1e-6) * (1 + m[i, 1]) + m[i, 0] for i in range(2)]
+    qkv = [lin(hs[i], ws[i]["w_qkv"], ws[i]["b_qkv"]) for i in range(2)]
+    q, k, v = (torch.cat([qkv[0][:, j * H:(j + 1) * H], qkv[1][:, j * H:(j + 1) * H]])
+               .view(-1, heads, d).transpose(0, 1) for j in range(3))
+    a = Fn.scaled_dot_product_attention(q, k, v).transpose(0, 1).reshape(-1, H)
+    a_s = [a[:L_img], a[L_img:]]
+    out = []
+    for i in range(2):
+        x1 = xs[i] + m[i, 2] * lin(a_s[i], ws[i]["w_o"], ws[i]["b_o"])
+        h2 = Fn.layer_norm(x1, (H,), eps=1e-6) * (1 + m[i, 4]) + m[i, 3]
+        mlp = lin(Fn.gelu(lin(h2, ws[i]["w_up"], ws[i]["b_up"]), approximate="tanh"),
+                  ws[i]["w_down"], ws[i]["b_down"])
+        out.append(x1 + m[i, 5] * mlp)
+    return torch.cat(out).numpy()
+
+
+def test_double_block_vs_torch():
+    _, w, x, m = _setup_double()
+    y, K, V = B.dense_block(x, w, m, 3, L_txt=8)
+    assert np.allclose(y, _torch_double_block(x, w, m, 3, 32), rtol=0, atol=1e-10)
+
+
+def test_double_block_same_weights_is_sequential():
+    """Both streams with the same weights and modulation reduce to the sequential block."""
+    g, w, x, m = _setup_double(seed=41)
+    w["txt"] = w["img"]
+    H = x.shape[1]
+    m[6 * H:] = m[:6 * H]
+    y, _, _ = B.dense_block(x, w, m, 3, L_txt=8)
+    y_seq, _, _ = B.dense_block(x, w["img"], m[:6 * H], 3)
+    assert np.allclose(y, y_seq, rtol=0, atol=1e-12)
+
+
+def test_double_streams_use_their_own_weights():
+    """Changing the text stream's MLP changes only text rows (token-wise outside attention)."""
+    g, w, x, m = _setup_double(seed=43)
+    y, _, _ = B.dense_block(x, w, m, 3, L_txt=8)
+    w2 = {"kind": "double", "img": w["img"], "txt": dict(w["txt"])}
+    w2["txt"]["b_down"] = w["txt"]["b_down"] + 1.0
+    y2, _, _ = B.dense_block(x, w2, m, 3, L_txt=8)
+    assert np.allclose(y2[:32], y[:32], atol=1e-12)
+    assert np.allclose(y2[32:] - y[32:], np.asarray(m, np.float64).reshape(2, 6, -1)[1, 5], atol=1e-9)
+
+
+@pytest.mark.parametrize("ratio", [0.0, 0.3, 1.0])
+def test_double_masked_equals_dense_under_identical_input_cache(ratio):
+    g, w, x, m = _setup_double(seed=45, L_img=64, L_txt=8)
+    mask = synth.token_mask(synth.mask_blobs(g, 8, 8, ratio), 8)
+    M, U = build_mask_index(mask)
+    y_ref, K, V = B.dense_block(x, w, m, 3, L_txt=8)
+    y_kv, K_M, V_M = B.masked_block_kv(x[M], M, U, K[U], V[U], w, m, 3, 72, L_txt=8)
+    y_y = B.masked_block_y(x[M], M, U, x[U], w, m, 3, 72, L_txt=8)
+    assert np.allclose(y_kv, y_ref[M], rtol=0, atol=1e-12)
+    assert np.allclose(y_y, y_ref[M], rtol=0, atol=1e-12)
+    assert np.allclose(K_M, K[M], atol=1e-12) and np.allclose(V_M, V[M], atol=1e-12)
+
+
+def test_double_cache_is_actually_used():
+    g, w, x, m = _setup_double(seed=47, L_img=64, L_txt=8)
+    mask = synth.token_mask(synth.mask_random(g, 64, 0.25), 8)
+    M, U = build_mask_index(mask)
+    x_t = synth.latent(g, 72, x.shape[1], "f32")
+    _, Kt, Vt = B.dense_block(x_t, w, m, 3, L_txt=8)
+    y_kv, _, _ = B.masked_block_kv(x[M], M, U, Kt[U], Vt[U], w, m, 3, 72, L_txt=8)
+    y_ref, _, _ = B.dense_block(x, w, m, 3, L_txt=8)
+    assert not np.allclose(y_kv, y_ref[M], atol=1e-3)
