@@ -8,8 +8,15 @@ from oracle import stack as S
 
 def _setup(N=3, steps=2, H=32, heads=2, F=64, L_img=36, L_txt=4, seed=0, kind="seq"):
     g = synth.rng(seed)
-    W = synth.stack_weights(g, N, H, F, "f32", kind)
-    mods = synth.mod_table(g, N, steps, H, "f32")
+    if kind == "flux":       # double-stream blocks then a single-stream block (R25, R23)
+        W = synth.stack_weights(g, N - 1, H, F, "f32", "double") + \
+            synth.stack_weights(g, 1, H, F, "f32", "par")
+    else:
+        W = synth.stack_weights(g, N, H, F, "f32", kind, D_ctx=24)
+    mods = synth.mod_table(g, N, steps, H, "f32", streams=2 if kind == "flux" else 1)
+    if kind == "flux":       # the single-stream block reads the first 6H of the 12H row
+        mods = [[mods[l][s] if l < N - 1 else mods[l][s][:6 * H] for s in range(steps)]
+                for l in range(N)]
     x0 = synth.latent(g, L_img + L_txt, H, "f32")
     return g, W, mods, x0, synth.delta_table(steps)
 
@@ -19,15 +26,16 @@ PLANS_Y = PLANS_KV + [[1, 0, 1], [1, 1, 0], [0, 1, 0], [1, 0, 0]]
 
 
 @pytest.mark.parametrize("mode,plan", [("kv", p) for p in PLANS_KV] + [("y", p) for p in PLANS_Y])
-@pytest.mark.parametrize("kind", ["seq", "par"])
+@pytest.mark.parametrize("kind", ["seq", "par", "sdxl", "flux"])
 def test_identical_input_cache_reproduces_template(mode, plan, kind):
     """L144/L157 + L211: with the cache from the template run on the identical input, every
-    feasible plan reproduces the dense trajectory over a whole stack and several steps (both
-    block kinds)."""
+    feasible plan reproduces the dense trajectory over a whole stack and several steps (every
+    block kind; SDXL with a prompt context, Flux-like double-stream + single-stream)."""
     g, W, mods, x0, deltas = _setup(kind=kind)
-    cache, xs = S.template_run(x0, W, mods, deltas, 2, 2)
+    ctx = synth.context(g, 5, 24, "f32") if kind == "sdxl" else None
+    cache, xs = S.template_run(x0, W, mods, deltas, 2, 2, ctx=ctx, L_txt=4)
     mask = synth.token_mask(synth.mask_blobs(g, 6, 6, 0.3), 4)
-    x = S.masked_run(x0, mask, W, mods, deltas, plan, mode, cache, 2, 2)
+    x = S.masked_run(x0, mask, W, mods, deltas, plan, mode, cache, 2, 2, ctx=ctx, L_txt=4)
     assert np.allclose(x, xs[2], rtol=0, atol=1e-11)
 
 
