@@ -407,6 +407,9 @@ def main():
     ap.add_argument("--copy-method", type=int, default=None, choices=[0, 1, 2],
                     help="H2D method: 0 SM zero-copy row gather, 1 batched DMA of the unmasked row "
                          "runs (host default), 2 whole-entry DMA (HBM default)")
+    ap.add_argument("--cross-step", type=int, default=1, choices=[0, 1],
+                    help="cross-step prefetch (R26): the next step's loads start as soon as their "
+                         "slots are consumed (1, default), or the per-step pipeline of Fig. 9 (0)")
     ap.add_argument("--no-extras", action="store_true", help="skip dense / Y-mode / profile legs")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()
@@ -446,6 +449,7 @@ def main():
                               "host_hugepage": "pinned host DRAM on 2 MiB pages"}[args.tier]
     base_cfg["h2d_method"] = ["SM row gather", "batched DMA of the unmasked row runs", "DMA of whole entries"][args.copy_method]
     base_cfg["parallelism"] = f"request-parallel x{world} (Alg. 2 routing)"
+    base_cfg["cross_step_prefetch"] = bool(args.cross_step)
 
     if args.impl == "reference":
         if rank != 0:
@@ -537,7 +541,7 @@ def main():
         return F.Engine(layers, w["heads"], F.MODE_CODE[mode], F.FPS_BF16, w["L_img"], w["L_txt"],
                         max(len(reqs_dev), 1), w["steps"], deltas, the_cache, mod_table=mod,
                         slots=0, plan_policy=policy, cost_model=cm.as_engine_model(), L_ctx=L_ctx,
-                        mod_width=MODW)
+                        mod_width=MODW, cross_step=bool(args.cross_step))
 
     eng = engine(0)
     log(f"[rank {rank}] timed run")
@@ -569,7 +573,7 @@ def main():
             eng_h = F.Engine(layers, w["heads"], F.MODE_CODE[args.mode], F.FPS_BF16, w["L_img"],
                              w["L_txt"], max(len(reqs_dev), 1), w["steps"], deltas, c_h,
                              mod_table=mod, slots=0, plan_policy=3, plan=list(plan), L_ctx=L_ctx,
-                             mod_width=MODW)
+                             mod_width=MODW, cross_step=bool(args.cross_step))
             noload_ms, _ = run_engine_timed(F, eng_h, reqs_dev, K, W, stream, load_stream, rank,
                                             world)
             del eng_h
@@ -592,7 +596,8 @@ def main():
             eng_o = F.Engine(layers, w["heads"], F.MODE_CODE[md], F.FPS_BF16, w["L_img"],
                              w["L_txt"], max(len(reqs_dev), 1), w["steps"], deltas, c2,
                              mod_table=mod, slots=0, plan_policy=0,
-                             cost_model=cm2.as_engine_model(), L_ctx=L_ctx, mod_width=MODW)
+                             cost_model=cm2.as_engine_model(), L_ctx=L_ctx, mod_width=MODW,
+                             cross_step=bool(args.cross_step))
             o_ms, _ = run_engine_timed(F, eng_o, reqs_dev, K, W, stream, load_stream, rank, world)
             tag = f"{md}_mode_{['host', 'hbm', 'host_hugepage'][loc]}"
             if cmeth != default_cm(loc):

@@ -330,6 +330,17 @@ fps_status fps_dense_block_forward(const fps_block_weights* w, const fps_varlen_
 fps_status fps_plan_pipeline(const double* c_cached, const double* c_dense, const double* load,
                              int32_t N, int32_t mode, double final_load, uint8_t* use_cache,
                              double* latency);
+/* Cross-step prefetch (NEXT-2, reading R26): loads of step s+1 may start as soon as the load
+ * stream is free and step s has consumed their staging slot (one slot per cached block), so
+ * the link does not idle at step boundaries.  The per-step latency of a plan is then the
+ * long-run step time of that multi-step pipeline (mean over steps 9..16 of a 16-step
+ * simulation); the planner scans the N+1 suffix plans.  Host only. */
+fps_status fps_plan_pipeline_cross(const double* c_cached, const double* c_dense,
+                                   const double* load, int32_t N, int32_t mode,
+                                   double final_load, uint8_t* use_cache, double* latency);
+double fps_pipeline_latency_cross(const uint8_t* use_cache, const double* c_cached,
+                                  const double* c_dense, const double* load, int32_t N,
+                                  int32_t mode, double final_load);
 /* The model itself (for tests and the balancer): latency of a given plan; +inf if infeasible. */
 double fps_pipeline_latency(const uint8_t* use_cache, const double* c_cached,
                             const double* c_dense, const double* load, int32_t N, int32_t mode,
@@ -358,6 +369,10 @@ typedef struct {
   int32_t mod_width;               /* elements per d_mod_table row: 0 = 6H; 12H when any
                                       layer is FPS_BLOCK_DOUBLE (image 6H, text 6H; other
                                       blocks read the first 6H)                              */
+  int32_t cross_step;              /* 1: cross-step prefetch (R26) -- the next step's loads
+                                      start as soon as their slots are consumed, and
+                                      plan_policy 0 uses fps_plan_pipeline_cross; needs one
+                                      slot per block (slots = 0 or >= n_layers)              */
 } fps_engine_desc;
 
 typedef struct fps_engine* fps_engine_t;

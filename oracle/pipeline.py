@@ -110,3 +110,87 @@ def plan_suffix_scan(Cw, Cwo, Lm, mode, final_load=0.0, slots=None):
         if v < best:
             best, best_plan = v, p
     return best, best_plan
+
+
+def simulate_steps(use, Cw, Cwo, Lm, mode, final_load=0.0, steps=1, cross_step=False):
+    """End time of `steps` consecutive denoising steps under plan `use` (R11 per step).
+
+    cross_step=False: each step's two streams start when the previous step has ended (the
+    per-step pipeline of Fig. 9).  cross_step=True (NEXT-2 "cross-step prefetch", reading R26):
+    the load stream runs on continuously -- load j of step s starts as soon as the stream is
+    free and its staging slot has been consumed in step s-1 (one slot per load; the final Y
+    rows' slot is consumed by the step-end replenish) -- while compute still runs the steps in
+    order (step s+1 starts after step s's last block and final load, i.e. its sampler update).
+    Returns (total end time, list of per-step end times)."""
+    N = len(use)
+    if not _feasible(use, mode):
+        return math.inf, []
+    loads = [l for l in range(N) if use[l]]
+    if mode == "kv" and loads:
+        loads.append(N)
+    dur = [Lm[l] if l < N else final_load for l in loads]
+    pos = {l: j for j, l in enumerate(loads)}
+    t_load, t_comp = 0.0, 0.0
+    prev_consumed = [0.0] * len(loads)     # when step s-1 released slot j
+    ends = []
+    for s in range(steps):
+        start = t_comp
+        if not cross_step:
+            t_load = max(t_load, start)
+        load_end = []
+        for j in range(len(loads)):         # the load stream issues in order
+            st = max(t_load, prev_consumed[j] if cross_step else start)
+            t_load = st + dur[j]
+            load_end.append(t_load)
+        t = start
+        end = [0.0] * N
+        for l in range(N):
+            dep = 0.0
+            if mode == "kv" and use[l]:
+                dep = load_end[pos[l]]
+            elif mode == "y" and l > 0 and use[l - 1]:
+                dep = load_end[pos[l - 1]]
+            t = max(t, dep) + (Cw[l] if use[l] else Cwo[l])
+            end[l] = t
+        if mode == "kv" and loads:
+            t = max(t, load_end[-1])
+        if mode == "y" and N and use[N - 1]:
+            t = max(t, load_end[pos[N - 1]])
+        for j, l in enumerate(loads):       # consumers: KV block l; Y block l+1 (or the end)
+            if l == N:
+                prev_consumed[j] = t
+            elif mode == "kv":
+                prev_consumed[j] = end[l]
+            else:
+                prev_consumed[j] = end[l + 1] if l + 1 < N else t
+        t_comp = t
+        ends.append(t)
+    return t_comp, ends
+
+
+STEADY_STEPS = 16
+
+
+def steady_step_latency(use, Cw, Cwo, Lm, mode, final_load=0.0, steps=STEADY_STEPS):
+    """Long-run per-step time with cross-step prefetch (R26): the mean step time over the
+    second half of `steps` simulated steps (past the pipeline's fill transient).  At least the
+    busier stream's total, max(sum of block times, sum of load times); more when a slot's
+    reuse cycle (its load in step s+1 waits for its consumer in step s) binds."""
+    if not _feasible(use, mode):
+        return math.inf
+    _, ends = simulate_steps(use, Cw, Cwo, Lm, mode, final_load, steps, cross_step=True)
+    h = steps // 2
+    return (ends[-1] - ends[h - 1]) / (steps - h)
+
+
+def plan_steady_suffix(Cw, Cwo, Lm, mode, final_load=0.0):
+    """Cross-step planner (R26): the suffix plan minimising steady_step_latency; ties -> fewer
+    cached blocks."""
+    N = len(Cw)
+    best, best_plan = math.inf, None
+    for k in range(N + 1):
+        p = [0] * (N - k) + [1] * k
+        v = steady_step_latency(p, Cw, Cwo, Lm, mode, final_load)
+        if v < best:
+            best, best_plan = v, p
+    return best, best_plan

@@ -249,22 +249,24 @@ def linear(a, w, bias=None, act=0, out=None, stream=None):
 
 
 # ---------------------------------------------------------------------------------------
-def plan_pipeline(c_cached, c_dense, load, mode, final_load=0.0):
-    """Alg. 1 (host, in the library). Returns (use_cache list, latency)."""
+def plan_pipeline(c_cached, c_dense, load, mode, final_load=0.0, cross_step=False):
+    """Alg. 1 (host, in the library). Returns (use_cache list, latency).  cross_step: the
+    cross-step prefetch planner (R26)."""
     N = len(c_cached)
     arr = lambda v: (C.c_double * N)(*map(float, v))
     use = (C.c_uint8 * max(N, 1))()
     lat = C.c_double()
-    _lib.fps_plan_pipeline(arr(c_cached), arr(c_dense), arr(load), N, mode, float(final_load),
-                           use, C.byref(lat))
+    f = _lib.fps_plan_pipeline_cross if cross_step else _lib.fps_plan_pipeline
+    f(arr(c_cached), arr(c_dense), arr(load), N, mode, float(final_load), use, C.byref(lat))
     return [int(use[i]) for i in range(N)], lat.value
 
 
-def pipeline_latency(use, c_cached, c_dense, load, mode, final_load=0.0):
+def pipeline_latency(use, c_cached, c_dense, load, mode, final_load=0.0, cross_step=False):
     N = len(use)
     arr = lambda v: (C.c_double * N)(*map(float, v))
-    return _lib.fps_pipeline_latency((C.c_uint8 * max(N, 1))(*use), arr(c_cached), arr(c_dense),
-                                     arr(load), N, mode, float(final_load))
+    f = _lib.fps_pipeline_latency_cross if cross_step else _lib.fps_pipeline_latency
+    return f((C.c_uint8 * max(N, 1))(*use), arr(c_cached), arr(c_dense), arr(load), N, mode,
+             float(final_load))
 
 
 class Cache:
@@ -315,7 +317,7 @@ class Engine:
 
     def __init__(self, layers, heads, mode, dtype, L_img, L_txt, max_batch, n_steps, deltas,
                  cache: Cache, mod_table=None, slots=0, plan_policy=0, plan=None,
-                 cost_model=(0.0, 0.0, 0.0, 0.0), L_ctx=0, mod_width=0):
+                 cost_model=(0.0, 0.0, 0.0, 0.0), L_ctx=0, mod_width=0, cross_step=False):
         self.layers = layers                      # list[BlockWeights] (keeps tensors alive)
         self._w = (fps_block_weights * len(layers))(*[l.c for l in layers])
         self._deltas = (C.c_float * n_steps)(*map(float, deltas))
@@ -328,7 +330,7 @@ class Engine:
                             C.cast(self._deltas, C.c_void_p), cache.h, slots, plan_policy,
                             C.cast(self._plan, C.c_void_p), (C.c_double * 4)(*cost_model),
                             L_ctx, max((getattr(l, "D_ctx", 0) for l in layers), default=0),
-                            mod_width)
+                            mod_width, int(cross_step))
         self.desc = d
         h = C.c_void_p()
         _lib.fps_engine_create(C.byref(d), C.byref(h))

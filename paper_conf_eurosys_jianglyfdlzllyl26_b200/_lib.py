@@ -63,7 +63,8 @@ class fps_engine_desc(C.Structure):
                 ("mode", i32), ("L_img", i32), ("L_txt", i32), ("max_batch", i32),
                 ("n_steps", i32), ("layers", vp), ("d_mod_table", vp), ("h_deltas", vp),
                 ("cache", vp), ("slots", i32), ("plan_policy", i32), ("h_plan", vp),
-                ("cost_model", dbl * 4), ("L_ctx", i32), ("D_ctx", i32), ("mod_width", i32)]
+                ("cost_model", dbl * 4), ("L_ctx", i32), ("D_ctx", i32), ("mod_width", i32),
+                ("cross_step", i32)]
 
 
 class fps_request(C.Structure):
@@ -104,6 +105,8 @@ _SIGS = [
      [C.POINTER(fps_block_weights), C.POINTER(fps_varlen_batch), vp, vp, vp, vp, sz, vp], True),
     ("fps_plan_pipeline", C.c_int, [P_dbl, P_dbl, P_dbl, i32, i32, dbl, P_u8, P_dbl], True),
     ("fps_pipeline_latency", dbl, [P_u8, P_dbl, P_dbl, P_dbl, i32, i32, dbl], False),
+    ("fps_plan_pipeline_cross", C.c_int, [P_dbl, P_dbl, P_dbl, i32, i32, dbl, P_u8, P_dbl], True),
+    ("fps_pipeline_latency_cross", dbl, [P_u8, P_dbl, P_dbl, P_dbl, i32, i32, dbl], False),
     ("fps_engine_create", C.c_int, [C.POINTER(fps_engine_desc), C.POINTER(vp)], True),
     ("fps_engine_destroy", C.c_int, [vp], True),
     ("fps_run_batch", C.c_int, [vp, C.POINTER(fps_request), i32, i32, vp, vp], True),

@@ -43,6 +43,11 @@ struct fps_engine {
   bool has_double = false;
   int MW = 0;                   // modulation elements per request and block
   int32_t *d_sm = nullptr, *h_sm = nullptr;
+  // cross-step prefetch (R26): loads of the previous step of the same batch, and the event
+  // after which the final-Y slot is free again
+  bool cross = false;
+  int prev_ring = 0;
+  cudaEvent_t final_consumed = nullptr;
   float* d_delta = nullptr;
   // pinned host staging
   int32_t* h_meta = nullptr;
@@ -78,6 +83,7 @@ static void free_engine(fps_engine* e) {
   for (auto ev : e->ready) if (ev) cudaEventDestroy(ev);
   for (auto ev : e->consumed) if (ev) cudaEventDestroy(ev);
   if (e->step_start) cudaEventDestroy(e->step_start);
+  if (e->final_consumed) cudaEventDestroy(e->final_consumed);
   if (e->admit_done) cudaEventDestroy(e->admit_done);
   delete e;
 }
@@ -159,6 +165,7 @@ fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out) {
     D = (int)std::max<size_t>(2, std::min<size_t>(d.n_layers, budget / std::max<size_t>(slot_bytes, 1)));
   }
   e->D = std::min(D, d.n_layers);
+  e->cross = d.cross_step != 0 && e->D >= d.n_layers;   // needs one slot per block
   cudaError_t err = cudaSuccess;
   auto dmal = [&](char** p, size_t bytes) {
     if (err == cudaSuccess) err = cudaMalloc((void**)p, std::max<size_t>(bytes, 256));
@@ -215,6 +222,7 @@ fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out) {
     if (err == cudaSuccess) err = cudaEventCreateWithFlags(&e->consumed[i], cudaEventDisableTiming);
   }
   if (err == cudaSuccess) err = cudaEventCreateWithFlags(&e->step_start, cudaEventDisableTiming);
+  if (err == cudaSuccess) err = cudaEventCreateWithFlags(&e->final_consumed, cudaEventDisableTiming);
   if (err == cudaSuccess) err = cudaEventCreateWithFlags(&e->admit_done, cudaEventDisableTiming);
   if (err != cudaSuccess) {
     cudaGetLastError();
@@ -404,13 +412,17 @@ static void make_plan(fps_engine* e, const Batch& B) {
   for (int l = 0; l < N; ++l) Lm[l] = by > 0 ? c * by + ec : 0.0;
   const double fin = byf > 0 ? c * byf + ec : 0.0;
   if (e->d.plan_policy == 0) {
-    fps_plan_pipeline(Cw.data(), Cwo.data(), Lm.data(), N, e->d.mode, fin, e->last_plan.data(),
-                      &e->last_latency);
+    if (e->cross)
+      fps_plan_pipeline_cross(Cw.data(), Cwo.data(), Lm.data(), N, e->d.mode, fin,
+                              e->last_plan.data(), &e->last_latency);
+    else
+      fps_plan_pipeline(Cw.data(), Cwo.data(), Lm.data(), N, e->d.mode, fin, e->last_plan.data(),
+                        &e->last_latency);
   } else {
     for (int l = 0; l < N; ++l)
       e->last_plan[l] = e->d.plan_policy == 1 ? 1 : e->d.plan_policy == 2 ? 0 : e->fixed_plan[l];
-    e->last_latency = fps_pipeline_latency(e->last_plan.data(), Cw.data(), Cwo.data(), Lm.data(),
-                                           N, e->d.mode, fin);
+    e->last_latency = (e->cross ? fps_pipeline_latency_cross : fps_pipeline_latency)(
+        e->last_plan.data(), Cw.data(), Cwo.data(), Lm.data(), N, e->d.mode, fin);
   }
 }
 
@@ -447,7 +459,9 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
   bool final_issued = false;
   std::vector<fps_prefetch_item> items(n);
   FPS_CUDA_TRY(cudaEventRecord(e->step_start, cs));
-  FPS_CUDA_TRY(stream_wait(ls, e->step_start, 0));
+  // per-step pipeline: this step's loads start with the step; cross-step prefetch (R26): a
+  // load waits only for the previous step's consumer of its slot (below)
+  if (!e->cross) FPS_CUDA_TRY(stream_wait(ls, e->step_start, 0));
   auto issue = [&](int block, char* dst, size_t row_bytes, cudaEvent_t ev) -> fps_status {
     for (int i = 0; i < n; ++i) {
       const fps_request& r = reqs[B.idx[i]];
@@ -466,10 +480,13 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
   auto try_issue = [&]() -> fps_status {
     while (issued < n_ring && (issued < e->D || consumed_rec[issued - e->D])) {
       if (issued >= e->D) FPS_CUDA_TRY(stream_wait(ls, e->consumed[issued - e->D], 0));
+      // the previous step's consumer of this slot (recorded before this step re-records it)
+      if (e->cross && issued < e->prev_ring) FPS_CUDA_TRY(stream_wait(ls, e->consumed[issued], 0));
       FPS_TRY(issue(loads[issued], e->slots[issued % e->D], e->row_w, e->ready[issued]));
       ++issued;
     }
     if (final_load && issued == n_ring && !final_issued) {
+      if (e->cross && e->prev_ring > 0) FPS_CUDA_TRY(stream_wait(ls, e->final_consumed, 0));
       FPS_TRY(issue(N, e->final_slot, e->row_h, e->ready[n_ring]));
       final_issued = true;
     }
@@ -604,12 +621,17 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
     const char* src = kv ? e->final_slot : e->slots[pos[N - 1] % e->D];
     FPS_CUDA_TRY(stream_wait(cs, e->ready[j], 0));
     FPS_TRY(launch_copy_rows(src, B.u_row, B.u_row, B.tu, (int)e->row_h, e->y_full, cs));
+    if (kv) FPS_CUDA_TRY(cudaEventRecord(e->final_consumed, cs));
+    else FPS_TRY(consume(j));          // Y-mode: block N-1's slot is read by the replenish
     y_src = e->y_full;
   }
   FPS_TRY(launch_euler(e->d.dtype, e->x_full, y_src, B.tk, H, B.cu_k, n, e->d_delta, cs));
-  // the load stream must not run ahead into the next step's slots before this step is done
-  FPS_CUDA_TRY(cudaEventRecord(e->step_start, cs));
-  FPS_CUDA_TRY(stream_wait(ls, e->step_start, 0));
+  e->prev_ring = n_ring;
+  if (!e->cross) {
+    // the load stream must not run ahead into the next step's slots before this step is done
+    FPS_CUDA_TRY(cudaEventRecord(e->step_start, cs));
+    FPS_CUDA_TRY(stream_wait(ls, e->step_start, 0));
+  }
   return FPS_OK;
 }
 
@@ -638,6 +660,10 @@ extern "C" fps_status fps_run_batch(fps_engine_t e, fps_request* reqs, int32_t n
     }
     if (live.empty()) break;
     Batch B;
+    // a new batch: its index arrays and slots are rewritten, so the load stream drains first
+    FPS_CUDA_TRY(cudaEventRecord(e->final_consumed, ls));
+    FPS_CUDA_TRY(stream_wait(cs, e->final_consumed, 0));
+    e->prev_ring = 0;
     FPS_TRY(admit(e, reqs, live, B, cs));
     // load each request's latent into the contiguous batch buffer
     for (int i = 0; i < B.n; ++i)

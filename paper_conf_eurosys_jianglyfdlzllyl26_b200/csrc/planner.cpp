@@ -137,9 +137,93 @@ double plan_y(const double* Cw, const double* Cwo, const double* Lm, int N, uint
   return best;
 }
 
+// Cross-step prefetch (reading R26): the load stream never waits for the step boundary --
+// load j of step s+1 starts when the stream is free and step s has consumed its slot (one slot
+// per load); compute runs the steps in order.  Steady per-step time = mean step time over the
+// second half of kSteadySteps simulated steps.
+constexpr int kSteadySteps = 16;
+
+double steady_of(const uint8_t* use, const double* Cw, const double* Cwo, const double* Lm,
+                 int N, int mode, double final_load) {
+  if (mode == FPS_MODE_KV) {
+    bool seen = false;
+    for (int l = 0; l < N; ++l) {
+      if (use[l]) seen = true;
+      else if (seen) return std::numeric_limits<double>::infinity();
+    }
+  }
+  std::vector<int> blk;                       // block of each load; N = final Y rows (KV)
+  std::vector<int> slot_of(N, -1);
+  for (int l = 0; l < N; ++l)
+    if (use[l]) {
+      slot_of[l] = (int)blk.size();
+      blk.push_back(l);
+    }
+  if (mode == FPS_MODE_KV && !blk.empty()) blk.push_back(N);
+  const int nl = (int)blk.size();
+  std::vector<double> freed(nl, 0.0), ready(nl, 0.0), end(N, 0.0);
+  double t_load = 0.0, t_comp = 0.0, half_end = 0.0;
+  for (int s = 0; s < kSteadySteps; ++s) {
+    for (int j = 0; j < nl; ++j) {
+      t_load = std::max(t_load, freed[j]) + (blk[j] < N ? Lm[blk[j]] : final_load);
+      ready[j] = t_load;
+    }
+    double t = t_comp;
+    for (int l = 0; l < N; ++l) {
+      double dep = 0.0;
+      if (mode == FPS_MODE_KV && use[l]) dep = ready[slot_of[l]];
+      if (mode == FPS_MODE_Y && l > 0 && use[l - 1]) dep = ready[slot_of[l - 1]];
+      t = std::max(t, dep) + (use[l] ? Cw[l] : Cwo[l]);
+      end[l] = t;
+    }
+    if (nl > 0) {
+      if (mode == FPS_MODE_KV) t = std::max(t, ready[nl - 1]);
+      if (mode == FPS_MODE_Y && use[N - 1]) t = std::max(t, ready[slot_of[N - 1]]);
+    }
+    for (int j = 0; j < nl; ++j) {
+      const int l = blk[j];
+      freed[j] = l == N ? t : mode == FPS_MODE_KV ? end[l] : (l + 1 < N ? end[l + 1] : t);
+    }
+    t_comp = t;
+    if (s == kSteadySteps / 2 - 1) half_end = t;
+  }
+  return (t_comp - half_end) / (kSteadySteps - kSteadySteps / 2);
+}
+
 }  // namespace
 
 extern "C" {
+
+double fps_pipeline_latency_cross(const uint8_t* use_cache, const double* c_cached,
+                                  const double* c_dense, const double* load, int32_t N,
+                                  int32_t mode, double final_load) {
+  if (N < 0 || (N > 0 && (!use_cache || !c_cached || !c_dense || !load)))
+    return std::numeric_limits<double>::quiet_NaN();
+  return N == 0 ? 0.0 : steady_of(use_cache, c_cached, c_dense, load, N, mode, final_load);
+}
+
+fps_status fps_plan_pipeline_cross(const double* c_cached, const double* c_dense,
+                                   const double* load, int32_t N, int32_t mode,
+                                   double final_load, uint8_t* use_cache, double* latency) {
+  if (N < 0 || !latency || (N > 0 && (!c_cached || !c_dense || !load || !use_cache)))
+    return FPS_EINVAL;
+  if (mode != FPS_MODE_KV && mode != FPS_MODE_Y) return FPS_EINVAL;
+  std::vector<uint8_t> p(N);
+  double best = std::numeric_limits<double>::infinity();
+  int best_k = 0;
+  for (int k = 0; k <= N; ++k) {                 // suffix plans, ties -> fewer cached blocks
+    for (int l = 0; l < N; ++l) p[l] = l >= N - k ? 1 : 0;
+    const double v = N == 0 ? 0.0 : steady_of(p.data(), c_cached, c_dense, load, N, mode, final_load);
+    if (v < best - 1e-12 * std::max(1.0, std::fabs(best)) || std::isinf(best)) {
+      best = v;
+      best_k = k;
+    }
+  }
+  for (int l = 0; l < N; ++l) use_cache[l] = l >= N - best_k ? 1 : 0;
+  *latency = best;
+  return FPS_OK;
+}
+
 
 double fps_pipeline_latency(const uint8_t* use_cache, const double* c_cached,
                             const double* c_dense, const double* load, int32_t N, int32_t mode,

@@ -20,7 +20,7 @@ def F():
 
 def _setup(F, mode, dtype, plan_policy, plan=None, N=3, steps=3, H=256, heads=2, Fd=512,
            L_img=256, L_txt=16, n_req=3, slots=0, copy_method=0, seed=5000, location=0,
-           kind="seq"):
+           kind="seq", cross_step=False):
     g = synth.rng(seed)
     W = synth.stack_weights(g, N, H, Fd, dtype, kind)
     mods = synth.mod_table(g, N, steps, H, dtype)
@@ -49,7 +49,7 @@ def _setup(F, mode, dtype, plan_policy, plan=None, N=3, steps=3, H=256, heads=2,
     layers = [F.BlockWeights(w, heads, dt) for w in W]
     eng = F.Engine(layers, heads, m, dt, L_img, L_txt, max_batch=4, n_steps=steps, deltas=deltas,
                    cache=cache, mod_table=to_dev(mods, dtype), slots=slots,
-                   plan_policy=plan_policy, plan=plan)
+                   plan_policy=plan_policy, plan=plan, cross_step=cross_step)
     reqs = []
     ratios = [0.1, 0.45, 0.25, 0.6][:n_req]
     for i in range(n_req):
@@ -327,3 +327,25 @@ def test_full_scale_stack_identical_input_invariant(F, mode):
     assert torch.isfinite(outs[0].float()).all()
     assert torch.equal(outs[0].view(torch.int16), outs[1].view(torch.int16)), \
         f"{mode}: max diff {(outs[0].float() - outs[1].float()).abs().max().item()}"
+
+
+@pytest.mark.parametrize("mode,plan,copy_method", [("kv", [0, 1, 1], 1), ("y", [1, 0, 1], 0),
+                                                   ("kv", [1, 1, 1], 2), ("y", [1, 1, 1], 1)])
+def test_cross_step_prefetch_matches_oracle_and_per_step_bits(F, mode, plan, copy_method):
+    """Cross-step prefetch (R26) only moves loads earlier: over 2 steps the latents match the
+    oracle and are bit-identical to the per-step pipeline's."""
+    outs = []
+    for cross in (False, True):
+        W, mods, deltas, cache_np, eng, reqs = _setup(F, mode, "bf16", 3, plan, steps=4,
+                                                      copy_method=copy_method, cross_step=cross)
+        for r in reqs:
+            r["step0"] = r["step"]
+        eng.run_batch(reqs, 2)
+        torch.cuda.synchronize()
+        outs.append([r["x"].clone() for r in reqs])
+        ref = _oracle(W, mods, deltas, cache_np, reqs, plan, mode, 2, 2)
+        for r, x in zip(reqs, ref):
+            check_close(to_np(r["x"]), x, stack_tol("bf16", 3),
+                        f"cross={cross} {mode} plan={plan}")
+    for a, b in zip(*outs):
+        assert torch.equal(a, b)

@@ -102,3 +102,25 @@ def test_planner_large_stack_properties():
             for _ in range(200):
                 use = [int(v) for v in g.integers(0, 2, N)]
                 assert lat <= P.simulate(use, Cw, Cwo, Lm, mode, fin) + 1e-9
+
+
+@pytest.mark.parametrize("mode", ["kv", "y"])
+def test_cross_step_planner_matches_oracle(mode):
+    """Cross-step prefetch (R26): the library's multi-step pipeline latency and its suffix
+    planner vs the oracle's multi-step simulator and exhaustive suffix scan."""
+    g = synth.rng(14)
+    m = fps.MODE_CODE[mode]
+    for _ in range(100):
+        N = int(g.integers(1, 14))
+        Cw, Cwo, Lm, fin = _rand_costs(g, N)
+        use = [0] * int(g.integers(0, N + 1))
+        use += [1] * (N - len(use))
+        if mode == "y" and g.uniform() < 0.5:
+            use = [int(v) for v in g.integers(0, 2, N)]
+        ref = P.steady_step_latency(use, Cw, Cwo, Lm, mode, fin)
+        got = fps.pipeline_latency(use, Cw, Cwo, Lm, m, fin, cross_step=True)
+        assert got == pytest.approx(ref, rel=1e-9)
+        best, bplan = P.plan_steady_suffix(Cw, Cwo, Lm, mode, fin)
+        plan, lat = fps.plan_pipeline(Cw, Cwo, Lm, m, fin, cross_step=True)
+        assert lat == pytest.approx(best, rel=1e-9)
+        assert P.steady_step_latency(plan, Cw, Cwo, Lm, mode, fin) == pytest.approx(best, rel=1e-9)

@@ -160,3 +160,69 @@ def test_sdxl_flops_match_matmul_shapes():
         assert count["f"] == C.block_flops("y", len(M), L, H, F, "sdxl", Lc) + cf
     finally:
         B.linear, B.attention = orig
+
+
+def test_multistep_without_cross_step_is_steps_times_alg1_model():
+    """cross_step=False: consecutive steps are independent copies of the pinned R11 model."""
+    g = synth.rng(61)
+    for mode in ("kv", "y"):
+        for _ in range(30):
+            N = int(g.integers(1, 9))
+            Cw, Cwo, Lm = g.uniform(0.1, 1, N), g.uniform(1, 2, N), g.uniform(0, 2, N)
+            fin = float(g.uniform(0, 0.5))
+            plan = [0] * int(g.integers(0, N + 1))
+            plan += [1] * (N - len(plan))
+            one = P.simulate(plan, Cw, Cwo, Lm, mode, fin)
+            tot, ends = P.simulate_steps(plan, Cw, Cwo, Lm, mode, fin, steps=4)
+            assert tot == pytest.approx(4 * one, rel=1e-12)
+            assert ends == pytest.approx([one * (s + 1) for s in range(4)], rel=1e-12)
+
+
+def test_cross_step_never_slower_and_converges_to_busier_stream():
+    """cross_step=True: never slower than per-step pipelines, and the long-run step time is
+    the busier stream's total (closed form) -- the link never idles when load-bound and the
+    compute stream never waits when compute-bound."""
+    g = synth.rng(62)
+    for mode in ("kv", "y"):
+        for _ in range(40):
+            N = int(g.integers(2, 10))
+            Cw, Cwo, Lm = g.uniform(0.1, 1, N), g.uniform(1, 2, N), g.uniform(0, 2.5, N)
+            fin = float(g.uniform(0, 0.5))
+            k = int(g.integers(1, N + 1))
+            plan = [0] * (N - k) + [1] * k
+            base, _ = P.simulate_steps(plan, Cw, Cwo, Lm, mode, fin, steps=40)
+            tot, ends = P.simulate_steps(plan, Cw, Cwo, Lm, mode, fin, steps=40, cross_step=True)
+            assert tot <= base + 1e-9
+            steady = P.steady_step_latency(plan, Cw, Cwo, Lm, mode, fin)
+            comp = sum(Cw[l] if plan[l] else Cwo[l] for l in range(N))
+            load = sum(Lm[l] for l in range(N) if plan[l]) + (fin if mode == "kv" else 0.0)
+            assert max(comp, load) - 1e-9 <= steady <= P.simulate(plan, Cw, Cwo, Lm, mode, fin) + 1e-9
+            # no load time at all: the compute stream alone sets the pace (closed form)
+            z = P.steady_step_latency(plan, Cw, Cwo, np.zeros(N), mode, 0.0)
+            assert z == pytest.approx(comp, rel=1e-12)
+
+
+def test_cross_step_busy_link_closed_form():
+    """Load-bound with a dense prefix long enough to cover every slot's reuse cycle: the link
+    never idles, one step = all loads + the final load (hand-derived)."""
+    N = 6
+    Cw, Cwo = [0.1] * N, [1.0] * N
+    Lm = [2.0] * N
+    plan = [0, 0, 0, 1, 1, 1]            # prefix compute 3.0, loads 6.0 + final 0.5
+    assert P.steady_step_latency(plan, Cw, Cwo, Lm, "kv", 0.5) == pytest.approx(6.5)
+    # all cached, Cw 0.5, loads 0.6: per step block l waits for load l -> 6 x 0.6 + 0.5 = 4.1;
+    # across steps the loads of step s+1 run under step s's compute -> the link's 3.6
+    Cw2, Lm2 = [0.5] * N, [0.6] * N
+    assert P.simulate([1] * N, Cw2, Cwo, Lm2, "kv", 0.0) == pytest.approx(4.1)
+    assert P.steady_step_latency([1] * N, Cw2, Cwo, Lm2, "kv", 0.0) == pytest.approx(3.6)
+
+
+def test_steady_planner_is_exhaustive_optimum_over_suffixes():
+    g = synth.rng(63)
+    for _ in range(50):
+        N = int(g.integers(1, 12))
+        Cw, Cwo, Lm = g.uniform(0.1, 1, N), g.uniform(1, 2, N), g.uniform(0, 2, N)
+        best, plan = P.plan_steady_suffix(Cw, Cwo, Lm, "kv", 0.2)
+        for k in range(N + 1):
+            p = [0] * (N - k) + [1] * k
+            assert best <= P.steady_step_latency(p, Cw, Cwo, Lm, "kv", 0.2) + 1e-12
