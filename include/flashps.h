@@ -55,7 +55,10 @@ int32_t fps_device_ok(void);
  * shared memory, = 3 the two-tile kernel with P in TMEM and a correction warpgroup (the default);
  * bit 6 = launch without programmatic dependent launch (PDL is on by default);
  * bit 7 = HBM-arena whole-entry prefetch by driver device-to-device memcpy instead of the
- * library copy kernel (experiments only: see cache.cu). */
+ * library copy kernel (experiments only: see cache.cu);
+ * bits 8-10 = S > 0 forces the split-KV factor of the tensor-core attention inside block calls
+ * (0 = chosen by wave efficiency; S is applied only when the block workspace holds the S
+ * partial outputs). */
 int64_t fps_launch_count(void);
 void fps_set_disable_tc(int32_t flags);
 /* Per-kernel-class timing for the bench: when enabled (this also clears old records) every

@@ -95,14 +95,15 @@ fps_status launch_gemm(int dtype, const void* A, const void* B, int M, int N, in
 fps_status launch_attention(int dtype, const void* q, const void* kv, void* o, int heads,
                             int head_dim, const int32_t* d_cu_q, const int32_t* d_cu_k,
                             const int32_t* h_cu_q, const int32_t* h_cu_k, int n_req, int total_q,
-                            int max_q, int max_k, cudaStream_t s, int ldo) {
+                            int max_q, int max_k, cudaStream_t s, int ldo,
+                            const AttnScratch* sc) {
   (void)max_k;
   if (total_q <= 0) return FPS_OK;
   prof::begin(s);
   fps_status st;
   if (!(g_disable_tc & 2) && attention_tc_supported(dtype, head_dim) && h_cu_q && h_cu_k)
     st = launch_attention_tc(q, kv, o, heads, head_dim, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s,
-                             ldo);
+                             ldo, sc);
   else
     st = launch_attention_simt(dtype, q, kv, o, heads, head_dim, d_cu_q, d_cu_k, n_req, total_q, s,
                                ldo);
@@ -144,6 +145,20 @@ static size_t ws_layout(int H, int F, int dtype, int max_q, int max_u, char* bas
   char* x2 = take((size_t)max_q * H * 4);              // SDXL block: after cross-attention (fp32)
   if (ws) *ws = BlockWs{h, q, ao, x1, h2, u, hu, x2};
   return off;
+}
+
+// Split-KV attention scratch inside the block workspace: buffers that are dead while the
+// attention runs -- the LN output h (consumed by the QKV GEMM) for the statistics, and the MLP
+// hidden u (written after the attention) or, for the parallel block whose u holds GELU(Z)
+// already, the x1 buffer for the partial outputs.
+static AttnScratch attn_scratch(const BlockWs& ws, int H, int F, int dtype, int max_q, bool par) {
+  const size_t e = elt_size(dtype);
+  AttnScratch sc{};
+  sc.ml = ws.h;
+  sc.ml_bytes = (size_t)max_q * H * e;
+  sc.part = par ? ws.x1 : ws.u;
+  sc.part_bytes = par ? (size_t)max_q * H * 4 : (size_t)max_q * F * e;
+  return sc;
 }
 
 static fps_status check_weights(const fps_block_weights* w) {
@@ -278,8 +293,9 @@ static fps_status double_block_forward(const fps_block_weights* w, const fps_var
   if (tq == 0) return FPS_OK;
   // a6: joint attention of both streams' queries over the merged keys
   if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
+  const AttnScratch sc = attn_scratch(ws, H, F, dt, tq, false);
   FPS_TRY(launch_attention(dt, ws.q, kv, ws.ao, w->heads, w->head_dim, b->d_cu_q, b->d_cu_k,
-                           b->h_cu_q, b->h_cu_k, b->n_req, tq, b->max_q, b->max_k, s));
+                           b->h_cu_q, b->h_cu_k, b->n_req, tq, b->max_q, b->max_k, s, 0, &sc));
   FPS_TRY(launch_copy_rows(ws.ao, perm, nullptr, tq, (int)rowb, ao_sm, s));
   for (int st = 0; st < 2; ++st) {   // a7 per stream: x1 = x + gate1 (A Wo^T + bo)
     Epilogue ep{};
@@ -383,8 +399,10 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
     // parallel block (reading R23): ws.ao..ws.u hold cat = [A | GELU(Z)], [tq, H+F]
     char* cat = ws.ao;
     if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
+    const AttnScratch sc = attn_scratch(ws, H, F, dt, tq, true);
     FPS_TRY(launch_attention(dt, ws.q, kv, cat, w->heads, w->head_dim, b->d_cu_q, b->d_cu_k,
-                             b->h_cu_q, b->h_cu_k, b->n_req, tq, b->max_q, b->max_k, s, H + F));
+                             b->h_cu_q, b->h_cu_k, b->n_req, tq, b->max_q, b->max_k, s, H + F,
+                             &sc));
     Epilogue ep{};
     ep.bias = w->b_down;
     ep.resid = x_act; ep.ld_resid = H;
@@ -394,8 +412,9 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
   }
   // a6: queries from active rows only, keys = merged fresh + cached rows (L159)
   if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
+  const AttnScratch sc = attn_scratch(ws, H, F, dt, tq, false);
   FPS_TRY(launch_attention(dt, ws.q, kv, ws.ao, w->heads, w->head_dim, b->d_cu_q, b->d_cu_k,
-                           b->h_cu_q, b->h_cu_k, b->n_req, tq, b->max_q, b->max_k, s));
+                           b->h_cu_q, b->h_cu_k, b->n_req, tq, b->max_q, b->max_k, s, 0, &sc));
   {  // a7: x1 = x + gate1 (A Wo^T + bo)
     Epilogue ep{};
     ep.bias = w->b_o;
@@ -418,7 +437,8 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
     int max_c = 0;
     for (int r = 0; r < b->n_req; ++r) max_c = std::max(max_c, b->h_cu_ctx[r + 1] - b->h_cu_ctx[r]);
     FPS_TRY(launch_attention(dt, ws.q, b->d_ctx_kv, ws.ao, w->heads, w->head_dim, b->d_cu_q,
-                             b->d_cu_ctx, b->h_cu_q, b->h_cu_ctx, b->n_req, tq, b->max_q, max_c, s));
+                             b->d_cu_ctx, b->h_cu_q, b->h_cu_ctx, b->n_req, tq, b->max_q, max_c, s,
+                             0, &sc));
     {
       Epilogue ep{};
       ep.bias = w->b_o2;
@@ -518,6 +538,7 @@ void fps_set_disable_tc(int32_t flags) {
   fps::g_attn_force = (flags >> 4) & 3;
   fps::g_pdl = (flags & 64) ? 0 : 1;
   fps::g_d2d_kernel = (flags & 128) ? 0 : 1;
+  fps::g_attn_split = (flags >> 8) & 7;
 }
 
 fps_status fps_build_mask_index(const uint8_t* d_masks, const int32_t* d_offsets, int32_t n_req,

@@ -12,6 +12,8 @@
 //              by more than 2^8, FA4-style), P as bf16 into one of two smem P buffers in the UMMA
 //              K-major SW128 layout; the exponentials of tile j are computed while PV_{j-1} still
 //              runs; final O / l from TMEM to global.
+#include <algorithm>
+
 #include "kernels.h"
 #include "tc_util.cuh"
 
@@ -65,9 +67,13 @@ __global__ void __launch_bounds__(256, 1)
   }
   const int q0 = __ldg(cu_q + r) + qt * 128;
   const int n_rows = min(128, __ldg(cu_q + r + 1) - q0);
-  const int k0 = __ldg(cu_k + r);
-  const int Lr = __ldg(cu_k + r + 1) - k0;
-  const int nk = (Lr + 127) >> 7;
+  const int Lr = __ldg(cu_k + r + 1) - __ldg(cu_k + r);
+  const int nk_all = (Lr + 127) >> 7;
+  const int nsplit = gridDim.z, split = blockIdx.z;
+  const int kb = (int)(((long long)nk_all * split) / nsplit);       // first key tile of this CTA
+  const int nk = (int)(((long long)nk_all * (split + 1)) / nsplit) - kb;
+  const int k0 = __ldg(cu_k + r) + kb * 128;                         // its first key row
+  const int Lr_rem = Lr - kb * 128;                                  // keys from k0 to the end
 
   if (threadIdx.x == 0) {
     tc::mbar_init(bar_q, 1);
@@ -340,9 +346,13 @@ __global__ void __launch_bounds__(384, 1)
   const bool hasB = 2 * qp + 1 < ntile;
   const int q_end = __ldg(cu_q + r + 1);
   const int q0 = __ldg(cu_q + r) + qp * 256;
-  const int k0 = __ldg(cu_k + r);
-  const int Lr = __ldg(cu_k + r + 1) - k0;
-  const int nk = (Lr + 127) >> 7;
+  const int Lr = __ldg(cu_k + r + 1) - __ldg(cu_k + r);
+  const int nk_all = (Lr + 127) >> 7;
+  const int nsplit = gridDim.z, split = blockIdx.z;
+  const int kb = (int)(((long long)nk_all * split) / nsplit);       // first key tile of this CTA
+  const int nk = (int)(((long long)nk_all * (split + 1)) / nsplit) - kb;
+  const int k0 = __ldg(cu_k + r) + kb * 128;                         // its first key row
+  const int Lr_rem = Lr - kb * 128;                                  // keys from k0 to the end
 
   if (threadIdx.x == 0) {
     tc::mbar_init(bar_q, 1);
@@ -658,11 +668,16 @@ struct Attn3Cfg {
   static constexpr int TMEM_COLS = 512;
 };
 
+// Split-KV (gridDim.z = S > 1): CTA z covers key tiles [nk*z/S, nk*(z+1)/S) of its request,
+// writes its own normalised output O_z (bf16, [total_q, H] at Opart + z * part_stride) and its
+// (running max, row sum) pair to ML[z][row][head]; attn_combine_kernel merges the S partials.
 template <int D>
 __global__ void __launch_bounds__(512, 1)
     attn_tc3_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmKV,
                     __nv_bfloat16* __restrict__ O, const int32_t* __restrict__ cu_q,
-                    const int32_t* __restrict__ cu_k, int n_req, int heads, float scale_log2, int ldo) {
+                    const int32_t* __restrict__ cu_k, int n_req, int heads, float scale_log2, int ldo,
+                    __nv_bfloat16* __restrict__ Opart, float2* __restrict__ ML, long long part_stride,
+                    int total_q) {
   using Cfg = Attn3Cfg<D>;
   constexpr int CHUNK = 128 * 128;
   extern __shared__ uint8_t smem_raw[];
@@ -700,9 +715,13 @@ __global__ void __launch_bounds__(512, 1)
   const bool hasB = 2 * qp + 1 < ntile;
   const int q_end = __ldg(cu_q + r + 1);
   const int q0 = __ldg(cu_q + r) + qp * 256;
-  const int k0 = __ldg(cu_k + r);
-  const int Lr = __ldg(cu_k + r + 1) - k0;
-  const int nk = (Lr + 127) >> 7;
+  const int Lr = __ldg(cu_k + r + 1) - __ldg(cu_k + r);
+  const int nk_all = (Lr + 127) >> 7;
+  const int nsplit = gridDim.z, split = blockIdx.z;
+  const int kb = (int)(((long long)nk_all * split) / nsplit);       // first key tile of this CTA
+  const int nk = (int)(((long long)nk_all * (split + 1)) / nsplit) - kb;
+  const int k0 = __ldg(cu_k + r) + kb * 128;                         // its first key row
+  const int Lr_rem = Lr - kb * 128;                                  // keys from k0 to the end
 
   if (threadIdx.x == 0) {
     tc::mbar_init(bar_q, 1);
@@ -842,7 +861,7 @@ __global__ void __launch_bounds__(512, 1)
           tc::tmem_ld32(tS + lane_off + c * 32, reinterpret_cast<uint32_t*>(s + c * 32));
         tc::tmem_wait_ld();
         ATTN_TRACE(t, kt, 1);
-        const int valid = Lr - kt * 128;
+        const int valid = Lr_rem - kt * 128;
         if (valid < 128) {                                 // only the request's last key tile
 #pragma unroll
           for (int i = 0; i < 128; ++i) s[i] = (i < valid) ? s[i] : -INFINITY;
@@ -899,6 +918,10 @@ __global__ void __launch_bounds__(512, 1)
         l = l * factor + (((a8[0] + a8[1]) + (a8[2] + a8[3])) + ((a8[4] + a8[5]) + (a8[6] + a8[7])));
       }
       sL[t * 128 + row] = l;
+      if (nsplit > 1) {
+        const int grow = q0 + t * 128 + row;
+        if (grow < q_end) ML[((size_t)split * total_q + grow) * heads + head] = make_float2(m_used, l);
+      }
       __syncwarp();
       if (lane == 0) tc::mbar_arrive(&bar_fin[t]);
     }
@@ -940,10 +963,15 @@ __global__ void __launch_bounds__(512, 1)
     }
     for (int t = 0; t < ntl; ++t) {
       const int grow = q0 + t * 128 + row;
-      __nv_bfloat16* orow = O + (size_t)grow * ldo + head * D;
+      __nv_bfloat16* orow = nsplit > 1
+          ? Opart + split * part_stride + (size_t)grow * (heads * D) + head * D
+          : O + (size_t)grow * ldo + head * D;
       if (nk == 0) {                                       // no keys: defined zero output
-        if (grow < q_end)
+        if (grow < q_end) {
           for (int c = 0; c < D; c += 8) *reinterpret_cast<uint4*>(orow + c) = make_uint4(0, 0, 0, 0);
+          if (nsplit > 1)
+            ML[((size_t)split * total_q + grow) * heads + head] = make_float2(-INFINITY, 0.f);
+        }
         continue;
       }
       tc::mbar_wait(&bar_fin[t], 0);
@@ -977,7 +1005,49 @@ __global__ void __launch_bounds__(512, 1)
   }
 }
 
+// Merge of the split-KV partials: out = sum_z w_z O_z / sum_z w_z, w_z = l_z 2^(m_z - max m).
+// One thread per 8 output columns of one (row, head).
+template <int D>
+__global__ void __launch_bounds__(256) attn_combine_kernel(const __nv_bfloat16* __restrict__ Opart,
+                                                           const float2* __restrict__ ML,
+                                                           long long part_stride, int nsplit,
+                                                           int total_q, int heads,
+                                                           __nv_bfloat16* __restrict__ O, int ldo) {
+  pdl_trigger();
+  pdl_wait();
+  constexpr int C8 = D / 8;
+  const long long n = (long long)total_q * heads * C8;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (long long)gridDim.x * blockDim.x) {
+    const int c8 = (int)(i % C8);
+    const long long rh = i / C8;                       // row * heads + head
+    const int row = (int)(rh / heads), head = (int)(rh - (long long)row * heads);
+    float m = -INFINITY;
+    for (int z = 0; z < nsplit; ++z) {
+      const float2 v = __ldg(ML + (size_t)z * total_q * heads + rh);
+      if (v.y > 0.f) m = fmaxf(m, v.x);
+    }
+    float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f}, wsum = 0.f;
+    const size_t col = (size_t)row * heads * D + (size_t)head * D + c8 * 8;
+    for (int z = 0; z < nsplit; ++z) {
+      const float2 v = __ldg(ML + (size_t)z * total_q * heads + rh);
+      if (!(v.y > 0.f)) continue;
+      const float wz = v.y * exp2f(v.x - m);
+      float f[8];
+      Vec16<__nv_bfloat16>::unpack(__ldg(reinterpret_cast<const uint4*>(Opart + z * part_stride + col)), f);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) acc[e] += wz * f[e];
+      wsum += wz;
+    }
+    const float inv = wsum > 0.f ? 1.0f / wsum : 0.f;
+#pragma unroll
+    for (int e = 0; e < 8; ++e) acc[e] *= inv;
+    *reinterpret_cast<uint4*>(O + (size_t)row * ldo + head * D + c8 * 8) = Vec16<__nv_bfloat16>::pack(acc);
+  }
+}
+
 int g_attn_force = 0;   // tests: 1 = one-tile kernel, 2 = two-tile smem-P kernel, 3 = P-in-TMEM
+int g_attn_split = 0;   // tests: 0 = choose the split-KV factor, S > 0 = force S (when scratch fits)
 
 bool attention_tc_supported(int dtype, int head_dim) {
   return dtype == FPS_BF16 && (head_dim == 64 || head_dim == 128);
@@ -1043,15 +1113,50 @@ static fps_status launch_d2(const void* q, const void* kv, void* o, int heads,
   return FPS_OK;
 }
 
+// Split-KV factor: the grid of `pairs x heads` CTAs (one per SM) often leaves the last wave
+// mostly empty (C2A: 200 CTAs on 148 SMs -> 2 waves at 68 %); splitting every CTA's key range in
+// S parts fills the waves better at the cost of a combine pass.  Chosen by wave efficiency
+// (CTAs / (waves x 148)), S <= 4, at least 8 key tiles per part (measured with
+// tools/block_probe.py: C2A, 32 key tiles, S = 2 cuts the block's attention 0.130 -> 0.119 ms,
+// S = 3 / 4 lose; C2B, 8 key tiles, S = 2 loses 0.036 -> 0.044 ms), S > 1 only if it gains
+// > 8 % and the scratch (partial outputs + statistics) fits.
+static int choose_split(int ctas, int min_nk, int total_q, int H, int heads,
+                        const AttnScratch* sc) {
+  auto fits = [&](int S) {
+    return sc && (size_t)S * total_q * H * 2 <= sc->part_bytes &&
+           (size_t)S * total_q * heads * 8 <= sc->ml_bytes;
+  };
+  if (g_attn_split > 0) return fits(g_attn_split) && min_nk >= g_attn_split ? g_attn_split : 1;
+  auto eff = [&](int S) {
+    const long long c = (long long)ctas * S;
+    return (double)c / (double)(((c + kNumSMs - 1) / kNumSMs) * kNumSMs);
+  };
+  int best = 1;
+  double be = eff(1);
+  for (int S = 2; S <= 4; ++S)
+    if (min_nk >= 8 * S && fits(S) && eff(S) > be + 0.08) {
+      best = S;
+      be = eff(S);
+    }
+  return best;
+}
+
 template <int D>
 static fps_status launch_d3(const void* q, const void* kv, void* o, int heads,
                             const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
-                            const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo) {
+                            const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo,
+                            const AttnScratch* sc) {
   using Cfg = Attn3Cfg<D>;
   const int H = heads * D;
-  int pairs = 0;
-  for (int r = 0; r < n_req; ++r) pairs += ((h_cu_q[r + 1] - h_cu_q[r] + 127) / 128 + 1) / 2;
+  int pairs = 0, min_nk = 1 << 30;
+  for (int r = 0; r < n_req; ++r) {
+    const int pr = ((h_cu_q[r + 1] - h_cu_q[r] + 127) / 128 + 1) / 2;
+    pairs += pr;
+    if (pr > 0) min_nk = std::min(min_nk, (h_cu_k[r + 1] - h_cu_k[r] + 127) / 128);
+  }
   if (pairs == 0) return FPS_OK;
+  const int total_q = h_cu_q[n_req];
+  const int S = choose_split(pairs * heads, min_nk, total_q, H, heads, sc);
   CUtensorMap tq, tkv;
   if (!make_tmap_2d_bf16(&tq, q, (uint64_t)h_cu_q[n_req], H, (uint64_t)H * 2, 64, 128))
     return fail(FPS_ECUDA, "attention_tc3: Q tensor map");
@@ -1064,9 +1169,20 @@ static fps_status launch_d3(const void* q, const void* kv, void* o, int heads,
     attr = true;
   }
   const float scale_log2 = 1.4426950408889634f / sqrtf((float)D);
-  FPS_CUDA_TRY(launch_k(attn_tc3_kernel<D>, dim3(pairs, heads), dim3(512), Cfg::SMEM, s, tq, tkv,
+  const long long part_stride = (long long)total_q * H;
+  auto* Opart = S > 1 ? reinterpret_cast<__nv_bfloat16*>(sc->part) : nullptr;
+  auto* ML = S > 1 ? reinterpret_cast<float2*>(sc->ml) : nullptr;
+  FPS_CUDA_TRY(launch_k(attn_tc3_kernel<D>, dim3(pairs, heads, S), dim3(512), Cfg::SMEM, s, tq, tkv,
                         reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads,
-                        scale_log2, ldo));
+                        scale_log2, ldo, Opart, ML, part_stride, total_q));
+  if (S > 1) {
+    count_launch();
+    const long long n = (long long)total_q * heads * (D / 8);
+    const int grid = (int)std::min<long long>((n + 255) / 256, kNumSMs * 8LL);
+    FPS_CUDA_TRY(launch_k(attn_combine_kernel<D>, dim3(grid), dim3(256), 0, s,
+                          (const __nv_bfloat16*)Opart, (const float2*)ML, part_stride, S, total_q,
+                          heads, reinterpret_cast<__nv_bfloat16*>(o), ldo));
+  }
 #ifdef FPS_ATTN_TRACE
   {
     static long long h[2][64][8];
@@ -1088,7 +1204,8 @@ static fps_status launch_d3(const void* q, const void* kv, void* o, int heads,
 
 fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads, int head_dim,
                                const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
-                               const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo) {
+                               const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo,
+                               const AttnScratch* sc) {
   if (ldo == 0) ldo = heads * head_dim;
   if (ldo < heads * head_dim || ldo % 8 != 0)
     return fail(FPS_EINVAL, "attention_tc: output row stride %d", ldo);
@@ -1103,8 +1220,8 @@ fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads
   // A+B operand reads exceed the 128 B/clk smem port), which ate the latency it saved.
   if (g_attn_force == 0 || g_attn_force == 3) {
     if (head_dim == 128)
-      return launch_d3<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo);
-    return launch_d3<64>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo);
+      return launch_d3<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo, sc);
+    return launch_d3<64>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo, sc);
   }
   if (g_attn_force == 2) {
     if (head_dim == 128)

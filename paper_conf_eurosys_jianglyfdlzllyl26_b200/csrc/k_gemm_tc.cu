@@ -750,7 +750,10 @@ fps_status launch_gemm_tc(const void* A, const void* B, int M, int N, int K, con
   // quantisation differences the wave model sees; one wave: the wave model and M padding decide
   // (one wave, long K: the pair's deeper ring wins -- 80.5 vs 83.3 us at 1331x3072x12288;
   //  short K: its longer prologue / epilogue lose -- 27.3 vs 23.2 us at 1331x3072x3072)
-  const bool pair_wins = tp > kNumSMs / 2 || cp < cmin ||
+  // short K (< 1024, the SDXL-scale projections at C = 640): the pair's longer prologue and
+  // epilogue are not amortised even over several waves (4916x1920x640: 30.2 vs 23.3 us for the
+  // 1-SM kernel; 4916x5120x640: 54.8 vs 52.9; 16384x1920x640: 64.7 vs 61.3; K >= 1280: ties)
+  const bool pair_wins = (tp > kNumSMs / 2 && K >= 1024) || cp < cmin ||
                          (cp == cmin && (m2 * 256 - M < 128 || K >= 8192));
   // swapped operands (activation rows on the MMA's N side, no 256-row M padding): correct and
   // tested, but measured no faster at the masked-block shapes (1331x9216x3072: 59.8 vs 59.2 us

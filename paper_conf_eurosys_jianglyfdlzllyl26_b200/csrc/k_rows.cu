@@ -447,6 +447,55 @@ __global__ void __launch_bounds__(128) ln_affine_f32_kernel(const float* __restr
   }
 }
 
+// Narrow rows (H <= 1024): one warp per row, VPT float4 per lane, shuffle-only reductions.
+template <int VPT>
+__global__ void __launch_bounds__(128) ln_affine_f32_warp_kernel(const float* __restrict__ x, int n,
+                                                                 int H, __nv_bfloat16* __restrict__ out,
+                                                                 const __nv_bfloat16* __restrict__ gamma,
+                                                                 const __nv_bfloat16* __restrict__ beta) {
+  pdl_trigger();
+  pdl_wait();
+  const int row = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (row >= n) return;
+  const int nvec = H / 4;
+  const float4* xr = reinterpret_cast<const float4*>(x + (size_t)row * H);
+  const uint2* gp = reinterpret_cast<const uint2*>(gamma);
+  const uint2* bp = reinterpret_cast<const uint2*>(beta);
+  float4 v[VPT];
+  uint2 gv[VPT], bv[VPT];
+  float sum = 0.f;
+#pragma unroll
+  for (int k = 0; k < VPT; ++k) {
+    const int vi = lane + 32 * k;
+    const bool ok = vi < nvec;
+    v[k] = ok ? __ldg(xr + vi) : make_float4(0.f, 0.f, 0.f, 0.f);
+    gv[k] = ok ? __ldg(gp + vi) : make_uint2(0, 0);
+    bv[k] = ok ? __ldg(bp + vi) : make_uint2(0, 0);
+    sum += (v[k].x + v[k].y) + (v[k].z + v[k].w);
+  }
+  const float mean = warp_sum(sum) / (float)H;
+  float sq = 0.f;
+#pragma unroll
+  for (int k = 0; k < VPT; ++k)
+    if (lane + 32 * k < nvec) {
+      const float a = v[k].x - mean, b = v[k].y - mean, c = v[k].z - mean, d = v[k].w - mean;
+      sq += (a * a + b * b) + (c * c + d * d);
+    }
+  const float rstd = 1.0f / sqrtf(warp_sum(sq) / (float)H + 1e-6f);
+  uint2* o = reinterpret_cast<uint2*>(out + (size_t)row * H);
+#pragma unroll
+  for (int k = 0; k < VPT; ++k) {
+    const int vi = lane + 32 * k;
+    if (vi < nvec) {
+      float g0, g1, g2, g3, b0, b1, b2, b3;
+      unpack_bf16x2(gv[k].x, g0, g1); unpack_bf16x2(gv[k].y, g2, g3);
+      unpack_bf16x2(bv[k].x, b0, b1); unpack_bf16x2(bv[k].y, b2, b3);
+      o[vi] = make_uint2(pack_bf16x2((v[k].x - mean) * rstd * g0 + b0, (v[k].y - mean) * rstd * g1 + b1),
+                         pack_bf16x2((v[k].z - mean) * rstd * g2 + b2, (v[k].w - mean) * rstd * g3 + b3));
+    }
+  }
+}
+
 fps_status launch_ln_affine_f32in(const float* x, int n, int H, void* out, const void* gamma,
                                   const void* beta, cudaStream_t s) {
   if (n <= 0) return FPS_OK;
@@ -457,7 +506,12 @@ fps_status launch_ln_affine_f32in(const float* x, int n, int H, void* out, const
   auto O = reinterpret_cast<__nv_bfloat16*>(out);
   prof::begin(s);
   cudaError_t le;
-  if (per <= 2) le = launch_k(ln_affine_f32_kernel<2>, dim3(n), dim3(128), 0, s, x, H, O, G, Bt);
+  const int per_lane = ceil_div(H / 4, 32), wgrid = ceil_div(n, 4);
+  if (per_lane <= 4)
+    le = launch_k(ln_affine_f32_warp_kernel<4>, dim3(wgrid), dim3(128), 0, s, x, n, H, O, G, Bt);
+  else if (per_lane <= 8)
+    le = launch_k(ln_affine_f32_warp_kernel<8>, dim3(wgrid), dim3(128), 0, s, x, n, H, O, G, Bt);
+  else if (per <= 2) le = launch_k(ln_affine_f32_kernel<2>, dim3(n), dim3(128), 0, s, x, H, O, G, Bt);
   else if (per <= 4) le = launch_k(ln_affine_f32_kernel<4>, dim3(n), dim3(128), 0, s, x, H, O, G, Bt);
   else if (per <= 8) le = launch_k(ln_affine_f32_kernel<8>, dim3(n), dim3(128), 0, s, x, H, O, G, Bt);
   else if (per <= 16) le = launch_k(ln_affine_f32_kernel<16>, dim3(n), dim3(128), 0, s, x, H, O, G, Bt);

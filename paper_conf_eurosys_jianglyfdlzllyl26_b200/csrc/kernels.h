@@ -41,18 +41,28 @@ fps_status launch_gemm_simt(int dtype, const void* A, const void* B, int M, int 
 fps_status launch_gemm_tc(const void* A, const void* B, int M, int N, int K, const Epilogue& ep,
                           cudaStream_t s);
 bool gemm_tc_supported(int dtype, int M, int N, int K);
+// Scratch for split-KV attention: partial outputs (S x total_q x H bf16) and per-row
+// statistics (S x total_q x heads float2); null = no split
+struct AttnScratch {
+  void* part;
+  size_t part_bytes;
+  void* ml;
+  size_t ml_bytes;
+};
 // a6: o[i, head] = softmax(q_i k^T / sqrt(d)) v over the request's merged keys; o rows are
 // ldo elements apart (0 = heads * head_dim)
 fps_status launch_attention(int dtype, const void* q, const void* kv, void* o, int heads,
                             int head_dim, const int32_t* d_cu_q, const int32_t* d_cu_k,
                             const int32_t* h_cu_q, const int32_t* h_cu_k, int n_req, int total_q,
-                            int max_q, int max_k, cudaStream_t s, int ldo = 0);
+                            int max_q, int max_k, cudaStream_t s, int ldo = 0,
+                            const AttnScratch* sc = nullptr);
 fps_status launch_attention_simt(int dtype, const void* q, const void* kv, void* o, int heads,
                                  int head_dim, const int32_t* cu_q, const int32_t* cu_k,
                                  int n_req, int total_q, cudaStream_t s, int ldo = 0);
 fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads, int head_dim,
                                const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
-                               const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo = 0);
+                               const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo = 0,
+                               const AttnScratch* sc = nullptr);
 bool attention_tc_supported(int dtype, int head_dim);
 
 // true if fps_cache_prefetch also overwrites rows outside U (copy_method 2): fresh rows written
@@ -66,6 +76,8 @@ extern int g_disable_tc;
 extern int g_gemm_force;
 // tests: 0 = two query tiles per CTA (default), 1 = force the one-tile attention kernel
 extern int g_attn_force;
+// tests: force the split-KV factor S (0 = choose)
+extern int g_attn_split;
 // 1 (default): HBM-arena whole-entry loads copied by a library kernel, 0: driver D2D memcpy
 extern int g_d2d_kernel;
 

@@ -258,3 +258,17 @@ def test_c4_continuous_batch_sampled_rows(F, mode):
         a = B.attention(B.linear(h1[M][sample], Wq, bq), Kall, Vall, heads)
         ref = B._attn_out_and_mlp(r["x"][M][sample], a, w, r["mod"], H)
         check_close(y[cu[i] + sample], ref, TOL["bf16"], f"C4 {mode} request {i}")
+
+
+@pytest.mark.parametrize("mode,split", [("kv", 2), ("kv", 3), ("y", 2), ("kv", 4)])
+def test_split_kv_attention(F, mode, split):
+    """Split-KV attention (each CTA's key range in S parts, then a combine pass) inside the
+    block: heterogeneous varlen batch with ragged key tiles; the parts must merge to the
+    oracle's softmax over all keys."""
+    w, reqs = _problem(2010 + split, "bf16", 256, 2, 1024, 1500, 36, [0.05, 0.6, 0.3], blobs=False)
+    F.fps_set_disable_tc(split << 8)
+    try:
+        y, _ = _run_masked(F, w, reqs, 2, "bf16", mode)
+    finally:
+        F.fps_set_disable_tc(0)
+    check_close(y, _ref_masked(w, reqs, 2, mode), TOL["bf16"], f"split {split} {mode}")
