@@ -4,8 +4,9 @@
 A step = one denoising step of the whole hot path for one batch of synthetic requests: mask-aware
 stack of N blocks (a4-a8) with the Alg. 1 plan, layer-ahead cache prefetch from pinned host DRAM
 (a3), replenish (a9) and the sampler update, through fps_run_batch.  Default workload: configs[2]
-(Flux-scale DiT stack, 4096 image + 512 text tokens, H 3072, 24x128 heads, bf16, 20% mask,
-cached K/V streamed from pinned host per layer).
+(Flux-scale DiT stack -- Flux's 19 double-stream + 38 single-stream blocks -- 4096 image + 512
+text tokens, H 3072, 24x128 heads, bf16, 20% mask, cached K/V streamed from pinned host per
+layer).
 
   python bench.py [--gpus N --steps K --warmup W --config C3|C4|C2A|C2B --mode kv|y]
   python bench.py --impl reference ...     (the CPU oracle on the same workload)
@@ -400,7 +401,7 @@ def main():
                          "single-stream) block with fused input / output projections, or the SDXL "
                          "block with cross-attention and GEGLU, or Flux's stack of 19 double-stream "
                          "then 38 single-stream blocks (NEXT-2); default: sdxl for the "
-                         "SDXL-scale configs (C2A/C2B), seq otherwise")
+                         "SDXL-scale configs (C2A/C2B), flux for the Flux-scale ones (C3/C4)")
     ap.add_argument("--tier", default="host", choices=["host", "hbm", "host_hugepage"],
                     help="template cache in pinned host DRAM (configs[2]) or HBM (NEXT-1)")
     ap.add_argument("--copy-ctas", type=int, default=0, help="CTAs of the SM row gather (0 = lib default)")
@@ -427,8 +428,8 @@ def main():
     rank = int(os.environ.get("RANK", 0))
     world = int(os.environ.get("WORLD_SIZE", 1))
     local = int(os.environ.get("LOCAL_RANK", 0))
-    if args.block is None:
-        args.block = "sdxl" if args.config.startswith("C2") else "seq"
+    if args.block is None:       # the evaluated models' own block structure (R24, R25)
+        args.block = "sdxl" if args.config.startswith("C2") else "flux"
     w = dict(WORKLOADS[args.config], block=args.block)
     K, W = args.steps, max(args.warmup, 0)
     if W + K > w["steps"]:

@@ -92,6 +92,24 @@ fps_status launch_gemm(int dtype, const void* A, const void* B, int M, int N, in
   return st;
 }
 
+fps_status launch_gemm_grouped(int dtype, const void* A, const void* B0, const void* B1, int M0,
+                               int M1, int N, int K, const Epilogue& ep0, const Epilogue& ep1,
+                               cudaStream_t s) {
+  if (M1 <= 0) return launch_gemm(dtype, A, B0, M0, N, K, ep0, s);
+  if (M0 <= 0) return launch_gemm(dtype, (const char*)A + (size_t)M0 * K * elt_size(dtype), B1, M1,
+                                  N, K, ep1, s);
+  if ((g_disable_tc & 1) || !gemm_tc_supported(dtype, M0 + M1, N, K)) {
+    FPS_TRY(launch_gemm(dtype, A, B0, M0, N, K, ep0, s));
+    return launch_gemm(dtype, (const char*)A + (size_t)M0 * K * elt_size(dtype), B1, M1, N, K, ep1,
+                       s);
+  }
+  prof::begin(s);
+  fps_status st = launch_gemm_tc_grouped(A, B0, B1, M0, M1, N, K, ep0, ep1, s);
+  const double e = elt_size(dtype), M = (double)M0 + M1;
+  prof::end(s, prof::GEMM, 2.0 * M * N * K, e * (M * K + 2.0 * N * K + M * N));
+  return st;
+}
+
 fps_status launch_attention(int dtype, const void* q, const void* kv, void* o, int heads,
                             int head_dim, const int32_t* d_cu_q, const int32_t* d_cu_k,
                             const int32_t* h_cu_q, const int32_t* h_cu_k, int n_req, int total_q,
@@ -266,17 +284,18 @@ static fps_status double_block_forward(const fps_block_weights* w, const fps_var
   };
   if (tq > 0) {
     FPS_TRY(launch_copy_rows(x_act, perm, nullptr, tq, (int)rowb, x_sm, s));
+    // a4 per stream; a5 for both streams in one grouped launch: Q -> request-major rows,
+    // K|V -> merged key rows
+    Epilogue ep[2] = {};
     for (int st = 0; st < 2; ++st) {
-      // a4 per stream, a5 per stream: Q -> request-major rows, K|V -> merged key rows
       FPS_TRY(launch_ln_mod(dt, at(x_sm, st), nullptr, nrows[st], H, at(ws.h, st), cu[st],
                             b->n_req, mod, 6 * H * st, s, nullptr, MS));
-      Epilogue ep{};
-      ep.bias = Bqkv[st];
-      ep.out0 = ws.q; ep.ld0 = H; ep.map0 = perm + rows0[st];
-      ep.out1 = kv; ep.ld1 = 2 * H; ep.map1 = kvrow + rows0[st];
-      ep.split = H;
-      FPS_TRY(launch_gemm(dt, at(ws.h, st), Wqkv[st], nrows[st], 3 * H, H, ep, s));
+      ep[st].bias = Bqkv[st];
+      ep[st].out0 = ws.q; ep[st].ld0 = H; ep[st].map0 = perm + rows0[st];
+      ep[st].out1 = kv; ep[st].ld1 = 2 * H; ep[st].map1 = kvrow + rows0[st];
+      ep[st].split = H;
     }
+    FPS_TRY(launch_gemm_grouped(dt, ws.h, Wqkv[0], Wqkv[1], ti, tt, 3 * H, H, ep[0], ep[1], s));
   }
   if (tu > 0) {
     // Y-mode: cached input rows U (image rows, R9) -> image-stream LN -> K|V projection
@@ -297,29 +316,28 @@ static fps_status double_block_forward(const fps_block_weights* w, const fps_var
   FPS_TRY(launch_attention(dt, ws.q, kv, ws.ao, w->heads, w->head_dim, b->d_cu_q, b->d_cu_k,
                            b->h_cu_q, b->h_cu_k, b->n_req, tq, b->max_q, b->max_k, s, 0, &sc));
   FPS_TRY(launch_copy_rows(ws.ao, perm, nullptr, tq, (int)rowb, ao_sm, s));
-  for (int st = 0; st < 2; ++st) {   // a7 per stream: x1 = x + gate1 (A Wo^T + bo)
-    Epilogue ep{};
-    ep.bias = Bo[st];
-    ep.resid = at(x_sm, st); ep.ld_resid = H;
-    ep.gate = modp(st, 2); ep.gate_stride = MS; ep.cu = cu[st]; ep.n_req = b->n_req;
-    ep.out0 = at(ws.x1, st); ep.ld0 = H; ep.split = H;
-    FPS_TRY(launch_gemm(dt, at(ao_sm, st), Wo[st], nrows[st], H, H, ep, s));
+  // a7, a8: each projection one grouped launch over both streams (their own weights, adaLN
+  // gates and request offsets); y written back in request-major order
+  Epilogue eo[2] = {}, eu[2] = {}, ed[2] = {};
+  for (int st = 0; st < 2; ++st) {   // x1 = x + gate1 (A Wo^T + bo)
+    eo[st].bias = Bo[st];
+    eo[st].resid = at(x_sm, st); eo[st].ld_resid = H;
+    eo[st].gate = modp(st, 2); eo[st].gate_stride = MS; eo[st].cu = cu[st]; eo[st].n_req = b->n_req;
+    eo[st].out0 = at(ws.x1, st); eo[st].ld0 = H; eo[st].split = H;
   }
-  for (int st = 0; st < 2; ++st) {   // a8 per stream; y written back in request-major order
+  FPS_TRY(launch_gemm_grouped(dt, ao_sm, Wo[0], Wo[1], ti, tt, H, H, eo[0], eo[1], s));
+  for (int st = 0; st < 2; ++st) {
     FPS_TRY(launch_ln_mod(dt, at(ws.x1, st), nullptr, nrows[st], H, at(ws.h2, st), cu[st],
                           b->n_req, mod, 6 * H * st + 3 * H, s, nullptr, MS));
-    Epilogue eu{};
-    eu.bias = Bup[st]; eu.act = 1;
-    eu.out0 = at(ws.u, st, (size_t)F * e); eu.ld0 = F; eu.split = F;
-    FPS_TRY(launch_gemm(dt, at(ws.h2, st), Wup[st], nrows[st], F, H, eu, s));
-    Epilogue ed{};
-    ed.bias = Bdn[st];
-    ed.resid = at(ws.x1, st); ed.ld_resid = H;
-    ed.gate = modp(st, 5); ed.gate_stride = MS; ed.cu = cu[st]; ed.n_req = b->n_req;
-    ed.out0 = y_act; ed.ld0 = H; ed.map0 = perm + rows0[st]; ed.split = H;
-    FPS_TRY(launch_gemm(dt, at(ws.u, st, (size_t)F * e), Wdn[st], nrows[st], H, F, ed, s));
+    eu[st].bias = Bup[st]; eu[st].act = 1;
+    eu[st].out0 = at(ws.u, st, (size_t)F * e); eu[st].ld0 = F; eu[st].split = F;
+    ed[st].bias = Bdn[st];
+    ed[st].resid = at(ws.x1, st); ed[st].ld_resid = H;
+    ed[st].gate = modp(st, 5); ed[st].gate_stride = MS; ed[st].cu = cu[st]; ed[st].n_req = b->n_req;
+    ed[st].out0 = y_act; ed[st].ld0 = H; ed[st].map0 = perm + rows0[st]; ed[st].split = H;
   }
-  return FPS_OK;
+  FPS_TRY(launch_gemm_grouped(dt, ws.h2, Wup[0], Wup[1], ti, tt, F, H, eu[0], eu[1], s));
+  return launch_gemm_grouped(dt, ws.u, Wdn[0], Wdn[1], ti, tt, H, F, ed[0], ed[1], s);
 }
 
 static fps_status block_forward(const fps_block_weights* w, const fps_varlen_batch* b,

@@ -38,6 +38,21 @@ __device__ __forceinline__ void tile_coords(int tile, int num_m, int num_n, int&
   n_blk = local / gm;
 }
 
+// Grouped launch (double-stream block, R25): problem 0 = rows [0, M) of A with B and `ep`,
+// problem 1 = rows [M, M + M1) with B1 and `ep1` (row-local epilogue indexing), same N and K.
+// Tiles [0, T0) belong to problem 0, the rest to problem 1.
+template <int GM>
+__device__ __forceinline__ void group_coords(int tile, int T0, int num_m0, int num_m1, int num_n,
+                                             int& p, int& m_blk, int& n_blk) {
+  if (tile < T0) {
+    p = 0;
+    tile_coords<GM>(tile, num_m0, num_n, m_blk, n_blk);
+  } else {
+    p = 1;
+    tile_coords<GM>(tile - T0, num_m1, num_n, m_blk, n_blk);
+  }
+}
+
 // Per-row epilogue context: gate vector of the row's request and the output rows of both
 // column ranges (K/V scatter into the merged key buffer).
 struct RowCtx {
@@ -215,7 +230,8 @@ struct GemmCfg {
 template <int BN, int STAGES>
 __global__ void __launch_bounds__(256, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                   int M, int N, int K, Epilogue ep) {
+                   const __grid_constant__ CUtensorMap tmB1, int M, int N, int K, Epilogue ep,
+                   int M1, Epilogue ep1) {
   using Cfg = GemmCfg<BN, STAGES>;
   constexpr int kGroupM = 16;                              // 2048 rows of A per group
   extern __shared__ uint8_t smem_raw[];
@@ -231,8 +247,10 @@ __global__ void __launch_bounds__(256, 1)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int num_m = (M + Cfg::BM - 1) / Cfg::BM;
+  const int num_m1 = (M1 + Cfg::BM - 1) / Cfg::BM;
   const int num_n = (N + BN - 1) / BN;
-  const int num_tiles = num_m * num_n;
+  const int T0 = num_m * num_n;
+  const int num_tiles = T0 + num_m1 * num_n;
   const int num_k = K / Cfg::BK;
 
   if (threadIdx.x == 0) {
@@ -249,6 +267,7 @@ __global__ void __launch_bounds__(256, 1)
   if (warp == 0 && lane == 0) {
     tc::tma_prefetch_desc(&tmA);
     tc::tma_prefetch_desc(&tmB);
+    if (M1 > 0) tc::tma_prefetch_desc(&tmB1);
   }
   if (warp == 2) tc::tmem_alloc<Cfg::TMEM_COLS>(tmem_holder);
   tc::fence_before();
@@ -263,14 +282,15 @@ __global__ void __launch_bounds__(256, 1)
       int stage = 0;
       uint32_t phase = 0;
       for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
-        int m_blk, n_blk;
-        tile_coords<kGroupM>(tile, num_m, num_n, m_blk, n_blk);
+        int p, m_blk, n_blk;
+        group_coords<kGroupM>(tile, T0, num_m, num_m1, num_n, p, m_blk, n_blk);
+        const CUtensorMap* tb = p ? &tmB1 : &tmB;
+        const int arow = (p ? M : 0) + m_blk * Cfg::BM;
         for (int kb = 0; kb < num_k; ++kb) {
           tc::mbar_wait(&empty[stage], phase ^ 1);
           tc::mbar_expect_tx(&full[stage], Cfg::STAGE_BYTES);
-          tc::tma_load_2d(sA + stage * Cfg::A_BYTES, &tmA, &full[stage], kb * Cfg::BK,
-                          m_blk * Cfg::BM);
-          tc::tma_load_2d(sB + stage * Cfg::B_BYTES, &tmB, &full[stage], kb * Cfg::BK, n_blk * BN);
+          tc::tma_load_2d(sA + stage * Cfg::A_BYTES, &tmA, &full[stage], kb * Cfg::BK, arow);
+          tc::tma_load_2d(sB + stage * Cfg::B_BYTES, tb, &full[stage], kb * Cfg::BK, n_blk * BN);
           if (++stage == STAGES) {
             stage = 0;
             phase ^= 1;
@@ -311,12 +331,12 @@ __global__ void __launch_bounds__(256, 1)
     const int q = warp & 3;
     int it = 0;
     for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++it) {
-      int m_blk, n_blk;
-      tile_coords<kGroupM>(tile, num_m, num_n, m_blk, n_blk);
+      int p, m_blk, n_blk;
+      group_coords<kGroupM>(tile, T0, num_m, num_m1, num_n, p, m_blk, n_blk);
       const int acc = it & 1;
       tc::mbar_wait(&tfull[acc], (it >> 1) & 1);
       tc::fence_after();
-      epilogue_tile<BN>(ep, M, N, m_blk * Cfg::BM + q * 32 + lane, n_blk * BN,
+      epilogue_tile<BN>(p ? ep1 : ep, p ? M1 : M, N, m_blk * Cfg::BM + q * 32 + lane, n_blk * BN,
                         tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN);
       tc::fence_before();
       __syncwarp();
@@ -345,7 +365,8 @@ struct Gemm2Cfg {
 template <int STAGES>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
     gemm_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                    int M, int N, int K, Epilogue ep) {
+                    const __grid_constant__ CUtensorMap tmB1, int M, int N, int K, Epilogue ep,
+                    int M1, Epilogue ep1) {
   using Cfg = Gemm2Cfg<STAGES>;
   constexpr int kGroupM = 8;                               // 2048 rows of A per group
   extern __shared__ uint8_t smem_raw[];
@@ -363,8 +384,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
   const uint32_t rank = tc::cluster_ctarank();
   const int pair = blockIdx.x >> 1, num_pairs = gridDim.x >> 1;
   const int num_m = (M + Cfg::BM - 1) / Cfg::BM;
+  const int num_m1 = (M1 + Cfg::BM - 1) / Cfg::BM;
   const int num_n = (N + Cfg::BN - 1) / Cfg::BN;
-  const int num_tiles = num_m * num_n;
+  const int T0 = num_m * num_n;
+  const int num_tiles = T0 + num_m1 * num_n;
   const int num_k = K / Cfg::BK;
 
   if (threadIdx.x == 0) {
@@ -381,6 +404,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
   if (warp == 0 && lane == 0) {
     tc::tma_prefetch_desc(&tmA);
     tc::tma_prefetch_desc(&tmB);
+    if (M1 > 0) tc::tma_prefetch_desc(&tmB1);
   }
   if (warp == 2) tc::tmem_alloc_2sm<Cfg::TMEM_COLS>(tmem_holder);
   tc::fence_before();
@@ -396,14 +420,16 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
       int stage = 0;
       uint32_t phase = 0;
       for (int tile = pair; tile < num_tiles; tile += num_pairs) {
-        int m_blk, n_blk;
-        tile_coords<kGroupM>(tile, num_m, num_n, m_blk, n_blk);
-        const int arow = m_blk * Cfg::BM + rank * 128, brow = n_blk * Cfg::BN + rank * 128;
+        int p, m_blk, n_blk;
+        group_coords<kGroupM>(tile, T0, num_m, num_m1, num_n, p, m_blk, n_blk);
+        const CUtensorMap* tb = p ? &tmB1 : &tmB;
+        const int arow = (p ? M : 0) + m_blk * Cfg::BM + rank * 128;
+        const int brow = n_blk * Cfg::BN + rank * 128;
         for (int kb = 0; kb < num_k; ++kb) {
           tc::mbar_wait(&empty[stage], phase ^ 1);
           if (rank == 0) tc::mbar_expect_tx(&full[stage], 2 * Cfg::STAGE_BYTES);
           tc::tma_load_2d_2sm(sA + stage * Cfg::A_BYTES, &tmA, &full[stage], kb * Cfg::BK, arow);
-          tc::tma_load_2d_2sm(sB + stage * Cfg::B_BYTES, &tmB, &full[stage], kb * Cfg::BK, brow);
+          tc::tma_load_2d_2sm(sB + stage * Cfg::B_BYTES, tb, &full[stage], kb * Cfg::BK, brow);
           if (++stage == STAGES) {
             stage = 0;
             phase ^= 1;
@@ -445,12 +471,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
     const uint32_t tempty_leader = tc::mapa(tc::smem_u32(tempty), 0);
     int it = 0;
     for (int tile = pair; tile < num_tiles; tile += num_pairs, ++it) {
-      int m_blk, n_blk;
-      tile_coords<kGroupM>(tile, num_m, num_n, m_blk, n_blk);
+      int p, m_blk, n_blk;
+      group_coords<kGroupM>(tile, T0, num_m, num_m1, num_n, p, m_blk, n_blk);
       const int acc = it & 1;
       tc::mbar_wait(&tfull[acc], (it >> 1) & 1);
       tc::fence_after();
-      epilogue_tile<256>(ep, M, N, m_blk * Cfg::BM + rank * 128 + q * 32 + lane, n_blk * Cfg::BN,
+      epilogue_tile<256>(p ? ep1 : ep, p ? M1 : M, N,
+                         m_blk * Cfg::BM + rank * 128 + q * 32 + lane, n_blk * Cfg::BN,
                          tmem_base + ((uint32_t)(q * 32) << 16) + acc * 256);
       tc::fence_before();
       __syncwarp();
@@ -644,24 +671,34 @@ bool gemm_tc_supported(int dtype, int M, int N, int K) {
 
 int g_gemm_force = 0;   // tests: 1 = force the 1-SM kernel, 2 = force the CTA-pair kernel
 
+// Optional second problem of a grouped launch (see group_coords): B1 [N, K], M1 rows of A after
+// the first M, its own epilogue.  M1 = 0: a plain GEMM.
+struct Group2 {
+  const void* B1;
+  int M1;
+  Epilogue ep1;
+};
+
 template <int BN, int STAGES>
 static fps_status launch_cfg(const void* A, const void* B, int M, int N, int K,
-                             const Epilogue& ep, cudaStream_t s) {
+                             const Epilogue& ep, cudaStream_t s, const Group2& g2 = Group2{}) {
   using Cfg = GemmCfg<BN, STAGES>;
-  CUtensorMap ta, tb;
-  if (!make_tmap_2d_bf16(&ta, A, M, K, (uint64_t)K * 2, Cfg::BK, Cfg::BM) ||
-      !make_tmap_2d_bf16(&tb, B, N, K, (uint64_t)K * 2, Cfg::BK, BN))
+  CUtensorMap ta, tb, tb1;
+  if (!make_tmap_2d_bf16(&ta, A, M + g2.M1, K, (uint64_t)K * 2, Cfg::BK, Cfg::BM) ||
+      !make_tmap_2d_bf16(&tb, B, N, K, (uint64_t)K * 2, Cfg::BK, BN) ||
+      (g2.M1 > 0 && !make_tmap_2d_bf16(&tb1, g2.B1, N, K, (uint64_t)K * 2, Cfg::BK, BN)))
     return fail(FPS_ECUDA, "gemm_tc: cuTensorMapEncodeTiled failed (M=%d N=%d K=%d)", M, N, K);
+  if (g2.M1 == 0) tb1 = tb;
   static bool attr_set = false;
   if (!attr_set) {
     FPS_CUDA_TRY(cudaFuncSetAttribute(gemm_tc_kernel<BN, STAGES>,
                                       cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
     attr_set = true;
   }
-  const int tiles = ceil_div(M, Cfg::BM) * ceil_div(N, BN);
+  const int tiles = (ceil_div(M, Cfg::BM) + ceil_div(g2.M1, Cfg::BM)) * ceil_div(N, BN);
   const int grid = tiles < kNumSMs ? tiles : kNumSMs;
   FPS_CUDA_TRY(launch_k(gemm_tc_kernel<BN, STAGES>, dim3(grid), dim3(256), Cfg::SMEM, s, ta, tb,
-                        M, N, K, ep));
+                        tb1, M, N, K, ep, g2.M1, g2.ep1));
   count_launch();
   FPS_LAUNCH_CHECK();
   return FPS_OK;
@@ -669,22 +706,24 @@ static fps_status launch_cfg(const void* A, const void* B, int M, int N, int K,
 
 template <int STAGES>
 static fps_status launch_pair(const void* A, const void* B, int M, int N, int K,
-                              const Epilogue& ep, cudaStream_t s) {
+                              const Epilogue& ep, cudaStream_t s, const Group2& g2 = Group2{}) {
   using Cfg = Gemm2Cfg<STAGES>;
-  CUtensorMap ta, tb;
-  if (!make_tmap_2d_bf16(&ta, A, M, K, (uint64_t)K * 2, Cfg::BK, 128) ||
-      !make_tmap_2d_bf16(&tb, B, N, K, (uint64_t)K * 2, Cfg::BK, 128))
+  CUtensorMap ta, tb, tb1;
+  if (!make_tmap_2d_bf16(&ta, A, M + g2.M1, K, (uint64_t)K * 2, Cfg::BK, 128) ||
+      !make_tmap_2d_bf16(&tb, B, N, K, (uint64_t)K * 2, Cfg::BK, 128) ||
+      (g2.M1 > 0 && !make_tmap_2d_bf16(&tb1, g2.B1, N, K, (uint64_t)K * 2, Cfg::BK, 128)))
     return fail(FPS_ECUDA, "gemm_tc2: cuTensorMapEncodeTiled failed (M=%d N=%d K=%d)", M, N, K);
+  if (g2.M1 == 0) tb1 = tb;
   static bool attr_set = false;
   if (!attr_set) {
     FPS_CUDA_TRY(cudaFuncSetAttribute(gemm_tc2_kernel<STAGES>,
                                       cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
     attr_set = true;
   }
-  const int tiles = ceil_div(M, Cfg::BM) * ceil_div(N, Cfg::BN);
+  const int tiles = (ceil_div(M, Cfg::BM) + ceil_div(g2.M1, Cfg::BM)) * ceil_div(N, Cfg::BN);
   const int pairs = tiles < kNumSMs / 2 ? tiles : kNumSMs / 2;
   FPS_CUDA_TRY(launch_k(gemm_tc2_kernel<STAGES>, dim3(2 * pairs), dim3(256), Cfg::SMEM, s, ta, tb,
-                        M, N, K, ep));
+                        tb1, M, N, K, ep, g2.M1, g2.ep1));
   count_launch();
   FPS_LAUNCH_CHECK();
   return FPS_OK;
@@ -728,6 +767,30 @@ static int swap_block(int M, int N, long* cost) {
   }
   *cost = bc;
   return best;
+}
+
+// Grouped pair of GEMMs in one launch (double-stream block: image rows on the image weights,
+// text rows on the text weights): both problems' tiles share the persistent grid, so the two
+// small problems fill the machine like one of their combined size.  Kernel choice as for one
+// GEMM with the combined tile counts.
+fps_status launch_gemm_tc_grouped(const void* A, const void* B0, const void* B1, int M0, int M1,
+                                  int N, int K, const Epilogue& ep0, const Epilogue& ep1,
+                                  cudaStream_t s) {
+  if (!aligned16(A) || !aligned16(B0) || !aligned16(B1))
+    return fail(FPS_EINVAL, "gemm_tc: unaligned operand");
+  const Group2 g2{B1, M1, ep1};
+  const int m1 = ceil_div(M0, 128) + ceil_div(M1, 128), m2 = ceil_div(M0, 256) + ceil_div(M1, 256);
+  const long t256 = (long)m1 * ceil_div(N, 256), t128 = (long)m1 * ceil_div(N, 128);
+  const long tp = (long)m2 * ceil_div(N, 256);
+  const long c256 = ((t256 + kNumSMs - 1) / kNumSMs) * 256;
+  const long c128 = ((t128 + kNumSMs - 1) / kNumSMs) * 128;
+  const long cp = ((tp + kNumSMs / 2 - 1) / (kNumSMs / 2)) * 256;
+  const long cmin = std::min(c256, c128);
+  const bool pair_wins = (tp > kNumSMs / 2 && K >= 1024) || cp < cmin;
+  if (g_gemm_force == 2 || (g_gemm_force != 1 && pair_wins))
+    return launch_pair<6>(A, B0, M0, N, K, ep0, s, g2);
+  if (c256 <= c128) return launch_cfg<256, 4>(A, B0, M0, N, K, ep0, s, g2);
+  return launch_cfg<128, 6>(A, B0, M0, N, K, ep0, s, g2);
 }
 
 fps_status launch_gemm_tc(const void* A, const void* B, int M, int N, int K, const Epilogue& ep,

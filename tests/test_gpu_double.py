@@ -85,17 +85,19 @@ def _ref(w, reqs, heads, mode, L_txt):
 
 
 @pytest.mark.parametrize("mode", ["kv", "y"])
-@pytest.mark.parametrize("simt", [False, True])
-def test_double_masked_varlen_batch(F, mode, simt):
+@pytest.mark.parametrize("flags", [0, 3, 4, 8])
+def test_double_masked_varlen_batch(F, mode, flags):
     """Three requests, masks 5-60 %, 40 text rows each: image rows of every request on the
-    image weights, text rows on the text weights, one joint attention launch."""
+    image weights, text rows on the text weights (one grouped GEMM launch per projection; flags
+    4 / 8 force its 1-SM / CTA-pair kernel, 3 the SIMT kernels as two launches), one joint
+    attention launch."""
     w, reqs = _problem(7100, "bf16", 256, 2, 1024, 576, 40, [0.05, 0.6, 0.3])
-    F.fps_set_disable_tc(3 if simt else 0)
+    F.fps_set_disable_tc(flags)
     try:
         y = _run(F, w, reqs, 2, "bf16", mode, 576)
     finally:
         F.fps_set_disable_tc(0)
-    check_close(y, _ref(w, reqs, 2, mode, 40), TOL["bf16"], f"double {mode} simt={simt}")
+    check_close(y, _ref(w, reqs, 2, mode, 40), TOL["bf16"], f"double {mode} flags={flags}")
 
 
 def test_double_fp32_and_dense(F):

@@ -45,3 +45,14 @@ def test_library_cost_equals_oracle_cost():
 def test_stats():
     s = PS.latency_stats({0: (0, 10), 1: (0, 20), 2: (5, 45)})
     assert s["p50_ms"] == 20 and s["p95_ms"] == 40 and s["mean_ms"] == pytest.approx(70 / 3)
+
+
+@pytest.mark.parametrize("kind,Lc", [("sdxl", 77), ("seq", 0)])
+def test_product_flops_match_oracle_counters(kind, Lc):
+    """The product's per-block FLOP count (planner / balancer cost input) equals the oracle's
+    Table 1 counters, including the SDXL block's cross-attention and GEGLU terms (R24)."""
+    from oracle import counters as OC
+    for mode in ("kv", "y", "dense"):
+        for n, L, H, F in ((410, 4096, 640, 2560), (307, 1024, 1280, 5120), (1331, 4608, 3072, 12288)):
+            assert PS.block_flops(mode, n, L, H, F, kind, Lc) == pytest.approx(
+                OC.block_flops(mode, n, L, H, F, kind, Lc), rel=1e-12)

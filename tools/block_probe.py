@@ -46,6 +46,22 @@ for _ in range(5):
 e1.record()
 torch.cuda.synchronize()
 per_block = e0.elapsed_time(e1) / (5 * len(layers))
+# the same blocks replayed from a CUDA graph (no host launch cost): if this is much faster, the
+# eager number above is host-bound
+g = torch.cuda.CUDAGraph()
+gs = torch.cuda.Stream()
+with torch.cuda.stream(gs):
+    with torch.cuda.graph(g, stream=gs):
+        for l in layers:
+            F.masked_block_forward(l, b, x, kv, y_act=y, ws=ws, stream=gs)
+g.replay()
+torch.cuda.synchronize()
+e0.record()
+for _ in range(5):
+    g.replay()
+e1.record()
+torch.cuda.synchronize()
+graph_block = e0.elapsed_time(e1) / (5 * len(layers))
 F.fps_profile_enable(1)
 for l in layers:
     F.masked_block_forward(l, b, x, kv, y_act=y, ws=ws)
@@ -55,6 +71,6 @@ P = C.POINTER(C.c_double)
 F.fps_profile_read(ms.ctypes.data_as(P), fl.ctypes.data_as(P), None, cnt.ctypes.data_as(C.POINTER(C.c_int64)))
 F.fps_profile_enable(0)
 names = ["gemm", "attn", "ln", "rows"]
-print(f"{cfg} {kind} flags={flags} rows={sum(ns)}: {per_block:.4f} ms/block | " +
+print(f"{cfg} {kind} flags={flags} rows={sum(ns)}: {per_block:.4f} ms/block (graph {graph_block:.4f}) | " +
       " ".join(f"{names[k]} {ms[k] / len(layers):.4f}ms" + (f" {fl[k] / ms[k] / 1e9:.0f}TF/s" if fl[k] else "")
                for k in range(4)))
