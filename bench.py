@@ -634,8 +634,9 @@ def main():
                 "achieved": gemm_achieved, "peak": bf16_sust, "unit": "TFLOP/s",
                 "frac": gemm_achieved / bf16_sust, "peak_source": f"{src} bf16_tflops_sustained",
                 "traffic": ncu_traffic("gemm_tcgen05"),
-                "traffic_source": "dram__bytes_read.sum + dram__bytes_write.sum per launch, "
-                                  "ncu --set full capture in profiles/ (one masked block's GEMMs)",
+                "traffic_source": "dram__bytes_read.sum + dram__bytes_write.sum per launch, from "
+                                  "the newest ncu --set full captures in profiles/*_traffic.json "
+                                  "(masked-block GEMMs at the bench's shapes)",
                 "algorithmic_bytes_per_launch": by[0] / max(cnt[0], 1),
                 "avg_launch_ms": gemm_avg_ms,
                 "flops_per_launch": fl[0] / max(cnt[0], 1)}
