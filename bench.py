@@ -506,6 +506,8 @@ def main():
     COPY_CTAS = args.copy_ctas
     layers, mod, cache = build_engine_inputs(F, w, args.mode, device, n_entries, location,
                                              args.copy_method)
+    wbytes = sum(t.numel() * t.element_size() for l in layers for t in l.t.values())
+    base_cfg["l2"] = f"inputs > L2 ({wbytes / 1e9:.1f} GB of weights streamed per step)"
     base_cfg["cache_tier"] = "pinned host DRAM" if location == 0 else "device HBM (NEXT-1)"
     base_cfg["h2d_method"] = ["SM row gather", "batched DMA of the unmasked row runs", "DMA of whole entries"][args.copy_method]
     torch.cuda.synchronize()
