@@ -68,3 +68,26 @@ def test_attention_large_logits_lazy_rescale(F, kernel):
     ref = attention(q, k, v, heads)
     check_close(to_np(out)[:n], ref, TOL["bf16"], "rescale")
     check_close(to_np(out)[n:], ref, TOL["bf16"], "rescale (second tile of the pair)")
+
+
+@pytest.mark.parametrize("d,heads", [(128, 3), (64, 10)])
+def test_short_key_sets(F, d, heads):
+    """Every request <= 128 keys (the SDXL cross-attention over a 77-token prompt): the
+    register-tile kernel, with key counts off every 8 / 16 boundary, ragged query tiles, an
+    empty request and large logits."""
+    g = synth.rng(700 + d)
+    H = d * heads
+    n_active = [300, 1, 0, 129, 77, 16]
+    L = [77, 1, 5, 128, 120, 33]
+    q = synth.latent(g, sum(n_active), H, "bf16")
+    kv = synth.bf16_round(synth.latent(g, sum(L), 2 * H, "bf16") * 3.0)
+    out = F.masked_attention(to_dev(q, "bf16"), to_dev(kv, "bf16"), n_active, L, heads)
+    torch.cuda.synchronize()
+    got = to_np(out)
+    qo, ko = 0, 0
+    for n, l in zip(n_active, L):
+        if n:
+            ref = attention(q[qo:qo + n], kv[ko:ko + l, :H], kv[ko:ko + l, H:], heads)
+            check_close(got[qo:qo + n], ref, TOL["bf16"], f"short attention n={n} L={l}")
+        qo += n
+        ko += l
