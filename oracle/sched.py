@@ -98,16 +98,32 @@ def route(req, workers, cost_fn, max_batch):
     return best
 
 
-def simulate_serving(reqs, n_workers, max_batch, step_latency, policy="mask_aware"):
+def masked_tokens(r):
+    """Token-granularity load of a request (§6.5): its masked image tokens."""
+    return int(math.floor(r.ratio * r.L_img + 0.5))
+
+
+def simulate_serving(reqs, n_workers, max_batch, step_latency, policy="mask_aware",
+                     batching="continuous", interrupt_ms=0.0):
     """Discrete-event simulation of the cluster (Fig. 8 workflow, L191-L199).
 
     reqs: list of Req sorted by arrival. step_latency(batch) -> ms of one denoising step.
-    policy: "mask_aware" (Alg. 2), "round_robin" (request-level), "least_requests".
-    Returns {rid: (arrival, finish)}."""
+    policy (router, §6.5): "mask_aware" (Alg. 2), "round_robin" and "least_requests"
+    (request granularity), "least_tokens" (token granularity: fewest masked tokens assigned).
+    batching (worker, §4.3, §6.4; reading R27):
+      "continuous"  FlashPS: requests join / leave the running batch at step boundaries (L237),
+                    pre- / post-processing run in other processes (disaggregated, L235);
+      "strawman"    the same, but each request's preprocessing (when it joins) and
+                    postprocessing (when it leaves) run in the worker's main process: every
+                    such event adds `interrupt_ms` before the worker's next step (L233);
+      "static"      a batch is formed only when the worker is idle and runs until all of its
+                    requests finish; later requests wait (L228).
+    Returns {rid: (arrival, finish of its last denoising step)}."""
     workers = [[] for _ in range(n_workers)]         # assigned, unfinished
     running = [[] for _ in range(n_workers)]         # joined the running batch
     remaining = {}
     busy = [False] * n_workers
+    joined = set()
     held = []
     out = {}
     ev = []
@@ -127,6 +143,8 @@ def simulate_serving(reqs, n_workers, max_batch, step_latency, policy="mask_awar
             elif policy == "round_robin":
                 wid = min(free, key=lambda w: ((w - rr[0]) % n_workers))
                 rr[0] = (wid + 1) % n_workers
+            elif policy == "least_tokens":
+                wid = min(free, key=lambda w: (sum(masked_tokens(q) for q in workers[w]), w))
             else:
                 wid = min(free, key=lambda w: (len(workers[w]), w))
         if wid is None:
@@ -135,16 +153,25 @@ def simulate_serving(reqs, n_workers, max_batch, step_latency, policy="mask_awar
         workers[wid].append(r)
         remaining[r.rid] = r.steps
         if not busy[wid]:
-            start_step(wid, now)
+            start_step(wid, now, 0)
 
-    def start_step(wid, now):
+    def start_step(wid, now, n_left):
         nonlocal seq
-        running[wid] = list(workers[wid])            # join at the step boundary (L237)
-        if not running[wid]:
+        if batching == "static":
+            batch = [r for r in running[wid] if remaining[r.rid] > 0]   # no newcomers ...
+            if not batch:
+                batch = list(workers[wid])           # ... until the whole batch is done
+        else:
+            batch = list(workers[wid])               # join at the step boundary (L237)
+        new = [r for r in batch if r.rid not in joined]
+        joined.update(r.rid for r in new)
+        running[wid] = batch
+        if not batch:
             busy[wid] = False
             return
         busy[wid] = True
-        heapq.heappush(ev, (now + step_latency(running[wid]), 0, seq, "step", wid))
+        extra = interrupt_ms * (len(new) + n_left) if batching == "strawman" else 0.0
+        heapq.heappush(ev, (now + extra + step_latency(batch), 0, seq, "step", wid))
         seq += 1
 
     while ev:
@@ -153,12 +180,14 @@ def simulate_serving(reqs, n_workers, max_batch, step_latency, policy="mask_awar
             assign(obj, now)
             continue
         wid = obj
+        n_left = 0
         for r in running[wid]:
             remaining[r.rid] -= 1
             if remaining[r.rid] == 0:
                 workers[wid].remove(r)               # leave at the step boundary (L237)
                 out[r.rid] = (r.arrival, now)
+                n_left += 1
         while held and len(workers[wid]) < max_batch:
             assign(held.pop(0), now)
-        start_step(wid, now)
+        start_step(wid, now, n_left)
     return out

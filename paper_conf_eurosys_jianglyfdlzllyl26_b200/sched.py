@@ -48,8 +48,10 @@ def fit_linear(x, y):
 class Request:
     """What the scheduler knows about a request: its active rows n and unmasked rows u."""
 
-    def __init__(self, rid, n_active, L, arrival=0.0, steps=28):
+    def __init__(self, rid, n_active, L, arrival=0.0, steps=28, tokens=None):
         self.rid, self.n, self.L, self.arrival, self.steps = rid, int(n_active), int(L), arrival, steps
+        # token-granularity load (§6.5): masked image tokens (defaults to the active rows)
+        self.tokens = int(n_active if tokens is None else tokens)
 
     @property
     def u(self):
@@ -131,10 +133,15 @@ def assign_all(reqs, n_workers, cost_fn, max_batch):
     return workers, held
 
 
-def simulate_serving(reqs, n_workers, max_batch, step_latency, policy="mask_aware"):
+def simulate_serving(reqs, n_workers, max_batch, step_latency, policy="mask_aware",
+                     batching="continuous", interrupt_ms=0.0):
     """Cluster of `n_workers` step-level continuous-batching workers (Fig. 8 workflow, L191-L199;
     L237: join / leave at step boundaries) fed by a router (Alg. 2, or a baseline policy:
-    "round_robin" = request-level, "least_requests" = fewest assigned requests).
+    "round_robin" = request-level, "least_requests" = fewest assigned requests, "least_tokens" =
+    fewest masked tokens assigned, §6.5).  Worker batching (§4.3, §6.4, reading R27):
+    "continuous" (FlashPS, pre/post-processing disaggregated), "strawman" (each join and leave
+    costs `interrupt_ms` of the worker's main process before its next step), "static" (a batch
+    forms only on an idle worker and runs until all its requests finish).
 
     reqs: Request objects with .arrival (ms) and .steps, sorted by arrival.
     step_latency(batch) -> ms of one denoising step of that batch (e.g. CostModel.step_latency,
@@ -144,18 +151,24 @@ def simulate_serving(reqs, n_workers, max_batch, step_latency, policy="mask_awar
     workers = [[] for _ in range(n_workers)]
     running = [[] for _ in range(n_workers)]
     remaining, busy, held, out, ev = {}, [False] * n_workers, [], {}, []
+    started = set()
     seq = 0
     for r in reqs:
         heapq.heappush(ev, (r.arrival, 1, seq, "arr", r))
         seq += 1
     rr = [0]
 
-    def start_step(wid, now):
+    def start_step(wid, now, finished=0):
         nonlocal seq
-        running[wid] = list(workers[wid])
+        cur = [r for r in running[wid] if remaining.get(r.rid, 0) > 0]
+        # static batching admits nobody while its batch still runs
+        running[wid] = cur if (batching == "static" and cur) else list(workers[wid])
         busy[wid] = bool(running[wid])
         if busy[wid]:
-            heapq.heappush(ev, (now + step_latency(running[wid]), 0, seq, "step", wid))
+            joining = [r for r in running[wid] if r.rid not in started]
+            started.update(r.rid for r in joining)
+            pause = interrupt_ms * (len(joining) + finished) if batching == "strawman" else 0.0
+            heapq.heappush(ev, (now + pause + step_latency(running[wid]), 0, seq, "step", wid))
             seq += 1
 
     def assign(r, now):
@@ -167,6 +180,8 @@ def simulate_serving(reqs, n_workers, max_batch, step_latency, policy="mask_awar
         elif policy == "round_robin":
             wid = min(free, key=lambda w: (w - rr[0]) % n_workers)
             rr[0] = (wid + 1) % n_workers
+        elif policy == "least_tokens":
+            wid = min(free, key=lambda w: (sum(q.tokens for q in workers[w]), w))
         else:
             wid = min(free, key=lambda w: (len(workers[w]), w))
         if wid is None:
@@ -183,14 +198,16 @@ def simulate_serving(reqs, n_workers, max_batch, step_latency, policy="mask_awar
             assign(obj, now)
             continue
         wid = obj
+        finished = 0
         for r in running[wid]:
             remaining[r.rid] -= 1
             if remaining[r.rid] == 0:
                 workers[wid].remove(r)
                 out[r.rid] = (r.arrival, now)
+                finished += 1
         while held and len(workers[wid]) < max_batch:
             assign(held.pop(0), now)
-        start_step(wid, now)
+        start_step(wid, now, finished)
     return out
 
 

@@ -15,8 +15,14 @@ def _pool(seed, n, rate_ms):
     return ratios, t
 
 
-@pytest.mark.parametrize("policy", ["mask_aware", "round_robin", "least_requests"])
-def test_des_matches_oracle(policy):
+@pytest.mark.parametrize("policy,batching", [("mask_aware", "continuous"),
+                                              ("round_robin", "continuous"),
+                                              ("least_requests", "continuous"),
+                                              ("least_tokens", "continuous"),
+                                              ("mask_aware", "static"),
+                                              ("mask_aware", "strawman"),
+                                              ("least_requests", "strawman")])
+def test_des_matches_oracle(policy, batching):
     ratios, t = _pool(3, 30, 40.0)
     L_img, L_txt = 4096, 512
     # one latency function for both sides: the oracle's cost model (suffix scan == library
@@ -25,9 +31,10 @@ def test_des_matches_oracle(policy):
     oreqs = [OS.Req(i, float(t[i]), float(ratios[i]), 6, L_img, L_txt) for i in range(30)]
     pcm = PS.CostModel(57, 3072, 12288, "kv", comp=(1 / 1.2e9, 0.05), load=(1 / 4.6e7, 0.01))
     preqs = [PS.Request(i, synth.n_masked_for(float(ratios[i]), L_img) + L_txt, L_img + L_txt,
-                        arrival=float(t[i]), steps=6) for i in range(30)]
-    o = OS.simulate_serving(oreqs, 3, 4, ocm.step_latency, policy)
-    p = PS.simulate_serving(preqs, 3, 4, pcm.step_latency, policy)
+                        arrival=float(t[i]), steps=6,
+                        tokens=synth.n_masked_for(float(ratios[i]), L_img)) for i in range(30)]
+    o = OS.simulate_serving(oreqs, 3, 4, ocm.step_latency, policy, batching, interrupt_ms=25.0)
+    p = PS.simulate_serving(preqs, 3, 4, pcm.step_latency, policy, batching, interrupt_ms=25.0)
     assert set(o) == set(p)
     for k in o:
         assert p[k][1] == pytest.approx(o[k][1], rel=1e-9)

@@ -5,7 +5,9 @@ L326).  Step latencies come from the Alg. 1 planner over the linear latency mode
 fitted on a B200 (`plan.fit` of a bench JSON line): a prediction from measured models, not a
 multi-GPU measurement (gpurun exposes one GPU).
 
-  python tools/serve_sweep.py profiles/r01_bench_c3_default.json > profiles/r01_serving_sim.json
+  python tools/serve_sweep.py profiles/r01e2_bench_c3.json > profiles/r01e2_serving_sim.json
+Also the NEXT-3 comparisons: router policies at token vs request granularity (§6.5) and the
+worker's batching policy -- static / strawman / disaggregated continuous (§6.4).
 """
 import json
 import os
@@ -37,19 +39,35 @@ def main():
     cap_img_s = 8 / (cm.step_latency(typical) * steps / 1e3)
     out = {"source_bench": sys.argv[1], "mode": mode, "fit": fit,
            "one_gpu_capacity_images_per_s": cap_img_s, "runs": []}
+    tokens = [synth.n_masked_for(float(m), L_img) for m in ratios]
+
+    def pool(rate):
+        t = np.cumsum(g.exponential(1e3 / rate, n_req))
+        return [sched.Request(i, n_active[i], L_img + L_txt, arrival=float(t[i]), steps=steps,
+                              tokens=tokens[i]) for i in range(n_req)]
+
     for n_gpu in (1, 2, 4, 8):
         for load_frac in (0.5, 0.8, 0.95):
-            rate = load_frac * cap_img_s * n_gpu                     # requests per second
-            gaps = g.exponential(1e3 / rate, n_req)
-            t = np.cumsum(gaps)
-            reqs = [sched.Request(i, n_active[i], L_img + L_txt, arrival=float(t[i]), steps=steps)
-                    for i in range(n_req)]
-            for pol in ("mask_aware", "least_requests", "round_robin"):
+            reqs = pool(load_frac * cap_img_s * n_gpu)              # requests per second
+            for pol in ("mask_aware", "least_requests", "least_tokens", "round_robin"):
                 res = sched.simulate_serving(reqs, n_gpu, 8, cm.step_latency, pol)
                 st = sched.latency_stats(res)
                 st.update(n_gpus=n_gpu, load=load_frac, policy=pol,
                           images_per_s=n_req / (st["makespan_ms"] / 1e3))
                 out["runs"].append(st)
+    # NEXT-3, §6.4 (Fig. 16-Left): one worker (max batch 8) with static batching, the strawman
+    # continuous batching whose pre/post-processing interrupts the denoising process (0.36 s per
+    # interruption, L398 -- the paper's CPU-side cost, taken as given), and FlashPS's
+    # disaggregated continuous batching; P95 latency at several loads
+    out["batching"] = []
+    for load_frac in (0.3, 0.5, 0.7):
+        reqs = pool(load_frac * cap_img_s)
+        for bat in ("continuous", "strawman", "static"):
+            res = sched.simulate_serving(reqs, 1, 8, cm.step_latency, "mask_aware", bat,
+                                         interrupt_ms=360.0)
+            st = sched.latency_stats(res)
+            st.update(n_gpus=1, load=load_frac, batching=bat, interrupt_ms=360.0)
+            out["batching"].append(st)
     print(json.dumps(out, indent=1))
 
 
