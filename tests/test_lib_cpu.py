@@ -124,3 +124,53 @@ def test_cross_step_planner_matches_oracle(mode):
         plan, lat = fps.plan_pipeline(Cw, Cwo, Lm, m, fin, cross_step=True)
         assert lat == pytest.approx(best, rel=1e-9)
         assert P.steady_step_latency(plan, Cw, Cwo, Lm, mode, fin) == pytest.approx(best, rel=1e-9)
+
+
+def _weights(kind, **kw):
+    """A descriptor with dummy (never dereferenced) 16-B aligned addresses."""
+    a = 1 << 20
+    w = fps.fps_block_weights(256, 2, 128, 512, _lib.FPS_BF16, a, 0, a, 0, a, 0, a, 0, kind)
+    for k, v in kw.items():
+        setattr(w, k, v)
+    return w
+
+
+def _batch(**kw):
+    b = fps.fps_varlen_batch()
+    b.n_req, b.total_q, b.total_k, b.max_q, b.max_k = 1, 8, 16, 8, 16
+    b.d_cu_q = b.d_cu_k = b.d_q_row = 1 << 20
+    for k, v in kw.items():
+        setattr(b, k, v)
+    return b
+
+
+@pytest.mark.parametrize("kind,wkw,bkw,what", [
+    (_lib.FPS_BLOCK_SDXL, {}, {}, "weight pointer"),                  # no cross-attention weights
+    (_lib.FPS_BLOCK_SDXL, dict(w_q2=1 << 20, w_kv2=1 << 20, w_o2=1 << 20), {}, "LayerNorm"),
+    (_lib.FPS_BLOCK_SDXL, dict(ln1_w=1 << 20, ln1_b=1 << 20, ln2_w=1 << 20, ln2_b=1 << 20,
+                               ln3_w=1 << 20, ln3_b=1 << 20, w_q2=1 << 20, w_kv2=1 << 20,
+                               w_o2=1 << 20, D_ctx=128), {}, "cu_ctx"),  # no prompt K|V
+    (_lib.FPS_BLOCK_DOUBLE, {}, {}, "text weight"),                    # no text-stream weights
+    (_lib.FPS_BLOCK_DOUBLE, dict(t_qkv=1 << 20, t_o=1 << 20, t_up=1 << 20, t_down=1 << 20), {},
+     "stream-major"),                                                  # no stream-major order
+    (7, {}, {}, "kind"),
+])
+def test_block_kind_validation_before_enqueue(kind, wkw, bkw, what):
+    """Missing per-kind inputs fail with FPS_EINVAL and a message, before anything is enqueued
+    (so this runs without a GPU)."""
+    w, b = _weights(kind, **wkw), _batch(**bkw)
+    import ctypes as C
+    with pytest.raises(fps.FlashPSError) as ei:
+        fps.fps_masked_block_forward(C.byref(w), C.byref(b), 1 << 20, 1 << 20, 1 << 20, None, None,
+                                     1 << 20, 1 << 30, None)
+    assert ei.value.code == _lib.FPS_EINVAL
+    assert what in str(ei.value)
+
+
+def test_geglu_pack_and_engine_desc_validation():
+    with pytest.raises(fps.FlashPSError) as ei:
+        fps.fps_geglu_pack(_lib.FPS_BF16, 1 << 20, None, 48, 64, 2 << 20, None, None)   # F % 32
+    assert ei.value.code == _lib.FPS_EINVAL
+    with pytest.raises(fps.FlashPSError) as ei:
+        fps.fps_geglu_pack(_lib.FPS_BF16, 1 << 20, None, 64, 64, 1 << 20, None, None)   # aliasing
+    assert ei.value.code == _lib.FPS_EINVAL
