@@ -172,3 +172,25 @@ def test_flux_stack_run_batch(F, mode, policy, plan):
         ref = S.masked_run(r["x0"], r["mask_np"], W, mods_o, deltas, used, mode, cache_np, heads,
                            n, step0=r["step0"], L_txt=L_txt)
         check_close(to_np(r["x"]), ref, stack_tol("bf16", N), f"Flux stack {mode} plan={used}")
+
+
+def test_double_c4_continuous_batch(F):
+    """configs[3] shapes on the double-stream block: 16 Flux-scale requests with masks 5-60 % in
+    one varlen batch (grouped GEMMs over ~21k image and 8k text rows, one joint attention); the
+    oracle checks the requests with the smallest and the largest mask, all rows."""
+    H, heads, Fd, L_img, L_txt = 3072, 24, 12288, 4096, 512
+    g = synth.rng(7300)
+    w = synth.block_weights(g, H, Fd, "bf16", "double")
+    reqs = []
+    for m in np.linspace(0.05, 0.60, 16):
+        mask = synth.token_mask(synth.mask_blobs(g, 64, 64, float(m)), L_txt)
+        M, U = build_mask_index(mask)
+        L = L_img + L_txt
+        reqs.append(dict(mask=mask, M=M, U=U, L=L, x=synth.latent(g, L, H, "bf16"),
+                         K=synth.latent(g, L, H, "bf16"), V=synth.latent(g, L, H, "bf16"),
+                         mod=synth.mod_table(g, 1, 1, H, "bf16", streams=2)[0, 0]))
+    y = _run(F, w, reqs, heads, "bf16", "kv", L_img)
+    cu = np.concatenate([[0], np.cumsum([len(r["M"]) for r in reqs])])
+    for i in (0, 15):
+        ref = _ref(w, [reqs[i]], heads, "kv", L_txt)
+        check_close(y[cu[i]:cu[i + 1]], ref, TOL["bf16"], f"C4 double request {i}")
