@@ -411,6 +411,9 @@ def main():
     ap.add_argument("--cross-step", type=int, default=1, choices=[0, 1],
                     help="cross-step prefetch (R26): the next step's loads start as soon as their "
                          "slots are consumed (1, default), or the per-step pipeline of Fig. 9 (0)")
+    ap.add_argument("--admission-reuse", type=int, default=1, choices=[0, 1],
+                    help="fps_run_batch reuses the previous call's admission when the batch is "
+                         "unchanged (1, default) or re-admits every call (0)")
     ap.add_argument("--no-extras", action="store_true", help="skip dense / Y-mode / profile legs")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()
@@ -549,6 +552,7 @@ def main():
                         mod_width=MODW, cross_step=bool(args.cross_step))
 
     eng = engine(0)
+    F.fps_engine_set_admission_reuse(eng.h, args.admission_reuse)
     log(f"[rank {rank}] timed run")
     with Clocks(local % n_dev) as clk:
         step_ms, launches = run_engine_timed(F, eng, reqs_dev, K, W, stream, load_stream, rank, world)

@@ -399,13 +399,21 @@ fps_status fps_engine_destroy(fps_engine_t e);
  * with the Alg. 1 plan, layer-ahead prefetch on `load_stream`, final replenish + Euler update
  * x <- x + delta_s * y (reading R21).  The engine's last plan is available below.
  * SDXL blocks: at admission the engine projects every request's d_ctx to the cross-attention
- * K|V of each SDXL block once (fps_context_kv); the prompt is fixed over the steps. */
+ * K|V of each SDXL block once (fps_context_kv); the prompt is fixed over the steps.
+ * Admission reuse: when a call's unfinished requests are exactly the previous call's (same
+ * order, same d_mask / d_x / d_ctx pointers and template_id) and none finished since, the call
+ * reuses that admission (mask index, batch metadata, prompt K|V, plan) and skips its host
+ * synchronisation -- so a serving loop that advances its batch one step per call pays it once
+ * per batch change.  Contract: a request's mask and prompt buffers must not be modified while
+ * the request is in flight (between its first and its last fps_run_batch call). */
 fps_status fps_run_batch(fps_engine_t e, fps_request* reqs, int32_t n_req, int32_t n_steps,
                          void* compute_stream, void* load_stream);
 /* Plan and predicted latency (ms) of the last step; use_cache may be NULL. */
 fps_status fps_engine_last_plan(fps_engine_t e, uint8_t* use_cache, double* latency_ms);
 /* Kernels the engine launched in its last fps_run_batch call (own kernels only). */
 int64_t fps_engine_last_launches(fps_engine_t e);
+/* Admission reuse on (default, on != 0) or off (every call re-admits; experiments). */
+void fps_engine_set_admission_reuse(fps_engine_t e, int32_t on);
 
 #ifdef __cplusplus
 }

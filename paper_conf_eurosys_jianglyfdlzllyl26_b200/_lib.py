@@ -112,6 +112,7 @@ _SIGS = [
     ("fps_run_batch", C.c_int, [vp, C.POINTER(fps_request), i32, i32, vp, vp], True),
     ("fps_engine_last_plan", C.c_int, [vp, P_u8, P_dbl], True),
     ("fps_engine_last_launches", i64, [vp], False),
+    ("fps_engine_set_admission_reuse", None, [vp, i32], False),
 ]
 
 EXPORTED = [s[0] for s in _SIGS]

@@ -17,6 +17,21 @@
 
 #include "kernels.h"
 
+namespace fps {
+struct Batch {
+  int n = 0;                       // requests in the running batch
+  std::vector<int> idx;            // index into the caller's reqs[]
+  std::vector<int> nq, nu;         // active / unmasked rows per request
+  int tq = 0, tu = 0, tk = 0, max_q = 0;
+  int32_t *cu_q, *cu_k, *cu_u, *q_row, *u_row, *mod_ids;      // device (inside d_meta)
+  int32_t *h_cu_q, *h_cu_k, *h_cu_u;                          // host (inside h_meta)
+  // double-stream blocks: [0] masked batch, [1] dense batch (device, inside e->d_sm)
+  int ti[2] = {0, 0};
+  int32_t *sm_perm[2] = {nullptr, nullptr}, *sm_kvrow[2] = {nullptr, nullptr};
+  int32_t *cu_img[2] = {nullptr, nullptr}, *cu_txt[2] = {nullptr, nullptr};
+};
+}  // namespace fps
+
 struct fps_engine {
   fps_engine_desc d{};
   std::vector<fps_block_weights> layers;
@@ -48,11 +63,25 @@ struct fps_engine {
   bool cross = false;
   int prev_ring = 0;
   cudaEvent_t final_consumed = nullptr;
+  // admission reuse: the last admitted batch and the identity of its live requests
+  fps::Batch last_B;
+  std::vector<const void*> last_key;
+  bool last_valid = false;
   float* d_delta = nullptr;
   // pinned host staging
   int32_t* h_meta = nullptr;
   int32_t *h_mids = nullptr, *h_uids = nullptr, *h_nm = nullptr, *h_off = nullptr;
   float* h_delta = nullptr;
+  // per-step host staging (modulation row ids, Euler coefficients): a small ring of pinned
+  // slots, each reused only after its previous H2D copy has executed -- the host may run
+  // several steps ahead of the device, and an async copy reads its pinned source when it runs
+  static constexpr int kStageRing = 4;
+  int32_t* h_stage = nullptr;
+  size_t stage_ints = 0;
+  cudaEvent_t stage_ev[kStageRing] = {};
+  long long stage_ctr = 0;
+  bool no_reuse = false;   // experiments: admit every call
+  bool call_start = false; // first step of a fps_run_batch call
   std::vector<cudaEvent_t> ready, consumed;
   cudaEvent_t step_start = nullptr, admit_done = nullptr;
   std::vector<uint8_t> last_plan;
@@ -78,7 +107,8 @@ static void free_engine(fps_engine* e) {
   int32_t* ib[] = {e->d_off, e->d_mids, e->d_uids, e->d_nm, e->d_meta};
   for (int32_t* p : ib) if (p) cudaFree(p);
   if (e->d_delta) cudaFree(e->d_delta);
-  void* hb[] = {e->h_meta, e->h_mids, e->h_uids, e->h_nm, e->h_off, e->h_delta};
+  void* hb[] = {e->h_meta, e->h_mids, e->h_uids, e->h_nm, e->h_off, e->h_delta, e->h_stage};
+  for (auto ev : e->stage_ev) if (ev) cudaEventDestroy(ev);
   for (void* p : hb) if (p) cudaFreeHost(p);
   for (auto ev : e->ready) if (ev) cudaEventDestroy(ev);
   for (auto ev : e->consumed) if (ev) cudaEventDestroy(ev);
@@ -215,6 +245,10 @@ fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out) {
   hmal((void**)&e->h_nm, d.max_batch * 4);
   hmal((void**)&e->h_off, (d.max_batch + 1) * 4);
   hmal((void**)&e->h_delta, d.max_batch * 4);
+  e->stage_ints = (size_t)d.n_layers * d.max_batch + d.max_batch;
+  hmal((void**)&e->h_stage, fps_engine::kStageRing * e->stage_ints * 4);
+  for (int i = 0; i < fps_engine::kStageRing && err == cudaSuccess; ++i)
+    err = cudaEventCreateWithFlags(&e->stage_ev[i], cudaEventDisableTiming);
   e->ready.assign(d.n_layers + 1, nullptr);
   e->consumed.assign(d.n_layers + 1, nullptr);
   for (int i = 0; i <= d.n_layers && err == cudaSuccess; ++i) {
@@ -249,22 +283,14 @@ fps_status fps_engine_last_plan(fps_engine_t e, uint8_t* use_cache, double* late
 
 int64_t fps_engine_last_launches(fps_engine_t e) { return e ? e->last_launches : -1; }
 
+void fps_engine_set_admission_reuse(fps_engine_t e, int32_t on) {
+  if (e) e->no_reuse = on == 0;
+}
+
 }  // extern "C"
 
 namespace fps {
 
-struct Batch {
-  int n = 0;                       // requests in the running batch
-  std::vector<int> idx;            // index into the caller's reqs[]
-  std::vector<int> nq, nu;         // active / unmasked rows per request
-  int tq = 0, tu = 0, tk = 0, max_q = 0;
-  int32_t *cu_q, *cu_k, *cu_u, *q_row, *u_row, *mod_ids;      // device (inside d_meta)
-  int32_t *h_cu_q, *h_cu_k, *h_cu_u;                          // host (inside h_meta)
-  // double-stream blocks: [0] masked batch, [1] dense batch (device, inside e->d_sm)
-  int ti[2] = {0, 0};
-  int32_t *sm_perm[2] = {nullptr, nullptr}, *sm_kvrow[2] = {nullptr, nullptr};
-  int32_t *cu_img[2] = {nullptr, nullptr}, *cu_txt[2] = {nullptr, nullptr};
-};
 
 static fps_status admit(fps_engine* e, fps_request* reqs, const std::vector<int>& live, Batch& B,
                         cudaStream_t cs) {
@@ -433,16 +459,20 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
   const bool kv = e->d.mode == FPS_MODE_KV;
   const std::vector<uint8_t>& use = e->last_plan;
   // adaLN vectors of every block for every request at its own step (rows of the table)
+  const int slot = (int)(e->stage_ctr++ % fps_engine::kStageRing);
+  FPS_CUDA_TRY(cudaEventSynchronize(e->stage_ev[slot]));   // its last copy has run
+  int32_t* mod_ids = e->h_stage + (size_t)slot * e->stage_ints;
+  float* h_delta = reinterpret_cast<float*>(mod_ids + (size_t)N * e->d.max_batch);
   if (e->d.d_mod_table) {
-    int32_t* mod_ids = e->h_meta + 3 * (e->d.max_batch + 1) + 2 * e->maxR;
     for (int l = 0; l < N; ++l)
       for (int i = 0; i < n; ++i) mod_ids[l * n + i] = l * e->d.n_steps + reqs[B.idx[i]].step;
     FPS_COPY_TRY(cs, cudaMemcpyAsync(B.mod_ids, mod_ids, (size_t)N * n * 4, cudaMemcpyHostToDevice, cs));
     FPS_TRY(launch_copy_rows(e->d.d_mod_table, B.mod_ids, nullptr, N * n, e->MW * e->elt,
                              e->mod_batch, cs));
   }
-  for (int i = 0; i < n; ++i) e->h_delta[i] = e->deltas[reqs[B.idx[i]].step];
-  FPS_COPY_TRY(cs, cudaMemcpyAsync(e->d_delta, e->h_delta, n * 4, cudaMemcpyHostToDevice, cs));
+  for (int i = 0; i < n; ++i) h_delta[i] = e->deltas[reqs[B.idx[i]].step];
+  FPS_COPY_TRY(cs, cudaMemcpyAsync(e->d_delta, h_delta, n * 4, cudaMemcpyHostToDevice, cs));
+  FPS_CUDA_TRY(cudaEventRecord(e->stage_ev[slot], cs));
 
   // ---- load schedule: ring loads (cached blocks in order) + KV-mode final Y load ----------
   std::vector<int> loads;                  // block of each ring load
@@ -461,7 +491,10 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
   FPS_CUDA_TRY(cudaEventRecord(e->step_start, cs));
   // per-step pipeline: this step's loads start with the step; cross-step prefetch (R26): a
   // load waits only for the previous step's consumer of its slot (below)
-  if (!e->cross) FPS_CUDA_TRY(stream_wait(ls, e->step_start, 0));
+  // (the first step of a call also waits: the caller's stream work before the call -- e.g. the
+  // host-to-device copy of the latents -- must not queue behind this step's cache loads)
+  if (!e->cross || e->call_start) FPS_CUDA_TRY(stream_wait(ls, e->step_start, 0));
+  e->call_start = false;
   auto issue = [&](int block, char* dst, size_t row_bytes, cudaEvent_t ev) -> fps_status {
     for (int i = 0; i < n; ++i) {
       const fps_request& r = reqs[B.idx[i]];
@@ -651,6 +684,7 @@ extern "C" fps_status fps_run_batch(fps_engine_t e, fps_request* reqs, int32_t n
   cudaStream_t cs = as_stream(compute_stream);
   cudaStream_t ls = load_stream ? as_stream(load_stream) : cs;
   const long long launches0 = g_launches;
+  e->call_start = true;
   int done_steps = 0;
   while (done_steps < n_steps) {
     std::vector<int> live;
@@ -659,17 +693,32 @@ extern "C" fps_status fps_run_batch(fps_engine_t e, fps_request* reqs, int32_t n
       if (!reqs[i].status) live.push_back(i);
     }
     if (live.empty()) break;
-    Batch B;
-    // a new batch: its index arrays and slots are rewritten, so the load stream drains first
-    FPS_CUDA_TRY(cudaEventRecord(e->final_consumed, ls));
-    FPS_CUDA_TRY(stream_wait(cs, e->final_consumed, 0));
-    e->prev_ring = 0;
-    FPS_TRY(admit(e, reqs, live, B, cs));
+    // the same live requests as the last admitted batch (same order, buffers and template):
+    // reuse its admission -- mask index, batch metadata, prompt K|V, plan -- without the host
+    // synchronisation (callers stepping one step per call, e.g. a serving loop, pay it once)
+    std::vector<const void*> key;
+    for (int i : live)
+      key.insert(key.end(), {reqs[i].d_mask, reqs[i].d_x, reqs[i].d_ctx,
+                             reinterpret_cast<const void*>((uintptr_t)reqs[i].template_id)});
+    const bool reuse = e->last_valid && !e->no_reuse && key == e->last_key;
+    Batch& B = e->last_B;
+    B.idx = live;           // same requests, possibly at other positions of the caller's array
+    if (!reuse) {
+      e->last_valid = false;
+      B = Batch{};
+      // a new batch: its index arrays and slots are rewritten, so the load stream drains first
+      FPS_CUDA_TRY(cudaEventRecord(e->final_consumed, ls));
+      FPS_CUDA_TRY(stream_wait(cs, e->final_consumed, 0));
+      e->prev_ring = 0;
+      FPS_TRY(admit(e, reqs, live, B, cs));
+      make_plan(e, B);
+      e->last_key = key;
+      e->last_valid = true;
+    }
     // load each request's latent into the contiguous batch buffer
     for (int i = 0; i < B.n; ++i)
       FPS_COPY_TRY(cs, cudaMemcpyAsync(e->x_full + (size_t)i * e->L * e->row_h, reqs[live[i]].d_x,
                                    (size_t)e->L * e->row_h, cudaMemcpyDeviceToDevice, cs));
-    make_plan(e, B);
     bool changed = false;
     while (done_steps < n_steps && !changed) {
       FPS_TRY(run_step(e, reqs, B, cs, ls));
@@ -680,6 +729,7 @@ extern "C" fps_status fps_run_batch(fps_engine_t e, fps_request* reqs, int32_t n
         if (r.step >= r.n_steps) {
           r.status = 1;
           changed = true;   // leaves at this step boundary (L237); the batch is rebuilt
+          e->last_valid = false;
         }
       }
     }

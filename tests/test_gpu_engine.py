@@ -349,3 +349,43 @@ def test_cross_step_prefetch_matches_oracle_and_per_step_bits(F, mode, plan, cop
                         f"cross={cross} {mode} plan={plan}")
     for a, b in zip(*outs):
         assert torch.equal(a, b)
+
+
+@pytest.mark.parametrize("mode", ["kv", "y"])
+def test_admission_reuse_step_by_step(F, mode):
+    """A serving loop advancing the batch one step per call (the same requests each call) reuses
+    the first call's admission -- no mask-index launch, no host sync -- and produces bit-identical
+    latents to one multi-step call; a changed request set is re-admitted."""
+    import ctypes as C
+    outs = []
+    for per_call in (False, True):
+        W, mods, deltas, cache_np, eng, reqs = _setup(F, mode, "bf16", 1, None, steps=4,
+                                                      cross_step=True)
+        for r in reqs:
+            r["step"] = 0
+        if per_call:
+            F.fps_profile_enable(1)
+            for _ in range(3):
+                eng.run_batch(reqs, 1)
+            torch.cuda.synchronize()
+            cnt = np.zeros(7, dtype=np.int64)
+            F.fps_profile_read(None, None, None, cnt.ctypes.data_as(C.POINTER(C.c_int64)))
+            F.fps_profile_enable(0)
+            assert cnt[6] == 1, f"mask index launched {cnt[6]} times for one batch"
+        else:
+            eng.run_batch(reqs, 3)
+        torch.cuda.synchronize()
+        outs.append([r["x"].clone() for r in reqs])
+    for a, b in zip(*outs):
+        assert torch.equal(a, b)
+    # a different request set (one request dropped) is admitted again and still matches the oracle
+    sub = reqs[:2]
+    for r in sub:
+        r["step0"] = r["step"]
+    F.fps_profile_enable(1)
+    eng.run_batch(sub, 1)
+    torch.cuda.synchronize()
+    cnt = np.zeros(7, dtype=np.int64)
+    F.fps_profile_read(None, None, None, cnt.ctypes.data_as(C.POINTER(C.c_int64)))
+    F.fps_profile_enable(0)
+    assert cnt[6] == 1
