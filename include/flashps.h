@@ -266,6 +266,9 @@ typedef struct {
   const int32_t* d_sm_kvrow;       /* [total_q] merged-buffer row of stream row i            */
   const int32_t* d_cu_img;         /* [n_req+1] prefix sums of active image rows            */
   const int32_t* d_cu_txt;         /* [n_req+1] prefix sums of text rows                    */
+  const int32_t* d_sm_inv;         /* [total_q] stream row of compact row r (the inverse of
+                                      d_sm_perm), or NULL: the block then reorders its rows
+                                      with two extra row copies                              */
 } fps_varlen_batch;
 
 /* SDXL block helpers (R24), run once per weight load / per request prompt, not per step.

@@ -144,7 +144,7 @@ class VarlenBatch:
 
     def __init__(self, n_active, L, q_row=None, mod=None, mode=FPS_MODE_KV, u_row=None,
                  u_src=None, n_unmasked=None, device="cuda", ctx_kv=None, n_ctx=None,
-                 act_ids=None, L_img=None, mod_stride=0):
+                 act_ids=None, L_img=None, mod_stride=0, stream_inverse=True):
         self.n_active = list(map(int, n_active))
         self.L = list(map(int, L))
         cu_q = np.concatenate([[0], np.cumsum(self.n_active)]).astype(np.int32)
@@ -174,12 +174,17 @@ class VarlenBatch:
                     perm.append(cu_q[r] + sel)
                     kvr.append(cu_k[r] + ids[sel])
                     (nt if st else ni).append(len(sel))
-            arrs = (np.concatenate(perm), np.concatenate(kvr),
-                    np.concatenate([[0], np.cumsum(ni)]), np.concatenate([[0], np.cumsum(nt)]))
+            pm = np.concatenate(perm)
+            inv = np.empty_like(pm)
+            inv[pm] = np.arange(len(pm))
+            arrs = (pm, np.concatenate(kvr), np.concatenate([[0], np.cumsum(ni)]),
+                    np.concatenate([[0], np.cumsum(nt)]), inv)
             self.sm = [torch.as_tensor(a.astype(np.int32), device=device) for a in arrs]
             self.c.total_q_img = int(sum(ni))
-            self.c.d_sm_perm, self.c.d_sm_kvrow, self.c.d_cu_img, self.c.d_cu_txt = \
-                (ptr(t) for t in self.sm)
+            (self.c.d_sm_perm, self.c.d_sm_kvrow, self.c.d_cu_img, self.c.d_cu_txt,
+             self.c.d_sm_inv) = (ptr(t) for t in self.sm)
+            if not stream_inverse:
+                self.c.d_sm_inv = None
         if ctx_kv is not None:       # SDXL blocks: request r's prompt K|V rows (n_ctx[r] each)
             cu_c = np.concatenate([[0], np.cumsum(n_ctx)]).astype(np.int32)
             self.h_cu_ctx, self.cu_ctx, self.ctx_kv = cu_c, torch.tensor(cu_c, device=device), ctx_kv

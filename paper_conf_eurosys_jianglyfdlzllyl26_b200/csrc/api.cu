@@ -114,17 +114,17 @@ fps_status launch_attention(int dtype, const void* q, const void* kv, void* o, i
                             int head_dim, const int32_t* d_cu_q, const int32_t* d_cu_k,
                             const int32_t* h_cu_q, const int32_t* h_cu_k, int n_req, int total_q,
                             int max_q, int max_k, cudaStream_t s, int ldo,
-                            const AttnScratch* sc) {
+                            const AttnScratch* sc, const int32_t* o_map) {
   (void)max_k;
   if (total_q <= 0) return FPS_OK;
   prof::begin(s);
   fps_status st;
   if (!(g_disable_tc & 2) && attention_tc_supported(dtype, head_dim) && h_cu_q && h_cu_k)
     st = launch_attention_tc(q, kv, o, heads, head_dim, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s,
-                             ldo, sc);
+                             ldo, sc, o_map);
   else
     st = launch_attention_simt(dtype, q, kv, o, heads, head_dim, d_cu_q, d_cu_k, n_req, total_q, s,
-                               ldo);
+                               ldo, o_map);
   if (prof::enabled() && h_cu_q && h_cu_k) {
     // algorithmic work: QK^T and PV, 4 n_r L_r H FLOPs; bytes: Q, O once + K|V once per request
     double fl = 0, by = 0;
@@ -282,14 +282,23 @@ static fps_status double_block_forward(const fps_block_weights* w, const fps_var
   auto at = [&](char* base, int st, size_t width = 0) {
     return base + (size_t)rows0[st] * (width ? width : rowb);
   };
+  // Without reordering copies: the norms read x through the stream-major order, the O
+  // projection reads its residual through it, and the attention writes its output rows
+  // straight to their stream-major positions (d_sm_inv).  The copy path remains for the
+  // attention kernels forced by tests.
+  const bool direct = b->d_sm_inv != nullptr && (g_attn_force == 0 || g_attn_force == 3);
   if (tq > 0) {
-    FPS_TRY(launch_copy_rows(x_act, perm, nullptr, tq, (int)rowb, x_sm, s));
+    if (!direct) FPS_TRY(launch_copy_rows(x_act, perm, nullptr, tq, (int)rowb, x_sm, s));
     // a4 per stream; a5 for both streams in one grouped launch: Q -> request-major rows,
     // K|V -> merged key rows
     Epilogue ep[2] = {};
     for (int st = 0; st < 2; ++st) {
-      FPS_TRY(launch_ln_mod(dt, at(x_sm, st), nullptr, nrows[st], H, at(ws.h, st), cu[st],
-                            b->n_req, mod, 6 * H * st, s, nullptr, MS));
+      if (direct)
+        FPS_TRY(launch_ln_mod(dt, x_act, perm + rows0[st], nrows[st], H, at(ws.h, st), cu[st],
+                              b->n_req, mod, 6 * H * st, s, nullptr, MS));
+      else
+        FPS_TRY(launch_ln_mod(dt, at(x_sm, st), nullptr, nrows[st], H, at(ws.h, st), cu[st],
+                              b->n_req, mod, 6 * H * st, s, nullptr, MS));
       ep[st].bias = Bqkv[st];
       ep[st].out0 = ws.q; ep[st].ld0 = H; ep[st].map0 = perm + rows0[st];
       ep[st].out1 = kv; ep[st].ld1 = 2 * H; ep[st].map1 = kvrow + rows0[st];
@@ -313,15 +322,26 @@ static fps_status double_block_forward(const fps_block_weights* w, const fps_var
   // a6: joint attention of both streams' queries over the merged keys
   if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
   const AttnScratch sc = attn_scratch(ws, H, F, dt, tq, false);
-  FPS_TRY(launch_attention(dt, ws.q, kv, ws.ao, w->heads, w->head_dim, b->d_cu_q, b->d_cu_k,
-                           b->h_cu_q, b->h_cu_k, b->n_req, tq, b->max_q, b->max_k, s, 0, &sc));
-  FPS_TRY(launch_copy_rows(ws.ao, perm, nullptr, tq, (int)rowb, ao_sm, s));
+  if (direct) {
+    FPS_TRY(launch_attention(dt, ws.q, kv, ao_sm, w->heads, w->head_dim, b->d_cu_q, b->d_cu_k,
+                             b->h_cu_q, b->h_cu_k, b->n_req, tq, b->max_q, b->max_k, s, 0, &sc,
+                             b->d_sm_inv));
+  } else {
+    FPS_TRY(launch_attention(dt, ws.q, kv, ws.ao, w->heads, w->head_dim, b->d_cu_q, b->d_cu_k,
+                             b->h_cu_q, b->h_cu_k, b->n_req, tq, b->max_q, b->max_k, s, 0, &sc));
+    FPS_TRY(launch_copy_rows(ws.ao, perm, nullptr, tq, (int)rowb, ao_sm, s));
+  }
   // a7, a8: each projection one grouped launch over both streams (their own weights, adaLN
   // gates and request offsets); y written back in request-major order
   Epilogue eo[2] = {}, eu[2] = {}, ed[2] = {};
   for (int st = 0; st < 2; ++st) {   // x1 = x + gate1 (A Wo^T + bo)
     eo[st].bias = Bo[st];
-    eo[st].resid = at(x_sm, st); eo[st].ld_resid = H;
+    if (direct) {
+      eo[st].resid = x_act; eo[st].resid_map = perm + rows0[st];
+    } else {
+      eo[st].resid = at(x_sm, st);
+    }
+    eo[st].ld_resid = H;
     eo[st].gate = modp(st, 2); eo[st].gate_stride = MS; eo[st].cu = cu[st]; eo[st].n_req = b->n_req;
     eo[st].out0 = at(ws.x1, st); eo[st].ld0 = H; eo[st].split = H;
   }

@@ -259,6 +259,8 @@ struct Epilogue {
   int act_from;
   // fp32 residual stream (SDXL block, tcgen05 path only): out0 and/or resid hold fp32 rows
   int out0_f32, resid_f32;
+  // residual row of output row r: resid_map[r] (null -> r)
+  const int32_t* resid_map;
 };
 
 }  // namespace fps

@@ -29,6 +29,7 @@ struct Batch {
   int ti[2] = {0, 0};
   int32_t *sm_perm[2] = {nullptr, nullptr}, *sm_kvrow[2] = {nullptr, nullptr};
   int32_t *cu_img[2] = {nullptr, nullptr}, *cu_txt[2] = {nullptr, nullptr};
+  int32_t* sm_inv[2] = {nullptr, nullptr};
 };
 }  // namespace fps
 
@@ -211,7 +212,7 @@ fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out) {
   e->ws_bytes = fps_block_workspace_bytes(d.H, d.F, d.dtype, (int)R, (int)R);
   dmal(&e->ws, e->ws_bytes);
   dmal(&e->mod_batch, (size_t)d.n_layers * d.max_batch * e->MW * e->elt);
-  const size_t sm_ints = 2 * (2 * R + 2 * (d.max_batch + 1));
+  const size_t sm_ints = 2 * (3 * R + 2 * (d.max_batch + 1));
   if (e->has_double) {
     if (err == cudaSuccess) err = cudaMalloc((void**)&e->d_sm, sm_ints * 4);
     if (err == cudaSuccess) err = cudaHostAlloc((void**)&e->h_sm, sm_ints * 4, cudaHostAllocDefault);
@@ -351,9 +352,11 @@ static fps_status admit(fps_engine* e, fps_request* reqs, const std::vector<int>
   if (e->has_double) {
     // stream-major order (all image rows, then all text rows) of the masked and dense batches
     const int R = e->maxR, nb1 = e->d.max_batch + 1, Li = e->d.L_img;
+    const size_t per = 3 * (size_t)R + 2 * nb1;
     for (int v = 0; v < 2; ++v) {
-      int32_t* base = e->h_sm + (size_t)v * (2 * R + 2 * nb1);
+      int32_t* base = e->h_sm + (size_t)v * per;
       int32_t *perm = base, *kvr = base + R, *ci = base + 2 * R, *ct = ci + nb1;
+      int32_t* inv = ct + nb1;
       int k = 0;
       ci[0] = ct[0] = 0;
       for (int i = 0; i < n; ++i) {          // image rows
@@ -379,14 +382,15 @@ static fps_status admit(fps_engine* e, fps_request* reqs, const std::vector<int>
         }
         ct[i + 1] = ct[i] + (cnt - first);
       }
-      int32_t* dbase = e->d_sm + (size_t)v * (2 * R + 2 * nb1);
+      for (int j = 0; j < k; ++j) inv[perm[j]] = j;
+      int32_t* dbase = e->d_sm + (size_t)v * per;
       B.sm_perm[v] = dbase;
       B.sm_kvrow[v] = dbase + R;
       B.cu_img[v] = dbase + 2 * R;
       B.cu_txt[v] = dbase + 2 * R + nb1;
+      B.sm_inv[v] = dbase + 2 * R + 2 * nb1;
     }
-    FPS_COPY_TRY(cs, cudaMemcpyAsync(e->d_sm, e->h_sm, (size_t)2 * (2 * R + 2 * nb1) * 4,
-                                     cudaMemcpyHostToDevice, cs));
+    FPS_COPY_TRY(cs, cudaMemcpyAsync(e->d_sm, e->h_sm, 2 * per * 4, cudaMemcpyHostToDevice, cs));
   }
   if (e->n_sdxl) {
     // SDXL blocks: the prompt is fixed over the steps, so each block's cross-attention K|V
@@ -555,12 +559,14 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
   vb.d_sm_kvrow = B.sm_kvrow[0];
   vb.d_cu_img = B.cu_img[0];
   vb.d_cu_txt = B.cu_txt[0];
+  vb.d_sm_inv = B.sm_inv[0];
   fps_varlen_batch vd = vb;             // dense: every row of every request is active
   vd.total_q_img = B.ti[1];
   vd.d_sm_perm = B.sm_perm[1];
   vd.d_sm_kvrow = B.sm_kvrow[1];
   vd.d_cu_img = B.cu_img[1];
   vd.d_cu_txt = B.cu_txt[1];
+  vd.d_sm_inv = B.sm_inv[1];
   vd.total_q = B.tk;
   vd.max_q = e->L;
   vd.d_cu_q = B.cu_k;

@@ -20,7 +20,8 @@ __device__ __forceinline__ void epilogue_store(const Epilogue& ep, int r, int c0
     for (int e = 0; e < NC; ++e) v[e] = gelu_tanh(v[e]);
   }
   if (ep.resid) {
-    const T* res = reinterpret_cast<const T*>(ep.resid) + (size_t)r * ep.ld_resid + c0;
+    const int rr = ep.resid_map ? __ldg(ep.resid_map + r) : r;
+    const T* res = reinterpret_cast<const T*>(ep.resid) + (size_t)rr * ep.ld_resid + c0;
     if (ep.gate) {
       const int q = find_req(ep.cu, ep.n_req, r);
       const T* g = reinterpret_cast<const T*>(ep.gate) + (size_t)q * ep.gate_stride + c0;

@@ -677,7 +677,7 @@ __global__ void __launch_bounds__(512, 1)
                     __nv_bfloat16* __restrict__ O, const int32_t* __restrict__ cu_q,
                     const int32_t* __restrict__ cu_k, int n_req, int heads, float scale_log2, int ldo,
                     __nv_bfloat16* __restrict__ Opart, float2* __restrict__ ML, long long part_stride,
-                    int total_q) {
+                    int total_q, const int32_t* __restrict__ o_map) {
   using Cfg = Attn3Cfg<D>;
   constexpr int CHUNK = 128 * 128;
   extern __shared__ uint8_t smem_raw[];
@@ -963,9 +963,10 @@ __global__ void __launch_bounds__(512, 1)
     }
     for (int t = 0; t < ntl; ++t) {
       const int grow = q0 + t * 128 + row;
+      const int orow_i = (o_map && grow < q_end) ? __ldg(o_map + grow) : grow;
       __nv_bfloat16* orow = nsplit > 1
           ? Opart + split * part_stride + (size_t)grow * (heads * D) + head * D
-          : O + (size_t)grow * ldo + head * D;
+          : O + (size_t)orow_i * ldo + head * D;
       if (nk == 0) {                                       // no keys: defined zero output
         if (grow < q_end) {
           for (int c = 0; c < D; c += 8) *reinterpret_cast<uint4*>(orow + c) = make_uint4(0, 0, 0, 0);
@@ -1012,7 +1013,8 @@ __global__ void __launch_bounds__(256) attn_combine_kernel(const __nv_bfloat16* 
                                                            const float2* __restrict__ ML,
                                                            long long part_stride, int nsplit,
                                                            int total_q, int heads,
-                                                           __nv_bfloat16* __restrict__ O, int ldo) {
+                                                           __nv_bfloat16* __restrict__ O, int ldo,
+                                                           const int32_t* __restrict__ o_map) {
   pdl_trigger();
   pdl_wait();
   constexpr int C8 = D / 8;
@@ -1042,7 +1044,8 @@ __global__ void __launch_bounds__(256) attn_combine_kernel(const __nv_bfloat16* 
     const float inv = wsum > 0.f ? 1.0f / wsum : 0.f;
 #pragma unroll
     for (int e = 0; e < 8; ++e) acc[e] *= inv;
-    *reinterpret_cast<uint4*>(O + (size_t)row * ldo + head * D + c8 * 8) = Vec16<__nv_bfloat16>::pack(acc);
+    const int orow = o_map ? __ldg(o_map + row) : row;
+    *reinterpret_cast<uint4*>(O + (size_t)orow * ldo + head * D + c8 * 8) = Vec16<__nv_bfloat16>::pack(acc);
   }
 }
 
@@ -1145,7 +1148,7 @@ template <int D>
 static fps_status launch_d3(const void* q, const void* kv, void* o, int heads,
                             const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
                             const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo,
-                            const AttnScratch* sc) {
+                            const AttnScratch* sc, const int32_t* o_map) {
   using Cfg = Attn3Cfg<D>;
   const int H = heads * D;
   int pairs = 0, min_nk = 1 << 30;
@@ -1174,14 +1177,14 @@ static fps_status launch_d3(const void* q, const void* kv, void* o, int heads,
   auto* ML = S > 1 ? reinterpret_cast<float2*>(sc->ml) : nullptr;
   FPS_CUDA_TRY(launch_k(attn_tc3_kernel<D>, dim3(pairs, heads, S), dim3(512), Cfg::SMEM, s, tq, tkv,
                         reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads,
-                        scale_log2, ldo, Opart, ML, part_stride, total_q));
+                        scale_log2, ldo, Opart, ML, part_stride, total_q, o_map));
   if (S > 1) {
     count_launch();
     const long long n = (long long)total_q * heads * (D / 8);
     const int grid = (int)std::min<long long>((n + 255) / 256, kNumSMs * 8LL);
     FPS_CUDA_TRY(launch_k(attn_combine_kernel<D>, dim3(grid), dim3(256), 0, s,
                           (const __nv_bfloat16*)Opart, (const float2*)ML, part_stride, S, total_q,
-                          heads, reinterpret_cast<__nv_bfloat16*>(o), ldo));
+                          heads, reinterpret_cast<__nv_bfloat16*>(o), ldo, o_map));
   }
 #ifdef FPS_ATTN_TRACE
   {
@@ -1205,7 +1208,7 @@ static fps_status launch_d3(const void* q, const void* kv, void* o, int heads,
 fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads, int head_dim,
                                const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
                                const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo,
-                               const AttnScratch* sc) {
+                               const AttnScratch* sc, const int32_t* o_map) {
   if (ldo == 0) ldo = heads * head_dim;
   if (ldo < heads * head_dim || ldo % 8 != 0)
     return fail(FPS_EINVAL, "attention_tc: output row stride %d", ldo);
@@ -1220,9 +1223,11 @@ fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads
   // A+B operand reads exceed the 128 B/clk smem port), which ate the latency it saved.
   if (g_attn_force == 0 || g_attn_force == 3) {
     if (head_dim == 128)
-      return launch_d3<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo, sc);
-    return launch_d3<64>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo, sc);
+      return launch_d3<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo, sc,
+                            o_map);
+    return launch_d3<64>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo, sc, o_map);
   }
+  if (o_map) return fail(FPS_EUNSUPPORTED, "attention: output row map needs the default kernel");
   if (g_attn_force == 2) {
     if (head_dim == 128)
       return launch_d2<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo);

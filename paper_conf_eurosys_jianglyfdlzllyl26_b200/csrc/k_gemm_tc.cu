@@ -57,12 +57,13 @@ __device__ __forceinline__ void group_coords(int tile, int T0, int num_m0, int n
 // column ranges (K/V scatter into the merged key buffer).
 struct RowCtx {
   const __nv_bfloat16* gate;
-  int row, orow0, orow1;
+  int row, orow0, orow1, rrow;
   bool ok;
 };
 __device__ __forceinline__ RowCtx row_ctx(const Epilogue& ep, int M, int row) {
-  RowCtx c{nullptr, row, row, row, row < M};
+  RowCtx c{nullptr, row, row, row, row, row < M};
   if (c.ok) {
+    if (ep.resid_map) c.rrow = __ldg(ep.resid_map + row);
     if (ep.gate)
       c.gate = reinterpret_cast<const __nv_bfloat16*>(ep.gate) +
                (size_t)find_req(ep.cu, ep.n_req, row) * ep.gate_stride;
@@ -86,12 +87,12 @@ __device__ __forceinline__ void chunk_load(const Epilogue& ep, const RowCtx& rc,
     const bool ok = rc.ok && c0 < N;
     in.bv[g] = (bias && ok) ? __ldg(reinterpret_cast<const uint4*>(bias + c0)) : make_uint4(0, 0, 0, 0);
     if (ep.resid_f32) {
-      const float* rf = reinterpret_cast<const float*>(ep.resid) + (size_t)row * ep.ld_resid + c0;
+      const float* rf = reinterpret_cast<const float*>(ep.resid) + (size_t)rc.rrow * ep.ld_resid + c0;
       in.rv[g] = (resid && ok) ? __ldg(reinterpret_cast<const uint4*>(rf)) : make_uint4(0, 0, 0, 0);
       in.rv[g + 4] = (resid && ok) ? __ldg(reinterpret_cast<const uint4*>(rf + 4)) : make_uint4(0, 0, 0, 0);
     } else {
       in.rv[g] = (resid && ok)
-                     ? __ldg(reinterpret_cast<const uint4*>(resid + (size_t)row * ep.ld_resid + c0))
+                     ? __ldg(reinterpret_cast<const uint4*>(resid + (size_t)rc.rrow * ep.ld_resid + c0))
                      : make_uint4(0, 0, 0, 0);
     }
     in.gv[g] = (rc.gate && ok) ? __ldg(reinterpret_cast<const uint4*>(rc.gate + c0))

@@ -76,7 +76,8 @@ __global__ void __launch_bounds__(128) attn_simt_kernel(const T* __restrict__ q,
                                                         T* __restrict__ o, int heads, int total_q,
                                                         const int32_t* __restrict__ cu_q,
                                                         const int32_t* __restrict__ cu_k,
-                                                        int n_req, int ldo) {
+                                                        int n_req, int ldo,
+                                                        const int32_t* __restrict__ o_map) {
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   const int i = gw / heads, j = gw - (gw / heads) * heads;
   if (i >= total_q) return;
@@ -106,7 +107,7 @@ __global__ void __launch_bounds__(128) attn_simt_kernel(const T* __restrict__ q,
     for (int e = 0; e < DPL; ++e) acc[e] = acc[e] * c + p * to_f(vr[e]);
     m = mn;
   }
-  T* op = o + (size_t)i * ldo + j * d + lane * DPL;
+  T* op = o + (size_t)(o_map ? __ldg(o_map + i) : i) * ldo + j * d + lane * DPL;
   const float inv = 1.0f / l;
 #pragma unroll
   for (int e = 0; e < DPL; ++e) op[e] = from_f<T>(acc[e] * inv);
@@ -114,7 +115,8 @@ __global__ void __launch_bounds__(128) attn_simt_kernel(const T* __restrict__ q,
 
 fps_status launch_attention_simt(int dtype, const void* q, const void* kv, void* o, int heads,
                                  int head_dim, const int32_t* cu_q, const int32_t* cu_k,
-                                 int n_req, int total_q, cudaStream_t s, int ldo) {
+                                 int n_req, int total_q, cudaStream_t s, int ldo,
+                                 const int32_t* o_map) {
   if (total_q <= 0) return FPS_OK;
   if (ldo == 0) ldo = heads * head_dim;
   const long long warps = (long long)total_q * heads;
@@ -124,10 +126,11 @@ fps_status launch_attention_simt(int dtype, const void* q, const void* kv, void*
     if (dtype == FPS_BF16)                                                                   \
       attn_simt_kernel<__nv_bfloat16, D / 32><<<grid, 128, 0, s>>>(                          \
           (const __nv_bfloat16*)q, (const __nv_bfloat16*)kv, (__nv_bfloat16*)o, heads,       \
-          total_q, cu_q, cu_k, n_req, ldo);                                                       \
+          total_q, cu_q, cu_k, n_req, ldo, o_map);                                                \
     else                                                                                     \
       attn_simt_kernel<float, D / 32><<<grid, 128, 0, s>>>(                                  \
-          (const float*)q, (const float*)kv, (float*)o, heads, total_q, cu_q, cu_k, n_req, ldo);  \
+          (const float*)q, (const float*)kv, (float*)o, heads, total_q, cu_q, cu_k, n_req, ldo, \
+          o_map);                                                                            \
     count_launch();                                                                          \
     FPS_LAUNCH_CHECK();                                                                      \
     return FPS_OK;                                                                           \

@@ -58,19 +58,21 @@ struct AttnScratch {
   size_t ml_bytes;
 };
 // a6: o[i, head] = softmax(q_i k^T / sqrt(d)) v over the request's merged keys; o rows are
-// ldo elements apart (0 = heads * head_dim)
+// ldo elements apart (0 = heads * head_dim); o_map: query row i is written to output row
+// o_map[i] (null -> i; default tensor-core and SIMT kernels only)
 fps_status launch_attention(int dtype, const void* q, const void* kv, void* o, int heads,
                             int head_dim, const int32_t* d_cu_q, const int32_t* d_cu_k,
                             const int32_t* h_cu_q, const int32_t* h_cu_k, int n_req, int total_q,
                             int max_q, int max_k, cudaStream_t s, int ldo = 0,
-                            const AttnScratch* sc = nullptr);
+                            const AttnScratch* sc = nullptr, const int32_t* o_map = nullptr);
 fps_status launch_attention_simt(int dtype, const void* q, const void* kv, void* o, int heads,
                                  int head_dim, const int32_t* cu_q, const int32_t* cu_k,
-                                 int n_req, int total_q, cudaStream_t s, int ldo = 0);
+                                 int n_req, int total_q, cudaStream_t s, int ldo = 0,
+                                 const int32_t* o_map = nullptr);
 fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads, int head_dim,
                                const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
                                const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo = 0,
-                               const AttnScratch* sc = nullptr);
+                               const AttnScratch* sc = nullptr, const int32_t* o_map = nullptr);
 bool attention_tc_supported(int dtype, int head_dim);
 
 // true if fps_cache_prefetch also overwrites rows outside U (copy_method 2): fresh rows written

@@ -38,7 +38,7 @@ def _problem(seed, dtype, H, heads, Fd, L_img, L_txt, ratios):
     return w, reqs
 
 
-def _run(F, w, reqs, heads, dtype, mode, L_img, dense=False):
+def _run(F, w, reqs, heads, dtype, mode, L_img, dense=False, inv=True):
     dt = F.DTYPE_CODE[dtype]
     H = w["img"]["w_o"].shape[0]
     bw = F.BlockWeights(w, heads, dt)
@@ -47,7 +47,8 @@ def _run(F, w, reqs, heads, dtype, mode, L_img, dense=False):
     mod = to_dev(np.stack([r["mod"] for r in reqs]), dtype)
     if dense:
         x = to_dev(np.concatenate([r["x"] for r in reqs]), dtype)
-        b = F.VarlenBatch(Ls, Ls, mod=mod, act_ids=[np.arange(L) for L in Ls], L_img=L_img)
+        b = F.VarlenBatch(Ls, Ls, mod=mod, act_ids=[np.arange(L) for L in Ls], L_img=L_img,
+                          stream_inverse=inv)
         y, _ = F.dense_block_forward(bw, b, x)
         torch.cuda.synchronize()
         return to_np(y)
@@ -65,7 +66,7 @@ def _run(F, w, reqs, heads, dtype, mode, L_img, dense=False):
     qd, ud = torch.as_tensor(q_row).cuda(), torch.as_tensor(u_row).cuda()
     b = F.VarlenBatch([len(r["M"]) for r in reqs], Ls, q_row=qd, mod=mod, mode=F.MODE_CODE[mode],
                       u_row=ud, u_src=ud, n_unmasked=[len(r["U"]) for r in reqs],
-                      act_ids=[r["M"] for r in reqs], L_img=L_img)
+                      act_ids=[r["M"] for r in reqs], L_img=L_img, stream_inverse=inv)
     y = F.masked_block_forward(bw, b, x_act, kv, xu=xu)
     torch.cuda.synchronize()
     return to_np(y)
@@ -194,3 +195,16 @@ def test_double_c4_continuous_batch(F):
     for i in (0, 15):
         ref = _ref(w, [reqs[i]], heads, "kv", L_txt)
         check_close(y[cu[i]:cu[i + 1]], ref, TOL["bf16"], f"C4 double request {i}")
+
+
+@pytest.mark.parametrize("mode,flags", [("kv", 0), ("y", 0), ("kv", 16)])
+def test_double_copy_path(F, mode, flags):
+    """Without the inverse stream order (or with a forced one-tile attention kernel, which has no
+    output row map) the block reorders its rows with explicit copies: same results."""
+    w, reqs = _problem(7110, "bf16", 256, 2, 1024, 576, 40, [0.1, 0.5])
+    F.fps_set_disable_tc(flags)
+    try:
+        y = _run(F, w, reqs, 2, "bf16", mode, 576, inv=flags != 0)
+    finally:
+        F.fps_set_disable_tc(0)
+    check_close(y, _ref(w, reqs, 2, mode, 40), TOL["bf16"], f"double copy path {mode} {flags}")
