@@ -291,14 +291,11 @@ static fps_status double_block_forward(const fps_block_weights* w, const fps_var
     if (!direct) FPS_TRY(launch_copy_rows(x_act, perm, nullptr, tq, (int)rowb, x_sm, s));
     // a4 per stream; a5 for both streams in one grouped launch: Q -> request-major rows,
     // K|V -> merged key rows
+    // both streams' norms in one launch (rows >= ti: the text stream's vectors)
+    FPS_TRY(launch_ln_mod2(dt, direct ? x_act : x_sm, direct ? perm : nullptr, tq, H, ws.h, cu[0],
+                           cu[1], ti, b->n_req, mod, 0, 6 * H, s, MS));
     Epilogue ep[2] = {};
     for (int st = 0; st < 2; ++st) {
-      if (direct)
-        FPS_TRY(launch_ln_mod(dt, x_act, perm + rows0[st], nrows[st], H, at(ws.h, st), cu[st],
-                              b->n_req, mod, 6 * H * st, s, nullptr, MS));
-      else
-        FPS_TRY(launch_ln_mod(dt, at(x_sm, st), nullptr, nrows[st], H, at(ws.h, st), cu[st],
-                              b->n_req, mod, 6 * H * st, s, nullptr, MS));
       ep[st].bias = Bqkv[st];
       ep[st].out0 = ws.q; ep[st].ld0 = H; ep[st].map0 = perm + rows0[st];
       ep[st].out1 = kv; ep[st].ld1 = 2 * H; ep[st].map1 = kvrow + rows0[st];
@@ -346,9 +343,9 @@ static fps_status double_block_forward(const fps_block_weights* w, const fps_var
     eo[st].out0 = at(ws.x1, st); eo[st].ld0 = H; eo[st].split = H;
   }
   FPS_TRY(launch_gemm_grouped(dt, ao_sm, Wo[0], Wo[1], ti, tt, H, H, eo[0], eo[1], s));
+  FPS_TRY(launch_ln_mod2(dt, ws.x1, nullptr, tq, H, ws.h2, cu[0], cu[1], ti, b->n_req, mod,
+                         3 * H, 6 * H, s, MS));
   for (int st = 0; st < 2; ++st) {
-    FPS_TRY(launch_ln_mod(dt, at(ws.x1, st), nullptr, nrows[st], H, at(ws.h2, st), cu[st],
-                          b->n_req, mod, 6 * H * st + 3 * H, s, nullptr, MS));
     eu[st].bias = Bup[st]; eu[st].act = 1;
     eu[st].out0 = at(ws.u, st, (size_t)F * e); eu[st].ld0 = F; eu[st].split = F;
     ed[st].bias = Bdn[st];

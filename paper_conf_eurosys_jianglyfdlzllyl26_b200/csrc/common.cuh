@@ -237,6 +237,11 @@ struct LnMod {
   float one;
   const int32_t* cu;
   int n_req;
+  // two row groups in one launch (double-stream block): rows >= split take their request
+  // from cu2 (indexed from split) and their vectors `soff` elements further on
+  int split;
+  int soff;
+  const int32_t* cu2;
 };
 
 struct Epilogue {

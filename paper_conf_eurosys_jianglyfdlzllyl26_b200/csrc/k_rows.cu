@@ -246,7 +246,10 @@ __global__ void __launch_bounds__(128) ln_mod_kernel(const T* __restrict__ x,
   const T* shift = nullptr;
   const T* scale = nullptr;
   if (mod) {
-    const size_t off = md.stride ? (size_t)find_req(md.cu, md.n_req, warp) * md.stride : 0;
+    const bool g2 = warp >= md.split;
+    const size_t off = (md.stride ? (size_t)find_req(g2 ? md.cu2 : md.cu, md.n_req,
+                                                     g2 ? warp - md.split : warp) * md.stride : 0) +
+                       (g2 ? md.soff : 0);
     shift = md.shift + off;
     scale = md.scale + off;
   }
@@ -291,7 +294,10 @@ __global__ void __launch_bounds__(128) ln_mod_row_kernel(const T* __restrict__ x
   const uint4* sh = nullptr;
   const uint4* sc = nullptr;
   if (mod) {
-    const size_t off = md.stride ? (size_t)find_req(md.cu, md.n_req, row) * md.stride : 0;
+    const bool g2 = row >= md.split;
+    const size_t off = (md.stride ? (size_t)find_req(g2 ? md.cu2 : md.cu, md.n_req,
+                                                     g2 ? row - md.split : row) * md.stride : 0) +
+                       (g2 ? md.soff : 0);
     sh = reinterpret_cast<const uint4*>(md.shift + off);
     sc = reinterpret_cast<const uint4*>(md.scale + off);
   }
@@ -525,9 +531,27 @@ fps_status launch_ln_affine_f32in(const float* x, int n, int H, void* out, const
 
 template <typename T>
 static LnMod<T> ln_params(const void* shift, const void* scale, int stride, float one,
-                          const int32_t* cu, int n_req) {
+                          const int32_t* cu, int n_req, int split = 0x7fffffff, int soff = 0,
+                          const int32_t* cu2 = nullptr) {
   return LnMod<T>{reinterpret_cast<const T*>(shift), reinterpret_cast<const T*>(scale), stride, one,
-                  cu, n_req};
+                  cu, n_req, split, soff, cu2};
+}
+
+fps_status launch_ln_mod2(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
+                          const int32_t* cu, const int32_t* cu2, int split, int n_req,
+                          const void* mod, int shift_off, int soff, cudaStream_t s,
+                          int mod_stride) {
+  if (n <= 0) return FPS_OK;
+  const size_t e = dtype == FPS_BF16 ? 2 : 4;
+  const char* sh = mod ? (const char*)mod + (size_t)shift_off * e : nullptr;
+  const char* sc = mod ? sh + (size_t)H * e : nullptr;
+  if (dtype == FPS_BF16)
+    return ln_mod_t<__nv_bfloat16>(
+        x, rows, n, H, out,
+        ln_params<__nv_bfloat16>(sh, sc, mod_stride, 1.0f, cu, n_req, split, soff, cu2), s, nullptr);
+  return ln_mod_t<float>(x, rows, n, H, out,
+                         ln_params<float>(sh, sc, mod_stride, 1.0f, cu, n_req, split, soff, cu2), s,
+                         nullptr);
 }
 
 fps_status launch_ln_mod(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,

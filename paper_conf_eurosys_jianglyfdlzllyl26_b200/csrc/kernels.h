@@ -19,6 +19,12 @@ fps_status launch_copy_rows(const void* src, const int32_t* src_ids, const int32
 fps_status launch_ln_mod(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
                          const int32_t* cu, int n_req, const void* mod, int shift_off,
                          cudaStream_t s, const int32_t* out_rows = nullptr, int mod_stride = 0);
+// a4 over two row groups in one launch (double-stream block): rows >= split use cu2 (rows
+// counted from split) and vectors soff elements after the first group's
+fps_status launch_ln_mod2(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
+                          const int32_t* cu, const int32_t* cu2, int split, int n_req,
+                          const void* mod, int shift_off, int soff, cudaStream_t s,
+                          int mod_stride);
 // a4 (SDXL block, R24): out[out_rows ? out_rows[i] : i] = LN(x[rows ? rows[i] : i]) * gamma + beta
 fps_status launch_ln_affine(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
                             const void* gamma, const void* beta, cudaStream_t s,
