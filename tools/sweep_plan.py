@@ -12,12 +12,13 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C3"); ap.add_argument("--mode", default="kv")
 ap.add_argument("--tier", default="host"); ap.add_argument("--steps", type=int, default=8)
 ap.add_argument("--cross-step", type=int, default=1)
+ap.add_argument("--block", default="flux")
 ap.add_argument("ks", type=int, nargs="+")
 a = ap.parse_args()
 w = bench.WORKLOADS[a.config]
 dev = torch.device("cuda", 0)
 loc = {"host": 0, "hbm": 1}[a.tier]
-w = dict(w, block="seq")
+w = dict(w, block=a.block)
 layers, mod, cache = bench.build_engine_inputs(F, w, a.mode, dev, 2 * (w["layers"] + 1), loc,
                                                2 if loc == 1 else 1)
 pool = bench.make_requests(w, w["batch"], bench.SEED)
@@ -32,7 +33,8 @@ for k in a.ks:
     plan = [0] * (N - k) + [1] * k
     eng = F.Engine(layers, w["heads"], F.MODE_CODE[a.mode], F.FPS_BF16, w["L_img"], w["L_txt"],
                    len(reqs), w["steps"], synth.delta_table(w["steps"]), cache, mod_table=mod,
-                   slots=0, plan_policy=3, plan=plan, cross_step=bool(a.cross_step))
+                   slots=0, plan_policy=3, plan=plan, cross_step=bool(a.cross_step),
+                   mod_width=12 * w["H"] if a.block == "flux" else 0)
     ms, _ = bench.run_engine_timed(F, eng, reqs, a.steps, 3, torch.cuda.current_stream(), ls, 0, 1)
     print(f"k={k:2d} cached: {ms:.2f} ms/step", flush=True)
     del eng
