@@ -174,3 +174,26 @@ def test_geglu_pack_and_engine_desc_validation():
     with pytest.raises(fps.FlashPSError) as ei:
         fps.fps_geglu_pack(_lib.FPS_BF16, 1 << 20, None, 64, 64, 1 << 20, None, None)   # aliasing
     assert ei.value.code == _lib.FPS_EINVAL
+
+
+def test_header_is_plain_c_and_links(tmp_path):
+    """include/flashps.h is a C ABI: it compiles as strict C99 and C++17, and a C program links
+    against libflashps.so and calls it (no torch, no Python)."""
+    import shutil
+    import subprocess
+    if not shutil.which("gcc"):
+        pytest.skip("no gcc")
+    inc = os.path.dirname(HDR)
+    src = tmp_path / "use.c"
+    src.write_text('#include "flashps.h"\n'
+                   'int main(void) { fps_block_weights w = {0}; fps_varlen_batch b = {0};\n'
+                   '  fps_engine_desc d = {0}; (void)w; (void)b; (void)d;\n'
+                   '  return fps_abi_version() == FPS_ABI_VERSION ? 0 : 1; }\n')
+    for cc, std in (("gcc", "-std=c99"), ("g++", "-std=c++17")):
+        subprocess.run([cc, std, "-Wall", "-Werror", "-I", inc, "-x", "c" if cc == "gcc" else "c++",
+                        "-c", str(src), "-o", str(tmp_path / "use.o")], check=True)
+    libdir = os.path.dirname(_lib.LIB_PATH)
+    exe = tmp_path / "use"
+    subprocess.run(["gcc", "-std=c99", "-I", inc, str(src), "-L", libdir, "-l:libflashps.so",
+                    f"-Wl,-rpath,{libdir}", "-o", str(exe)], check=True)
+    assert subprocess.run([str(exe)]).returncode == 0
