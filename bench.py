@@ -414,6 +414,9 @@ def main():
     ap.add_argument("--admission-reuse", type=int, default=1, choices=[0, 1],
                     help="fps_run_batch reuses the previous call's admission when the batch is "
                          "unchanged (1, default) or re-admits every call (0)")
+    ap.add_argument("--kv-transition", type=int, default=1, choices=[0, 1],
+                    help="KV-mode: run the last dense block before the cached suffix as a masked "
+                         "block over the fresh full input (R28; 0 = dense, for A/B)")
     ap.add_argument("--no-extras", action="store_true", help="skip dense / Y-mode / profile legs")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()
@@ -456,6 +459,7 @@ def main():
     base_cfg["h2d_method"] = ["SM row gather", "batched DMA of the unmasked row runs", "DMA of whole entries"][args.copy_method]
     base_cfg["parallelism"] = f"request-parallel x{world} (Alg. 2 routing)"
     base_cfg["cross_step_prefetch"] = bool(args.cross_step)
+    base_cfg["kv_transition_block"] = bool(args.kv_transition) and args.mode == "kv"
 
     if args.impl == "reference":
         if rank != 0:
@@ -546,10 +550,12 @@ def main():
     deltas = synth.delta_table(w["steps"])
 
     def engine(policy, mode=args.mode, the_cache=cache):
-        return F.Engine(layers, w["heads"], F.MODE_CODE[mode], F.FPS_BF16, w["L_img"], w["L_txt"],
-                        max(len(reqs_dev), 1), w["steps"], deltas, the_cache, mod_table=mod,
-                        slots=0, plan_policy=policy, cost_model=cm.as_engine_model(), L_ctx=L_ctx,
-                        mod_width=MODW, cross_step=bool(args.cross_step))
+        e = F.Engine(layers, w["heads"], F.MODE_CODE[mode], F.FPS_BF16, w["L_img"], w["L_txt"],
+                     max(len(reqs_dev), 1), w["steps"], deltas, the_cache, mod_table=mod,
+                     slots=0, plan_policy=policy, cost_model=cm.as_engine_model(), L_ctx=L_ctx,
+                     mod_width=MODW, cross_step=bool(args.cross_step))
+        F.fps_engine_set_kv_transition(e.h, args.kv_transition)
+        return e
 
     eng = engine(0)
     F.fps_engine_set_admission_reuse(eng.h, args.admission_reuse)

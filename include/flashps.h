@@ -417,6 +417,13 @@ fps_status fps_engine_last_plan(fps_engine_t e, uint8_t* use_cache, double* late
 int64_t fps_engine_last_launches(fps_engine_t e);
 /* Admission reuse on (default, on != 0) or off (every call re-admits; experiments). */
 void fps_engine_set_admission_reuse(fps_engine_t e, int32_t on);
+/* KV-mode transition block on (default, on != 0) or off (experiments).  In a KV-mode plan the
+ * last uncached block before the cached suffix has only its active rows' outputs read later
+ * (the next block takes its unmasked K|V from the cache), so the engine runs it as a masked
+ * block whose K|V projection covers every row of the fresh full input: the same values for
+ * every row read afterwards at the cost of the active rows' attention and MLP (R28).
+ * Off: that block runs densely over all rows. */
+void fps_engine_set_kv_transition(fps_engine_t e, int32_t on);
 
 #ifdef __cplusplus
 }

@@ -114,6 +114,7 @@ _SIGS = [
     ("fps_engine_last_plan", C.c_int, [vp, P_u8, P_dbl], True),
     ("fps_engine_last_launches", i64, [vp], False),
     ("fps_engine_set_admission_reuse", None, [vp, i32], False),
+    ("fps_engine_set_kv_transition", None, [vp, i32], False),
 ]
 
 EXPORTED = [s[0] for s in _SIGS]

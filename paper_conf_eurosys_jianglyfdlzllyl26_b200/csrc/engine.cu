@@ -82,6 +82,7 @@ struct fps_engine {
   cudaEvent_t stage_ev[kStageRing] = {};
   long long stage_ctr = 0;
   bool no_reuse = false;   // experiments: admit every call
+  bool no_transition = false;   // experiments: run a KV-mode plan's last dense block densely
   bool call_start = false; // first step of a fps_run_batch call
   std::vector<cudaEvent_t> ready, consumed;
   cudaEvent_t step_start = nullptr, admit_done = nullptr;
@@ -286,6 +287,10 @@ int64_t fps_engine_last_launches(fps_engine_t e) { return e ? e->last_launches :
 
 void fps_engine_set_admission_reuse(fps_engine_t e, int32_t on) {
   if (e) e->no_reuse = on == 0;
+}
+
+void fps_engine_set_kv_transition(fps_engine_t e, int32_t on) {
+  if (e) e->no_transition = on == 0;
 }
 
 }  // extern "C"
@@ -595,7 +600,21 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
     vd.d_ctx_kv = vb.d_ctx_kv;
     vd.d_cu_ctx = vb.d_cu_ctx;
     vd.h_cu_ctx = vb.h_cu_ctx;
-    if (!use[l]) {
+    if (!use[l] && kv && rep_full && !e->no_transition && l + 1 < N && use[l + 1]) {
+      // KV-mode transition block (reading R28): the last uncached block before the cached
+      // suffix.  Block l+1 reads only its masked rows' input (its unmasked K|V come from the
+      // cache), so block l's unmasked output rows are dead: run it as a masked block over the
+      // fresh full input -- K|V of all rows from cur_full (the Y-mode path with d_xu = the
+      // full input), Q / attention / O / MLP on the active rows only.  Same values for every
+      // row that is read afterwards; nothing loaded for it.
+      FPS_TRY(launch_copy_rows(cur_full, B.q_row, nullptr, B.tq, (int)e->row_h, e->act[act_cur], cs));
+      fps_varlen_batch vt = vb;
+      vt.mode = FPS_MODE_Y;
+      FPS_TRY(fps_masked_block_forward(w, &vt, e->act[act_cur], e->act[act_cur ^ 1], e->kv_scratch,
+                                       cur_full, nullptr, e->ws, e->ws_bytes, cs));
+      act_cur ^= 1;
+      rep_full = false;
+    } else if (!use[l]) {
       if (!rep_full) {
         // Y-mode cached -> uncached: rebuild the full input from act rows M and the cached
         // output rows U of block l-1 (reading R11)

@@ -389,3 +389,26 @@ def test_admission_reuse_step_by_step(F, mode):
     F.fps_profile_read(None, None, None, cnt.ctypes.data_as(C.POINTER(C.c_int64)))
     F.fps_profile_enable(0)
     assert cnt[6] == 1
+
+
+@pytest.mark.parametrize("kind", ["seq", "par"])
+@pytest.mark.parametrize("plan", [[0, 0, 1, 1], [0, 1, 1, 1]])
+def test_kv_transition_block_matches_oracle_and_dense_run(F, kind, plan):
+    """KV-mode transition block (R28): the last uncached block before the cached suffix runs as
+    a masked block over the fresh full input.  With it on (default) and off (dense), the latents
+    match the oracle's plan (whose uncached blocks are dense over all rows) and each other."""
+    outs = []
+    for on in (1, 0):
+        W, mods, deltas, cache_np, eng, reqs = _setup(F, "kv", "bf16", 3, plan, N=4, kind=kind)
+        F.fps_engine_set_kv_transition(eng.h, on)
+        for r in reqs:
+            r["step0"] = r["step"]
+        eng.run_batch(reqs, 2)
+        torch.cuda.synchronize()
+        assert eng.last_plan()[0] == plan
+        ref = _oracle(W, mods, deltas, cache_np, reqs, plan, "kv", 2, 2)
+        for r, x in zip(reqs, ref):
+            check_close(to_np(r["x"]), x, stack_tol("bf16", 4), f"transition={on} {kind} {plan}")
+        outs.append([to_np(r["x"]) for r in reqs])
+    for a, b in zip(*outs):
+        check_close(a, b, stack_tol("bf16", 4), "transition on vs off")
