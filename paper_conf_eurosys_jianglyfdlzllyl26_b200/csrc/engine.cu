@@ -12,6 +12,7 @@
 //            block on all tokens (L211); transitions gather / rebuild rows;
 //   replenish: y[M] from the last block, y[U] from the cache (L157); Euler x += delta_s y (R21).
 #include <algorithm>
+#include <cmath>
 #include <cstring>
 #include <vector>
 
@@ -290,7 +291,10 @@ void fps_engine_set_admission_reuse(fps_engine_t e, int32_t on) {
 }
 
 void fps_engine_set_kv_transition(fps_engine_t e, int32_t on) {
-  if (e) e->no_transition = on == 0;
+  if (e && e->no_transition != (on == 0)) {
+    e->no_transition = on == 0;
+    e->last_valid = false;             // the plan depends on it: re-admit on the next call
+  }
 }
 
 }  // extern "C"
@@ -427,16 +431,18 @@ static void make_plan(fps_engine* e, const Batch& B) {
   const double ec = e->d.cost_model[3] > 0 ? e->d.cost_model[3] : 0.01;
   double by = 0, byf = 0;
   const double H = e->d.H, F = e->d.F, L = e->L, Lc = e->d.L_ctx;
-  std::vector<double> Cw(N), Cwo(N), Lm(N);
+  std::vector<double> Cw(N), Cwo(N), Ct(N), Lm(N);
   for (int l = 0; l < N; ++l) {
     const int kind = e->layers[l].kind;
-    double fm = 0, fd = 0;
+    double fm = 0, fd = 0, ft = 0;
     for (int i = 0; i < B.n; ++i) {
       fm += flops_block(e->d.mode, B.nq[i], L, H, F, kind, Lc);
       fd += flops_block(FPS_MODE_KV, L, L, H, F, kind, Lc);
+      ft += flops_block(FPS_MODE_Y, B.nq[i], L, H, F, kind, Lc);
     }
     Cw[l] = a * fm + b;
     Cwo[l] = a * fd + b;
+    Ct[l] = a * ft + b;     // transition block (R28): Y-mode work over the fresh full input
   }
   for (int i = 0; i < B.n; ++i) {
     // rows the load moves: U, or the whole entry for the whole-entry DMA method
@@ -446,7 +452,32 @@ static void make_plan(fps_engine* e, const Batch& B) {
   }
   for (int l = 0; l < N; ++l) Lm[l] = by > 0 ? c * by + ec : 0.0;
   const double fin = byf > 0 ? c * byf + ec : 0.0;
-  if (e->d.plan_policy == 0) {
+  const bool trans = e->d.mode == FPS_MODE_KV && !e->no_transition;
+  auto latency = e->cross ? fps_pipeline_latency_cross : fps_pipeline_latency;
+  // KV-mode plans are the N+1 suffixes; with the transition block (R28) the prefix's last block
+  // costs Ct instead of Cwo, so each suffix is priced with its own cost vector.
+  auto priced = [&](const uint8_t* use) {
+    int k = 0;
+    while (k < N && !use[k]) ++k;
+    if (!trans || k == 0 || k == N) return latency(use, Cw.data(), Cwo.data(), Lm.data(), N,
+                                                   e->d.mode, fin);
+    std::vector<double> C2(Cwo);
+    C2[k - 1] = Ct[k - 1];
+    return latency(use, Cw.data(), C2.data(), Lm.data(), N, e->d.mode, fin);
+  };
+  if (e->d.plan_policy == 0 && trans) {
+    std::vector<uint8_t> use(N);
+    double best = 0;
+    for (int k = 0; k <= N; ++k) {        // k = uncached prefix length; ties -> more cached
+      for (int l = 0; l < N; ++l) use[l] = l >= k ? 1 : 0;
+      const double t = priced(use.data());
+      if (k == 0 || t < best - 1e-12 * std::max(1.0, std::fabs(best))) {
+        best = t;
+        e->last_plan = use;
+      }
+    }
+    e->last_latency = best;
+  } else if (e->d.plan_policy == 0) {
     if (e->cross)
       fps_plan_pipeline_cross(Cw.data(), Cwo.data(), Lm.data(), N, e->d.mode, fin,
                               e->last_plan.data(), &e->last_latency);
@@ -456,8 +487,7 @@ static void make_plan(fps_engine* e, const Batch& B) {
   } else {
     for (int l = 0; l < N; ++l)
       e->last_plan[l] = e->d.plan_policy == 1 ? 1 : e->d.plan_policy == 2 ? 0 : e->fixed_plan[l];
-    e->last_latency = (e->cross ? fps_pipeline_latency_cross : fps_pipeline_latency)(
-        e->last_plan.data(), Cw.data(), Cwo.data(), Lm.data(), N, e->d.mode, fin);
+    e->last_latency = priced(e->last_plan.data());
   }
 }
 

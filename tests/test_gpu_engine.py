@@ -20,7 +20,7 @@ def F():
 
 def _setup(F, mode, dtype, plan_policy, plan=None, N=3, steps=3, H=256, heads=2, Fd=512,
            L_img=256, L_txt=16, n_req=3, slots=0, copy_method=0, seed=5000, location=0,
-           kind="seq", cross_step=False):
+           kind="seq", cross_step=False, cost_model=(0.0, 0.0, 0.0, 0.0)):
     g = synth.rng(seed)
     W = synth.stack_weights(g, N, H, Fd, dtype, kind)
     mods = synth.mod_table(g, N, steps, H, dtype)
@@ -49,7 +49,8 @@ def _setup(F, mode, dtype, plan_policy, plan=None, N=3, steps=3, H=256, heads=2,
     layers = [F.BlockWeights(w, heads, dt) for w in W]
     eng = F.Engine(layers, heads, m, dt, L_img, L_txt, max_batch=4, n_steps=steps, deltas=deltas,
                    cache=cache, mod_table=to_dev(mods, dtype), slots=slots,
-                   plan_policy=plan_policy, plan=plan, cross_step=cross_step)
+                   plan_policy=plan_policy, plan=plan, cross_step=cross_step,
+                   cost_model=cost_model)
     reqs = []
     ratios = [0.1, 0.45, 0.25, 0.6][:n_req]
     for i in range(n_req):
@@ -412,3 +413,44 @@ def test_kv_transition_block_matches_oracle_and_dense_run(F, kind, plan):
         outs.append([to_np(r["x"]) for r in reqs])
     for a, b in zip(*outs):
         check_close(a, b, stack_tol("bf16", 4), "transition on vs off")
+
+
+@pytest.mark.parametrize("cross", [False, True])
+def test_kv_transition_planner_prices_each_suffix(F, cross):
+    """With the transition block (R28) the engine's KV-mode planner prices every suffix plan
+    with its prefix's last block at the transition cost (Y-mode FLOPs over the fresh input):
+    its plan and latency are the argmin of the library's pipeline model over the N+1 suffixes
+    with those cost vectors; off, it is the library planner's."""
+    from paper_conf_eurosys_jianglyfdlzllyl26_b200 import sched as Sd
+    N, H, Fd, L_img, L_txt = 6, 256, 512, 256, 16
+    L = L_img + L_txt
+    cm = (1.0e-9, 0.01, 1.3e-6, 0.01)      # ms / FLOP, ms, ms / byte, ms: a dense-prefix optimum
+    for on in (1, 0):
+        W, mods, deltas, cache_np, eng, reqs = _setup(F, "kv", "bf16", 0, None, N=N,
+                                                      cross_step=cross, cost_model=cm)
+        F.fps_engine_set_kv_transition(eng.h, on)
+        eng.run_batch(reqs, 1)
+        torch.cuda.synchronize()
+        plan, lat = eng.last_plan()
+        nq = [int(r["mask_np"].sum()) for r in reqs]
+        Cw = [cm[0] * sum(Sd.block_flops("kv", n, L, H, Fd) for n in nq) + cm[1]] * N
+        Cwo = [cm[0] * sum(Sd.block_flops("dense", n, L, H, Fd) for n in nq) + cm[1]] * N
+        Ct = cm[0] * sum(Sd.block_flops("y", n, L, H, Fd) for n in nq) + cm[1]
+        nu = sum(L - n for n in nq)
+        Lm = [cm[2] * nu * 2 * H * 2 + cm[3]] * N
+        fin = cm[2] * nu * H * 2 + cm[3]
+        best = None
+        for k in range(N + 1):
+            use = [0] * k + [1] * (N - k)
+            C2 = list(Cwo)
+            if on and 0 < k < N:
+                C2[k - 1] = Ct
+            t = F.pipeline_latency(use, Cw, C2, Lm, F.FPS_MODE_KV, fin, cross_step=cross)
+            if best is None or t < best[0] - 1e-12 * max(1.0, abs(best[0])):
+                best = (t, use)
+        if not on:
+            ref_plan, ref_lat = F.plan_pipeline(Cw, Cwo, Lm, F.FPS_MODE_KV, fin, cross_step=cross)
+            assert list(ref_plan) == best[1] and ref_lat == pytest.approx(best[0], rel=1e-9)
+        assert plan == best[1], (on, plan, best)
+        assert 0 < sum(plan) < N, plan
+        assert lat == pytest.approx(best[0], rel=1e-9)
