@@ -13,6 +13,7 @@ ap.add_argument("--config", default="C3"); ap.add_argument("--mode", default="kv
 ap.add_argument("--tier", default="host"); ap.add_argument("--steps", type=int, default=8)
 ap.add_argument("--cross-step", type=int, default=1)
 ap.add_argument("--block", default="flux")
+ap.add_argument("--kv-transition", type=int, default=1)
 ap.add_argument("ks", type=int, nargs="+")
 a = ap.parse_args()
 w = bench.WORKLOADS[a.config]
@@ -27,6 +28,10 @@ g = torch.Generator(device=dev).manual_seed(bench.SEED)
 reqs = [dict(template_id=i, step=0, n_steps=w["steps"], mask=torch.as_tensor(p["mask_np"]).to(dev),
              x=torch.randn(L, w["H"], generator=g, device=dev).to(torch.bfloat16))
         for i, p in enumerate(pool)]
+L_ctx = bench.SDXL_CTX[0] if a.block == "sdxl" else 0
+for r in reqs:
+    if L_ctx:
+        r["ctx"] = torch.randn(*bench.SDXL_CTX, generator=g, device=dev).to(torch.bfloat16)
 ls = torch.cuda.Stream()
 N = w["layers"]
 for k in a.ks:
@@ -34,7 +39,8 @@ for k in a.ks:
     eng = F.Engine(layers, w["heads"], F.MODE_CODE[a.mode], F.FPS_BF16, w["L_img"], w["L_txt"],
                    len(reqs), w["steps"], synth.delta_table(w["steps"]), cache, mod_table=mod,
                    slots=0, plan_policy=3, plan=plan, cross_step=bool(a.cross_step),
-                   mod_width=12 * w["H"] if a.block == "flux" else 0)
+                   mod_width=12 * w["H"] if a.block == "flux" else 0, L_ctx=L_ctx)
+    F.fps_engine_set_kv_transition(eng.h, a.kv_transition)
     ms, _ = bench.run_engine_timed(F, eng, reqs, a.steps, 3, torch.cuda.current_stream(), ls, 0, 1)
     print(f"k={k:2d} cached: {ms:.2f} ms/step", flush=True)
     del eng
