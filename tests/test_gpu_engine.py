@@ -278,7 +278,8 @@ def test_full_scale_stack_identical_input_invariant(F, mode):
     """configs[2] at its full size (57 Flux-scale blocks, 4096 + 512 tokens, m = 0.2): with the
     cache taken from the GPU's own dense template run on the identical input, the mask-aware
     step (every block cached) reproduces the dense step bit-for-bit -- a property that holds at
-    any size (L144/L157), checked where the fp64 oracle cannot run the whole stack."""
+    any size (L144/L157), checked where the fp64 oracle cannot run the whole stack.  So does
+    the bench's plan shape (uncached prefix, cached suffix)."""
     H, heads, Fd, L_img, L_txt, N, steps = 3072, 24, 12288, 4096, 512, 57, 1
     L = L_img + L_txt
     dev = torch.device("cuda")
@@ -315,9 +316,13 @@ def test_full_scale_stack_identical_input_invariant(F, mode):
         cache.store(0, 0, N, cur)
     torch.cuda.synchronize()
     outs = []
-    for policy in (1, 2):                 # every block cached vs every block dense
+    # every block cached, a 15-block uncached prefix (the bench's C3 plan: in KV-mode its last
+    # block is the transition block, R28), every block dense (the reference, last)
+    prefix = [0] * 15 + [1] * (N - 15)
+    for policy in (1, 3, 2):
         eng = F.Engine(layers, heads, m, dt, L_img, L_txt, 1, steps, synth.delta_table(steps),
-                       cache, mod_table=mods, plan_policy=policy)
+                       cache, mod_table=mods, plan_policy=policy,
+                       plan=prefix if policy == 3 else None)
         req = dict(template_id=0, step=0, n_steps=steps, mask=torch.as_tensor(mask).cuda(),
                    x=x0.clone())
         eng.run_batch([req], 1)
@@ -325,9 +330,10 @@ def test_full_scale_stack_identical_input_invariant(F, mode):
         outs.append(req["x"].clone())
         eng.close()
     cache.close()
-    assert torch.isfinite(outs[0].float()).all()
-    assert torch.equal(outs[0].view(torch.int16), outs[1].view(torch.int16)), \
-        f"{mode}: max diff {(outs[0].float() - outs[1].float()).abs().max().item()}"
+    for o in outs[:2]:
+        assert torch.isfinite(o.float()).all()
+        assert torch.equal(o.view(torch.int16), outs[2].view(torch.int16)), \
+            f"{mode}: max diff {(o.float() - outs[2].float()).abs().max().item()}"
 
 
 @pytest.mark.parametrize("mode,plan,copy_method", [("kv", [0, 1, 1], 1), ("y", [1, 0, 1], 0),
