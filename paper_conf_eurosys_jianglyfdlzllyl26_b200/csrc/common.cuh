@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <atomic>
 #include <cstdarg>
 #include <cstdio>
 #include <string>
@@ -29,6 +30,22 @@ fps_status fail(fps_status code, const char* fmt, ...);
     if (_e != cudaSuccess)                                                                  \
       return ::fps::fail(FPS_ECUDA, "%s:%d %s: %s", __FILE__, __LINE__, #expr,              \
                          cudaGetErrorString(_e));                                           \
+  } while (0)
+
+// Dynamic shared memory above 48 KB needs cudaFuncSetAttribute once per kernel AND per device:
+// each call site keeps a bit per device it has already set up (atomic: engines on different
+// devices may launch from different threads).  Wrap a templated kernel name in parentheses.
+#define FPS_SMEM_ATTR(kernel, bytes)                                                        \
+  do {                                                                                      \
+    static std::atomic<unsigned long long> fps_attr_mask_{0};                               \
+    int fps_dev_ = 0;                                                                       \
+    FPS_CUDA_TRY(cudaGetDevice(&fps_dev_));                                                 \
+    const unsigned long long fps_bit_ = 1ull << (fps_dev_ & 63);                            \
+    if (!(fps_attr_mask_.load(std::memory_order_acquire) & fps_bit_)) {                     \
+      FPS_CUDA_TRY(cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, \
+                                        (int)(bytes)));                                     \
+      fps_attr_mask_.fetch_or(fps_bit_, std::memory_order_acq_rel);                         \
+    }                                                                                       \
   } while (0)
 
 #define FPS_LAUNCH_CHECK()                                                                  \

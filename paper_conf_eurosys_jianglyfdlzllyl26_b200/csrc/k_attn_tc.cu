@@ -1072,12 +1072,7 @@ static fps_status launch_d(const void* q, const void* kv, void* o, int heads,
     return fail(FPS_ECUDA, "attention_tc: Q tensor map");
   if (!make_tmap_2d_bf16(&tkv, kv, (uint64_t)h_cu_k[n_req], 2 * H, (uint64_t)H * 4, 64, 128))
     return fail(FPS_ECUDA, "attention_tc: KV tensor map");
-  static bool attr = false;
-  if (!attr) {
-    FPS_CUDA_TRY(cudaFuncSetAttribute(attn_tc_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      Cfg::SMEM));
-    attr = true;
-  }
+  FPS_SMEM_ATTR((attn_tc_kernel<D>), Cfg::SMEM);
   const float scale_log2 = 1.4426950408889634f / sqrtf((float)D);
   FPS_CUDA_TRY(launch_k(attn_tc_kernel<D>, dim3(tiles, heads), dim3(256), Cfg::SMEM, s, tq, tkv,
                         reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads,
@@ -1101,12 +1096,7 @@ static fps_status launch_d2(const void* q, const void* kv, void* o, int heads,
     return fail(FPS_ECUDA, "attention_tc2: Q tensor map");
   if (!make_tmap_2d_bf16(&tkv, kv, (uint64_t)h_cu_k[n_req], 2 * H, (uint64_t)H * 4, 64, 128))
     return fail(FPS_ECUDA, "attention_tc2: KV tensor map");
-  static bool attr = false;
-  if (!attr) {
-    FPS_CUDA_TRY(cudaFuncSetAttribute(attn_tc2_kernel<D>,
-                                      cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
-    attr = true;
-  }
+  FPS_SMEM_ATTR((attn_tc2_kernel<D>), Cfg::SMEM);
   const float scale_log2 = 1.4426950408889634f / sqrtf((float)D);
   FPS_CUDA_TRY(launch_k(attn_tc2_kernel<D>, dim3(pairs, heads), dim3(384), Cfg::SMEM, s, tq, tkv,
                         reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads,
@@ -1165,12 +1155,7 @@ static fps_status launch_d3(const void* q, const void* kv, void* o, int heads,
     return fail(FPS_ECUDA, "attention_tc3: Q tensor map");
   if (!make_tmap_2d_bf16(&tkv, kv, (uint64_t)h_cu_k[n_req], 2 * H, (uint64_t)H * 4, 64, 128))
     return fail(FPS_ECUDA, "attention_tc3: KV tensor map");
-  static bool attr = false;
-  if (!attr) {
-    FPS_CUDA_TRY(cudaFuncSetAttribute(attn_tc3_kernel<D>,
-                                      cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
-    attr = true;
-  }
+  FPS_SMEM_ATTR((attn_tc3_kernel<D>), Cfg::SMEM);
   const float scale_log2 = 1.4426950408889634f / sqrtf((float)D);
   const long long part_stride = (long long)total_q * H;
   auto* Opart = S > 1 ? reinterpret_cast<__nv_bfloat16*>(sc->part) : nullptr;

@@ -690,12 +690,7 @@ static fps_status launch_cfg(const void* A, const void* B, int M, int N, int K,
       (g2.M1 > 0 && !make_tmap_2d_bf16(&tb1, g2.B1, N, K, (uint64_t)K * 2, Cfg::BK, BN)))
     return fail(FPS_ECUDA, "gemm_tc: cuTensorMapEncodeTiled failed (M=%d N=%d K=%d)", M, N, K);
   if (g2.M1 == 0) tb1 = tb;
-  static bool attr_set = false;
-  if (!attr_set) {
-    FPS_CUDA_TRY(cudaFuncSetAttribute(gemm_tc_kernel<BN, STAGES>,
-                                      cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
-    attr_set = true;
-  }
+  FPS_SMEM_ATTR((gemm_tc_kernel<BN, STAGES>), Cfg::SMEM);
   const int tiles = (ceil_div(M, Cfg::BM) + ceil_div(g2.M1, Cfg::BM)) * ceil_div(N, BN);
   const int grid = tiles < kNumSMs ? tiles : kNumSMs;
   FPS_CUDA_TRY(launch_k(gemm_tc_kernel<BN, STAGES>, dim3(grid), dim3(256), Cfg::SMEM, s, ta, tb,
@@ -715,12 +710,7 @@ static fps_status launch_pair(const void* A, const void* B, int M, int N, int K,
       (g2.M1 > 0 && !make_tmap_2d_bf16(&tb1, g2.B1, N, K, (uint64_t)K * 2, Cfg::BK, 128)))
     return fail(FPS_ECUDA, "gemm_tc2: cuTensorMapEncodeTiled failed (M=%d N=%d K=%d)", M, N, K);
   if (g2.M1 == 0) tb1 = tb;
-  static bool attr_set = false;
-  if (!attr_set) {
-    FPS_CUDA_TRY(cudaFuncSetAttribute(gemm_tc2_kernel<STAGES>,
-                                      cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
-    attr_set = true;
-  }
+  FPS_SMEM_ATTR((gemm_tc2_kernel<STAGES>), Cfg::SMEM);
   const int tiles = (ceil_div(M, Cfg::BM) + ceil_div(g2.M1, Cfg::BM)) * ceil_div(N, Cfg::BN);
   const int pairs = tiles < kNumSMs / 2 ? tiles : kNumSMs / 2;
   FPS_CUDA_TRY(launch_k(gemm_tc2_kernel<STAGES>, dim3(2 * pairs), dim3(256), Cfg::SMEM, s, ta, tb,
@@ -738,12 +728,7 @@ static fps_status launch_pair_swap(const void* A, const void* B, int M, int N, i
   if (!make_tmap_2d_bf16(&ta, A, M, K, (uint64_t)K * 2, Cfg::BK, NA / 2) ||
       !make_tmap_2d_bf16(&tb, B, N, K, (uint64_t)K * 2, Cfg::BK, 128))
     return fail(FPS_ECUDA, "gemm_tc2s: cuTensorMapEncodeTiled failed (M=%d N=%d K=%d)", M, N, K);
-  static bool attr_set = false;
-  if (!attr_set) {
-    FPS_CUDA_TRY(cudaFuncSetAttribute(gemm_tc2s_kernel<STAGES>,
-                                      cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
-    attr_set = true;
-  }
+  FPS_SMEM_ATTR((gemm_tc2s_kernel<STAGES>), Cfg::SMEM);
   const int tiles = ceil_div(M, NA) * ceil_div(N, 256);
   const int pairs = tiles < kNumSMs / 2 ? tiles : kNumSMs / 2;
   FPS_CUDA_TRY(launch_k(gemm_tc2s_kernel<STAGES>, dim3(2 * pairs), dim3(256), Cfg::SMEM, s, ta,
