@@ -347,6 +347,16 @@ fps_status fps_plan_pipeline_cross(const double* c_cached, const double* c_dense
 double fps_pipeline_latency_cross(const uint8_t* use_cache, const double* c_cached,
                                   const double* c_dense, const double* load, int32_t N,
                                   int32_t mode, double final_load);
+/* KV-mode with the transition block (reading R28): the N+1 suffix plans, each priced with its
+ * uncached prefix's last block at c_transition[l] (a masked block whose K|V projection covers
+ * every row, Y-mode work) instead of c_dense[l] -- when both the prefix and the cached suffix
+ * are non-empty.  cross_step 0: the R11 model (fps_pipeline_latency); 1: the R26 steady-state
+ * model (fps_pipeline_latency_cross).  Ties -> fewer cached blocks.  c_transition[N] as the
+ * other cost arrays.  Host only; FPS_EINVAL on NULL arrays or N < 0. */
+fps_status fps_plan_pipeline_kv_transition(const double* c_cached, const double* c_dense,
+                                           const double* c_transition, const double* load,
+                                           int32_t N, double final_load, int32_t cross_step,
+                                           uint8_t* use_cache, double* latency);
 /* The model itself (for tests and the balancer): latency of a given plan; +inf if infeasible. */
 double fps_pipeline_latency(const uint8_t* use_cache, const double* c_cached,
                             const double* c_dense, const double* load, int32_t N, int32_t mode,

@@ -194,3 +194,23 @@ def plan_steady_suffix(Cw, Cwo, Lm, mode, final_load=0.0):
         if v < best:
             best, best_plan = v, p
     return best, best_plan
+
+
+def plan_transition_suffix(Cw, Cwo, Ct, Lm, final_load=0.0, cross_step=False):
+    """KV-mode Alg. 1 with the transition block (reading R28): the N+1 plans
+    'uncached prefix, cached suffix', each priced with the prefix's last block at Ct[l] (it runs
+    as a masked block over the fresh full input) instead of Cwo[l] when both parts are
+    non-empty; latency = simulate (R11) or steady_step_latency (R26, cross_step).  Ties ->
+    fewer cached blocks.  Returns (latency, plan)."""
+    N = len(Cw)
+    best, best_plan = math.inf, None
+    for k in range(N + 1):
+        p = [0] * (N - k) + [1] * k
+        c = list(Cwo)
+        if 0 < k < N:
+            c[N - k - 1] = Ct[N - k - 1]
+        v = (steady_step_latency(p, Cw, c, Lm, "kv", final_load) if cross_step
+             else simulate(p, Cw, c, Lm, "kv", final_load))
+        if v < best:
+            best, best_plan = v, p
+    return best, best_plan

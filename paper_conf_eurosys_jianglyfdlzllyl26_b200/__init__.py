@@ -266,6 +266,19 @@ def plan_pipeline(c_cached, c_dense, load, mode, final_load=0.0, cross_step=Fals
     return [int(use[i]) for i in range(N)], lat.value
 
 
+def plan_pipeline_kv_transition(c_cached, c_dense, c_transition, load, final_load=0.0,
+                                cross_step=False):
+    """KV-mode Alg. 1 with the transition block (R28). Returns (use_cache list, latency)."""
+    N = len(c_cached)
+    arr = lambda v: (C.c_double * max(N, 1))(*map(float, v))
+    use = (C.c_uint8 * max(N, 1))()
+    lat = C.c_double()
+    _lib.fps_plan_pipeline_kv_transition(arr(c_cached), arr(c_dense), arr(c_transition), arr(load),
+                                         N, float(final_load), int(bool(cross_step)), use,
+                                         C.byref(lat))
+    return [int(use[i]) for i in range(N)], lat.value
+
+
 def pipeline_latency(use, c_cached, c_dense, load, mode, final_load=0.0, cross_step=False):
     N = len(use)
     arr = lambda v: (C.c_double * N)(*map(float, v))

@@ -108,6 +108,7 @@ _SIGS = [
     ("fps_pipeline_latency", dbl, [P_u8, P_dbl, P_dbl, P_dbl, i32, i32, dbl], False),
     ("fps_plan_pipeline_cross", C.c_int, [P_dbl, P_dbl, P_dbl, i32, i32, dbl, P_u8, P_dbl], True),
     ("fps_pipeline_latency_cross", dbl, [P_u8, P_dbl, P_dbl, P_dbl, i32, i32, dbl], False),
+    ("fps_plan_pipeline_kv_transition", C.c_int, [P_dbl, P_dbl, P_dbl, P_dbl, i32, dbl, i32, P_u8, P_dbl], True),
     ("fps_engine_create", C.c_int, [C.POINTER(fps_engine_desc), C.POINTER(vp)], True),
     ("fps_engine_destroy", C.c_int, [vp], True),
     ("fps_run_batch", C.c_int, [vp, C.POINTER(fps_request), i32, i32, vp, vp], True),

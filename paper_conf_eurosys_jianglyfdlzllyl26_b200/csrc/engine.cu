@@ -466,17 +466,8 @@ static void make_plan(fps_engine* e, const Batch& B) {
     return latency(use, Cw.data(), C2.data(), Lm.data(), N, e->d.mode, fin);
   };
   if (e->d.plan_policy == 0 && trans) {
-    std::vector<uint8_t> use(N);
-    double best = 0;
-    for (int k = 0; k <= N; ++k) {        // k = uncached prefix length; ties -> more cached
-      for (int l = 0; l < N; ++l) use[l] = l >= k ? 1 : 0;
-      const double t = priced(use.data());
-      if (k == 0 || t < best - 1e-12 * std::max(1.0, std::fabs(best))) {
-        best = t;
-        e->last_plan = use;
-      }
-    }
-    e->last_latency = best;
+    fps_plan_pipeline_kv_transition(Cw.data(), Cwo.data(), Ct.data(), Lm.data(), N, fin,
+                                    e->cross ? 1 : 0, e->last_plan.data(), &e->last_latency);
   } else if (e->d.plan_policy == 0) {
     if (e->cross)
       fps_plan_pipeline_cross(Cw.data(), Cwo.data(), Lm.data(), N, e->d.mode, fin,

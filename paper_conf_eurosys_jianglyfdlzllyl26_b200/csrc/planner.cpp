@@ -248,4 +248,33 @@ fps_status fps_plan_pipeline(const double* c_cached, const double* c_dense, cons
   return FPS_OK;
 }
 
+fps_status fps_plan_pipeline_kv_transition(const double* c_cached, const double* c_dense,
+                                           const double* c_transition, const double* load,
+                                           int32_t N, double final_load, int32_t cross_step,
+                                           uint8_t* use_cache, double* latency) {
+  if (N < 0 || !latency ||
+      (N > 0 && (!c_cached || !c_dense || !c_transition || !load || !use_cache)))
+    return FPS_EINVAL;
+  std::vector<uint8_t> p(N);
+  std::vector<double> cd(c_dense, c_dense + N);
+  double best = std::numeric_limits<double>::infinity();
+  int best_k = 0;
+  for (int k = 0; k <= N; ++k) {                 // k cached blocks; ties -> fewer cached
+    for (int l = 0; l < N; ++l) p[l] = l >= N - k ? 1 : 0;
+    const int t = N - k - 1;                     // the prefix's last block, if both parts exist
+    if (k > 0 && t >= 0) cd[t] = c_transition[t];
+    const double v = N == 0 ? 0.0
+                     : cross_step ? steady_of(p.data(), c_cached, cd.data(), load, N, FPS_MODE_KV, final_load)
+                                  : latency_of(p.data(), c_cached, cd.data(), load, N, FPS_MODE_KV, final_load);
+    if (k > 0 && t >= 0) cd[t] = c_dense[t];
+    if (v < best - 1e-12 * std::max(1.0, std::fabs(best)) || std::isinf(best)) {
+      best = v;
+      best_k = k;
+    }
+  }
+  for (int l = 0; l < N; ++l) use_cache[l] = l >= N - best_k ? 1 : 0;
+  *latency = N == 0 ? 0.0 : best;
+  return FPS_OK;
+}
+
 }  // extern "C"

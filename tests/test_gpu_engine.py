@@ -446,7 +446,8 @@ def test_kv_transition_planner_prices_each_suffix(F, cross):
         Lm = [cm[2] * nu * 2 * H * 2 + cm[3]] * N
         fin = cm[2] * nu * H * 2 + cm[3]
         best = None
-        for k in range(N + 1):
+        for kc in range(N + 1):               # k cached blocks; ties -> fewer cached
+            k = N - kc
             use = [0] * k + [1] * (N - k)
             C2 = list(Cwo)
             if on and 0 < k < N:
@@ -457,6 +458,10 @@ def test_kv_transition_planner_prices_each_suffix(F, cross):
         if not on:
             ref_plan, ref_lat = F.plan_pipeline(Cw, Cwo, Lm, F.FPS_MODE_KV, fin, cross_step=cross)
             assert list(ref_plan) == best[1] and ref_lat == pytest.approx(best[0], rel=1e-9)
+        if on:
+            lib_plan, lib_lat = F.plan_pipeline_kv_transition(Cw, Cwo, [Ct] * N, Lm, fin,
+                                                              cross_step=cross)
+            assert lib_plan == best[1] and lib_lat == pytest.approx(best[0], rel=1e-9)
         assert plan == best[1], (on, plan, best)
         assert 0 < sum(plan) < N, plan
         assert lat == pytest.approx(best[0], rel=1e-9)

@@ -197,3 +197,25 @@ def test_header_is_plain_c_and_links(tmp_path):
     subprocess.run(["gcc", "-std=c99", "-I", inc, str(src), "-L", libdir, "-l:libflashps.so",
                     f"-Wl,-rpath,{libdir}", "-o", str(exe)], check=True)
     assert subprocess.run([str(exe)]).returncode == 0
+
+
+@pytest.mark.parametrize("cross", [False, True])
+def test_transition_planner_matches_oracle(cross):
+    """KV-mode planner with the transition block (R28): the library vs the oracle's exhaustive
+    suffix scan with the prefix's last block at its transition cost."""
+    g = synth.rng(29)
+    for _ in range(100):
+        N = int(g.integers(1, 14))
+        Cw, Cwo, Lm, fin = _rand_costs(g, N)
+        Ct = [c + float(g.uniform(0, 1)) * max(d - c, 0.0) for c, d in zip(Cw, Cwo)]
+        best, bplan = P.plan_transition_suffix(Cw, Cwo, Ct, Lm, fin, cross)
+        plan, lat = fps.plan_pipeline_kv_transition(Cw, Cwo, Ct, Lm, fin, cross_step=cross)
+        assert lat == pytest.approx(best, rel=1e-9)
+        if plan != bplan:                   # a tie: the library's plan prices at the optimum
+            k = N - sum(plan)
+            c = list(Cwo)
+            if 0 < k < N:
+                c[k - 1] = Ct[k - 1]
+            f = P.steady_step_latency if cross else P.simulate
+            assert f(plan, Cw, c, Lm, "kv", fin) == pytest.approx(best, rel=1e-9)
+    assert fps.plan_pipeline_kv_transition([], [], [], [], 0.0) == ([], 0.0)

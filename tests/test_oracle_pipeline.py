@@ -226,3 +226,38 @@ def test_steady_planner_is_exhaustive_optimum_over_suffixes():
         for k in range(N + 1):
             p = [0] * (N - k) + [1] * k
             assert best <= P.steady_step_latency(p, Cw, Cwo, Lm, "kv", 0.2) + 1e-12
+
+
+def test_transition_planner_hand_case_flips_the_plan():
+    """KV-mode transition block (R28), a timeline derived by hand under the R11 model: N = 2,
+    C_w = [1, 1], C_w/o = [3, 3], C_t = [1.5, 1.5], loads [1, 1], no final load.
+    Without the transition: [0,0] = 6; [0,1]: block 0 ends 3, block 1 at max(3, 1) -> 4;
+    [1,1]: loads end 1, 2; block 0 1 -> 2, block 1 max(2, 2) -> 3  => [1,1] at 3.
+    With it, [0,1]: block 0 (transition) ends 1.5, block 1 at max(1.5, 1) -> 2.5  => [0,1]."""
+    Cw, Cwo, Ct, Lm = [1.0, 1.0], [3.0, 3.0], [1.5, 1.5], [1.0, 1.0]
+    assert P.plan_suffix_scan(Cw, Cwo, Lm, "kv") == (3.0, [1, 1])
+    assert P.plan_transition_suffix(Cw, Cwo, Ct, Lm) == (2.5, [0, 1])
+    # cross-step (R26): the [0,1] plan's loads hide (1 per step against 2.5 of compute), so its
+    # steady step is the compute stream's sum 1.5 + 1
+    lat, plan = P.plan_transition_suffix(Cw, Cwo, Ct, Lm, cross_step=True)
+    assert P.steady_step_latency([0, 1], Cw, [1.5, 3.0], Lm, "kv") == pytest.approx(2.5)
+    assert lat <= 2.5 + 1e-12
+
+
+@pytest.mark.parametrize("cross", [False, True])
+def test_transition_planner_reduces_to_alg1_and_never_loses(cross):
+    """With C_t = C_w/o the transition planner is the suffix planner (R11 / R26); with
+    C_t <= C_w/o it is never slower."""
+    g = synth.rng(28)
+    for _ in range(60):
+        N = int(g.integers(1, 10))
+        Cw = list(g.uniform(0.1, 1.0, N))
+        Cwo = [c + float(g.uniform(0.2, 2.0)) for c in Cw]
+        Lm = list(g.uniform(0.05, 1.5, N))
+        fin = float(g.uniform(0, 0.5))
+        ref = (P.plan_steady_suffix if cross else P.plan_suffix_scan)(Cw, Cwo, Lm, "kv", fin)
+        same = P.plan_transition_suffix(Cw, Cwo, Cwo, Lm, fin, cross)
+        assert same[0] == pytest.approx(ref[0], rel=1e-12) and same[1] == ref[1]
+        Ct = [c + float(g.uniform(0, 1)) * (d - c) for c, d in zip(Cw, Cwo)]
+        lat, plan = P.plan_transition_suffix(Cw, Cwo, Ct, Lm, fin, cross)
+        assert lat <= ref[0] + 1e-12
