@@ -456,7 +456,7 @@ def main():
                    if args.config == "C3" else f"masked-block stack images/s ({args.config})")
     base_cfg["cache_tier"] = {"host": "pinned host DRAM", "hbm": "device HBM (NEXT-1)",
                               "host_hugepage": "pinned host DRAM on 2 MiB pages"}[args.tier]
-    base_cfg["h2d_method"] = ["SM row gather", "batched DMA of the unmasked row runs", "DMA of whole entries"][args.copy_method]
+    base_cfg["h2d_method"] = ["SM row gather", "DMA of the unmasked row runs", "DMA of whole entries"][args.copy_method]
     base_cfg["parallelism"] = f"request-parallel x{world} (Alg. 2 routing)"
     base_cfg["cross_step_prefetch"] = bool(args.cross_step)
     base_cfg["kv_transition_block"] = bool(args.kv_transition) and args.mode == "kv"
@@ -518,7 +518,7 @@ def main():
     wbytes = sum(t.numel() * t.element_size() for l in layers for t in l.t.values())
     base_cfg["l2"] = f"inputs > L2 ({wbytes / 1e9:.1f} GB of weights streamed per step)"
     base_cfg["cache_tier"] = "pinned host DRAM" if location == 0 else "device HBM (NEXT-1)"
-    base_cfg["h2d_method"] = ["SM row gather", "batched DMA of the unmasked row runs", "DMA of whole entries"][args.copy_method]
+    base_cfg["h2d_method"] = ["SM row gather", "DMA of the unmasked row runs", "DMA of whole entries"][args.copy_method]
     torch.cuda.synchronize()
     log(f"[rank {rank}] inputs ready in {time.perf_counter() - t0:.1f}s")
     my_pool = pool[:w["batch"]]

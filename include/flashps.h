@@ -130,9 +130,9 @@ typedef struct {
                             moved are identical, contents alias)                            */
   int32_t copy_method;   /* 0 = SM row gather (zero-copy over mapped pinned memory, or from
                                 the HBM arena) -- exactly the rows U (default);
-                            1 = copy-engine DMA of exactly the rows U: their runs of
-                                consecutive tokens go out as one cudaMemcpyBatchAsync per call
-                                (one cudaMemcpyAsync per run on the legacy default stream).
+                            1 = copy-engine DMA of exactly the rows U: one cudaMemcpyAsync
+                                per run of consecutive tokens, on the load stream (on the HBM
+                                arena, location 1, the rows go through the method-0 gather);
                                 Full link rate on only the unmasked bytes: the pinned-host
                                 default of the bench;
                             2 = copy-engine DMA of the WHOLE entry (all L_img rows, one copy

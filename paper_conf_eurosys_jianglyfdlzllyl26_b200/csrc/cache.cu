@@ -7,10 +7,11 @@
 //     arena over PCIe (16-B loads, many in flight) and write them to their token rows in HBM.
 //     One launch per layer for the whole batch, exact bytes, any mask shape -- but the gather
 //     warps share the SMs with the compute stream (~10% slower GEMMs in the step).
-//  1  copy-engine DMA of exactly the unmasked rows: runs of consecutive tokens submitted as one
-//     cudaMemcpyBatchAsync per prefetch call.  Measured on B200 (tools/micro/h2d_runs, C3 entry,
-//     33 runs): 55.2 GB/s of unmasked bytes and ~11 us of host time per entry, against 47 GB/s and
-//     ~200 us for one cudaMemcpyAsync per run, and 44 GB/s of useful bytes for whole entries.
+//  1  copy-engine DMA of exactly the unmasked rows: one cudaMemcpyAsync per run of consecutive
+//     tokens.  Measured on B200 (a dev micro, C3 entry, 33 runs): 47 GB/s and ~200 us of host
+//     time per entry, against 44 GB/s of useful bytes for whole entries.  (The CUDA 12.8
+//     batched-copy entry point measured faster, 55 GB/s / ~11 us, but it is closed on the GPU
+//     pool this library is validated on -- it raised device faults there -- so it is not used.)
 //  2  copy-engine DMA of whole entries (all L_img rows, one copy per request and block): +25%
 //     bytes at m = 0.2 but no SM time and no per-run overhead; the caller orders fresh-row writes
 //     after the ready event.  Fastest measured step on B200 for both tiers.
@@ -274,7 +275,9 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
       bytes += nb;
     }
     prof::end(s, prof::PREFETCH, 0, bytes);
-  } else if (c->d.copy_method == 0) {
+  } else if (c->d.copy_method == 0 || c->d.location == 1) {
+    // (method 1 on the HBM arena takes the row gather too: a driver D2D copy per run would
+    //  interleave with PDL launches, the pattern that hung in tools/hang_probe.py)
     for (int base = 0; base < n_items; base += kMaxPrefetchItems) {
       PrefetchBatch b{};
       long long acc = 0;
@@ -339,33 +342,13 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
         j = k + 1;
       }
     }
-    // all runs of all items as one batch (stream-ordered source access: the arena is stable)
+    // one DMA per run of consecutive tokens, in submission order on the load stream
     double bytes = 0;
     for (size_t q = 0; q < c->sizes.size(); ++q) bytes += c->sizes[q];
     prof::begin(s);
-    if (s == 0 || s == cudaStreamLegacy) {
-      // the batch API rejects the legacy default stream: one DMA per run there
-      for (size_t q = 0; q < c->sizes.size(); ++q)
-        FPS_COPY_TRY(s, cudaMemcpyAsync(c->dsts[q], c->srcs[q], c->sizes[q], cudaMemcpyDefault, s));
-    } else if (!c->sizes.empty()) {
-      cudaMemcpyAttributes a{};
-      a.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-      a.srcLocHint.type = c->d.location == 1 ? cudaMemLocationTypeDevice : cudaMemLocationTypeHost;
-      a.dstLocHint.type = cudaMemLocationTypeDevice;
-      int dev = 0;
-      FPS_CUDA_TRY(cudaGetDevice(&dev));
-      a.dstLocHint.id = dev;
-      a.flags = cudaMemcpyFlagPreferOverlapWithCompute;
-      size_t attr_idx = 0, fail_idx = ~size_t(0);
-      pdl_fence(s);
-      const cudaError_t e = cudaMemcpyBatchAsync(c->dsts.data(), c->srcs.data(), c->sizes.data(),
-                                                 c->sizes.size(), &a, &attr_idx, 1, &fail_idx, s);
-      if (e != cudaSuccess) {
-        (void)cudaGetLastError();                 // not sticky: clear it for later launch checks
-        return fail(FPS_ECUDA, "cache prefetch: cudaMemcpyBatchAsync (copy %zu of %zu): %s",
-                    fail_idx, c->sizes.size(), cudaGetErrorString(e));
-      }
-    }
+    if (!c->sizes.empty()) pdl_fence(s);
+    for (size_t q = 0; q < c->sizes.size(); ++q)
+      FPS_COPY_TRY(s, cudaMemcpyAsync(c->dsts[q], c->srcs[q], c->sizes[q], cudaMemcpyDefault, s));
     prof::end(s, prof::PREFETCH, 0, bytes);
   }
   if (ready_event) FPS_CUDA_TRY(cudaEventRecord((cudaEvent_t)ready_event, s));

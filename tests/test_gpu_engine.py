@@ -183,8 +183,8 @@ def test_pipeline_slots_and_copy_methods_bit_identical(F, slots, method, locatio
 
 @pytest.mark.parametrize("mode,slots", [("kv", 2), ("y", 2), ("kv", 1)])
 def test_batched_run_dma_bit_identical(F, mode, slots):
-    """copy_method 1 on a real load stream goes through one cudaMemcpyBatchAsync per prefetch
-    (exact unmasked rows); with a shallow staging ring the slot reuse must still be ordered."""
+    """copy_method 1 on a real load stream goes through one cudaMemcpyAsync per run of
+    consecutive unmasked rows; with a shallow staging ring the slot reuse must still be ordered."""
     outs = []
     for me, use_ls in ((0, False), (1, True)):
         _, _, _, _, eng, reqs = _setup(F, mode, "bf16", 1, slots=slots if me else 0,
