@@ -406,8 +406,8 @@ def main():
                     help="template cache in pinned host DRAM (configs[2]) or HBM (NEXT-1)")
     ap.add_argument("--copy-ctas", type=int, default=0, help="CTAs of the SM row gather (0 = lib default)")
     ap.add_argument("--copy-method", type=int, default=None, choices=[0, 1, 2],
-                    help="H2D method: 0 SM zero-copy row gather, 1 batched DMA of the unmasked row "
-                         "runs (host default), 2 whole-entry DMA (HBM default)")
+                    help="H2D method: 0 SM zero-copy row gather, 1 one DMA per unmasked row run, "
+                         "2 whole-entry DMA (default, both tiers)")
     ap.add_argument("--cross-step", type=int, default=1, choices=[0, 1],
                     help="cross-step prefetch (R26): the next step's loads start as soon as their "
                          "slots are consumed (1, default), or the per-step pipeline of Fig. 9 (0)")
@@ -425,11 +425,10 @@ def main():
     faulthandler.dump_traceback_later(900, exit=True)
     faulthandler.register(signal.SIGUSR1, all_threads=True)   # `timeout -s USR1`: dump stacks
     if args.copy_method is None:
-        # measured on B200 (C3): pinned host tier -- batched DMA of the unmasked row runs 32.8
-        # ms/step vs 36.7 with whole-entry DMA (-20% bytes at the same 55 GB/s) and 43.3 with the
-        # SM row gather (SM interference); HBM tier -- whole-entry DMA 21.6 vs 44.4 for the run
-        # batch (device-to-device run copies reach only ~145 GB/s on the copy engine)
-        args.copy_method = 2 if args.tier == "hbm" else 1
+        # measured on B200 (C3, profiles/r01f5_*): pinned host tier -- whole-entry DMA 34.6
+        # ms/step vs 36.2 with one DMA per unmasked row run (~200 us of host time per entry) and
+        # 48.5 with the SM row gather (SM interference); HBM tier -- whole-entry DMA 21.2
+        args.copy_method = 2
 
     rank = int(os.environ.get("RANK", 0))
     world = int(os.environ.get("WORLD_SIZE", 1))
@@ -598,7 +597,7 @@ def main():
         # the other caching mode, and both modes with the other cache tier, on the same batch
         other = "y" if args.mode == "kv" else "kv"
         other_loc = 0 if location == 1 else 1
-        default_cm = lambda loc: 2 if loc == 1 else 1
+        default_cm = lambda loc: 2
         other_cm = default_cm(other_loc)
         for md, loc, cmeth in ((other, location, args.copy_method),
                                (args.mode, other_loc, other_cm), (other, other_loc, other_cm),
