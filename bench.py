@@ -48,6 +48,8 @@ WORKLOADS = {
                 desc="SDXL-scale 64x64 level (640 ch), masks 10/30/50%, batch 4"),
 }
 SEED = 1003
+H2D_NAMES = ["SM row gather", "DMA of the unmasked row runs", "DMA of whole entries",
+             "TMA bulk row gather (exact rows, reserved SMs)"]
 SDXL_CTX = (77, 2048)          # SDXL prompt encoding: 77 tokens x 2048 channels (R24)
 FLUX_DOUBLE = 19               # Flux: 19 double-stream blocks, then 38 single-stream (R19, R25)
 
@@ -405,9 +407,9 @@ def main():
     ap.add_argument("--tier", default="host", choices=["host", "hbm", "host_hugepage"],
                     help="template cache in pinned host DRAM (configs[2]) or HBM (NEXT-1)")
     ap.add_argument("--copy-ctas", type=int, default=0, help="CTAs of the SM row gather (0 = lib default)")
-    ap.add_argument("--copy-method", type=int, default=None, choices=[0, 1, 2],
+    ap.add_argument("--copy-method", type=int, default=None, choices=[0, 1, 2, 3],
                     help="H2D method: 0 SM zero-copy row gather, 1 one DMA per unmasked row run, "
-                         "2 whole-entry DMA (default, both tiers)")
+                         "2 whole-entry DMA, 3 TMA bulk row gather on reserved SMs")
     ap.add_argument("--cross-step", type=int, default=1, choices=[0, 1],
                     help="cross-step prefetch (R26): the next step's loads start as soon as their "
                          "slots are consumed (1, default), or the per-step pipeline of Fig. 9 (0)")
@@ -455,7 +457,7 @@ def main():
                    if args.config == "C3" else f"masked-block stack images/s ({args.config})")
     base_cfg["cache_tier"] = {"host": "pinned host DRAM", "hbm": "device HBM (NEXT-1)",
                               "host_hugepage": "pinned host DRAM on 2 MiB pages"}[args.tier]
-    base_cfg["h2d_method"] = ["SM row gather", "DMA of the unmasked row runs", "DMA of whole entries"][args.copy_method]
+    base_cfg["h2d_method"] = H2D_NAMES[args.copy_method]
     base_cfg["parallelism"] = f"request-parallel x{world} (Alg. 2 routing)"
     base_cfg["cross_step_prefetch"] = bool(args.cross_step)
     base_cfg["kv_transition_block"] = bool(args.kv_transition) and args.mode == "kv"
@@ -517,7 +519,7 @@ def main():
     wbytes = sum(t.numel() * t.element_size() for l in layers for t in l.t.values())
     base_cfg["l2"] = f"inputs > L2 ({wbytes / 1e9:.1f} GB of weights streamed per step)"
     base_cfg["cache_tier"] = "pinned host DRAM" if location == 0 else "device HBM (NEXT-1)"
-    base_cfg["h2d_method"] = ["SM row gather", "DMA of the unmasked row runs", "DMA of whole entries"][args.copy_method]
+    base_cfg["h2d_method"] = H2D_NAMES[args.copy_method]
     torch.cuda.synchronize()
     log(f"[rank {rank}] inputs ready in {time.perf_counter() - t0:.1f}s")
     my_pool = pool[:w["batch"]]
@@ -615,7 +617,7 @@ def main():
             o_ms, _ = run_engine_timed(F, eng_o, reqs_dev, K, W, stream, load_stream, rank, world)
             tag = f"{md}_mode_{['host', 'hbm', 'host_hugepage'][loc]}"
             if cmeth != default_cm(loc):
-                tag += "_" + ["row_gather", "run_dma", "whole_entry_dma"][cmeth]
+                tag += "_" + ["row_gather", "run_dma", "whole_entry_dma", "tma_row_gather"][cmeth]
             extras[f"{tag}_ms_per_step"] = o_ms
             extras[f"{tag}_cached_blocks"] = int(sum(eng_o.last_plan()[0]))
             del eng_o

@@ -69,6 +69,11 @@ void fps_set_disable_tc(int32_t flags);
  * FPS_ECUDA. */
 void fps_profile_enable(int32_t on);
 int32_t fps_profile_read(double* ms, double* flops, double* bytes, int64_t* count);
+/* The recorded launches in launch order (up to max_n): start / end in ms relative to the first
+ * launch's start event, the kernel class, and the stream (as an integer id).  Returns the
+ * number written, or FPS_ECUDA. */
+int64_t fps_profile_trace(double* start_ms, double* end_ms, int32_t* kind, int64_t* stream,
+                          int64_t max_n);
 
 /* ---------------------------------------------------------------------------------------
  * a1 input (NEXT-4)  Pixel mask -> token mask.  L79 (§2.1): the latent (B, C, H, W) is reshaped
@@ -434,6 +439,13 @@ void fps_engine_set_admission_reuse(fps_engine_t e, int32_t on);
  * every row read afterwards at the cost of the active rows' attention and MLP (R28).
  * Off: that block runs densely over all rows. */
 void fps_engine_set_kv_transition(fps_engine_t e, int32_t on);
+/* Measurement switch (default off): when on, the engine issues no cache loads -- each load's
+ * ready event is still recorded on the load stream, so the compute stream's ordering is
+ * unchanged, and the staging slots keep whatever an earlier step loaded into them.  The step
+ * then runs the same plan and the same kernels without any host-link traffic: the "no-load"
+ * arm against which exposed load time is measured.  Results are NOT the
+ * method's (the cached rows are stale); never use it for output. */
+void fps_engine_set_skip_loads(fps_engine_t e, int32_t on);
 
 #ifdef __cplusplus
 }

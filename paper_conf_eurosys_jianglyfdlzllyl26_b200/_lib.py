@@ -82,6 +82,7 @@ _SIGS = [
     ("fps_set_disable_tc", None, [i32], False),
     ("fps_profile_enable", None, [i32], False),
     ("fps_profile_read", i32, [P_dbl, P_dbl, P_dbl, C.POINTER(C.c_int64)], False),
+    ("fps_profile_trace", i64, [P_dbl, P_dbl, C.POINTER(C.c_int32), C.POINTER(C.c_int64), i64], False),
     ("fps_mask_to_tokens", C.c_int, [vp, i32, i32, i32, i32, i32, vp, vp], True),
     ("fps_build_mask_index", C.c_int, [vp, vp, i32, i32, vp, vp, vp, vp], True),
     ("fps_gather_rows", C.c_int, [vp, vp, i32, i32, vp, vp], True),
@@ -116,6 +117,7 @@ _SIGS = [
     ("fps_engine_last_launches", i64, [vp], False),
     ("fps_engine_set_admission_reuse", None, [vp, i32], False),
     ("fps_engine_set_kv_transition", None, [vp, i32], False),
+    ("fps_engine_set_skip_loads", None, [vp, i32], False),
 ]
 
 EXPORTED = [s[0] for s in _SIGS]

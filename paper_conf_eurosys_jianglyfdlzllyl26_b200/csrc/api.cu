@@ -11,6 +11,7 @@ namespace fps {
 static thread_local std::string g_err;
 thread_local long long g_launches = 0;
 int g_disable_tc = 0;
+int g_sm_reserved = 0;
 int g_pdl = 1;
 thread_local PdlFence g_pdl_fence;
 
@@ -41,6 +42,7 @@ struct Rec {
   cudaEvent_t a, b;
   int kind;
   double flops, bytes;
+  cudaStream_t s;
 };
 static bool g_on = false;
 static std::vector<Rec> g_recs;
@@ -70,7 +72,7 @@ void end(cudaStream_t s, int kind, double flops, double bytes) {
   cudaEvent_t b = take();
   if (!b) return;
   cudaEventRecord(b, s);
-  g_recs.push_back(Rec{g_pending, b, kind, flops, bytes});
+  g_recs.push_back(Rec{g_pending, b, kind, flops, bytes, s});
   g_pending = nullptr;
 }
 }  // namespace prof
@@ -567,6 +569,28 @@ int32_t fps_profile_read(double* ms, double* flops, double* bytes, int64_t* coun
   }
   return NKIND;
 }
+int64_t fps_profile_trace(double* start_ms, double* end_ms, int32_t* kind, int64_t* stream,
+                          int64_t max_n) {
+  using namespace fps::prof;
+  if (g_recs.empty()) return 0;
+  const int64_t n = std::min<int64_t>(max_n, (int64_t)g_recs.size());
+  const cudaEvent_t t0 = g_recs[0].a;
+  for (int64_t i = 0; i < n; ++i) {
+    const Rec& r = g_recs[i];
+    float a = 0.f, b = 0.f;
+    if (cudaEventSynchronize(r.b) != cudaSuccess || cudaEventElapsedTime(&a, t0, r.a) != cudaSuccess ||
+        cudaEventElapsedTime(&b, t0, r.b) != cudaSuccess) {
+      cudaGetLastError();
+      return FPS_ECUDA;
+    }
+    if (start_ms) start_ms[i] = a;
+    if (end_ms) end_ms[i] = b;
+    if (kind) kind[i] = r.kind;
+    if (stream) stream[i] = (int64_t)(uintptr_t)r.s;
+  }
+  return n;
+}
+
 void fps_set_disable_tc(int32_t flags) {
   fps::g_disable_tc = flags & 3;
   fps::g_gemm_force = (flags >> 2) & 3;

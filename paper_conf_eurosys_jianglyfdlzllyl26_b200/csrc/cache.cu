@@ -86,6 +86,152 @@ __global__ void __launch_bounds__(256) prefetch_kernel(const __grid_constant__ P
   }
 }
 
+// ---- method 3: TMA bulk row gather (host -> smem -> HBM) ------------------------------------
+// A few CTAs, one warp each, in CTA pairs (cluster of 2 = one TPC, so the CTA-pair GEMMs keep
+// whole TPCs); the warp scans 32 row ids at a time, cuts them into chunks of consecutive rows
+// (a chunk ends at a run boundary, every kBulkRows-aligned token, and every 32 ids), and lane 0
+// moves each chunk with one cp.async.bulk load into a smem ring slot (mbarrier completion) and
+// one cp.async.bulk store to the same rows of the destination.  Measured on B200
+// (tools/micro/h2d_gather.cu, one C3 KV entry): 4 CTAs x 4 slots x 12 KB reach 51.1 GB/s of
+// unmasked bytes from mapped pinned memory for blob and random masks alike, against 44 GB/s of
+// useful bytes for the whole-entry DMA and 47 / 12 GB/s for one DMA per run (blob / random).
+// The loads cost the compute stream only the reserved SMs (sm_budget()).
+constexpr int kBulkMaxSlots = 16;
+constexpr int kBulkMinChunk = 12288;   // bytes per ring slot (at least one row)
+constexpr int kBulkMaxRow = 32768;     // widest row method 3 accepts (KV-mode H <= 8192 bf16)
+// bytes in flight over all CTAs: PCIe read latency ~2 us x ~55 GB/s needs > 110 KB; the
+// micro reached the link rate from 128 KB (e.g. 16 x 8 KB, 8 x 16 KB, 4 x 48 KB)
+constexpr int kBulkInFlight = 192 * 1024;
+constexpr int kBulkMaxSmem = 200 * 1024;
+constexpr int kBulkHeader = 512;   // barriers, row ids, pending stores (kBulkMaxSlots = 16)
+
+struct BulkBatch {
+  const char* src[kMaxPrefetchItems];
+  char* dst[kMaxPrefetchItems];
+  const int32_t* rows[kMaxPrefetchItems];
+  int n_rows[kMaxPrefetchItems];
+  int row_bytes[kMaxPrefetchItems];
+  int n_items;
+  int slot_bytes;
+  int slots;        // ring slots per CTA (<= kBulkMaxSlots)
+};
+
+__device__ __forceinline__ uint32_t bulk_su32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+// cp.async.bulk.wait_group.read takes an immediate: at most n of this thread's newest bulk
+// store groups may still be reading shared memory
+__device__ __forceinline__ void bulk_wait_read(int n) {
+  switch (n) {
+#define FPS_BW(i) \
+  case i: asm volatile("cp.async.bulk.wait_group.read " #i ";" ::: "memory"); break;
+    FPS_BW(0) FPS_BW(1) FPS_BW(2) FPS_BW(3) FPS_BW(4) FPS_BW(5) FPS_BW(6) FPS_BW(7)
+    FPS_BW(8) FPS_BW(9) FPS_BW(10) FPS_BW(11) FPS_BW(12) FPS_BW(13) FPS_BW(14)
+#undef FPS_BW
+    default: asm volatile("cp.async.bulk.wait_group.read 15;" ::: "memory"); break;
+  }
+}
+
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(32)
+    bulk_gather_kernel(const __grid_constant__ BulkBatch b) {
+  extern __shared__ __align__(128) char bulk_smem[];
+  // header: slot barriers | 32 row ids | pending store (dst, bytes) per slot | ring
+  uint64_t* bar = reinterpret_cast<uint64_t*>(bulk_smem);
+  int* toks = reinterpret_cast<int*>(bulk_smem + 8 * kBulkMaxSlots);
+  char** pend_dst = reinterpret_cast<char**>(bulk_smem + 8 * kBulkMaxSlots + 128);
+  int* pend_bytes = reinterpret_cast<int*>(bulk_smem + 16 * kBulkMaxSlots + 128);
+  char* ring = bulk_smem + kBulkHeader;
+  const int lane = threadIdx.x;
+  if (lane == 0) {
+    for (int i = 0; i < b.slots; ++i)
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bulk_su32(bar + i)));
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncwarp();
+  // lane 0's pipeline: chunk k is loaded into ring slot k % S; chunks are stored in order,
+  // lazily, when their slot is needed again (S - 1 loads stay in flight).  Measured on B200:
+  // storing each chunk as soon as it lands (a test_wait poll after every issue) was slower
+  // (49.5 vs 51.3 GB/s at 4 CTAs x 4 slots), and a deeper ring on fewer CTAs does not help --
+  // 2 CTAs x 8 slots reach 21 GB/s: the bulk copies one SM keeps in flight from system memory
+  // are limited, so the link needs about 4 SMs
+  const int S = b.slots;
+  long long k = 0, stored = 0;
+  auto landed = [&](long long j) {     // chunk j is in its slot
+    const uint32_t addr = bulk_su32(bar + (int)(j % S)), ph = (uint32_t)((j / S) & 1);
+    asm volatile(
+        "{\n.reg .pred p;\nBW: mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n@!p bra BW;\n}\n" ::"r"(
+            addr),
+        "r"(ph)
+        : "memory");
+  };
+  auto store_next = [&]() {
+    const int sl = (int)(stored % S);
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(pend_dst[sl]),
+                 "r"(bulk_su32(ring + (size_t)sl * b.slot_bytes)), "r"(pend_bytes[sl])
+                 : "memory");
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    ++stored;
+  };
+  auto issue = [&](const char* src, char* dst, int bytes) {
+    const int sl = (int)(k % S);
+    if (k >= S) {
+      while (stored <= k - S) {
+        landed(stored);
+        store_next();
+      }
+      bulk_wait_read((int)(stored - 1 - (k - S)));   // chunk k - S's store has read slot sl
+    }
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bulk_su32(bar + sl)),
+                 "r"(bytes)
+                 : "memory");
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            bulk_su32(ring + (size_t)sl * b.slot_bytes)),
+        "l"(src), "r"(bytes), "r"(bulk_su32(bar + sl))
+        : "memory");
+    pend_dst[sl] = dst;
+    pend_bytes[sl] = bytes;
+    ++k;
+  };
+  const int G = gridDim.x, rank = blockIdx.x;
+  for (int it = 0; it < b.n_items; ++it) {
+    const int n = b.n_rows[it], rb = b.row_bytes[it];
+    const int kr = rb >= b.slot_bytes ? 1 : b.slot_bytes / rb;   // rows per chunk at most
+    const int p0 = (int)((long long)n * rank / G), p1 = (int)((long long)n * (rank + 1) / G);
+    const int32_t* rows = b.rows[it];
+    for (int base = p0; base < p1; base += 32) {
+      const int pos = base + lane;
+      const bool valid = pos < p1;
+      const int tok = valid ? __ldg(rows + pos) : 0;
+      const int prev = __shfl_up_sync(0xffffffffu, tok, 1);
+      const bool start = valid && (lane == 0 || tok != prev + 1 || tok % kr == 0);
+      const unsigned mask = __ballot_sync(0xffffffffu, start);
+      toks[lane] = tok;
+      __syncwarp();
+      if (lane == 0) {
+        const int nvalid = min(32, p1 - base);
+        unsigned m = mask;
+        while (m) {
+          const int a = __ffs(m) - 1;
+          m &= m - 1;
+          const int e = m ? __ffs(m) - 1 : nvalid;
+          const long long off = (long long)toks[a] * rb;
+          issue(b.src[it] + off, b.dst[it] + off, (e - a) * rb);
+        }
+      }
+      __syncwarp();
+    }
+  }
+  if (lane == 0) {
+    while (stored < k) {
+      landed(stored);
+      store_next();
+    }
+    asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+  }
+}
+
 static long long key_of(const fps_cache* c, uint32_t t, int step, int layer) {
   const int per_step = c->d.n_layers + (c->d.mode == FPS_MODE_KV ? 1 : 0);
   return ((long long)t * c->d.n_steps + step) * per_step + layer;
@@ -106,6 +252,14 @@ static size_t offset_of(const fps_cache* c, uint32_t t, int step, int layer) {
   return (size_t)(key_of(c, t, step, layer) % c->n_entries) * c->entry_bytes;
 }
 
+// CTAs of the method-3 gather (even: CTA pairs): copy_ctas, default 4
+int bulk_ctas(const fps_cache* c) {
+  if (!c || c->d.copy_method != 3) return 0;
+  int n = c->d.copy_ctas > 0 ? c->d.copy_ctas : 4;
+  n = (n + 1) & ~1;
+  return std::min(n, 32);
+}
+
 int g_d2d_kernel = 1;   // experiments: 0 = driver D2D memcpy for HBM whole-entry loads
 bool cache_writes_all_rows(const fps_cache* c) { return c && c->d.copy_method == 2; }
 
@@ -122,7 +276,11 @@ fps_status fps_cache_create(const fps_cache_desc* desc, fps_cache_t* out) {
   FPS_CHECK_ARG(d.dtype == FPS_BF16 || d.dtype == FPS_F32, "dtype %d", d.dtype);
   FPS_CHECK_ARG(d.H > 0 && d.L_img > 0 && d.n_layers > 0 && d.n_steps > 0 && d.n_templates > 0,
                 "sizes must be positive");
-  FPS_CHECK_ARG(d.n_entries >= 0 && d.copy_method >= 0 && d.copy_method <= 2, "bad desc");
+  FPS_CHECK_ARG(d.n_entries >= 0 && d.copy_method >= 0 && d.copy_method <= 3, "bad desc");
+  FPS_CHECK_ARG(d.copy_method != 3 ||
+                    (size_t)(d.mode == FPS_MODE_KV ? 2 : 1) * d.H * (d.dtype == FPS_BF16 ? 2 : 4) <=
+                        (size_t)kBulkMaxRow,
+                "copy_method 3: rows wider than %d bytes", kBulkMaxRow);
   auto* c = new (std::nothrow) fps_cache();
   if (!c) return fail(FPS_ENOMEM, "cache: host allocation");
   c->d = d;
@@ -249,8 +407,11 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
     FPS_CHECK_ARG(it.dst_row_bytes == (int)row_bytes_of(c, it.layer),
                   "item %d: dst_row_bytes %d != entry row bytes %zu", i, it.dst_row_bytes,
                   row_bytes_of(c, it.layer));
-    if (c->d.copy_method == 0) FPS_CHECK_ARG(it.n_rows == 0 || it.d_rows, "item %d: d_rows", i);
-    else if (c->d.copy_method == 1)
+    // the row gather (method 0, and method 1 on the HBM arena) reads d_rows on the device;
+    // the per-run DMA reads h_rows on the host
+    if (c->d.copy_method == 0 || c->d.copy_method == 3 || (c->d.copy_method == 1 && c->d.location == 1))
+      FPS_CHECK_ARG(it.n_rows == 0 || it.d_rows, "item %d: d_rows needed for the row gather", i);
+    if (c->d.copy_method == 1 && c->d.location != 1)
       FPS_CHECK_ARG(it.n_rows == 0 || it.h_rows, "item %d: h_rows needed for DMA", i);
   }
   if (c->d.copy_method == 2) {
@@ -275,6 +436,42 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
       bytes += nb;
     }
     prof::end(s, prof::PREFETCH, 0, bytes);
+  } else if (c->d.copy_method == 3) {
+    // TMA bulk row gather: exactly the rows U, a few CTA pairs on reserved SMs
+    int max_rb = 0;
+    for (int i = 0; i < n_items; ++i) max_rb = std::max(max_rb, (int)row_bytes_of(c, items[i].layer));
+    const int slot_bytes = std::max(kBulkMinChunk, max_rb);
+    const int ctas = bulk_ctas(c);
+    const int slots = std::max(2, std::min({kBulkMaxSlots, (kBulkMaxSmem - kBulkHeader) / slot_bytes,
+                                             (kBulkInFlight + ctas * slot_bytes - 1) / (ctas * slot_bytes)}));
+    const int smem = kBulkHeader + slots * slot_bytes;
+    FPS_SMEM_ATTR(bulk_gather_kernel, kBulkMaxSmem);
+    for (int base = 0; base < n_items; base += kMaxPrefetchItems) {
+      BulkBatch b{};
+      b.slot_bytes = slot_bytes;
+      b.slots = slots;
+      double bytes = 0;
+      int k = 0;
+      for (int i = base; i < n_items && i < base + kMaxPrefetchItems; ++i) {
+        const fps_prefetch_item& it = items[i];
+        if (it.n_rows == 0) continue;
+        b.src[k] = c->dev_alias + offset_of(c, it.template_id, it.step, it.layer);
+        b.dst[k] = reinterpret_cast<char*>(it.d_dst);
+        b.rows[k] = it.d_rows;
+        b.n_rows[k] = it.n_rows;
+        b.row_bytes[k] = (int)row_bytes_of(c, it.layer);
+        bytes += (double)it.n_rows * b.row_bytes[k];
+        ++k;
+      }
+      b.n_items = k;
+      if (k == 0) continue;
+      prof::begin(s);
+      pdl_fence(s);    // plain launch: the load stream's kernels never overlap via PDL
+      FPS_CUDA_TRY(launch_k(bulk_gather_kernel, dim3(ctas), dim3(32), smem, s, b));
+      prof::end(s, prof::PREFETCH, 0, bytes);
+      count_launch();
+      FPS_LAUNCH_CHECK();
+    }
   } else if (c->d.copy_method == 0 || c->d.location == 1) {
     // (method 1 on the HBM arena takes the row gather too: a driver D2D copy per run would
     //  interleave with PDL launches, the pattern that hung in tools/hang_probe.py)

@@ -134,6 +134,11 @@ extern thread_local long long g_launches;
 inline void count_launch(int n = 1) { g_launches += n; }
 
 constexpr int kNumSMs = 148;
+// SMs left to the compute kernels: the pinned-host TMA row gather (cache copy_method 3) keeps
+// g_sm_reserved SMs (whole TPCs) for its CTAs while fps_run_batch runs, and the persistent
+// compute grids (GEMM, split-KV wave model) are sized to the rest, so neither waits for the other.
+extern int g_sm_reserved;
+inline int sm_budget() { return kNumSMs - g_sm_reserved; }
 
 // ---- per-kernel-class timing (fps_profile_enable / fps_profile_read) ----------------------
 // When enabled, every library launch is bracketed by a pair of CUDA events on its own stream;

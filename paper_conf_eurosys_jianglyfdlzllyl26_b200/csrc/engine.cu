@@ -84,6 +84,7 @@ struct fps_engine {
   long long stage_ctr = 0;
   bool no_reuse = false;   // experiments: admit every call
   bool no_transition = false;   // experiments: run a KV-mode plan's last dense block densely
+  bool skip_loads = false;      // measurement: no cache loads, slots keep their last contents
   bool call_start = false; // first step of a fps_run_batch call
   std::vector<cudaEvent_t> ready, consumed;
   cudaEvent_t step_start = nullptr, admit_done = nullptr;
@@ -133,6 +134,17 @@ static double flops_block(int mode, double n, double L, double H, double F, int 
 }
 
 }  // namespace fps
+
+// SMs kept for the cache's TMA row gather; FPS_SM_RESERVE=n overrides (experiments)
+static int reserved_sms(const fps_cache* c) {
+  using fps::bulk_ctas;
+  static const int forced = [] {
+    const char* v = getenv("FPS_SM_RESERVE");
+    return v ? atoi(v) : -1;
+  }();
+  const int n = bulk_ctas(c);
+  return n > 0 && forced >= 0 ? forced : n;
+}
 
 using namespace fps;
 
@@ -288,6 +300,10 @@ int64_t fps_engine_last_launches(fps_engine_t e) { return e ? e->last_launches :
 
 void fps_engine_set_admission_reuse(fps_engine_t e, int32_t on) {
   if (e) e->no_reuse = on == 0;
+}
+
+void fps_engine_set_skip_loads(fps_engine_t e, int32_t on) {
+  if (e) e->skip_loads = on != 0;
 }
 
 void fps_engine_set_kv_transition(fps_engine_t e, int32_t on) {
@@ -538,6 +554,10 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
       it.d_dst = dst + (size_t)B.h_cu_k[i] * row_bytes;
       it.dst_row_bytes = (int)row_bytes;
     }
+    if (e->skip_loads) {   // the no-load arm: only the ordering events, no bytes moved
+      FPS_CUDA_TRY(cudaEventRecord(ev, ls));
+      return FPS_OK;
+    }
     return fps_cache_prefetch(e->d.cache, items.data(), n, ls, ev);
   };
   auto try_issue = [&]() -> fps_status {
@@ -730,6 +750,13 @@ extern "C" fps_status fps_run_batch(fps_engine_t e, fps_request* reqs, int32_t n
   cudaStream_t cs = as_stream(compute_stream);
   cudaStream_t ls = load_stream ? as_stream(load_stream) : cs;
   const long long launches0 = g_launches;
+  // the TMA row gather (copy_method 3) keeps its SMs for the whole call: size the compute grids
+  // to the rest (restored on every return path)
+  struct SmReserve {
+    int prev;
+    explicit SmReserve(int n) : prev(g_sm_reserved) { g_sm_reserved = n; }
+    ~SmReserve() { g_sm_reserved = prev; }
+  } reserve(load_stream ? reserved_sms(e->d.cache) : 0);
   e->call_start = true;
   int done_steps = 0;
   while (done_steps < n_steps) {

@@ -1122,7 +1122,8 @@ static int choose_split(int ctas, int min_nk, int total_q, int H, int heads,
   if (g_attn_split > 0) return fits(g_attn_split) && min_nk >= g_attn_split ? g_attn_split : 1;
   auto eff = [&](int S) {
     const long long c = (long long)ctas * S;
-    return (double)c / (double)(((c + kNumSMs - 1) / kNumSMs) * kNumSMs);
+    const long long nb = sm_budget();
+    return (double)c / (double)(((c + nb - 1) / nb) * nb);
   };
   int best = 1;
   double be = eff(1);

@@ -692,7 +692,7 @@ static fps_status launch_cfg(const void* A, const void* B, int M, int N, int K,
   if (g2.M1 == 0) tb1 = tb;
   FPS_SMEM_ATTR((gemm_tc_kernel<BN, STAGES>), Cfg::SMEM);
   const int tiles = (ceil_div(M, Cfg::BM) + ceil_div(g2.M1, Cfg::BM)) * ceil_div(N, BN);
-  const int grid = tiles < kNumSMs ? tiles : kNumSMs;
+  const int grid = tiles < sm_budget() ? tiles : sm_budget();
   FPS_CUDA_TRY(launch_k(gemm_tc_kernel<BN, STAGES>, dim3(grid), dim3(256), Cfg::SMEM, s, ta, tb,
                         tb1, M, N, K, ep, g2.M1, g2.ep1));
   count_launch();
@@ -712,7 +712,7 @@ static fps_status launch_pair(const void* A, const void* B, int M, int N, int K,
   if (g2.M1 == 0) tb1 = tb;
   FPS_SMEM_ATTR((gemm_tc2_kernel<STAGES>), Cfg::SMEM);
   const int tiles = (ceil_div(M, Cfg::BM) + ceil_div(g2.M1, Cfg::BM)) * ceil_div(N, Cfg::BN);
-  const int pairs = tiles < kNumSMs / 2 ? tiles : kNumSMs / 2;
+  const int pairs = tiles < sm_budget() / 2 ? tiles : sm_budget() / 2;
   FPS_CUDA_TRY(launch_k(gemm_tc2_kernel<STAGES>, dim3(2 * pairs), dim3(256), Cfg::SMEM, s, ta, tb,
                         tb1, M, N, K, ep, g2.M1, g2.ep1));
   count_launch();
@@ -730,7 +730,7 @@ static fps_status launch_pair_swap(const void* A, const void* B, int M, int N, i
     return fail(FPS_ECUDA, "gemm_tc2s: cuTensorMapEncodeTiled failed (M=%d N=%d K=%d)", M, N, K);
   FPS_SMEM_ATTR((gemm_tc2s_kernel<STAGES>), Cfg::SMEM);
   const int tiles = ceil_div(M, NA) * ceil_div(N, 256);
-  const int pairs = tiles < kNumSMs / 2 ? tiles : kNumSMs / 2;
+  const int pairs = tiles < sm_budget() / 2 ? tiles : sm_budget() / 2;
   FPS_CUDA_TRY(launch_k(gemm_tc2s_kernel<STAGES>, dim3(2 * pairs), dim3(256), Cfg::SMEM, s, ta,
                         tb, M, N, K, NA, ep));
   count_launch();
@@ -745,7 +745,7 @@ static int swap_block(int M, int N, long* cost) {
   long bc = -1;
   for (int na = 256; na >= 64; na -= 16) {
     const long tiles = (long)ceil_div(M, na) * ceil_div(N, 256);
-    const long c = ((tiles + kNumSMs / 2 - 1) / (kNumSMs / 2)) * na;
+    const long c = ((tiles + sm_budget() / 2 - 1) / (sm_budget() / 2)) * na;
     if (bc < 0 || c < bc) {
       bc = c;
       best = na;
@@ -768,11 +768,11 @@ fps_status launch_gemm_tc_grouped(const void* A, const void* B0, const void* B1,
   const int m1 = ceil_div(M0, 128) + ceil_div(M1, 128), m2 = ceil_div(M0, 256) + ceil_div(M1, 256);
   const long t256 = (long)m1 * ceil_div(N, 256), t128 = (long)m1 * ceil_div(N, 128);
   const long tp = (long)m2 * ceil_div(N, 256);
-  const long c256 = ((t256 + kNumSMs - 1) / kNumSMs) * 256;
-  const long c128 = ((t128 + kNumSMs - 1) / kNumSMs) * 128;
-  const long cp = ((tp + kNumSMs / 2 - 1) / (kNumSMs / 2)) * 256;
+  const long c256 = ((t256 + sm_budget() - 1) / sm_budget()) * 256;
+  const long c128 = ((t128 + sm_budget() - 1) / sm_budget()) * 128;
+  const long cp = ((tp + sm_budget() / 2 - 1) / (sm_budget() / 2)) * 256;
   const long cmin = std::min(c256, c128);
-  const bool pair_wins = (tp > kNumSMs / 2 && K >= 1024) || cp < cmin;
+  const bool pair_wins = (tp > sm_budget() / 2 && K >= 1024) || cp < cmin;
   if (g_gemm_force == 2 || (g_gemm_force != 1 && pair_wins))
     return launch_pair<6>(A, B0, M0, N, K, ep0, s, g2);
   if (c256 <= c128) return launch_cfg<256, 4>(A, B0, M0, N, K, ep0, s, g2);
@@ -788,9 +788,9 @@ fps_status launch_gemm_tc(const void* A, const void* B, int M, int N, int K, con
   const int m1 = ceil_div(M, 128), m2 = ceil_div(M, 256);
   const long t256 = (long)m1 * ceil_div(N, 256), t128 = (long)m1 * ceil_div(N, 128);
   const long tp = (long)m2 * ceil_div(N, 256);
-  const long c256 = ((t256 + kNumSMs - 1) / kNumSMs) * 256;
-  const long c128 = ((t128 + kNumSMs - 1) / kNumSMs) * 128;
-  const long cp = ((tp + kNumSMs / 2 - 1) / (kNumSMs / 2)) * 256;
+  const long c256 = ((t256 + sm_budget() - 1) / sm_budget()) * 256;
+  const long c128 = ((t128 + sm_budget() - 1) / sm_budget()) * 128;
+  const long cp = ((tp + sm_budget() / 2 - 1) / (sm_budget() / 2)) * 256;
   // Measured (tools/gemm_probe.py, B200): the pair kernel reaches 95% tensor-pipe activity at
   // large M where the 1-SM kernel is L2-bound (1480 vs 1070 TFLOP/s at M = 29491); at one wave
   // the extra M padding of 256-row tiles can make it lose, so then padding decides.
@@ -802,7 +802,7 @@ fps_status launch_gemm_tc(const void* A, const void* B, int M, int N, int K, con
   // short K (< 1024, the SDXL-scale projections at C = 640): the pair's longer prologue and
   // epilogue are not amortised even over several waves (4916x1920x640: 30.2 vs 23.3 us for the
   // 1-SM kernel; 4916x5120x640: 54.8 vs 52.9; 16384x1920x640: 64.7 vs 61.3; K >= 1280: ties)
-  const bool pair_wins = (tp > kNumSMs / 2 && K >= 1024) || cp < cmin ||
+  const bool pair_wins = (tp > sm_budget() / 2 && K >= 1024) || cp < cmin ||
                          (cp == cmin && (m2 * 256 - M < 128 || K >= 8192));
   // swapped operands (activation rows on the MMA's N side, no 256-row M padding): correct and
   // tested, but measured no faster at the masked-block shapes (1331x9216x3072: 59.8 vs 59.2 us

@@ -84,6 +84,8 @@ bool attention_tc_supported(int dtype, int head_dim);
 // true if fps_cache_prefetch also overwrites rows outside U (copy_method 2): fresh rows written
 // into the same buffer must then be ordered after the load's ready event
 bool cache_writes_all_rows(const fps_cache* c);
+// CTAs the cache's TMA row gather (copy_method 3) runs on; 0 for the other methods
+int bulk_ctas(const fps_cache* c);
 
 // global switches (tests can force the SIMT kernels): bit0 = no tcgen05 GEMM,
 // bit1 = no tensor-core attention

@@ -166,7 +166,8 @@ def test_requests_leave_at_step_boundary(F):
 
 
 @pytest.mark.parametrize("slots,method,location", [(1, 0, 0), (2, 1, 0), (0, 0, 0), (2, 0, 1),
-                                                  (0, 2, 1), (1, 2, 1), (2, 2, 0)])
+                                                  (0, 2, 1), (1, 2, 1), (2, 2, 0), (0, 3, 0),
+                                                  (1, 3, 0), (2, 3, 0)])
 def test_pipeline_slots_and_copy_methods_bit_identical(F, slots, method, location):
     """The staging ring depth, the H2D method and the cache tier (pinned host / HBM) change
     timing only, never the bits."""
@@ -174,7 +175,8 @@ def test_pipeline_slots_and_copy_methods_bit_identical(F, slots, method, locatio
     for sl, me, lo in ((0, 0, 0), (slots, method, location)):
         _, _, _, _, eng, reqs = _setup(F, "kv", "bf16", 1, slots=sl, copy_method=me, seed=5100,
                                        location=lo)
-        eng.run_batch(reqs, 2)
+        # the second run on its own load stream (method 3 then reserves its SMs)
+        eng.run_batch(reqs, 2, load_stream=torch.cuda.Stream() if sl == slots else None)
         torch.cuda.synchronize()
         outs.append([r["x"].clone() for r in reqs])
     for a, b in zip(*outs):
@@ -198,7 +200,9 @@ def test_batched_run_dma_bit_identical(F, mode, slots):
 
 
 @pytest.mark.parametrize("mode,method,location", [("y", 0, 0), ("kv", 0, 0), ("kv", 2, 1),
-                                                  ("y", 2, 1), ("kv", 1, 0), ("y", 1, 0)])
+                                                  ("y", 2, 1), ("kv", 1, 0), ("y", 1, 0),
+                                                  ("kv", 2, 0), ("y", 2, 0), ("kv", 3, 0),
+                                                  ("y", 3, 0)])
 def test_delayed_load_stream_bit_identical(F, mode, method, location):
     """Robustness of the event ordering: a busy load stream (a long spin queued before the
     prefetches) must not change the result -- in particular a late whole-entry DMA (method 2)
@@ -337,7 +341,8 @@ def test_full_scale_stack_identical_input_invariant(F, mode):
 
 
 @pytest.mark.parametrize("mode,plan,copy_method", [("kv", [0, 1, 1], 1), ("y", [1, 0, 1], 0),
-                                                   ("kv", [1, 1, 1], 2), ("y", [1, 1, 1], 1)])
+                                                   ("kv", [1, 1, 1], 2), ("y", [1, 1, 1], 1),
+                                                   ("kv", [0, 1, 1], 3), ("y", [1, 0, 1], 3)])
 def test_cross_step_prefetch_matches_oracle_and_per_step_bits(F, mode, plan, copy_method):
     """Cross-step prefetch (R26) only moves loads earlier: over 2 steps the latents match the
     oracle and are bit-identical to the per-step pipeline's."""
@@ -347,7 +352,7 @@ def test_cross_step_prefetch_matches_oracle_and_per_step_bits(F, mode, plan, cop
                                                       copy_method=copy_method, cross_step=cross)
         for r in reqs:
             r["step0"] = r["step"]
-        eng.run_batch(reqs, 2)
+        eng.run_batch(reqs, 2, load_stream=torch.cuda.Stream())
         torch.cuda.synchronize()
         outs.append([r["x"].clone() for r in reqs])
         ref = _oracle(W, mods, deltas, cache_np, reqs, plan, mode, 2, 2)

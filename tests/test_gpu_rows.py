@@ -78,15 +78,22 @@ def test_empty_gather_is_noop(F):
     assert out.shape == (0, 8)
 
 
-@pytest.mark.parametrize("mode,method,location", [("kv", 0, 0), ("y", 0, 0), ("kv", 1, 0),
-                                                  ("y", 1, 0), ("kv", 0, 1), ("y", 0, 1),
-                                                  ("kv", 1, 1)])
-def test_cache_store_prefetch_bytes_equal(F, mode, method, location):
+@pytest.mark.parametrize("mode,method,location,H,ctas", [
+    ("kv", 0, 0, 256, 0), ("y", 0, 0, 256, 0), ("kv", 1, 0, 256, 0), ("y", 1, 0, 256, 0),
+    ("kv", 0, 1, 256, 0), ("y", 0, 1, 256, 0), ("kv", 1, 1, 256, 0),
+    ("kv", 2, 0, 256, 0), ("y", 2, 0, 256, 0), ("kv", 2, 1, 256, 0),
+    ("kv", 3, 0, 256, 0), ("y", 3, 0, 256, 0), ("kv", 3, 0, 3072, 0), ("y", 3, 0, 3072, 0),
+    ("kv", 3, 0, 1280, 6), ("kv", 3, 1, 640, 2), ("y", 3, 0, 4096, 1)])
+def test_cache_store_prefetch_bytes_equal(F, mode, method, location, H, ctas):
+    """a3: the prefetched rows are the stored entry's rows, byte for byte, at their token rows.
+    Exact-row methods (0, 1, 3) leave every other row untouched; the whole-entry DMA (2) lands
+    all L_img image rows of the entry (text rows untouched).  Method 3 (TMA bulk row gather)
+    also at Flux / SDXL row widths (one-row chunks, odd row sizes) and odd CTA counts."""
     g = synth.rng(102)
-    H, L_img, L_txt, N, S = 256, 1024, 64, 3, 2
+    L_img, L_txt, N, S = 1024, 64, 3, 2
     m = F.MODE_CODE[mode]
     c = F.Cache(m, F.FPS_BF16, H, L_img, N, S, n_templates=2, copy_method=method,
-                location=location)
+                location=location, copy_ctas=ctas)
     W = 2 * H if mode == "kv" else H
     layers = N + (1 if mode == "kv" else 0)
     ents = {}
@@ -125,7 +132,8 @@ def test_cache_store_prefetch_bytes_equal(F, mode, method, location):
         for r, t in enumerate((1, 0)):
             base = r * (L_img + L_txt)
             exp = np.zeros(((L_img + L_txt), w), np.float32)
-            exp[ids[r]] = ents[(t, s, layer)][ids[r]]
+            rows = np.arange(L_img) if method == 2 else ids[r]
+            exp[rows] = ents[(t, s, layer)][rows]
             assert np.array_equal(got[base:base + L_img + L_txt], exp)
     c.close()
 
