@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define FPS_ABI_VERSION 2
+#define FPS_ABI_VERSION 3
 
 typedef enum {
   FPS_OK = 0,
@@ -394,7 +394,21 @@ typedef struct {
                                       start as soon as their slots are consumed, and
                                       plan_policy 0 uses fps_plan_pipeline_cross; needs one
                                       slot per block (slots = 0 or >= n_layers)              */
+  int32_t sampler;                 /* the update after the stack (a9):
+                                      FPS_SAMPLER_EULER (0): synthetic x += h_deltas[s] * y
+                                        over the whole latent (reading R21);
+                                      FPS_SAMPLER_FLOW_BLEND (1): flow-matching Euler with
+                                        inpainting blend (reading R29): masked image rows
+                                        x += (sigma_{s+1} - sigma_s) y, unmasked image rows
+                                        x = (1 - sigma_{s+1}) z + sigma_{s+1} eps (the
+                                        request's template latent z re-noised with its noise
+                                        eps), text rows unchanged                            */
+  const float* h_sigmas;           /* [n_steps + 1] noise levels sigma_0 > ... > sigma_S
+                                      (FPS_SAMPLER_FLOW_BLEND; copied at create), else NULL  */
 } fps_engine_desc;
+
+#define FPS_SAMPLER_EULER 0
+#define FPS_SAMPLER_FLOW_BLEND 1
 
 typedef struct fps_engine* fps_engine_t;
 
@@ -406,6 +420,8 @@ typedef struct {
   void* d_x;               /* [L, H] device latent tokens, updated in place                 */
   int32_t status;          /* out: 0 = running, 1 = finished                                */
   const void* d_ctx;       /* [L_ctx, D_ctx] device prompt encoding (SDXL blocks), or NULL  */
+  const void* d_z;         /* [L_img, H] device template latent (FPS_SAMPLER_FLOW_BLEND)    */
+  const void* d_noise;     /* [L_img, H] device noise of the request (FPS_SAMPLER_FLOW_BLEND) */
 } fps_request;
 
 fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out);
@@ -446,6 +462,13 @@ void fps_engine_set_kv_transition(fps_engine_t e, int32_t on);
  * arm against which exposed load time is measured.  Results are NOT the
  * method's (the cached rows are stale); never use it for output. */
 void fps_engine_set_skip_loads(fps_engine_t e, int32_t on);
+/* Template run (L130 "prior full inference", L203 the activation store): when on, every block
+ * the step runs densely also stores its cache entry (template_id, step, layer) of each request
+ * -- KV-mode its K|V rows, Y-mode its output rows, rows [0, L_img) -- with fps_cache_store on
+ * the compute stream, and a KV-mode step that ends dense stores the final Y entry (layer =
+ * n_layers).  Run the template's requests with plan_policy 2 (all dense) to fill the cache.
+ * Default off. */
+void fps_engine_set_record(fps_engine_t e, int32_t on);
 
 #ifdef __cplusplus
 }

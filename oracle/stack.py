@@ -16,13 +16,16 @@ import numpy as np
 
 from .block import dense_block, f64, masked_block_kv, masked_block_y
 from .index import build_mask_index, gather_rows, scatter_rows
+from .sampler import flow_blend_update
 
 
-def template_run(x0, weights, mods, deltas, heads, steps, ctx=None, L_txt=0):
+def template_run(x0, weights, mods, deltas, heads, steps, ctx=None, L_txt=0, sampler=None):
     """Full (dense) inference of the template: the producer of the activation cache (L130,
     L203). mods[l][s] is block l's adaLN vector at step s.
 
     ctx: the request's prompt encoding (SDXL blocks only); L_txt: text rows (double-stream).
+    sampler: None = the synthetic update (R21); {"sigmas", "z", "eps"} = the flow-blend sampler
+    (R29) with no image row masked, i.e. the template's own latent re-noised along the schedule.
     Returns (cache, xs): cache[s][l] = {"K", "V", "Y"} full-L arrays; xs[s] = latent entering
     step s (xs[steps] = final latent)."""
     x = f64(x0)
@@ -36,7 +39,12 @@ def template_run(x0, weights, mods, deltas, heads, steps, ctx=None, L_txt=0):
             entries.append({"K": K, "V": V, "Y": y})
             cur = y
         cache.append(entries)
-        x = x + float(deltas[s]) * cur
+        if sampler is None:
+            x = x + float(deltas[s]) * cur
+        else:
+            L = x.shape[0]
+            x = flow_blend_update(x, cur, np.zeros(L, np.uint8), sampler["z"], sampler["eps"],
+                                  sampler["sigmas"][s], sampler["sigmas"][s + 1], L - L_txt)
     xs.append(x)
     return cache, xs
 
@@ -100,11 +108,16 @@ def euler_update(x, y, delta):
 
 
 def masked_run(x0, mask, weights, mods, deltas, use_cache, mode, cache, heads, steps,
-               step0=0, ctx=None, L_txt=0):
-    """Steps step0..step0+steps-1 of one request against the template cache."""
+               step0=0, ctx=None, L_txt=0, sampler=None):
+    """Steps step0..step0+steps-1 of one request against the template cache.  sampler: None =
+    the synthetic update (R21), or {"sigmas", "z", "eps"} for the flow-blend sampler (R29)."""
     x = f64(x0)
     for s in range(step0, step0 + steps):
         mods_s = [mods[l][s] for l in range(len(weights))]
         y = masked_stack(x, mask, weights, mods_s, use_cache, mode, cache[s], heads, ctx, L_txt)
-        x = euler_update(x, y, deltas[s])
+        if sampler is None:
+            x = euler_update(x, y, deltas[s])
+        else:
+            x = flow_blend_update(x, y, mask, sampler["z"], sampler["eps"], sampler["sigmas"][s],
+                                  sampler["sigmas"][s + 1], len(mask) - L_txt)
     return x

@@ -335,11 +335,13 @@ class Engine:
 
     def __init__(self, layers, heads, mode, dtype, L_img, L_txt, max_batch, n_steps, deltas,
                  cache: Cache, mod_table=None, slots=0, plan_policy=0, plan=None,
-                 cost_model=(0.0, 0.0, 0.0, 0.0), L_ctx=0, mod_width=0, cross_step=False):
+                 cost_model=(0.0, 0.0, 0.0, 0.0), L_ctx=0, mod_width=0, cross_step=False,
+                 sampler=0, sigmas=None):
         self.layers = layers                      # list[BlockWeights] (keeps tensors alive)
         self._w = (fps_block_weights * len(layers))(*[l.c for l in layers])
         self._deltas = (C.c_float * n_steps)(*map(float, deltas))
         self._plan = (C.c_uint8 * len(layers))(*(plan or [0] * len(layers)))
+        self._sigmas = (C.c_float * (n_steps + 1))(*map(float, sigmas)) if sigmas is not None else None
         self.mod_table = mod_table
         self.cache = cache
         H, F = layers[0].H, layers[0].F
@@ -348,7 +350,8 @@ class Engine:
                             C.cast(self._deltas, C.c_void_p), cache.h, slots, plan_policy,
                             C.cast(self._plan, C.c_void_p), (C.c_double * 4)(*cost_model),
                             L_ctx, max((getattr(l, "D_ctx", 0) for l in layers), default=0),
-                            mod_width, int(cross_step))
+                            mod_width, int(cross_step), int(sampler),
+                            C.cast(self._sigmas, C.c_void_p) if self._sigmas is not None else None)
         self.desc = d
         h = C.c_void_p()
         _lib.fps_engine_create(C.byref(d), C.byref(h))
@@ -372,7 +375,8 @@ class Engine:
         arr = (fps_request * max(len(reqs), 1))()
         for i, r in enumerate(reqs):
             arr[i] = fps_request(r["template_id"], r["step"], r["n_steps"], ptr(r["mask"]),
-                                 ptr(r["x"]), 0, ptr(r.get("ctx")))
+                                 ptr(r["x"]), 0, ptr(r.get("ctx")), ptr(r.get("z")),
+                                 ptr(r.get("noise")))
         ls = stream_ptr(load_stream) if load_stream is not None else None
         _lib.fps_run_batch(self.h, arr, len(reqs), n_steps, stream_ptr(stream), ls)
         for i, r in enumerate(reqs):

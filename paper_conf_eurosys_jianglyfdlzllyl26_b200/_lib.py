@@ -17,6 +17,7 @@ FPS_OK, FPS_EINVAL, FPS_ECUDA, FPS_ENOMEM, FPS_EUNSUPPORTED, FPS_ESTATE = 0, -1,
 FPS_F32, FPS_BF16 = 0, 1
 FPS_MODE_KV, FPS_MODE_Y = 0, 1
 FPS_BLOCK_SEQ, FPS_BLOCK_PAR, FPS_BLOCK_SDXL, FPS_BLOCK_DOUBLE = 0, 1, 2, 3
+FPS_SAMPLER_EULER, FPS_SAMPLER_FLOW_BLEND = 0, 1
 
 vp, i32, u32, i64, sz, dbl = C.c_void_p, C.c_int32, C.c_uint32, C.c_int64, C.c_size_t, C.c_double
 P_i32, P_u8, P_dbl, P_f32 = C.POINTER(C.c_int32), C.POINTER(C.c_uint8), C.POINTER(C.c_double), C.POINTER(C.c_float)
@@ -65,12 +66,12 @@ class fps_engine_desc(C.Structure):
                 ("n_steps", i32), ("layers", vp), ("d_mod_table", vp), ("h_deltas", vp),
                 ("cache", vp), ("slots", i32), ("plan_policy", i32), ("h_plan", vp),
                 ("cost_model", dbl * 4), ("L_ctx", i32), ("D_ctx", i32), ("mod_width", i32),
-                ("cross_step", i32)]
+                ("cross_step", i32), ("sampler", i32), ("h_sigmas", vp)]
 
 
 class fps_request(C.Structure):
     _fields_ = [("template_id", u32), ("step", i32), ("n_steps", i32), ("d_mask", vp),
-                ("d_x", vp), ("status", i32), ("d_ctx", vp)]
+                ("d_x", vp), ("status", i32), ("d_ctx", vp), ("d_z", vp), ("d_noise", vp)]
 
 
 # (name, restype, argtypes, checked)
@@ -118,6 +119,7 @@ _SIGS = [
     ("fps_engine_set_admission_reuse", None, [vp, i32], False),
     ("fps_engine_set_kv_transition", None, [vp, i32], False),
     ("fps_engine_set_skip_loads", None, [vp, i32], False),
+    ("fps_engine_set_record", None, [vp, i32], False),
 ]
 
 EXPORTED = [s[0] for s in _SIGS]

@@ -38,6 +38,7 @@ struct fps_engine {
   fps_engine_desc d{};
   std::vector<fps_block_weights> layers;
   std::vector<float> deltas;
+  std::vector<float> sigmas;          // flow-blend sampler (R29): sigma_0 .. sigma_S
   std::vector<uint8_t> fixed_plan;
   int L = 0, elt = 2, W = 0, D = 0;
   size_t row_h = 0, row_w = 0;  // bytes of an H row / a W row
@@ -85,6 +86,11 @@ struct fps_engine {
   bool no_reuse = false;   // experiments: admit every call
   bool no_transition = false;   // experiments: run a KV-mode plan's last dense block densely
   bool skip_loads = false;      // measurement: no cache loads, slots keep their last contents
+  bool record = false;          // template run: store the K|V / Y rows of every dense block
+  // flow-blend sampler: per-request (template latent, noise) pointers and step coefficients
+  void** h_zeps = nullptr;
+  void** d_zeps = nullptr;
+  float* d_coef = nullptr;
   bool call_start = false; // first step of a fps_run_batch call
   std::vector<cudaEvent_t> ready, consumed;
   cudaEvent_t step_start = nullptr, admit_done = nullptr;
@@ -111,6 +117,9 @@ static void free_engine(fps_engine* e) {
   int32_t* ib[] = {e->d_off, e->d_mids, e->d_uids, e->d_nm, e->d_meta};
   for (int32_t* p : ib) if (p) cudaFree(p);
   if (e->d_delta) cudaFree(e->d_delta);
+  if (e->d_coef) cudaFree(e->d_coef);
+  if (e->d_zeps) cudaFree(e->d_zeps);
+  if (e->h_zeps) cudaFreeHost(e->h_zeps);
   void* hb[] = {e->h_meta, e->h_mids, e->h_uids, e->h_nm, e->h_off, e->h_delta, e->h_stage};
   for (auto ev : e->stage_ev) if (ev) cudaEventDestroy(ev);
   for (void* p : hb) if (p) cudaFreeHost(p);
@@ -160,6 +169,9 @@ fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out) {
   FPS_CHECK_ARG(d.L_img > 0 && d.L_txt >= 0 && d.max_batch > 0 && d.n_steps > 0, "bad sizes");
   FPS_CHECK_ARG(d.layers && d.h_deltas && d.cache, "layers, h_deltas and cache are required");
   FPS_CHECK_ARG(d.plan_policy >= 0 && d.plan_policy <= 3, "plan_policy");
+  FPS_CHECK_ARG(d.sampler == FPS_SAMPLER_EULER || d.sampler == FPS_SAMPLER_FLOW_BLEND, "sampler %d",
+                d.sampler);
+  FPS_CHECK_ARG(d.sampler != FPS_SAMPLER_FLOW_BLEND || d.h_sigmas, "flow-blend sampler needs h_sigmas");
   FPS_CHECK_ARG(d.plan_policy != 3 || d.h_plan, "plan_policy 3 needs h_plan");
   if (d.plan_policy == 3 && d.mode == FPS_MODE_KV) {
     bool seen = false;
@@ -186,6 +198,8 @@ fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out) {
   e->d = d;
   e->layers.assign(d.layers, d.layers + d.n_layers);
   e->deltas.assign(d.h_deltas, d.h_deltas + d.n_steps);
+  if (d.sampler == FPS_SAMPLER_FLOW_BLEND) e->sigmas.assign(d.h_sigmas, d.h_sigmas + d.n_steps + 1);
+  e->d.h_sigmas = nullptr;
   if (d.plan_policy == 3) e->fixed_plan.assign(d.h_plan, d.h_plan + d.n_layers);
   e->d.layers = nullptr;
   e->d.h_deltas = nullptr;
@@ -251,6 +265,10 @@ fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out) {
   imal(&e->d_nm, d.max_batch);
   imal(&e->d_meta, meta_ints);
   if (err == cudaSuccess) err = cudaMalloc((void**)&e->d_delta, d.max_batch * 4);
+  if (err == cudaSuccess) err = cudaMalloc((void**)&e->d_coef, d.max_batch * 8);
+  if (err == cudaSuccess) err = cudaMalloc((void**)&e->d_zeps, std::max(1, 2 * d.max_batch) * sizeof(void*));
+  if (err == cudaSuccess)
+    err = cudaHostAlloc((void**)&e->h_zeps, std::max(1, 2 * d.max_batch) * sizeof(void*), cudaHostAllocDefault);
   auto hmal = [&](void** p, size_t bytes) {
     if (err == cudaSuccess) err = cudaHostAlloc(p, std::max<size_t>(bytes, 16), cudaHostAllocDefault);
   };
@@ -260,7 +278,7 @@ fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out) {
   hmal((void**)&e->h_nm, d.max_batch * 4);
   hmal((void**)&e->h_off, (d.max_batch + 1) * 4);
   hmal((void**)&e->h_delta, d.max_batch * 4);
-  e->stage_ints = (size_t)d.n_layers * d.max_batch + d.max_batch;
+  e->stage_ints = (size_t)d.n_layers * d.max_batch + 3 * (size_t)d.max_batch;   // mod ids | delta | coef
   hmal((void**)&e->h_stage, fps_engine::kStageRing * e->stage_ints * 4);
   for (int i = 0; i < fps_engine::kStageRing && err == cudaSuccess; ++i)
     err = cudaEventCreateWithFlags(&e->stage_ev[i], cudaEventDisableTiming);
@@ -302,6 +320,10 @@ void fps_engine_set_admission_reuse(fps_engine_t e, int32_t on) {
   if (e) e->no_reuse = on == 0;
 }
 
+void fps_engine_set_record(fps_engine_t e, int32_t on) {
+  if (e) e->record = on != 0;
+}
+
 void fps_engine_set_skip_loads(fps_engine_t e, int32_t on) {
   if (e) e->skip_loads = on != 0;
 }
@@ -330,6 +352,16 @@ static fps_status admit(fps_engine* e, fps_request* reqs, const std::vector<int>
   }
   e->h_off[n] = n * L;
   FPS_COPY_TRY(cs, cudaMemcpyAsync(e->d_off, e->h_off, (n + 1) * 4, cudaMemcpyHostToDevice, cs));
+  if (e->d.sampler == FPS_SAMPLER_FLOW_BLEND) {
+    for (int i = 0; i < n; ++i) {
+      FPS_CHECK_ARG(reqs[live[i]].d_z && reqs[live[i]].d_noise,
+                    "request %d: the flow-blend sampler needs d_z and d_noise", live[i]);
+      e->h_zeps[2 * i] = const_cast<void*>(reqs[live[i]].d_z);
+      e->h_zeps[2 * i + 1] = const_cast<void*>(reqs[live[i]].d_noise);
+    }
+    FPS_COPY_TRY(cs, cudaMemcpyAsync(e->d_zeps, e->h_zeps, 2 * n * sizeof(void*),
+                                     cudaMemcpyHostToDevice, cs));
+  }
   FPS_TRY(launch_mask_index(e->d_masks, e->d_off, n, L, e->d_mids, e->d_uids, e->d_nm, cs));
   FPS_COPY_TRY(cs, cudaMemcpyAsync(e->h_nm, e->d_nm, n * 4, cudaMemcpyDeviceToHost, cs));
   FPS_COPY_TRY(cs, cudaMemcpyAsync(e->h_mids, e->d_mids, (size_t)n * L * 4, cudaMemcpyDeviceToHost, cs));
@@ -518,6 +550,15 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
   }
   for (int i = 0; i < n; ++i) h_delta[i] = e->deltas[reqs[B.idx[i]].step];
   FPS_COPY_TRY(cs, cudaMemcpyAsync(e->d_delta, h_delta, n * 4, cudaMemcpyHostToDevice, cs));
+  if (e->d.sampler == FPS_SAMPLER_FLOW_BLEND) {
+    float* h_coef = h_delta + e->d.max_batch;
+    for (int i = 0; i < n; ++i) {
+      const int st = reqs[B.idx[i]].step;
+      h_coef[2 * i] = e->sigmas[st + 1] - e->sigmas[st];
+      h_coef[2 * i + 1] = e->sigmas[st + 1];
+    }
+    FPS_COPY_TRY(cs, cudaMemcpyAsync(e->d_coef, h_coef, n * 8, cudaMemcpyHostToDevice, cs));
+  }
   FPS_CUDA_TRY(cudaEventRecord(e->stage_ev[slot], cs));
 
   // ---- load schedule: ring loads (cached blocks in order) + KV-mode final Y load ----------
@@ -670,6 +711,14 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
       }
       char* dst = e->full[full_toggle];
       FPS_TRY(fps_dense_block_forward(w, &vd, cur_full, dst, e->kv_scratch, e->ws, e->ws_bytes, cs));
+      if (e->record)     // template run (L130, L203): this block's cache entry of every request
+        for (int i = 0; i < n; ++i) {
+          const fps_request& r = reqs[B.idx[i]];
+          const char* src = kv ? e->kv_scratch + (size_t)B.h_cu_k[i] * 2 * e->row_h
+                               : dst + (size_t)B.h_cu_k[i] * e->row_h;
+          FPS_TRY(fps_cache_store(e->d.cache, r.template_id, r.step, l, src,
+                                  (int)(kv ? 2 * e->row_h : e->row_h), cs));
+        }
       cur_full = dst;
       full_toggle ^= 1;
       rep_full = true;
@@ -724,7 +773,17 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
     else FPS_TRY(consume(j));          // Y-mode: block N-1's slot is read by the replenish
     y_src = e->y_full;
   }
-  FPS_TRY(launch_euler(e->d.dtype, e->x_full, y_src, B.tk, H, B.cu_k, n, e->d_delta, cs));
+  if (e->record && kv && rep_full)   // KV-mode replenish entry: the final block's Y rows
+    for (int i = 0; i < n; ++i) {
+      const fps_request& r = reqs[B.idx[i]];
+      FPS_TRY(fps_cache_store(e->d.cache, r.template_id, r.step, N,
+                              y_src + (size_t)B.h_cu_k[i] * e->row_h, (int)e->row_h, cs));
+    }
+  if (e->d.sampler == FPS_SAMPLER_FLOW_BLEND)
+    FPS_TRY(launch_flow_blend(e->d.dtype, e->x_full, y_src, n, e->L, e->d.L_img, H, e->d_masks,
+                              reinterpret_cast<const float2*>(e->d_coef), e->d_zeps, cs));
+  else
+    FPS_TRY(launch_euler(e->d.dtype, e->x_full, y_src, B.tk, H, B.cu_k, n, e->d_delta, cs));
   e->prev_ring = n_ring;
   if (!e->cross) {
     // the load stream must not run ahead into the next step's slots before this step is done
@@ -771,7 +830,8 @@ extern "C" fps_status fps_run_batch(fps_engine_t e, fps_request* reqs, int32_t n
     // synchronisation (callers stepping one step per call, e.g. a serving loop, pay it once)
     std::vector<const void*> key;
     for (int i : live)
-      key.insert(key.end(), {reqs[i].d_mask, reqs[i].d_x, reqs[i].d_ctx,
+      key.insert(key.end(), {reqs[i].d_mask, reqs[i].d_x, reqs[i].d_ctx, reqs[i].d_z,
+                             reqs[i].d_noise,
                              reinterpret_cast<const void*>((uintptr_t)reqs[i].template_id)});
     const bool reuse = e->last_valid && !e->no_reuse && key == e->last_key;
     Batch& B = e->last_B;

@@ -603,6 +603,70 @@ __global__ void __launch_bounds__(256) euler_kernel(T* __restrict__ x, const T* 
   }
 }
 
+// Flow-matching Euler step with inpainting blend (reading R29, NEXT-4; PAPER.md L73-L79 the
+// latent goes through N denoising steps, L157 masked rows computed / unmasked rows kept from the
+// template).  Per request r at its step s (coefficients coef[r] = (sigma_{s+1} - sigma_s,
+// sigma_{s+1})), row t of its latent:
+//   text row (t >= L_img)          unchanged (the prompt tokens are re-fed every step)
+//   masked image row (mask[t] != 0) x += (sigma_{s+1} - sigma_s) * y      (Euler on the velocity)
+//   unmasked image row               x  = (1 - sigma_{s+1}) * z[t] + sigma_{s+1} * eps[t]
+//                                        (the template latent re-noised to the next level)
+template <typename T>
+__global__ void __launch_bounds__(256) flow_blend_kernel(T* __restrict__ x, const T* __restrict__ y,
+                                                         long long nvec, int vpr, int L, int L_img,
+                                                         const uint8_t* __restrict__ mask,
+                                                         const float2* __restrict__ coef,
+                                                         const void* const* __restrict__ zeps) {
+  constexpr int NV = Vec16<T>::N;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nvec;
+       i += (long long)gridDim.x * blockDim.x) {
+    const int row = (int)(i / vpr), c = (int)(i - (long long)row * vpr);
+    const int r = row / L, t = row - r * L;
+    if (t >= L_img) continue;
+    const float2 cf = __ldg(coef + r);
+    float a[NV];
+    if (__ldg(mask + row)) {
+      float b[NV];
+      Vec16<T>::unpack(reinterpret_cast<const uint4*>(x)[i], a);
+      Vec16<T>::unpack(reinterpret_cast<const uint4*>(y)[i], b);
+#pragma unroll
+      for (int e = 0; e < NV; ++e) a[e] = a[e] + cf.x * b[e];
+    } else {
+      const uint4* z = reinterpret_cast<const uint4*>(zeps[2 * r]);
+      const uint4* ep = reinterpret_cast<const uint4*>(zeps[2 * r + 1]);
+      float b[NV];
+      Vec16<T>::unpack(z[(long long)t * vpr + c], a);
+      Vec16<T>::unpack(ep[(long long)t * vpr + c], b);
+#pragma unroll
+      for (int e = 0; e < NV; ++e) a[e] = (1.0f - cf.y) * a[e] + cf.y * b[e];
+    }
+    reinterpret_cast<uint4*>(x)[i] = Vec16<T>::pack(a);
+  }
+}
+
+fps_status launch_flow_blend(int dtype, void* x, const void* y, int n_req, int L, int L_img, int H,
+                             const uint8_t* mask, const float2* coef, const void* const* zeps,
+                             cudaStream_t s) {
+  const int n = n_req * L;
+  if (n <= 0) return FPS_OK;
+  const int elt = dtype == FPS_BF16 ? 2 : 4;
+  const int vpr = H * elt / 16;
+  const long long nvec = (long long)n * vpr;
+  int grid = (int)((nvec + 255) / 256);
+  if (grid > kNumSMs * 16) grid = kNumSMs * 16;
+  prof::begin(s);
+  if (dtype == FPS_BF16)
+    flow_blend_kernel<__nv_bfloat16><<<grid, 256, 0, s>>>(
+        (__nv_bfloat16*)x, (const __nv_bfloat16*)y, nvec, vpr, L, L_img, mask, coef, zeps);
+  else
+    flow_blend_kernel<float><<<grid, 256, 0, s>>>((float*)x, (const float*)y, nvec, vpr, L, L_img,
+                                                  mask, coef, zeps);
+  prof::end(s, prof::EULER, 2.0 * n * H, 3.0 * n * H * elt);
+  count_launch();
+  FPS_LAUNCH_CHECK();
+  return FPS_OK;
+}
+
 fps_status launch_euler(int dtype, void* x, const void* y, int n, int H, const int32_t* cu,
                         int n_req, const float* delta, cudaStream_t s) {
   if (n <= 0) return FPS_OK;

@@ -39,6 +39,12 @@ fps_status launch_geglu_pack(int dtype, const void* w, const void* b, int F, int
 // x[i] += delta[req(i)] * y[i] over rows of width H (req via cu over rows)
 fps_status launch_euler(int dtype, void* x, const void* y, int n, int H, const int32_t* cu,
                         int n_req, const float* delta, cudaStream_t s);
+// flow-matching Euler + inpainting blend (R29) over n_req request latents of L rows each:
+// masked image rows x += coef[r].x * y; unmasked image rows x = (1 - coef[r].y) z + coef[r].y eps
+// (zeps[2r], zeps[2r+1]: the request's [L_img, H] template latent and noise); text rows kept
+fps_status launch_flow_blend(int dtype, void* x, const void* y, int n_req, int L, int L_img, int H,
+                             const uint8_t* mask, const float2* coef, const void* const* zeps,
+                             cudaStream_t s);
 // GEMM C = A[M,K] B[N,K]^T with the fused epilogue
 fps_status launch_gemm(int dtype, const void* A, const void* B, int M, int N, int K,
                        const Epilogue& ep, cudaStream_t s);

@@ -5,6 +5,7 @@ import pytest
 import torch
 
 import synth
+from oracle import sampler as SM
 from oracle import stack as S
 from gpu_util import TOL, check_close, stack_tol, to_dev, to_np
 
@@ -20,7 +21,7 @@ def F():
 
 def _setup(F, mode, dtype, plan_policy, plan=None, N=3, steps=3, H=256, heads=2, Fd=512,
            L_img=256, L_txt=16, n_req=3, slots=0, copy_method=0, seed=5000, location=0,
-           kind="seq", cross_step=False, cost_model=(0.0, 0.0, 0.0, 0.0)):
+           kind="seq", cross_step=False, cost_model=(0.0, 0.0, 0.0, 0.0), sampler=0):
     g = synth.rng(seed)
     W = synth.stack_weights(g, N, H, Fd, dtype, kind)
     mods = synth.mod_table(g, N, steps, H, dtype)
@@ -50,7 +51,8 @@ def _setup(F, mode, dtype, plan_policy, plan=None, N=3, steps=3, H=256, heads=2,
     eng = F.Engine(layers, heads, m, dt, L_img, L_txt, max_batch=4, n_steps=steps, deltas=deltas,
                    cache=cache, mod_table=to_dev(mods, dtype), slots=slots,
                    plan_policy=plan_policy, plan=plan, cross_step=cross_step,
-                   cost_model=cost_model)
+                   cost_model=cost_model, sampler=sampler,
+                   sigmas=SM.flow_sigmas(steps, 3.0) if sampler else None)
     reqs = []
     ratios = [0.1, 0.45, 0.25, 0.6][:n_req]
     for i in range(n_req):
@@ -58,6 +60,9 @@ def _setup(F, mode, dtype, plan_policy, plan=None, N=3, steps=3, H=256, heads=2,
         x0 = synth.latent(g, L, H, dtype)
         reqs.append(dict(template_id=i % n_t, step=i % 2, n_steps=steps, mask_np=mask, x0=x0,
                          mask=torch.as_tensor(mask).cuda(), x=to_dev(x0, dtype)))
+        if sampler:      # flow-blend sampler (R29): the request's template latent and noise
+            z, eps = synth.latent(g, L_img, H, dtype), synth.latent(g, L_img, H, dtype)
+            reqs[-1].update(z_np=z, eps_np=eps, z=to_dev(z, dtype), noise=to_dev(eps, dtype))
     return W, mods, deltas, cache_np, eng, reqs
 
 
@@ -470,3 +475,84 @@ def test_kv_transition_planner_prices_each_suffix(F, cross):
         assert plan == best[1], (on, plan, best)
         assert 0 < sum(plan) < N, plan
         assert lat == pytest.approx(best[0], rel=1e-9)
+
+
+@pytest.mark.parametrize("mode,dtype,policy,plan", [
+    ("kv", "bf16", 1, None), ("y", "bf16", 3, [1, 0, 1]), ("kv", "f32", 3, [0, 1, 1]),
+    ("y", "f32", 1, None)])
+def test_flow_blend_sampler_matches_oracle(F, mode, dtype, policy, plan):
+    """NEXT-4 / R29: the flow-matching Euler sampler with inpainting blend after the stack --
+    masked image rows x += (sigma_{s+1} - sigma_s) y, unmasked image rows reset to the template
+    latent re-noised to sigma_{s+1}, text rows kept -- each request at its own step, over two
+    steps of a continuous batch, against the oracle's masked_run with the same sampler."""
+    W, mods, deltas, cache_np, eng, reqs = _setup(F, mode, dtype, policy, plan, sampler=1)
+    for r in reqs:
+        r["step0"] = r["step"]
+    eng.run_batch(reqs, 2, load_stream=torch.cuda.Stream())
+    torch.cuda.synchronize()
+    used = eng.last_plan()[0]
+    sig = SM.flow_sigmas(3, 3.0)
+    for r in reqs:
+        s0 = r["step0"]
+        n = min(2, r["n_steps"] - s0)
+        ref = S.masked_run(r["x0"], r["mask_np"], W, mods, deltas, used, mode,
+                           cache_np[r["template_id"]], 2, n, step0=s0, L_txt=16,
+                           sampler={"sigmas": sig, "z": r["z_np"], "eps": r["eps_np"]})
+        got = to_np(r["x"])
+        check_close(got, ref, stack_tol(dtype, 3), f"flow-blend {mode} {dtype} plan={used}")
+        # after the schedule's last step the unmasked image rows ARE the template latent
+        if s0 + n == r["n_steps"]:
+            U = np.flatnonzero(r["mask_np"][:256] == 0)
+            assert np.array_equal(got[U], to_np(r["z"])[U])
+
+
+def test_flow_blend_sampler_needs_template_latent(F):
+    W, mods, deltas, cache_np, eng, reqs = _setup(F, "kv", "bf16", 1, None, sampler=1)
+    del reqs[0]["noise"]
+    with pytest.raises(F.FlashPSError):
+        eng.run_batch(reqs, 1)
+
+
+@pytest.mark.parametrize("mode", ["kv", "y"])
+def test_record_cache_is_the_template_run(F, mode):
+    """fps_engine_set_record: a dense engine run stores each block's K|V (KV-mode) or output
+    (Y-mode) rows -- and KV-mode's final Y -- as the template's cache entries of that step;
+    they match the oracle's template run, and a masked run of the same request against them
+    reproduces the dense run bit for bit (L130 / L203: the cache is the template's prior full
+    inference)."""
+    g = synth.rng(5600)
+    N, steps, Hh, heads, Fd, L_img, L_txt = 3, 2, 256, 2, 512, 256, 16
+    L = L_img + L_txt
+    W = synth.stack_weights(g, N, Hh, Fd, "bf16")
+    mods = synth.mod_table(g, N, steps, Hh, "bf16")
+    deltas = synth.delta_table(steps)
+    m = F.MODE_CODE[mode]
+    cache = F.Cache(m, F.FPS_BF16, Hh, L_img, N, steps, n_templates=1)
+    layers = [F.BlockWeights(w, heads, F.FPS_BF16) for w in W]
+    x0 = synth.latent(g, L, Hh, "bf16")
+    mask = synth.token_mask(synth.mask_blobs(g, 16, 16, 0.3), L_txt)
+    outs = []
+    for policy, record in ((2, 1), (1, 0)):
+        eng = F.Engine(layers, heads, m, F.FPS_BF16, L_img, L_txt, 1, steps, deltas, cache,
+                       mod_table=to_dev(mods, "bf16"), plan_policy=policy, cross_step=True)
+        F.fps_engine_set_record(eng.h, record)
+        req = dict(template_id=0, step=0, n_steps=steps, mask=torch.as_tensor(mask).cuda(),
+                   x=to_dev(x0, "bf16"))
+        eng.run_batch([req], steps, load_stream=torch.cuda.Stream())
+        torch.cuda.synchronize()
+        outs.append(req["x"].clone())
+        eng.close()
+    assert torch.equal(outs[0].view(torch.int16), outs[1].view(torch.int16))
+    ref_cache, _ = S.template_run(x0, W, mods, deltas, heads, steps)
+    for s in range(steps):
+        for l in range(N + (1 if mode == "kv" else 0)):
+            e = cache.entry_numpy(0, s, l)
+            got = torch.as_tensor(e.view(np.int16)).view(torch.bfloat16).float().numpy()
+            if l == N:
+                ref = ref_cache[s][N - 1]["Y"][:L_img]
+            elif mode == "kv":
+                ref = np.concatenate([ref_cache[s][l]["K"], ref_cache[s][l]["V"]], 1)[:L_img]
+            else:
+                ref = ref_cache[s][l]["Y"][:L_img]
+            check_close(got, ref, stack_tol("bf16", (l + 1) + s * N), f"{mode} entry ({s},{l})")
+    cache.close()

@@ -33,7 +33,7 @@ def test_exports_every_declared_symbol():
 
 
 def test_abi_version():
-    assert fps.fps_abi_version() == 2
+    assert fps.fps_abi_version() == 3
 
 
 @pytest.mark.skipif(torch.cuda.is_available(), reason="CPU-only check")
