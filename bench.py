@@ -48,6 +48,9 @@ WORKLOADS = {
                 desc="SDXL-scale 64x64 level (640 ch), masks 10/30/50%, batch 4"),
 }
 SEED = 1003
+TIER_NAMES = {"host": "pinned host DRAM", "hbm": "device HBM (NEXT-1)",
+              "host_hugepage": "pinned host DRAM on 2 MiB pages",
+              "host_shared": "pinned host DRAM, one arena shared by all ranks (memfd)"}
 H2D_NAMES = ["SM row gather", "DMA of the unmasked row runs", "DMA of whole entries",
              "TMA bulk row gather (exact rows, reserved SMs)"]
 SDXL_CTX = (77, 2048)          # SDXL prompt encoding: 77 tokens x 2048 channels (R24)
@@ -58,14 +61,12 @@ def log(*a):
     print(*a, file=sys.stderr, flush=True)
 
 
-def ncu_traffic(kernel):
-    """DRAM bytes per launch of `kernel` from the newest committed ncu capture (profiles/)."""
-    import glob
-    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_traffic.json")))
-    if not files:
-        return None
-    d = json.load(open(files[-1]))
-    return d.get(kernel, {}).get("dram_bytes_per_launch")
+def ncu_summary(config, what):
+    """The committed ncu summary of the bench's own command for this config (profiles/ncu/):
+    what = "classes" (per-class kernel time of one step from the launch list) or "traffic"
+    (DRAM bytes per launch of each class over one step's launch mix).  None if absent."""
+    p = os.path.join(ROOT, "profiles", "ncu", f"{config}_{what}.json")
+    return json.load(open(p)) if os.path.exists(p) else None
 
 
 def peaks():
@@ -136,6 +137,17 @@ def make_requests(w, n_requests, seed):
     return reqs
 
 
+def route_job(pool, w, world, rank, cm):
+    """Alg. 2 over the job's request pool (L263-L287): every rank routes the same pool with the
+    same cost model (rank 0's fit), so all ranks agree on the assignment without any data-path
+    communication; each keeps its share.  Max batch per GPU = the config's batch (C4: 16 of a
+    16 x N pool of heterogeneous masks; C3: one request per GPU).
+    Returns (this rank's pool indices, the assignment of every rank, held requests)."""
+    from paper_conf_eurosys_jianglyfdlzllyl26_b200 import sched
+    L = w["L_img"] + w["L_txt"]
+    return sched.shard_requests([p["n_active"] for p in pool], L, world, rank, cm, w["batch"])
+
+
 COPY_CTAS = 0
 # Timing the calibration blocks under concurrent loads was tried: the noisier fit (R^2 0.84)
 # over-weights the intercept, the planner caches too many blocks and the step gets slower
@@ -143,10 +155,28 @@ COPY_CTAS = 0
 LOADED_CALIBRATION = False
 
 
+SHM_PATH = None      # location 3: the shared arena file every rank maps
+
+
 def make_cache(F, w, mode, n_entries, location=0, copy_method=0):
     return F.Cache(F.MODE_CODE[mode], F.FPS_BF16, w["H"], w["L_img"], w["layers"], w["steps"],
                    n_templates=64, n_entries=n_entries, copy_method=copy_method, location=location,
-                   copy_ctas=COPY_CTAS if location == 0 else 0)
+                   copy_ctas=COPY_CTAS if location != 1 else 0,
+                   shm_path=SHM_PATH if location == 3 else None)
+
+
+def weight_bytes(w):
+    """bf16 bytes of the stack's block weights (what every step streams from HBM)."""
+    H, Fd, N, blk = w["H"], w["F"], w["layers"], w.get("block", "seq")
+    seq = 3 * H * H + 3 * H + H * H + H + Fd * H + Fd + H * Fd + H
+    par = (3 * H + Fd) * H + 3 * H + Fd + H * (H + Fd) + H
+    D = SDXL_CTX[1]
+    sdxl = 3 * H * H + H * H + H + 2 * Fd * H + 2 * Fd + H * Fd + H + H * H + 2 * H * D + H * H + H + 6 * H
+    if blk == "flux":
+        n = FLUX_DOUBLE * 2 * seq + (N - FLUX_DOUBLE) * par
+    else:
+        n = N * {"seq": seq, "par": par, "sdxl": sdxl}[blk]
+    return 2 * n
 
 
 def build_engine_inputs(F, w, mode, device, n_entries, location=0, copy_method=0):
@@ -216,8 +246,48 @@ def build_engine_inputs(F, w, mode, device, n_entries, location=0, copy_method=0
 
 
 def calibrate(F, w, mode, layers, cache, reqs, device):
-    """Fit the §4.4 linear latency models on this GPU (L255-L257): masked / dense block time vs
-    FLOPs, and per-layer cache-load time vs bytes.  Returns (CostModel, fit info)."""
+    """Fit the §4.4 linear latency models on this GPU (L255-L257): block time vs FLOPs per block
+    kind (Flux's stack: the double-stream and the single-stream blocks separately), and
+    per-layer cache-load time vs bytes.  Returns (CostModel, fit info)."""
+    from paper_conf_eurosys_jianglyfdlzllyl26_b200 import sched
+    link = host_link_gbs(w, mode, device)
+    if w.get("block") == "flux":
+        fits = [_calibrate_one(F, w, mode, layers, cache, reqs, device, first=f)
+                for f in (0, FLUX_DOUBLE)]
+        cm, info = fits[0]
+        cm_p, info_p = fits[1]
+        N = w["layers"]
+        cm.layer_comp = [cm.comp] * FLUX_DOUBLE + [cm_p.comp] * (N - FLUX_DOUBLE)
+        # the stack-wide (a, b): FLOP-weighted mix, for the callers that take one model
+        fd = FLUX_DOUBLE / N
+        cm.comp = (fd * cm.comp[0] + (1 - fd) * cm_p.comp[0], fd * cm.comp[1] + (1 - fd) * cm_p.comp[1])
+        info = dict(info, comp_double=(info["comp_ms_per_tflop"], info["comp_b_ms"], info["comp_r2"]),
+                    comp_single=(info_p["comp_ms_per_tflop"], info_p["comp_b_ms"], info_p["comp_r2"]),
+                    comp_ms_per_tflop=cm.comp[0] * 1e12, comp_b_ms=cm.comp[1], link_gbs=link)
+        return cm, info
+    cm, info = _calibrate_one(F, w, mode, layers, cache, reqs, device)
+    info["link_gbs"] = link
+    return cm, info
+
+
+def host_link_gbs(w, mode, device, reps=8):
+    """The host link's copy-engine rate: pinned host -> HBM cudaMemcpyAsync of one cache entry
+    (L_img rows of the mode's width), back to back (the step roofline's link peak)."""
+    nb = w["L_img"] * (2 if mode == "kv" else 1) * w["H"] * 2
+    h = torch.empty(nb, dtype=torch.uint8).pin_memory()
+    d = torch.empty(nb, dtype=torch.uint8, device=device)
+    d.copy_(h, non_blocking=True)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(reps):
+        d.copy_(h, non_blocking=True)
+    e1.record()
+    torch.cuda.synchronize()
+    return reps * nb / (e0.elapsed_time(e1) * 1e-3) / 1e9
+
+
+def _calibrate_one(F, w, mode, layers, cache, reqs, device, first=0):
     from paper_conf_eurosys_jianglyfdlzllyl26_b200 import sched
     H, Fd, L = w["H"], w["F"], w["L_img"] + w["L_txt"]
     B = len(reqs)
@@ -234,7 +304,7 @@ def calibrate(F, w, mode, layers, cache, reqs, device):
                                     ld_dst[i * L].data_ptr(), Wl * 2) for i in range(B)]
     ld_stream = torch.cuda.Stream(device=device)
     kind = w.get("block", "seq")
-    kind = "double" if kind == "flux" else kind         # FLOPs per row: double == seq
+    kind = "double" if kind == "flux" else kind         # FLOPs per row: double == seq == par
     Lc = SDXL_CTX[0] if kind == "sdxl" else 0
     ctx_kv = (torch.randn(B * Lc, 2 * H, device=device).to(torch.bfloat16) if Lc else None)
     for m in (0.05, 0.2, 0.4, 0.7, 1.0):
@@ -250,9 +320,9 @@ def calibrate(F, w, mode, layers, cache, reqs, device):
         # consecutive blocks with their own weights, as in the stack (weights stream from HBM,
         # 226 MB per Flux block > L2), after enough work for the clocks to settle at the
         # power-capped level the step runs at
-        nl = min(8, len(layers))
+        nl = min(8, len(layers) - first)
         def fn():
-            for i in range(nl):
+            for i in range(first, first + nl):
                 F.masked_block_forward(layers[i], b, x, kv, y_act=y, ws=ws)
         # (a 1.5 s clock-settling burst before the fits made the predicted step match the
         # measured one within 1% but moved the plan to 45-46 cached blocks, measured slower than
@@ -317,8 +387,10 @@ def calibrate(F, w, mode, layers, cache, reqs, device):
     return cm, info
 
 
-def run_engine_timed(F, eng, reqs_dev, K, W, stream, load_stream, rank, world):
-    """W warm-up steps, then exactly K timed steps bracketed by barrier + synchronize."""
+def run_engine_timed(F, eng, reqs_dev, K, W, stream, load_stream, rank, world, ranged=False):
+    """W warm-up steps, then exactly K timed steps bracketed by barrier + synchronize.
+    ranged: bracket the K steps with cudaProfilerStart / Stop when FPS_PROFILE_RANGE is set
+    (ncu --profile-from-start off then records exactly the timed region's launches)."""
     import torch.distributed as dist
     for r in reqs_dev:
         r["step"], r["status"] = 0, 0
@@ -330,10 +402,15 @@ def run_engine_timed(F, eng, reqs_dev, K, W, stream, load_stream, rank, world):
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     l0 = F.fps_launch_count()
+    prof_range = ranged and os.environ.get("FPS_PROFILE_RANGE")
+    if prof_range:
+        torch.cuda.profiler.start()
     e0.record(stream)
     eng.run_batch(reqs_dev, K, stream=stream, load_stream=load_stream)
     e1.record(stream)
     torch.cuda.synchronize()
+    if prof_range:
+        torch.cuda.profiler.stop()
     launches = F.fps_launch_count() - l0
     ms = e0.elapsed_time(e1)
     if world > 1:
@@ -353,16 +430,18 @@ def dist_max(v):
     return float(t.item())
 
 
-def oracle_block_sample(w, mode, ratio, seed=7):
+def oracle_block_sample(w, mode, ratio, seed=7, kind=None):
     """CPU oracle: one mask-aware block for one request of the workload (fp64 numpy, all host
-    cores).  Returns seconds."""
+    cores).  Returns (seconds, the block's algorithmic FLOPs)."""
+    from paper_conf_eurosys_jianglyfdlzllyl26_b200.sched import block_flops
     from oracle import block as OB
     from oracle.index import build_mask_index
     g = synth.rng(seed)
     H, Fd, L_img, L_txt = w["H"], w["F"], w["L_img"], w["L_txt"]
     L = L_img + L_txt
-    kind = w.get("block", "seq")
-    kind = "double" if kind == "flux" else kind
+    if kind is None:
+        kind = w.get("block", "seq")
+        kind = "double" if kind == "flux" else kind
     wt = synth.block_weights(g, H, Fd, "bf16", kind, D_ctx=SDXL_CTX[1])
     ctx = synth.context(g, *SDXL_CTX, "bf16") if kind == "sdxl" else None
     mask = synth.token_mask(synth.mask_blobs(g, *w["grid"], ratio), L_txt)
@@ -375,7 +454,9 @@ def oracle_block_sample(w, mode, ratio, seed=7):
         OB.masked_block_kv(x[M], M, U, K[U], V[U], wt, mod, w["heads"], L, ctx, L_txt)
     else:
         OB.masked_block_y(x[M], M, U, x[U], wt, mod, w["heads"], L, ctx, L_txt)
-    return time.perf_counter() - t0
+    t = time.perf_counter() - t0
+    Lc = SDXL_CTX[0] if kind == "sdxl" else 0
+    return t, block_flops(mode, len(M), L, H, Fd, "sdxl" if kind == "sdxl" else "seq", Lc)
 
 
 def cpu_threads():
@@ -404,8 +485,13 @@ def main():
                          "block with cross-attention and GEGLU, or Flux's stack of 19 double-stream "
                          "then 38 single-stream blocks (NEXT-2); default: sdxl for the "
                          "SDXL-scale configs (C2A/C2B), flux for the Flux-scale ones (C3/C4)")
-    ap.add_argument("--tier", default="host", choices=["host", "hbm", "host_hugepage"],
-                    help="template cache in pinned host DRAM (configs[2]) or HBM (NEXT-1)")
+    ap.add_argument("--tier", default=None, choices=["host", "hbm", "host_hugepage", "host_shared"],
+                    help="template cache in pinned host DRAM (configs[2]), HBM (NEXT-1), on 2 MiB "
+                         "pages, or one pinned arena shared by all ranks of the box (default "
+                         "host at 1 GPU, host_shared with more ranks)")
+    ap.add_argument("--sampler", default="euler", choices=["euler", "flow"],
+                    help="update after the stack: the synthetic Euler step (R21) or the "
+                         "flow-matching Euler step with inpainting blend (R29)")
     ap.add_argument("--copy-ctas", type=int, default=0, help="CTAs of the SM row gather (0 = lib default)")
     ap.add_argument("--copy-method", type=int, default=None, choices=[0, 1, 2, 3],
                     help="H2D method: 0 SM zero-copy row gather, 1 one DMA per unmasked row run, "
@@ -422,9 +508,25 @@ def main():
     ap.add_argument("--no-extras", action="store_true", help="skip dense / Y-mode / profile legs")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        # one process per GPU: start the N ranks ourselves (the driver's own launch sets
+        # WORLD_SIZE and lands in the branch below)
+        import socket
+        with socket.socket() as so:
+            so.bind(("127.0.0.1", 0))
+            port = so.getsockname()[1]
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+               f"--nproc-per-node={args.gpus}", "--master-addr", "127.0.0.1",
+               "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+        log(f"launching {args.gpus} ranks: {' '.join(cmd)}")
+        sys.exit(subprocess.call(cmd))
+    if int(os.environ.get("WORLD_SIZE", 1)) != args.gpus:
+        log(f"--gpus {args.gpus} but WORLD_SIZE={os.environ.get('WORLD_SIZE', 1)}: refusing to "
+            f"report a {os.environ.get('WORLD_SIZE', 1)}-rank run as {args.gpus} GPUs")
+        sys.exit(2)
     import faulthandler                   # a stuck run dumps every thread's stack and exits
     import signal
-    faulthandler.dump_traceback_later(900, exit=True)
+    faulthandler.dump_traceback_later(int(os.environ.get("FPS_BENCH_TIMEOUT", 900)), exit=True)
     faulthandler.register(signal.SIGUSR1, all_threads=True)   # `timeout -s USR1`: dump stacks
     if args.copy_method is None:
         # measured on B200 (C3, profiles/r01f5_*): pinned host tier -- whole-entry DMA 34.6
@@ -435,6 +537,8 @@ def main():
     rank = int(os.environ.get("RANK", 0))
     world = int(os.environ.get("WORLD_SIZE", 1))
     local = int(os.environ.get("LOCAL_RANK", 0))
+    if args.tier is None:
+        args.tier = "host_shared" if world > 1 else "host"
     if args.block is None:       # the evaluated models' own block structure (R24, R25)
         args.block = "sdxl" if args.config.startswith("C2") else "flux"
     w = dict(WORKLOADS[args.config], block=args.block)
@@ -449,14 +553,14 @@ def main():
                 "head_dim": w["H"] // w["heads"], "mlp": w["F"], "tokens": L,
                 "image_tokens": w["L_img"], "text_tokens": w["L_txt"], "blocks": w["layers"],
                 "denoise_steps": S_IMG, "cache_mode": args.mode,
-                "batch_per_gpu": w["batch"], "block": args.block, "l2": "inputs > L2 (12.9 GB of weights streamed per step)"}
-    if w["L_txt"] == 0:
-        base_cfg["l2"] = "inputs > L2 (weights + activations streamed per step)"
+                "batch_per_gpu": w["batch"], "block": args.block,
+                "l2": f"inputs > L2 ({weight_bytes(w) / 1e9:.1f} GB of weights streamed per step)",
+                "sampler": {"euler": "synthetic Euler (R21)",
+                            "flow": "flow-matching Euler + inpainting blend (R29)"}[args.sampler]}
 
     metric_name = ("masked-block stack images/s (Flux-scale, 20% mask) [ms/step alongside]"
                    if args.config == "C3" else f"masked-block stack images/s ({args.config})")
-    base_cfg["cache_tier"] = {"host": "pinned host DRAM", "hbm": "device HBM (NEXT-1)",
-                              "host_hugepage": "pinned host DRAM on 2 MiB pages"}[args.tier]
+    base_cfg["cache_tier"] = TIER_NAMES[args.tier]
     base_cfg["h2d_method"] = H2D_NAMES[args.copy_method]
     base_cfg["parallelism"] = f"request-parallel x{world} (Alg. 2 routing)"
     base_cfg["cross_step_prefetch"] = bool(args.cross_step)
@@ -468,7 +572,7 @@ def main():
         # the oracle as it stands, one block of one request per step; extrapolated to the step
         times = []
         for i in range(W + K):
-            t = oracle_block_sample(w, args.mode, float(w["ratios"][0]), seed=11 + i)
+            t, _ = oracle_block_sample(w, args.mode, float(w["ratios"][0]), seed=11 + i)
             if i >= W:
                 times.append(t)
         block_s = statistics.mean(times)
@@ -511,30 +615,48 @@ def main():
     pool = make_requests(w, w["batch"] * world, SEED)
     t0 = time.perf_counter()
     n_entries = 2 * (w["layers"] + 1)
-    location = {"host": 0, "hbm": 1, "host_hugepage": 2}[args.tier]
-    global COPY_CTAS
+    location = {"host": 0, "hbm": 1, "host_hugepage": 2, "host_shared": 3}[args.tier]
+    global COPY_CTAS, SHM_PATH
     COPY_CTAS = args.copy_ctas
+    shm_fd = None
+    if location == 3:
+        # one pinned arena for every rank of the box: rank 0 makes a memfd, the others map it
+        # through /proc (setup only; host control, not the data path)
+        if rank == 0:
+            shm_fd = os.memfd_create("flashps_arena")
+            SHM_PATH = f"/proc/{os.getpid()}/fd/{shm_fd}"
+        if world > 1:
+            import torch.distributed as dist
+            obj = [SHM_PATH]
+            dist.broadcast_object_list(obj, src=0)
+            SHM_PATH = obj[0]
     layers, mod, cache = build_engine_inputs(F, w, args.mode, device, n_entries, location,
                                              args.copy_method)
     wbytes = sum(t.numel() * t.element_size() for l in layers for t in l.t.values())
-    base_cfg["l2"] = f"inputs > L2 ({wbytes / 1e9:.1f} GB of weights streamed per step)"
-    base_cfg["cache_tier"] = "pinned host DRAM" if location == 0 else "device HBM (NEXT-1)"
-    base_cfg["h2d_method"] = H2D_NAMES[args.copy_method]
+    assert abs(wbytes - weight_bytes(w)) < 1e6, (wbytes, weight_bytes(w))
     torch.cuda.synchronize()
     log(f"[rank {rank}] inputs ready in {time.perf_counter() - t0:.1f}s")
     my_pool = pool[:w["batch"]]
     log(f"[rank {rank}] calibrating")
-    cm, fit = calibrate(F, w, args.mode, layers, cache, [dict()] * w["batch"], device)
+    if world > 1 and n_dev < world:
+        # ranks sharing a device (the functional check of the multi-rank path on one GPU):
+        # calibrate one rank at a time so the fits do not time each other's kernels
+        import torch.distributed as dist
+        for r in range(world):
+            if r == rank:
+                cm, fit = calibrate(F, w, args.mode, layers, cache, [dict()] * w["batch"], device)
+            dist.barrier()
+    else:
+        cm, fit = calibrate(F, w, args.mode, layers, cache, [dict()] * w["batch"], device)
     log(f"[rank {rank}] fit {fit}")
     if world > 1:
         # every rank routes the same pool with Alg. 2; the cost models must be identical for the
         # assignments to agree, so all ranks use rank 0's fit (setup only, not on the data path)
         import torch.distributed as dist
-        obj = [(cm.comp, cm.load, fit)]
+        obj = [(cm.comp, cm.load, cm.layer_comp, fit)]
         dist.broadcast_object_list(obj, src=0)
-        cm.comp, cm.load, fit = obj[0]
-    my_ids, assign, held = sched.shard_requests([p["n_active"] for p in pool], L, world, rank, cm,
-                                                w["batch"])
+        cm.comp, cm.load, cm.layer_comp, fit = obj[0]
+    my_ids, assign, held = route_job(pool, w, world, rank, cm)
     mine = [pool[i] for i in my_ids]
     g = torch.Generator(device=device).manual_seed(SEED + rank)
     reqs_dev = []
@@ -546,15 +668,27 @@ def main():
                              x=torch.randn(L, w["H"], generator=g, device=device).to(torch.bfloat16)))
         if L_ctx:
             reqs_dev[-1]["ctx"] = torch.randn(*SDXL_CTX, generator=g, device=device).to(torch.bfloat16)
+        if args.sampler == "flow":     # the request's template latent and noise (R29)
+            reqs_dev[-1]["z"] = torch.randn(w["L_img"], w["H"], generator=g, device=device).to(torch.bfloat16)
+            reqs_dev[-1]["noise"] = torch.randn(w["L_img"], w["H"], generator=g, device=device).to(torch.bfloat16)
     stream = torch.cuda.current_stream()
     load_stream = torch.cuda.Stream(device=device)
     deltas = synth.delta_table(w["steps"])
 
-    def engine(policy, mode=args.mode, the_cache=cache):
+    sigmas = None
+    if args.sampler == "flow":
+        from oracle.sampler import FLUX_SHIFT      # a constant, not the oracle's arithmetic
+        t = 1.0 - np.arange(w["steps"]) / w["steps"]
+        sigmas = list(FLUX_SHIFT * t / (1.0 + (FLUX_SHIFT - 1.0) * t)) + [0.0]
+
+    def engine(policy, mode=args.mode, the_cache=cache, plan=None, model=None):
+        model = model or cm
         e = F.Engine(layers, w["heads"], F.MODE_CODE[mode], F.FPS_BF16, w["L_img"], w["L_txt"],
                      max(len(reqs_dev), 1), w["steps"], deltas, the_cache, mod_table=mod,
-                     slots=0, plan_policy=policy, cost_model=cm.as_engine_model(), L_ctx=L_ctx,
-                     mod_width=MODW, cross_step=bool(args.cross_step))
+                     slots=0, plan_policy=policy, plan=plan, cost_model=model.as_engine_model(),
+                     L_ctx=L_ctx, mod_width=MODW, cross_step=bool(args.cross_step),
+                     sampler=1 if args.sampler == "flow" else 0, sigmas=sigmas,
+                     layer_comp=model.layer_comp)
         F.fps_engine_set_kv_transition(e.h, args.kv_transition)
         return e
 
@@ -562,7 +696,8 @@ def main():
     F.fps_engine_set_admission_reuse(eng.h, args.admission_reuse)
     log(f"[rank {rank}] timed run")
     with Clocks(local % n_dev) as clk:
-        step_ms, launches = run_engine_timed(F, eng, reqs_dev, K, W, stream, load_stream, rank, world)
+        step_ms, launches = run_engine_timed(F, eng, reqs_dev, K, W, stream, load_stream, rank, world,
+                                             ranged=True)
     plan, pred_ms = eng.last_plan()
     imgs = sum(len(a) for a in assign)
     value = imgs / (step_ms * 1e-3 * S_IMG)
@@ -581,21 +716,17 @@ def main():
         cached_ms, _ = run_engine_timed(F, eng_c, reqs_dev, K, W, stream, load_stream, rank, world)
         del eng_c
         extras.update(dense_ms_per_step=dense_ms, all_cached_ms_per_step=cached_ms)
-        # the same plan with every cache entry already resident in HBM: the step without any
-        # host-link load; exposed load = this step - that step
-        if location != 1:
-            log(f"[rank {rank}] extras: same plan, HBM-resident cache")
-            c_h = make_cache(F, w, args.mode, n_entries, 1, 2)
-            eng_h = F.Engine(layers, w["heads"], F.MODE_CODE[args.mode], F.FPS_BF16, w["L_img"],
-                             w["L_txt"], max(len(reqs_dev), 1), w["steps"], deltas, c_h,
-                             mod_table=mod, slots=0, plan_policy=3, plan=list(plan), L_ctx=L_ctx,
-                             mod_width=MODW, cross_step=bool(args.cross_step))
-            noload_ms, _ = run_engine_timed(F, eng_h, reqs_dev, K, W, stream, load_stream, rank,
-                                            world)
-            del eng_h
-            c_h.close()
-            extras["same_plan_no_load_ms_per_step"] = noload_ms
-            extras["exposed_load_ms_per_step"] = max(step_ms - noload_ms, 0.0)
+        # the same plan, same engine and cache, with the loads switched off
+        # (fps_engine_set_skip_loads: ready events still recorded, no bytes moved; the staging
+        # slots keep an earlier step's rows): the step without host-link load. Exposed load =
+        # this step - that step, signed
+        log(f"[rank {rank}] extras: same plan, loads skipped")
+        eng_n = engine(3, plan=list(plan))
+        F.fps_engine_set_skip_loads(eng_n.h, 1)
+        noload_ms, _ = run_engine_timed(F, eng_n, reqs_dev, K, W, stream, load_stream, rank, world)
+        del eng_n
+        extras["same_plan_no_load_ms_per_step"] = noload_ms
+        extras["exposed_load_ms_per_step"] = step_ms - noload_ms
         # the other caching mode, and both modes with the other cache tier, on the same batch
         other = "y" if args.mode == "kv" else "kv"
         other_loc = 0 if location == 1 else 1
@@ -606,16 +737,13 @@ def main():
                                (args.mode, location, 2 if args.copy_method != 2 else 1)):
             if loc == 1 and cmeth == 1:
                 continue
+            loc = 0 if loc == 3 else loc        # the shared arena file belongs to `cache`
             log(f"[rank {rank}] extras: mode {md} location {loc} copy method {cmeth}")
             c2 = make_cache(F, w, md, n_entries, loc, cmeth)
             cm2, _ = calibrate(F, w, md, layers, c2, [dict()] * w["batch"], device)
-            eng_o = F.Engine(layers, w["heads"], F.MODE_CODE[md], F.FPS_BF16, w["L_img"],
-                             w["L_txt"], max(len(reqs_dev), 1), w["steps"], deltas, c2,
-                             mod_table=mod, slots=0, plan_policy=0,
-                             cost_model=cm2.as_engine_model(), L_ctx=L_ctx, mod_width=MODW,
-                             cross_step=bool(args.cross_step))
+            eng_o = engine(0, mode=md, the_cache=c2, model=cm2)
             o_ms, _ = run_engine_timed(F, eng_o, reqs_dev, K, W, stream, load_stream, rank, world)
-            tag = f"{md}_mode_{['host', 'hbm', 'host_hugepage'][loc]}"
+            tag = f"{md}_mode_{['host', 'hbm', 'host_hugepage', 'host_shared'][loc]}"
             if cmeth != default_cm(loc):
                 tag += "_" + ["row_gather", "run_dma", "whole_entry_dma", "tma_row_gather"][cmeth]
             extras[f"{tag}_ms_per_step"] = o_ms
@@ -635,8 +763,29 @@ def main():
     P = C.POINTER(C.c_double)
     F.fps_profile_read(ms.ctypes.data_as(P), fl.ctypes.data_as(P), by.ctypes.data_as(P),
                        cnt.ctypes.data_as(C.POINTER(C.c_int64)))
-    F.fps_profile_enable(0)
     names = ["gemm_tcgen05", "attention", "rownorm", "row_copy", "cache_prefetch", "sampler", "mask_index"]
+    # launch timeline of the same pass: the compute stream's and the load stream's classes
+    # separately (the load stream overlaps the compute stream, so only the compute stream's
+    # classes add up to the step)
+    nmax = 400000
+    st_, en_ = np.zeros(nmax), np.zeros(nmax)
+    kd_, sid_ = np.zeros(nmax, np.int32), np.zeros(nmax, np.int64)
+    ntr = F.fps_profile_trace(st_.ctypes.data_as(P), en_.ctypes.data_as(P),
+                              kd_.ctypes.data_as(C.POINTER(C.c_int32)),
+                              sid_.ctypes.data_as(C.POINTER(C.c_int64)), nmax)
+    F.fps_profile_enable(0)
+    comp_sid = stream.cuda_stream
+    on_comp = sid_[:ntr] == comp_sid
+    dur = en_[:ntr] - st_[:ntr]
+    stream_split = {
+        "compute_stream_ms_per_step": float(dur[on_comp].sum()) / (W + K),
+        "load_stream_ms_per_step": float(dur[~on_comp].sum()) / (W + K),
+        "compute_stream_by_class": {names[k]: float(dur[on_comp & (kd_[:ntr] == k)].sum()) / (W + K)
+                                    for k in range(7) if (on_comp & (kd_[:ntr] == k)).any()},
+        "note": "CUDA events around every library launch on its own stream (the events break "
+                "PDL overlap, so the profiled step runs a little longer than the timed one); "
+                "per-class times of the undisturbed step come from the ncu launch list "
+                "(kernels_ncu)"}
     # the profiled pass covers warm-up + timed steps; report per step of the timed region share
     per = {names[k]: {"ms_per_step": ms[k] / (W + K), "launches_per_step": cnt[k] / (W + K),
                       "tflops": (fl[k] / (ms[k] * 1e-3) / 1e12) if ms[k] > 0 and fl[k] > 0 else None,
@@ -648,13 +797,32 @@ def main():
     roofline = {"bound": "tensor", "kernel": "gemm_tcgen05 (a5/a7/a8 projections + MLP)",
                 "achieved": gemm_achieved, "peak": bf16_sust, "unit": "TFLOP/s",
                 "frac": gemm_achieved / bf16_sust, "peak_source": f"{src} bf16_tflops_sustained",
-                "traffic": ncu_traffic("gemm_tcgen05"),
-                "traffic_source": "dram__bytes_read.sum + dram__bytes_write.sum per launch, from "
-                                  "the newest ncu --set full captures in profiles/*_traffic.json "
-                                  "(masked-block GEMMs at the bench's shapes)",
+                "traffic": None, "traffic_source": None,
                 "algorithmic_bytes_per_launch": by[0] / max(cnt[0], 1),
                 "avg_launch_ms": gemm_avg_ms,
                 "flops_per_launch": fl[0] / max(cnt[0], 1)}
+    tr = ncu_summary(args.config, "traffic")
+    if tr and "gemm_tcgen05" in tr:
+        roofline["traffic"] = tr["gemm_tcgen05"]["dram_bytes_per_launch"]
+        roofline["traffic_source"] = tr["source"]
+    # step roofline for the chosen plan: the slower of the tensor work at the sustained peak,
+    # the exact unmasked rows over the host link at its measured rate, and one pass of the
+    # weights over HBM
+    step_flops = (fl[0] + fl[1]) / (W + K)
+    n_cached = int(sum(plan))
+    Wl = (2 if args.mode == "kv" else 1) * w["H"] * 2
+    u_rows = sum(w["L_img"] - (p["n_active"] - w["L_txt"]) for p in mine)   # unmasked rows U
+    exact_bytes = n_cached * u_rows * Wl + ((u_rows * w["H"] * 2) if (args.mode == "kv" and n_cached) else 0)
+    link_gbs = fit.get("link_gbs") or fit.get("load_gbs")
+    t_comp = step_flops / (bf16_sust * 1e12) * 1e3
+    t_link = exact_bytes / (link_gbs * 1e9) * 1e3 if (location != 1 and link_gbs) else 0.0
+    t_hbm = weight_bytes(w) / (hbm * 1e9) * 1e3
+    ideal = max(t_comp, t_link, t_hbm)
+    step_roofline = {"ideal_ms": ideal, "frac": ideal / step_ms, "compute_ms": t_comp,
+                     "link_ms": t_link, "hbm_ms": t_hbm, "step_tflop": step_flops / 1e12,
+                     "exact_row_link_bytes": exact_bytes, "link_gbs": link_gbs,
+                     "link_source": "copy-engine DMA rate of whole entries, measured in the calibration",
+                     "bound": ["tensor", "host link", "hbm"][[t_comp, t_link, t_hbm].index(ideal)]}
 
     log(f"[rank {rank}] e2e")
     # e2e through the public call with HOST buffers: per step H2D latents, one step, D2H latents
@@ -685,15 +853,23 @@ def main():
     if rank == 0:
         cpu = None
         if not args.no_cpu and world == 1:
-            times = [oracle_block_sample(w, args.mode, float(w["ratios"][0]), seed=11 + i)
-                     for i in range(3)]
-            blk = statistics.mean(times)
-            cpu_step_ms = blk * 1e3 * w["layers"] * w["batch"]
-            cpu = {"value": w["batch"] / (cpu_step_ms * 1e-3 * S_IMG), "unit": metric_unit,
+            # the oracle's FLOP rate on one mask-aware block of each kind in the stack, then the
+            # timed plan's FLOPs (dense prefix, transition block, cached suffix) at that rate
+            kinds = ["double", "par"] if args.block == "flux" else [args.block]
+            secs, flops = 0.0, 0.0
+            for i, kd in enumerate(kinds):
+                t, f = oracle_block_sample(w, args.mode, float(w["ratios"][0]), seed=11 + i, kind=kd)
+                secs += t
+                flops += f
+            rate = flops / secs
+            cpu_step_ms = step_flops / rate * 1e3
+            cpu = {"value": imgs / (cpu_step_ms * 1e-3 * S_IMG), "unit": metric_unit,
                    "cores": cpu_threads(), "kind": "oracle",
-                   "sample": f"3 x (1 mask-aware block x 1 request, fp64 numpy, m={w['ratios'][0]}),"
-                             f" extrapolated x{w['layers']} blocks x{w['batch']} requests x{S_IMG} steps",
-                   "block_s": blk}
+                   "sample": f"{len(kinds)} mask-aware block(s) ({'/'.join(kinds)}) x 1 request, fp64 "
+                             f"numpy, m={w['ratios'][0]}: {secs:.1f} s for {flops / 1e9:.0f} GFLOP; "
+                             f"the timed plan's {step_flops / 1e12:.2f} TFLOP/step ({n_cached} cached "
+                             f"of {len(plan)} blocks) priced at that rate, x{S_IMG} steps",
+                   "oracle_gflops": rate / 1e9, "step_ms": cpu_step_ms}
         mean_n = statistics.mean(p["n_active"] for p in mine) if mine else 0
         out = {
             "metric": metric_name,
@@ -710,6 +886,9 @@ def main():
             "plan": {"cached_blocks": int(sum(plan)), "blocks": len(plan),
                      "predicted_ms_per_step": pred_ms, "fit": fit},
             "kernels": per,
+            "kernels_stream_split": stream_split,
+            "kernels_ncu": ncu_summary(args.config, "classes"),
+            "step_roofline": step_roofline,
             "extras": extras,
         }
         if extras.get("dense_ms_per_step"):
@@ -724,10 +903,12 @@ def main():
                 out["extras"]["saving_vs_ideal_literal"] = (dms - step_ms) / (dms * (1 - m))
                 out["extras"]["saving_vs_ideal_active_rows"] = (dms - step_ms) / (dms * (1 - frac_active))
         if "exposed_load_ms_per_step" in extras:
-            load_ms = per["cache_prefetch"]["ms_per_step"]
+            load_ms = stream_split["load_stream_ms_per_step"]
+            ex = extras["exposed_load_ms_per_step"]
             out["extras"]["load_ms_per_step"] = load_ms
-            out["extras"]["load_overlap_frac"] = (1 - extras["exposed_load_ms_per_step"] / load_ms
-                                                  if load_ms > 0 else None)
+            # hidden share of the load time; a negative exposed time (the step with loads ran
+            # faster than the one without, i.e. within run-to-run noise) is reported as is
+            out["extras"]["load_overlap_frac"] = (1 - max(ex, 0.0) / load_ms) if load_ms > 0 else None
         print(json.dumps(out), flush=True)
     if world > 1:
         import torch.distributed as dist

@@ -133,25 +133,41 @@ typedef struct {
   int32_t n_entries;     /* physical entries in the pinned arena; 0 = one per key.  When
                             smaller, key k maps to entry k % n_entries (perf runs only: bytes
                             moved are identical, contents alias)                            */
-  int32_t copy_method;   /* 0 = SM row gather (zero-copy over mapped pinned memory, or from
-                                the HBM arena) -- exactly the rows U (default);
+  int32_t copy_method;   /* how fps_cache_prefetch moves an entry's rows U (all four give the
+                            same bytes at rows U; DESIGN.md §6 has the measurements):
+                            0 = SM row gather (zero-copy over mapped pinned memory, or from
+                                the HBM arena) -- exactly the rows U, but its warps share the
+                                SMs with the compute stream;
                             1 = copy-engine DMA of exactly the rows U: one cudaMemcpyAsync
-                                per run of consecutive tokens, on the load stream (on the HBM
+                                per run of consecutive tokens on the load stream (on the HBM
                                 arena, location 1, the rows go through the method-0 gather);
-                                Full link rate on only the unmasked bytes: the pinned-host
-                                default of the bench;
+                                per-copy overhead: ~47 GB/s on blob masks, ~12 GB/s on
+                                random masks (hundreds of runs);
                             2 = copy-engine DMA of the WHOLE entry (all L_img rows, one copy
-                                per request): no SM time, but rows outside U are overwritten
-                                too, so fresh K/V must be written only after `ready_event`
-                                (fps_run_batch orders this itself).  Meant for the HBM tier,
-                                where the extra bytes are cheap and SM time is not.            */
+                                per request): no SM time, full link rate on 1/(1-m) more
+                                bytes; rows outside U are overwritten too, so fresh K/V must
+                                be written only after `ready_event` (fps_run_batch orders
+                                this itself).  The bench default on both tiers;
+                            3 = TMA bulk row gather: exactly the rows U, moved host -> smem
+                                -> HBM by cp.async.bulk from copy_ctas CTAs (default 4, in
+                                TPC pairs) at ~51 GB/s of useful bytes; fps_run_batch with a
+                                load stream sizes its compute grids to the other SMs.  Pinned
+                                host tiers only need it; rows <= 32 KB                       */
   int32_t copy_ctas;     /* CTAs used by method 0 (0 = default: 16 for the host link -- enough
                             for PCIe, few enough not to crowd out the compute stream -- and 64
-                            for the HBM tier)                                               */
+                            for the HBM tier) and by method 3 (0 = 4)                        */
   int32_t location;      /* 0 = pinned host DRAM (L203, streamed over PCIe);
                             1 = device HBM: the template tier one level above host DRAM
                             (the paper's "ideal" no-load case of Fig. 4-Left,
-                            L108), prefetch becomes an HBM row gather                        */
+                            L108), prefetch becomes an HBM row gather;
+                            2 = pinned host DRAM on 2 MiB pages (THP);
+                            3 = pinned host DRAM SHARED by the worker processes of a box
+                                (SURVEY §8(e)): the file at shm_path (created / grown to the
+                                arena size if needed) is mapped MAP_SHARED and page-locked by
+                                each process -- one copy of the templates for all GPUs       */
+  const char* shm_path;  /* location 3: path of the shared arena file (e.g. a memfd opened
+                            as /proc/<pid>/fd/<n>, or /dev/shm/<name>); the caller removes
+                            it; NULL otherwise                                               */
 } fps_cache_desc;
 
 typedef struct fps_cache* fps_cache_t;
@@ -177,9 +193,11 @@ typedef struct {
   int32_t step;
   int32_t layer;
   int32_t n_rows;
-  const int32_t* d_rows;   /* device, [n_rows] local row ids (unmasked tokens U)          */
-  const int32_t* h_rows;   /* host mirror of d_rows (used by copy_method 1; may be NULL
-                              for method 0)                                                */
+  const int32_t* d_rows;   /* device, [n_rows] local row ids (unmasked tokens U); read by
+                              the row gathers: methods 0 and 3, and method 1 on the HBM
+                              arena (FPS_EINVAL if NULL there)                             */
+  const int32_t* h_rows;   /* host mirror of d_rows: read by method 1 on a host arena (one
+                              DMA per run); may be NULL otherwise                          */
   void* d_dst;             /* device row 0 of this request's [L, W] region                */
   int32_t dst_row_bytes;
 } fps_prefetch_item;
@@ -405,6 +423,10 @@ typedef struct {
                                         eps), text rows unchanged                            */
   const float* h_sigmas;           /* [n_steps + 1] noise levels sigma_0 > ... > sigma_S
                                       (FPS_SAMPLER_FLOW_BLEND; copied at create), else NULL  */
+  const double* h_layer_comp;      /* [n_layers][2] per-block compute models (a_l, b_l) in
+                                      cost_model units -- e.g. fitted per block kind (§4.4
+                                      regression per block type); NULL = cost_model[0..1] for
+                                      every block.  Copied at create.                        */
 } fps_engine_desc;
 
 #define FPS_SAMPLER_EULER 0

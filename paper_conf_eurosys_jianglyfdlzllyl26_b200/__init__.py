@@ -291,9 +291,10 @@ class Cache:
     """fps_cache_t: pinned host arena of template activations (L203)."""
 
     def __init__(self, mode, dtype, H, L_img, n_layers, n_steps, n_templates=1, n_entries=0,
-                 copy_method=0, copy_ctas=0, location=0):
+                 copy_method=0, copy_ctas=0, location=0, shm_path=None):
+        self._shm = shm_path.encode() if shm_path else None
         self.desc = fps_cache_desc(mode, dtype, H, L_img, n_layers, n_steps, n_templates,
-                                   n_entries, copy_method, copy_ctas, location)
+                                   n_entries, copy_method, copy_ctas, location, self._shm)
         h = C.c_void_p()
         _lib.fps_cache_create(C.byref(self.desc), C.byref(h))
         self.h = h
@@ -336,12 +337,14 @@ class Engine:
     def __init__(self, layers, heads, mode, dtype, L_img, L_txt, max_batch, n_steps, deltas,
                  cache: Cache, mod_table=None, slots=0, plan_policy=0, plan=None,
                  cost_model=(0.0, 0.0, 0.0, 0.0), L_ctx=0, mod_width=0, cross_step=False,
-                 sampler=0, sigmas=None):
+                 sampler=0, sigmas=None, layer_comp=None):
         self.layers = layers                      # list[BlockWeights] (keeps tensors alive)
         self._w = (fps_block_weights * len(layers))(*[l.c for l in layers])
         self._deltas = (C.c_float * n_steps)(*map(float, deltas))
         self._plan = (C.c_uint8 * len(layers))(*(plan or [0] * len(layers)))
         self._sigmas = (C.c_float * (n_steps + 1))(*map(float, sigmas)) if sigmas is not None else None
+        self._layer_comp = ((C.c_double * (2 * len(layers)))(*[float(v) for ab in layer_comp for v in ab])
+                            if layer_comp is not None else None)
         self.mod_table = mod_table
         self.cache = cache
         H, F = layers[0].H, layers[0].F
@@ -351,7 +354,8 @@ class Engine:
                             C.cast(self._plan, C.c_void_p), (C.c_double * 4)(*cost_model),
                             L_ctx, max((getattr(l, "D_ctx", 0) for l in layers), default=0),
                             mod_width, int(cross_step), int(sampler),
-                            C.cast(self._sigmas, C.c_void_p) if self._sigmas is not None else None)
+                            C.cast(self._sigmas, C.c_void_p) if self._sigmas is not None else None,
+                            C.cast(self._layer_comp, C.c_void_p) if self._layer_comp is not None else None)
         self.desc = d
         h = C.c_void_p()
         _lib.fps_engine_create(C.byref(d), C.byref(h))

@@ -32,7 +32,8 @@ class FlashPSError(RuntimeError):
 class fps_cache_desc(C.Structure):
     _fields_ = [("mode", i32), ("dtype", i32), ("H", i32), ("L_img", i32), ("n_layers", i32),
                 ("n_steps", i32), ("n_templates", i32), ("n_entries", i32),
-                ("copy_method", i32), ("copy_ctas", i32), ("location", i32)]
+                ("copy_method", i32), ("copy_ctas", i32), ("location", i32),
+                ("shm_path", C.c_char_p)]
 
 
 class fps_prefetch_item(C.Structure):
@@ -66,7 +67,7 @@ class fps_engine_desc(C.Structure):
                 ("n_steps", i32), ("layers", vp), ("d_mod_table", vp), ("h_deltas", vp),
                 ("cache", vp), ("slots", i32), ("plan_policy", i32), ("h_plan", vp),
                 ("cost_model", dbl * 4), ("L_ctx", i32), ("D_ctx", i32), ("mod_width", i32),
-                ("cross_step", i32), ("sampler", i32), ("h_sigmas", vp)]
+                ("cross_step", i32), ("sampler", i32), ("h_sigmas", vp), ("h_layer_comp", vp)]
 
 
 class fps_request(C.Structure):

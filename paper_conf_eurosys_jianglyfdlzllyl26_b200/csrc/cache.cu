@@ -15,7 +15,10 @@
 //  2  copy-engine DMA of whole entries (all L_img rows, one copy per request and block): +25%
 //     bytes at m = 0.2 but no SM time and no per-run overhead; the caller orders fresh-row writes
 //     after the ready event.  Fastest measured step on B200 for both tiers.
+#include <fcntl.h>
 #include <sys/mman.h>
+#include <sys/stat.h>
+#include <unistd.h>
 
 #include <algorithm>
 #include <cstring>
@@ -292,7 +295,8 @@ fps_status fps_cache_create(const fps_cache_desc* desc, fps_cache_t* out) {
   c->n_keys = (long long)d.n_templates * d.n_steps * per_step;
   c->n_entries = d.n_entries > 0 ? std::min<long long>(d.n_entries, c->n_keys) : c->n_keys;
   const size_t bytes = (size_t)c->n_entries * c->entry_bytes;
-  FPS_CHECK_ARG(d.location >= 0 && d.location <= 2, "location %d", d.location);
+  FPS_CHECK_ARG(d.location >= 0 && d.location <= 3, "location %d", d.location);
+  FPS_CHECK_ARG(d.location != 3 || (d.shm_path && d.shm_path[0]), "location 3 needs shm_path");
   if (d.location == 1) {
     // HBM tier: the arena lives in device memory; "host" then names that device buffer
     cudaError_t e = cudaMalloc((void**)&c->host, bytes);
@@ -307,7 +311,38 @@ fps_status fps_cache_create(const fps_cache_desc* desc, fps_cache_t* out) {
     return FPS_OK;
   }
   cudaError_t e;
-  if (d.location == 2) {
+  if (d.location == 3) {
+    // one pinned arena shared by the worker processes of a box (SURVEY §8(e) "shared
+    // resource"): every process maps the same file (e.g. a memfd as /proc/<pid>/fd/<n>, or a
+    // /dev/shm file) MAP_SHARED and page-locks its own mapping for its device
+    const int fd = open(d.shm_path, O_RDWR | O_CREAT, 0600);
+    if (fd < 0) {
+      delete c;
+      return fail(FPS_EINVAL, "cache: open(%s) failed", d.shm_path);
+    }
+    struct stat st {};
+    if (fstat(fd, &st) != 0 || ((size_t)st.st_size < bytes && ftruncate(fd, (off_t)bytes) != 0)) {
+      close(fd);
+      delete c;
+      return fail(FPS_ENOMEM, "cache: sizing %s to %zu bytes failed", d.shm_path, bytes);
+    }
+    void* p = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+    close(fd);
+    if (p == MAP_FAILED) {
+      delete c;
+      return fail(FPS_ENOMEM, "cache: mmap(%s, %zu) failed", d.shm_path, bytes);
+    }
+    e = cudaHostRegister(p, bytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      munmap(p, bytes);
+      delete c;
+      return fail(FPS_ECUDA, "cache: cudaHostRegister(shared arena): %s", cudaGetErrorString(e));
+    }
+    c->host = static_cast<char*>(p);
+    c->mmap_base = p;
+    c->mmap_bytes = bytes;
+  } else if (d.location == 2) {
     // pinned host DRAM backed by transparent huge pages (fewer IOMMU translations per byte on
     // the PCIe path): 2 MiB-aligned anonymous mapping, MADV_HUGEPAGE, then page-locked+mapped
     const size_t align = size_t(2) << 20;
@@ -355,7 +390,7 @@ fps_status fps_cache_destroy(fps_cache_t c) {
   if (c->host) {
     if (c->d.location == 1) {
       cudaFree(c->host);
-    } else if (c->d.location == 2) {
+    } else if (c->d.location == 2 || c->d.location == 3) {
       cudaHostUnregister(c->host);
       munmap(c->mmap_base, c->mmap_bytes);
     } else {

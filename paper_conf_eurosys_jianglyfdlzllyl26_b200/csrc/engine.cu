@@ -39,6 +39,7 @@ struct fps_engine {
   std::vector<fps_block_weights> layers;
   std::vector<float> deltas;
   std::vector<float> sigmas;          // flow-blend sampler (R29): sigma_0 .. sigma_S
+  std::vector<double> layer_comp;     // per-block compute model (a_l, b_l), or empty
   std::vector<uint8_t> fixed_plan;
   int L = 0, elt = 2, W = 0, D = 0;
   size_t row_h = 0, row_w = 0;  // bytes of an H row / a W row
@@ -200,6 +201,8 @@ fps_status fps_engine_create(const fps_engine_desc* desc, fps_engine_t* out) {
   e->deltas.assign(d.h_deltas, d.h_deltas + d.n_steps);
   if (d.sampler == FPS_SAMPLER_FLOW_BLEND) e->sigmas.assign(d.h_sigmas, d.h_sigmas + d.n_steps + 1);
   e->d.h_sigmas = nullptr;
+  if (d.h_layer_comp) e->layer_comp.assign(d.h_layer_comp, d.h_layer_comp + 2 * d.n_layers);
+  e->d.h_layer_comp = nullptr;
   if (d.plan_policy == 3) e->fixed_plan.assign(d.h_plan, d.h_plan + d.n_layers);
   e->d.layers = nullptr;
   e->d.h_deltas = nullptr;
@@ -488,9 +491,12 @@ static void make_plan(fps_engine* e, const Batch& B) {
       fd += flops_block(FPS_MODE_KV, L, L, H, F, kind, Lc);
       ft += flops_block(FPS_MODE_Y, B.nq[i], L, H, F, kind, Lc);
     }
-    Cw[l] = a * fm + b;
-    Cwo[l] = a * fd + b;
-    Ct[l] = a * ft + b;     // transition block (R28): Y-mode work over the fresh full input
+    // the block's own compute model (fitted per block kind) when given, else the stack's
+    const double al = e->layer_comp.empty() ? a : e->layer_comp[2 * l];
+    const double bl = e->layer_comp.empty() ? b : e->layer_comp[2 * l + 1];
+    Cw[l] = al * fm + bl;
+    Cwo[l] = al * fd + bl;
+    Ct[l] = al * ft + bl;   // transition block (R28): Y-mode work over the fresh full input
   }
   for (int i = 0; i < B.n; ++i) {
     // rows the load moves: U, or the whole entry for the whole-entry DMA method

@@ -62,10 +62,12 @@ class CostModel:
     """Per-block costs of a batch for Alg. 1 from the two fitted linear models."""
 
     def __init__(self, n_layers, H, F, mode, comp=(1e-12, 0.01), load=(2e-8, 0.01), elt=2,
-                 full_entry_rows=None, kind="seq", Lc=0):
+                 full_entry_rows=None, kind="seq", Lc=0, layer_comp=None):
         self.n_layers, self.H, self.F, self.mode, self.elt = n_layers, H, F, mode, elt
         self.kind, self.Lc = kind, Lc
         self.comp, self.load = comp, load
+        # per-block compute models (a_l, b_l), e.g. fitted per block kind; None = comp for all
+        self.layer_comp = layer_comp
         # whole-entry DMA loads (copy_method 2) move L_img rows whatever the mask
         self.full_entry_rows = full_entry_rows
 
@@ -80,8 +82,9 @@ class CostModel:
         by = sum(cache_bytes(self.mode, self._rows(r), self.H, self.elt) for r in batch)
         byf = sum(cache_bytes("y", self._rows(r), self.H, self.elt) for r in batch)
         N = self.n_layers
-        Cw = [a * fm + b] * N
-        Cwo = [a * fd + b] * N
+        ab = self.layer_comp or [(a, b)] * N
+        Cw = [al * fm + bl for al, bl in ab]
+        Cwo = [al * fd + bl for al, bl in ab]
         Lm = [c * by + e if by > 0 else 0.0] * N
         fin = (c * byf + e) if (self.mode == "kv" and byf > 0) else 0.0
         return Cw, Cwo, Lm, fin

@@ -76,3 +76,59 @@ def test_mask_aware_routing_balances_predicted_latency():
     rr = [[reqs[i] for i in range(w, 16, 4)] for w in range(4)]
     worst = lambda ws: max(cm.step_latency(w) for w in ws)
     assert worst(ma) <= worst(rr) + 1e-9
+
+
+def _bench_worker(rank, world, port, out_dir):
+    """One rank of bench.py's multi-GPU routing path (bench.make_requests + bench.route_job) on
+    a C4 job: a pool of 16 x world heterogeneous masks (5-60 %), max batch 16 per GPU."""
+    import sys
+    sys.path.insert(0, ROOT)
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK=str(rank),
+                      WORLD_SIZE=str(world))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import bench
+    from paper_conf_eurosys_jianglyfdlzllyl26_b200 import sched
+    w = dict(bench.WORKLOADS["C4"], block="flux")
+    pool = bench.make_requests(w, w["batch"] * world, bench.SEED)
+    # per-block-kind compute models as the bench fits them (double-stream / single-stream)
+    cm = sched.CostModel(57, 3072, 12288, "kv", comp=(7.3e-13, 0.10), load=(1 / 5.5e7, 0.003),
+                         full_entry_rows=4096, kind="double",
+                         layer_comp=[(7.4e-13, 0.10)] * 19 + [(7.2e-13, 0.09)] * 38)
+    mine, assign, held = bench.route_job(pool, w, world, rank, cm)
+    gathered = [None] * world
+    dist.all_gather_object(gathered, assign)
+    lat = cm.step_latency([sched.Request(i, pool[i]["n_active"], 4608) for i in mine])
+    lats = [None] * world
+    dist.all_gather_object(lats, lat)
+    np.save(os.path.join(out_dir, f"b{rank}.npy"),
+            np.array([mine, gathered, held, lats, [p["ratio"] for p in pool]], dtype=object),
+            allow_pickle=True)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_bench_routing_path_world2(tmp_path):
+    """bench.py's own N > 1 routing (the function its main() calls) on 2 gloo ranks: identical
+    assignment on every rank, a disjoint cover of the heterogeneous pool, 16 requests per GPU,
+    and predicted step latencies within 5 % of each other (Alg. 2 balances mask sizes, L261)."""
+    world = 2
+    mp.spawn(_bench_worker, args=(world, _free_port(), str(tmp_path)), nprocs=world, join=True)
+    res = [np.load(tmp_path / f"b{r}.npy", allow_pickle=True) for r in range(world)]
+    for r in res:
+        assert all(a == r[1][0] for a in r[1])
+    mines = [list(r[0]) for r in res]
+    assert sorted(i for m in mines for i in m) == list(range(32)) and not list(res[0][2])
+    assert all(len(m) == 16 for m in mines)
+    assert len(set(res[0][4])) == 16                  # the pool really is heterogeneous
+    lats = res[0][3]
+    assert max(lats) <= 1.05 * min(lats), lats
+
+
+def test_bench_refuses_mismatched_world(tmp_path):
+    """`bench.py --gpus 2` inside a 1-rank launch must not report a 1-rank run as 2 GPUs."""
+    import subprocess
+    import sys
+    env = dict(os.environ, WORLD_SIZE="1", RANK="0", LOCAL_RANK="0")
+    p = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2"],
+                       env=env, capture_output=True, text=True, timeout=120)
+    assert p.returncode == 2, p.stderr[-2000:]
