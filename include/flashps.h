@@ -164,10 +164,20 @@ typedef struct {
                             3 = pinned host DRAM SHARED by the worker processes of a box
                                 (SURVEY §8(e)): the file at shm_path (created / grown to the
                                 arena size if needed) is mapped MAP_SHARED and page-locked by
-                                each process -- one copy of the templates for all GPUs       */
+                                each process -- one copy of the templates for all GPUs;
+                            4 = a PEER GPU's HBM tier (NEXT-1, the NVLink / NVSwitch level
+                                of the hierarchical store, L222-L224): the arena another
+                                process exported with fps_cache_export_ipc, opened with CUDA
+                                IPC (peer access enabled lazily); loads read it over NVLink
+                                exactly like the local HBM tier (methods 0 / 2 / 3 on the
+                                device, method 1 takes the gather).  The desc must match the
+                                exporter's (same sizes and n_entries); stores write through to
+                                the peer                                                     */
   const char* shm_path;  /* location 3: path of the shared arena file (e.g. a memfd opened
                             as /proc/<pid>/fd/<n>, or /dev/shm/<name>); the caller removes
                             it; NULL otherwise                                               */
+  const void* peer_ipc_handle;   /* location 4: the 64-byte cudaIpcMemHandle_t written by the
+                            owner's fps_cache_export_ipc; NULL otherwise                     */
 } fps_cache_desc;
 
 typedef struct fps_cache* fps_cache_t;
@@ -179,6 +189,10 @@ void* fps_cache_entry_host_ptr(fps_cache_t c, uint32_t template_id, int32_t step
 /* Address of an entry in whichever memory holds the arena (host or device); NULL if out of range. */
 void* fps_cache_entry_ptr(fps_cache_t c, uint32_t template_id, int32_t step, int32_t layer);
 size_t fps_cache_entry_bytes(fps_cache_t c, int32_t layer);
+/* NEXT-1 peer tier: export an HBM-tier cache's arena (location 1) as a 64-byte CUDA IPC
+ * handle for other processes (another GPU's worker opens it as location 4).  The exporting
+ * cache must outlive every importer. */
+fps_status fps_cache_export_ipc(fps_cache_t c, void* handle_out);
 /* D2H: store rows [0, L_img) of d_src (row pitch src_row_bytes >= W*elt) as entry
  * (template_id, step, layer).  Asynchronous on `stream`. */
 fps_status fps_cache_store(fps_cache_t c, uint32_t template_id, int32_t step, int32_t layer,

@@ -291,10 +291,12 @@ class Cache:
     """fps_cache_t: pinned host arena of template activations (L203)."""
 
     def __init__(self, mode, dtype, H, L_img, n_layers, n_steps, n_templates=1, n_entries=0,
-                 copy_method=0, copy_ctas=0, location=0, shm_path=None):
+                 copy_method=0, copy_ctas=0, location=0, shm_path=None, peer_handle=None):
         self._shm = shm_path.encode() if shm_path else None
+        self._peer = (C.c_uint8 * 64).from_buffer_copy(peer_handle) if peer_handle else None
         self.desc = fps_cache_desc(mode, dtype, H, L_img, n_layers, n_steps, n_templates,
-                                   n_entries, copy_method, copy_ctas, location, self._shm)
+                                   n_entries, copy_method, copy_ctas, location, self._shm,
+                                   C.cast(self._peer, C.c_void_p) if self._peer is not None else None)
         h = C.c_void_p()
         _lib.fps_cache_create(C.byref(self.desc), C.byref(h))
         self.h = h
@@ -310,6 +312,12 @@ class Cache:
             self.close()
         except Exception:
             pass
+
+    def export_ipc(self):
+        """64-byte CUDA IPC handle of an HBM-tier arena (NEXT-1 peer tier)."""
+        h = (C.c_uint8 * 64)()
+        _lib.fps_cache_export_ipc(self.h, h)
+        return bytes(h)
 
     def entry_numpy(self, template_id, step, layer):
         """Host view of an entry as raw uint16 (bf16) / float32 numpy array [L_img, width]."""

@@ -33,7 +33,7 @@ class fps_cache_desc(C.Structure):
     _fields_ = [("mode", i32), ("dtype", i32), ("H", i32), ("L_img", i32), ("n_layers", i32),
                 ("n_steps", i32), ("n_templates", i32), ("n_entries", i32),
                 ("copy_method", i32), ("copy_ctas", i32), ("location", i32),
-                ("shm_path", C.c_char_p)]
+                ("shm_path", C.c_char_p), ("peer_ipc_handle", vp)]
 
 
 class fps_prefetch_item(C.Structure):
@@ -95,6 +95,7 @@ _SIGS = [
     ("fps_cache_entry_host_ptr", vp, [vp, u32, i32, i32], False),
     ("fps_cache_entry_ptr", vp, [vp, u32, i32, i32], False),
     ("fps_cache_entry_bytes", sz, [vp, i32], False),
+    ("fps_cache_export_ipc", C.c_int, [vp, vp], True),
     ("fps_cache_store", C.c_int, [vp, u32, i32, i32, vp, i32, vp], True),
     ("fps_cache_prefetch", C.c_int, [vp, C.POINTER(fps_prefetch_item), i32, vp, vp], True),
     ("fps_geglu_pack", C.c_int, [i32, vp, vp, i32, i32, vp, vp, vp], True),

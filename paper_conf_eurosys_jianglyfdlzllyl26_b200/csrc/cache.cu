@@ -263,6 +263,10 @@ int bulk_ctas(const fps_cache* c) {
   return std::min(n, 32);
 }
 
+// the arena lives in device memory: this GPU's HBM (location 1) or a peer GPU's, opened
+// through a CUDA IPC handle and read over NVLink / NVSwitch (location 4)
+static bool in_device_memory(const fps_cache* c) { return c->d.location == 1 || c->d.location == 4; }
+
 int g_d2d_kernel = 1;   // experiments: 0 = driver D2D memcpy for HBM whole-entry loads
 bool cache_writes_all_rows(const fps_cache* c) { return c && c->d.copy_method == 2; }
 
@@ -295,7 +299,8 @@ fps_status fps_cache_create(const fps_cache_desc* desc, fps_cache_t* out) {
   c->n_keys = (long long)d.n_templates * d.n_steps * per_step;
   c->n_entries = d.n_entries > 0 ? std::min<long long>(d.n_entries, c->n_keys) : c->n_keys;
   const size_t bytes = (size_t)c->n_entries * c->entry_bytes;
-  FPS_CHECK_ARG(d.location >= 0 && d.location <= 3, "location %d", d.location);
+  FPS_CHECK_ARG(d.location >= 0 && d.location <= 4, "location %d", d.location);
+  FPS_CHECK_ARG(d.location != 4 || d.peer_ipc_handle, "location 4 needs peer_ipc_handle");
   FPS_CHECK_ARG(d.location != 3 || (d.shm_path && d.shm_path[0]), "location 3 needs shm_path");
   if (d.location == 1) {
     // HBM tier: the arena lives in device memory; "host" then names that device buffer
@@ -305,6 +310,22 @@ fps_status fps_cache_create(const fps_cache_desc* desc, fps_cache_t* out) {
       delete c;
       return fail(e == cudaErrorMemoryAllocation ? FPS_ENOMEM : FPS_ECUDA,
                   "cache: cudaMalloc(%zu bytes): %s", bytes, cudaGetErrorString(e));
+    }
+    c->dev_alias = c->host;
+    *out = c;
+    return FPS_OK;
+  }
+  if (d.location == 4) {
+    // NEXT-1, the peer tier: the template arena of another GPU (its HBM tier, exported with
+    // fps_cache_export_ipc), mapped into this process; loads read it over NVLink / NVSwitch.
+    // Same layout and size rules as the exporter's cache (the caller passes the same desc).
+    cudaIpcMemHandle_t h;
+    memcpy(&h, d.peer_ipc_handle, sizeof(h));
+    cudaError_t e = cudaIpcOpenMemHandle((void**)&c->host, h, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      delete c;
+      return fail(FPS_ECUDA, "cache: cudaIpcOpenMemHandle: %s", cudaGetErrorString(e));
     }
     c->dev_alias = c->host;
     *out = c;
@@ -390,6 +411,8 @@ fps_status fps_cache_destroy(fps_cache_t c) {
   if (c->host) {
     if (c->d.location == 1) {
       cudaFree(c->host);
+    } else if (c->d.location == 4) {
+      cudaIpcCloseMemHandle(c->host);
     } else if (c->d.location == 2 || c->d.location == 3) {
       cudaHostUnregister(c->host);
       munmap(c->mmap_base, c->mmap_bytes);
@@ -407,8 +430,19 @@ void* fps_cache_entry_ptr(fps_cache_t c, uint32_t template_id, int32_t step, int
 }
 
 void* fps_cache_entry_host_ptr(fps_cache_t c, uint32_t template_id, int32_t step, int32_t layer) {
-  if (!c || c->d.location == 1) return nullptr;
+  if (!c || in_device_memory(c)) return nullptr;
   return fps_cache_entry_ptr(c, template_id, step, layer);
+}
+
+static_assert(sizeof(cudaIpcMemHandle_t) == 64, "the ABI passes IPC handles as 64 bytes");
+
+fps_status fps_cache_export_ipc(fps_cache_t c, void* handle_out) {
+  FPS_CHECK_ARG(c && handle_out, "NULL argument");
+  FPS_CHECK_ARG(c->d.location == 1, "only an HBM-tier cache (location 1) can be exported");
+  cudaIpcMemHandle_t h;
+  FPS_CUDA_TRY(cudaIpcGetMemHandle(&h, c->host));
+  memcpy(handle_out, &h, sizeof(h));
+  return FPS_OK;
 }
 
 size_t fps_cache_entry_bytes(fps_cache_t c, int32_t layer) {
@@ -444,9 +478,9 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
                   row_bytes_of(c, it.layer));
     // the row gather (method 0, and method 1 on the HBM arena) reads d_rows on the device;
     // the per-run DMA reads h_rows on the host
-    if (c->d.copy_method == 0 || c->d.copy_method == 3 || (c->d.copy_method == 1 && c->d.location == 1))
+    if (c->d.copy_method == 0 || c->d.copy_method == 3 || (c->d.copy_method == 1 && in_device_memory(c)))
       FPS_CHECK_ARG(it.n_rows == 0 || it.d_rows, "item %d: d_rows needed for the row gather", i);
-    if (c->d.copy_method == 1 && c->d.location != 1)
+    if (c->d.copy_method == 1 && !in_device_memory(c))
       FPS_CHECK_ARG(it.n_rows == 0 || it.h_rows, "item %d: h_rows needed for DMA", i);
   }
   if (c->d.copy_method == 2) {
@@ -458,7 +492,7 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
       if (it.n_rows == 0) continue;
       const size_t nb = (size_t)c->d.L_img * row_bytes_of(c, it.layer);
       const char* src = c->host + offset_of(c, it.template_id, it.step, it.layer);
-      if (c->d.location == 1 && g_d2d_kernel) {
+      if (in_device_memory(c) && g_d2d_kernel) {
         // HBM arena: device-to-device entry copy by our own kernel (launched without PDL).
         // A driver cudaMemcpyAsync D2D here, with PDL launches on the compute stream, hung
         // the C2B stack deterministically (tools/hang_probe.py: plan 21 dense + 39 cached).
@@ -507,7 +541,7 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
       count_launch();
       FPS_LAUNCH_CHECK();
     }
-  } else if (c->d.copy_method == 0 || c->d.location == 1) {
+  } else if (c->d.copy_method == 0 || in_device_memory(c)) {
     // (method 1 on the HBM arena takes the row gather too: a driver D2D copy per run would
     //  interleave with PDL launches, the pattern that hung in tools/hang_probe.py)
     for (int base = 0; base < n_items; base += kMaxPrefetchItems) {
@@ -541,7 +575,7 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
           if (sscanf(e, "%d,%d", &g_pf_threads, &g_pf_unroll) != 2) g_pf_threads = 64, g_pf_unroll = 16;
       }
       const int thr = g_pf_threads, unr = g_pf_unroll;
-      int ctas = c->d.copy_ctas > 0 ? c->d.copy_ctas : (c->d.location == 1 ? 64 : 16);
+      int ctas = c->d.copy_ctas > 0 ? c->d.copy_ctas : (in_device_memory(c) ? 64 : 16);
       ctas = (int)((long long)ctas * 2048 / (thr * unr));  // same loads in flight as 256 x 8
       long long want = (acc + (long long)thr * unr - 1) / ((long long)thr * unr);
       if (want < ctas) ctas = (int)want;

@@ -48,10 +48,13 @@ def fit_linear(x, y):
 class Request:
     """What the scheduler knows about a request: its active rows n and unmasked rows u."""
 
-    def __init__(self, rid, n_active, L, arrival=0.0, steps=28, tokens=None):
+    def __init__(self, rid, n_active, L, arrival=0.0, steps=28, tokens=None, model="flux",
+                 ratio=None):
         self.rid, self.n, self.L, self.arrival, self.steps = rid, int(n_active), int(L), arrival, steps
         # token-granularity load (§6.5): masked image tokens (defaults to the active rows)
         self.tokens = int(n_active if tokens is None else tokens)
+        # which model's stack serves it, and its image-token mask ratio (multi-level models)
+        self.model, self.ratio = model, ratio
 
     @property
     def u(self):
@@ -100,6 +103,40 @@ class CostModel:
     def as_engine_model(self):
         """(a, b, c, e) in the units fps_engine_desc.cost_model expects (ms/FLOP, ms, ms/B, ms)."""
         return (self.comp[0], self.comp[1], self.load[0], self.load[1])
+
+
+class SdxlCost:
+    """SDXL's transformer blocks sit at two UNet levels (reading R19): a
+    request's step runs the 64 x 64 level's stack (640 channels) and the 32 x 32 level's (1280
+    channels), each with the request's mask pooled to that level (fps_mask_to_tokens, R8).  The
+    step latency is the sum of the two levels' Alg. 1 pipeline latencies under their own fitted
+    models; a request's mask ratio sets its active rows at each level."""
+
+    def __init__(self, level_models, level_tokens):
+        self.levels = list(zip(level_models, level_tokens))
+
+    def step_latency(self, batch):
+        if not batch:
+            return 0.0
+        t = 0.0
+        for cm, Lv in self.levels:
+            t += cm.step_latency([Request(r.rid, max(1, round(r.ratio * Lv)), Lv) for r in batch])
+        return t
+
+
+class MixedCost:
+    """A worker holding both models' stacks (Flux 12.9 GB + SDXL 2.4 GB of weights
+    in 180 GB of HBM) runs each model's sub-batch of its running batch in turn every step; the
+    step latency is their sum (configs[4]: mixed SDXL / Flux traffic)."""
+
+    def __init__(self, models):
+        self.models = models          # model name -> object with step_latency(batch)
+
+    def step_latency(self, batch):
+        by = {}
+        for r in batch:
+            by.setdefault(r.model, []).append(r)
+        return sum(self.models[m].step_latency(b) for m, b in by.items())
 
 
 def route(req, workers, cost_fn, max_batch):

@@ -63,3 +63,28 @@ def test_product_flops_match_oracle_counters(kind, Lc):
         for n, L, H, F in ((410, 4096, 640, 2560), (307, 1024, 1280, 5120), (1331, 4608, 3072, 12288)):
             assert PS.block_flops(mode, n, L, H, F, kind, Lc) == pytest.approx(
                 OC.block_flops(mode, n, L, H, F, kind, Lc), rel=1e-12)
+
+
+def test_mixed_and_sdxl_costs_are_sums_of_their_parts():
+    """configs[4] mixed traffic: a worker's step over a mixed batch = the Flux sub-batch's
+    latency + the SDXL sub-batch's, and an SDXL step = its two UNet levels' pipeline latencies
+    with the request's mask ratio pooled to each level (R19, R8)."""
+    from paper_conf_eurosys_jianglyfdlzllyl26_b200 import sched
+    flux = sched.CostModel(57, 3072, 12288, "kv", comp=(7e-13, 0.1), load=(1 / 5.5e7, 0.003))
+    A = sched.CostModel(10, 640, 2560, "kv", comp=(1.6e-12, 0.08), load=(1 / 5.4e7, 0.002),
+                        kind="sdxl", Lc=77)
+    Bm = sched.CostModel(60, 1280, 5120, "kv", comp=(1.0e-12, 0.1), load=(1 / 5.3e7, 0.004),
+                         kind="sdxl", Lc=77)
+    sd = sched.SdxlCost([A, Bm], [4096, 1024])
+    mix = sched.MixedCost({"flux": flux, "sdxl": sd})
+    f = [sched.Request(0, 1331, 4608, model="flux"), sched.Request(1, 900, 4608, model="flux")]
+    s = [sched.Request(2, 0, 4096, model="sdxl", ratio=0.25)]
+    assert mix.step_latency(f + s) == pytest.approx(flux.step_latency(f) + sd.step_latency(s))
+    assert sd.step_latency(s) == pytest.approx(
+        A.step_latency([sched.Request(2, 1024, 4096)]) + Bm.step_latency([sched.Request(2, 256, 1024)]))
+    assert mix.step_latency([]) == 0.0
+    # Alg. 2 over a mixed pool sends an SDXL request to the worker whose batch it costs least
+    workers = [list(f), list(s)]
+    w = sched.route(sched.Request(3, 0, 4096, model="sdxl", ratio=0.1), workers, mix.step_latency, 8)
+    costs = [mix.step_latency(wk + [sched.Request(3, 0, 4096, model="sdxl", ratio=0.1)]) for wk in workers]
+    assert w == int(np.argmin(costs))
