@@ -273,18 +273,21 @@ def calibrate(F, w, mode, layers, cache, reqs, device):
 def host_link_gbs(w, mode, device, reps=8):
     """The host link's copy-engine rate: pinned host -> HBM cudaMemcpyAsync of one cache entry
     (L_img rows of the mode's width), back to back (the step roofline's link peak)."""
-    nb = w["L_img"] * (2 if mode == "kv" else 1) * w["H"] * 2
+    nb = max(w["L_img"] * (2 if mode == "kv" else 1) * w["H"] * 2, 64 << 20)
     h = torch.empty(nb, dtype=torch.uint8).pin_memory()
     d = torch.empty(nb, dtype=torch.uint8, device=device)
     d.copy_(h, non_blocking=True)
     torch.cuda.synchronize()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record()
-    for _ in range(reps):
-        d.copy_(h, non_blocking=True)
-    e1.record()
-    torch.cuda.synchronize()
-    return reps * nb / (e0.elapsed_time(e1) * 1e-3) / 1e9
+    best = 0.0
+    for _ in range(3):                     # best of 3 (the link is shared with nothing here)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(reps):
+            d.copy_(h, non_blocking=True)
+        e1.record()
+        torch.cuda.synchronize()
+        best = max(best, reps * nb / (e0.elapsed_time(e1) * 1e-3) / 1e9)
+    return best
 
 
 def _calibrate_one(F, w, mode, layers, cache, reqs, device, first=0):
@@ -327,6 +330,11 @@ def _calibrate_one(F, w, mode, layers, cache, reqs, device, first=0):
         # (a 1.5 s clock-settling burst before the fits made the predicted step match the
         # measured one within 1% but moved the plan to 45-46 cached blocks, measured slower than
         # the 41-44 this fit picks: tools/sweep_plan.py, C3 k = 41..44 within noise at ~32.5 ms)
+        settle = float(os.environ.get("FPS_CALIB_SETTLE", 0.5))
+        t_end = time.perf_counter() + settle
+        while time.perf_counter() < t_end:
+            fn()
+            torch.cuda.synchronize()
         fn()
         torch.cuda.synchronize()
         if LOADED_CALIBRATION:
