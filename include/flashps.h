@@ -306,6 +306,11 @@ typedef struct {
   const int32_t* d_sm_inv;         /* [total_q] stream row of compact row r (the inverse of
                                       d_sm_perm), or NULL: the block then reorders its rows
                                       with two extra row copies                              */
+  /* a2 fused into the block (NEXT-4): 1 = d_x_act is the FULL merged buffer [total_k, H] and
+   * active row i is its row d_q_row[i] (d_sm_kvrow for DOUBLE blocks) -- the first norm and
+   * the residual read the rows there, so no gathered copy of the active rows is needed;
+   * 0 = d_x_act is compact [total_q, H] (request-major).  Requires d_q_row.                */
+  int32_t x_full_rows;
 } fps_varlen_batch;
 
 /* SDXL block helpers (R24), run once per weight load / per request prompt, not per step.

@@ -58,7 +58,7 @@ class fps_varlen_batch(C.Structure):
                 ("d_cu_u", vp), ("d_u_src", vp), ("d_u_row", vp), ("d_ctx_kv", vp),
                 ("d_cu_ctx", vp), ("h_cu_ctx", vp), ("mod_stride", i32), ("total_q_img", i32),
                 ("d_sm_perm", vp), ("d_sm_kvrow", vp), ("d_cu_img", vp), ("d_cu_txt", vp),
-                ("d_sm_inv", vp)]
+                ("d_sm_inv", vp), ("x_full_rows", i32)]
 
 
 class fps_engine_desc(C.Structure):

@@ -269,6 +269,9 @@ static fps_status double_block_forward(const fps_block_weights* w, const fps_var
   };
   const int32_t* perm = b->d_sm_perm;
   const int32_t* kvrow = b->d_sm_kvrow;
+  // a2 fused into the consumers: x_act may be the full merged buffer, read at the active rows'
+  // merged rows (stream-major order -> d_sm_kvrow) instead of a compact gathered copy
+  const int32_t* xperm = b->x_full_rows ? kvrow : perm;
   const int32_t* cu[2] = {b->d_cu_img, b->d_cu_txt};
   const int rows0[2] = {0, ti}, nrows[2] = {ti, tt};
   const void* Wqkv[2] = {w->w_qkv, w->t_qkv};
@@ -290,11 +293,11 @@ static fps_status double_block_forward(const fps_block_weights* w, const fps_var
   // attention kernels forced by tests.
   const bool direct = b->d_sm_inv != nullptr && (g_attn_force == 0 || g_attn_force == 3);
   if (tq > 0) {
-    if (!direct) FPS_TRY(launch_copy_rows(x_act, perm, nullptr, tq, (int)rowb, x_sm, s));
+    if (!direct) FPS_TRY(launch_copy_rows(x_act, xperm, nullptr, tq, (int)rowb, x_sm, s));
     // a4 per stream; a5 for both streams in one grouped launch: Q -> request-major rows,
     // K|V -> merged key rows
     // both streams' norms in one launch (rows >= ti: the text stream's vectors)
-    FPS_TRY(launch_ln_mod2(dt, direct ? x_act : x_sm, direct ? perm : nullptr, tq, H, ws.h, cu[0],
+    FPS_TRY(launch_ln_mod2(dt, direct ? x_act : x_sm, direct ? xperm : nullptr, tq, H, ws.h, cu[0],
                            cu[1], ti, b->n_req, mod, 0, 6 * H, s, MS));
     Epilogue ep[2] = {};
     for (int st = 0; st < 2; ++st) {
@@ -336,7 +339,7 @@ static fps_status double_block_forward(const fps_block_weights* w, const fps_var
   for (int st = 0; st < 2; ++st) {   // x1 = x + gate1 (A Wo^T + bo)
     eo[st].bias = Bo[st];
     if (direct) {
-      eo[st].resid = x_act; eo[st].resid_map = perm + rows0[st];
+      eo[st].resid = x_act; eo[st].resid_map = xperm + rows0[st];
     } else {
       eo[st].resid = at(x_sm, st);
     }
@@ -375,6 +378,9 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
   const int MS = b->mod_stride > 0 ? b->mod_stride : 6 * H;
   const char* mod = sdxl ? nullptr : (const char*)b->d_mod;
   auto modp = [&](int off) -> const void* { return mod ? mod + (size_t)off * H * e : nullptr; };
+  // a2 fused into the consumers: with x_full_rows the block reads its active input rows
+  // straight out of the full merged buffer at d_q_row (first norm + residual), no gathered copy
+  const int32_t* xr = b->x_full_rows ? b->d_q_row : nullptr;
   // a4, the first norm: adaLN-modulated LN, or the SDXL block's affine LN (reading R24)
   auto ln1 = [&](const void* x, const int32_t* rows, int n, void* out, const int32_t* cu,
                  const int32_t* out_rows) -> fps_status {
@@ -388,12 +394,12 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
   // the M/U split (C3: 6 + 1 waves instead of 3 + 5)
   const bool y_split = tu > 0 && tq > 0 && w->kind != FPS_BLOCK_PAR;
   if (y_split) {
-    FPS_TRY(ln1(x_act, nullptr, tq, ws.h, b->d_cu_q, nullptr));
+    FPS_TRY(ln1(x_act, xr, tq, ws.h, b->d_cu_q, nullptr));
     Epilogue eq{};
     eq.bias = w->b_qkv;
     eq.out0 = ws.q; eq.ld0 = H; eq.split = H;
     FPS_TRY(launch_gemm(dt, ws.h, w->w_qkv, tq, H, H, eq, s));
-    FPS_TRY(ln1(x_act, nullptr, tq, ws.hu, b->d_cu_q, b->d_q_row));
+    FPS_TRY(ln1(x_act, xr, tq, ws.hu, b->d_cu_q, b->d_q_row));
     if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
     kv_ready = nullptr;
     FPS_TRY(ln1(xu, b->d_u_src, tu, ws.hu, b->d_cu_u, b->d_u_row));
@@ -405,7 +411,7 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
   }
   if (tq > 0 && !y_split) {
     // a4: h1 = LN(x)(1+scale1)+shift1 on active rows
-    FPS_TRY(ln1(x_act, nullptr, tq, ws.h, b->d_cu_q, nullptr));
+    FPS_TRY(ln1(x_act, xr, tq, ws.h, b->d_cu_q, nullptr));
     // a5: [tq,H] x [3H,H]^T; Q -> compact, K|V -> merged key rows at original positions
     Epilogue ep{};
     ep.bias = w->b_qkv;
@@ -442,7 +448,7 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
                              &sc));
     Epilogue ep{};
     ep.bias = w->b_down;
-    ep.resid = x_act; ep.ld_resid = H;
+    ep.resid = x_act; ep.ld_resid = H; ep.resid_map = xr;
     ep.gate = modp(2); ep.gate_stride = MS; ep.cu = b->d_cu_q; ep.n_req = b->n_req;
     ep.out0 = y_act; ep.ld0 = H; ep.split = H;
     return launch_gemm(dt, cat, w->w_down, tq, H, H + F, ep, s);
@@ -455,7 +461,7 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
   {  // a7: x1 = x + gate1 (A Wo^T + bo)
     Epilogue ep{};
     ep.bias = w->b_o;
-    ep.resid = x_act; ep.ld_resid = H;
+    ep.resid = x_act; ep.ld_resid = H; ep.resid_map = xr;
     ep.gate = modp(2); ep.gate_stride = MS; ep.cu = b->d_cu_q; ep.n_req = b->n_req;
     ep.out0 = ws.x1; ep.ld0 = H; ep.split = H;
     ep.out0_f32 = sdxl;          // SDXL: keep the residual stream x1, x2 in fp32 (R24)
@@ -665,6 +671,9 @@ fps_status fps_masked_block_forward(const fps_block_weights* w, const fps_varlen
   if (b->mode == FPS_MODE_Y && b->total_u > 0) FPS_CHECK_ARG(d_xu && d_kv, "Y-mode needs d_xu");
   if (b->total_q > 0 && b->d_q_row == nullptr)
     FPS_CHECK_ARG(b->total_q == b->total_k, "d_q_row NULL requires total_q == total_k");
+  if (b->x_full_rows && b->total_q > 0)
+    FPS_CHECK_ARG(b->d_q_row && (w->kind != FPS_BLOCK_DOUBLE || b->d_sm_kvrow),
+                  "x_full_rows needs d_q_row (and d_sm_kvrow for double-stream blocks)");
   FPS_CHECK_ARG(w->heads * w->head_dim == w->H, "heads*head_dim != H");
   FPS_TRY(check_ctx(w, b));
   FPS_TRY(check_streams(w, b));

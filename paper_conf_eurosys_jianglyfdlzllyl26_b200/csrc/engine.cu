@@ -695,10 +695,11 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
       // fresh full input -- K|V of all rows from cur_full (the Y-mode path with d_xu = the
       // full input), Q / attention / O / MLP on the active rows only.  Same values for every
       // row that is read afterwards; nothing loaded for it.
-      FPS_TRY(launch_copy_rows(cur_full, B.q_row, nullptr, B.tq, (int)e->row_h, e->act[act_cur], cs));
+      // (its active rows are read straight from the full input: a2 fused into the block)
       fps_varlen_batch vt = vb;
       vt.mode = FPS_MODE_Y;
-      FPS_TRY(fps_masked_block_forward(w, &vt, e->act[act_cur], e->act[act_cur ^ 1], e->kv_scratch,
+      vt.x_full_rows = 1;
+      FPS_TRY(fps_masked_block_forward(w, &vt, cur_full, e->act[act_cur ^ 1], e->kv_scratch,
                                        cur_full, nullptr, e->ws, e->ws_bytes, cs));
       act_cur ^= 1;
       rep_full = false;
@@ -733,15 +734,19 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
       const char* xu = nullptr;
       cudaEvent_t ev = nullptr;
       int consumed_after = -1;
+      fps_varlen_batch vx = vb;
+      x_in = e->act[act_cur];
       if (rep_full) {
-        FPS_TRY(launch_copy_rows(cur_full, B.q_row, nullptr, B.tq, (int)e->row_h, e->act[act_cur], cs));
+        // a2 fused into the block: the first cached block reads its active rows straight out
+        // of the full activations (first norm and residual at d_q_row), no gathered copy
+        x_in = cur_full;
+        vx.x_full_rows = 1;
         xu = cur_full;
       } else if (!kv) {
         xu = e->slots[pos[l - 1] % e->D];
         ev = e->ready[pos[l - 1]];
         consumed_after = pos[l - 1];
       }
-      x_in = e->act[act_cur];
       char* kvbuf;
       if (kv) {
         kvbuf = e->slots[pos[l] % e->D];
@@ -756,7 +761,7 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
       } else {
         kvbuf = e->kv_scratch;
       }
-      FPS_TRY(fps_masked_block_forward(w, &vb, x_in, e->act[act_cur ^ 1], kvbuf, kv ? nullptr : xu,
+      FPS_TRY(fps_masked_block_forward(w, &vx, x_in, e->act[act_cur ^ 1], kvbuf, kv ? nullptr : xu,
                                        ev, e->ws, e->ws_bytes, cs));
       if (consumed_after >= 0) FPS_TRY(consume(consumed_after));
       act_cur ^= 1;

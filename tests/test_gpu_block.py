@@ -272,3 +272,24 @@ def test_split_kv_attention(F, mode, split):
     finally:
         F.fps_set_disable_tc(0)
     check_close(y, _ref_masked(w, reqs, 2, mode), TOL["bf16"], f"split {split} {mode}")
+
+
+@pytest.mark.parametrize("kind,mode", [("seq", "kv"), ("seq", "y"), ("par", "kv"), ("par", "y")])
+def test_active_rows_read_from_full_buffer_bit_identical(F, kind, mode):
+    """a2 fused into the block (x_full_rows): reading the active input rows straight out of the
+    full merged buffer at d_q_row gives the same bits as the compact gathered rows."""
+    w, reqs = _problem(4100 + (kind == "par"), "bf16", 256, 2, 1024, 576, 40, [0.05, 0.6, 0.3],
+                       blobs=True, kind=kind)
+    y_ref, _ = _run_masked(F, w, reqs, 2, "bf16", mode)
+    orig = F.masked_block_forward
+    full = to_dev(np.concatenate([r["x"] for r in reqs]), "bf16")      # [sum L, H]
+
+    def fused(bw, b, x_act, kv, xu=None, **kw):
+        b.c.x_full_rows = 1
+        return orig(bw, b, full, kv, xu=xu, y_act=torch.empty_like(x_act), **kw)
+    F.masked_block_forward = fused
+    try:
+        y, _ = _run_masked(F, w, reqs, 2, "bf16", mode)
+    finally:
+        F.masked_block_forward = orig
+    assert np.array_equal(y, y_ref)
