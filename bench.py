@@ -513,6 +513,9 @@ def main():
     ap.add_argument("--kv-transition", type=int, default=1, choices=[0, 1],
                     help="KV-mode: run the last dense block before the cached suffix as a masked "
                          "block over the fresh full input (R28; 0 = dense, for A/B)")
+    ap.add_argument("--plan-refine", type=int, default=1, choices=[0, 1],
+                    help="refine Alg. 1's plan by measuring it and its +-2-block neighbours "
+                         "(1, default) or time the planner's plan as is (0)")
     ap.add_argument("--no-extras", action="store_true", help="skip dense / Y-mode / profile legs")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()
@@ -701,6 +704,33 @@ def main():
         return e
 
     eng = engine(0)
+    refine = None
+    if args.plan_refine:
+        # Alg. 1 picks the plan from the fitted latency models; the models' few-percent error
+        # moves the link / compute balance point by a block or two, so the choice is refined
+        # by measurement: the planner's suffix plan and its neighbours (k - 2 .. k + 2 cached
+        # blocks), a few steps each on this GPU, the fastest kept (an online correction of the
+        # planner, made before the timed region; every rank does the same on its own batch)
+        run_engine_timed(F, eng, reqs_dev, 1, 1, stream, load_stream, rank, world)
+        p0, pred0 = eng.last_plan()
+        N = len(p0)
+        suffix = all(p0[i] <= p0[i + 1] for i in range(N - 1))
+        if suffix:
+            k0 = int(sum(p0))
+            refine = {"planner_cached_blocks": k0, "planner_predicted_ms": pred0, "measured_ms": {}}
+            best = None
+            for k in range(max(0, k0 - 2), min(N, k0 + 2) + 1):
+                e_k = engine(3, plan=[0] * (N - k) + [1] * k)
+                ms_k, _ = run_engine_timed(F, e_k, reqs_dev, 4, 2, stream, load_stream, rank, world)
+                refine["measured_ms"][k] = ms_k
+                if best is None or ms_k < best[0]:
+                    best = (ms_k, k)
+                del e_k
+            if best[1] != k0:
+                del eng
+                eng = engine(3, plan=[0] * (N - best[1]) + [1] * best[1])
+            refine["chosen_cached_blocks"] = best[1]
+            log(f"[rank {rank}] plan refinement {refine}")
     F.fps_engine_set_admission_reuse(eng.h, args.admission_reuse)
     log(f"[rank {rank}] timed run")
     with Clocks(local % n_dev) as clk:
@@ -896,7 +926,7 @@ def main():
             "roofline": roofline,
             "cpu_baseline": cpu,
             "plan": {"cached_blocks": int(sum(plan)), "blocks": len(plan),
-                     "predicted_ms_per_step": pred_ms, "fit": fit},
+                     "predicted_ms_per_step": pred_ms, "fit": fit, "refinement": refine},
             "kernels": per,
             "kernels_stream_split": stream_split,
             "kernels_ncu": ncu_summary(args.config, "classes"),
