@@ -78,9 +78,10 @@ struct ChunkIn {
   uint4 bv[4], rv[8], gv[4];   // rv[4..7]: second halves of an fp32 residual
 };
 __device__ __forceinline__ void chunk_load(const Epilogue& ep, const RowCtx& rc, int N, int row,
-                                           int col0, ChunkIn& in) {
+                                           int col0, ChunkIn& in, bool skip_resid = false) {
   const __nv_bfloat16* __restrict__ bias = reinterpret_cast<const __nv_bfloat16*>(ep.bias);
-  const __nv_bfloat16* __restrict__ resid = reinterpret_cast<const __nv_bfloat16*>(ep.resid);
+  const __nv_bfloat16* __restrict__ resid =
+      skip_resid ? nullptr : reinterpret_cast<const __nv_bfloat16*>(ep.resid);
 #pragma unroll
   for (int g = 0; g < 4; ++g) {
     const int c0 = col0 + g * 8;
@@ -184,10 +185,98 @@ __device__ __forceinline__ void geglu_store(const Epilogue& ep, const RowCtx& rc
   }
 }
 
+#ifdef FPS_GEMM_TRACE
+// developer instrumentation (separate build, `make VARIANT=gtrace EXTRA=-DFPS_GEMM_TRACE`):
+// %globaltimer stamps of every CTA of the last 1-SM GEMM launch -- entry, setup done, PDL wait
+// done, first stage landed (MMA warp), last MMA of its first tile issued, its accumulator
+// ready (epilogue warp 4), its epilogue done, exit
+__device__ unsigned long long g_gemm_trace[160][8];
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+#define GEMM_TRACE(slot) g_gemm_trace[blockIdx.x < 160 ? blockIdx.x : 159][slot] = gtimer()
+#else
+#define GEMM_TRACE(slot) do {} while (0)
+#endif
+
+// Row-major tiles are written through a warp-private shared-memory transpose: the thread that
+// owns a row (TMEM lane) leaves its 32 packed outputs there, then the warp stores 8 rows x 64 B
+// per instruction (4 lanes per row segment) instead of 32 rows x 16 B -- whole, contiguous
+// sectors.  Measured on B200 (tools/gemm_trace.py, one 128 x 256 tile per CTA, no fused ops):
+// the epilogue took 8.5 us against 3.1 us of MMAs with per-row stores and the descriptor read
+// from kernel parameters per chunk, 6.7 us with both changes (4916 x 640 x 640: 19.7 -> 13.9 us;
+// 4916 x 5120 x 640: 63.3 -> 51.6 us); the SDXL block 0.279 -> 0.272 ms, the Flux-scale blocks
+// and the C3 step unchanged within noise (tools/scripts/r02y_epi5.sh).  Handling 64 columns per
+// iteration (two TMEM loads in flight) measured slower (254 registers).
+// Layout: 32 rows x 64 B per warp; piece p (16 B) of row r at r * 64 + ((p ^ (r >> 1 & 3)) << 4)
+// (conflict-free for both the row-per-lane writes and the 4-lanes-per-row reads).
+constexpr int kXsWarpBytes = 32 * 64;
+constexpr int kXsBytes = 4 * kXsWarpBytes;
+
+__device__ __forceinline__ uint32_t xs_off(int r, int p) { return r * 64 + ((p ^ ((r >> 1) & 3)) << 4); }
+
+// Destination of output columns col0..col0+31 of the row (one column region: out0 / out1 /
+// out2, as chunk_store decides per 8 columns); nullptr = nothing to store.
+__device__ __forceinline__ __nv_bfloat16* chunk_dst(const Epilogue& ep, const RowCtx& rc, int N,
+                                                    int col0) {
+  if (!rc.ok || col0 >= N) return nullptr;
+  if (col0 < ep.split)
+    return reinterpret_cast<__nv_bfloat16*>(ep.out0) + (size_t)rc.orow0 * ep.ld0 + col0;
+  if (ep.out2 && col0 >= ep.split2)
+    return reinterpret_cast<__nv_bfloat16*>(ep.out2) + (size_t)rc.row * ep.ld2 + (col0 - ep.split2);
+  return reinterpret_cast<__nv_bfloat16*>(ep.out1) + (size_t)rc.orow1 * ep.ld1 + (col0 - ep.split);
+}
+
+// Fused ops of 32 accumulator values (fp32 bits) of one row -> 4 x 8 packed bf16 (as chunk_store)
+__device__ __forceinline__ void chunk_values(const Epilogue& ep, const RowCtx& rc, int col0,
+                                             const uint32_t* r, const ChunkIn& in, uint4* out) {
+#pragma unroll
+  for (int g = 0; g < 4; ++g) {
+    const int c0 = col0 + g * 8;
+    float v[8], t[8];
+#pragma unroll
+    for (int e = 0; e < 8; ++e) v[e] = __uint_as_float(r[g * 8 + e]);
+    if (ep.bias) {
+      Vec16<__nv_bfloat16>::unpack(in.bv[g], t);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) v[e] += t[e];
+    }
+    if (ep.act == 1 && c0 >= ep.act_from) {
+#pragma unroll
+      for (int e = 0; e < 8; ++e) v[e] = gelu_tanh_fast(v[e]);
+    }
+    if (ep.resid) {
+      float rr[8];
+      if (ep.resid_f32) {
+        Vec16<float>::unpack(in.rv[g], rr);
+        Vec16<float>::unpack(in.rv[g + 4], rr + 4);
+      } else {
+        Vec16<__nv_bfloat16>::unpack(in.rv[g], rr);
+      }
+      if (rc.gate) {
+        Vec16<__nv_bfloat16>::unpack(in.gv[g], t);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) v[e] = rr[e] + t[e] * v[e];
+      } else {
+#pragma unroll
+        for (int e = 0; e < 8; ++e) v[e] = rr[e] + v[e];
+      }
+    }
+    out[g] = Vec16<__nv_bfloat16>::pack(v);
+  }
+}
+
 // Epilogue of one accumulator tile for the calling thread's output row (thread = TMEM lane).
+// xs: this warp's kXsWarpBytes of shared memory (transposed stores), or nullptr.
 template <int BN>
-__device__ __forceinline__ void epilogue_tile(const Epilogue& ep, int M, int N, int row,
-                                              int col_base, uint32_t taddr) {
+__device__ __forceinline__ void epilogue_tile(const Epilogue& ep_param, int M, int N, int row,
+                                              int col_base, uint32_t taddr, uint8_t* xs) {
+  // one copy of the epilogue descriptor in registers per tile: the caller's `p ? ep1 : ep`
+  // is an indexed kernel-parameter access, which re-read field by field (register-indexed
+  // constant loads) cost ~300 cycles per 32-column chunk
+  const Epilogue ep = ep_param;
   const RowCtx rc = row_ctx(ep, M, row);
   if (ep.act == 2) {
 #pragma unroll 1
@@ -204,15 +293,78 @@ __device__ __forceinline__ void epilogue_tile(const Epilogue& ep, int M, int N, 
     }
     return;
   }
+  // the transposed path needs every 32-column chunk inside one output region and bf16 rows
+  const bool staged = xs != nullptr && !ep.out0_f32 && (ep.split & 31) == 0 &&
+                      (!ep.out2 || (ep.split2 & 31) == 0) && (ep.act != 1 || (ep.act_from & 31) == 0);
+  const int lane = threadIdx.x & 31;
+  const uint32_t xs_base = tc::smem_u32(xs);
+  // bf16 residual rows read the same way: 8 rows x 64 B per warp instruction into the staging
+  // buffer, then each thread takes its row (the per-row 16-B loads touched 32 lines per
+  // instruction)
+  const bool coop_resid = staged && ep.resid && !ep.resid_f32;
+  const unsigned long long res_row =
+      (coop_resid && rc.ok)
+          ? reinterpret_cast<unsigned long long>(reinterpret_cast<const __nv_bfloat16*>(ep.resid) +
+                                                 (size_t)rc.rrow * ep.ld_resid)
+          : 0ull;
 #pragma unroll 1
   for (int c = 0; c < BN / 32; ++c) {
     uint32_t r[32];
     tc::tmem_ld32(taddr + c * 32, r);
     const int col0 = col_base + c * 32;
     ChunkIn in;
-    chunk_load(ep, rc, N, row, col0, in);
+    chunk_load(ep, rc, N, row, col0, in, coop_resid);
+    if (coop_resid) {
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int rr = j * 8 + (lane >> 2), piece = lane & 3;
+        const unsigned long long p = __shfl_sync(0xffffffffu, res_row, rr);
+        uint4 v = make_uint4(0, 0, 0, 0);
+        if (p && col0 + piece * 8 < N)
+          v = __ldg(reinterpret_cast<const uint4*>(reinterpret_cast<const char*>(p) +
+                                                    (size_t)col0 * 2 + piece * 16));
+        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(xs_base + xs_off(rr, piece)),
+                     "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+                     : "memory");
+      }
+      __syncwarp();
+#pragma unroll
+      for (int g = 0; g < 4; ++g)
+        asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
+                     : "=r"(in.rv[g].x), "=r"(in.rv[g].y), "=r"(in.rv[g].z), "=r"(in.rv[g].w)
+                     : "r"(xs_base + xs_off(lane, g))
+                     : "memory");
+      __syncwarp();
+    }
     tc::tmem_wait_ld();
-    chunk_store(ep, rc, N, col0, r, in);
+    if (!staged) {
+      chunk_store(ep, rc, N, col0, r, in);
+      continue;
+    }
+    uint4 pk[4];
+    chunk_values(ep, rc, col0, r, in, pk);
+#pragma unroll
+    for (int g = 0; g < 4; ++g)
+      asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(xs_base + xs_off(lane, g)),
+                   "r"(pk[g].x), "r"(pk[g].y), "r"(pk[g].z), "r"(pk[g].w)
+                   : "memory");
+    const unsigned long long dst =
+        reinterpret_cast<unsigned long long>(chunk_dst(ep, rc, N, col0));
+    __syncwarp();
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int rr = j * 8 + (lane >> 2), piece = lane & 3;
+      const unsigned long long p = __shfl_sync(0xffffffffu, dst, rr);
+      if (p && col0 + piece * 8 < N) {
+        uint4 v;
+        asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
+                     : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+                     : "r"(xs_base + xs_off(rr, piece))
+                     : "memory");
+        *reinterpret_cast<uint4*>(reinterpret_cast<char*>(p) + piece * 16) = v;
+      }
+    }
+    __syncwarp();
   }
 }
 
@@ -225,8 +377,10 @@ struct GemmCfg {
   static constexpr int B_BYTES = BN * BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
   static constexpr int TMEM_COLS = 2 * BN;
-  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 + 256;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + kXsBytes + 1024 + 256;
 };
+
+
 
 template <int BN, int STAGES>
 __global__ void __launch_bounds__(256, 1)
@@ -240,13 +394,15 @@ __global__ void __launch_bounds__(256, 1)
                                              ~uintptr_t(1023));
   uint8_t* sA = smem;
   uint8_t* sB = smem + STAGES * Cfg::A_BYTES;
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + STAGES * Cfg::STAGE_BYTES);
+  uint8_t* sXs = smem + STAGES * Cfg::STAGE_BYTES;           // epilogue transpose staging
+  uint64_t* full = reinterpret_cast<uint64_t*>(sXs + kXsBytes);
   uint64_t* empty = full + STAGES;
   uint64_t* tfull = empty + STAGES;
   uint64_t* tempty = tfull + 2;
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(tempty + 2);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) GEMM_TRACE(0);
   const int num_m = (M + Cfg::BM - 1) / Cfg::BM;
   const int num_m1 = (M1 + Cfg::BM - 1) / Cfg::BM;
   const int num_n = (N + BN - 1) / BN;
@@ -275,8 +431,10 @@ __global__ void __launch_bounds__(256, 1)
   __syncthreads();
   tc::fence_after();
   const uint32_t tmem_base = *tmem_holder;
+  if (threadIdx.x == 0) GEMM_TRACE(1);
   pdl_trigger();   // setup done: let the next kernel's CTAs start as ours retire
   pdl_wait();      // inputs of this GEMM come from the previous kernel
+  if (threadIdx.x == 0) GEMM_TRACE(2);
 
   if (warp == 0) {
     if (lane == 0) {
@@ -313,6 +471,7 @@ __global__ void __launch_bounds__(256, 1)
         for (int kb = 0; kb < num_k; ++kb) {
           tc::mbar_wait(&full[stage], phase);
           tc::fence_after();
+          if (it == 0 && kb == 0) GEMM_TRACE(3);
           const uint32_t a0 = tc::smem_u32(sA + stage * Cfg::A_BYTES);
           const uint32_t b0 = tc::smem_u32(sB + stage * Cfg::B_BYTES);
 #pragma unroll
@@ -326,6 +485,7 @@ __global__ void __launch_bounds__(256, 1)
           }
         }
         tc::mma_commit(&tfull[acc]);
+        if (it == 0) GEMM_TRACE(4);
       }
     }
   } else if (warp >= 4) {
@@ -337,19 +497,33 @@ __global__ void __launch_bounds__(256, 1)
       const int acc = it & 1;
       tc::mbar_wait(&tfull[acc], (it >> 1) & 1);
       tc::fence_after();
+      if (it == 0 && warp == 4 && lane == 0) GEMM_TRACE(5);
       epilogue_tile<BN>(p ? ep1 : ep, p ? M1 : M, N, m_blk * Cfg::BM + q * 32 + lane, n_blk * BN,
-                        tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN);
+                        tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN,
+                        sXs + q * kXsWarpBytes);
+      if (it == 0 && warp == 4 && lane == 0) GEMM_TRACE(6);
       tc::fence_before();
       __syncwarp();
       if (lane == 0) tc::mbar_arrive(&tempty[acc]);
     }
   }
+  __syncwarp();     // each role warp reconverged (lane 0 ran the producer / MMA loop alone)
   __syncthreads();
+  if (threadIdx.x == 0) GEMM_TRACE(7);
   if (warp == 2) {
     tc::fence_after();
     tc::tmem_dealloc<Cfg::TMEM_COLS>(tmem_base);
   }
 }
+
+#ifdef FPS_GEMM_TRACE
+}  // namespace fps
+extern "C" int fps_debug_gemm_trace(unsigned long long* out) {
+  return (int)cudaMemcpyFromSymbol(out, fps::g_gemm_trace, sizeof(fps::g_gemm_trace));
+}
+
+namespace fps {
+#endif
 
 // ============================================================================================
 // CTA-pair kernel (cta_group::2): 256 x 256 tile per pair
@@ -360,7 +534,7 @@ struct Gemm2Cfg {
   static constexpr int B_BYTES = 128 * BK * 2;             // per CTA: its 128 rows of B
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
   static constexpr int TMEM_COLS = 512;                    // 2 accumulators x 256 columns
-  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 + 256;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + kXsBytes + 1024 + 256;
 };
 
 template <int STAGES>
@@ -375,7 +549,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
                                              ~uintptr_t(1023));
   uint8_t* sA = smem;
   uint8_t* sB = smem + STAGES * Cfg::A_BYTES;
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + STAGES * Cfg::STAGE_BYTES);
+  uint8_t* sXs = smem + STAGES * Cfg::STAGE_BYTES;           // epilogue transpose staging
+  uint64_t* full = reinterpret_cast<uint64_t*>(sXs + kXsBytes);
   uint64_t* empty = full + STAGES;
   uint64_t* tfull = empty + STAGES;
   uint64_t* tempty = tfull + 2;
@@ -479,7 +654,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
       tc::fence_after();
       epilogue_tile<256>(p ? ep1 : ep, p ? M1 : M, N,
                          m_blk * Cfg::BM + rank * 128 + q * 32 + lane, n_blk * Cfg::BN,
-                         tmem_base + ((uint32_t)(q * 32) << 16) + acc * 256);
+                         tmem_base + ((uint32_t)(q * 32) << 16) + acc * 256,
+                         sXs + q * kXsWarpBytes);
       tc::fence_before();
       __syncwarp();
       if (lane == 0) tc::mbar_arrive_cluster(tempty_leader + acc * 8);
