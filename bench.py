@@ -709,8 +709,9 @@ def main():
         # Alg. 1 picks the plan from the fitted latency models; the models' few-percent error
         # moves the link / compute balance point by a block or two, so the choice is refined
         # by measurement: the planner's suffix plan and its neighbours (k - 2 .. k + 2 cached
-        # blocks), a few steps each on this GPU, the fastest kept (an online correction of the
-        # planner, made before the timed region; every rank does the same on its own batch)
+        # blocks, extended while the best sits at an edge and keeps improving), a few steps
+        # each on this GPU, the fastest kept (an online correction of the planner, made before
+        # the timed region; every rank does the same on its own batch)
         run_engine_timed(F, eng, reqs_dev, 1, 1, stream, load_stream, rank, world)
         p0, pred0 = eng.last_plan()
         N = len(p0)
@@ -718,14 +719,25 @@ def main():
         if suffix:
             k0 = int(sum(p0))
             refine = {"planner_cached_blocks": k0, "planner_predicted_ms": pred0, "measured_ms": {}}
-            best = None
-            for k in range(max(0, k0 - 2), min(N, k0 + 2) + 1):
+            def measure(k):
                 e_k = engine(3, plan=[0] * (N - k) + [1] * k)
                 ms_k, _ = run_engine_timed(F, e_k, reqs_dev, 4, 2, stream, load_stream, rank, world)
                 refine["measured_ms"][k] = ms_k
-                if best is None or ms_k < best[0]:
-                    best = (ms_k, k)
                 del e_k
+                return ms_k
+            for k in range(max(0, k0 - 2), min(N, k0 + 2) + 1):
+                measure(k)
+            # the best at an edge of the window: keep walking that way while it improves
+            while True:
+                kb = min(refine["measured_ms"], key=refine["measured_ms"].get)
+                lo, hi = min(refine["measured_ms"]), max(refine["measured_ms"])
+                nxt = kb - 1 if (kb == lo and lo > 0) else kb + 1 if (kb == hi and hi < N) else None
+                if nxt is None or len(refine["measured_ms"]) >= 12:
+                    break
+                if measure(nxt) >= refine["measured_ms"][kb]:
+                    break
+            kb = min(refine["measured_ms"], key=refine["measured_ms"].get)
+            best = (refine["measured_ms"][kb], kb)
             if best[1] != k0:
                 del eng
                 eng = engine(3, plan=[0] * (N - best[1]) + [1] * best[1])
