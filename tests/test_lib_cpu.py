@@ -122,8 +122,36 @@ def test_cross_step_planner_matches_oracle(mode):
         assert got == pytest.approx(ref, rel=1e-9)
         best, bplan = P.plan_steady_suffix(Cw, Cwo, Lm, mode, fin)
         plan, lat = fps.plan_pipeline(Cw, Cwo, Lm, m, fin, cross_step=True)
-        assert lat == pytest.approx(best, rel=1e-9)
-        assert P.steady_step_latency(plan, Cw, Cwo, Lm, mode, fin) == pytest.approx(best, rel=1e-9)
+        # the returned latency is the oracle model's value of the returned plan
+        assert P.steady_step_latency(plan, Cw, Cwo, Lm, mode, fin) == pytest.approx(lat, rel=1e-9)
+        if mode == "kv":
+            assert lat == pytest.approx(best, rel=1e-9)      # the N+1 suffixes are all plans
+        else:
+            assert lat <= best * (1 + 1e-9)                   # local search from the best suffix
+
+
+def test_cross_step_y_planner_local_search_vs_brute_force():
+    """Y-mode cross-step plans (any pattern): the library's local search over the steady-state
+    model (seeded by the best suffix and the per-step Pareto plan) against exhaustive search
+    on heterogeneous random stacks of up to 10 blocks: never worse than the suffix scan, exact
+    in at least 90 % of the cases and within 10 % of the optimum in all."""
+    import itertools
+    g = synth.rng(15)
+    exact = worse_than_suffix = 0
+    n_cases = 60
+    for _ in range(n_cases):
+        N = int(g.integers(2, 11))
+        Cw, Cwo, Lm, fin = _rand_costs(g, N)
+        Lm = [v * float(g.uniform(0.2, 3.0)) for v in Lm]         # heterogeneous loads
+        plan, lat = fps.plan_pipeline(Cw, Cwo, Lm, fps.FPS_MODE_Y, fin, cross_step=True)
+        opt = min(P.steady_step_latency(list(u), Cw, Cwo, Lm, "y", fin)
+                  for u in itertools.product([0, 1], repeat=N))
+        suffix, _ = P.plan_steady_suffix(Cw, Cwo, Lm, "y", fin)
+        assert lat >= opt * (1 - 1e-9) and lat <= opt * 1.10, (N, lat, opt)
+        worse_than_suffix += lat > suffix * (1 + 1e-9)
+        exact += abs(lat - opt) <= 1e-9 * max(1.0, opt)
+    assert worse_than_suffix == 0
+    assert exact >= 0.9 * n_cases, exact
 
 
 def _weights(kind, **kw):
