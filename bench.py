@@ -621,6 +621,9 @@ def main():
             dist.init_process_group("gloo")
             DIST_DEVICE = torch.device("cpu")
             log(f"[rank {rank}] {world} ranks on {n_dev} GPU(s): shared devices, gloo reductions")
+            # processes time-sharing one GPU: launch without programmatic dependent launch (two
+            # such runs hung a rank's step -- device work never completed -- out of eight)
+            F.fps_set_disable_tc(int(os.environ.get("FPS_KERNEL_FLAGS", 0)) | 64)
 
     # requests of the whole job, routed to GPUs by Alg. 2 (identical on every rank: no comms)
     pool = make_requests(w, w["batch"] * world, SEED)
