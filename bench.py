@@ -580,6 +580,10 @@ def main():
     if args.impl == "reference":
         if rank != 0:
             return
+        # the same config keys as our arm's line (one GPU: the whole pool is this rank's)
+        ref_pool = make_requests(w, w["batch"], SEED)
+        base_cfg.update(mask_ratios=sorted({p["ratio"] for p in ref_pool}),
+                        mean_active_rows=statistics.mean(p["n_active"] for p in ref_pool))
         # the oracle as it stands, one block of one request per step; extrapolated to the step
         times = []
         for i in range(W + K):

@@ -26,6 +26,8 @@ def main():
     bench.COPY_CTAS = int(os.environ.get("PROBE_CTAS", 0))
     import paper_conf_eurosys_jianglyfdlzllyl26_b200 as F
     F.require_gpu()
+    if os.environ.get("FPS_KERNEL_FLAGS"):
+        F.fps_set_disable_tc(int(os.environ["FPS_KERNEL_FLAGS"]))
     dev = torch.device("cuda", 0)
     w = dict(bench.WORKLOADS[cfg], block="sdxl" if cfg.startswith("C2") else "flux")
     w["steps"] = max(w["steps"], 3 + K)
