@@ -654,7 +654,7 @@ __device__ __forceinline__ constexpr bool attn_poly(int i) {
 __device__ long long g_attn_trace[2][64][8];
 #define ATTN_TRACE(t, kt, slot)                                                     \
   do {                                                                              \
-    if (blockIdx.x == 5 && blockIdx.y == 3 && (threadIdx.x & 31) == 0 && (kt) < 64) \
+    if (blockIdx.x == 2 && blockIdx.y == 3 && (threadIdx.x & 31) == 0 && (kt) < 64) \
       g_attn_trace[t][kt][slot] = clock64();                                        \
   } while (0)
 #else
@@ -1225,3 +1225,9 @@ fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads
 }
 
 }  // namespace fps
+
+#ifdef FPS_ATTN_TRACE
+extern "C" int fps_debug_attn_trace(long long* out) {
+  return (int)cudaMemcpyFromSymbol(out, fps::g_attn_trace, sizeof(fps::g_attn_trace));
+}
+#endif
