@@ -58,7 +58,9 @@ int32_t fps_device_ok(void);
  * library copy kernel (experiments only: see cache.cu);
  * bits 8-10 = S > 0 forces the split-KV factor of the tensor-core attention inside block calls
  * (0 = chosen by wave efficiency; S is applied only when the block workspace holds the S
- * partial outputs). */
+ * partial outputs);
+ * bit 11 = the 1-SM tcgen05 GEMM with 4 epilogue warps instead of 8 (A/B experiments);
+ * bit 12 = the CTA-pair attention kernel (attn_tc4, head_dim 128). */
 int64_t fps_launch_count(void);
 void fps_set_disable_tc(int32_t flags);
 /* Per-kernel-class timing for the bench: when enabled (this also clears old records) every

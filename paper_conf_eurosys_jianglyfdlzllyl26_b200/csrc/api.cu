@@ -604,6 +604,8 @@ void fps_set_disable_tc(int32_t flags) {
   fps::g_pdl = (flags & 64) ? 0 : 1;
   fps::g_d2d_kernel = (flags & 128) ? 0 : 1;
   fps::g_attn_split = (flags >> 8) & 7;
+  fps::g_gemm_epi4 = (flags >> 11) & 1;
+  fps::g_attn_pair = (flags >> 12) & 1;
 }
 
 fps_status fps_build_mask_index(const uint8_t* d_masks, const int32_t* d_offsets, int32_t n_req,

@@ -213,7 +213,7 @@ __device__ __forceinline__ unsigned long long gtimer() {
 // Layout: 32 rows x 64 B per warp; piece p (16 B) of row r at r * 64 + ((p ^ (r >> 1 & 3)) << 4)
 // (conflict-free for both the row-per-lane writes and the 4-lanes-per-row reads).
 constexpr int kXsWarpBytes = 32 * 64;
-constexpr int kXsBytes = 4 * kXsWarpBytes;
+constexpr int kXsBytes = 4 * kXsWarpBytes;      // pair kernels: 4 epilogue warps per CTA
 
 __device__ __forceinline__ uint32_t xs_off(int r, int p) { return r * 64 + ((p ^ ((r >> 1) & 3)) << 4); }
 
@@ -307,11 +307,146 @@ __device__ __forceinline__ void epilogue_tile(const Epilogue& ep_param, int M, i
           ? reinterpret_cast<unsigned long long>(reinterpret_cast<const __nv_bfloat16*>(ep.resid) +
                                                  (size_t)rc.rrow * ep.ld_resid)
           : 0ull;
+  // Whole 32-column chunks inside one output region (the common case) take a branch-light path:
+  // the fused-op flags are tested once per chunk, not per 8 columns, and no operand is
+  // zero-filled (the generic path below costs ~330 instructions per chunk, ~half of them guards)
+  const bool aligned = (ep.split & 31) == 0 && (!ep.out2 || (ep.split2 & 31) == 0) &&
+                       (ep.act != 1 || (ep.act_from & 31) == 0);
 #pragma unroll 1
   for (int c = 0; c < BN / 32; ++c) {
     uint32_t r[32];
     tc::tmem_ld32(taddr + c * 32, r);
     const int col0 = col_base + c * 32;
+    if (aligned && col0 + 32 <= N) {
+      const bool f_bias = ep.bias != nullptr;
+      const bool f_res = ep.resid != nullptr && rc.ok;
+      const bool f_gate = rc.gate != nullptr;
+      uint4 bv[4], gv[4], rv[8];
+      if (f_bias) {
+        const uint4* b = reinterpret_cast<const uint4*>(reinterpret_cast<const __nv_bfloat16*>(ep.bias) + col0);
+#pragma unroll
+        for (int g = 0; g < 4; ++g) bv[g] = __ldg(b + g);
+      }
+      if (f_gate) {
+        const uint4* gp = reinterpret_cast<const uint4*>(rc.gate + col0);
+#pragma unroll
+        for (int g = 0; g < 4; ++g) gv[g] = __ldg(gp + g);
+      }
+      if (ep.resid_f32) {
+        if (f_res) {
+          const uint4* rp = reinterpret_cast<const uint4*>(reinterpret_cast<const float*>(ep.resid) +
+                                                           (size_t)rc.rrow * ep.ld_resid + col0);
+#pragma unroll
+          for (int g = 0; g < 8; ++g) rv[g] = __ldg(rp + g);
+        }
+      } else if (coop_resid) {
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const int rr = j * 8 + (lane >> 2), piece = lane & 3;
+          const unsigned long long pr = __shfl_sync(0xffffffffu, res_row, rr);
+          uint4 v = make_uint4(0, 0, 0, 0);
+          if (pr) v = __ldg(reinterpret_cast<const uint4*>(reinterpret_cast<const char*>(pr) +
+                                                           (size_t)col0 * 2 + piece * 16));
+          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(xs_base + xs_off(rr, piece)),
+                       "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+                       : "memory");
+        }
+        __syncwarp();
+#pragma unroll
+        for (int g = 0; g < 4; ++g)
+          asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
+                       : "=r"(rv[g].x), "=r"(rv[g].y), "=r"(rv[g].z), "=r"(rv[g].w)
+                       : "r"(xs_base + xs_off(lane, g))
+                       : "memory");
+        __syncwarp();
+      } else if (f_res) {
+        const uint4* rp = reinterpret_cast<const uint4*>(reinterpret_cast<const __nv_bfloat16*>(ep.resid) +
+                                                         (size_t)rc.rrow * ep.ld_resid + col0);
+#pragma unroll
+        for (int g = 0; g < 4; ++g) rv[g] = __ldg(rp + g);
+      }
+      tc::tmem_wait_ld();
+      float v[32];
+#pragma unroll
+      for (int e = 0; e < 32; ++e) v[e] = __uint_as_float(r[e]);
+      if (f_bias) {
+#pragma unroll
+        for (int g = 0; g < 4; ++g) {
+          float t[8];
+          Vec16<__nv_bfloat16>::unpack(bv[g], t);
+#pragma unroll
+          for (int e = 0; e < 8; ++e) v[g * 8 + e] += t[e];
+        }
+      }
+      if (ep.act == 1 && col0 >= ep.act_from) {
+#pragma unroll
+        for (int e = 0; e < 32; ++e) v[e] = gelu_tanh_fast(v[e]);
+      }
+      if (f_res) {
+        float rr[32];
+        if (ep.resid_f32) {
+#pragma unroll
+          for (int g = 0; g < 8; ++g) Vec16<float>::unpack(rv[g], rr + g * 4);
+        } else {
+#pragma unroll
+          for (int g = 0; g < 4; ++g) Vec16<__nv_bfloat16>::unpack(rv[g], rr + g * 8);
+        }
+        if (f_gate) {
+#pragma unroll
+          for (int g = 0; g < 4; ++g) {
+            float t[8];
+            Vec16<__nv_bfloat16>::unpack(gv[g], t);
+#pragma unroll
+            for (int e = 0; e < 8; ++e) v[g * 8 + e] = rr[g * 8 + e] + t[e] * v[g * 8 + e];
+          }
+        } else {
+#pragma unroll
+          for (int e = 0; e < 32; ++e) v[e] += rr[e];
+        }
+      }
+      if (ep.out0_f32 && col0 < ep.split) {                // fp32 rows: 128 B per row per chunk
+        if (rc.ok) {
+          uint4* df = reinterpret_cast<uint4*>(reinterpret_cast<float*>(ep.out0) +
+                                               (size_t)rc.orow0 * ep.ld0 + col0);
+#pragma unroll
+          for (int g = 0; g < 8; ++g) df[g] = Vec16<float>::pack(v + g * 4);
+        }
+        continue;
+      }
+      uint4 pk[4];
+#pragma unroll
+      for (int g = 0; g < 4; ++g) pk[g] = Vec16<__nv_bfloat16>::pack(v + g * 8);
+      __nv_bfloat16* const dst = chunk_dst(ep, rc, N, col0);
+      if (!staged) {
+        if (dst) {
+#pragma unroll
+          for (int g = 0; g < 4; ++g) reinterpret_cast<uint4*>(dst)[g] = pk[g];
+        }
+        continue;
+      }
+#pragma unroll
+      for (int g = 0; g < 4; ++g)
+        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(xs_base + xs_off(lane, g)),
+                     "r"(pk[g].x), "r"(pk[g].y), "r"(pk[g].z), "r"(pk[g].w)
+                     : "memory");
+      const unsigned long long dd = reinterpret_cast<unsigned long long>(dst);
+      __syncwarp();
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int rr = j * 8 + (lane >> 2), piece = lane & 3;
+        const unsigned long long p = __shfl_sync(0xffffffffu, dd, rr);
+        if (p) {
+          uint4 v4;
+          asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
+                       : "=r"(v4.x), "=r"(v4.y), "=r"(v4.z), "=r"(v4.w)
+                       : "r"(xs_base + xs_off(rr, piece))
+                       : "memory");
+          *reinterpret_cast<uint4*>(reinterpret_cast<char*>(p) + piece * 16) = v4;
+        }
+      }
+      __syncwarp();
+      continue;
+    }
     ChunkIn in;
     chunk_load(ep, rc, N, row, col0, in, coop_resid);
     if (coop_resid) {
@@ -370,24 +505,31 @@ __device__ __forceinline__ void epilogue_tile(const Epilogue& ep_param, int M, i
 
 // ============================================================================================
 // 1-SM kernel
-template <int BN, int STAGES>
+// EPI epilogue warps: 4 (thread = TMEM lane = output row, all BN columns) or 8 (two warps per
+// TMEM lane quarter, BN / 2 columns each).  The epilogue of a 128-row tile is issue-bound in
+// its warp (~330 instructions per 32-column chunk with the fused-op guards), so for short-K
+// problems -- the SDXL-scale projections at K = 640, one tile per CTA -- it, not the MMAs, sets
+// the CTA's time; two warps per quarter halve that chain.
+template <int BN, int STAGES, int EPI = 8>
 struct GemmCfg {
   static constexpr int BM = 128, BK = 64;
   static constexpr int A_BYTES = BM * BK * 2;
   static constexpr int B_BYTES = BN * BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
   static constexpr int TMEM_COLS = 2 * BN;
-  static constexpr int SMEM = STAGES * STAGE_BYTES + kXsBytes + 1024 + 256;
+  static constexpr int XS_BYTES = EPI * kXsWarpBytes;
+  static constexpr int THREADS = 128 + 32 * EPI;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + XS_BYTES + 1024 + 256;
 };
 
 
 
-template <int BN, int STAGES>
-__global__ void __launch_bounds__(256, 1)
+template <int BN, int STAGES, int EPI>
+__global__ void __launch_bounds__(GemmCfg<BN, STAGES, EPI>::THREADS, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const __grid_constant__ CUtensorMap tmB1, int M, int N, int K, Epilogue ep,
                    int M1, Epilogue ep1) {
-  using Cfg = GemmCfg<BN, STAGES>;
+  using Cfg = GemmCfg<BN, STAGES, EPI>;
   constexpr int kGroupM = 16;                              // 2048 rows of A per group
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
@@ -395,7 +537,7 @@ __global__ void __launch_bounds__(256, 1)
   uint8_t* sA = smem;
   uint8_t* sB = smem + STAGES * Cfg::A_BYTES;
   uint8_t* sXs = smem + STAGES * Cfg::STAGE_BYTES;           // epilogue transpose staging
-  uint64_t* full = reinterpret_cast<uint64_t*>(sXs + kXsBytes);
+  uint64_t* full = reinterpret_cast<uint64_t*>(sXs + Cfg::XS_BYTES);
   uint64_t* empty = full + STAGES;
   uint64_t* tfull = empty + STAGES;
   uint64_t* tempty = tfull + 2;
@@ -417,7 +559,7 @@ __global__ void __launch_bounds__(256, 1)
     }
     for (int a = 0; a < 2; ++a) {
       tc::mbar_init(&tfull[a], 1);
-      tc::mbar_init(&tempty[a], 4);
+      tc::mbar_init(&tempty[a], EPI);
     }
     tc::fence_mbar_init();
   }
@@ -436,6 +578,7 @@ __global__ void __launch_bounds__(256, 1)
   pdl_wait();      // inputs of this GEMM come from the previous kernel
   if (threadIdx.x == 0) GEMM_TRACE(2);
 
+  if (EPI == 8 && warp < 4) tc::regs_dec<72>();
   if (warp == 0) {
     if (lane == 0) {
       int stage = 0;
@@ -489,7 +632,10 @@ __global__ void __launch_bounds__(256, 1)
       }
     }
   } else if (warp >= 4) {
-    const int q = warp & 3;
+    if (EPI == 8) tc::regs_inc<216>();
+    const int q = warp & 3;                                // TMEM lane quarter (warp id % 4)
+    constexpr int CW = BN * 4 / EPI;                       // columns per epilogue warp
+    const int h = (warp - 4) >> 2;                         // column part of this warp
     int it = 0;
     for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++it) {
       int p, m_blk, n_blk;
@@ -498,9 +644,10 @@ __global__ void __launch_bounds__(256, 1)
       tc::mbar_wait(&tfull[acc], (it >> 1) & 1);
       tc::fence_after();
       if (it == 0 && warp == 4 && lane == 0) GEMM_TRACE(5);
-      epilogue_tile<BN>(p ? ep1 : ep, p ? M1 : M, N, m_blk * Cfg::BM + q * 32 + lane, n_blk * BN,
-                        tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN,
-                        sXs + q * kXsWarpBytes);
+      epilogue_tile<CW>(p ? ep1 : ep, p ? M1 : M, N, m_blk * Cfg::BM + q * 32 + lane,
+                        n_blk * BN + h * CW,
+                        tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + h * CW,
+                        sXs + (warp - 4) * kXsWarpBytes);
       if (it == 0 && warp == 4 && lane == 0) GEMM_TRACE(6);
       tc::fence_before();
       __syncwarp();
@@ -856,24 +1003,33 @@ struct Group2 {
   Epilogue ep1;
 };
 
-template <int BN, int STAGES>
-static fps_status launch_cfg(const void* A, const void* B, int M, int N, int K,
-                             const Epilogue& ep, cudaStream_t s, const Group2& g2 = Group2{}) {
-  using Cfg = GemmCfg<BN, STAGES>;
+int g_gemm_epi4 = 0;    // tests / A-B: 1 = the 1-SM kernel with 4 epilogue warps instead of 8
+
+template <int BN, int STAGES, int EPI>
+static fps_status launch_cfg_e(const void* A, const void* B, int M, int N, int K,
+                               const Epilogue& ep, cudaStream_t s, const Group2& g2) {
+  using Cfg = GemmCfg<BN, STAGES, EPI>;
   CUtensorMap ta, tb, tb1;
   if (!make_tmap_2d_bf16(&ta, A, M + g2.M1, K, (uint64_t)K * 2, Cfg::BK, Cfg::BM) ||
       !make_tmap_2d_bf16(&tb, B, N, K, (uint64_t)K * 2, Cfg::BK, BN) ||
       (g2.M1 > 0 && !make_tmap_2d_bf16(&tb1, g2.B1, N, K, (uint64_t)K * 2, Cfg::BK, BN)))
     return fail(FPS_ECUDA, "gemm_tc: cuTensorMapEncodeTiled failed (M=%d N=%d K=%d)", M, N, K);
   if (g2.M1 == 0) tb1 = tb;
-  FPS_SMEM_ATTR((gemm_tc_kernel<BN, STAGES>), Cfg::SMEM);
+  FPS_SMEM_ATTR((gemm_tc_kernel<BN, STAGES, EPI>), Cfg::SMEM);
   const int tiles = (ceil_div(M, Cfg::BM) + ceil_div(g2.M1, Cfg::BM)) * ceil_div(N, BN);
   const int grid = tiles < sm_budget() ? tiles : sm_budget();
-  FPS_CUDA_TRY(launch_k(gemm_tc_kernel<BN, STAGES>, dim3(grid), dim3(256), Cfg::SMEM, s, ta, tb,
+  FPS_CUDA_TRY(launch_k(gemm_tc_kernel<BN, STAGES, EPI>, dim3(grid), dim3(Cfg::THREADS), Cfg::SMEM, s, ta, tb,
                         tb1, M, N, K, ep, g2.M1, g2.ep1));
   count_launch();
   FPS_LAUNCH_CHECK();
   return FPS_OK;
+}
+
+template <int BN, int STAGES>
+static fps_status launch_cfg(const void* A, const void* B, int M, int N, int K,
+                             const Epilogue& ep, cudaStream_t s, const Group2& g2 = Group2{}) {
+  if (g_gemm_epi4) return launch_cfg_e<BN, STAGES, 4>(A, B, M, N, K, ep, s, g2);
+  return launch_cfg_e<BN, STAGES, 8>(A, B, M, N, K, ep, s, g2);
 }
 
 template <int STAGES>

@@ -98,8 +98,10 @@ int bulk_ctas(const fps_cache* c);
 extern int g_disable_tc;
 // tests: 0 = choose, 1 = force the 1-SM tcgen05 GEMM, 2 = force the CTA-pair GEMM
 extern int g_gemm_force;
+extern int g_gemm_epi4;
 // tests: 0 = two query tiles per CTA (default), 1 = force the one-tile attention kernel
 extern int g_attn_force;
+extern int g_attn_pair;
 // tests: force the split-KV factor S (0 = choose)
 extern int g_attn_split;
 // 1 (default): HBM-arena whole-entry loads copied by a library kernel, 0: driver D2D memcpy
