@@ -1006,6 +1006,349 @@ __global__ void __launch_bounds__(512, 1)
   }
 }
 
+// ============================================================================================
+// attn_tc4: CTA-pair (cta_group::2) attention, head_dim 128.  A cluster of two CTAs on two SMs
+// takes two query tiles of one request (128 rows each, one per CTA); every MMA is issued by the
+// leader for both:
+//   S  = Q K^T   M = 256 (both tiles), N = 128 keys: each CTA stages its Q tile and HALF of the
+//                key tile (64 keys) -- per SM half the K bytes of the 1-SM kernel, both from TMA
+//                and from the smem port the MMA reads operands through;
+//   O += P V     M = 256, N = 128: each CTA stages half of V's columns, P from each CTA's TMEM.
+// S is double-buffered in TMEM (cols 0-127 / 128-255, O at 256-383), so S(j+1) is computed
+// while the softmax works on S(j): the tensor pipe no longer waits for the exponentials of the
+// tile it has just produced (attn_tc3's chain S -> softmax -> PV -> next S, measured 3066 cycles
+// per key tile for two query tiles against 2048 of MMAs, tools/attn_trace.py).
+// Warps: 0 K/Q producer, 1 MMA issuer (leader CTA), 2 TMEM allocator, 3 V producer,
+// 4-11 softmax (two warps per TMEM lane quarter, 64 key columns each; the row max is exchanged
+// through shared memory with a 64-thread named barrier), 12-15 correction + epilogue.
+// Barriers on the leader count both CTAs' arrivals (P stored: softmax + correction warps of
+// the two CTAs); MMA completions are multicast to both CTAs.
+#ifndef FPS_ATTN4_POLY
+#define FPS_ATTN4_POLY 4
+#endif
+struct Attn4Cfg {
+  static constexpr int D = 128;
+  static constexpr int KS = 3, VS = 3;                      // K / V ring depths
+  static constexpr int Q_BYTES = 128 * D * 2;               // this CTA's query tile
+  static constexpr int K_HALF = 64 * D * 2;                 // 64 keys x 128 (2 chunks of 8 KB)
+  static constexpr int V_HALF = 128 * 64 * 2;               // 128 keys x 64 columns
+  static constexpr int SMEM = Q_BYTES + KS * K_HALF + VS * V_HALF + (4 + 2 + 2 + 1) * 128 * 4 + 1024 + 512;
+  static constexpr int TMEM_COLS = 512;
+};
+
+__device__ __forceinline__ void named_bar_sync(int id, int n) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(512, 1)
+    attn_tc4_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
+                    const __grid_constant__ CUtensorMap tmV, __nv_bfloat16* __restrict__ O,
+                    const int32_t* __restrict__ cu_q, const int32_t* __restrict__ cu_k, int n_req,
+                    int heads, float scale_log2, int ldo, __nv_bfloat16* __restrict__ Opart,
+                    float2* __restrict__ ML, long long part_stride, int total_q,
+                    const int32_t* __restrict__ o_map) {
+  using Cfg = Attn4Cfg;
+  constexpr int D = Cfg::D;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~uintptr_t(1023));
+  uint8_t* sQ = smem;
+  uint8_t* sK = sQ + Cfg::Q_BYTES;
+  uint8_t* sV = sK + Cfg::KS * Cfg::K_HALF;
+  float* sMax = reinterpret_cast<float*>(sV + Cfg::VS * Cfg::V_HALF);   // [buf][half][row]
+  float* sScale = sMax + 4 * 128;                                        // [buf][row]
+  float* sL = sScale + 2 * 128;                                          // [half][row]
+  float* sM = sL + 2 * 128;                                              // [row] final max
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sM + 128);
+  uint64_t* bar_q = bars;                  // leader: both Q tiles landed
+  uint64_t* k_full = bars + 1;             // [KS] leader: both K halves landed
+  uint64_t* k_empty = bars + 4;            // [KS] both: S MMA done with the stage (multicast)
+  uint64_t* v_full = bars + 7;             // [VS] leader
+  uint64_t* v_empty = bars + 10;           // [VS] both (multicast)
+  uint64_t* bar_s = bars + 13;             // [buf] both: S(j) in TMEM (multicast)
+  uint64_t* bar_p = bars + 15;             // [buf] leader: keys 0-63 of P + O rescaled (2 x 8 warps)
+  uint64_t* bar_p2 = bars + 17;            // [buf] leader: keys 64-127 of P (2 x 4 warps)
+  uint64_t* bar_stat = bars + 19;          // [buf] local: scale of step j in smem (4 warps)
+  uint64_t* bar_pv = bars + 21;            // both: PV(j) complete (multicast)
+  uint64_t* bar_o = bars + 22;             // both: last PV complete (multicast)
+  uint64_t* bar_fin = bars + 23;           // local: row-sum halves in smem (8 warps)
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + 24);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = tc::cluster_ctarank();
+  const int head = blockIdx.y;
+  const int H = heads * D;
+  int r = 0, qp = blockIdx.x >> 1, ntile = 0;
+  for (; r < n_req; ++r) {
+    ntile = (__ldg(cu_q + r + 1) - __ldg(cu_q + r) + 127) >> 7;
+    const int np = (ntile + 1) >> 1;
+    if (qp < np) break;
+    qp -= np;
+  }
+  const int q_end = __ldg(cu_q + r + 1);
+  const int q0 = __ldg(cu_q + r) + qp * 256 + (int)rank * 128;   // this CTA's first query row
+  const int Lr = __ldg(cu_k + r + 1) - __ldg(cu_k + r);
+  const int nk_all = (Lr + 127) >> 7;
+  const int nsplit = gridDim.z, split = blockIdx.z;
+  const int kb = (int)(((long long)nk_all * split) / nsplit);
+  const int nk = (int)(((long long)nk_all * (split + 1)) / nsplit) - kb;
+  const int k0 = __ldg(cu_k + r) + kb * 128;
+  const int Lr_rem = Lr - kb * 128;
+
+  if (threadIdx.x == 0) {
+    tc::mbar_init(bar_q, 1);
+    for (int s = 0; s < Cfg::KS; ++s) {
+      tc::mbar_init(&k_full[s], 1);
+      tc::mbar_init(&k_empty[s], 1);
+    }
+    for (int s = 0; s < Cfg::VS; ++s) {
+      tc::mbar_init(&v_full[s], 1);
+      tc::mbar_init(&v_empty[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      tc::mbar_init(&bar_s[b], 1);
+      tc::mbar_init(&bar_p[b], 16);
+      tc::mbar_init(&bar_p2[b], 8);
+      tc::mbar_init(&bar_stat[b], 4);
+    }
+    tc::mbar_init(bar_pv, 1);
+    tc::mbar_init(bar_o, 1);
+    tc::mbar_init(bar_fin, 8);
+    tc::fence_mbar_init();
+  }
+  if (warp == 0 && lane == 0) {
+    tc::tma_prefetch_desc(&tmQ);
+    tc::tma_prefetch_desc(&tmK);
+    tc::tma_prefetch_desc(&tmV);
+  }
+  if (warp == 2) tc::tmem_alloc_2sm<Cfg::TMEM_COLS>(tmem_holder);
+  tc::fence_before();
+  __syncthreads();
+  tc::cluster_sync();                                      // peer barriers initialised
+  tc::fence_after();
+  const uint32_t tmem = *tmem_holder;
+  pdl_trigger();
+  pdl_wait();
+
+  if (warp < 4) {
+    tc::regs_dec<88>();
+    if (warp == 0) {
+      if (lane == 0 && nk > 0) {
+        if (rank == 0) tc::mbar_expect_tx(bar_q, 2 * Cfg::Q_BYTES);
+#pragma unroll
+        for (int c = 0; c < D / 64; ++c)
+          tc::tma_load_2d_2sm(sQ + c * (Cfg::Q_BYTES / 2), &tmQ, bar_q, head * D + c * 64, q0);
+        for (int kt = 0; kt < nk; ++kt) {
+          const int st = kt % Cfg::KS;
+          tc::mbar_wait_sleep(&k_empty[st], ((kt / Cfg::KS) & 1) ^ 1);
+          if (rank == 0) tc::mbar_expect_tx(&k_full[st], 2 * Cfg::K_HALF);
+#pragma unroll
+          for (int c = 0; c < D / 64; ++c)
+            tc::tma_load_2d_2sm(sK + st * Cfg::K_HALF + c * (Cfg::K_HALF / 2), &tmK, &k_full[st],
+                                head * D + c * 64, k0 + kt * 128 + (int)rank * 64);
+        }
+      }
+    } else if (warp == 3) {
+      if (lane == 0) {
+        for (int kt = 0; kt < nk; ++kt) {
+          const int st = kt % Cfg::VS;
+          tc::mbar_wait_sleep(&v_empty[st], ((kt / Cfg::VS) & 1) ^ 1);
+          if (rank == 0) tc::mbar_expect_tx(&v_full[st], 2 * Cfg::V_HALF);
+          tc::tma_load_2d_2sm(sV + st * Cfg::V_HALF, &tmV, &v_full[st], H + head * D + (int)rank * 64,
+                              k0 + kt * 128);
+        }
+      }
+    } else if (warp == 1) {
+      if (rank == 0 && nk > 0) {
+        constexpr uint32_t idesc_s = tc::idesc_bf16(256, 128);
+        constexpr uint32_t idesc_o = tc::idesc_bf16(256, 128, /*b_mn_major=*/true);
+        tc::mbar_wait_sleep(bar_q, 0);
+        const uint64_t dq = tc::sdesc_k_sw128(tc::smem_u32(sQ));
+        const uint64_t dk = tc::sdesc_k_sw128(tc::smem_u32(sK));
+        const uint64_t dv = tc::sdesc_mn_sw128(tc::smem_u32(sV), Cfg::V_HALF);
+        auto issue_s = [&](int j) {                        // S(j) -> TMEM buffer j & 1
+          const int st = j % Cfg::KS;
+          tc::mbar_wait_sleep(&k_full[st], (j / Cfg::KS) & 1);
+          tc::fence_after();
+          tc::mma2_ss_k8<(Cfg::Q_BYTES / 2) / 16, (Cfg::K_HALF / 2) / 16>(
+              (j & 1) * 128, dq, dk + ((st * Cfg::K_HALF) >> 4), idesc_s);
+          tc::mma2_commit_w(&k_empty[st]);
+          tc::mma2_commit_w(&bar_s[j & 1]);
+        };
+        issue_s(0);
+        if (nk > 1) issue_s(1);
+        for (int kt = 0; kt < nk; ++kt) {
+          const int b = kt & 1, st = kt % Cfg::VS;
+          const uint64_t v = dv + ((st * Cfg::V_HALF) >> 4);
+          tc::mbar_wait_sleep(&v_full[st], (kt / Cfg::VS) & 1);
+          ATTN_MMA_WAIT(&bar_p[b], (kt >> 1) & 1);
+          tc::fence_after();
+          tc::mma2_ts_k4(256, b * 128 + 64, v, idesc_o, kt != 0);
+          ATTN_MMA_WAIT(&bar_p2[b], (kt >> 1) & 1);
+          tc::fence_after();
+          tc::mma2_ts_k4(256, b * 128 + 96, v + (4 * 2048 >> 4), idesc_o, 1);
+          tc::mma2_commit_w(&v_empty[st]);
+          tc::mma2_commit_w(bar_pv);
+          if (kt + 1 == nk) tc::mma2_commit_w(bar_o);
+          if (kt + 2 < nk) issue_s(kt + 2);                // into buffer b: after PV(kt) in order
+        }
+      }
+    }
+  } else if (warp < 12) {
+    // ---------------- softmax: warps 4-7 keys 0-63, 8-11 keys 64-127 of each S tile ----------
+    tc::regs_inc<168>();
+    const int q = warp & 3, h = (warp - 4) >> 2;
+    const int row = q * 32 + lane;
+    const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+    const uint32_t leader_p = tc::mapa(tc::smem_u32(h == 0 ? bar_p : bar_p2), 0);
+    float m_used = -INFINITY, l = 0.f;
+    for (int kt = 0; kt < nk; ++kt) {
+      const int b = kt & 1;
+      const uint32_t tS = tmem + lane_off + b * 128;
+      tc::mbar_wait(&bar_s[b], (kt >> 1) & 1);
+      tc::fence_after();
+      float s[64];
+      tc::tmem_ld32(tS + h * 64, reinterpret_cast<uint32_t*>(s));
+      tc::tmem_ld32(tS + h * 64 + 32, reinterpret_cast<uint32_t*>(s + 32));
+      tc::tmem_wait_ld();
+      const int valid = Lr_rem - kt * 128 - h * 64;
+      if (valid < 64) {
+#pragma unroll
+        for (int i = 0; i < 64; ++i) s[i] = (i < valid) ? s[i] : -INFINITY;
+      }
+      float m4[4] = {s[0], s[1], s[2], s[3]};
+#pragma unroll
+      for (int i = 4; i < 60; i += 8)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) m4[j] = tc::fmax3(m4[j], s[i + j], s[i + 4 + j]);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) m4[j] = fmaxf(m4[j], s[60 + j]);
+      const float pm = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3]));
+      sMax[(b * 2 + h) * 128 + row] = pm;
+      named_bar_sync(1 + q, 64);                           // both halves' S loaded, maxima out
+      const float mx = fmaxf(pm, sMax[(b * 2 + (h ^ 1)) * 128 + row]) * scale_log2;
+      float factor = 1.0f;
+      if (mx > m_used + 8.0f) {                            // lazy rescale (threshold 2^8)
+        factor = tc::ex2(m_used - mx);
+        m_used = mx;
+      }
+      if (h == 0) {
+        sScale[b * 128 + row] = factor;
+        __syncwarp();
+        if (lane == 0) tc::mbar_arrive(&bar_stat[b]);
+      }
+      const float nm = -m_used;
+      float a8[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+      for (int c = 0; c < 2; ++c) {
+        uint32_t p[16];
+#pragma unroll
+        for (int i = c * 32; i < c * 32 + 32; i += 2) {
+          tc::ffma2(s[i], s[i + 1], s[i], s[i + 1], scale_log2, scale_log2, nm, nm);
+          if (FPS_ATTN4_POLY > 0 && ((i >> 3) % (FPS_ATTN4_POLY > 0 ? FPS_ATTN4_POLY : 1)) ==
+                                        (FPS_ATTN4_POLY > 0 ? FPS_ATTN4_POLY : 1) - 1) {
+            tc::ex2_poly2(s[i], s[i + 1]);
+          } else {
+            s[i] = tc::ex2(s[i]);
+            s[i + 1] = tc::ex2(s[i + 1]);
+          }
+          p[(i - c * 32) >> 1] = tc::pack_bf16x2_rn(s[i], s[i + 1]);
+        }
+        tc::tmem_st16(tS + 64 + h * 32 + c * 16, p);
+      }
+      tc::tmem_wait_st();
+      tc::fence_before();
+      __syncwarp();
+      if (lane == 0) tc::mbar_arrive_cluster(leader_p + b * 8);
+#pragma unroll
+      for (int i = 0; i < 64; i += 2) {
+        const int j = (i >> 1) & 3;
+        tc::fadd2(a8[2 * j], a8[2 * j + 1], a8[2 * j], a8[2 * j + 1], s[i], s[i + 1]);
+      }
+      l = l * factor + (((a8[0] + a8[1]) + (a8[2] + a8[3])) + ((a8[4] + a8[5]) + (a8[6] + a8[7])));
+    }
+    sL[h * 128 + row] = l;
+    if (nsplit > 1 && h == 0) sM[row] = m_used;            // final statistics: m for ML below
+    __syncwarp();
+    if (lane == 0) tc::mbar_arrive(bar_fin);
+  } else {
+    // ---------------- correction + epilogue (warps 12-15) ----------------
+    tc::regs_dec<88>();
+    const int q = warp & 3;
+    const int row = q * 32 + lane;
+    const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+    const uint32_t leader_p = tc::mapa(tc::smem_u32(bar_p), 0);
+    const uint32_t tO = tmem + 256 + lane_off;
+    for (int kt = 0; kt < nk; ++kt) {
+      const int b = kt & 1;
+      tc::mbar_wait(&bar_stat[b], (kt >> 1) & 1);
+      const float f = sScale[b * 128 + row];
+      if (kt > 0 && __any_sync(0xffffffffu, f != 1.0f)) {
+        tc::mbar_wait(bar_pv, (kt - 1) & 1);               // O(kt-1) complete
+        tc::fence_after();
+#pragma unroll 1
+        for (int c = 0; c < D / 32; ++c) {
+          uint32_t o[32];
+          tc::tmem_ld32(tO + c * 32, o);
+          tc::tmem_wait_ld();
+#pragma unroll
+          for (int e = 0; e < 32; e += 2) {
+            float x0 = __uint_as_float(o[e]), x1 = __uint_as_float(o[e + 1]);
+            tc::ffma2(x0, x1, x0, x1, f, f, 0.f, 0.f);
+            o[e] = __float_as_uint(x0);
+            o[e + 1] = __float_as_uint(x1);
+          }
+          tc::tmem_st32(tO + c * 32, o);
+        }
+        tc::tmem_wait_st();
+      }
+      tc::fence_before();
+      __syncwarp();
+      if (lane == 0) tc::mbar_arrive_cluster(leader_p + b * 8);
+    }
+    const int grow = q0 + row;
+    const int orow_i = (o_map && grow < q_end) ? __ldg(o_map + grow) : grow;
+    __nv_bfloat16* orow = nsplit > 1 ? Opart + split * part_stride + (size_t)grow * (heads * D) + head * D
+                                     : O + (size_t)orow_i * ldo + head * D;
+    if (nk == 0) {
+      if (grow < q_end) {
+        for (int c = 0; c < D; c += 8) *reinterpret_cast<uint4*>(orow + c) = make_uint4(0, 0, 0, 0);
+        if (nsplit > 1) ML[((size_t)split * total_q + grow) * heads + head] = make_float2(-INFINITY, 0.f);
+      }
+    } else {
+      tc::mbar_wait(bar_fin, 0);
+      tc::mbar_wait(bar_o, 0);
+      tc::fence_after();
+      const float l = sL[row] + sL[128 + row];
+      if (nsplit > 1 && grow < q_end)
+        ML[((size_t)split * total_q + grow) * heads + head] = make_float2(sM[row], l);
+      const float inv = (l > 0.f) ? 1.0f / l : 0.f;
+#pragma unroll 1
+      for (int c = 0; c < D / 32; ++c) {
+        uint32_t o[32];
+        tc::tmem_ld32(tO + c * 32, o);
+        tc::tmem_wait_ld();
+        if (grow < q_end) {
+#pragma unroll
+          for (int g = 0; g < 4; ++g) {
+            float f[8];
+#pragma unroll
+            for (int e = 0; e < 8; ++e) f[e] = __uint_as_float(o[g * 8 + e]) * inv;
+            *reinterpret_cast<uint4*>(orow + c * 32 + g * 8) = Vec16<__nv_bfloat16>::pack(f);
+          }
+        }
+      }
+    }
+  }
+  tc::fence_before();
+  __syncthreads();
+  tc::cluster_sync();                                      // both CTAs done with TMEM / barriers
+  if (warp == 2) {
+    tc::fence_after();
+    tc::tmem_dealloc_2sm<Cfg::TMEM_COLS>(tmem);
+  }
+}
+
 // Merge of the split-KV partials: out = sum_z w_z O_z / sum_z w_z, w_z = l_z 2^(m_z - max m).
 // One thread per 8 output columns of one (row, head).
 template <int D>
@@ -1191,6 +1534,51 @@ static fps_status launch_d3(const void* q, const void* kv, void* o, int heads,
   return FPS_OK;
 }
 
+int g_attn_pair = 0;    // 1 = the CTA-pair kernel (attn_tc4) for head_dim 128
+
+static fps_status launch_d4(const void* q, const void* kv, void* o, int heads,
+                            const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
+                            const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo,
+                            const AttnScratch* sc, const int32_t* o_map) {
+  using Cfg = Attn4Cfg;
+  constexpr int D = Cfg::D;
+  const int H = heads * D;
+  int pairs = 0, min_nk = 1 << 30;
+  for (int r = 0; r < n_req; ++r) {
+    const int pr = ((h_cu_q[r + 1] - h_cu_q[r] + 127) / 128 + 1) / 2;
+    pairs += pr;
+    if (pr > 0) min_nk = std::min(min_nk, (h_cu_k[r + 1] - h_cu_k[r] + 127) / 128);
+  }
+  if (pairs == 0) return FPS_OK;
+  const int total_q = h_cu_q[n_req];
+  const int S = choose_split(2 * pairs * heads, min_nk, total_q, H, heads, sc);
+  CUtensorMap tq, tk, tv;
+  if (!make_tmap_2d_bf16(&tq, q, (uint64_t)h_cu_q[n_req], H, (uint64_t)H * 2, 64, 128))
+    return fail(FPS_ECUDA, "attention_tc4: Q tensor map");
+  if (!make_tmap_2d_bf16(&tk, kv, (uint64_t)h_cu_k[n_req], 2 * H, (uint64_t)H * 4, 64, 64) ||
+      !make_tmap_2d_bf16(&tv, kv, (uint64_t)h_cu_k[n_req], 2 * H, (uint64_t)H * 4, 64, 128))
+    return fail(FPS_ECUDA, "attention_tc4: KV tensor maps");
+  FPS_SMEM_ATTR(attn_tc4_kernel, Cfg::SMEM);
+  const float scale_log2 = 1.4426950408889634f / sqrtf((float)D);
+  const long long part_stride = (long long)total_q * H;
+  auto* Opart = S > 1 ? reinterpret_cast<__nv_bfloat16*>(sc->part) : nullptr;
+  auto* ML = S > 1 ? reinterpret_cast<float2*>(sc->ml) : nullptr;
+  FPS_CUDA_TRY(launch_k(attn_tc4_kernel, dim3(2 * pairs, heads, S), dim3(512), Cfg::SMEM, s, tq, tk,
+                        tv, reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads,
+                        scale_log2, ldo, Opart, ML, part_stride, total_q, o_map));
+  if (S > 1) {
+    count_launch();
+    const long long n = (long long)total_q * heads * (D / 8);
+    const int grid = (int)std::min<long long>((n + 255) / 256, kNumSMs * 8LL);
+    FPS_CUDA_TRY(launch_k(attn_combine_kernel<D>, dim3(grid), dim3(256), 0, s,
+                          (const __nv_bfloat16*)Opart, (const float2*)ML, part_stride, S, total_q,
+                          heads, reinterpret_cast<__nv_bfloat16*>(o), ldo, o_map));
+  }
+  count_launch();
+  FPS_LAUNCH_CHECK();
+  return FPS_OK;
+}
+
 fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads, int head_dim,
                                const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
                                const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo,
@@ -1207,6 +1595,8 @@ fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads
   // double-buffered per tile (no S -> softmax -> PV -> S chain) measured 1113 at best: M=128 N=64
   // SS MMAs run at 66% of the tensor rate (48.6 instead of 32 cycles each, tools/micro/mma_rate:
   // A+B operand reads exceed the 128 B/clk smem port), which ate the latency it saved.
+  if (g_attn_force == 0 && g_attn_pair && head_dim == 128)
+    return launch_d4(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo, sc, o_map);
   if (g_attn_force == 0 || g_attn_force == 3) {
     if (head_dim == 128)
       return launch_d3<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo, sc,

@@ -347,6 +347,67 @@ __device__ __forceinline__ void mma_ts_k8(uint32_t d, uint32_t a_tmem, uint64_t 
       "r"(a_tmem), "r"(blo), "r"(bhi), "r"(idesc), "r"(acc)
       : "memory");
 }
+// ---- CTA-pair (cta_group::2) groups for the attention: issued by the leader CTA's MMA warp
+// (warp-wide, one elected lane), M = 256 rows = 128 per CTA, B operand split along N between the
+// two CTAs (same smem offset in each), A from smem (S = Q K^T) or from TMEM (O += P V).
+// SS group, 8 x K=16 (d = 128), no commit; A_CH / B_CH = 64-column chunk strides (16-B units).
+template <int A_CH, int B_CH>
+__device__ __forceinline__ void mma2_ss_k8(uint32_t d, uint64_t adesc, uint64_t bdesc,
+                                           uint32_t idesc) {
+  const uint32_t alo = (uint32_t)adesc, ahi = (uint32_t)(adesc >> 32);
+  const uint32_t blo = (uint32_t)bdesc, bhi = (uint32_t)(bdesc >> 32);
+  asm volatile(
+      "{\n.reg .pred e;\n.reg .b32 al, bl;\n.reg .b64 ad, bd;\n"
+      "elect.sync _|e, 0xffffffff;\n"
+      "mov.b64 ad, {%1, %2};\nmov.b64 bd, {%3, %4};\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], ad, bd, %5, 0;\n"
+      "add.s32 al, %1, 2;\nadd.s32 bl, %3, 2;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "add.s32 al, %1, 4;\nadd.s32 bl, %3, 4;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "add.s32 al, %1, 6;\nadd.s32 bl, %3, 6;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "add.s32 al, %1, %6;\nadd.s32 bl, %3, %7;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "add.s32 al, al, 2;\nadd.s32 bl, bl, 2;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "add.s32 al, al, 2;\nadd.s32 bl, bl, 2;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "add.s32 al, al, 2;\nadd.s32 bl, bl, 2;\nmov.b64 ad, {al, %2};\nmov.b64 bd, {bl, %4};\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], ad, bd, %5, 1;\n"
+      "}\n" ::"r"(d),
+      "r"(alo), "r"(ahi), "r"(blo), "r"(bhi), "r"(idesc), "n"(A_CH), "n"(B_CH)
+      : "memory");
+}
+// TS group, 4 x K=16 (64 keys): A = P from TMEM (8 columns per step, both CTAs' TMEM at the same
+// address), B = V MN-major SW128 (2048 B per 16 keys); acc = 0 only for the first group.
+__device__ __forceinline__ void mma2_ts_k4(uint32_t d, uint32_t a_tmem, uint64_t bdesc,
+                                           uint32_t idesc, uint32_t acc) {
+  const uint32_t blo = (uint32_t)bdesc, bhi = (uint32_t)(bdesc >> 32);
+  asm volatile(
+      "{\n.reg .pred e, p;\n.reg .b32 ta, bl;\n.reg .b64 bd;\n"
+      "elect.sync _|e, 0xffffffff;\n"
+      "setp.ne.b32 p, %5, 0;\n"
+      "mov.b64 bd, {%2, %3};\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], [%1], bd, %4, p;\n"
+      "add.s32 ta, %1, 8;\nadd.s32 bl, %2, 128;\nmov.b64 bd, {bl, %3};\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], [ta], bd, %4, 1;\n"
+      "add.s32 ta, %1, 16;\nadd.s32 bl, %2, 256;\nmov.b64 bd, {bl, %3};\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], [ta], bd, %4, 1;\n"
+      "add.s32 ta, %1, 24;\nadd.s32 bl, %2, 384;\nmov.b64 bd, {bl, %3};\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], [ta], bd, %4, 1;\n"
+      "}\n" ::"r"(d),
+      "r"(a_tmem), "r"(blo), "r"(bhi), "r"(idesc), "r"(acc)
+      : "memory");
+}
+// warp-wide commit of the leader's MMAs to the barrier at this offset in both CTAs
+__device__ __forceinline__ void mma2_commit_w(uint64_t* bar) {
+  asm volatile(
+      "{\n.reg .pred e;\n.reg .b16 m;\nmov.b16 m, 3;\nelect.sync _|e, 0xffffffff;\n"
+      "@e tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64"
+      " [%0], m;\n}\n" ::"r"(smem_u32(bar))
+      : "memory");
+}
 __device__ __forceinline__ void mma_commit(uint64_t* bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
                    smem_u32(bar))

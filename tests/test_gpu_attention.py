@@ -19,7 +19,7 @@ def F():
     return fps
 
 
-KERNEL_FLAGS = {"auto": 0, "p_tmem": 48, "two_tile": 32, "one_tile": 16, "simt": 2}
+KERNEL_FLAGS = {"auto": 0, "pair": 4096, "p_tmem": 48, "two_tile": 32, "one_tile": 16, "simt": 2}
 
 
 @pytest.mark.parametrize("d,heads", [(128, 3), (64, 4)])
@@ -47,7 +47,7 @@ def test_varlen_attention(F, d, heads, kernel):
         ko += l
 
 
-@pytest.mark.parametrize("kernel", ["auto", "p_tmem", "two_tile", "one_tile"])
+@pytest.mark.parametrize("kernel", ["auto", "pair", "p_tmem", "two_tile", "one_tile"])
 def test_attention_large_logits_lazy_rescale(F, kernel):
     """Keys whose scores grow along the sequence force the lazy-max rescale of O in TMEM."""
     g = synth.rng(5)

@@ -260,13 +260,14 @@ def test_c4_continuous_batch_sampled_rows(F, mode):
         check_close(y[cu[i] + sample], ref, TOL["bf16"], f"C4 {mode} request {i}")
 
 
+@pytest.mark.parametrize("pair", [0, 1])
 @pytest.mark.parametrize("mode,split", [("kv", 2), ("kv", 3), ("y", 2), ("kv", 4)])
-def test_split_kv_attention(F, mode, split):
+def test_split_kv_attention(F, mode, split, pair):
     """Split-KV attention (each CTA's key range in S parts, then a combine pass) inside the
     block: heterogeneous varlen batch with ragged key tiles; the parts must merge to the
     oracle's softmax over all keys."""
     w, reqs = _problem(2010 + split, "bf16", 256, 2, 1024, 1500, 36, [0.05, 0.6, 0.3], blobs=False)
-    F.fps_set_disable_tc(split << 8)
+    F.fps_set_disable_tc(split << 8 | pair << 12)      # pair: the CTA-pair kernel (attn_tc4)
     try:
         y, _ = _run_masked(F, w, reqs, 2, "bf16", mode)
     finally:
