@@ -60,7 +60,8 @@ int32_t fps_device_ok(void);
  * (0 = chosen by wave efficiency; S is applied only when the block workspace holds the S
  * partial outputs);
  * bit 11 = the 1-SM tcgen05 GEMM with 4 epilogue warps instead of 8 (A/B experiments);
- * bit 12 = the CTA-pair attention kernel (attn_tc4, head_dim 128). */
+ * bit 12 = the CTA-pair attention kernel (attn_tc4, head_dim 128);
+ * bits 13-14 = 1 / 2 force the 1-SM GEMM's 128- / 256-column tile (A/B experiments). */
 int64_t fps_launch_count(void);
 void fps_set_disable_tc(int32_t flags);
 /* Per-kernel-class timing for the bench: when enabled (this also clears old records) every

@@ -1026,6 +1026,30 @@ __global__ void __launch_bounds__(512, 1)
 #ifndef FPS_ATTN4_POLY
 #define FPS_ATTN4_POLY 4
 #endif
+// the leader's MMA warp waits for P (arrivals from both CTAs) spinning (1) or in the
+// suspend-hinted try_wait (0)
+#ifndef FPS_ATTN4_SPIN
+#define FPS_ATTN4_SPIN 0
+#endif
+// MMA issue split over two warps on two SM sub-partitions (S: warp 1, PV: warp 2) instead of
+// one: a tcgen05.mma issue occupies its sub-partition's dispatch, which the trace showed as the
+// two softmax warps sharing the MMA warp's sub-partition running ~1000 cycles late per tile
+#ifndef FPS_ATTN4_SPLIT
+#define FPS_ATTN4_SPLIT 1
+#endif
+#ifndef FPS_ATTN4_CLUSTER_RELEASE
+#define FPS_ATTN4_CLUSTER_RELEASE 0
+#endif
+#if FPS_ATTN4_CLUSTER_RELEASE
+#define ATTN4_ARRIVE(a) tc::mbar_arrive_cluster(a)
+#else
+#define ATTN4_ARRIVE(a) tc::mbar_arrive_remote(a)
+#endif
+#if FPS_ATTN4_SPIN
+#define ATTN4_MMA_WAIT(bar, par) tc::mbar_wait(bar, par)
+#else
+#define ATTN4_MMA_WAIT(bar, par) tc::mbar_wait_sleep(bar, par)
+#endif
 struct Attn4Cfg {
   static constexpr int D = 128;
   static constexpr int KS = 3, VS = 3;                      // K / V ring depths
@@ -1036,6 +1060,25 @@ struct Attn4Cfg {
   static constexpr int TMEM_COLS = 512;
 };
 
+#ifdef FPS_ATTN_TRACE
+__device__ long long g_attn4_trace[4][64][8];
+#define ATTN4_TRACE(t, kt, slot)                                                    \
+  do {                                                                              \
+    if (blockIdx.x == 2 && blockIdx.y == 3 && (threadIdx.x & 31) == 0 && (kt) < 64) \
+      g_attn4_trace[t][kt][slot] = clock64();                                       \
+  } while (0)
+// every warp of both CTAs of pair 1 / head 3: [rank][warp][kt][slot], %globaltimer-free clock64
+// of each SM (the two SMs' clocks are not aligned: compare within a rank)
+__device__ long long g_attn4_warps[2][16][64][2];
+#define ATTN4_WTRACE(kt, slot)                                                                 \
+  do {                                                                                         \
+    if ((blockIdx.x >> 1) == 1 && blockIdx.y == 3 && (threadIdx.x & 31) == 0 && (kt) < 64)     \
+      g_attn4_warps[blockIdx.x & 1][threadIdx.x >> 5][kt][slot] = clock64();                   \
+  } while (0)
+#else
+#define ATTN4_TRACE(t, kt, slot) do {} while (0)
+#define ATTN4_WTRACE(kt, slot) do {} while (0)
+#endif
 __device__ __forceinline__ void named_bar_sync(int id, int n) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
 }
@@ -1072,7 +1115,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(512, 1)
   uint64_t* bar_pv = bars + 21;            // both: PV(j) complete (multicast)
   uint64_t* bar_o = bars + 22;             // both: last PV complete (multicast)
   uint64_t* bar_fin = bars + 23;           // local: row-sum halves in smem (8 warps)
-  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + 24);
+  uint64_t* pv_iss = bars + 24;            // [buf] leader: PV(j) issued (split issue: S warp waits)
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + 26);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t rank = tc::cluster_ctarank();
@@ -1114,6 +1158,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(512, 1)
     tc::mbar_init(bar_pv, 1);
     tc::mbar_init(bar_o, 1);
     tc::mbar_init(bar_fin, 8);
+    tc::mbar_init(&pv_iss[0], 1);
+    tc::mbar_init(&pv_iss[1], 1);
     tc::fence_mbar_init();
   }
   if (warp == 0 && lane == 0) {
@@ -1158,11 +1204,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(512, 1)
                               k0 + kt * 128);
         }
       }
-    } else if (warp == 1) {
+    } else if (warp == 1 || (FPS_ATTN4_SPLIT && warp == 2)) {
       if (rank == 0 && nk > 0) {
         constexpr uint32_t idesc_s = tc::idesc_bf16(256, 128);
         constexpr uint32_t idesc_o = tc::idesc_bf16(256, 128, /*b_mn_major=*/true);
-        tc::mbar_wait_sleep(bar_q, 0);
         const uint64_t dq = tc::sdesc_k_sw128(tc::smem_u32(sQ));
         const uint64_t dk = tc::sdesc_k_sw128(tc::smem_u32(sK));
         const uint64_t dv = tc::sdesc_mn_sw128(tc::smem_u32(sV), Cfg::V_HALF);
@@ -1175,22 +1220,52 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(512, 1)
           tc::mma2_commit_w(&k_empty[st]);
           tc::mma2_commit_w(&bar_s[j & 1]);
         };
-        issue_s(0);
-        if (nk > 1) issue_s(1);
-        for (int kt = 0; kt < nk; ++kt) {
+        auto issue_pv = [&](int kt) {                      // O += P(kt) V(kt), both halves
           const int b = kt & 1, st = kt % Cfg::VS;
           const uint64_t v = dv + ((st * Cfg::V_HALF) >> 4);
           tc::mbar_wait_sleep(&v_full[st], (kt / Cfg::VS) & 1);
-          ATTN_MMA_WAIT(&bar_p[b], (kt >> 1) & 1);
+          ATTN4_TRACE(2, kt, 0);
+          ATTN4_MMA_WAIT(&bar_p[b], (kt >> 1) & 1);
           tc::fence_after();
+          ATTN4_TRACE(2, kt, 1);
+          ATTN4_WTRACE(kt, 0);
           tc::mma2_ts_k4(256, b * 128 + 64, v, idesc_o, kt != 0);
-          ATTN_MMA_WAIT(&bar_p2[b], (kt >> 1) & 1);
+          ATTN4_MMA_WAIT(&bar_p2[b], (kt >> 1) & 1);
           tc::fence_after();
+          ATTN4_TRACE(2, kt, 2);
+          ATTN4_WTRACE(kt, 1);
           tc::mma2_ts_k4(256, b * 128 + 96, v + (4 * 2048 >> 4), idesc_o, 1);
           tc::mma2_commit_w(&v_empty[st]);
           tc::mma2_commit_w(bar_pv);
           if (kt + 1 == nk) tc::mma2_commit_w(bar_o);
-          if (kt + 2 < nk) issue_s(kt + 2);                // into buffer b: after PV(kt) in order
+        };
+        if (!FPS_ATTN4_SPLIT) {                            // one issuing warp: program order
+          tc::mbar_wait_sleep(bar_q, 0);
+          issue_s(0);
+          if (nk > 1) issue_s(1);
+          for (int kt = 0; kt < nk; ++kt) {
+            issue_pv(kt);
+            if (kt + 2 < nk) issue_s(kt + 2);              // into buffer b: after PV(kt) in order
+            ATTN4_TRACE(2, kt, 3);
+          }
+        } else if (warp == 1) {                            // S issuer
+          tc::mbar_wait_sleep(bar_q, 0);
+          issue_s(0);
+          if (nk > 1) issue_s(1);
+          for (int j = 2; j < nk; ++j) {
+            // buffer j & 1 still holds P(j - 2): issue after PV(j - 2) (same tensor-pipe queue)
+            tc::mbar_wait_sleep(&pv_iss[j & 1], ((j - 2) >> 1) & 1);
+            tc::fence_after();
+            issue_s(j);
+            ATTN4_TRACE(2, j - 2, 3);
+          }
+        } else {                                           // PV issuer (warp 2)
+          for (int kt = 0; kt < nk; ++kt) {
+            issue_pv(kt);
+            tc::fence_before();
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(&pv_iss[kt & 1]);
+          }
         }
       }
     }
@@ -1207,10 +1282,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(512, 1)
       const uint32_t tS = tmem + lane_off + b * 128;
       tc::mbar_wait(&bar_s[b], (kt >> 1) & 1);
       tc::fence_after();
+      if (q == 0) ATTN4_TRACE(h, kt, 0);
       float s[64];
       tc::tmem_ld32(tS + h * 64, reinterpret_cast<uint32_t*>(s));
       tc::tmem_ld32(tS + h * 64 + 32, reinterpret_cast<uint32_t*>(s + 32));
       tc::tmem_wait_ld();
+      if (q == 0) ATTN4_TRACE(h, kt, 1);
       const int valid = Lr_rem - kt * 128 - h * 64;
       if (valid < 64) {
 #pragma unroll
@@ -1226,6 +1303,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(512, 1)
       const float pm = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3]));
       sMax[(b * 2 + h) * 128 + row] = pm;
       named_bar_sync(1 + q, 64);                           // both halves' S loaded, maxima out
+      if (q == 0) ATTN4_TRACE(h, kt, 2);
+      ATTN4_WTRACE(kt, 0);
       const float mx = fmaxf(pm, sMax[(b * 2 + (h ^ 1)) * 128 + row]) * scale_log2;
       float factor = 1.0f;
       if (mx > m_used + 8.0f) {                            // lazy rescale (threshold 2^8)
@@ -1237,7 +1316,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(512, 1)
         __syncwarp();
         if (lane == 0) tc::mbar_arrive(&bar_stat[b]);
       }
-      const float nm = -m_used;
+      // the exponentials below are plain (non-volatile) arithmetic the compiler may hoist above
+      // the arrive, which then only issues near the end of the tile and holds the correction
+      // warps (and PV) back by ~1000 cycles: make them depend on a volatile move after it
+      float nm;
+      asm volatile("mov.b32 %0, %1;" : "=f"(nm) : "f"(-m_used));
       float a8[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
 #pragma unroll
       for (int c = 0; c < 2; ++c) {
@@ -1254,12 +1337,17 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(512, 1)
           }
           p[(i - c * 32) >> 1] = tc::pack_bf16x2_rn(s[i], s[i + 1]);
         }
+        if (c == 1 && q == 0) ATTN4_TRACE(h, kt, 3);
         tc::tmem_st16(tS + 64 + h * 32 + c * 16, p);
       }
       tc::tmem_wait_st();
+      if (q == 0) ATTN4_TRACE(h, kt, 4);
       tc::fence_before();
       __syncwarp();
-      if (lane == 0) tc::mbar_arrive_cluster(leader_p + b * 8);
+      if (q == 0) ATTN4_TRACE(h, kt, 5);
+      if (lane == 0) ATTN4_ARRIVE(leader_p + b * 8);
+      if (q == 0) ATTN4_TRACE(h, kt, 6);
+      ATTN4_WTRACE(kt, 1);
 #pragma unroll
       for (int i = 0; i < 64; i += 2) {
         const int j = (i >> 1) & 3;
@@ -1281,7 +1369,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(512, 1)
     const uint32_t tO = tmem + 256 + lane_off;
     for (int kt = 0; kt < nk; ++kt) {
       const int b = kt & 1;
-      tc::mbar_wait(&bar_stat[b], (kt >> 1) & 1);
+      tc::mbar_wait_sleep(&bar_stat[b], (kt >> 1) & 1);   // off the softmax warps' issue slots
+      if (q == 0) ATTN4_TRACE(3, kt, 0);
+      ATTN4_WTRACE(kt, 0);
       const float f = sScale[b * 128 + row];
       if (kt > 0 && __any_sync(0xffffffffu, f != 1.0f)) {
         tc::mbar_wait(bar_pv, (kt - 1) & 1);               // O(kt-1) complete
@@ -1304,7 +1394,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(512, 1)
       }
       tc::fence_before();
       __syncwarp();
-      if (lane == 0) tc::mbar_arrive_cluster(leader_p + b * 8);
+      if (lane == 0) ATTN4_ARRIVE(leader_p + b * 8);
+      if (q == 0) ATTN4_TRACE(3, kt, 1);
+      ATTN4_WTRACE(kt, 1);
     }
     const int grow = q0 + row;
     const int orow_i = (o_map && grow < q_end) ? __ldg(o_map + grow) : grow;
@@ -1619,5 +1711,11 @@ fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads
 #ifdef FPS_ATTN_TRACE
 extern "C" int fps_debug_attn_trace(long long* out) {
   return (int)cudaMemcpyFromSymbol(out, fps::g_attn_trace, sizeof(fps::g_attn_trace));
+}
+extern "C" int fps_debug_attn4_trace(long long* out) {
+  return (int)cudaMemcpyFromSymbol(out, fps::g_attn4_trace, sizeof(fps::g_attn4_trace));
+}
+extern "C" int fps_debug_attn4_warps(long long* out) {
+  return (int)cudaMemcpyFromSymbol(out, fps::g_attn4_warps, sizeof(fps::g_attn4_warps));
 }
 #endif

@@ -1070,6 +1070,18 @@ static fps_status launch_pair_swap(const void* A, const void* B, int M, int N, i
   return FPS_OK;
 }
 
+int g_gemm_bn = 0;      // tests / A-B: 1 = force the 1-SM kernel's 128-column tile, 2 = 256
+
+// 1-SM tile width: the wave model's per-SM tensor time (waves x BN), ties to the 256 tile.
+// An epilogue-aware tie-break (the 128 tile's last epilogue is half as long) measured worse
+// where it changed the choice: 4916 x 640 x 2560 29.4 vs 20.5 us, 4916 x 640 x 640 11.7 vs
+// 11.0 us (tools/gemm_probe.py, flag bits 13-14) -- with twice the tiles the 128 tile reads the
+// activation panel twice as often and the short-K problems are L2-bound at one wave.
+static bool prefer_bn256(long c256, long c128, int) {
+  if (g_gemm_bn) return g_gemm_bn == 2;
+  return c256 <= c128;
+}
+
 // Activation-block height for the swapped pair kernel: minimise waves x NA (per-SM tensor work
 // of the critical path), ties to the larger NA (fewer tiles, fewer epilogue passes).
 static int swap_block(int M, int N, long* cost) {
@@ -1107,7 +1119,7 @@ fps_status launch_gemm_tc_grouped(const void* A, const void* B0, const void* B1,
   const bool pair_wins = (tp > sm_budget() / 2 && K >= 1024) || cp < cmin;
   if (g_gemm_force == 2 || (g_gemm_force != 1 && pair_wins))
     return launch_pair<6>(A, B0, M0, N, K, ep0, s, g2);
-  if (c256 <= c128) return launch_cfg<256, 4>(A, B0, M0, N, K, ep0, s, g2);
+  if (prefer_bn256(c256, c128, K)) return launch_cfg<256, 4>(A, B0, M0, N, K, ep0, s, g2);
   return launch_cfg<128, 6>(A, B0, M0, N, K, ep0, s, g2);
 }
 
@@ -1146,7 +1158,7 @@ fps_status launch_gemm_tc(const void* A, const void* B, int M, int N, int K, con
   }
   if (g_gemm_force == 2 || (g_gemm_force == 0 && pair_wins))
     return launch_pair<6>(A, B, M, N, K, ep, s);
-  if (c256 <= c128) return launch_cfg<256, 4>(A, B, M, N, K, ep, s);
+  if (prefer_bn256(c256, c128, K)) return launch_cfg<256, 4>(A, B, M, N, K, ep, s);
   return launch_cfg<128, 6>(A, B, M, N, K, ep, s);
 }
 

@@ -99,6 +99,7 @@ extern int g_disable_tc;
 // tests: 0 = choose, 1 = force the 1-SM tcgen05 GEMM, 2 = force the CTA-pair GEMM
 extern int g_gemm_force;
 extern int g_gemm_epi4;
+extern int g_gemm_bn;
 // tests: 0 = two query tiles per CTA (default), 1 = force the one-tile attention kernel
 extern int g_attn_force;
 extern int g_attn_pair;

@@ -126,6 +126,12 @@ __device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
   asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr)
                : "memory");
 }
+// remote arrive with the default (.release.cta) semantics, as CUTLASS's ClusterBarrier::arrive:
+// the payload it publishes (tcgen05 stores, ordered by tcgen05.fence::before_thread_sync) is read
+// by the tensor core, not by the peer's threads, so no cluster-scope release is needed
+__device__ __forceinline__ void mbar_arrive_remote(uint32_t cluster_addr) {
+  asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
 // 2-SM TMA: data lands in the issuing CTA, the transaction bytes count on CTA 0's barrier
 constexpr uint32_t kPeerBitMask = 0xFEFFFFFFu;
 __device__ __forceinline__ void tma_load_2d_2sm(void* smem_dst, const void* desc, uint64_t* bar,
