@@ -59,7 +59,7 @@ int32_t fps_device_ok(void);
  * bits 8-10 = S > 0 forces the split-KV factor of the tensor-core attention inside block calls
  * (0 = chosen by wave efficiency; S is applied only when the block workspace holds the S
  * partial outputs);
- * bit 11 = the 1-SM tcgen05 GEMM with 4 epilogue warps instead of 8 (A/B experiments);
+ * bit 11 = the tcgen05 GEMMs (1-SM and CTA-pair) with 4 epilogue warps instead of 8 (A/B);
  * bit 12 = the CTA-pair attention kernel (attn_tc4, head_dim 128);
  * bits 13-14 = 1 / 2 force the 1-SM GEMM's 128- / 256-column tile (A/B experiments). */
 int64_t fps_launch_count(void);

@@ -213,7 +213,6 @@ __device__ __forceinline__ unsigned long long gtimer() {
 // Layout: 32 rows x 64 B per warp; piece p (16 B) of row r at r * 64 + ((p ^ (r >> 1 & 3)) << 4)
 // (conflict-free for both the row-per-lane writes and the 4-lanes-per-row reads).
 constexpr int kXsWarpBytes = 32 * 64;
-constexpr int kXsBytes = 4 * kXsWarpBytes;      // pair kernels: 4 epilogue warps per CTA
 
 __device__ __forceinline__ uint32_t xs_off(int r, int p) { return r * 64 + ((p ^ ((r >> 1) & 3)) << 4); }
 
@@ -674,22 +673,26 @@ namespace fps {
 
 // ============================================================================================
 // CTA-pair kernel (cta_group::2): 256 x 256 tile per pair
-template <int STAGES>
+// EPI epilogue warps per CTA: 4 or 8 (two per TMEM lane quarter, 128 columns each), as the
+// 1-SM kernel; the epilogue of the last wave's tiles is exposed
+template <int STAGES, int EPI = 4>
 struct Gemm2Cfg {
   static constexpr int BM = 256, BN = 256, BK = 64;        // per pair
   static constexpr int A_BYTES = 128 * BK * 2;             // per CTA: its 128 rows of A
   static constexpr int B_BYTES = 128 * BK * 2;             // per CTA: its 128 rows of B
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
   static constexpr int TMEM_COLS = 512;                    // 2 accumulators x 256 columns
-  static constexpr int SMEM = STAGES * STAGE_BYTES + kXsBytes + 1024 + 256;
+  static constexpr int XS_BYTES = EPI * kXsWarpBytes;
+  static constexpr int THREADS = 128 + 32 * EPI;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + XS_BYTES + 1024 + 256;
 };
 
-template <int STAGES>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
+template <int STAGES, int EPI>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Gemm2Cfg<STAGES, EPI>::THREADS, 1)
     gemm_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     const __grid_constant__ CUtensorMap tmB1, int M, int N, int K, Epilogue ep,
                     int M1, Epilogue ep1) {
-  using Cfg = Gemm2Cfg<STAGES>;
+  using Cfg = Gemm2Cfg<STAGES, EPI>;
   constexpr int kGroupM = 8;                               // 2048 rows of A per group
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
@@ -697,7 +700,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
   uint8_t* sA = smem;
   uint8_t* sB = smem + STAGES * Cfg::A_BYTES;
   uint8_t* sXs = smem + STAGES * Cfg::STAGE_BYTES;           // epilogue transpose staging
-  uint64_t* full = reinterpret_cast<uint64_t*>(sXs + kXsBytes);
+  uint64_t* full = reinterpret_cast<uint64_t*>(sXs + Cfg::XS_BYTES);
   uint64_t* empty = full + STAGES;
   uint64_t* tfull = empty + STAGES;
   uint64_t* tempty = tfull + 2;
@@ -720,7 +723,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
     }
     for (int a = 0; a < 2; ++a) {
       tc::mbar_init(&tfull[a], 1);                         // both: multicast commit
-      tc::mbar_init(&tempty[a], 8);                        // leader: 4 epilogue warps x 2 CTAs
+      tc::mbar_init(&tempty[a], 2 * EPI);                  // leader: EPI epilogue warps x 2 CTAs
     }
     tc::fence_mbar_init();
   }
@@ -738,6 +741,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
   pdl_trigger();   // setup done: let the next kernel's CTAs start as ours retire
   pdl_wait();      // inputs of this GEMM come from the previous kernel
 
+  if (EPI == 8 && warp < 4) tc::regs_dec<72>();
   if (warp == 0) {
     if (lane == 0) {
       int stage = 0;
@@ -790,7 +794,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
       }
     }
   } else if (warp >= 4) {
+    if (EPI == 8) tc::regs_inc<216>();
     const int q = warp & 3;
+    constexpr int CW = 256 * 4 / EPI;                      // columns per epilogue warp
+    const int h = (warp - 4) >> 2;
     const uint32_t tempty_leader = tc::mapa(tc::smem_u32(tempty), 0);
     int it = 0;
     for (int tile = pair; tile < num_tiles; tile += num_pairs, ++it) {
@@ -799,10 +806,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
       const int acc = it & 1;
       tc::mbar_wait(&tfull[acc], (it >> 1) & 1);
       tc::fence_after();
-      epilogue_tile<256>(p ? ep1 : ep, p ? M1 : M, N,
-                         m_blk * Cfg::BM + rank * 128 + q * 32 + lane, n_blk * Cfg::BN,
-                         tmem_base + ((uint32_t)(q * 32) << 16) + acc * 256,
-                         sXs + q * kXsWarpBytes);
+      epilogue_tile<CW>(p ? ep1 : ep, p ? M1 : M, N,
+                        m_blk * Cfg::BM + rank * 128 + q * 32 + lane, n_blk * Cfg::BN + h * CW,
+                        tmem_base + ((uint32_t)(q * 32) << 16) + acc * 256 + h * CW,
+                        sXs + (warp - 4) * kXsWarpBytes);
       tc::fence_before();
       __syncwarp();
       if (lane == 0) tc::mbar_arrive_cluster(tempty_leader + acc * 8);
@@ -1003,7 +1010,7 @@ struct Group2 {
   Epilogue ep1;
 };
 
-int g_gemm_epi4 = 0;    // tests / A-B: 1 = the 1-SM kernel with 4 epilogue warps instead of 8
+int g_gemm_epi4 = 0;    // tests / A-B: 1 = 4 epilogue warps instead of 8 (1-SM and pair kernels)
 
 template <int BN, int STAGES, int EPI>
 static fps_status launch_cfg_e(const void* A, const void* B, int M, int N, int K,
@@ -1032,24 +1039,31 @@ static fps_status launch_cfg(const void* A, const void* B, int M, int N, int K,
   return launch_cfg_e<BN, STAGES, 8>(A, B, M, N, K, ep, s, g2);
 }
 
-template <int STAGES>
-static fps_status launch_pair(const void* A, const void* B, int M, int N, int K,
-                              const Epilogue& ep, cudaStream_t s, const Group2& g2 = Group2{}) {
-  using Cfg = Gemm2Cfg<STAGES>;
+template <int STAGES, int EPI>
+static fps_status launch_pair_e(const void* A, const void* B, int M, int N, int K,
+                                const Epilogue& ep, cudaStream_t s, const Group2& g2) {
+  using Cfg = Gemm2Cfg<STAGES, EPI>;
   CUtensorMap ta, tb, tb1;
   if (!make_tmap_2d_bf16(&ta, A, M + g2.M1, K, (uint64_t)K * 2, Cfg::BK, 128) ||
       !make_tmap_2d_bf16(&tb, B, N, K, (uint64_t)K * 2, Cfg::BK, 128) ||
       (g2.M1 > 0 && !make_tmap_2d_bf16(&tb1, g2.B1, N, K, (uint64_t)K * 2, Cfg::BK, 128)))
     return fail(FPS_ECUDA, "gemm_tc2: cuTensorMapEncodeTiled failed (M=%d N=%d K=%d)", M, N, K);
   if (g2.M1 == 0) tb1 = tb;
-  FPS_SMEM_ATTR((gemm_tc2_kernel<STAGES>), Cfg::SMEM);
+  FPS_SMEM_ATTR((gemm_tc2_kernel<STAGES, EPI>), Cfg::SMEM);
   const int tiles = (ceil_div(M, Cfg::BM) + ceil_div(g2.M1, Cfg::BM)) * ceil_div(N, Cfg::BN);
   const int pairs = tiles < sm_budget() / 2 ? tiles : sm_budget() / 2;
-  FPS_CUDA_TRY(launch_k(gemm_tc2_kernel<STAGES>, dim3(2 * pairs), dim3(256), Cfg::SMEM, s, ta, tb,
-                        tb1, M, N, K, ep, g2.M1, g2.ep1));
+  FPS_CUDA_TRY(launch_k(gemm_tc2_kernel<STAGES, EPI>, dim3(2 * pairs), dim3(Cfg::THREADS), Cfg::SMEM,
+                        s, ta, tb, tb1, M, N, K, ep, g2.M1, g2.ep1));
   count_launch();
   FPS_LAUNCH_CHECK();
   return FPS_OK;
+}
+
+template <int STAGES>
+static fps_status launch_pair(const void* A, const void* B, int M, int N, int K,
+                              const Epilogue& ep, cudaStream_t s, const Group2& g2 = Group2{}) {
+  if (g_gemm_epi4) return launch_pair_e<STAGES, 4>(A, B, M, N, K, ep, s, g2);
+  return launch_pair_e<STAGES, 8>(A, B, M, N, K, ep, s, g2);
 }
 
 template <int STAGES>

@@ -22,13 +22,13 @@ def F():
                                    (1331, 3072, 12288), (409, 1920, 640), (2048, 2560, 1280),
                                    (300, 640, 2560), (4608, 3072, 3072)])
 @pytest.mark.parametrize("act", [0, 1])
-@pytest.mark.parametrize("kernel", ["auto", "1sm", "1sm_epi4", "pair", "swap"])
+@pytest.mark.parametrize("kernel", ["auto", "1sm", "1sm_epi4", "pair", "pair_epi4", "swap"])
 def test_linear_bf16(F, M, N, K, act, kernel):
     g = synth.rng(M * 7 + N + K + act)
     a = synth.latent(g, M, K, "bf16")
     w = synth.bf16_round(g.standard_normal((N, K), dtype=np.float32) / np.sqrt(K))
     b = synth.bf16_round(0.1 * g.standard_normal(N, dtype=np.float32))
-    F.fps_set_disable_tc({"auto": 0, "1sm": 4, "1sm_epi4": 4 | 2048, "pair": 8, "swap": 12}[kernel])
+    F.fps_set_disable_tc({"auto": 0, "1sm": 4, "1sm_epi4": 4 | 2048, "pair": 8, "pair_epi4": 8 | 2048, "swap": 12}[kernel])
     try:
         out = F.linear(to_dev(a, "bf16"), to_dev(w, "bf16"), to_dev(b, "bf16"), act=act)
         torch.cuda.synchronize()
