@@ -39,7 +39,11 @@ WORKLOADS = {
                batch=1, layers=57, steps=28, desc="Flux-scale DiT stack, 20% mask, batch 1"),
     "C4": dict(H=3072, heads=24, F=12288, L_img=4096, L_txt=512, grid=(64, 64),
                ratios=list(np.linspace(0.05, 0.60, 16)), batch=16, layers=57, steps=28,
-               desc="continuous batch of 16 heterogeneous masks (5-60%), Flux-scale"),
+               desc="continuous batch of 16 heterogeneous masks (5-60%), Flux-scale",
+               # H2D default (profiles/r02/c4_h2d/): whole entries move 1.48x the unmasked bytes
+               # here (mean m 0.33), so the exact-row TMA gather on 8 reserved SMs wins (525 vs
+               # 614 ms/step); at C3 (1.25x) the reserved SMs cost more than the bytes saved
+               copy_method=3, copy_ctas=8),
     "C2B": dict(H=1280, heads=20, F=5120, L_img=1024, L_txt=0, grid=(32, 32),
                 ratios=[0.1, 0.3, 0.5, 0.3], batch=4, layers=60, steps=50,
                 desc="SDXL-scale 32x32 level (1280 ch), masks 10/30/50%, batch 4"),
@@ -149,6 +153,7 @@ def route_job(pool, w, world, rank, cm):
 
 
 COPY_CTAS = 0
+LOAD_PRIORITY = 0     # CUDA priority of the cache-load streams (--load-priority)
 # Timing the calibration blocks under concurrent loads was tried: the noisier fit (R^2 0.84)
 # over-weights the intercept, the planner caches too many blocks and the step gets slower
 # (49.9 vs 43.0 ms on C3), so the models are fitted on isolated timings (as the paper does).
@@ -305,7 +310,7 @@ def _calibrate_one(F, w, mode, layers, cache, reqs, device, first=0):
     h_ld_rows = np.arange(w["L_img"], dtype=np.int32)
     ld_items = [F.fps_prefetch_item(i, 0, 0, w["L_img"], ld_rows.data_ptr(), h_ld_rows.ctypes.data,
                                     ld_dst[i * L].data_ptr(), Wl * 2) for i in range(B)]
-    ld_stream = torch.cuda.Stream(device=device)
+    ld_stream = torch.cuda.Stream(device=device, priority=LOAD_PRIORITY)
     kind = w.get("block", "seq")
     kind = "double" if kind == "flux" else kind         # FLOPs per row: double == seq == par
     Lc = SDXL_CTX[0] if kind == "sdxl" else 0
@@ -352,7 +357,7 @@ def _calibrate_one(F, w, mode, layers, cache, reqs, device, first=0):
     # loads: rows of one layer for the batch at several unmasked counts
     W = (2 if mode == "kv" else 1) * H
     dst = torch.empty(B * L, W, dtype=torch.bfloat16, device=device)
-    ls = torch.cuda.Stream(device=device)
+    ls = torch.cuda.Stream(device=device, priority=LOAD_PRIORITY)
     whole = cache.desc.copy_method == 2
     for k, m in enumerate((0.05, 0.3, 0.6, 0.9)):
         u = w["L_img"] - synth.n_masked_for(m, w["L_img"])
@@ -504,6 +509,11 @@ def main():
     ap.add_argument("--copy-method", type=int, default=None, choices=[0, 1, 2, 3],
                     help="H2D method: 0 SM zero-copy row gather, 1 one DMA per unmasked row run, "
                          "2 whole-entry DMA, 3 TMA bulk row gather on reserved SMs")
+    ap.add_argument("--load-priority", type=int, default=None,
+                    help="CUDA priority of the cache-load stream (lower = higher; 0 = the compute "
+                         "stream's). Default: highest (-5) with the TMA row gather (method 3), whose "
+                         "CTAs then take the reserved SMs ahead of queued compute CTAs (C4: 525 "
+                         "vs 548 ms/step), else 0")
     ap.add_argument("--cross-step", type=int, default=1, choices=[0, 1],
                     help="cross-step prefetch (R26): the next step's loads start as soon as their "
                          "slots are consumed (1, default), or the per-step pipeline of Fig. 9 (0)")
@@ -539,11 +549,19 @@ def main():
     import signal
     faulthandler.dump_traceback_later(int(os.environ.get("FPS_BENCH_TIMEOUT", 900)), exit=True)
     faulthandler.register(signal.SIGUSR1, all_threads=True)   # `timeout -s USR1`: dump stacks
+    global LOAD_PRIORITY
     if args.copy_method is None:
         # measured on B200 (C3, profiles/r01f5_*): pinned host tier -- whole-entry DMA 34.6
         # ms/step vs 36.2 with one DMA per unmasked row run (~200 us of host time per entry) and
-        # 48.5 with the SM row gather (SM interference); HBM tier -- whole-entry DMA 21.2
-        args.copy_method = 2
+        # 48.5 with the SM row gather (SM interference); HBM tier -- whole-entry DMA 21.2.
+        # C4 (pinned host): the TMA row gather (WORKLOADS["C4"])
+        wl = WORKLOADS[args.config]
+        args.copy_method = wl.get("copy_method", 2) if args.tier != "hbm" else 2
+        if args.copy_method == 3 and args.copy_ctas == 0:
+            args.copy_ctas = wl.get("copy_ctas", 0)
+    if args.load_priority is None:
+        args.load_priority = -5 if args.copy_method == 3 else 0
+    LOAD_PRIORITY = args.load_priority
 
     rank = int(os.environ.get("RANK", 0))
     world = int(os.environ.get("WORLD_SIZE", 1))
@@ -573,6 +591,10 @@ def main():
                    if args.config == "C3" else f"masked-block stack images/s ({args.config})")
     base_cfg["cache_tier"] = TIER_NAMES[args.tier]
     base_cfg["h2d_method"] = H2D_NAMES[args.copy_method]
+    if args.copy_method == 3:
+        base_cfg["h2d_reserved_sms"] = args.copy_ctas or 4
+    if args.load_priority:
+        base_cfg["load_stream_priority"] = args.load_priority
     base_cfg["parallelism"] = f"request-parallel x{world} (Alg. 2 routing)"
     base_cfg["cross_step_prefetch"] = bool(args.cross_step)
     base_cfg["kv_transition_block"] = bool(args.kv_transition) and args.mode == "kv"
@@ -690,7 +712,7 @@ def main():
             reqs_dev[-1]["z"] = torch.randn(w["L_img"], w["H"], generator=g, device=device).to(torch.bfloat16)
             reqs_dev[-1]["noise"] = torch.randn(w["L_img"], w["H"], generator=g, device=device).to(torch.bfloat16)
     stream = torch.cuda.current_stream()
-    load_stream = torch.cuda.Stream(device=device)
+    load_stream = torch.cuda.Stream(device=device, priority=LOAD_PRIORITY)
     deltas = synth.delta_table(w["steps"])
 
     sigmas = None

@@ -155,10 +155,15 @@ typedef struct {
                                 -> HBM by cp.async.bulk from copy_ctas CTAs (default 4, in
                                 TPC pairs) at ~51 GB/s of useful bytes; fps_run_batch with a
                                 load stream sizes its compute grids to the other SMs.  Pinned
-                                host tiers only need it; rows <= 32 KB                       */
+                                host tiers only need it; rows <= 32 KB.  Give the load stream
+                                a high CUDA priority: its gather CTAs then take the reserved
+                                SMs ahead of queued compute CTAs (non-persistent grids, PDL
+                                early launches).  Inside a step 6-8 CTAs keep the link busy
+                                (bench default at configs[3], where whole entries would move
+                                1.48x the unmasked bytes)                                    */
   int32_t copy_ctas;     /* CTAs used by method 0 (0 = default: 16 for the host link -- enough
                             for PCIe, few enough not to crowd out the compute stream -- and 64
-                            for the HBM tier) and by method 3 (0 = 4)                        */
+                            for the HBM tier) and by method 3 (0 = 4; even)                        */
   int32_t location;      /* 0 = pinned host DRAM (L203, streamed over PCIe);
                             1 = device HBM: the template tier one level above host DRAM
                             (the paper's "ideal" no-load case of Fig. 4-Left,

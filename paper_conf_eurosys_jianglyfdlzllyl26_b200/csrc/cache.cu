@@ -102,9 +102,11 @@ __global__ void __launch_bounds__(256) prefetch_kernel(const __grid_constant__ P
 constexpr int kBulkMaxSlots = 16;
 constexpr int kBulkMinChunk = 12288;   // bytes per ring slot (at least one row)
 constexpr int kBulkMaxRow = 32768;     // widest row method 3 accepts (KV-mode H <= 8192 bf16)
-// bytes in flight over all CTAs: PCIe read latency ~2 us x ~55 GB/s needs > 110 KB; the
-// micro reached the link rate from 128 KB (e.g. 16 x 8 KB, 8 x 16 KB, 4 x 48 KB)
-constexpr int kBulkInFlight = 192 * 1024;
+// bytes in flight per CTA: PCIe read latency ~2 us x ~55 GB/s needs > 110 KB over all CTAs; the
+// micro reached the link rate from 128 KB (e.g. 16 x 8 KB, 8 x 16 KB, 4 x 48 KB).  Inside the
+// C4 step the link needs 6-8 CTAs (C4: 4 CTAs 603 ms/step, 6 527, 8 524, 12 536) and a deeper
+// ring per CTA does not help (8 CTAs: 48 KB 523.5, 96 KB 525.0, 192 KB 529.8 ms/step)
+constexpr int kBulkInFlightPerCta = 48 * 1024;
 constexpr int kBulkMaxSmem = 200 * 1024;
 constexpr int kBulkHeader = 512;   // barriers, row ids, pending stores (kBulkMaxSlots = 16)
 
@@ -511,8 +513,14 @@ fps_status fps_cache_prefetch(fps_cache_t c, const fps_prefetch_item* items, int
     for (int i = 0; i < n_items; ++i) max_rb = std::max(max_rb, (int)row_bytes_of(c, items[i].layer));
     const int slot_bytes = std::max(kBulkMinChunk, max_rb);
     const int ctas = bulk_ctas(c);
+    static int inflight_env = -1;     // FPS_BULK_INFLIGHT: bytes over all CTAs (experiments)
+    if (inflight_env < 0) {
+      const char* v = getenv("FPS_BULK_INFLIGHT");
+      inflight_env = v ? std::max(1, atoi(v)) : 0;
+    }
+    const int inflight = inflight_env > 0 ? inflight_env : kBulkInFlightPerCta * ctas;
     const int slots = std::max(2, std::min({kBulkMaxSlots, (kBulkMaxSmem - kBulkHeader) / slot_bytes,
-                                             (kBulkInFlight + ctas * slot_bytes - 1) / (ctas * slot_bytes)}));
+                                             (inflight + ctas * slot_bytes - 1) / (ctas * slot_bytes)}));
     const int smem = kBulkHeader + slots * slot_bytes;
     FPS_SMEM_ATTR(bulk_gather_kernel, kBulkMaxSmem);
     for (int base = 0; base < n_items; base += kMaxPrefetchItems) {

@@ -43,7 +43,9 @@ def main():
                          x=torch.randn(L, w["H"], generator=g, device=dev).to(torch.bfloat16)))
         if L_ctx:
             reqs[-1]["ctx"] = torch.randn(*bench.SDXL_CTX, generator=g, device=dev).to(torch.bfloat16)
-    stream, ls = torch.cuda.current_stream(), torch.cuda.Stream(device=dev)
+    # PROBE_LOAD_PRIO: priority of the load stream (lower = higher; torch range [-3, 0] or so)
+    prio = int(os.environ.get("PROBE_LOAD_PRIO", 0))
+    stream, ls = torch.cuda.current_stream(), torch.cuda.Stream(device=dev, priority=prio)
     deltas = synth.delta_table(w["steps"])
     out = []
     for me in methods:
