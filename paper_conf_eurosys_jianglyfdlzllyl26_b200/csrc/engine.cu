@@ -87,6 +87,7 @@ struct fps_engine {
   bool no_reuse = false;   // experiments: admit every call
   bool no_transition = false;   // experiments: run a KV-mode plan's last dense block densely
   bool skip_loads = false;      // measurement: no cache loads, slots keep their last contents
+  int sm_reserve_call = 0;      // SMs the call keeps for the TMA row gather (method 3)
   bool record = false;          // template run: store the K|V / Y rows of every dense block
   // flow-blend sampler: per-request (template latent, noise) pointers and step coefficients
   void** h_zeps = nullptr;
@@ -577,6 +578,10 @@ static fps_status run_step(fps_engine* e, fps_request* reqs, Batch& B, cudaStrea
     }
   const int n_ring = (int)loads.size();
   const bool final_load = kv && n_ring > 0;
+  // the gather's SMs are kept only in steps that load: a plan without cached blocks (the dense
+  // reference) and the no-load arm compute on every SM, so the reservation's compute cost
+  // counts as load cost in the exposed-load measurement
+  g_sm_reserved = (n_ring > 0 && !e->skip_loads) ? e->sm_reserve_call : 0;
   std::vector<char> consumed_rec(n_ring + 1, 0);
   int issued = 0;
   bool final_issued = false;
@@ -827,6 +832,7 @@ extern "C" fps_status fps_run_batch(fps_engine_t e, fps_request* reqs, int32_t n
     explicit SmReserve(int n) : prev(g_sm_reserved) { g_sm_reserved = n; }
     ~SmReserve() { g_sm_reserved = prev; }
   } reserve(load_stream ? reserved_sms(e->d.cache) : 0);
+  e->sm_reserve_call = g_sm_reserved;
   e->call_start = true;
   int done_steps = 0;
   while (done_steps < n_steps) {

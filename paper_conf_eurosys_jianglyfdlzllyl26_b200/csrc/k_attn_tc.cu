@@ -654,7 +654,7 @@ __device__ __forceinline__ constexpr bool attn_poly(int i) {
 __device__ long long g_attn_trace[2][64][8];
 #define ATTN_TRACE(t, kt, slot)                                                     \
   do {                                                                              \
-    if (blockIdx.x == 2 && blockIdx.y == 3 && (threadIdx.x & 31) == 0 && (kt) < 64) \
+    if (blockIdx.x == 3 && blockIdx.y == 2 && (threadIdx.x & 31) == 0 && (kt) < 64) \
       g_attn_trace[t][kt][slot] = clock64();                                        \
   } while (0)
 #else
@@ -703,9 +703,13 @@ __global__ void __launch_bounds__(512, 1)
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + 21);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int head = blockIdx.y;
+  // grid (heads, query-tile pairs, splits): heads vary fastest, so the CTAs the block scheduler
+  // places last are the highest pair index -- for a single request its odd last tile, a short
+  // CTA -- and a grid a few CTAs over the SMs left beside the method-3 gather (sm_budget())
+  // costs one short CTA, not a second full-length wave
+  const int head = blockIdx.x;
   const int H = heads * D;
-  int r = 0, qp = blockIdx.x, ntile = 0;
+  int r = 0, qp = blockIdx.y, ntile = 0;
   for (; r < n_req; ++r) {
     ntile = (__ldg(cu_q + r + 1) - __ldg(cu_q + r) + 127) >> 7;
     const int np = (ntile + 1) >> 1;
@@ -1596,7 +1600,7 @@ static fps_status launch_d3(const void* q, const void* kv, void* o, int heads,
   const long long part_stride = (long long)total_q * H;
   auto* Opart = S > 1 ? reinterpret_cast<__nv_bfloat16*>(sc->part) : nullptr;
   auto* ML = S > 1 ? reinterpret_cast<float2*>(sc->ml) : nullptr;
-  FPS_CUDA_TRY(launch_k(attn_tc3_kernel<D>, dim3(pairs, heads, S), dim3(512), Cfg::SMEM, s, tq, tkv,
+  FPS_CUDA_TRY(launch_k(attn_tc3_kernel<D>, dim3(heads, pairs, S), dim3(512), Cfg::SMEM, s, tq, tkv,
                         reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads,
                         scale_log2, ldo, Opart, ML, part_stride, total_q, o_map));
   if (S > 1) {

@@ -1130,7 +1130,8 @@ fps_status launch_gemm_tc_grouped(const void* A, const void* B0, const void* B1,
   const long c128 = ((t128 + sm_budget() - 1) / sm_budget()) * 128;
   const long cp = ((tp + sm_budget() / 2 - 1) / (sm_budget() / 2)) * 256;
   const long cmin = std::min(c256, c128);
-  const bool pair_wins = (tp > sm_budget() / 2 && K >= 1024) || cp < cmin;
+  const long pair_multi = g_sm_reserved > 0 ? 2L * (sm_budget() / 2) : sm_budget() / 2;
+  const bool pair_wins = (tp > pair_multi && K >= 1024) || cp < cmin;
   if (g_gemm_force == 2 || (g_gemm_force != 1 && pair_wins))
     return launch_pair<6>(A, B0, M0, N, K, ep0, s, g2);
   if (prefer_bn256(c256, c128, K)) return launch_cfg<256, 4>(A, B0, M0, N, K, ep0, s, g2);
@@ -1160,7 +1161,11 @@ fps_status launch_gemm_tc(const void* A, const void* B, int M, int N, int K, con
   // short K (< 1024, the SDXL-scale projections at C = 640): the pair's longer prologue and
   // epilogue are not amortised even over several waves (4916x1920x640: 30.2 vs 23.3 us for the
   // 1-SM kernel; 4916x5120x640: 54.8 vs 52.9; 16384x1920x640: 64.7 vs 61.3; K >= 1280: ties)
-  const bool pair_wins = (tp > sm_budget() / 2 && K >= 1024) || cp < cmin ||
+  // with SMs reserved for the method-3 gather (sm_budget() < 148) a problem just over one pair
+  // wave (C3's W2: 72 pair tiles on 70 pairs) would take two; there the pair kernel's L2
+  // advantage must span at least two full waves to outweigh the wave model
+  const long pair_multi = g_sm_reserved > 0 ? 2L * (sm_budget() / 2) : sm_budget() / 2;
+  const bool pair_wins = (tp > pair_multi && K >= 1024) || cp < cmin ||
                          (cp == cmin && (m2 * 256 - M < 128 || K >= 8192));
   // swapped operands (activation rows on the MMA's N side, no 256-row M padding): correct and
   // tested, but measured no faster at the masked-block shapes (1331x9216x3072: 59.8 vs 59.2 us
