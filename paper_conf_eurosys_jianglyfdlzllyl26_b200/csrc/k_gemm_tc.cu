@@ -1131,7 +1131,16 @@ fps_status launch_gemm_tc_grouped(const void* A, const void* B0, const void* B1,
   const long cp = ((tp + sm_budget() / 2 - 1) / (sm_budget() / 2)) * 256;
   const long cmin = std::min(c256, c128);
   const long pair_multi = g_sm_reserved > 0 ? 2L * (sm_budget() / 2) : sm_budget() / 2;
-  const bool pair_wins = (tp > pair_multi && K >= 1024) || cp < cmin;
+  // a tie in the wave model goes to the pair kernel (FPS_GROUPED_TIE overrides: 0 never, 1 at
+  // K >= 8192, 2 always): the double-stream block's O and down projections at C3's masked size
+  // (819 image + 512 text rows, 72 pair tiles) run one pair wave instead of 132 1-SM tiles --
+  // Y-mode C3 step 27.40 -> 27.03 ms (mean of 2 runs each, profiles/r02/grouped_tie.txt)
+  static const int tie = [] {
+    const char* v = getenv("FPS_GROUPED_TIE");
+    return v ? atoi(v) : 2;
+  }();
+  const bool pair_wins = (tp > pair_multi && K >= 1024) || cp < cmin ||
+                         (cp == cmin && (tie == 2 || (tie == 1 && K >= 8192)));
   if (g_gemm_force == 2 || (g_gemm_force != 1 && pair_wins))
     return launch_pair<6>(A, B0, M0, N, K, ep0, s, g2);
   if (prefer_bn256(c256, c128, K)) return launch_cfg<256, 4>(A, B0, M0, N, K, ep0, s, g2);
