@@ -96,19 +96,22 @@ fps_status launch_gemm(int dtype, const void* A, const void* B, int M, int N, in
 
 fps_status launch_gemm_grouped(int dtype, const void* A, const void* B0, const void* B1, int M0,
                                int M1, int N, int K, const Epilogue& ep0, const Epilogue& ep1,
-                               cudaStream_t s) {
+                               cudaStream_t s, int N1) {
+  if (N1 <= 0) N1 = N;
   if (M1 <= 0) return launch_gemm(dtype, A, B0, M0, N, K, ep0, s);
   if (M0 <= 0) return launch_gemm(dtype, (const char*)A + (size_t)M0 * K * elt_size(dtype), B1, M1,
-                                  N, K, ep1, s);
-  if ((g_disable_tc & 1) || !gemm_tc_supported(dtype, M0 + M1, N, K)) {
+                                  N1, K, ep1, s);
+  if ((g_disable_tc & 1) || !gemm_tc_supported(dtype, M0 + M1, N, K) ||
+      !gemm_tc_supported(dtype, M0 + M1, N1, K)) {
     FPS_TRY(launch_gemm(dtype, A, B0, M0, N, K, ep0, s));
-    return launch_gemm(dtype, (const char*)A + (size_t)M0 * K * elt_size(dtype), B1, M1, N, K, ep1,
-                       s);
+    return launch_gemm(dtype, (const char*)A + (size_t)M0 * K * elt_size(dtype), B1, M1, N1, K,
+                       ep1, s);
   }
   prof::begin(s);
-  fps_status st = launch_gemm_tc_grouped(A, B0, B1, M0, M1, N, K, ep0, ep1, s);
+  fps_status st = launch_gemm_tc_grouped(A, B0, B1, M0, M1, N, K, ep0, ep1, s, N1);
   const double e = elt_size(dtype), M = (double)M0 + M1;
-  prof::end(s, prof::GEMM, 2.0 * M * N * K, e * (M * K + 2.0 * N * K + M * N));
+  const double MN = (double)M0 * N + (double)M1 * N1;
+  prof::end(s, prof::GEMM, 2.0 * MN * K, e * (M * K + (double)(N + N1) * K + MN));
   return st;
 }
 
@@ -409,9 +412,19 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
     FPS_TRY(launch_gemm(dt, ws.hu, (const char*)w->w_qkv + (size_t)H * H * e, b->total_k, 2 * H, H,
                         ek, s));
   }
+  // Y-mode parallel block: the W1 GEMM of rows M ([Q|K|V|Z]) and the K|V GEMM of the cached
+  // rows U in ONE grouped launch (A = both rows' LN outputs, stacked in ws.hu): the persistent
+  // grid runs both problems' tiles back to back, so the K|V problem's partial last wave is
+  // filled (C3: 504 + 312 pair tiles = 11.03 waves in one launch vs 7 + 5 in two).  Per element
+  // the arithmetic is unchanged (same K order and epilogue), so outputs are bit-identical.
+  static const bool y_grouped = [] {
+    const char* v = getenv("FPS_Y_GROUPED");
+    return v ? atoi(v) != 0 : true;
+  }();
+  const bool par_group = w->kind == FPS_BLOCK_PAR && tq > 0 && tu > 0 && y_grouped;
   if (tq > 0 && !y_split) {
     // a4: h1 = LN(x)(1+scale1)+shift1 on active rows
-    FPS_TRY(ln1(x_act, xr, tq, ws.h, b->d_cu_q, nullptr));
+    FPS_TRY(ln1(x_act, xr, tq, par_group ? ws.hu : ws.h, b->d_cu_q, nullptr));
     // a5: [tq,H] x [3H,H]^T; Q -> compact, K|V -> merged key rows at original positions
     Epilogue ep{};
     ep.bias = w->b_qkv;
@@ -424,9 +437,23 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
       ep.act = 1; ep.act_from = 3 * H;
       n_out += F;
     }
-    FPS_TRY(launch_gemm(dt, ws.h, w->w_qkv, tq, n_out, H, ep, s));
+    if (par_group) {
+      // Y-mode: cached block-input rows U -> LN (rows [tq, tq + tu) of ws.hu) -> K|V
+      if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
+      kv_ready = nullptr;
+      char* hu_rows = ws.hu + (size_t)tq * H * e;
+      FPS_TRY(ln1(xu, b->d_u_src, tu, hu_rows, b->d_cu_u, nullptr));
+      Epilogue ek{};
+      ek.bias = w->b_qkv ? (const char*)w->b_qkv + (size_t)H * e : nullptr;
+      ek.out0 = kv; ek.ld0 = 2 * H; ek.map0 = b->d_u_row;
+      ek.split = 2 * H;
+      FPS_TRY(launch_gemm_grouped(dt, ws.hu, w->w_qkv, (const char*)w->w_qkv + (size_t)H * H * e,
+                                  tq, tu, n_out, H, ep, ek, s, 2 * H));
+    } else {
+      FPS_TRY(launch_gemm(dt, ws.h, w->w_qkv, tq, n_out, H, ep, s));
+    }
   }
-  if (tu > 0 && !y_split) {
+  if (tu > 0 && !y_split && !par_group) {
     // Y-mode: cached block-input rows U -> LN -> K|V projection (Fig. 5-Bottom, reading R5)
     if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
     kv_ready = nullptr;

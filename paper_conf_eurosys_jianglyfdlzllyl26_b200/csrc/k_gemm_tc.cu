@@ -38,18 +38,21 @@ __device__ __forceinline__ void tile_coords(int tile, int num_m, int num_n, int&
   n_blk = local / gm;
 }
 
-// Grouped launch (double-stream block, R25): problem 0 = rows [0, M) of A with B and `ep`,
-// problem 1 = rows [M, M + M1) with B1 and `ep1` (row-local epilogue indexing), same N and K.
-// Tiles [0, T0) belong to problem 0, the rest to problem 1.
+// Grouped launch: problem 0 = rows [0, M) of A with B [N, K] and `ep`, problem 1 = rows
+// [M, M + M1) with B1 [N1, K] and `ep1` (row-local epilogue indexing), the same K.  Used by the
+// double-stream block (R25: image / text rows on their own weights, N1 = N) and by the Y-mode
+// parallel block (rows M on [Q|K|V|Z], cached rows U on [K|V]: N1 = 2H < N), so one persistent
+// grid covers both problems' tiles -- no second partial wave.  Tiles [0, T0) belong to
+// problem 0, the rest to problem 1.
 template <int GM>
-__device__ __forceinline__ void group_coords(int tile, int T0, int num_m0, int num_m1, int num_n,
-                                             int& p, int& m_blk, int& n_blk) {
+__device__ __forceinline__ void group_coords(int tile, int T0, int num_m0, int num_m1, int num_n0,
+                                             int num_n1, int& p, int& m_blk, int& n_blk) {
   if (tile < T0) {
     p = 0;
-    tile_coords<GM>(tile, num_m0, num_n, m_blk, n_blk);
+    tile_coords<GM>(tile, num_m0, num_n0, m_blk, n_blk);
   } else {
     p = 1;
-    tile_coords<GM>(tile - T0, num_m1, num_n, m_blk, n_blk);
+    tile_coords<GM>(tile - T0, num_m1, num_n1, m_blk, n_blk);
   }
 }
 
@@ -527,7 +530,7 @@ template <int BN, int STAGES, int EPI>
 __global__ void __launch_bounds__(GemmCfg<BN, STAGES, EPI>::THREADS, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const __grid_constant__ CUtensorMap tmB1, int M, int N, int K, Epilogue ep,
-                   int M1, Epilogue ep1) {
+                   int M1, Epilogue ep1, int N1) {
   using Cfg = GemmCfg<BN, STAGES, EPI>;
   constexpr int kGroupM = 16;                              // 2048 rows of A per group
   extern __shared__ uint8_t smem_raw[];
@@ -547,8 +550,9 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, EPI>::THREADS, 1)
   const int num_m = (M + Cfg::BM - 1) / Cfg::BM;
   const int num_m1 = (M1 + Cfg::BM - 1) / Cfg::BM;
   const int num_n = (N + BN - 1) / BN;
+  const int num_n1 = M1 > 0 ? (N1 + BN - 1) / BN : 0;
   const int T0 = num_m * num_n;
-  const int num_tiles = T0 + num_m1 * num_n;
+  const int num_tiles = T0 + num_m1 * num_n1;
   const int num_k = K / Cfg::BK;
 
   if (threadIdx.x == 0) {
@@ -584,7 +588,7 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, EPI>::THREADS, 1)
       uint32_t phase = 0;
       for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
         int p, m_blk, n_blk;
-        group_coords<kGroupM>(tile, T0, num_m, num_m1, num_n, p, m_blk, n_blk);
+        group_coords<kGroupM>(tile, T0, num_m, num_m1, num_n, num_n1, p, m_blk, n_blk);
         const CUtensorMap* tb = p ? &tmB1 : &tmB;
         const int arow = (p ? M : 0) + m_blk * Cfg::BM;
         for (int kb = 0; kb < num_k; ++kb) {
@@ -638,12 +642,12 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, EPI>::THREADS, 1)
     int it = 0;
     for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++it) {
       int p, m_blk, n_blk;
-      group_coords<kGroupM>(tile, T0, num_m, num_m1, num_n, p, m_blk, n_blk);
+      group_coords<kGroupM>(tile, T0, num_m, num_m1, num_n, num_n1, p, m_blk, n_blk);
       const int acc = it & 1;
       tc::mbar_wait(&tfull[acc], (it >> 1) & 1);
       tc::fence_after();
       if (it == 0 && warp == 4 && lane == 0) GEMM_TRACE(5);
-      epilogue_tile<CW>(p ? ep1 : ep, p ? M1 : M, N, m_blk * Cfg::BM + q * 32 + lane,
+      epilogue_tile<CW>(p ? ep1 : ep, p ? M1 : M, p ? N1 : N, m_blk * Cfg::BM + q * 32 + lane,
                         n_blk * BN + h * CW,
                         tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + h * CW,
                         sXs + (warp - 4) * kXsWarpBytes);
@@ -691,7 +695,7 @@ template <int STAGES, int EPI>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Gemm2Cfg<STAGES, EPI>::THREADS, 1)
     gemm_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     const __grid_constant__ CUtensorMap tmB1, int M, int N, int K, Epilogue ep,
-                    int M1, Epilogue ep1) {
+                    int M1, Epilogue ep1, int N1) {
   using Cfg = Gemm2Cfg<STAGES, EPI>;
   constexpr int kGroupM = 8;                               // 2048 rows of A per group
   extern __shared__ uint8_t smem_raw[];
@@ -712,8 +716,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Gemm2Cfg<STAGES, EPI
   const int num_m = (M + Cfg::BM - 1) / Cfg::BM;
   const int num_m1 = (M1 + Cfg::BM - 1) / Cfg::BM;
   const int num_n = (N + Cfg::BN - 1) / Cfg::BN;
+  const int num_n1 = M1 > 0 ? (N1 + Cfg::BN - 1) / Cfg::BN : 0;
   const int T0 = num_m * num_n;
-  const int num_tiles = T0 + num_m1 * num_n;
+  const int num_tiles = T0 + num_m1 * num_n1;
   const int num_k = K / Cfg::BK;
 
   if (threadIdx.x == 0) {
@@ -748,7 +753,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Gemm2Cfg<STAGES, EPI
       uint32_t phase = 0;
       for (int tile = pair; tile < num_tiles; tile += num_pairs) {
         int p, m_blk, n_blk;
-        group_coords<kGroupM>(tile, T0, num_m, num_m1, num_n, p, m_blk, n_blk);
+        group_coords<kGroupM>(tile, T0, num_m, num_m1, num_n, num_n1, p, m_blk, n_blk);
         const CUtensorMap* tb = p ? &tmB1 : &tmB;
         const int arow = (p ? M : 0) + m_blk * Cfg::BM + rank * 128;
         const int brow = n_blk * Cfg::BN + rank * 128;
@@ -802,11 +807,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Gemm2Cfg<STAGES, EPI
     int it = 0;
     for (int tile = pair; tile < num_tiles; tile += num_pairs, ++it) {
       int p, m_blk, n_blk;
-      group_coords<kGroupM>(tile, T0, num_m, num_m1, num_n, p, m_blk, n_blk);
+      group_coords<kGroupM>(tile, T0, num_m, num_m1, num_n, num_n1, p, m_blk, n_blk);
       const int acc = it & 1;
       tc::mbar_wait(&tfull[acc], (it >> 1) & 1);
       tc::fence_after();
-      epilogue_tile<CW>(p ? ep1 : ep, p ? M1 : M, N,
+      epilogue_tile<CW>(p ? ep1 : ep, p ? M1 : M, p ? N1 : N,
                         m_blk * Cfg::BM + rank * 128 + q * 32 + lane, n_blk * Cfg::BN + h * CW,
                         tmem_base + ((uint32_t)(q * 32) << 16) + acc * 256 + h * CW,
                         sXs + (warp - 4) * kXsWarpBytes);
@@ -1002,12 +1007,13 @@ bool gemm_tc_supported(int dtype, int M, int N, int K) {
 
 int g_gemm_force = 0;   // tests: 1 = force the 1-SM kernel, 2 = force the CTA-pair kernel
 
-// Optional second problem of a grouped launch (see group_coords): B1 [N, K], M1 rows of A after
+// Optional second problem of a grouped launch (see group_coords): B1 [N1, K], M1 rows of A after
 // the first M, its own epilogue.  M1 = 0: a plain GEMM.
 struct Group2 {
   const void* B1;
   int M1;
   Epilogue ep1;
+  int N1;
 };
 
 int g_gemm_epi4 = 0;    // tests / A-B: 1 = 4 epilogue warps instead of 8 (1-SM and pair kernels)
@@ -1019,14 +1025,14 @@ static fps_status launch_cfg_e(const void* A, const void* B, int M, int N, int K
   CUtensorMap ta, tb, tb1;
   if (!make_tmap_2d_bf16(&ta, A, M + g2.M1, K, (uint64_t)K * 2, Cfg::BK, Cfg::BM) ||
       !make_tmap_2d_bf16(&tb, B, N, K, (uint64_t)K * 2, Cfg::BK, BN) ||
-      (g2.M1 > 0 && !make_tmap_2d_bf16(&tb1, g2.B1, N, K, (uint64_t)K * 2, Cfg::BK, BN)))
+      (g2.M1 > 0 && !make_tmap_2d_bf16(&tb1, g2.B1, g2.N1, K, (uint64_t)K * 2, Cfg::BK, BN)))
     return fail(FPS_ECUDA, "gemm_tc: cuTensorMapEncodeTiled failed (M=%d N=%d K=%d)", M, N, K);
   if (g2.M1 == 0) tb1 = tb;
   FPS_SMEM_ATTR((gemm_tc_kernel<BN, STAGES, EPI>), Cfg::SMEM);
-  const int tiles = (ceil_div(M, Cfg::BM) + ceil_div(g2.M1, Cfg::BM)) * ceil_div(N, BN);
+  const int tiles = ceil_div(M, Cfg::BM) * ceil_div(N, BN) + ceil_div(g2.M1, Cfg::BM) * ceil_div(g2.N1, BN);
   const int grid = tiles < sm_budget() ? tiles : sm_budget();
   FPS_CUDA_TRY(launch_k(gemm_tc_kernel<BN, STAGES, EPI>, dim3(grid), dim3(Cfg::THREADS), Cfg::SMEM, s, ta, tb,
-                        tb1, M, N, K, ep, g2.M1, g2.ep1));
+                        tb1, M, N, K, ep, g2.M1, g2.ep1, g2.N1));
   count_launch();
   FPS_LAUNCH_CHECK();
   return FPS_OK;
@@ -1046,14 +1052,15 @@ static fps_status launch_pair_e(const void* A, const void* B, int M, int N, int 
   CUtensorMap ta, tb, tb1;
   if (!make_tmap_2d_bf16(&ta, A, M + g2.M1, K, (uint64_t)K * 2, Cfg::BK, 128) ||
       !make_tmap_2d_bf16(&tb, B, N, K, (uint64_t)K * 2, Cfg::BK, 128) ||
-      (g2.M1 > 0 && !make_tmap_2d_bf16(&tb1, g2.B1, N, K, (uint64_t)K * 2, Cfg::BK, 128)))
+      (g2.M1 > 0 && !make_tmap_2d_bf16(&tb1, g2.B1, g2.N1, K, (uint64_t)K * 2, Cfg::BK, 128)))
     return fail(FPS_ECUDA, "gemm_tc2: cuTensorMapEncodeTiled failed (M=%d N=%d K=%d)", M, N, K);
   if (g2.M1 == 0) tb1 = tb;
   FPS_SMEM_ATTR((gemm_tc2_kernel<STAGES, EPI>), Cfg::SMEM);
-  const int tiles = (ceil_div(M, Cfg::BM) + ceil_div(g2.M1, Cfg::BM)) * ceil_div(N, Cfg::BN);
+  const int tiles = ceil_div(M, Cfg::BM) * ceil_div(N, Cfg::BN) +
+                    ceil_div(g2.M1, Cfg::BM) * ceil_div(g2.N1, Cfg::BN);
   const int pairs = tiles < sm_budget() / 2 ? tiles : sm_budget() / 2;
   FPS_CUDA_TRY(launch_k(gemm_tc2_kernel<STAGES, EPI>, dim3(2 * pairs), dim3(Cfg::THREADS), Cfg::SMEM,
-                        s, ta, tb, tb1, M, N, K, ep, g2.M1, g2.ep1));
+                        s, ta, tb, tb1, M, N, K, ep, g2.M1, g2.ep1, g2.N1));
   count_launch();
   FPS_LAUNCH_CHECK();
   return FPS_OK;
@@ -1119,13 +1126,16 @@ static int swap_block(int M, int N, long* cost) {
 // GEMM with the combined tile counts.
 fps_status launch_gemm_tc_grouped(const void* A, const void* B0, const void* B1, int M0, int M1,
                                   int N, int K, const Epilogue& ep0, const Epilogue& ep1,
-                                  cudaStream_t s) {
+                                  cudaStream_t s, int N1) {
   if (!aligned16(A) || !aligned16(B0) || !aligned16(B1))
     return fail(FPS_EINVAL, "gemm_tc: unaligned operand");
-  const Group2 g2{B1, M1, ep1};
-  const int m1 = ceil_div(M0, 128) + ceil_div(M1, 128), m2 = ceil_div(M0, 256) + ceil_div(M1, 256);
-  const long t256 = (long)m1 * ceil_div(N, 256), t128 = (long)m1 * ceil_div(N, 128);
-  const long tp = (long)m2 * ceil_div(N, 256);
+  if (N1 <= 0) N1 = N;
+  if (N1 % 8 != 0) return fail(FPS_EINVAL, "gemm_tc: N1 %% 8 != 0");
+  const Group2 g2{B1, M1, ep1, N1};
+  // tile counts of both problems (problem 1 has N1 columns)
+  const long t256 = (long)ceil_div(M0, 128) * ceil_div(N, 256) + (long)ceil_div(M1, 128) * ceil_div(N1, 256);
+  const long t128 = (long)ceil_div(M0, 128) * ceil_div(N, 128) + (long)ceil_div(M1, 128) * ceil_div(N1, 128);
+  const long tp = (long)ceil_div(M0, 256) * ceil_div(N, 256) + (long)ceil_div(M1, 256) * ceil_div(N1, 256);
   const long c256 = ((t256 + sm_budget() - 1) / sm_budget()) * 256;
   const long c128 = ((t128 + sm_budget() - 1) / sm_budget()) * 128;
   const long cp = ((tp + sm_budget() / 2 - 1) / (sm_budget() / 2)) * 256;

@@ -55,12 +55,14 @@ fps_status launch_gemm_tc(const void* A, const void* B, int M, int N, int K, con
 bool gemm_tc_supported(int dtype, int M, int N, int K);
 // two GEMMs sharing N and K in one launch: rows [0, M0) of A with B0 / ep0, rows [M0, M0 + M1)
 // with B1 / ep1 (ep1 indexes its rows from 0)
+// Two GEMMs in one launch: rows [0, M0) of A times B0 [N, K] (ep0), rows [M0, M0 + M1) times
+// B1 [N1, K] (ep1); N1 = 0 means N1 = N
 fps_status launch_gemm_grouped(int dtype, const void* A, const void* B0, const void* B1, int M0,
                                int M1, int N, int K, const Epilogue& ep0, const Epilogue& ep1,
-                               cudaStream_t s);
+                               cudaStream_t s, int N1 = 0);
 fps_status launch_gemm_tc_grouped(const void* A, const void* B0, const void* B1, int M0, int M1,
                                   int N, int K, const Epilogue& ep0, const Epilogue& ep1,
-                                  cudaStream_t s);
+                                  cudaStream_t s, int N1 = 0);
 // Scratch for split-KV attention: partial outputs (S x total_q x H bf16) and per-row
 // statistics (S x total_q x heads float2); null = no split
 struct AttnScratch {
