@@ -61,7 +61,9 @@ int32_t fps_device_ok(void);
  * partial outputs);
  * bit 11 = the tcgen05 GEMMs (1-SM and CTA-pair) with 4 epilogue warps instead of 8 (A/B);
  * bit 12 = the CTA-pair attention kernel (attn_tc4, head_dim 128);
- * bits 13-14 = 1 / 2 force the 1-SM GEMM's 128- / 256-column tile (A/B experiments). */
+ * bits 13-14 = 1 / 2 force the 1-SM GEMM's 128- / 256-column tile (A/B experiments);
+ * bit 15 = the Y-mode parallel block's two projections (rows M on W1, cached rows U on K|V) as two
+ *          launches instead of one grouped launch (A/B; outputs are bit-identical). */
 int64_t fps_launch_count(void);
 void fps_set_disable_tc(int32_t flags);
 /* Per-kernel-class timing for the bench: when enabled (this also clears old records) every

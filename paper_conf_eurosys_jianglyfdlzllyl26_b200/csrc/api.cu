@@ -13,6 +13,7 @@ thread_local long long g_launches = 0;
 int g_disable_tc = 0;
 int g_sm_reserved = 0;
 int g_pdl = 1;
+int g_y_grouped = 1;   // Y-mode parallel block: one grouped launch for W1(M) + K|V(U) (bit 15 off)
 thread_local PdlFence g_pdl_fence;
 
 void set_error(const char* fmt, ...) {
@@ -417,11 +418,7 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
   // grid runs both problems' tiles back to back, so the K|V problem's partial last wave is
   // filled (C3: 504 + 312 pair tiles = 11.03 waves in one launch vs 7 + 5 in two).  Per element
   // the arithmetic is unchanged (same K order and epilogue), so outputs are bit-identical.
-  static const bool y_grouped = [] {
-    const char* v = getenv("FPS_Y_GROUPED");
-    return v ? atoi(v) != 0 : true;
-  }();
-  const bool par_group = w->kind == FPS_BLOCK_PAR && tq > 0 && tu > 0 && y_grouped;
+  const bool par_group = w->kind == FPS_BLOCK_PAR && tq > 0 && tu > 0 && g_y_grouped;
   if (tq > 0 && !y_split) {
     // a4: h1 = LN(x)(1+scale1)+shift1 on active rows
     FPS_TRY(ln1(x_act, xr, tq, par_group ? ws.hu : ws.h, b->d_cu_q, nullptr));
@@ -634,6 +631,7 @@ void fps_set_disable_tc(int32_t flags) {
   fps::g_gemm_epi4 = (flags >> 11) & 1;
   fps::g_attn_pair = (flags >> 12) & 1;
   fps::g_gemm_bn = (flags >> 13) & 3;
+  fps::g_y_grouped = (flags >> 15) & 1 ? 0 : 1;
 }
 
 fps_status fps_build_mask_index(const uint8_t* d_masks, const int32_t* d_offsets, int32_t n_req,

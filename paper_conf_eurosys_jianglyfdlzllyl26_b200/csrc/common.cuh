@@ -75,6 +75,7 @@ __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;"
 __device__ __forceinline__ void pdl_trigger() {
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 }
+extern int g_y_grouped;   // 1 = Y-mode parallel block's two projections in one launch
 extern int g_pdl;   // 1 = launch with PDL (default), 0 = plain launches (fps_set_disable_tc bit 6)
 // Set by every cross-stream wait / copy the library enqueues: the next kernel is launched
 // WITHOUT the PDL attribute, so PDL only ever overlaps two back-to-back library kernels.

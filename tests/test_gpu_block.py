@@ -294,3 +294,25 @@ def test_active_rows_read_from_full_buffer_bit_identical(F, kind, mode):
     finally:
         F.masked_block_forward = orig
     assert np.array_equal(y, y_ref)
+
+
+@pytest.mark.parametrize("H,heads,Fd,L_img,L_txt,ratios", [
+    (256, 2, 1024, 576, 40, [0.05, 0.6, 0.3]),          # several tiles per problem, ragged
+    (3072, 24, 12288, 4096, 512, [0.2]),                # the C3 single-stream block
+])
+def test_y_parallel_grouped_projections_bit_identical(F, H, heads, Fd, L_img, L_txt, ratios):
+    """Y-mode parallel block: W1 over rows M and K|V over cached rows U in ONE grouped launch
+    (per-problem N: 3H + F and 2H) gives the same bits as two launches (flag bit 15), and both
+    match the oracle (masked_block_y)."""
+    w, reqs = _problem(4200 + H, "bf16", H, heads, Fd, L_img, L_txt, ratios, blobs=True,
+                       kind="par")
+    y_grouped, kv_grouped = _run_masked(F, w, reqs, heads, "bf16", "y")
+    F.fps_set_disable_tc(1 << 15)
+    try:
+        y_two, kv_two = _run_masked(F, w, reqs, heads, "bf16", "y")
+    finally:
+        F.fps_set_disable_tc(0)
+    assert np.array_equal(y_grouped, y_two)
+    assert torch.equal(kv_grouped, kv_two)
+    if H <= 256:
+        check_close(y_grouped, _ref_masked(w, reqs, heads, "y"), TOL["bf16"])
