@@ -63,7 +63,8 @@ int32_t fps_device_ok(void);
  * bit 12 = the CTA-pair attention kernel (attn_tc4, head_dim 128);
  * bits 13-14 = 1 / 2 force the 1-SM GEMM's 128- / 256-column tile (A/B experiments);
  * bit 15 = the Y-mode parallel block's two projections (rows M on W1, cached rows U on K|V) as two
- *          launches instead of one grouped launch (A/B; outputs are bit-identical). */
+ *          launches instead of one grouped launch (A/B; outputs are bit-identical);
+ * bit 16 = head_dim 64 attention on attn_tc3 instead of attn_tc5 (three rotating S buffers). */
 int64_t fps_launch_count(void);
 void fps_set_disable_tc(int32_t flags);
 /* Per-kernel-class timing for the bench: when enabled (this also clears old records) every

@@ -632,6 +632,7 @@ void fps_set_disable_tc(int32_t flags) {
   fps::g_attn_pair = (flags >> 12) & 1;
   fps::g_gemm_bn = (flags >> 13) & 3;
   fps::g_y_grouped = (flags >> 15) & 1 ? 0 : 1;
+  fps::g_attn_rot = (flags >> 16) & 1 ? 0 : 1;
 }
 
 fps_status fps_build_mask_index(const uint8_t* d_masks, const int32_t* d_offsets, int32_t n_req,

@@ -644,6 +644,36 @@ __global__ void __launch_bounds__(384, 1)
 #else
 #define ATTN_MMA_WAIT(bar, par) tc::mbar_wait_sleep(bar, par)
 #endif
+// Row max of 128 fp32 scores in C independent FMNMX3 chains.  16 chains (depth 5 + a 3-level
+// tree) measured no faster than 4 (tools/scripts/r02z20_max16.sh: 1038 / 1205 vs 1044 / 1211
+// TF/s at the C3 masked / dense shapes): the max phase is issue-shared, not latency-bound
+#ifndef FPS_ATTN_MAX_CHAINS
+#define FPS_ATTN_MAX_CHAINS 4
+#endif
+__device__ __forceinline__ float row_max128(const float* s) {
+  constexpr int C = FPS_ATTN_MAX_CHAINS;
+  float m[C];
+#pragma unroll
+  for (int j = 0; j < C; ++j) m[j] = s[j];
+  int k = C;
+#pragma unroll
+  for (; k + 2 * C <= 128; k += 2 * C)
+#pragma unroll
+    for (int j = 0; j < C; ++j) m[j] = tc::fmax3(m[j], s[k + j], s[k + C + j]);
+#pragma unroll
+  for (; k < 128; k += C)
+#pragma unroll
+    for (int j = 0; j < C; ++j) m[j] = fmaxf(m[j], s[k + j]);
+#pragma unroll
+  for (int w = C; w > 1; w = (w + 2) / 3) {
+#pragma unroll
+    for (int j = 0; j < (w + 2) / 3; ++j) {
+      const float a = m[3 * j], b = 3 * j + 1 < w ? m[3 * j + 1] : a, c = 3 * j + 2 < w ? m[3 * j + 2] : a;
+      m[j] = tc::fmax3(a, b, c);
+    }
+  }
+  return m[0];
+}
 template <int D>
 __device__ __forceinline__ constexpr bool attn_poly(int i) {
   constexpr int N = D == 64 ? FPS_ATTN_POLY64 : FPS_ATTN_POLY;
@@ -870,14 +900,7 @@ __global__ void __launch_bounds__(512, 1)
 #pragma unroll
           for (int i = 0; i < 128; ++i) s[i] = (i < valid) ? s[i] : -INFINITY;
         }
-        float m4[4] = {s[0], s[1], s[2], s[3]};
-#pragma unroll
-        for (int i = 4; i < 124; i += 8)
-#pragma unroll
-          for (int j = 0; j < 4; ++j) m4[j] = tc::fmax3(m4[j], s[i + j], s[i + 4 + j]);
-#pragma unroll
-        for (int j = 0; j < 4; ++j) m4[j] = fmaxf(m4[j], s[124 + j]);
-        const float mx = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) * scale_log2;
+        const float mx = row_max128(s) * scale_log2;
         float factor = 1.0f;
         if (mx > m_used + 8.0f) {                          // lazy rescale (threshold 2^8)
           factor = tc::ex2(m_used - mx);
@@ -985,6 +1008,361 @@ __global__ void __launch_bounds__(512, 1)
       const float l = sL[t * 128 + row];
       const float inv = (l > 0.f) ? 1.0f / l : 0.f;
       const uint32_t tO = tmem + 256 + t * 128 + lane_off;
+#pragma unroll 1
+      for (int c = 0; c < D / 32; ++c) {
+        uint32_t o[32];
+        tc::tmem_ld32(tO + c * 32, o);
+        tc::tmem_wait_ld();
+        if (grow < q_end) {
+#pragma unroll
+          for (int g = 0; g < 4; ++g) {
+            float f[8];
+#pragma unroll
+            for (int e = 0; e < 8; ++e) f[e] = __uint_as_float(o[g * 8 + e]) * inv;
+            *reinterpret_cast<uint4*>(orow + c * 32 + g * 8) = Vec16<__nv_bfloat16>::pack(f);
+          }
+        }
+      }
+    }
+  }
+  tc::fence_before();
+  __syncthreads();
+  if (warp == 2) {
+    tc::fence_after();
+    tc::tmem_dealloc<Cfg::TMEM_COLS>(tmem);
+  }
+}
+
+// ============================================================================================
+// attn_tc5: head_dim 64, two query tiles per CTA (as attn_tc3) with THREE S buffers in TMEM
+// rotating over the two tiles.  At d = 64 the outputs need only 2 x 64 TMEM columns, so the 512
+// columns hold S buffers at [0,128), [128,256), [256,384) and O_A [384,448), O_B [448,512).
+// S of "index" i = 2 kt + t (tile t, key tile kt) lives in buffer i % 3, its P in that buffer's
+// upper half.  The MMA warp issues S(i + 3) right after PV(i) into PV(i)'s buffer (tcgen05 MMAs
+// execute in issue order), so the order is
+//     S(0) S(1) S(2) | PV(0) S(3) | PV(1) S(4) | PV(2) S(5) | ...
+// and S_t(kt+1) is issued after the OTHER tile's PV, not after PV_t(kt): a tile's softmax no
+// longer waits for its own PV and next QK^T (attn_tc3's S -> softmax -> PV -> S chain, ~2850
+// cycles per key tile at d = 64 against 1024 of MMAs), and the two softmax warpgroups can run
+// back to back, bounded by MUFU / issue.
+// Because S_t(kt+1) may now be computed before PV_t(kt), the correction warps wait for PV_t(kt)
+// to complete (bar_pv) before rescaling O_t for key tile kt+1.  Barriers that a warpgroup may
+// reach one key tile ahead of its consumer are double-buffered ([tile][kt & 1], parity
+// (kt >> 1) & 1), so no phase can be overtaken.
+struct Attn5Cfg {
+  static constexpr int D = 64;
+  static constexpr int Q_BYTES = 128 * D * 2;
+  static constexpr int KV_TILE = 128 * D * 2;
+  static constexpr int SMEM = 2 * Q_BYTES + 4 * KV_TILE + 2 * 2 * 128 * 4 + 1024 + 512;
+  static constexpr int TMEM_COLS = 512;
+  static constexpr int O_COL = 384;                         // O_t at O_COL + 64 t
+};
+
+__global__ void __launch_bounds__(512, 1)
+    attn_tc5_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmKV,
+                    __nv_bfloat16* __restrict__ O, const int32_t* __restrict__ cu_q,
+                    const int32_t* __restrict__ cu_k, int n_req, int heads, float scale_log2, int ldo,
+                    __nv_bfloat16* __restrict__ Opart, float2* __restrict__ ML, long long part_stride,
+                    int total_q, const int32_t* __restrict__ o_map) {
+  using Cfg = Attn5Cfg;
+  constexpr int D = Cfg::D;
+  constexpr int CHUNK = 128 * 128;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~uintptr_t(1023));
+  uint8_t* sQ = smem;                                       // [2 tiles]
+  uint8_t* sK = sQ + 2 * Cfg::Q_BYTES;                      // [2 stages]
+  uint8_t* sV = sK + 2 * Cfg::KV_TILE;
+  float* sScale = reinterpret_cast<float*>(sV + 2 * Cfg::KV_TILE);   // [tile][row]
+  float* sL = sScale + 2 * 128;                                      // [tile][row]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sL + 2 * 128);
+  uint64_t* bar_q = bars;
+  uint64_t* k_full = bars + 1;      // [stage]
+  uint64_t* k_empty = bars + 3;
+  uint64_t* v_full = bars + 5;
+  uint64_t* v_empty = bars + 7;
+  uint64_t* bar_s = bars + 9;       // [buffer 0..2] S(i) in TMEM                 (MMA commit)
+  uint64_t* bar_p = bars + 12;      // [tile][kt&1] P half 1 stored + O rescaled  (4 softmax + 4 corr.)
+  uint64_t* bar_p2 = bars + 16;     // [tile][kt&1] P half 2 stored               (4 softmax + 4 corr.)
+  uint64_t* bar_stat = bars + 20;   // [tile][kt&1] scale in smem                 (4 softmax)
+  uint64_t* bar_pv = bars + 24;     // [tile][kt&1] PV_t(kt) complete             (MMA commit)
+  uint64_t* bar_o = bars + 28;      // [tile] final PV done                       (MMA commit)
+  uint64_t* bar_fin = bars + 30;    // [tile] row sum l in smem                   (4 softmax)
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + 32);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  // grid (heads, query-tile pairs, splits) as attn_tc3
+  const int head = blockIdx.x;
+  const int H = heads * D;
+  int r = 0, qp = blockIdx.y, ntile = 0;
+  for (; r < n_req; ++r) {
+    ntile = (__ldg(cu_q + r + 1) - __ldg(cu_q + r) + 127) >> 7;
+    const int np = (ntile + 1) >> 1;
+    if (qp < np) break;
+    qp -= np;
+  }
+  const bool hasB = 2 * qp + 1 < ntile;
+  const int q_end = __ldg(cu_q + r + 1);
+  const int q0 = __ldg(cu_q + r) + qp * 256;
+  const int Lr = __ldg(cu_k + r + 1) - __ldg(cu_k + r);
+  const int nk_all = (Lr + 127) >> 7;
+  const int nsplit = gridDim.z, split = blockIdx.z;
+  const int kb = (int)(((long long)nk_all * split) / nsplit);
+  const int nk = (int)(((long long)nk_all * (split + 1)) / nsplit) - kb;
+  const int k0 = __ldg(cu_k + r) + kb * 128;
+  const int Lr_rem = Lr - kb * 128;
+
+  if (threadIdx.x == 0) {
+    tc::mbar_init(bar_q, 1);
+    for (int s = 0; s < 2; ++s) {
+      tc::mbar_init(&k_full[s], 1);
+      tc::mbar_init(&k_empty[s], 1);
+      tc::mbar_init(&v_full[s], 1);
+      tc::mbar_init(&v_empty[s], 1);
+      tc::mbar_init(&bar_o[s], 1);
+      tc::mbar_init(&bar_fin[s], 4);
+    }
+    for (int b = 0; b < 3; ++b) tc::mbar_init(&bar_s[b], 1);
+    for (int b = 0; b < 4; ++b) {
+      tc::mbar_init(&bar_p[b], 8);
+      tc::mbar_init(&bar_p2[b], 8);
+      tc::mbar_init(&bar_stat[b], 4);
+      tc::mbar_init(&bar_pv[b], 1);
+    }
+    tc::fence_mbar_init();
+  }
+  if (warp == 0 && lane == 0) {
+    tc::tma_prefetch_desc(&tmQ);
+    tc::tma_prefetch_desc(&tmKV);
+  }
+  if (warp == 2) tc::tmem_alloc<Cfg::TMEM_COLS>(tmem_holder);
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tmem = *tmem_holder;
+  pdl_trigger();
+  pdl_wait();
+
+  if (warp < 4) {
+    tc::regs_dec<56>();
+    if (warp == 0) {
+      if (lane == 0 && nk > 0) {
+        tc::mbar_expect_tx(bar_q, (hasB ? 2 : 1) * Cfg::Q_BYTES);
+        for (int t = 0; t < (hasB ? 2 : 1); ++t)
+          tc::tma_load_2d(sQ + t * Cfg::Q_BYTES, &tmQ, bar_q, head * D, q0 + t * 128);
+        for (int kt = 0; kt < nk; ++kt) {
+          const int st = kt & 1;
+          tc::mbar_wait_sleep(&k_empty[st], ((kt >> 1) & 1) ^ 1);
+          tc::mbar_expect_tx(&k_full[st], Cfg::KV_TILE);
+          tc::tma_load_2d(sK + st * Cfg::KV_TILE, &tmKV, &k_full[st], head * D, k0 + kt * 128);
+        }
+      }
+    } else if (warp == 3) {
+      if (lane == 0) {
+        for (int kt = 0; kt < nk; ++kt) {
+          const int st = kt & 1;
+          tc::mbar_wait_sleep(&v_empty[st], ((kt >> 1) & 1) ^ 1);
+          tc::mbar_expect_tx(&v_full[st], Cfg::KV_TILE);
+          tc::tma_load_2d(sV + st * Cfg::KV_TILE, &tmKV, &v_full[st], H + head * D, k0 + kt * 128);
+        }
+      }
+    } else if (warp == 1) {
+      if (nk > 0) {
+        constexpr uint32_t idesc_s = tc::idesc_bf16(128, 128);
+        constexpr uint32_t idesc_o = tc::idesc_bf16(128, D, /*b_mn_major=*/true);
+        tc::mbar_wait_sleep(bar_q, 0);
+        const uint64_t dq = tc::sdesc_k_sw128(tc::smem_u32(sQ));
+        const uint64_t dk = tc::sdesc_k_sw128(tc::smem_u32(sK));
+        const uint64_t dv = tc::sdesc_mn_sw128(tc::smem_u32(sV), CHUNK);
+        // S(i) = Q_t K_kt^T into buffer i % 3 (i = 2 kt + t); a K tile is released after the
+        // last S that reads it (tile B's, or tile A's when the CTA has one tile)
+        auto issue_s = [&](int i) {
+          const int t = i & 1, kt = i >> 1;
+          const uint64_t a = dq + ((t * Cfg::Q_BYTES) >> 4);
+          const uint64_t b = dk + (((kt & 1) * Cfg::KV_TILE) >> 4);
+          tc::mma_ss_k4_commit((uint32_t)((i % 3) * 128), a, b, idesc_s, &bar_s[i % 3]);
+          if (t == 1 || !hasB) tc::mma_commit_w(&k_empty[kt & 1]);
+        };
+        auto wait_k = [&](int kt) {
+          tc::mbar_wait_sleep(&k_full[kt & 1], (kt >> 1) & 1);
+          tc::fence_after();
+        };
+        // O_t += P_t V_kt: keys 0-63 once bar_p, keys 64-127 once bar_p2
+        auto issue_pv = [&](int i) {
+          const int t = i & 1, kt = i >> 1, pb = t * 2 + (kt & 1);
+          const uint32_t ph = (kt >> 1) & 1;
+          const uint64_t b = dv + (((kt & 1) * Cfg::KV_TILE) >> 4);
+          const uint32_t p = (uint32_t)((i % 3) * 128);
+          ATTN_MMA_WAIT(&bar_p[pb], ph);
+          tc::fence_after();
+          tc::mma_ts_k4(Cfg::O_COL + t * 64, p + 64, b, idesc_o, kt != 0);
+          ATTN_MMA_WAIT(&bar_p2[pb], ph);
+          tc::fence_after();
+          tc::mma_ts_k4(Cfg::O_COL + t * 64, p + 96, b + (4 * 2048 >> 4), idesc_o, 1);
+          tc::mma_commit_w(&bar_pv[pb]);
+          if (kt + 1 == nk) tc::mma_commit_w(&bar_o[t]);
+          if (t == 1 || !hasB) tc::mma_commit_w(&v_empty[kt & 1]);
+        };
+        // prologue: S(0), S(1), S(2) (indices of a missing tile B are skipped)
+        wait_k(0);
+        issue_s(0);
+        if (hasB) issue_s(1);
+        if (nk > 1) {
+          wait_k(1);
+          issue_s(2);
+        }
+        for (int kt = 0; kt < nk; ++kt) {
+          tc::mbar_wait_sleep(&v_full[kt & 1], (kt >> 1) & 1);
+          issue_pv(2 * kt);                                  // PV_A(kt)
+          if (kt + 1 < nk && hasB) issue_s(2 * kt + 3);      // S_B(kt+1) into PV_A(kt)'s buffer
+          if (hasB) issue_pv(2 * kt + 1);                    // PV_B(kt)
+          if (kt + 2 < nk) {                                 // S_A(kt+2) into PV_B(kt)'s buffer
+            wait_k(kt + 2);
+            issue_s(2 * kt + 4);
+          }
+        }
+      }
+    }
+  } else if (warp < 12) {
+    // ---------------- softmax (warps 4-7: tile A, 8-11: tile B), as attn_tc3 ----------------
+    tc::regs_inc<192>();
+    const int t = (warp >= 8) ? 1 : 0;
+    if (t == 0 || hasB) {
+      const int q = warp & 3;
+      const int row = q * 32 + lane;
+      const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+      float m_used = -INFINITY, l = 0.f;
+      for (int kt = 0; kt < nk; ++kt) {
+        const int i = 2 * kt + t, pb = t * 2 + (kt & 1);
+        // buffer i % 3 is used by indices b, b + 3, ... (one tile: only the even indices, so
+        // the n-th use of a buffer is key tile 3n + ..)
+        const int n_use = hasB ? i / 3 : kt / 3;
+        tc::mbar_wait(&bar_s[i % 3], (uint32_t)(n_use & 1));
+        tc::fence_after();
+        const uint32_t tS = tmem + (uint32_t)((i % 3) * 128);
+        float s[128];
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+          tc::tmem_ld32(tS + lane_off + c * 32, reinterpret_cast<uint32_t*>(s + c * 32));
+        tc::tmem_wait_ld();
+        const int valid = Lr_rem - kt * 128;
+        if (valid < 128) {
+#pragma unroll
+          for (int k = 0; k < 128; ++k) s[k] = (k < valid) ? s[k] : -INFINITY;
+        }
+        const float mx = row_max128(s) * scale_log2;
+        float factor = 1.0f;
+        if (mx > m_used + 8.0f) {
+          factor = tc::ex2(m_used - mx);
+          m_used = mx;
+        }
+        sScale[t * 128 + row] = factor;
+        __syncwarp();
+        if (lane == 0) tc::mbar_arrive(&bar_stat[pb]);
+        const float nm = -m_used;
+        float a8[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          uint32_t p[16];
+#pragma unroll
+          for (int k = c * 32; k < c * 32 + 32; k += 2) {
+            tc::ffma2(s[k], s[k + 1], s[k], s[k + 1], scale_log2, scale_log2, nm, nm);
+            if (attn_poly<D>(k)) {
+              tc::ex2_poly2(s[k], s[k + 1]);
+            } else {
+              s[k] = tc::ex2(s[k]);
+              s[k + 1] = tc::ex2(s[k + 1]);
+            }
+            p[(k - c * 32) >> 1] = tc::pack_bf16x2_rn(s[k], s[k + 1]);
+          }
+          tc::tmem_st16(tS + lane_off + 64 + c * 16, p);
+          if (c & 1) {
+            tc::tmem_wait_st();
+            tc::fence_before();
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(c == 1 ? &bar_p[pb] : &bar_p2[pb]);
+          }
+        }
+#pragma unroll
+        for (int k = 0; k < 128; k += 2) {
+          const int j = (k >> 1) & 3;
+          tc::fadd2(a8[2 * j], a8[2 * j + 1], a8[2 * j], a8[2 * j + 1], s[k], s[k + 1]);
+        }
+        l = l * factor + (((a8[0] + a8[1]) + (a8[2] + a8[3])) + ((a8[4] + a8[5]) + (a8[6] + a8[7])));
+      }
+      sL[t * 128 + row] = l;
+      if (nsplit > 1) {
+        const int grow = q0 + t * 128 + row;
+        if (grow < q_end) ML[((size_t)split * total_q + grow) * heads + head] = make_float2(m_used, l);
+      }
+      __syncwarp();
+      if (lane == 0) tc::mbar_arrive(&bar_fin[t]);
+    }
+  } else {
+    // ---------------- correction + epilogue (warps 12-15) ----------------
+    tc::regs_dec<72>();
+    const int q = warp & 3;
+    const int row = q * 32 + lane;
+    const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+    const int ntl = hasB ? 2 : 1;
+    for (int kt = 0; kt < nk; ++kt) {
+      for (int t = 0; t < ntl; ++t) {
+        const int pb = t * 2 + (kt & 1);
+        tc::mbar_wait(&bar_stat[pb], (uint32_t)((kt >> 1) & 1));
+        if (kt > 0) {
+          // PV_t(kt-1) must be complete before O_t is rescaled for key tile kt (its S may have
+          // been computed first) -- and before this warp's arrival for kt can complete a phase
+          const int pp = t * 2 + ((kt - 1) & 1);
+          tc::mbar_wait(&bar_pv[pp], (uint32_t)(((kt - 1) >> 1) & 1));
+        }
+        const float f = sScale[t * 128 + row];
+        if (kt > 0 && __any_sync(0xffffffffu, f != 1.0f)) {
+          tc::fence_after();
+          const uint32_t tO = tmem + Cfg::O_COL + t * 64 + lane_off;
+#pragma unroll 1
+          for (int c = 0; c < D / 32; ++c) {
+            uint32_t o[32];
+            tc::tmem_ld32(tO + c * 32, o);
+            tc::tmem_wait_ld();
+#pragma unroll
+            for (int e = 0; e < 32; e += 2) {
+              float x0 = __uint_as_float(o[e]), x1 = __uint_as_float(o[e + 1]);
+              tc::ffma2(x0, x1, x0, x1, f, f, 0.f, 0.f);
+              o[e] = __float_as_uint(x0);
+              o[e + 1] = __float_as_uint(x1);
+            }
+            tc::tmem_st32(tO + c * 32, o);
+          }
+          tc::tmem_wait_st();
+        }
+        tc::fence_before();
+        __syncwarp();
+        if (lane == 0) {
+          tc::mbar_arrive(&bar_p[pb]);
+          tc::mbar_arrive(&bar_p2[pb]);
+        }
+      }
+    }
+    for (int t = 0; t < ntl; ++t) {
+      const int grow = q0 + t * 128 + row;
+      const int orow_i = (o_map && grow < q_end) ? __ldg(o_map + grow) : grow;
+      __nv_bfloat16* orow = nsplit > 1
+          ? Opart + split * part_stride + (size_t)grow * (heads * D) + head * D
+          : O + (size_t)orow_i * ldo + head * D;
+      if (nk == 0) {
+        if (grow < q_end) {
+          for (int c = 0; c < D; c += 8) *reinterpret_cast<uint4*>(orow + c) = make_uint4(0, 0, 0, 0);
+          if (nsplit > 1)
+            ML[((size_t)split * total_q + grow) * heads + head] = make_float2(-INFINITY, 0.f);
+        }
+        continue;
+      }
+      tc::mbar_wait(&bar_fin[t], 0);
+      tc::mbar_wait(&bar_o[t], 0);
+      tc::fence_after();
+      const float l = sL[t * 128 + row];
+      const float inv = (l > 0.f) ? 1.0f / l : 0.f;
+      const uint32_t tO = tmem + Cfg::O_COL + t * 64 + lane_off;
 #pragma unroll 1
       for (int c = 0; c < D / 32; ++c) {
         uint32_t o[32];
@@ -1630,6 +2008,48 @@ static fps_status launch_d3(const void* q, const void* kv, void* o, int heads,
   return FPS_OK;
 }
 
+int g_attn_rot = 1;     // 1 = attn_tc5 (three rotating S buffers) for head_dim 64; 0 = attn_tc3
+
+static fps_status launch_d5(const void* q, const void* kv, void* o, int heads,
+                            const int32_t* d_cu_q, const int32_t* d_cu_k, const int32_t* h_cu_q,
+                            const int32_t* h_cu_k, int n_req, cudaStream_t s, int ldo,
+                            const AttnScratch* sc, const int32_t* o_map) {
+  using Cfg = Attn5Cfg;
+  constexpr int D = Cfg::D;
+  const int H = heads * D;
+  int pairs = 0, min_nk = 1 << 30;
+  for (int r = 0; r < n_req; ++r) {
+    const int pr = ((h_cu_q[r + 1] - h_cu_q[r] + 127) / 128 + 1) / 2;
+    pairs += pr;
+    if (pr > 0) min_nk = std::min(min_nk, (h_cu_k[r + 1] - h_cu_k[r] + 127) / 128);
+  }
+  if (pairs == 0) return FPS_OK;
+  const int total_q = h_cu_q[n_req];
+  const int S = choose_split(pairs * heads, min_nk, total_q, H, heads, sc);
+  CUtensorMap tq, tkv;
+  if (!make_tmap_2d_bf16(&tq, q, (uint64_t)h_cu_q[n_req], H, (uint64_t)H * 2, 64, 128))
+    return fail(FPS_ECUDA, "attention_tc5: Q tensor map");
+  if (!make_tmap_2d_bf16(&tkv, kv, (uint64_t)h_cu_k[n_req], 2 * H, (uint64_t)H * 4, 64, 128))
+    return fail(FPS_ECUDA, "attention_tc5: KV tensor map");
+  FPS_SMEM_ATTR(attn_tc5_kernel, Cfg::SMEM);
+  const float scale_log2 = 1.4426950408889634f / sqrtf((float)D);
+  const long long part_stride = (long long)total_q * H;
+  auto* Opart = S > 1 ? reinterpret_cast<__nv_bfloat16*>(sc->part) : nullptr;
+  auto* ML = S > 1 ? reinterpret_cast<float2*>(sc->ml) : nullptr;
+  FPS_CUDA_TRY(launch_k(attn_tc5_kernel, dim3(heads, pairs, S), dim3(512), Cfg::SMEM, s, tq, tkv,
+                        reinterpret_cast<__nv_bfloat16*>(o), d_cu_q, d_cu_k, n_req, heads,
+                        scale_log2, ldo, Opart, ML, part_stride, total_q, o_map));
+  if (S > 1) {
+    count_launch();
+    const long long n = (long long)total_q * heads * (D / 8);
+    const int grid = (int)std::min<long long>((n + 255) / 256, kNumSMs * 8LL);
+    FPS_CUDA_TRY(launch_k(attn_combine_kernel<D>, dim3(grid), dim3(256), 0, s,
+                          (const __nv_bfloat16*)Opart, (const float2*)ML, part_stride, S, total_q,
+                          heads, reinterpret_cast<__nv_bfloat16*>(o), ldo, o_map));
+  }
+  return FPS_OK;
+}
+
 int g_attn_pair = 0;    // 1 = the CTA-pair kernel (attn_tc4) for head_dim 128
 
 static fps_status launch_d4(const void* q, const void* kv, void* o, int heads,
@@ -1697,6 +2117,8 @@ fps_status launch_attention_tc(const void* q, const void* kv, void* o, int heads
     if (head_dim == 128)
       return launch_d3<128>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo, sc,
                             o_map);
+    if (g_attn_force == 0 && g_attn_rot)
+      return launch_d5(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo, sc, o_map);
     return launch_d3<64>(q, kv, o, heads, d_cu_q, d_cu_k, h_cu_q, h_cu_k, n_req, s, ldo, sc, o_map);
   }
   if (o_map) return fail(FPS_EUNSUPPORTED, "attention: output row map needs the default kernel");

@@ -105,6 +105,7 @@ extern int g_gemm_bn;
 // tests: 0 = two query tiles per CTA (default), 1 = force the one-tile attention kernel
 extern int g_attn_force;
 extern int g_attn_pair;
+extern int g_attn_rot;
 // tests: force the split-KV factor S (0 = choose)
 extern int g_attn_split;
 // 1 (default): HBM-arena whole-entry loads copied by a library kernel, 0: driver D2D memcpy
