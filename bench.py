@@ -46,10 +46,14 @@ WORKLOADS = {
                copy_method=3, copy_ctas=8),
     "C2B": dict(H=1280, heads=20, F=5120, L_img=1024, L_txt=0, grid=(32, 32),
                 ratios=[0.1, 0.3, 0.5, 0.3], batch=4, layers=60, steps=50,
-                desc="SDXL-scale 32x32 level (1280 ch), masks 10/30/50%, batch 4"),
+                desc="SDXL-scale 32x32 level (1280 ch), masks 10/30/50%, batch 4",
+               # cache mode: Y (Fig. 5-Bottom, the paper's default; configs[1] does not name
+               # one): 12.31 vs 14.49 ms/step for KV in the same run (profiles/r02/c2_y/)
+               mode="y"),
     "C2A": dict(H=640, heads=10, F=2560, L_img=4096, L_txt=0, grid=(64, 64),
                 ratios=[0.1, 0.3, 0.5, 0.3], batch=4, layers=10, steps=50,
-                desc="SDXL-scale 64x64 level (640 ch), masks 10/30/50%, batch 4"),
+                desc="SDXL-scale 64x64 level (640 ch), masks 10/30/50%, batch 4",
+                mode="y"),      # 3.66 vs 4.46 ms/step for KV in the same run
 }
 SEED = 1003
 TIER_NAMES = {"host": "pinned host DRAM", "hbm": "device HBM (NEXT-1)",
@@ -491,7 +495,10 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C3", choices=list(WORKLOADS))
-    ap.add_argument("--mode", default="kv", choices=["kv", "y"])
+    ap.add_argument("--mode", default=None, choices=["kv", "y"],
+                    help="cache mode: K|V of the unmasked rows (KV-mode, L161) or the block "
+                         "outputs Y (Y-mode, the paper's default, L157). Default: kv for C3 / C4 "
+                         "(configs[2] names cached KV), y for the SDXL-scale levels C2A / C2B")
     ap.add_argument("--block", default=None, choices=["seq", "par", "sdxl", "flux"],
                     help="block kind: sequential attention -> MLP, the parallel (Flux "
                          "single-stream) block with fused input / output projections, or the SDXL "
@@ -550,6 +557,8 @@ def main():
     faulthandler.dump_traceback_later(int(os.environ.get("FPS_BENCH_TIMEOUT", 900)), exit=True)
     faulthandler.register(signal.SIGUSR1, all_threads=True)   # `timeout -s USR1`: dump stacks
     global LOAD_PRIORITY
+    if args.mode is None:
+        args.mode = WORKLOADS[args.config].get("mode", "kv")
     if args.copy_method is None:
         # measured on B200 (C3, profiles/r01f5_*): pinned host tier -- whole-entry DMA 34.6
         # ms/step vs 36.2 with one DMA per unmasked row run (~200 us of host time per entry) and

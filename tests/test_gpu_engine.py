@@ -21,7 +21,8 @@ def F():
 
 def _setup(F, mode, dtype, plan_policy, plan=None, N=3, steps=3, H=256, heads=2, Fd=512,
            L_img=256, L_txt=16, n_req=3, slots=0, copy_method=0, seed=5000, location=0,
-           kind="seq", cross_step=False, cost_model=(0.0, 0.0, 0.0, 0.0), sampler=0):
+           kind="seq", cross_step=False, cost_model=(0.0, 0.0, 0.0, 0.0), sampler=0,
+           copy_ctas=0):
     g = synth.rng(seed)
     W = synth.stack_weights(g, N, H, Fd, dtype, kind)
     mods = synth.mod_table(g, N, steps, H, dtype)
@@ -35,7 +36,7 @@ def _setup(F, mode, dtype, plan_policy, plan=None, N=3, steps=3, H=256, heads=2,
     dt = F.DTYPE_CODE[dtype]
     m = F.MODE_CODE[mode]
     cache = F.Cache(m, dt, H, L_img, N, steps, n_templates=n_t, copy_method=copy_method,
-                    location=location)
+                    location=location, copy_ctas=copy_ctas)
     for t in range(n_t):
         for s in range(steps):
             for l in range(N):
@@ -226,6 +227,23 @@ def test_delayed_load_stream_bit_identical(F, mode, method, location):
     torch.cuda.synchronize()
     for a, r in zip(ref, reqs):
         assert torch.equal(a.view(torch.int16), r["x"].view(torch.int16))
+
+
+@pytest.mark.parametrize("mode,ctas,prio", [("kv", 8, -5), ("y", 8, -5), ("kv", 6, 0)])
+def test_row_gather_wide_high_priority_bit_identical(F, mode, ctas, prio):
+    """configs[3]'s H2D setting: the TMA row gather on 8 CTAs (8 reserved SMs, compute grids on
+    the other 140) from a high-priority load stream, cross-step prefetch on, gives the bits of
+    the SM row gather (method 0) without a load stream."""
+    outs = []
+    for me, ct, use_ls in ((0, 0, False), (3, ctas, True)):
+        _, _, _, _, eng, reqs = _setup(F, mode, "bf16", 1, copy_method=me, seed=5250,
+                                       copy_ctas=ct, cross_step=True)
+        ls = torch.cuda.Stream(priority=prio) if use_ls else None
+        eng.run_batch(reqs, 3, load_stream=ls)
+        torch.cuda.synchronize()
+        outs.append([r["x"].clone() for r in reqs])
+    for a, b in zip(*outs):
+        assert torch.equal(a.view(torch.int16), b.view(torch.int16))
 
 
 def test_identical_input_cache_gpu_internal_invariant(F):

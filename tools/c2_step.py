@@ -12,7 +12,10 @@ convolutions / resamplers between the levels are out of scope: e
 its own hidden state.  Reports ms per step, images/s (50 steps), the dense step on the same
 kernels, and per-level times.
 
-  python tools/c2_step.py [steps=10] [warmup=3] > profiles/r02/c2_two_level_step.json
+  python tools/c2_step.py [steps=10] [warmup=3] [mode=y|kv] > profiles/r02/c2_two_level_step.json
+
+(mode: the cache mode, default y -- the paper's Y caching, Fig. 5-Bottom, which bench.py uses for
+the SDXL-scale levels)
 """
 import json
 import os
@@ -31,6 +34,7 @@ import synth
 def main():
     K = int(sys.argv[1]) if len(sys.argv) > 1 else 10
     W = int(sys.argv[2]) if len(sys.argv) > 2 else 3
+    mode = sys.argv[3] if len(sys.argv) > 3 else "y"
     import paper_conf_eurosys_jianglyfdlzllyl26_b200 as F
     F.require_gpu()
     dev = torch.device("cuda", 0)
@@ -49,8 +53,8 @@ def main():
     built = []
     for name, cfg, nl, tok in levels:
         w = dict(bench.WORKLOADS[cfg], block="sdxl", layers=nl, steps=max(S_IMG, W + K + 2))
-        layers, mod, cache = bench.build_engine_inputs(F, w, "kv", dev, 2 * (nl + 1), 0, 2)
-        cm, fit = bench.calibrate(F, w, "kv", layers, cache, [dict()] * B, dev)
+        layers, mod, cache = bench.build_engine_inputs(F, w, mode, dev, 2 * (nl + 1), 0, 2)
+        cm, fit = bench.calibrate(F, w, mode, layers, cache, [dict()] * B, dev)
         L = w["L_img"]
         reqs = [dict(template_id=i, step=0, n_steps=w["steps"], mask=tok[i].contiguous(),
                      x=torch.randn(L, w["H"], generator=gen, device=dev).to(torch.bfloat16),
@@ -62,7 +66,7 @@ def main():
         es = []
         for b in built:
             w = b["w"]
-            es.append(F.Engine(b["layers"], w["heads"], F.FPS_MODE_KV, F.FPS_BF16, w["L_img"], 0, B,
+            es.append(F.Engine(b["layers"], w["heads"], F.MODE_CODE[mode], F.FPS_BF16, w["L_img"], 0, B,
                                w["steps"], synth.delta_table(w["steps"]), b["cache"], mod_table=None,
                                plan_policy=policy, cost_model=b["cm"].as_engine_model(),
                                L_ctx=bench.SDXL_CTX[0], cross_step=True))
@@ -97,6 +101,7 @@ def main():
 
     out = {"workload": "configs[1] SDXL-scale: one request step over both UNet levels, A(4) -> "
                        "B(60) -> A(6) blocks, batch 4, pixel masks 10/30/50/30 % pooled per level",
+           "cache_mode": mode,
            "images_per_step": B, "denoise_steps": S_IMG, "steps": K, "warmup": W}
     ms, per, plans = run(engines(0))
     dms, dper, _ = run(engines(2))
