@@ -40,10 +40,13 @@ WORKLOADS = {
     "C4": dict(H=3072, heads=24, F=12288, L_img=4096, L_txt=512, grid=(64, 64),
                ratios=list(np.linspace(0.05, 0.60, 16)), batch=16, layers=57, steps=28,
                desc="continuous batch of 16 heterogeneous masks (5-60%), Flux-scale",
-               # H2D default (profiles/r02/c4_h2d/): whole entries move 1.48x the unmasked bytes
-               # here (mean m 0.33), so the exact-row TMA gather on 8 reserved SMs wins (525 vs
-               # 614 ms/step); at C3 (1.25x) the reserved SMs cost more than the bytes saved
-               copy_method=3, copy_ctas=8),
+               # cache mode: Y (the paper's default; configs[3] does not name one): 473.6
+               # ms/step with whole-entry DMA vs 486.7 with the row gather and 522.1 for KV-mode
+               # (profiles/r02/c4_mode/).  KV-mode here streams exactly the unmasked rows with the
+               # TMA row gather on 8 reserved SMs: whole entries move 1.48x the unmasked bytes
+               # (mean m 0.33) -- 524 vs 614 ms/step (profiles/r02/c4_h2d/); at C3 (1.25x) the
+               # reserved SMs cost more than the bytes saved
+               mode="y", kv_copy_method=3, kv_copy_ctas=8),
     "C2B": dict(H=1280, heads=20, F=5120, L_img=1024, L_txt=0, grid=(32, 32),
                 ratios=[0.1, 0.3, 0.5, 0.3], batch=4, layers=60, steps=50,
                 desc="SDXL-scale 32x32 level (1280 ch), masks 10/30/50%, batch 4",
@@ -559,15 +562,18 @@ def main():
     global LOAD_PRIORITY
     if args.mode is None:
         args.mode = WORKLOADS[args.config].get("mode", "kv")
+    cm_given = args.copy_method is not None
     if args.copy_method is None:
         # measured on B200 (C3, profiles/r01f5_*): pinned host tier -- whole-entry DMA 34.6
         # ms/step vs 36.2 with one DMA per unmasked row run (~200 us of host time per entry) and
         # 48.5 with the SM row gather (SM interference); HBM tier -- whole-entry DMA 21.2.
         # C4 (pinned host): the TMA row gather (WORKLOADS["C4"])
         wl = WORKLOADS[args.config]
-        args.copy_method = wl.get("copy_method", 2) if args.tier != "hbm" else 2
-        if args.copy_method == 3 and args.copy_ctas == 0:
-            args.copy_ctas = wl.get("copy_ctas", 0)
+        args.copy_method = 2
+        if args.mode == "kv" and args.tier != "hbm" and "kv_copy_method" in wl:
+            args.copy_method = wl["kv_copy_method"]
+            if args.copy_ctas == 0:
+                args.copy_ctas = wl.get("kv_copy_ctas", 0)
     if args.load_priority is None:
         args.load_priority = -5 if args.copy_method == 3 else 0
     LOAD_PRIORITY = args.load_priority
@@ -818,21 +824,32 @@ def main():
         # the other caching mode, and both modes with the other cache tier, on the same batch
         other = "y" if args.mode == "kv" else "kv"
         other_loc = 0 if location == 1 else 1
-        default_cm = lambda loc: 2
-        other_cm = default_cm(other_loc)
-        for md, loc, cmeth in ((other, location, args.copy_method),
-                               (args.mode, other_loc, other_cm), (other, other_loc, other_cm),
+        wl = WORKLOADS[args.config]
+
+        def default_cm(md, loc):     # the bench's default H2D method of a mode on a tier
+            return wl.get("kv_copy_method", 2) if (md == "kv" and loc != 1) else 2
+        other_cm = default_cm(other, other_loc)
+        for md, loc, cmeth in ((other, location, args.copy_method if cm_given
+                                else default_cm(other, location)),
+                               (args.mode, other_loc, default_cm(args.mode, other_loc)),
+                               (other, other_loc, other_cm),
                                (args.mode, location, 2 if args.copy_method != 2 else 1)):
             if loc == 1 and cmeth == 1:
                 continue
             loc = 0 if loc == 3 else loc        # the shared arena file belongs to `cache`
             log(f"[rank {rank}] extras: mode {md} location {loc} copy method {cmeth}")
+            ctas_saved = COPY_CTAS
+            ls_o = load_stream
+            if cmeth == 3 and not cm_given:   # that mode's default gather setting (C4 KV-mode)
+                COPY_CTAS = wl.get("kv_copy_ctas", 0)
+                ls_o = torch.cuda.Stream(device=device, priority=-5)
             c2 = make_cache(F, w, md, n_entries, loc, cmeth)
+            COPY_CTAS = ctas_saved
             cm2, _ = calibrate(F, w, md, layers, c2, [dict()] * w["batch"], device)
             eng_o = engine(0, mode=md, the_cache=c2, model=cm2)
-            o_ms, _ = run_engine_timed(F, eng_o, reqs_dev, K, W, stream, load_stream, rank, world)
+            o_ms, _ = run_engine_timed(F, eng_o, reqs_dev, K, W, stream, ls_o, rank, world)
             tag = f"{md}_mode_{['host', 'hbm', 'host_hugepage', 'host_shared'][loc]}"
-            if cmeth != default_cm(loc):
+            if cmeth != default_cm(md, loc):
                 tag += "_" + ["row_gather", "run_dma", "whole_entry_dma", "tma_row_gather"][cmeth]
             extras[f"{tag}_ms_per_step"] = o_ms
             extras[f"{tag}_cached_blocks"] = int(sum(eng_o.last_plan()[0]))

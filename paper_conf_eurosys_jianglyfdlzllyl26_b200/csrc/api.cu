@@ -420,8 +420,16 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
   // the arithmetic is unchanged (same K order and epilogue), so outputs are bit-identical.
   const bool par_group = w->kind == FPS_BLOCK_PAR && tq > 0 && tu > 0 && g_y_grouped;
   if (tq > 0 && !y_split) {
-    // a4: h1 = LN(x)(1+scale1)+shift1 on active rows
-    FPS_TRY(ln1(x_act, xr, tq, par_group ? ws.hu : ws.h, b->d_cu_q, nullptr));
+    // a4: h1 = LN(x)(1+scale1)+shift1 on active rows (Y-mode parallel block: and on the cached
+    // rows U in the same launch, rows [tq, tq + tu) of ws.hu -- after the load of x[U])
+    if (par_group) {
+      if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
+      kv_ready = nullptr;
+      FPS_TRY(launch_ln_mod_2src(dt, x_act, xr, tq, xu, b->d_u_src, tu, H, ws.hu, b->d_cu_q,
+                                 b->d_cu_u, b->n_req, mod, 0, s, MS));
+    } else {
+      FPS_TRY(ln1(x_act, xr, tq, ws.h, b->d_cu_q, nullptr));
+    }
     // a5: [tq,H] x [3H,H]^T; Q -> compact, K|V -> merged key rows at original positions
     Epilogue ep{};
     ep.bias = w->b_qkv;
@@ -435,11 +443,7 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
       n_out += F;
     }
     if (par_group) {
-      // Y-mode: cached block-input rows U -> LN (rows [tq, tq + tu) of ws.hu) -> K|V
-      if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
-      kv_ready = nullptr;
-      char* hu_rows = ws.hu + (size_t)tq * H * e;
-      FPS_TRY(ln1(xu, b->d_u_src, tu, hu_rows, b->d_cu_u, nullptr));
+      // Y-mode: K|V of the cached block-input rows U (normalised above)
       Epilogue ek{};
       ek.bias = w->b_qkv ? (const char*)w->b_qkv + (size_t)H * e : nullptr;
       ek.out0 = kv; ek.ld0 = 2 * H; ek.map0 = b->d_u_row;

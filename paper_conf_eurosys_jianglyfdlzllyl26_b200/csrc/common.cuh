@@ -265,6 +265,10 @@ struct LnMod {
   int split;
   int soff;
   const int32_t* cu2;
+  // optional second SOURCE for rows >= split (Y-mode parallel block: rows M from the active
+  // input, rows U from the cached input): row split + i reads x2 at rows2[i] (or i)
+  const T* x2;
+  const int32_t* rows2;
 };
 
 struct Epilogue {

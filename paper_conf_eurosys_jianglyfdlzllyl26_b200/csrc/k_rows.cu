@@ -211,9 +211,12 @@ __global__ void __launch_bounds__(128) ln_mod_kernel(const T* __restrict__ x,
   constexpr int NV = Vec16<T>::N;
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (warp >= n) return;
-  const int src_row = rows ? __ldg(rows + warp) : warp;
+  const bool src2 = md.x2 != nullptr && warp >= md.split;
+  const int32_t* rmap = src2 ? md.rows2 : rows;
+  const int ridx = src2 ? warp - md.split : warp;
+  const int src_row = rmap ? __ldg(rmap + ridx) : ridx;
   const int nvec = H / NV;
-  const uint4* xr = reinterpret_cast<const uint4*>(x + (size_t)src_row * H);
+  const uint4* xr = reinterpret_cast<const uint4*>((src2 ? md.x2 : x) + (size_t)src_row * H);
   float v[VPT][NV];
   float sum = 0.f;
 #pragma unroll
@@ -288,8 +291,11 @@ __global__ void __launch_bounds__(128) ln_mod_row_kernel(const T* __restrict__ x
   pdl_wait();
   const int row = blockIdx.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int nvec = H / NV;
-  const int src_row = rows ? __ldg(rows + row) : row;
-  const uint4* xr = reinterpret_cast<const uint4*>(x + (size_t)src_row * H);
+  const bool src2 = md.x2 != nullptr && row >= md.split;
+  const int32_t* rmap = src2 ? md.rows2 : rows;
+  const int ridx = src2 ? row - md.split : row;
+  const int src_row = rmap ? __ldg(rmap + ridx) : ridx;
+  const uint4* xr = reinterpret_cast<const uint4*>((src2 ? md.x2 : x) + (size_t)src_row * H);
   const bool mod = md.shift != nullptr;
   const uint4* sh = nullptr;
   const uint4* sc = nullptr;
@@ -532,9 +538,10 @@ fps_status launch_ln_affine_f32in(const float* x, int n, int H, void* out, const
 template <typename T>
 static LnMod<T> ln_params(const void* shift, const void* scale, int stride, float one,
                           const int32_t* cu, int n_req, int split = 0x7fffffff, int soff = 0,
-                          const int32_t* cu2 = nullptr) {
+                          const int32_t* cu2 = nullptr, const void* x2 = nullptr,
+                          const int32_t* rows2 = nullptr) {
   return LnMod<T>{reinterpret_cast<const T*>(shift), reinterpret_cast<const T*>(scale), stride, one,
-                  cu, n_req, split, soff, cu2};
+                  cu, n_req, split, soff, cu2, reinterpret_cast<const T*>(x2), rows2};
 }
 
 fps_status launch_ln_mod2(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
@@ -568,6 +575,29 @@ fps_status launch_ln_mod(int dtype, const void* x, const int32_t* rows, int n, i
                                    s, out_rows);
   return ln_mod_t<float>(x, rows, n, H, out, ln_params<float>(sh, sc, mod_stride, 1.0f, cu, n_req),
                          s, out_rows);
+}
+
+// Two row sources in one launch, one output: rows [0, n0) are LN-mod of x0 at rows0 (requests
+// from cu0), rows [n0, n0 + n1) of x1 at rows1 (requests from cu1); the same modulation vectors
+fps_status launch_ln_mod_2src(int dtype, const void* x0, const int32_t* rows0, int n0,
+                              const void* x1, const int32_t* rows1, int n1, int H, void* out,
+                              const int32_t* cu0, const int32_t* cu1, int n_req, const void* mod,
+                              int shift_off, cudaStream_t s, int mod_stride) {
+  if (n1 <= 0) return launch_ln_mod(dtype, x0, rows0, n0, H, out, cu0, n_req, mod, shift_off, s,
+                                    nullptr, mod_stride);
+  if (mod_stride <= 0) mod_stride = 6 * H;
+  const size_t e = dtype == FPS_BF16 ? 2 : 4;
+  const char* sh = mod ? (const char*)mod + (size_t)shift_off * e : nullptr;
+  const char* sc = mod ? sh + (size_t)H * e : nullptr;
+  if (dtype == FPS_BF16)
+    return ln_mod_t<__nv_bfloat16>(x0, rows0, n0 + n1, H, out,
+                                   ln_params<__nv_bfloat16>(sh, sc, mod_stride, 1.0f, cu0, n_req, n0,
+                                                            0, cu1, x1, rows1),
+                                   s, nullptr);
+  return ln_mod_t<float>(x0, rows0, n0 + n1, H, out,
+                         ln_params<float>(sh, sc, mod_stride, 1.0f, cu0, n_req, n0, 0, cu1, x1,
+                                          rows1),
+                         s, nullptr);
 }
 
 fps_status launch_ln_affine(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
