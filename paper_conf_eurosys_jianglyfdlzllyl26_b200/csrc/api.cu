@@ -398,15 +398,17 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
   // the M/U split (C3: 6 + 1 waves instead of 3 + 5)
   const bool y_split = tu > 0 && tq > 0 && w->kind != FPS_BLOCK_PAR;
   if (y_split) {
-    FPS_TRY(ln1(x_act, xr, tq, ws.h, b->d_cu_q, nullptr));
+    // one norm launch for both row sets (after the load of x[U]): rows M -> ws.h (compact, the Q
+    // GEMM's A) and ws.hu at their token rows; cached rows U -> ws.hu at theirs
+    if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
+    kv_ready = nullptr;
+    FPS_TRY(launch_ln_ysplit(dt, x_act, xr, tq, xu, b->d_u_src, tu, H, ws.h, ws.hu, b->d_q_row,
+                             b->d_u_row, b->d_cu_q, b->d_cu_u, b->n_req, mod, 0, MS,
+                             sdxl ? w->ln1_w : nullptr, sdxl ? w->ln1_b : nullptr, s));
     Epilogue eq{};
     eq.bias = w->b_qkv;
     eq.out0 = ws.q; eq.ld0 = H; eq.split = H;
     FPS_TRY(launch_gemm(dt, ws.h, w->w_qkv, tq, H, H, eq, s));
-    FPS_TRY(ln1(x_act, xr, tq, ws.hu, b->d_cu_q, b->d_q_row));
-    if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
-    kv_ready = nullptr;
-    FPS_TRY(ln1(xu, b->d_u_src, tu, ws.hu, b->d_cu_u, b->d_u_row));
     Epilogue ek{};
     ek.bias = w->b_qkv ? (const char*)w->b_qkv + (size_t)H * e : nullptr;
     ek.out0 = kv; ek.ld0 = 2 * H; ek.split = 2 * H;

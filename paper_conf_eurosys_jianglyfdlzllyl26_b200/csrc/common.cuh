@@ -269,6 +269,13 @@ struct LnMod {
   // input, rows U from the cached input): row split + i reads x2 at rows2[i] (or i)
   const T* x2;
   const int32_t* rows2;
+  // optional SECOND OUTPUT (Y-mode sequential / SDXL block: the normalised rows M also land in
+  // the all-rows buffer at their token rows, next to the normalised cached rows U): row r < split
+  // is also stored at outb[outb_rows1[r]]; with x2, rows >= split are stored ONLY there, at
+  // outb[outb_rows2[r - split]]
+  T* outb;
+  const int32_t* outb_rows1;
+  const int32_t* outb_rows2;
 };
 
 struct Epilogue {

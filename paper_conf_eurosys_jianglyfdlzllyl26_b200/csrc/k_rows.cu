@@ -256,7 +256,12 @@ __global__ void __launch_bounds__(128) ln_mod_kernel(const T* __restrict__ x,
     shift = md.shift + off;
     scale = md.scale + off;
   }
-  uint4* o = reinterpret_cast<uint4*>(out + (size_t)(out_rows ? __ldg(out_rows + warp) : warp) * H);
+  uint4* o = (src2 && md.outb) ? nullptr
+                               : reinterpret_cast<uint4*>(out + (size_t)(out_rows ? __ldg(out_rows + warp) : warp) * H);
+  uint4* ob = md.outb ? reinterpret_cast<uint4*>(
+                            md.outb + (size_t)(src2 ? __ldg(md.outb_rows2 + warp - md.split)
+                                                    : __ldg(md.outb_rows1 + warp)) * H)
+                      : nullptr;
 #pragma unroll
   for (int k = 0; k < VPT; ++k) {
     int vi = lane + 32 * k;
@@ -272,7 +277,9 @@ __global__ void __launch_bounds__(128) ln_mod_kernel(const T* __restrict__ x,
 #pragma unroll
         for (int e = 0; e < NV; ++e) r[e] = (v[k][e] - mean) * rstd;
       }
-      o[vi] = Vec16<T>::pack(r);
+      const uint4 pr = Vec16<T>::pack(r);
+      if (o) o[vi] = pr;
+      if (ob) ob[vi] = pr;
     }
   }
 }
@@ -344,7 +351,12 @@ __global__ void __launch_bounds__(128) ln_mod_row_kernel(const T* __restrict__ x
   if (lane == 0) red[warp] = sq;
   __syncthreads();
   const float rstd = 1.0f / sqrtf((red[0] + red[1] + red[2] + red[3]) / (float)H + 1e-6f);
-  uint4* o = reinterpret_cast<uint4*>(out + (size_t)(out_rows ? __ldg(out_rows + row) : row) * H);
+  uint4* o = (src2 && md.outb) ? nullptr
+                               : reinterpret_cast<uint4*>(out + (size_t)(out_rows ? __ldg(out_rows + row) : row) * H);
+  uint4* ob = md.outb ? reinterpret_cast<uint4*>(
+                            md.outb + (size_t)(src2 ? __ldg(md.outb_rows2 + row - md.split)
+                                                    : __ldg(md.outb_rows1 + row)) * H)
+                      : nullptr;
 #pragma unroll
   for (int k = 0; k < VPT; ++k) {
     const int vi = tid + 128 * k;
@@ -354,7 +366,9 @@ __global__ void __launch_bounds__(128) ln_mod_row_kernel(const T* __restrict__ x
       Vec16<T>::unpack(scv[k], b);
 #pragma unroll
       for (int e = 0; e < NV; ++e) r[e] = (v[k][e] - mean) * rstd * (md.one + b[e]) + a[e];
-      o[vi] = Vec16<T>::pack(r);
+      const uint4 pr = Vec16<T>::pack(r);
+      if (o) o[vi] = pr;
+      if (ob) ob[vi] = pr;
     }
   }
 }
@@ -598,6 +612,38 @@ fps_status launch_ln_mod_2src(int dtype, const void* x0, const int32_t* rows0, i
                          ln_params<float>(sh, sc, mod_stride, 1.0f, cu0, n_req, n0, 0, cu1, x1,
                                           rows1),
                          s, nullptr);
+}
+
+// The y_split norm in one launch: rows [0, n0) of x0 at rows0 -> out[r] and outb[outb_rows0[r]];
+// rows [n0, n0 + n1) of x1 at rows1 -> outb[outb_rows1[r - n0]] only.  Modulation as
+// launch_ln_mod_2src (cu0 / cu1), or the affine LN (gamma / beta) when `gamma` is given.
+fps_status launch_ln_ysplit(int dtype, const void* x0, const int32_t* rows0, int n0,
+                            const void* x1, const int32_t* rows1, int n1, int H, void* out,
+                            void* outb, const int32_t* outb_rows0, const int32_t* outb_rows1,
+                            const int32_t* cu0, const int32_t* cu1, int n_req, const void* mod,
+                            int shift_off, int mod_stride, const void* gamma, const void* beta,
+                            cudaStream_t s) {
+  if (n0 + n1 <= 0) return FPS_OK;
+  if (mod_stride <= 0) mod_stride = 6 * H;
+  const size_t e = dtype == FPS_BF16 ? 2 : 4;
+  const char* sh = gamma ? (const char*)beta : mod ? (const char*)mod + (size_t)shift_off * e : nullptr;
+  const char* sc = gamma ? (const char*)gamma : mod ? sh + (size_t)H * e : nullptr;
+  const int stride = gamma ? 0 : mod_stride;
+  const float one = gamma ? 0.0f : 1.0f;
+  if (dtype == FPS_BF16) {
+    auto md = ln_params<__nv_bfloat16>(sh, sc, stride, one, gamma ? nullptr : cu0, n_req, n0, 0,
+                                       gamma ? nullptr : cu1, x1, rows1);
+    md.outb = reinterpret_cast<__nv_bfloat16*>(outb);
+    md.outb_rows1 = outb_rows0;
+    md.outb_rows2 = outb_rows1;
+    return ln_mod_t<__nv_bfloat16>(x0, rows0, n0 + n1, H, out, md, s, nullptr);
+  }
+  auto md = ln_params<float>(sh, sc, stride, one, gamma ? nullptr : cu0, n_req, n0, 0,
+                             gamma ? nullptr : cu1, x1, rows1);
+  md.outb = reinterpret_cast<float*>(outb);
+  md.outb_rows1 = outb_rows0;
+  md.outb_rows2 = outb_rows1;
+  return ln_mod_t<float>(x0, rows0, n0 + n1, H, out, md, s, nullptr);
 }
 
 fps_status launch_ln_affine(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,

@@ -19,6 +19,12 @@ fps_status launch_copy_rows(const void* src, const int32_t* src_ids, const int32
 fps_status launch_ln_mod(int dtype, const void* x, const int32_t* rows, int n, int H, void* out,
                          const int32_t* cu, int n_req, const void* mod, int shift_off,
                          cudaStream_t s, const int32_t* out_rows = nullptr, int mod_stride = 0);
+fps_status launch_ln_ysplit(int dtype, const void* x0, const int32_t* rows0, int n0,
+                            const void* x1, const int32_t* rows1, int n1, int H, void* out,
+                            void* outb, const int32_t* outb_rows0, const int32_t* outb_rows1,
+                            const int32_t* cu0, const int32_t* cu1, int n_req, const void* mod,
+                            int shift_off, int mod_stride, const void* gamma, const void* beta,
+                            cudaStream_t s);
 fps_status launch_ln_mod_2src(int dtype, const void* x0, const int32_t* rows0, int n0,
                               const void* x1, const int32_t* rows1, int n1, int H, void* out,
                               const int32_t* cu0, const int32_t* cu1, int n_req, const void* mod,
