@@ -2047,6 +2047,8 @@ static fps_status launch_d5(const void* q, const void* kv, void* o, int heads,
                           (const __nv_bfloat16*)Opart, (const float2*)ML, part_stride, S, total_q,
                           heads, reinterpret_cast<__nv_bfloat16*>(o), ldo, o_map));
   }
+  count_launch();
+  FPS_LAUNCH_CHECK();
   return FPS_OK;
 }
 
