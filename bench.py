@@ -491,6 +491,28 @@ def cpu_threads():
 
 
 # ---------------------------------------------------------------------------------------
+def resolve_defaults(args):
+    """Per-config defaults of the cache mode and the H2D path (flags the user gave win).
+    Mode: KV for C3 (configs[2] names cached KV), Y -- the paper's default (L157) -- for the
+    configs that name none (C2A / C2B / C4; measured faster there, profiles/r02/c2_y, c4_mode).
+    H2D: whole-entry DMA (measured on B200, C3, profiles/r01f5_*: 34.6 ms/step vs 36.2 with one
+    DMA per unmasked row run and 48.5 with the SM row gather; HBM tier 21.2), except KV-mode at
+    C4 on the host tier: the TMA row gather on 8 SMs (WORKLOADS["C4"]).  Load-stream priority:
+    highest with the row gather, else the compute stream's."""
+    wl = WORKLOADS[args.config]
+    if args.mode is None:
+        args.mode = wl.get("mode", "kv")
+    if args.copy_method is None:
+        args.copy_method = 2
+        if args.mode == "kv" and args.tier != "hbm" and "kv_copy_method" in wl:
+            args.copy_method = wl["kv_copy_method"]
+            if args.copy_ctas == 0:
+                args.copy_ctas = wl.get("kv_copy_ctas", 0)
+    if args.load_priority is None:
+        args.load_priority = -5 if args.copy_method == 3 else 0
+    return args
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -560,22 +582,8 @@ def main():
     faulthandler.dump_traceback_later(int(os.environ.get("FPS_BENCH_TIMEOUT", 900)), exit=True)
     faulthandler.register(signal.SIGUSR1, all_threads=True)   # `timeout -s USR1`: dump stacks
     global LOAD_PRIORITY
-    if args.mode is None:
-        args.mode = WORKLOADS[args.config].get("mode", "kv")
     cm_given = args.copy_method is not None
-    if args.copy_method is None:
-        # measured on B200 (C3, profiles/r01f5_*): pinned host tier -- whole-entry DMA 34.6
-        # ms/step vs 36.2 with one DMA per unmasked row run (~200 us of host time per entry) and
-        # 48.5 with the SM row gather (SM interference); HBM tier -- whole-entry DMA 21.2.
-        # C4 (pinned host): the TMA row gather (WORKLOADS["C4"])
-        wl = WORKLOADS[args.config]
-        args.copy_method = 2
-        if args.mode == "kv" and args.tier != "hbm" and "kv_copy_method" in wl:
-            args.copy_method = wl["kv_copy_method"]
-            if args.copy_ctas == 0:
-                args.copy_ctas = wl.get("kv_copy_ctas", 0)
-    if args.load_priority is None:
-        args.load_priority = -5 if args.copy_method == 3 else 0
+    resolve_defaults(args)
     LOAD_PRIORITY = args.load_priority
 
     rank = int(os.environ.get("RANK", 0))
