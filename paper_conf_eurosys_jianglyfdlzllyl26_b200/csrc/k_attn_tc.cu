@@ -1234,8 +1234,9 @@ __global__ void __launch_bounds__(512, 1)
       float m_used = -INFINITY, l = 0.f;
       for (int kt = 0; kt < nk; ++kt) {
         const int i = 2 * kt + t, pb = t * 2 + (kt & 1);
-        // buffer i % 3 is used by indices b, b + 3, ... (one tile: only the even indices, so
-        // the n-th use of a buffer is key tile 3n + ..)
+        // how many times buffer i % 3 was filled before: with two tiles every index is used
+        // (buffer b holds indices b, b + 3, b + 6, ...: use i / 3); with one tile only the even
+        // indices 2 kt are (buffer (2 kt) % 3 cycles with period 3 in kt: use kt / 3)
         const int n_use = hasB ? i / 3 : kt / 3;
         tc::mbar_wait(&bar_s[i % 3], (uint32_t)(n_use & 1));
         tc::fence_after();
