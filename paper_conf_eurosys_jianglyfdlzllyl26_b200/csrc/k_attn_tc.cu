@@ -636,6 +636,9 @@ __global__ void __launch_bounds__(384, 1)
 #ifndef FPS_ATTN_POLY64          // the same for head_dim 64 (twice the exponentials per MMA FLOP)
 #define FPS_ATTN_POLY64 4
 #endif
+#ifndef FPS_ATTN_PQ               // P release granularity of attn_tc3: 2 halves or 4 quarters
+#define FPS_ATTN_PQ 2             // (quarters measured 1030 vs 1047 TF/s at C3's masked shape)
+#endif
 #ifndef FPS_ATTN_MMA_SPIN
 #define FPS_ATTN_MMA_SPIN 0
 #endif
@@ -730,7 +733,11 @@ __global__ void __launch_bounds__(512, 1)
   uint64_t* bar_o = bars + 15;      // [tile] final PV_t done              (MMA commit)
   uint64_t* bar_fin = bars + 17;    // [tile] row sum l in smem            (4 softmax warps)
   uint64_t* bar_p2 = bars + 19;     // [tile] second half of P_t(j) stored (4 softmax warps)
-  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + 21);
+  // FPS_ATTN_PQ = 4: P released in quarters -- bar_p (keys 0-31, + the correction warps),
+  // bar_p2 (32-63), bar_p3 (64-95), bar_p4 (96-127); 2: halves (bar_p 0-63, bar_p2 64-127)
+  uint64_t* bar_p3 = bars + 21;
+  uint64_t* bar_p4 = bars + 23;
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + 25);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   // grid (heads, query-tile pairs, splits): heads vary fastest, so the CTAs the block scheduler
@@ -770,6 +777,8 @@ __global__ void __launch_bounds__(512, 1)
       tc::mbar_init(&bar_o[s], 1);
       tc::mbar_init(&bar_fin[s], 4);
       tc::mbar_init(&bar_p2[s], 4);
+      tc::mbar_init(&bar_p3[s], 4);
+      tc::mbar_init(&bar_p4[s], 4);
     }
     tc::fence_mbar_init();
   }
@@ -837,14 +846,25 @@ __global__ void __launch_bounds__(512, 1)
         // stored them (bar_p), keys 64-127 after the rest (bar_p2)
         auto issue_pv = [&](int t, int kt) {
           const uint64_t b = dv + (((kt & 1) * Cfg::KV_TILE) >> 4);
-          ATTN_MMA_WAIT(&bar_p[t], kt & 1);
-          tc::fence_after();
-          ATTN_TRACE(t, kt, 5);
-          tc::mma_ts_k4(256 + t * 128, t * 128 + 64, b, idesc_o, kt != 0);
-          ATTN_MMA_WAIT(&bar_p2[t], kt & 1);
-          tc::fence_after();
-          ATTN_TRACE(t, kt, 6);
-          tc::mma_ts_k4(256 + t * 128, t * 128 + 96, b + (4 * 2048 >> 4), idesc_o, 1);
+          if constexpr (FPS_ATTN_PQ == 4) {
+            uint64_t* qb[4] = {&bar_p[t], &bar_p2[t], &bar_p3[t], &bar_p4[t]};
+#pragma unroll
+            for (int qq = 0; qq < 4; ++qq) {
+              ATTN_MMA_WAIT(qb[qq], kt & 1);
+              tc::fence_after();
+              tc::mma_ts_k2(256 + t * 128, t * 128 + 64 + 16 * qq, b + ((2 * 2048 * qq) >> 4),
+                            idesc_o, (kt != 0 || qq != 0) ? 1u : 0u);
+            }
+          } else {
+            ATTN_MMA_WAIT(&bar_p[t], kt & 1);
+            tc::fence_after();
+            ATTN_TRACE(t, kt, 5);
+            tc::mma_ts_k4(256 + t * 128, t * 128 + 64, b, idesc_o, kt != 0);
+            ATTN_MMA_WAIT(&bar_p2[t], kt & 1);
+            tc::fence_after();
+            ATTN_TRACE(t, kt, 6);
+            tc::mma_ts_k4(256 + t * 128, t * 128 + 96, b + (4 * 2048 >> 4), idesc_o, 1);
+          }
         };
         tc::mbar_wait_sleep(&k_full[0], 0);
         tc::fence_after();
@@ -929,11 +949,16 @@ __global__ void __launch_bounds__(512, 1)
             p[(i - c * 32) >> 1] = tc::pack_bf16x2_rn(s[i], s[i + 1]);
           }
           tc::tmem_st16(tS + lane_off + 64 + c * 16, p);
-          if (c & 1) {                                     // keys 0-63, then 64-127, released
+          if (FPS_ATTN_PQ == 4 || (c & 1)) {               // keys released by halves / quarters
             tc::tmem_wait_st();
             tc::fence_before();
             __syncwarp();
-            if (lane == 0) tc::mbar_arrive(c == 1 ? &bar_p[t] : &bar_p2[t]);
+            if (lane == 0) {
+              if (FPS_ATTN_PQ == 4)
+                tc::mbar_arrive(c == 0 ? &bar_p[t] : c == 1 ? &bar_p2[t] : c == 2 ? &bar_p3[t] : &bar_p4[t]);
+              else
+                tc::mbar_arrive(c == 1 ? &bar_p[t] : &bar_p2[t]);
+            }
             ATTN_TRACE(t, kt, 2 + (c >> 1) + 1);
           }
         }

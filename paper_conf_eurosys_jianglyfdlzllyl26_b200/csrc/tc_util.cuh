@@ -320,6 +320,22 @@ __device__ __forceinline__ void mma_ts_k4(uint32_t d, uint32_t a_tmem, uint64_t 
       "r"(a_tmem), "r"(blo), "r"(bhi), "r"(idesc), "r"(acc)
       : "memory");
 }
+// TS group of 2 steps (32 keys): as mma_ts_k4, half the keys
+__device__ __forceinline__ void mma_ts_k2(uint32_t d, uint32_t a_tmem, uint64_t bdesc,
+                                          uint32_t idesc, uint32_t acc) {
+  const uint32_t blo = (uint32_t)bdesc, bhi = (uint32_t)(bdesc >> 32);
+  asm volatile(
+      "{\n.reg .pred e, p;\n.reg .b32 ta, bl;\n.reg .b64 bd;\n"
+      "elect.sync _|e, 0xffffffff;\n"
+      "setp.ne.b32 p, %5, 0;\n"
+      "mov.b64 bd, {%2, %3};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], bd, %4, p;\n"
+      "add.s32 ta, %1, 8;\nadd.s32 bl, %2, 128;\nmov.b64 bd, {bl, %3};\n"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ta], bd, %4, 1;\n"
+      "}\n" ::"r"(d),
+      "r"(a_tmem), "r"(blo), "r"(bhi), "r"(idesc), "r"(acc)
+      : "memory");
+}
 __device__ __forceinline__ void mma_ts_k4_commit(uint32_t d, uint32_t a_tmem, uint64_t bdesc,
                                                  uint32_t idesc, uint32_t acc, uint64_t* bar) {
   mma_ts_k4(d, a_tmem, bdesc, idesc, acc);
