@@ -165,7 +165,10 @@ static size_t ws_layout(int H, int F, int dtype, int max_q, int max_u, char* bas
   char* x1 = take((size_t)max_q * H * 4);              // fp32 for the SDXL block's residual stream
   char* h2 = take((size_t)max_q * H * e);
   char* u = take((size_t)max_q * F * e);
-  char* hu = take((size_t)(max_q + max_u) * H * e);   // Y-mode: LN of all rows, token order
+  // Y-mode: LN of all rows in token order; max_q rows of headroom in front, where the
+  // sequential / SDXL block puts the compact rows M right before it (one A operand for the
+  // grouped Q + K|V launch)
+  char* hu = take((size_t)(2 * max_q + max_u) * H * e) + (base ? (size_t)max_q * H * e : 0);
   char* x2 = take((size_t)max_q * H * 4);              // SDXL block: after cross-attention (fp32)
   if (ws) *ws = BlockWs{h, q, ao, x1, h2, u, hu, x2};
   return off;
@@ -402,18 +405,27 @@ static fps_status block_forward(const fps_block_weights* w, const fps_varlen_bat
     // GEMM's A) and ws.hu at their token rows; cached rows U -> ws.hu at theirs
     if (kv_ready) FPS_CUDA_TRY(stream_wait(s, kv_ready, 0));
     kv_ready = nullptr;
-    FPS_TRY(launch_ln_ysplit(dt, x_act, xr, tq, xu, b->d_u_src, tu, H, ws.h, ws.hu, b->d_q_row,
+    // the compact rows M sit right before ws.hu (its headroom), so Q over rows M and K|V over
+    // all rows are ONE grouped launch on one A operand (per-problem N: H and 2H); bit-identical
+    // to two launches (flag bit 15 selects those)
+    char* hq = g_y_grouped ? ws.hu - (size_t)tq * H * e : ws.h;
+    FPS_TRY(launch_ln_ysplit(dt, x_act, xr, tq, xu, b->d_u_src, tu, H, hq, ws.hu, b->d_q_row,
                              b->d_u_row, b->d_cu_q, b->d_cu_u, b->n_req, mod, 0, MS,
                              sdxl ? w->ln1_w : nullptr, sdxl ? w->ln1_b : nullptr, s));
     Epilogue eq{};
     eq.bias = w->b_qkv;
     eq.out0 = ws.q; eq.ld0 = H; eq.split = H;
-    FPS_TRY(launch_gemm(dt, ws.h, w->w_qkv, tq, H, H, eq, s));
     Epilogue ek{};
     ek.bias = w->b_qkv ? (const char*)w->b_qkv + (size_t)H * e : nullptr;
     ek.out0 = kv; ek.ld0 = 2 * H; ek.split = 2 * H;
-    FPS_TRY(launch_gemm(dt, ws.hu, (const char*)w->w_qkv + (size_t)H * H * e, b->total_k, 2 * H, H,
-                        ek, s));
+    if (g_y_grouped) {
+      FPS_TRY(launch_gemm_grouped(dt, hq, w->w_qkv, (const char*)w->w_qkv + (size_t)H * H * e, tq,
+                                  b->total_k, H, H, eq, ek, s, 2 * H));
+    } else {
+      FPS_TRY(launch_gemm(dt, hq, w->w_qkv, tq, H, H, eq, s));
+      FPS_TRY(launch_gemm(dt, ws.hu, (const char*)w->w_qkv + (size_t)H * H * e, b->total_k, 2 * H,
+                          H, ek, s));
+    }
   }
   // Y-mode parallel block: the W1 GEMM of rows M ([Q|K|V|Z]) and the K|V GEMM of the cached
   // rows U in ONE grouped launch (A = both rows' LN outputs, stacked in ws.hu): the persistent

@@ -296,16 +296,19 @@ def test_active_rows_read_from_full_buffer_bit_identical(F, kind, mode):
     assert np.array_equal(y, y_ref)
 
 
-@pytest.mark.parametrize("H,heads,Fd,L_img,L_txt,ratios", [
-    (256, 2, 1024, 576, 40, [0.05, 0.6, 0.3]),          # several tiles per problem, ragged
-    (3072, 24, 12288, 4096, 512, [0.2]),                # the C3 single-stream block
+@pytest.mark.parametrize("kind,H,heads,Fd,L_img,L_txt,ratios", [
+    ("par", 256, 2, 1024, 576, 40, [0.05, 0.6, 0.3]),   # several tiles per problem, ragged
+    ("par", 3072, 24, 12288, 4096, 512, [0.2]),         # the C3 single-stream block
+    ("seq", 256, 2, 1024, 576, 40, [0.05, 0.6, 0.3]),   # sequential block: Q(M) + K|V(all rows)
+    ("seq", 1280, 20, 5120, 1024, 0, [0.1, 0.3, 0.5, 0.3]),   # the C2B level's width
 ])
-def test_y_parallel_grouped_projections_bit_identical(F, H, heads, Fd, L_img, L_txt, ratios):
-    """Y-mode parallel block: W1 over rows M and K|V over cached rows U in ONE grouped launch
-    (per-problem N: 3H + F and 2H) gives the same bits as two launches (flag bit 15), and both
-    match the oracle (masked_block_y)."""
+def test_y_parallel_grouped_projections_bit_identical(F, kind, H, heads, Fd, L_img, L_txt, ratios):
+    """Y-mode projections in ONE grouped launch -- parallel block: W1 over rows M and K|V over
+    the cached rows U (per-problem N: 3H + F and 2H); sequential block: Q over rows M and K|V over
+    all rows (N: H and 2H) -- give the same bits as two launches (flag bit 15), and match the
+    oracle (masked_block_y)."""
     w, reqs = _problem(4200 + H, "bf16", H, heads, Fd, L_img, L_txt, ratios, blobs=True,
-                       kind="par")
+                       kind=kind)
     y_grouped, kv_grouped = _run_masked(F, w, reqs, heads, "bf16", "y")
     F.fps_set_disable_tc(1 << 15)
     try:
