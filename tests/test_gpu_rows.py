@@ -83,7 +83,8 @@ def test_empty_gather_is_noop(F):
     ("kv", 0, 1, 256, 0), ("y", 0, 1, 256, 0), ("kv", 1, 1, 256, 0),
     ("kv", 2, 0, 256, 0), ("y", 2, 0, 256, 0), ("kv", 2, 1, 256, 0),
     ("kv", 3, 0, 256, 0), ("y", 3, 0, 256, 0), ("kv", 3, 0, 3072, 0), ("y", 3, 0, 3072, 0),
-    ("kv", 3, 0, 1280, 6), ("kv", 3, 1, 640, 2), ("y", 3, 0, 4096, 1)])
+    ("kv", 3, 0, 1280, 6), ("kv", 3, 1, 640, 2), ("y", 3, 0, 4096, 1),
+    ("kv", 3, 0, 3072, 8)])                             # configs[3]'s KV-mode setting
 def test_cache_store_prefetch_bytes_equal(F, mode, method, location, H, ctas):
     """a3: the prefetched rows are the stored entry's rows, byte for byte, at their token rows.
     Exact-row methods (0, 1, 3) leave every other row untouched; the whole-entry DMA (2) lands
